@@ -1,0 +1,186 @@
+"""Pins for the host-side oracle: fusion index mapping (Fig. 5/6), PTB coverage (Fig. 7),
+fusion budget (§V-C), predictor (§VI), manager (§VII) and metrics (Eqs. 10/11)."""
+import json
+import os
+
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st
+
+from oracle import fusion, manager_ref as mr, metrics, predictor
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def gold(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+# ------------------------------------------------------------------ Fig. 6 worked example
+def test_fig6_direct_fusion_worked_example():
+    g = gold("fig6_direct_fusion.json")
+    grid, block, role = fusion.direct_fusion_map(g["block_num_tc"], g["thread_num_tc"],
+                                                 g["block_num_cd"], g["thread_num_cd"])
+    assert (grid, block) == (g["fused_grid"], g["fused_block"])
+    lo, hi = g["cd_thread_range"]
+    for b in range(grid):
+        for t in range(lo, hi + 1):
+            assert role[b][t] == ("cd", b, t - lo)
+        for t in range(lo):
+            if b in g["idle_tc_blocks"]:
+                assert role[b][t] is None
+            else:
+                assert role[b][t] == ("tc", b, t)
+
+
+# ------------------------------------------------------------------ Fig. 7 PTB
+@settings(max_examples=200, deadline=None)
+@given(st.integers(0, 3000), st.integers(1, 400))
+def test_ptb_visits_every_block_exactly_once(orig, issued):
+    v = fusion.ptb_visits(orig, issued)
+    flat = sorted(x for row in v for x in row)
+    assert flat == list(range(orig))
+
+
+def test_ptb_figure_bound_reading():
+    # Fig. 7 literally uses `<=`, which would visit block `original_block_num`: reading `<`.
+    assert fusion.ptb_visits(4, 3) == [[0, 3], [1], [2]]
+
+
+# ------------------------------------------------------------------ §V-C budget
+def test_sec5c_budget_example():
+    g = gold("sec5c_budget.json")
+    cap = g["smem_capacity"]
+    assert g["tc_smem"] + g["cd_smem"] == g["one_to_one_block_smem"]
+    assert fusion.fused_blocks_per_sm(1, g["tc_smem"], 1, g["cd_smem"], cap) == g["one_to_one_blocks_per_sm"]
+    r = fusion.flexible_ratio(g["tc_blocks_needed"], g["tc_smem"], g["cd_smem"], cap)
+    assert list(r) == g["flexible_ratio"]
+    assert fusion.fused_blocks_per_sm(r[0], g["tc_smem"], r[1], g["cd_smem"], cap) == g["flexible_blocks_per_sm"]
+    assert fusion.fused_blocks_per_sm(3, g["tc_smem"], 1, g["cd_smem"], cap) == 0   # over budget: no fusion
+
+
+# ------------------------------------------------------------------ predictor
+def test_ols_matches_polyfit():
+    rng = np.random.default_rng(0)
+    x = rng.uniform(1, 100, 20)
+    y = 0.37 * x + 5.0 + rng.normal(0, 0.3, 20)
+    a, b = predictor.ols(list(x), list(y))
+    pa, pb = np.polyfit(x, y, 1)
+    assert abs(a - pa) < 1e-12 and abs(b - pb) < 1e-10
+
+
+def test_kernel_lr_exact_recovery():
+    m = predictor.KernelLR()
+    for blocks in (16, 32, 64, 128, 256, 512):
+        m.add(blocks, 0.002 * blocks + 0.011)
+    a, b = m.fit()
+    assert abs(a - 0.002) < 1e-15 and abs(b - 0.011) < 1e-13
+    assert abs(m.predict(1000) - 2.011) < 1e-12
+
+
+def closed_form_tau(r, r_o=0.8, tau_o=1.25):
+    # Eqs. 3-6 reading: stage 1 linear from tau(0)=1 to (r_o, tau_o); stage 2 slope 1 after r_o
+    return 1 + (tau_o - 1) * r / r_o if r <= r_o else tau_o + (r - r_o)
+
+
+def test_two_stage_recovers_closed_form():
+    m = predictor.TwoStage()
+    xtc = 3.0
+    for r in predictor.TRAIN_RATIOS:
+        m.add(xtc, r * xtc, xtc * closed_form_tau(r))
+    m.fit()
+    assert abs(m.inflection() - 0.8) < 1e-12
+    assert abs(m.l2[1] - 1.0) < 1e-12   # slope 1 after the inflection
+    for r in np.linspace(0.01, 3, 40):
+        for x in (0.5, 3.0, 11.0):      # linear in X_tc at fixed r (Fig. 11)
+            assert abs(m.predict(x, r * x) - x * closed_form_tau(r)) < 1e-10
+
+
+def test_two_stage_online_refit():
+    m = predictor.TwoStage()
+    for r in predictor.TRAIN_RATIOS:
+        m.add(1.0, r, closed_form_tau(r))
+    m.fit()
+    assert not m.observe(1.0, 0.5, closed_form_tau(0.5) * 1.05)      # 5 % error: keep
+    assert m.observe(1.0, 0.5, closed_form_tau(0.5) * 1.3)           # 30 % error: refit
+    assert len(m.samples) == 5
+
+
+# ------------------------------------------------------------------ manager
+def heads_and_pred(spec):
+    heads = [(a, tcd, True) for a, tcd, _ in spec["heads"]]
+    tf = {a: f for a, _, f in spec["heads"]}
+    return heads, (lambda a: tf[a])
+
+
+@pytest.mark.parametrize("sid", ["S1", "S2", "S3", "S4", "S6"])
+def test_manager_scenarios(sid):
+    s = gold("manager_scenarios.json")[sid]
+    heads, fp = heads_and_pred(s)
+    fused, reorder, thr, gain = mr.decide(s["ttc"], True, s["thr"], heads, mr.TACKER, fp)
+    assert fused == s["fused"]
+    assert reorder == s["reorder"]
+    assert abs(thr - s["thr_after"]) < 1e-12
+    if "gain" in s:
+        assert abs(gain - s["gain"]) < 1e-12
+
+
+def test_manager_baymax_never_fuses():
+    s = gold("manager_scenarios.json")["S1"]
+    heads, fp = heads_and_pred(s)
+    fused, reorder, thr, _ = mr.decide(s["ttc"], True, s["thr"], heads, mr.BAYMAX, fp)
+    assert fused == -1 and reorder == [0] and thr == 37
+
+
+def test_manager_eq9_headroom_two_queries():
+    s = gold("manager_scenarios.json")["S5"]
+    # earlier query (12 ms remaining) still active when Q (Tori_solo 10) is issued
+    q_old = mr.Query(0, 0.0, [(True, 12.0)])
+    q_new = mr.Query(1, 0.0, [(True, 5.0), (True, 5.0)])
+    res = mr.simulate([q_old, q_new], [], s["qos"], mr.TACKER, lambda a, b: None)
+    # q_new issues at t=12 after q_old; Tqueue = 12 so Thr = 50 - 12 - 10 - 0 = 28 (== S5)
+    assert res["latency"] == {0: 12.0, 1: 22.0}
+    q_new2 = mr.Query(1, 0.0, [(True, 5.0), (True, 5.0)])
+    thr = s["qos"] - s["tqueue"] - s["tori_solo"] - sum(s["earlier_remaining"])
+    assert thr == s["thr"] and q_new2.remaining() == 10.0
+
+
+def test_manager_fig13_schedule():
+    # Fig. 13: Q = [TC1, CD1, ..., TCn]; BE task 0 = [CD1, CD2]: Q-TC1 fuses with
+    # a BE CD kernel, later Q-CD kernels are followed by reordered BE kernels while headroom lasts.
+    q = mr.Query(0, 0.0, [(True, 2.0), (False, 1.0), (True, 2.0)])
+    apps = [mr.App([(True, 3.0), (True, 3.0)])]
+    fp = lambda ttc, tcd: 4.0 if ttc == 2.0 else None
+    res = mr.simulate([q], apps, 50.0, mr.TACKER, fp)
+    kinds = [e[0] for e in res["timeline"]]
+    assert kinds[0] == "fused"                   # FUSE1 = Q-TC1 + B-CD
+    assert "be" in kinds[1:]                     # a reordered BE kernel follows
+    assert res["latency"][0] <= 50.0
+
+
+def test_manager_qos_holds_and_tacker_beats_baymax():
+    rng = np.random.default_rng(3)
+    arrivals = np.cumsum(rng.exponential(20.0, 200))
+    mk = lambda: [mr.Query(i, float(t), [(True, 1.5), (False, 0.5)] * 4) for i, t in enumerate(arrivals)]
+    apps = lambda: [mr.App([(True, 2.0)]), mr.App([(True, 3.0), (True, 1.0)])]
+    fp = lambda ttc, tcd: max(ttc, tcd) + 0.2 * min(ttc, tcd)
+    out = {}
+    for pol in (mr.BAYMAX, mr.TACKER):
+        a = apps()
+        res = mr.simulate(mk(), a, 50.0, pol, fp, idle_cap=5.0)
+        assert max(res["latency"].values()) <= 50.0 + 1e-9
+        out[pol] = sum(x.completed for x in a) / res["t"]
+    assert out[mr.TACKER] > out[mr.BAYMAX]
+
+
+# ------------------------------------------------------------------ metrics
+def test_overlap_rate_bounds():
+    assert metrics.overlap_rate(1.0, 1.0, 1.0) == 0.5      # perfect overlap
+    assert metrics.overlap_rate(1.0, 1.0, 2.0) == 0.0      # sequential
+    assert metrics.throughput_improvement(118.6, 100.0) == pytest.approx(0.186)
+
+
+def test_rel_err_uses_abs_sum():
+    assert metrics.max_rel_err([1e-3], [0.0], [1.0]) == pytest.approx(1e-3)
+    assert metrics.max_rel_err([2.0], [1.0]) == 1.0
