@@ -1,0 +1,303 @@
+/*
+ * tacker.h — C ABI of the B200-native Tacker hot path (libtacker.so).
+ *
+ * Tacker (Zhao et al., HPCA'22; /root/reference/PAPER.md, cited P:a-b) co-runs a latency-
+ * critical (LC) tensor-core kernel and a best-effort (BE) CUDA-core kernel inside ONE fused
+ * kernel so both core types are busy at once (§III-B, §V), predicts the
+ * fused duration with a two-stage linear model (§VI) and decides at run time,
+ * from each LC query's QoS headroom, whether to launch the fused or the original kernels
+ * (§VII).  This header is the boundary: every call below is implemented by
+ * hand-written sm_100a CUDA (tcgen05/TMEM/TMA for LC, CUDA-core bodies for BE) and C++ host
+ * code; there is no CPU fallback.
+ *
+ * Conventions (all calls):
+ *   Errors     Every call returns tacker_status; nothing throws across the ABI.  The
+ *              thread-local message of the last failure is tacker_last_error().  CUDA runtime
+ *              failures map to TACKER_ECUDA.
+ *   Memory     Pointers inside descriptors are DEVICE pointers owned by the caller (e.g. torch
+ *              tensors).  The library never allocates or frees them.  Descriptors are copied at
+ *              tacker_fuse(); buffers must outlive every launch of the handle.  Handles own
+ *              their own small device workspace.
+ *   Streams    tacker_stream_t is a cudaStream_t (NULL = legacy default stream).  Launches are
+ *              asynchronous on that stream; predictor calls never touch the GPU.
+ *   Threads    Fused handles are immutable after tacker_fuse() and may be launched from any
+ *              thread.  A manager is single-threaded.  The model store is mutex-protected.
+ */
+#ifndef TACKER_H
+#define TACKER_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *tacker_stream_t;
+
+typedef enum {
+  TACKER_OK = 0,
+  TACKER_EINVAL = -1,        /* bad argument (null, negative size, inconsistent shape) */
+  TACKER_ERESOURCE = -2,     /* fused budget exceeds one SM: do not fuse */
+  TACKER_EUNSUPPORTED = -3,  /* shape/alignment/kind the kernels do not implement */
+  TACKER_ECUDA = -4,         /* CUDA runtime / driver error */
+  TACKER_ENOMODEL = -5,      /* predictor has no fitted model for this key */
+  TACKER_ENOMEM = -6
+} tacker_status;
+
+const char *tacker_last_error(void);
+/* Library version string and the SM count of the current device (0 without a GPU). */
+const char *tacker_version(void);
+int tacker_device_sm_count(void);
+
+/* ======================================================================== LC descriptors
+ * The LC part is the TC kernel "Kt" of the paper: an fp16 GEMM on tensor cores,
+ * or a convolution lowered to GEMM (§VIII-H, here as an implicit GEMM).
+ *
+ * GEMM   D[M,N] = A[M,K] . B[N,K]^T, A and B fp16 row-major with K contiguous ("K-major"),
+ *        fp32 accumulation in TMEM.  Constraints: K % 8 == 0 and N % 8 == 0 (16-byte TMA row
+ *        pitch), M >= 1 arbitrary (masked epilogue).  D row-major [M,N], fp32 or fp16 (RNE).
+ * CONV   out[n,p,q,k] = sum_{c,r,s} x[n, p*stride-pad+r, q*stride-pad+s, c] * w[k,r,s,c], x = 0
+ *        outside the image; x NHWC fp16 (A), w KRSC fp16 (B), out NHWC (D).  As a GEMM:
+ *        M = n*p*q, N = k, K = c*r*s.  Constraints: c % 64 == 0 or (r == s == 1 and c % 8 == 0)
+ *        or c == 8 (conv1 padded); k % 8 == 0.
+ * Epilogue (both): D = act(acc + bias[j] + residual[i,j]) with optional fp32 bias [N], fp16
+ *        residual with D's layout, ReLU.
+ */
+typedef enum { TACKER_LC_NONE = 0, TACKER_LC_GEMM_F16 = 1, TACKER_LC_CONV_F16 = 2 } tacker_lc_kind;
+enum { TACKER_F32 = 0, TACKER_F16 = 1 };
+enum { TACKER_EPI_BIAS = 1, TACKER_EPI_RELU = 2, TACKER_EPI_RESIDUAL = 4 };
+
+typedef struct {
+  int32_t kind;                       /* tacker_lc_kind */
+  int32_t M, N, K;                    /* GEMM shape (ignored for CONV: derived) */
+  int32_t n, h, w, c, k, r, s, stride, pad; /* CONV shape */
+  const void *A;                      /* GEMM A [M,K] fp16 | CONV x NHWC fp16 */
+  const void *B;                      /* GEMM B [N,K] fp16 | CONV w KRSC fp16 */
+  void *D;                            /* output, d_dtype */
+  const float *bias;                  /* [N] fp32 or NULL (requires TACKER_EPI_BIAS) */
+  const void *residual;               /* fp16 like D, or NULL (requires TACKER_EPI_RESIDUAL) */
+  int32_t d_dtype;                    /* TACKER_F32 | TACKER_F16 */
+  int32_t epi_flags;                  /* TACKER_EPI_* */
+  int32_t tile_n;                     /* LC tile N: 0 = auto, else 64 | 128 | 256 */
+} tacker_lc_desc;
+
+/* ======================================================================== BE descriptors
+ * The BE part is a CUDA-core kernel (Parboil-style, Table II).  Each kind defines
+ * its "original block" (one virtual block = 128 threads = 4 warps); `orig_blocks` is the
+ * PTB runtime argument of Fig. 7: 0 = the whole problem, else only blocks
+ * [0, orig_blocks) run (must not exceed the whole-problem count).  Bodies use fixed
+ * per-element arithmetic order, so a fused launch is bit-identical to the original one.
+ */
+typedef enum {
+  TACKER_BE_NONE = 0,
+  TACKER_BE_SGEMM = 1,        /* C = alpha A.B + beta C; block = 64x64 tile of C          */
+  TACKER_BE_STENCIL = 2,      /* 7-point Jacobi sweep; block = 32x4 columns, all z        */
+  TACKER_BE_MRIQ_PHIMAG = 3,  /* phiMag = phiR^2 + phiI^2; block = 512 k                   */
+  TACKER_BE_MRIQ_Q = 4,       /* Qr/Qi += sum_k phiMag cos/sin(2pi k.x); block = 256 voxels */
+  TACKER_BE_CUTCP = 5,        /* cutoff Coulomb potential; block = 4x4x8 lattice points    */
+  TACKER_BE_LBM = 6,          /* D3Q19 BGK push step; block = 128 cells along x            */
+  TACKER_BE_SPMV_JDS = 7,     /* y[perm[i]] = sum_d val*x[col]; block = 128 rows           */
+  TACKER_BE_HISTO = 8,        /* count[in[i]] += 1 (u32); block = 8192 inputs              */
+  TACKER_BE_BFS_EXPAND = 9,   /* Rodinia BFS kernel 1; block = 128 nodes                   */
+  TACKER_BE_BFS_COMMIT = 10,  /* Rodinia BFS kernel 2; block = 128 nodes                   */
+  TACKER_BE_FMA_BURN = 11,    /* register-only FMA chains (Kc, §III-B); block = 128 thr.   */
+  TACKER_BE_KIND_COUNT = 12
+} tacker_be_kind;
+
+typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
+typedef struct { int32_t nx, ny, nz; float c0, c1; const float *A0; float *Anext; } tacker_be_stencil;
+typedef struct { int32_t numK; const float *phiR, *phiI; float *phiMag; } tacker_be_mriq_phimag;
+typedef struct { int32_t numX, numK; const float *x, *y, *z, *kx, *ky, *kz, *phiMag; float *Qr, *Qi; } tacker_be_mriq_q;
+typedef struct {
+  int32_t nx, ny, nz;        /* lattice points per axis, point (i,j,k) at h*(i,j,k) */
+  float h, cutoff, excl;     /* spacing, cutoff radius, exclusion radius (Angstrom) */
+  int32_t bdim_x, bdim_y, bdim_z; /* atom bin grid (bin side = bin_size) */
+  float bin_size;
+  int32_t bin_depth;         /* atom slots per bin; unused slots have q == 0 and far coords */
+  const float *bins;         /* float4 (x,y,z,q) [bdim_z][bdim_y][bdim_x][bin_depth] */
+  float *V;                  /* [nz][ny][nx] */
+} tacker_be_cutcp;
+typedef struct { int32_t nx, ny, nz; const float *src; float *dst; const uint32_t *flags; } tacker_be_lbm;
+typedef struct { int32_t rows; const int32_t *perm, *row_len, *jds_ptr, *col; const float *val, *x; float *y; } tacker_be_spmv;
+typedef struct { int32_t n, nbins; const uint32_t *in; uint32_t *count; } tacker_be_histo;
+typedef struct { int32_t V; const int32_t *row_ptr, *col; int32_t *level; uint8_t *mask; const uint8_t *visited; uint8_t *upd; } tacker_be_bfs_expand;
+typedef struct { int32_t V; uint8_t *mask, *visited, *upd; int32_t *over; } tacker_be_bfs_commit;
+typedef struct { int32_t n_threads, iters; float a; float b; float *out; } tacker_be_fma_burn;
+
+typedef struct {
+  int32_t kind;              /* tacker_be_kind */
+  int32_t orig_blocks;       /* PTB original block count (0 = whole problem) */
+  union {
+    tacker_be_sgemm sgemm;
+    tacker_be_stencil stencil;
+    tacker_be_mriq_phimag mriq_phimag;
+    tacker_be_mriq_q mriq_q;
+    tacker_be_cutcp cutcp;
+    tacker_be_lbm lbm;
+    tacker_be_spmv spmv;
+    tacker_be_histo histo;
+    tacker_be_bfs_expand bfs_expand;
+    tacker_be_bfs_commit bfs_commit;
+    tacker_be_fma_burn fma_burn;
+    uint8_t _pad[128];
+  } p;
+} tacker_be_desc;
+
+/* Whole-problem block counts ("number of blocks in non-PTB mode", §VI-C). */
+tacker_status tacker_be_num_blocks(const tacker_be_desc *be, int64_t *out);
+tacker_status tacker_lc_num_tiles(const tacker_lc_desc *lc, int32_t tile_n, int64_t *out);
+
+/* ======================================================================== fusion (a1)
+ * tacker_fuse: admission + resource split of one fused kernel (§V-B/C P:1117-1309,
+ * §VIII-I).  One fused CTA per SM, persistent (PTB, Fig. 7):
+ *   warps [0,6)            LC: warp 0 TMA producer, warp 1 single-thread tcgen05.mma issuer
+ *                          (+ TMEM owner), warps 2..5 TMEM->register epilogue
+ *   warps [6, 6+warp_split) BE: block_ratio.be virtual blocks of 4 warps, each with its own
+ *                          named barrier (bar.sync 1+j, 128; Fig. 9) and SMEM slice
+ * warp_split  BE warps per CTA, a multiple of 4 in [4, 24] (0 = LC only; requires be NULL/NONE)
+ * block_ratio.lc  LC accumulator pipelines per CTA (TMEM stages, 1 or 2; 0 = auto)
+ * block_ratio.be  BE virtual blocks per CTA = warp_split/4 (0 = auto)
+ * LC is budgeted first (SMEM ring stages, TMEM columns), BE gets the rest (TC-first, §V-C).
+ * Returns TACKER_ERESOURCE when the aggregate does not fit (232,448 B SMEM, 512 TMEM columns,
+ * 64K registers, 32 warps, 16 barriers).  The handle owns encoded TMA tensor maps.
+ */
+typedef struct { uint8_t lc, be; } tacker_ratio;
+typedef struct tacker_fused_s *tacker_fused_t;
+
+tacker_status tacker_fuse(const tacker_lc_desc *lc, const tacker_be_desc *be, int32_t warp_split,
+                          tacker_ratio block_ratio, tacker_fused_t *out);
+tacker_status tacker_fused_destroy(tacker_fused_t f);
+
+typedef struct {
+  int32_t grid, block_threads, smem_bytes;
+  int32_t lc_warps, be_warps, be_vblocks_per_cta;
+  int32_t lc_tile_m, lc_tile_n, lc_tile_k, lc_stages, lc_acc_stages, tmem_cols;
+  int64_t lc_tiles, be_blocks;
+  int32_t be_smem_per_vblock, regs_per_thread;
+} tacker_fused_info_t;
+tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *out);
+/* Model-store keys of the handle's LC kernel, BE kernel and fused pair (for the predictor). */
+tacker_status tacker_fused_keys(tacker_fused_t f, char *lc_key, char *be_key, char *pair_key, size_t buflen);
+
+/* Retarget an existing handle to new buffers/PTB block count of the SAME shape class (no
+ * re-planning; used by the manager to reuse a plan).  NULL leaves that part unchanged. */
+tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, const tacker_be_desc *be);
+
+/* ======================================================================== launches (a2-a8)
+ * tacker_launch_fused    one fused kernel: LC tiles and BE blocks co-run in every CTA.
+ * tacker_launch_original the original kernels one after the other on the same stream (LC then
+ *                        BE); either may be NULL.  LC original = the same LC device code in a
+ *                        persistent LC-only grid; BE original = the same BE body in a
+ *                        non-persistent grid of orig_blocks CTAs of 128 threads (Fig. 7 "CD_kernel").
+ */
+tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream);
+tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be,
+                                     tacker_stream_t stream);
+
+/* ======================================================================== predictor (a9, a10)
+ * Per-kernel LR (§VI-C): X = a * blocks + b, keyed by kernel class.
+ * Two-stage fused model (Eqs. 1-6): r = X_cd / X_tc; T = X_tc * max(l1(r), l2(r)),
+ * fitted from samples at r in {0.1, 0.2, 1.8, 1.9}, refit online when the error
+ * exceeds 10%.  Keys are NUL-terminated strings (< 256 bytes).
+ */
+tacker_status tacker_model_add_sample(const char *key, double blocks, double ms);
+tacker_status tacker_model_fit(const char *key, double *a_out, double *b_out);
+tacker_status tacker_model_predict(const char *key, double blocks, double *ms_out);
+tacker_status tacker_pair_add_sample(const char *key, double x_tc, double x_cd, double t_fused);
+tacker_status tacker_pair_fit(const char *key, double coef_out[4] /* a1,b1,a2,b2; nullable */);
+tacker_status tacker_pair_predict(const char *key, double x_tc, double x_cd, double *ms_out);
+tacker_status tacker_pair_observe(const char *key, double x_tc, double x_cd, double t_meas, int32_t *refit_out);
+tacker_status tacker_model_clear(void);
+tacker_status tacker_model_save(const char *path);
+tacker_status tacker_model_load(const char *path);
+/* Fused duration of a handle: X_tc and X_cd from the kernel LRs of its LC/BE keys at the
+ * handle's tile / block counts, then the pair's two-stage model. */
+tacker_status tacker_predict_duration(tacker_fused_t f, double *ms_out);
+
+/* ======================================================================== manager (a11)
+ * QoS-aware kernel manager (§VII).  Rules: Eq. 9 headroom at the first issue of
+ * the newest query; per TC kernel Eq. 8 admission over ready BE heads, max Tgain, then
+ * Thr -= Tk_fuse - Ttc; otherwise original launch and reorder of ready BE heads with
+ * Ttmp < Thr.  Only the newest query fuses/reorders; Baymax policy = fusion disabled.
+ * The manager keeps its own clock: in simulation mode (stream == NULL and simulate != 0)
+ * kernels take their predicted duration; otherwise launches go to `stream` and completions
+ * are observed with CUDA events.
+ */
+typedef enum { TACKER_POLICY_TACKER = 0, TACKER_POLICY_BAYMAX = 1 } tacker_policy;
+typedef enum {
+  TACKER_DEC_FUSED = 0, TACKER_DEC_ORIGINAL_LC = 1, TACKER_DEC_REORDER_BE = 2,
+  TACKER_DEC_IDLE_BE = 3, TACKER_DEC_NOTHING = 4
+} tacker_action;
+#define TACKER_MAX_APPS 64
+#define TACKER_MAX_REORDER 64
+
+typedef struct {
+  int32_t is_tc;             /* 1: tensor-core kernel (fusable as LC); 0: CUDA-core kernel */
+  double t_pred_ms;          /* predicted standalone duration */
+  tacker_lc_desc lc;         /* used when is_tc */
+  tacker_be_desc cd;         /* used when !is_tc (an LC CUDA-core kernel launched original) */
+} tacker_lc_kernel;
+
+typedef struct {
+  int32_t n_kernels;
+  const tacker_lc_kernel *kernels;   /* copied at submit */
+} tacker_lc_query;
+
+typedef struct {
+  int32_t is_cd;             /* 1: CUDA-core kernel (fusable as BE) */
+  double t_pred_ms;
+  tacker_be_desc be;
+  int32_t warp_split;        /* fusion plan for this kernel (0 = library default 16) */
+} tacker_be_kernel;
+
+typedef struct {
+  int32_t n_kernels;
+  const tacker_be_kernel *kernels;   /* copied; the app cycles through them forever */
+} tacker_be_app;
+
+typedef struct {
+  int32_t action;            /* tacker_action */
+  int32_t query, lc_index;   /* LC kernel decided (-1 if none) */
+  int32_t fused_app;         /* BE app fused with it (-1 if none) */
+  int32_t n_reorder;
+  int32_t reorder_apps[TACKER_MAX_REORDER];
+  double thr_ms;             /* headroom after the decision */
+  double gain_ms;            /* Tgain of the fused pair */
+  double t_start_ms, t_end_ms; /* manager clock: predicted (sim) or issue time (GPU) */
+} tacker_decision;
+
+typedef struct {
+  double direct_eps_ms;      /* Thr <= this at first issue -> launch the query directly */
+  double idle_cap_ms;        /* idle GPU: launch BE heads no longer than this (<=0: any) */
+  int32_t max_inflight;      /* GPU mode: kernels allowed in flight on the stream (>=1) */
+  int32_t simulate;          /* 1: no GPU, durations = predictions */
+} tacker_manager_params;
+
+typedef struct tacker_manager_s *tacker_manager_t;
+
+tacker_status tacker_manager_create(int32_t policy, const tacker_manager_params *params,
+                                    tacker_stream_t stream, tacker_manager_t *out);
+tacker_status tacker_manager_destroy(tacker_manager_t m);
+tacker_status tacker_manager_submit_lc(tacker_manager_t m, const tacker_lc_query *q, double arrival_ms,
+                                       int32_t *query_id_out);
+tacker_status tacker_manager_submit_be(tacker_manager_t m, const tacker_be_app *app, int32_t *app_id_out);
+/* Register the predicted fused duration for (LC kernel t_pred class, BE app kernel); the
+ * manager asks the model store with the pair key of the fused handle it would build. */
+tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms);
+/* One decision at the manager's clock.  headroom_ms (in/out): on input the newest query's
+ * headroom, or NAN to use the manager's Eq. 9 value; on output the updated headroom. */
+tacker_status tacker_manager_step(tacker_manager_t m, double qos_target_ms, double *headroom_ms,
+                                  tacker_decision *out);
+typedef struct {
+  int64_t lc_queries_done, be_kernels_done, fused_launches, original_lc, reordered_be, idle_be;
+  double now_ms;
+} tacker_manager_stats;
+tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
+/* Completion time (manager clock) of a finished query, or -1 if unfinished. */
+tacker_status tacker_manager_query_latency(tacker_manager_t m, int32_t query_id, double *latency_ms);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TACKER_H */

@@ -1,0 +1,448 @@
+// be_bodies.cuh — BE (best-effort, CUDA-core) kernel bodies.
+//
+// Each body executes ONE original thread block ("virtual block", 128 threads = 4 warps) of a
+// Parboil/Rodinia-style kernel given its block id `vb` and the thread id `tid` rebased into
+// [0,128) (the "thread_step" of Fig. 5).  Partial-CTA synchronisation uses
+// `bar.sync bar_id, 128` (Fig. 9), never __syncthreads().  The same body is
+// called by the fused kernel (PTB loop, Fig. 7) and by the original non-persistent kernel,
+// so their outputs are bit-identical: all floating-point arithmetic uses explicit
+// round-to-nearest intrinsics (no FMA contraction differences between call sites) and a
+// per-element order that does not depend on which CTA runs the block.
+#pragma once
+#include <cuda_fp16.h>
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "tacker.h"
+
+namespace tk {
+
+constexpr int kVbThreads = 128;
+
+template <int KIND> struct BeBody;
+
+// ---------------------------------------------------------------- sgemm (Parboil)
+// C[M,N] = alpha * A[M,K] . B[K,N] + beta * C, row-major fp32.  Block = 64x64 tile of C,
+// thread (ty = tid/16, tx = tid%16) owns rows 8ty..8ty+7, cols 4tx..4tx+3.  K is staged in
+// chunks of 16 through double-buffered shared memory.  acc = fma(a_k, b_k, acc), k ascending.
+template <> struct BeBody<TACKER_BE_SGEMM> {
+  static constexpr int BM = 64, BN = 64, BK = 16;
+  static constexpr uint32_t kSmem = 2 * BK * (BM + 4) * 4 + 2 * BK * BN * 4;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_sgemm &p) {
+    return (int64_t)((p.M + BM - 1) / BM) * ((p.N + BN - 1) / BN);
+  }
+  static __device__ __forceinline__ void run(const tacker_be_sgemm &p, int64_t vb, int tid, uint32_t bar,
+                                             uint8_t *smem) {
+    float(*As)[BK][BM + 4] = reinterpret_cast<float(*)[BK][BM + 4]>(smem);
+    float(*Bs)[BK][BN] = reinterpret_cast<float(*)[BK][BN]>(smem + 2 * BK * (BM + 4) * 4);
+    const int tiles_n = (p.N + BN - 1) / BN;
+    const int m0 = (int)(vb / tiles_n) * BM, n0 = (int)(vb % tiles_n) * BN;
+    const int ty = tid >> 4, tx = tid & 15;
+    float acc[8][4];
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+
+    float4 ra[2], rb[2];
+    auto load = [&](int k0) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int idx = tid + h * 128;          // 256 float4 per operand tile
+        const int ar = idx >> 2, ac = (idx & 3) * 4;   // A: 64 rows x 4 float4
+        const int gm = m0 + ar, gk = k0 + ac;
+        ra[h] = (gm < p.M && gk < p.K) ? __ldg(reinterpret_cast<const float4 *>(p.A + (size_t)gm * p.K + gk))
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+        const int br = idx >> 4, bc = (idx & 15) * 4;  // B: 16 rows x 16 float4
+        const int gk2 = k0 + br, gn = n0 + bc;
+        rb[h] = (gk2 < p.K && gn < p.N) ? __ldg(reinterpret_cast<const float4 *>(p.B + (size_t)gk2 * p.N + gn))
+                                       : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    };
+    auto store = [&](int buf) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int idx = tid + h * 128;
+        const int ar = idx >> 2, ac = (idx & 3) * 4;
+        As[buf][ac + 0][ar] = ra[h].x;
+        As[buf][ac + 1][ar] = ra[h].y;
+        As[buf][ac + 2][ar] = ra[h].z;
+        As[buf][ac + 3][ar] = ra[h].w;
+        const int br = idx >> 4, bc = (idx & 15) * 4;
+        *reinterpret_cast<float4 *>(&Bs[buf][br][bc]) = rb[h];
+      }
+    };
+    const int nk = (p.K + BK - 1) / BK;
+    load(0);
+    store(0);
+    named_bar_sync(bar, kVbThreads);
+    for (int kc = 0; kc < nk; ++kc) {
+      const int buf = kc & 1;
+      if (kc + 1 < nk) load((kc + 1) * BK);
+#pragma unroll
+      for (int k = 0; k < BK; ++k) {
+        const float4 a0 = *reinterpret_cast<const float4 *>(&As[buf][k][ty * 8]);
+        const float4 a1 = *reinterpret_cast<const float4 *>(&As[buf][k][ty * 8 + 4]);
+        const float4 b = *reinterpret_cast<const float4 *>(&Bs[buf][k][tx * 4]);
+        const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const float bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+      }
+      if (kc + 1 < nk) store(buf ^ 1);
+      named_bar_sync(bar, kVbThreads);
+    }
+    const int gn = n0 + tx * 4;
+    if (gn >= p.N) return;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int gm = m0 + ty * 8 + i;
+      if (gm >= p.M) break;
+      float *c = p.C + (size_t)gm * p.N + gn;
+      float4 o;
+      if (p.beta != 0.f) {
+        const float4 ci = *reinterpret_cast<const float4 *>(c);
+        o.x = __fadd_rn(__fmul_rn(p.alpha, acc[i][0]), __fmul_rn(p.beta, ci.x));
+        o.y = __fadd_rn(__fmul_rn(p.alpha, acc[i][1]), __fmul_rn(p.beta, ci.y));
+        o.z = __fadd_rn(__fmul_rn(p.alpha, acc[i][2]), __fmul_rn(p.beta, ci.z));
+        o.w = __fadd_rn(__fmul_rn(p.alpha, acc[i][3]), __fmul_rn(p.beta, ci.w));
+      } else {
+        o.x = __fmul_rn(p.alpha, acc[i][0]);
+        o.y = __fmul_rn(p.alpha, acc[i][1]);
+        o.z = __fmul_rn(p.alpha, acc[i][2]);
+        o.w = __fmul_rn(p.alpha, acc[i][3]);
+      }
+      *reinterpret_cast<float4 *>(c) = o;
+    }
+  }
+};
+
+// ---------------------------------------------------------------- fma_burn ("Kc", §III-B)
+// Register-only FMA chains: thread g = vb*128+tid runs x_j <- fma(x_j, a, (j+1) b), j < 4,
+// from x_j = (g%97 + j)/128, for `iters` steps; out[g] = ((x0+x1)+x2)+x3.
+template <> struct BeBody<TACKER_BE_FMA_BURN> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_fma_burn &p) {
+    return (p.n_threads + kVbThreads - 1) / kVbThreads;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_fma_burn &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+    const int64_t g = vb * kVbThreads + tid;
+    if (g >= p.n_threads) return;
+    const float base = (float)(g % 97);
+    float x0 = __fdiv_rn(base + 0.f, 128.f), x1 = __fdiv_rn(base + 1.f, 128.f);
+    float x2 = __fdiv_rn(base + 2.f, 128.f), x3 = __fdiv_rn(base + 3.f, 128.f);
+    const float a = p.a, b0 = p.b, b1 = __fmul_rn(2.f, p.b), b2 = __fmul_rn(3.f, p.b), b3 = __fmul_rn(4.f, p.b);
+#pragma unroll 4
+    for (int it = 0; it < p.iters; ++it) {
+      x0 = __fmaf_rn(x0, a, b0);
+      x1 = __fmaf_rn(x1, a, b1);
+      x2 = __fmaf_rn(x2, a, b2);
+      x3 = __fmaf_rn(x3, a, b3);
+    }
+    p.out[g] = __fadd_rn(__fadd_rn(__fadd_rn(x0, x1), x2), x3);
+  }
+};
+
+// ---------------------------------------------------------------- stencil (Parboil)
+// One 7-point Jacobi sweep over A0[nz][ny][nx] (x fastest).  Block = 32x4 (x,y) columns,
+// swept over all z with the column's z-1/z/z+1 values in registers; x+-1, y+-1 neighbours come
+// through L1.  Interior: An = c1*(((((W+E)+S)+N)+B)+T) - c0*A; boundary cells copied.
+template <> struct BeBody<TACKER_BE_STENCIL> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_stencil &p) {
+    return (int64_t)((p.nx + 31) / 32) * ((p.ny + 3) / 4);
+  }
+  static __device__ __forceinline__ void run(const tacker_be_stencil &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+    const int bx = (p.nx + 31) / 32;
+    const int x = (int)(vb % bx) * 32 + (tid & 31);
+    const int y = (int)(vb / bx) * 4 + (tid >> 5);
+    if (x >= p.nx || y >= p.ny) return;
+    const size_t plane = (size_t)p.nx * p.ny;
+    const float *A = p.A0;
+    float *An = p.Anext;
+    const size_t col = (size_t)y * p.nx + x;
+    const bool border = (x == 0) | (x == p.nx - 1) | (y == 0) | (y == p.ny - 1) | (p.nz < 3);
+    if (border) {
+      for (int z = 0; z < p.nz; ++z) An[z * plane + col] = __ldg(A + z * plane + col);
+      return;
+    }
+    float below = __ldg(A + col);
+    float cur = __ldg(A + plane + col);
+    An[col] = below;
+    for (int z = 1; z < p.nz - 1; ++z) {
+      const size_t o = z * plane + col;
+      const float above = __ldg(A + o + plane);
+      const float w = __ldg(A + o - 1), e = __ldg(A + o + 1);
+      const float s = __ldg(A + o - p.nx), n = __ldg(A + o + p.nx);
+      float sum = __fadd_rn(w, e);
+      sum = __fadd_rn(sum, s);
+      sum = __fadd_rn(sum, n);
+      sum = __fadd_rn(sum, below);
+      sum = __fadd_rn(sum, above);
+      An[o] = __fsub_rn(__fmul_rn(p.c1, sum), __fmul_rn(p.c0, cur));
+      below = cur;
+      cur = above;
+    }
+    An[(size_t)(p.nz - 1) * plane + col] = cur;
+  }
+};
+
+// ---------------------------------------------------------------- mri-q (Parboil)
+template <> struct BeBody<TACKER_BE_MRIQ_PHIMAG> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_phimag &p) { return (p.numK + 511) / 512; }
+  static __device__ __forceinline__ void run(const tacker_be_mriq_phimag &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+#pragma unroll
+    for (int h = 0; h < 4; ++h) {
+      const int64_t k = vb * 512 + h * 128 + tid;
+      if (k < p.numK) {
+        const float r = p.phiR[k], i = p.phiI[k];
+        p.phiMag[k] = __fadd_rn(__fmul_rn(r, r), __fmul_rn(i, i));
+      }
+    }
+  }
+};
+
+// Q: block = 256 voxels (thread owns tid and tid+128); k staged through shared memory in
+// chunks of 512 as float4 (kx, ky, kz, phiMag).  Phase in turns t = kx x + ky y + kz z is
+// range-reduced exactly (t - rint(t), Sterbenz) before the MUFU sin/cos of 2*pi*t.
+template <> struct BeBody<TACKER_BE_MRIQ_Q> {
+  static constexpr int KC = 512;
+  static constexpr uint32_t kSmem = KC * 16;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) { return (p.numX + 255) / 256; }
+  static __device__ __forceinline__ void run(const tacker_be_mriq_q &p, int64_t vb, int tid, uint32_t bar,
+                                             uint8_t *smem) {
+    float4 *ks = reinterpret_cast<float4 *>(smem);
+    const float kTwoPi = 6.2831853071795864769f;
+    int64_t v[2] = {vb * 256 + tid, vb * 256 + 128 + tid};
+    float xs[2], ys[2], zs[2], qr[2], qi[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const bool ok = v[h] < p.numX;
+      xs[h] = ok ? p.x[v[h]] : 0.f;
+      ys[h] = ok ? p.y[v[h]] : 0.f;
+      zs[h] = ok ? p.z[v[h]] : 0.f;
+      qr[h] = ok ? p.Qr[v[h]] : 0.f;
+      qi[h] = ok ? p.Qi[v[h]] : 0.f;
+    }
+    for (int k0 = 0; k0 < p.numK; k0 += KC) {
+      const int kn = min(KC, p.numK - k0);
+      named_bar_sync(bar, kVbThreads);  // previous chunk fully consumed
+      for (int k = tid; k < kn; k += kVbThreads)
+        ks[k] = make_float4(p.kx[k0 + k], p.ky[k0 + k], p.kz[k0 + k], p.phiMag[k0 + k]);
+      named_bar_sync(bar, kVbThreads);
+#pragma unroll 4
+      for (int k = 0; k < kn; ++k) {
+        const float4 kv = ks[k];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          float t = __fmaf_rn(kv.z, zs[h], __fmaf_rn(kv.y, ys[h], __fmul_rn(kv.x, xs[h])));
+          t = __fsub_rn(t, rintf(t));
+          const float arg = __fmul_rn(kTwoPi, t);
+          float s, c;
+          __sincosf(arg, &s, &c);
+          qr[h] = __fmaf_rn(kv.w, c, qr[h]);
+          qi[h] = __fmaf_rn(kv.w, s, qi[h]);
+        }
+      }
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+      if (v[h] < p.numX) {
+        p.Qr[v[h]] = qr[h];
+        p.Qi[v[h]] = qi[h];
+      }
+  }
+};
+
+// ---------------------------------------------------------------- lbm (Parboil)
+// D3Q19 BGK push step, SoA src/dst [19][cells], block = 128 consecutive cells (x fastest).
+// Direction order C N S E W T B NE NW SE SW NT NB ST SB ET EB WT WB.
+__constant__ int8_t kLbmE[19][3] = {{0, 0, 0},  {0, 1, 0},  {0, -1, 0}, {1, 0, 0},   {-1, 0, 0},
+                                    {0, 0, 1},  {0, 0, -1}, {1, 1, 0},  {-1, 1, 0},  {1, -1, 0},
+                                    {-1, -1, 0}, {0, 1, 1}, {0, 1, -1}, {0, -1, 1},  {0, -1, -1},
+                                    {1, 0, 1},  {1, 0, -1}, {-1, 0, 1}, {-1, 0, -1}};
+__constant__ int8_t kLbmOpp[19] = {0, 2, 1, 4, 3, 6, 5, 10, 9, 8, 7, 14, 13, 12, 11, 18, 17, 16, 15};
+
+template <> struct BeBody<TACKER_BE_LBM> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_lbm &p) {
+    return ((int64_t)p.nx * p.ny * p.nz + 127) / 128;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_lbm &p, int64_t vb, int tid, uint32_t, uint8_t *) {
+    const int64_t cells = (int64_t)p.nx * p.ny * p.nz;
+    const int64_t idx = vb * 128 + tid;
+    if (idx >= cells) return;
+    const int x = (int)(idx % p.nx), y = (int)((idx / p.nx) % p.ny), z = (int)(idx / ((int64_t)p.nx * p.ny));
+    const uint32_t flag = p.flags[idx];
+    float f[19];
+#pragma unroll
+    for (int i = 0; i < 19; ++i) f[i] = __ldg(p.src + i * cells + idx);
+    const float w[19] = {1.f / 3.f,  1.f / 18.f, 1.f / 18.f, 1.f / 18.f, 1.f / 18.f, 1.f / 18.f, 1.f / 18.f,
+                         1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f,
+                         1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f, 1.f / 36.f};
+    if (flag == 1u) {  // OBSTACLE: dst_{opp(i)}[x + e_opp(i)] = src_i[x]
+#pragma unroll
+      for (int i = 0; i < 19; ++i) {
+        const int j = kLbmOpp[i];
+        const int tx = x + kLbmE[j][0], ty = y + kLbmE[j][1], tz = z + kLbmE[j][2];
+        if (tx >= 0 && tx < p.nx && ty >= 0 && ty < p.ny && tz >= 0 && tz < p.nz)
+          p.dst[j * cells + ((int64_t)tz * p.ny + ty) * p.nx + tx] = f[i];
+      }
+      return;
+    }
+    float rho = 0.f, ux = 0.f, uy = 0.f, uz = 0.f;
+#pragma unroll
+    for (int i = 0; i < 19; ++i) {
+      rho = __fadd_rn(rho, f[i]);
+      if (kLbmE[i][0] > 0) ux = __fadd_rn(ux, f[i]);
+      if (kLbmE[i][0] < 0) ux = __fsub_rn(ux, f[i]);
+      if (kLbmE[i][1] > 0) uy = __fadd_rn(uy, f[i]);
+      if (kLbmE[i][1] < 0) uy = __fsub_rn(uy, f[i]);
+      if (kLbmE[i][2] > 0) uz = __fadd_rn(uz, f[i]);
+      if (kLbmE[i][2] < 0) uz = __fsub_rn(uz, f[i]);
+    }
+    ux = __fdiv_rn(ux, rho);
+    uy = __fdiv_rn(uy, rho);
+    uz = __fdiv_rn(uz, rho);
+    if (flag == 2u) {  // ACCEL
+      ux = 0.005f;
+      uy = 0.002f;
+      uz = 0.f;
+    }
+    const float u2 = __fadd_rn(__fadd_rn(__fmul_rn(ux, ux), __fmul_rn(uy, uy)), __fmul_rn(uz, uz));
+    const float omega = 1.95f;
+    const float one_m = __fsub_rn(1.f, omega);
+#pragma unroll
+    for (int i = 0; i < 19; ++i) {
+      float eu = 0.f;
+      if (kLbmE[i][0] != 0) eu = __fadd_rn(eu, kLbmE[i][0] > 0 ? ux : -ux);
+      if (kLbmE[i][1] != 0) eu = __fadd_rn(eu, kLbmE[i][1] > 0 ? uy : -uy);
+      if (kLbmE[i][2] != 0) eu = __fadd_rn(eu, kLbmE[i][2] > 0 ? uz : -uz);
+      // feq = w rho (1 + 3 eu + 4.5 eu^2 - 1.5 u2)
+      float poly = __fadd_rn(1.f, __fmul_rn(3.f, eu));
+      poly = __fadd_rn(poly, __fmul_rn(4.5f, __fmul_rn(eu, eu)));
+      poly = __fsub_rn(poly, __fmul_rn(1.5f, u2));
+      const float feq = __fmul_rn(__fmul_rn(w[i], rho), poly);
+      const float out = __fadd_rn(__fmul_rn(one_m, f[i]), __fmul_rn(omega, feq));
+      const int tx = x + kLbmE[i][0], ty = y + kLbmE[i][1], tz = z + kLbmE[i][2];
+      if (tx >= 0 && tx < p.nx && ty >= 0 && ty < p.ny && tz >= 0 && tz < p.nz)
+        p.dst[i * cells + ((int64_t)tz * p.ny + ty) * p.nx + tx] = out;
+    }
+  }
+};
+
+// ---------------------------------------------------------------- spmv JDS (Parboil)
+// Thread per JDS row i (block = 128 rows): y[perm[i]] = sum_{d<row_len[i]} val*x[col] at
+// jds_ptr[d]+i, d ascending; consecutive i touch consecutive addresses of each diagonal.
+template <> struct BeBody<TACKER_BE_SPMV_JDS> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_spmv &p) { return (p.rows + 127) / 128; }
+  static __device__ __forceinline__ void run(const tacker_be_spmv &p, int64_t vb, int tid, uint32_t, uint8_t *) {
+    const int64_t i = vb * 128 + tid;
+    if (i >= p.rows) return;
+    const int len = p.row_len[i];
+    float acc = 0.f;
+    for (int d = 0; d < len; ++d) {
+      const int64_t e = (int64_t)__ldg(p.jds_ptr + d) + i;
+      acc = __fmaf_rn(__ldg(p.val + e), __ldg(p.x + __ldg(p.col + e)), acc);
+    }
+    p.y[p.perm[i]] = acc;
+  }
+};
+
+// ---------------------------------------------------------------- histo
+// Block = 32768 inputs: a private u32 histogram of nbins (<= 8192) in shared memory, then one
+// global atomicAdd per non-empty bin.  Integer adds commute: bit-exact whatever the order.
+template <> struct BeBody<TACKER_BE_HISTO> {
+  static constexpr int PER_BLOCK = 32768;
+  static constexpr uint32_t kSmem = 8192 * 4;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_histo &p) {
+    return ((int64_t)p.n + PER_BLOCK - 1) / PER_BLOCK;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_histo &p, int64_t vb, int tid, uint32_t bar,
+                                             uint8_t *smem) {
+    uint32_t *h = reinterpret_cast<uint32_t *>(smem);
+    for (int b = tid; b < p.nbins; b += kVbThreads) h[b] = 0;
+    named_bar_sync(bar, kVbThreads);
+    const int64_t base = vb * PER_BLOCK;
+    const int64_t end = min((int64_t)p.n, base + PER_BLOCK);
+    if (base + PER_BLOCK <= p.n && (p.n & 3) == 0) {
+      const uint4 *in4 = reinterpret_cast<const uint4 *>(p.in + base);
+#pragma unroll 4
+      for (int i = tid; i < PER_BLOCK / 4; i += kVbThreads) {
+        const uint4 v = __ldg(in4 + i);
+        atomicAdd(&h[v.x], 1u);
+        atomicAdd(&h[v.y], 1u);
+        atomicAdd(&h[v.z], 1u);
+        atomicAdd(&h[v.w], 1u);
+      }
+    } else {
+      for (int64_t i = base + tid; i < end; i += kVbThreads) atomicAdd(&h[__ldg(p.in + i)], 1u);
+    }
+    named_bar_sync(bar, kVbThreads);
+    for (int b = tid; b < p.nbins; b += kVbThreads) {
+      const uint32_t c = h[b];
+      if (c) atomicAdd(p.count + b, c);
+    }
+    named_bar_sync(bar, kVbThreads);  // shared histogram reusable by the next block
+  }
+};
+
+// ---------------------------------------------------------------- bfs (Rodinia kernels 1 and 2)
+template <> struct BeBody<TACKER_BE_BFS_EXPAND> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_bfs_expand &p) { return (p.V + 127) / 128; }
+  static __device__ __forceinline__ void run(const tacker_be_bfs_expand &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+    const int64_t v = vb * 128 + tid;
+    if (v >= p.V || !p.mask[v]) return;
+    p.mask[v] = 0;
+    const int lv = p.level[v] + 1;
+    for (int e = p.row_ptr[v]; e < p.row_ptr[v + 1]; ++e) {
+      const int u = p.col[e];
+      if (!p.visited[u]) {
+        p.level[u] = lv;
+        p.upd[u] = 1;
+      }
+    }
+  }
+};
+template <> struct BeBody<TACKER_BE_BFS_COMMIT> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_bfs_commit &p) { return (p.V + 127) / 128; }
+  static __device__ __forceinline__ void run(const tacker_be_bfs_commit &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+    const int64_t u = vb * 128 + tid;
+    if (u >= p.V || !p.upd[u]) return;
+    p.mask[u] = 1;
+    p.visited[u] = 1;
+    p.upd[u] = 0;
+    *p.over = 1;
+  }
+};
+
+// ---------------------------------------------------------------- dispatch helpers
+template <int KIND> struct BeSel;
+#define TK_BE_SEL(K, FIELD)                                                            \
+  template <> struct BeSel<K> {                                                        \
+    static __host__ __device__ const auto &get(const tacker_be_desc &d) { return d.p.FIELD; } \
+  };
+TK_BE_SEL(TACKER_BE_SGEMM, sgemm)
+TK_BE_SEL(TACKER_BE_STENCIL, stencil)
+TK_BE_SEL(TACKER_BE_MRIQ_PHIMAG, mriq_phimag)
+TK_BE_SEL(TACKER_BE_MRIQ_Q, mriq_q)
+TK_BE_SEL(TACKER_BE_LBM, lbm)
+TK_BE_SEL(TACKER_BE_SPMV_JDS, spmv)
+TK_BE_SEL(TACKER_BE_HISTO, histo)
+TK_BE_SEL(TACKER_BE_BFS_EXPAND, bfs_expand)
+TK_BE_SEL(TACKER_BE_BFS_COMMIT, bfs_commit)
+TK_BE_SEL(TACKER_BE_FMA_BURN, fma_burn)
+#undef TK_BE_SEL
+
+}  // namespace tk

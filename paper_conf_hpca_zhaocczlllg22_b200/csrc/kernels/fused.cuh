@@ -1,0 +1,322 @@
+// fused.cuh — the Tensor-CUDA core fused kernel for sm_100a (Tacker §V).
+//
+// One persistent CTA per SM (PTB, Fig. 7).  Warp roles (the B200 analogue of
+// Fig. 5's thread ranges):
+//   warp 0            LC TMA producer (one elected lane): A/B k-blocks into an S-stage ring
+//   warp 1            LC MMA issuer (one lane) + TMEM owner: tcgen05.mma kind::f16 into TMEM
+//   warps 2..5        LC epilogue: tcgen05.ld 32x32b -> bias/residual/ReLU -> st.global
+//   warps 6..6+4V-1   BE: V virtual blocks of 4 warps; vblock j uses bar.sync 1+j, 128 (Fig. 9)
+// LC-only (original LC) launches have V = 0; the BE original kernel is be_original_kernel.
+// LC and BE share no barrier inside the main loops; bar.sync 0 is used only in the prologue
+// (barrier init, TMEM alloc) and the teardown (TMEM dealloc).
+#pragma once
+#include <cuda_fp16.h>
+#include <cstdint>
+
+#include "be_bodies.cuh"
+#include "ptx.cuh"
+#include "tacker.h"
+
+namespace tk {
+
+constexpr int kLcWarps = 6;
+constexpr int kBM = 128;   // UMMA M
+constexpr int kBK = 64;    // one 128-byte swizzle row of fp16
+constexpr int kUK = 16;    // UMMA K for kind::f16
+
+struct LcParams {
+  int32_t kind;            // tacker_lc_kind (0 = no LC part)
+  int32_t M, N, K;         // GEMM view
+  int32_t tiles_m, tiles_n, num_kb;
+  int32_t num_tiles;
+  void *D;
+  int32_t d_f16, epi;
+  const float *bias;
+  const __half *residual;
+  // implicit-GEMM conv view (kind == CONV)
+  int32_t n, h, w, c, k, r, s, stride, pad, p, q;
+  int32_t tp, tq;          // output tile = tp x tq positions (tp*tq == 128)
+  int32_t tiles_p, tiles_q, c_blocks;
+  int32_t conv_direct_gemm;  // 1x1 stride-1 conv handled as a plain GEMM over [n*h*w, c]
+};
+
+struct BeWork {
+  uint32_t ticket;         // next virtual block (atomic, self-resetting)
+  uint32_t done;           // vblock groups that finished
+};
+
+struct alignas(64) FusedParams {
+  CUtensorMap tmap_a;      // A / x operand
+  CUtensorMap tmap_b;      // B / w operand
+  LcParams lc;
+  tacker_be_desc be;
+  int64_t be_blocks;       // original blocks to run (PTB original_block_num)
+  BeWork *work;            // device workspace for the BE ticket
+  int32_t be_vb_per_cta;   // virtual blocks per CTA
+  int32_t lc_warps;        // 6 or 0
+  int32_t stages;          // SMEM ring depth
+  int32_t acc_stages;      // TMEM accumulator buffers
+  uint32_t tmem_cols;
+  uint32_t lc_smem_bytes;  // ring + barriers, 1024-aligned start
+  uint32_t be_smem_per_vb; // per-vblock slice (incl. 16 B ticket slot)
+};
+
+// ------------------------------------------------------------------------ LC roles
+template <int BN>
+struct LcGemm {
+  static constexpr uint32_t kStageA = kBM * kBK * 2;
+  static constexpr uint32_t kStageB = BN * kBK * 2;
+  static constexpr uint32_t kStage = kStageA + kStageB;
+  static constexpr uint32_t kIdesc = umma_idesc_f16(kBM, BN);
+
+  struct Bars {
+    uint64_t *full, *empty, *tfull, *tempty;
+    uint32_t *tmem_holder;
+  };
+  static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages) {
+    uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * kStage);
+    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4)};
+  }
+
+  static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
+    // N-tiles fastest: consecutive CTAs share the A rows (L2 reuse of the activation tile)
+    mt = t / L.tiles_n;
+    nt = t % L.tiles_n;
+  }
+
+  static __device__ __forceinline__ void producer(const FusedParams &P, uint8_t *lc, const Bars &bb) {
+    const LcParams &L = P.lc;
+    int stage = 0;
+    uint32_t phase = 0;
+    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
+      int mt, nt;
+      tile_coords(L, t, mt, nt);
+      for (int kb = 0; kb < L.num_kb; ++kb) {
+        mbar_wait(&bb.empty[stage], phase ^ 1);
+        uint8_t *sa = lc + stage * kStage;
+        uint8_t *sb = sa + kStageA;
+        mbar_arrive_expect_tx(&bb.full[stage], kStage);
+        if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
+          // k-block -> (filter tap r,s ; channel block cb); A = shifted NHWC window (implicit im2col)
+          const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
+          const int rr = rs / L.s, ss = rs % L.s;
+          const int img = mt / (L.tiles_p * L.tiles_q);
+          const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
+          const int h0 = pt * L.tp * L.stride - L.pad + rr;
+          const int w0 = qt * L.tq * L.stride - L.pad + ss;
+          tma_load_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, w0, h0, img);
+          // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
+          tma_load_2d(&P.tmap_b, &bb.full[stage], sb, rs * L.c + cb * kBK, nt * BN);
+        } else {
+          tma_load_2d(&P.tmap_a, &bb.full[stage], sa, kb * kBK, mt * kBM);
+          tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);
+        }
+        if (++stage == P.stages) {
+          stage = 0;
+          phase ^= 1;
+        }
+      }
+    }
+  }
+
+  static __device__ __forceinline__ void mma(const FusedParams &P, uint8_t *lc, const Bars &bb, uint32_t tmem) {
+    const LcParams &L = P.lc;
+    int stage = 0, acc = 0;
+    uint32_t phase = 0, acc_phase = 0;
+    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
+      mbar_wait(&bb.tempty[acc], acc_phase ^ 1);
+      tc_fence_after();
+      const uint32_t d = tmem + acc * BN;
+      for (int kb = 0; kb < L.num_kb; ++kb) {
+        mbar_wait(&bb.full[stage], phase);
+        tc_fence_after();
+        const uint32_t sa = smem_u32(lc + stage * kStage);
+        const uint32_t sb = sa + kStageA;
+#pragma unroll
+        for (int k = 0; k < kBK / kUK; ++k) {
+          umma_f16(d, umma_desc_sw128(sa + k * kUK * 2), umma_desc_sw128(sb + k * kUK * 2), kIdesc,
+                   (kb | k) != 0);
+        }
+        umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
+        if (++stage == P.stages) {
+          stage = 0;
+          phase ^= 1;
+        }
+      }
+      umma_commit(&bb.tfull[acc]);        // accumulator ready for the epilogue
+      if (++acc == P.acc_stages) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+  }
+
+  static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem) {
+    const LcParams &L = P.lc;
+    const int quarter = warp_id() & 3;          // TMEM lanes 32*quarter .. +31
+    const int row_in_tile = quarter * 32 + lane_id();
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
+      int mt, nt;
+      tile_coords(L, t, mt, nt);
+      mbar_wait(&bb.tfull[acc], acc_phase);
+      tc_fence_after();
+      // output row of this thread
+      int64_t orow = -1;
+      if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
+        const int img = mt / (L.tiles_p * L.tiles_q);
+        const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
+        const int pp = pt * L.tp + row_in_tile / L.tq, qq = qt * L.tq + row_in_tile % L.tq;
+        if (pp < L.p && qq < L.q) orow = ((int64_t)img * L.p + pp) * L.q + qq;
+      } else {
+        const int m = mt * kBM + row_in_tile;
+        if (m < L.M) orow = m;
+      }
+      const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN; c0 += 32) {
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(tbase + c0, v);
+        tmem_ld_wait();
+        const int n0 = nt * BN + c0;
+        if (orow >= 0 && n0 < L.N) {
+          float f[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) f[j] = __uint_as_float(v[j]);
+          if (L.epi & TACKER_EPI_BIAS) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (n0 + j < L.N) f[j] = __fadd_rn(f[j], __ldg(L.bias + n0 + j));
+          }
+          if (L.epi & TACKER_EPI_RESIDUAL) {
+            const __half *rp = L.residual + orow * L.N + n0;
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (n0 + j < L.N) f[j] = __fadd_rn(f[j], __half2float(rp[j]));
+          }
+          if (L.epi & TACKER_EPI_RELU) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) f[j] = fmaxf(f[j], 0.f);
+          }
+          if (L.d_f16) {
+            __half *dp = reinterpret_cast<__half *>(L.D) + orow * L.N + n0;
+#pragma unroll
+            for (int j = 0; j < 32; j += 8) {
+              if (n0 + j < L.N) {  // N % 8 == 0: a group of 8 is all in or all out
+                __align__(16) __half2 hv[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) hv[u] = __floats2half2_rn(f[j + 2 * u], f[j + 2 * u + 1]);
+                *reinterpret_cast<uint4 *>(dp + j) = *reinterpret_cast<uint4 *>(hv);
+              }
+            }
+          } else {
+            float *dp = reinterpret_cast<float *>(L.D) + orow * L.N + n0;
+#pragma unroll
+            for (int j = 0; j < 32; j += 4)
+              if (n0 + j < L.N) *reinterpret_cast<float4 *>(dp + j) = make_float4(f[j], f[j + 1], f[j + 2], f[j + 3]);
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&bb.tempty[acc]);
+      if (++acc == P.acc_stages) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+  }
+};
+
+// ------------------------------------------------------------------------ BE PTB loop
+template <int BE_KIND>
+__device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_smem) {
+  const int be_warp = warp_id() - P.lc_warps;
+  const int j = be_warp >> 2;                       // virtual block slot in this CTA
+  const int tid = threadIdx.x - 32 * P.lc_warps - kVbThreads * j;   // thread_step rebase (Fig. 5)
+  const uint32_t bar = 1 + j;                       // named barrier id (0 is reserved)
+  uint8_t *slice = be_smem + (size_t)j * P.be_smem_per_vb;
+  volatile uint32_t *s_ticket = reinterpret_cast<volatile uint32_t *>(slice);
+  uint8_t *body_smem = slice + 16;
+  const auto &bp = BeSel<BE_KIND>::get(P.be);
+  for (;;) {
+    if (tid == 0) *s_ticket = atomicAdd(&P.work->ticket, 1u);
+    named_bar_sync(bar, kVbThreads);
+    const int64_t vb = *s_ticket;
+    named_bar_sync(bar, kVbThreads);
+    if (vb >= P.be_blocks) break;
+    BeBody<BE_KIND>::run(bp, vb, tid, bar, body_smem);
+  }
+  if (tid == 0) {
+    __threadfence();
+    const uint32_t groups = gridDim.x * (uint32_t)P.be_vb_per_cta;
+    if (atomicAdd(&P.work->done, 1u) == groups - 1) {   // last group: reset for the next launch
+      P.work->ticket = 0;
+      P.work->done = 0;
+      __threadfence();
+    }
+  }
+}
+
+// ------------------------------------------------------------------------ the fused kernel
+template <int BN, int BE_KIND>
+__global__ void __launch_bounds__(32 * (kLcWarps + 16), 1) fused_kernel(const __grid_constant__ FusedParams P) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t *lc = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t *be_smem = lc + P.lc_smem_bytes;
+  const int warp = warp_id();
+  const bool has_lc = P.lc_warps > 0 && P.lc.num_tiles > 0;
+  typename LcGemm<BN>::Bars bb{};
+  if (P.lc_warps > 0) {
+    bb = LcGemm<BN>::bars(lc, P.stages);
+    if (warp == 0 && lane_id() == 0) {
+      tma_prefetch_desc(&P.tmap_a);
+      tma_prefetch_desc(&P.tmap_b);
+      for (int s = 0; s < P.stages; ++s) {
+        mbar_init(&bb.full[s], 1);
+        mbar_init(&bb.empty[s], 1);
+      }
+      for (int a = 0; a < 2; ++a) {
+        mbar_init(&bb.tfull[a], 1);
+        mbar_init(&bb.tempty[a], 4 * 32);
+      }
+      fence_barrier_init();
+    }
+    if (warp == 1 && has_lc) tmem_alloc(bb.tmem_holder, P.tmem_cols);
+  }
+  tc_fence_before();
+  __syncthreads();   // bar.sync 0: prologue only
+  tc_fence_after();
+
+  if (warp < P.lc_warps) {
+    if (has_lc) {
+      const uint32_t tmem = *bb.tmem_holder;
+      if (warp == 0) {
+        if (lane_id() == 0) LcGemm<BN>::producer(P, lc, bb);
+      } else if (warp == 1) {
+        if (lane_id() == 0) LcGemm<BN>::mma(P, lc, bb, tmem);
+      } else {
+        LcGemm<BN>::epilogue(P, bb, tmem);
+      }
+    }
+  } else if constexpr (BE_KIND != TACKER_BE_NONE) {
+    be_ptb_loop<BE_KIND>(P, be_smem);
+  }
+
+  tc_fence_before();
+  __syncthreads();   // teardown: every role done
+  if (warp == 1 && has_lc) {
+    tc_fence_after();
+    tmem_dealloc(*bb.tmem_holder, P.tmem_cols);
+  }
+}
+
+// ------------------------------------------------------------------------ BE original kernel
+// The non-persistent "CD_kernel" of Fig. 7: one CTA of 128 threads per original block.
+template <int BE_KIND>
+__global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ tacker_be_desc D) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  BeBody<BE_KIND>::run(BeSel<BE_KIND>::get(D), (int64_t)blockIdx.x, threadIdx.x, 1u, smem_raw);
+}
+
+}  // namespace tk

@@ -1,0 +1,438 @@
+// manager.cpp — Tacker's runtime QoS-aware kernel manager (a11; §VII).
+//
+// Per LC kernel of the oldest active query:
+//   * Eq. 9: at the first issue of the newest query Q,
+//       Thr = T_qos - T_queue - T_ori_solo(Q) - sum_i T_lc_i(remaining, earlier queries),
+//     T_queue = issue time - arrival (reading).  Thr <= direct_eps -> Q runs direct.
+//   * Only the newest query fuses/reorders.
+//   * TC kernel: Eq. 8 over the ready BE heads with a fitted pair model:
+//       Ttc + Tcd > Tk_fuse  &&  Tk_fuse - Ttc < Thr;  max Tgain = Tcd - (Tk_fuse - Ttc)
+//     (P:2045-2056), ties -> lowest app index; Thr -= Tk_fuse - Ttc.
+//   * No fusion: original launch, then reorder ready BE heads with Ttmp < Thr.
+//   * Baymax policy: identical with fusion disabled ("static scheduling").
+//   * Idle GPU (paper silent): one ready BE head no longer than idle_cap.
+// In simulation mode every kernel takes its predicted time on a serial virtual stream (the
+// discrete-event reference oracle/manager_ref.py follows the same rules); in GPU mode the
+// manager launches on its stream and observes completion with CUDA events.
+#include <cuda_runtime.h>
+
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <deque>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "runtime.h"
+#include "tacker.h"
+
+namespace tkrt {
+bool make_keys(const tacker_lc_desc *lc, const tacker_be_desc *be, int warp_split, std::string *lk, std::string *bk,
+               std::string *pk);
+}
+using namespace tkrt;
+
+namespace {
+
+struct Query {
+  int id;
+  double arrival;
+  std::vector<tacker_lc_kernel> ks;
+  size_t pos = 0;
+  bool issued = false, direct = false, has_thr = false;
+  double thr = 0;
+  double done_at = -1;
+  cudaEvent_t last_ev = nullptr;  // GPU mode: event after its last kernel
+  double remaining() const {
+    double s = 0;
+    for (size_t i = pos; i < ks.size(); ++i) s += ks[i].t_pred_ms;
+    return s;
+  }
+};
+
+struct App {
+  std::vector<tacker_be_kernel> ks;
+  size_t pos = 0;
+  double ready_at = 0;
+  int64_t completed = 0;
+  cudaEvent_t pending = nullptr;   // GPU mode: last launched kernel of this app
+  const tacker_be_kernel &head() const { return ks[pos % ks.size()]; }
+};
+
+}  // namespace
+
+struct tacker_manager_s {
+  int policy;
+  tacker_manager_params prm;
+  cudaStream_t stream;
+  double now = 0;
+  bool external_clock = false;
+  std::chrono::steady_clock::time_point t0;
+  cudaEvent_t base_ev = nullptr;
+  std::vector<Query> queries;        // by id
+  std::vector<int> pending;          // ids not yet admitted, arrival order
+  size_t next_pending = 0;
+  std::deque<int> active;
+  std::vector<App> apps;
+  tacker_manager_stats st{};
+  std::map<std::string, tacker_fused_t> cache;
+  std::deque<cudaEvent_t> inflight;
+  std::vector<cudaEvent_t> free_events;
+
+  bool sim() const { return prm.simulate != 0; }
+};
+
+static double host_now(tacker_manager_s *m) {
+  if (m->external_clock || m->sim()) return m->now;
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - m->t0).count();
+}
+
+static cudaEvent_t get_event(tacker_manager_s *m) {
+  if (!m->free_events.empty()) {
+    cudaEvent_t e = m->free_events.back();
+    m->free_events.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// GPU completion time of an event on the manager clock (ms since creation)
+static double event_time(tacker_manager_s *m, cudaEvent_t e) {
+  float ms = 0;
+  cudaEventElapsedTime(&ms, m->base_ev, e);
+  return (double)ms;
+}
+
+static void poll(tacker_manager_s *m) {
+  if (m->sim()) return;
+  while (!m->inflight.empty() && cudaEventQuery(m->inflight.front()) == cudaSuccess) m->inflight.pop_front();
+  for (auto &a : m->apps)
+    if (a.pending && cudaEventQuery(a.pending) == cudaSuccess) {
+      a.ready_at = event_time(m, a.pending);
+      a.pending = nullptr;
+    }
+  for (int id : m->active) {
+    Query &q = m->queries[id];
+    if (q.pos == q.ks.size() && q.done_at < 0 && q.last_ev && cudaEventQuery(q.last_ev) == cudaSuccess) {
+      q.done_at = event_time(m, q.last_ev);
+      m->st.lc_queries_done++;
+    }
+  }
+}
+
+static bool app_ready(tacker_manager_s *m, const App &a, double t) {
+  if (m->sim()) return a.ready_at <= t;
+  return a.pending == nullptr;
+}
+
+static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, double *tf) {
+  std::string lk, bk, pk;
+  const int ws = b.warp_split ? b.warp_split : 16;
+  if (!make_keys(&k.lc, &b.be, ws, &lk, &bk, &pk)) return false;
+  return pair_predict(pk, k.t_pred_ms, b.t_pred_ms, tf);
+}
+
+// ---------------------------------------------------------------- GPU launches
+static tacker_status launch_lc(tacker_manager_s *m, const tacker_lc_kernel &k) {
+  if (k.is_tc) return tacker_launch_original(&k.lc, nullptr, reinterpret_cast<tacker_stream_t>(m->stream));
+  return tacker_launch_original(nullptr, &k.cd, reinterpret_cast<tacker_stream_t>(m->stream));
+}
+
+static tacker_status launch_be(tacker_manager_s *m, const tacker_be_kernel &b) {
+  return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
+}
+
+static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b) {
+  const int ws = b.warp_split ? b.warp_split : 16;
+  char key[256];
+  snprintf(key, sizeof key, "%p/%p/%p/%p/%d/%d", k.lc.A, k.lc.B, k.lc.D, (const void *)&b, ws, b.be.orig_blocks);
+  auto it = m->cache.find(key);
+  tacker_fused_t f = nullptr;
+  if (it == m->cache.end()) {
+    tacker_status s = tacker_fuse(&k.lc, &b.be, ws, tacker_ratio{0, 0}, &f);
+    if (s) return s;
+    m->cache[key] = f;
+  } else {
+    f = it->second;
+  }
+  return tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
+}
+
+static cudaEvent_t record(tacker_manager_s *m) {
+  cudaEvent_t e = get_event(m);
+  cudaEventRecord(e, m->stream);
+  m->inflight.push_back(e);
+  return e;
+}
+
+extern "C" {
+
+tacker_status tacker_manager_create(int32_t policy, const tacker_manager_params *params, tacker_stream_t stream,
+                                    tacker_manager_t *out) {
+  if (!out || !params) return set_error("null argument"), TACKER_EINVAL;
+  if (policy != TACKER_POLICY_TACKER && policy != TACKER_POLICY_BAYMAX) return set_error("bad policy"), TACKER_EINVAL;
+  auto *m = new (std::nothrow) tacker_manager_s();
+  if (!m) return TACKER_ENOMEM;
+  m->policy = policy;
+  m->prm = *params;
+  if (m->prm.max_inflight < 1) m->prm.max_inflight = 1;
+  m->stream = reinterpret_cast<cudaStream_t>(stream);
+  m->t0 = std::chrono::steady_clock::now();
+  if (!m->sim()) {
+    cudaError_t e = cudaEventCreate(&m->base_ev);
+    if (e == cudaSuccess) e = cudaEventRecord(m->base_ev, m->stream);
+    if (e != cudaSuccess) {
+      delete m;
+      return cuda_fail("manager events", e);
+    }
+  }
+  *out = m;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_destroy(tacker_manager_t m) {
+  if (!m) return TACKER_OK;
+  if (!m->sim()) {
+    cudaStreamSynchronize(m->stream);
+    for (auto &kv : m->cache) tacker_fused_destroy(kv.second);
+    for (auto e : m->inflight) cudaEventDestroy(e);
+    for (auto e : m->free_events) cudaEventDestroy(e);
+    if (m->base_ev) cudaEventDestroy(m->base_ev);
+  }
+  delete m;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_submit_lc(tacker_manager_t m, const tacker_lc_query *q, double arrival_ms, int32_t *id) {
+  if (!m || !q || q->n_kernels <= 0 || !q->kernels) return set_error("bad query"), TACKER_EINVAL;
+  Query Q;
+  Q.id = (int)m->queries.size();
+  Q.arrival = arrival_ms;
+  Q.ks.assign(q->kernels, q->kernels + q->n_kernels);
+  m->queries.push_back(Q);
+  // keep pending sorted by arrival (stable)
+  auto pos = m->pending.begin() + (long)m->next_pending;
+  while (pos != m->pending.end() && m->queries[*pos].arrival <= arrival_ms) ++pos;
+  m->pending.insert(pos, Q.id);
+  if (id) *id = Q.id;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_submit_be(tacker_manager_t m, const tacker_be_app *app, int32_t *id) {
+  if (!m || !app || app->n_kernels <= 0 || !app->kernels) return set_error("bad BE app"), TACKER_EINVAL;
+  if (m->apps.size() >= TACKER_MAX_APPS) return set_error("too many BE apps"), TACKER_ERESOURCE;
+  App A;
+  A.ks.assign(app->kernels, app->kernels + app->n_kernels);
+  A.ready_at = m->now;
+  m->apps.push_back(A);
+  if (id) *id = (int)m->apps.size() - 1;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms) {
+  if (!m) return set_error("null manager"), TACKER_EINVAL;
+  m->now = now_ms;
+  m->external_clock = true;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headroom, tacker_decision *out) {
+  if (!m || !out) return set_error("null argument"), TACKER_EINVAL;
+  memset(out, 0, sizeof *out);
+  out->action = TACKER_DEC_NOTHING;
+  out->query = out->lc_index = out->fused_app = -1;
+  poll(m);
+  const double t = host_now(m);
+  m->now = t;
+  out->t_start_ms = out->t_end_ms = t;
+  while (m->next_pending < m->pending.size() && m->queries[m->pending[m->next_pending]].arrival <= t)
+    m->active.push_back(m->pending[m->next_pending++]);
+  // retire finished queries
+  while (!m->active.empty()) {
+    Query &q = m->queries[m->active.front()];
+    if (q.pos < q.ks.size()) break;
+    if (m->sim() || q.done_at >= 0) m->active.pop_front();
+    else break;
+  }
+  if (!m->sim() && (int)m->inflight.size() >= m->prm.max_inflight) return TACKER_OK;   // stream is busy
+
+  // oldest query with kernels still to issue
+  int qid = -1;
+  for (int id : m->active)
+    if (m->queries[id].pos < m->queries[id].ks.size()) {
+      qid = id;
+      break;
+    }
+  std::vector<int> heads;
+  for (size_t a = 0; a < m->apps.size(); ++a)
+    if (app_ready(m, m->apps[a], t)) heads.push_back((int)a);
+
+  if (qid < 0) {
+    // idle GPU (or only tails of earlier queries still running): one bounded BE kernel
+    for (int a : heads) {
+      const tacker_be_kernel &b = m->apps[a].head();
+      if (m->prm.idle_cap_ms > 0 && b.t_pred_ms > m->prm.idle_cap_ms) continue;
+      if (!m->active.empty()) break;   // do not delay a running query's completion
+      out->action = TACKER_DEC_IDLE_BE;
+      out->n_reorder = 1;
+      out->reorder_apps[0] = a;
+      App &A = m->apps[a];
+      if (m->sim()) {
+        m->now += b.t_pred_ms;
+        A.ready_at = m->now;
+      } else {
+        tacker_status s = launch_be(m, b);
+        if (s) return s;
+        A.pending = record(m);
+      }
+      A.pos++;
+      A.completed++;
+      m->st.be_kernels_done++;
+      m->st.idle_be++;
+      out->t_end_ms = m->now;
+      return TACKER_OK;
+    }
+    if (m->sim()) {   // advance the virtual clock to the next event
+      double nxt = INFINITY;
+      if (m->next_pending < m->pending.size()) nxt = m->queries[m->pending[m->next_pending]].arrival;
+      for (auto &A : m->apps)
+        if (A.ready_at > t) nxt = std::min(nxt, A.ready_at);
+      if (std::isfinite(nxt)) m->now = nxt;
+      out->t_end_ms = m->now;
+    }
+    return TACKER_OK;
+  }
+
+  Query &q = m->queries[qid];
+  const bool newest = (qid == m->active.back());
+  if (!q.issued) {
+    q.issued = true;
+    if (newest) {
+      double earlier = 0;
+      for (int id : m->active)
+        if (id != qid) earlier += m->queries[id].remaining();
+      q.thr = qos - (t - q.arrival) - q.remaining() - earlier;   // Eq. 9
+      q.has_thr = true;
+      q.direct = q.thr <= m->prm.direct_eps_ms;
+    }
+  }
+  const bool allow = newest && q.has_thr && !q.direct;
+  double thr = q.has_thr ? q.thr : 0.0;
+  if (allow && headroom && !std::isnan(*headroom)) thr = *headroom;
+  const tacker_lc_kernel &k = q.ks[q.pos];
+  const double ttc = k.t_pred_ms;
+
+  int fused = -1;
+  double best_gain = 0, best_tf = 0;
+  if (allow && m->policy == TACKER_POLICY_TACKER && k.is_tc) {
+    for (int a : heads) {
+      const tacker_be_kernel &b = m->apps[a].head();
+      if (!b.is_cd) continue;
+      double tf;
+      if (!pair_time(k, b, &tf)) continue;
+      if (ttc + b.t_pred_ms > tf && tf - ttc < thr) {   // Eq. 8
+        const double gain = b.t_pred_ms - (tf - ttc);
+        if (fused < 0 || gain > best_gain) {
+          fused = a;
+          best_gain = gain;
+          best_tf = tf;
+        }
+      }
+    }
+  }
+  std::vector<int> reorder;
+  if (fused >= 0) {
+    thr -= best_tf - ttc;
+  } else if (allow) {
+    for (int a : heads) {
+      const double tt = m->apps[a].head().t_pred_ms;
+      if (tt < thr) {
+        reorder.push_back(a);
+        thr -= tt;
+      }
+    }
+  }
+  if (allow) q.thr = thr;
+
+  // execute
+  out->query = qid;
+  out->lc_index = (int)q.pos;
+  out->fused_app = fused;
+  out->gain_ms = fused >= 0 ? best_gain : 0;
+  out->thr_ms = thr;
+  if (headroom) *headroom = thr;
+  if (fused >= 0) {
+    App &A = m->apps[fused];
+    if (m->sim()) {
+      m->now += best_tf;
+      A.ready_at = m->now;
+    } else {
+      tacker_status s = launch_fused(m, k, A.head());
+      if (s) return s;
+      cudaEvent_t e = record(m);
+      A.pending = e;
+      if (q.pos + 1 == q.ks.size()) q.last_ev = e;
+    }
+    A.pos++;
+    A.completed++;
+    m->st.fused_launches++;
+    m->st.be_kernels_done++;
+    out->action = TACKER_DEC_FUSED;
+  } else {
+    if (m->sim()) {
+      m->now += ttc;
+    } else {
+      tacker_status s = launch_lc(m, k);
+      if (s) return s;
+      cudaEvent_t e = record(m);
+      if (q.pos + 1 == q.ks.size()) q.last_ev = e;
+    }
+    m->st.original_lc++;
+    out->action = reorder.empty() ? TACKER_DEC_ORIGINAL_LC : TACKER_DEC_REORDER_BE;
+  }
+  q.pos++;
+  if (m->sim() && q.pos == q.ks.size()) {
+    q.done_at = m->now;
+    m->st.lc_queries_done++;
+  }
+  for (int a : reorder) {
+    App &A = m->apps[a];
+    const tacker_be_kernel &b = A.head();
+    if (m->sim()) {
+      m->now += b.t_pred_ms;
+      A.ready_at = m->now;
+    } else {
+      tacker_status s = launch_be(m, b);
+      if (s) return s;
+      A.pending = record(m);
+    }
+    A.pos++;
+    A.completed++;
+    m->st.be_kernels_done++;
+    m->st.reordered_be++;
+    if (out->n_reorder < TACKER_MAX_REORDER) out->reorder_apps[out->n_reorder++] = a;
+  }
+  out->t_end_ms = m->now;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *o) {
+  if (!m || !o) return set_error("null argument"), TACKER_EINVAL;
+  poll(m);
+  *o = m->st;
+  o->now_ms = m->sim() ? m->now : host_now(m);
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_query_latency(tacker_manager_t m, int32_t id, double *lat) {
+  if (!m || !lat || id < 0 || id >= (int)m->queries.size()) return set_error("bad query id"), TACKER_EINVAL;
+  poll(m);
+  const Query &q = m->queries[id];
+  *lat = q.done_at >= 0 ? q.done_at - q.arrival : -1.0;
+  return TACKER_OK;
+}
+
+}  // extern "C"

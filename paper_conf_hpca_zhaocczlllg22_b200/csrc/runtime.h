@@ -1,0 +1,20 @@
+// runtime.h — internal host-side declarations shared by the C ABI translation units.
+#pragma once
+#include <string>
+
+#include "tacker.h"
+
+namespace tkrt {
+
+void set_error(const char *fmt, ...);
+tacker_status cuda_fail(const char *what, int err);
+int sm_count();
+
+// model store (predictor.cpp)
+bool model_predict(const std::string &key, double x, double *y);
+bool pair_predict(const std::string &key, double x_tc, double x_cd, double *y);
+
+// kind names
+const char *be_kind_name(int kind);
+
+}  // namespace tkrt

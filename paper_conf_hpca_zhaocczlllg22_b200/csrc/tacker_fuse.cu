@@ -1,0 +1,633 @@
+// tacker_fuse.cu — fusion planner (a1), tensor-map encoding, fused / original launches (a2-a8).
+//
+// tacker_fuse implements Tacker's offline fusion step on B200 (§V-B/C P:1117-1309): PTB with
+// one persistent CTA per SM, LC budgeted first (SMEM ring stages, TMEM accumulator columns),
+// BE virtual blocks added with what remains, and admission by aggregate per-SM resources
+// (§VIII-I).  Instead of generating code it selects one of the
+// compiled template instantiations fused_kernel<BN, BE_KIND>.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "kernels/fused.cuh"
+#include "runtime.h"
+#include "tacker.h"
+
+using namespace tk;
+
+namespace tkrt {
+
+static thread_local std::string g_err;
+
+void set_error(const char *fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+
+tacker_status cuda_fail(const char *what, int err) {
+  set_error("%s: CUDA error %d (%s)", what, err, cudaGetErrorString((cudaError_t)err));
+  return TACKER_ECUDA;
+}
+
+int sm_count() {
+  static int n = -1;
+  if (n < 0) {
+    int dev = 0, v = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+      cudaGetLastError();
+      return 0;
+    }
+    n = v;
+  }
+  return n;
+}
+
+const char *be_kind_name(int kind) {
+  static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
+                                "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn"};
+  return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
+}
+
+}  // namespace tkrt
+
+using namespace tkrt;
+
+// ============================================================================ constants
+static constexpr int kSmemCap = 232448;      // max dynamic SMEM per CTA on sm_100 (227 KB)
+static constexpr int kTmemCols = 512;
+static constexpr int kMaxBeWarps = 16;       // fused_kernel __launch_bounds__ sizing
+static constexpr int kMaxWarps = 32;
+static constexpr int kMinLcSmem = 120 * 1024;  // forces one LC CTA per SM (TMEM ownership)
+
+// ============================================================================ BE helpers
+template <int K>
+static int64_t be_blocks_t(const tacker_be_desc &d) {
+  return BeBody<K>::num_blocks(BeSel<K>::get(d));
+}
+
+static bool be_num_blocks(const tacker_be_desc &d, int64_t *out) {
+  switch (d.kind) {
+#define C(K) \
+  case K: *out = be_blocks_t<K>(d); return true;
+    C(TACKER_BE_SGEMM)
+    C(TACKER_BE_STENCIL)
+    C(TACKER_BE_MRIQ_PHIMAG)
+    C(TACKER_BE_MRIQ_Q)
+    C(TACKER_BE_LBM)
+    C(TACKER_BE_SPMV_JDS)
+    C(TACKER_BE_HISTO)
+    C(TACKER_BE_BFS_EXPAND)
+    C(TACKER_BE_BFS_COMMIT)
+    C(TACKER_BE_FMA_BURN)
+#undef C
+    default: return false;
+  }
+}
+
+static uint32_t be_smem_bytes(int kind) {
+  switch (kind) {
+#define C(K) \
+  case K: return BeBody<K>::kSmem;
+    C(TACKER_BE_SGEMM)
+    C(TACKER_BE_STENCIL)
+    C(TACKER_BE_MRIQ_PHIMAG)
+    C(TACKER_BE_MRIQ_Q)
+    C(TACKER_BE_LBM)
+    C(TACKER_BE_SPMV_JDS)
+    C(TACKER_BE_HISTO)
+    C(TACKER_BE_BFS_EXPAND)
+    C(TACKER_BE_BFS_COMMIT)
+    C(TACKER_BE_FMA_BURN)
+#undef C
+    default: return 0;
+  }
+}
+
+static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
+  int64_t full = 0;
+  if (!be_num_blocks(d, &full)) {
+    set_error("BE kind %d not supported", d.kind);
+    return TACKER_EUNSUPPORTED;
+  }
+  switch (d.kind) {
+    case TACKER_BE_SGEMM: {
+      const auto &p = d.p.sgemm;
+      if (p.M < 0 || p.N < 0 || p.K < 0 || !p.A || !p.B || !p.C) return set_error("sgemm: bad args"), TACKER_EINVAL;
+      if (p.N % 4 || p.K % 4) return set_error("sgemm: N and K must be multiples of 4"), TACKER_EUNSUPPORTED;
+      break;
+    }
+    case TACKER_BE_STENCIL: {
+      const auto &p = d.p.stencil;
+      if (p.nx <= 0 || p.ny <= 0 || p.nz <= 0 || !p.A0 || !p.Anext) return set_error("stencil: bad args"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_MRIQ_PHIMAG:
+      if (d.p.mriq_phimag.numK < 0 || !d.p.mriq_phimag.phiMag) return set_error("mriq_phimag: bad args"), TACKER_EINVAL;
+      break;
+    case TACKER_BE_MRIQ_Q:
+      if (d.p.mriq_q.numX < 0 || d.p.mriq_q.numK < 0 || !d.p.mriq_q.Qr) return set_error("mriq_q: bad args"), TACKER_EINVAL;
+      break;
+    case TACKER_BE_LBM:
+      if (d.p.lbm.nx <= 0 || !d.p.lbm.src || !d.p.lbm.dst || !d.p.lbm.flags || d.p.lbm.src == d.p.lbm.dst)
+        return set_error("lbm: bad args (src and dst must differ)"), TACKER_EINVAL;
+      break;
+    case TACKER_BE_SPMV_JDS:
+      if (d.p.spmv.rows < 0 || !d.p.spmv.y) return set_error("spmv: bad args"), TACKER_EINVAL;
+      break;
+    case TACKER_BE_HISTO:
+      if (d.p.histo.n < 0 || d.p.histo.nbins <= 0 || d.p.histo.nbins > 8192 || !d.p.histo.count)
+        return set_error("histo: nbins must be in [1, 8192]"), TACKER_EUNSUPPORTED;
+      break;
+    case TACKER_BE_BFS_EXPAND:
+    case TACKER_BE_BFS_COMMIT:
+      break;
+    case TACKER_BE_FMA_BURN:
+      if (d.p.fma_burn.n_threads < 0 || d.p.fma_burn.iters < 0 || !d.p.fma_burn.out)
+        return set_error("fma_burn: bad args"), TACKER_EINVAL;
+      break;
+  }
+  if (d.orig_blocks < 0 || d.orig_blocks > full) {
+    set_error("orig_blocks %d outside [0, %lld]", d.orig_blocks, (long long)full);
+    return TACKER_EINVAL;
+  }
+  *blocks = d.orig_blocks ? d.orig_blocks : full;
+  return TACKER_OK;
+}
+
+// ============================================================================ LC helpers
+static tacker_status lc_view(const tacker_lc_desc &d, LcParams &L) {
+  memset(&L, 0, sizeof L);
+  L.kind = d.kind;
+  if (d.kind == TACKER_LC_GEMM_F16) {
+    L.M = d.M;
+    L.N = d.N;
+    L.K = d.K;
+  } else if (d.kind == TACKER_LC_CONV_F16) {
+    if (d.n <= 0 || d.h <= 0 || d.w <= 0 || d.c <= 0 || d.k <= 0 || d.r <= 0 || d.s <= 0 || d.stride <= 0 || d.pad < 0)
+      return set_error("conv: bad shape"), TACKER_EINVAL;
+    L.n = d.n; L.h = d.h; L.w = d.w; L.c = d.c; L.k = d.k; L.r = d.r; L.s = d.s; L.stride = d.stride; L.pad = d.pad;
+    L.p = (d.h + 2 * d.pad - d.r) / d.stride + 1;
+    L.q = (d.w + 2 * d.pad - d.s) / d.stride + 1;
+    if (L.p <= 0 || L.q <= 0) return set_error("conv: empty output"), TACKER_EINVAL;
+    L.M = d.n * L.p * L.q;
+    L.N = d.k;
+    L.K = d.c * d.r * d.s;
+    L.conv_direct_gemm = (d.r == 1 && d.s == 1 && d.stride == 1 && d.pad == 0);
+    if (!L.conv_direct_gemm && d.c % 64 != 0)
+      return set_error("conv: C must be a multiple of 64 for implicit GEMM (got %d)", d.c), TACKER_EUNSUPPORTED;
+  } else {
+    return set_error("LC kind %d not supported", d.kind), TACKER_EUNSUPPORTED;
+  }
+  if (L.M <= 0 || L.N <= 0 || L.K <= 0) return set_error("LC: empty GEMM"), TACKER_EINVAL;
+  if (L.K % 8 || L.N % 8) return set_error("LC: K and N must be multiples of 8 (16-byte TMA pitch)"), TACKER_EUNSUPPORTED;
+  if (!d.A || !d.B || !d.D) return set_error("LC: null pointer"), TACKER_EINVAL;
+  if ((d.epi_flags & TACKER_EPI_BIAS) && !d.bias) return set_error("LC: bias flag without bias"), TACKER_EINVAL;
+  if ((d.epi_flags & TACKER_EPI_RESIDUAL) && !d.residual) return set_error("LC: residual flag without residual"), TACKER_EINVAL;
+  if (d.d_dtype != TACKER_F32 && d.d_dtype != TACKER_F16) return set_error("LC: bad d_dtype"), TACKER_EINVAL;
+  L.D = d.D;
+  L.d_f16 = d.d_dtype == TACKER_F16;
+  L.epi = d.epi_flags;
+  L.bias = d.bias;
+  L.residual = reinterpret_cast<const __half *>(d.residual);
+  return TACKER_OK;
+}
+
+static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
+  if (d.tile_n == 64 || d.tile_n == 128 || d.tile_n == 256) return d.tile_n;
+  if (L.N <= 64) return 64;
+  const int sms = sm_count() > 0 ? sm_count() : 148;
+  if (L.N >= 256 && (int64_t)((L.M + 127) / 128) * ((L.N + 255) / 256) >= 2LL * sms) return 256;
+  return 128;
+}
+
+static void lc_tiles(LcParams &L, int BN) {
+  L.tiles_n = (L.N + BN - 1) / BN;
+  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
+    // output tile of 128 positions: tq along q (power of two <= 32 covering q), tp = 128/tq
+    int tq = 1;
+    while (tq < L.q && tq < 32) tq <<= 1;
+    if (tq < 8) tq = 8;
+    L.tq = tq;
+    L.tp = kBM / tq;
+    L.tiles_p = (L.p + L.tp - 1) / L.tp;
+    L.tiles_q = (L.q + L.tq - 1) / L.tq;
+    L.tiles_m = L.n * L.tiles_p * L.tiles_q;
+    L.c_blocks = L.c / kBK;
+    L.num_kb = L.r * L.s * L.c_blocks;
+  } else {
+    L.tiles_m = (L.M + kBM - 1) / kBM;
+    L.num_kb = (L.K + kBK - 1) / kBK;
+  }
+  L.num_tiles = L.tiles_m * L.tiles_n;
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+static tacker_status encode_2d(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                               uint32_t box_outer) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {inner * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(2d) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, const LcParams &L) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)d.c, (cuuint64_t)d.w, (cuuint64_t)d.h, (cuuint64_t)d.n};
+  cuuint64_t strides[3] = {(cuuint64_t)d.c * 2, (cuuint64_t)d.c * d.w * 2, (cuuint64_t)d.c * d.w * d.h * 2};
+  cuuint32_t box[4] = {(cuuint32_t)kBK, (cuuint32_t)(L.tq * d.stride), (cuuint32_t)(L.tp * d.stride), 1};
+  cuuint32_t es[4] = {1, (cuuint32_t)d.stride, (cuuint32_t)d.stride, 1};
+  if (box[1] > 256 || box[2] > 256) return set_error("conv: TMA box too large"), TACKER_EUNSUPPORTED;
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void *>(d.A), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv x) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+// ============================================================================ kernel table
+using KernelFn = void (*)(FusedParams);
+
+template <int BN>
+static KernelFn fused_fn(int be_kind) {
+  switch (be_kind) {
+    case TACKER_BE_NONE: return fused_kernel<BN, TACKER_BE_NONE>;
+#define C(K) \
+  case K: return fused_kernel<BN, K>;
+    C(TACKER_BE_SGEMM)
+    C(TACKER_BE_STENCIL)
+    C(TACKER_BE_MRIQ_PHIMAG)
+    C(TACKER_BE_MRIQ_Q)
+    C(TACKER_BE_LBM)
+    C(TACKER_BE_SPMV_JDS)
+    C(TACKER_BE_HISTO)
+    C(TACKER_BE_BFS_EXPAND)
+    C(TACKER_BE_BFS_COMMIT)
+    C(TACKER_BE_FMA_BURN)
+#undef C
+    default: return nullptr;
+  }
+}
+static KernelFn pick_fused(int BN, int be_kind) {
+  if (BN == 64) return fused_fn<64>(be_kind);
+  if (BN == 128) return fused_fn<128>(be_kind);
+  if (BN == 256) return fused_fn<256>(be_kind);
+  return nullptr;
+}
+
+using BeFn = void (*)(tacker_be_desc);
+static BeFn pick_be_original(int kind) {
+  switch (kind) {
+#define C(K) \
+  case K: return be_original_kernel<K>;
+    C(TACKER_BE_SGEMM)
+    C(TACKER_BE_STENCIL)
+    C(TACKER_BE_MRIQ_PHIMAG)
+    C(TACKER_BE_MRIQ_Q)
+    C(TACKER_BE_LBM)
+    C(TACKER_BE_SPMV_JDS)
+    C(TACKER_BE_HISTO)
+    C(TACKER_BE_BFS_EXPAND)
+    C(TACKER_BE_BFS_COMMIT)
+    C(TACKER_BE_FMA_BURN)
+#undef C
+    default: return nullptr;
+  }
+}
+
+static tacker_status set_smem_attr(const void *fn, int bytes) {
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e != cudaSuccess) return cuda_fail("cudaFuncSetAttribute", e);
+  return TACKER_OK;
+}
+
+// ============================================================================ fused handle
+struct tacker_fused_s {
+  FusedParams P;
+  KernelFn fn;
+  tacker_lc_desc lc;
+  tacker_be_desc be;
+  int warp_split;
+  int grid, block, smem;
+  int BN;
+  int regs;
+  std::string lc_key, be_key, pair_key;
+};
+
+static std::string lc_key_of(const tacker_lc_desc &d, const LcParams &L, int BN) {
+  char b[256];
+  if (d.kind == TACKER_LC_GEMM_F16)
+    snprintf(b, sizeof b, "lc:gemm:N%d:K%d:bn%d:%s", L.N, L.K, BN, L.d_f16 ? "f16" : "f32");
+  else
+    snprintf(b, sizeof b, "lc:conv:h%dw%dc%d:k%dr%ds%d:st%dp%d:bn%d", d.h, d.w, d.c, d.k, d.r, d.s, d.stride, d.pad, BN);
+  return b;
+}
+
+static std::string be_key_of(const tacker_be_desc &d) {
+  char b[256];
+  switch (d.kind) {
+    case TACKER_BE_SGEMM: snprintf(b, sizeof b, "be:sgemm:N%d:K%d", d.p.sgemm.N, d.p.sgemm.K); break;
+    case TACKER_BE_STENCIL: snprintf(b, sizeof b, "be:stencil:nz%d", d.p.stencil.nz); break;
+    case TACKER_BE_MRIQ_Q: snprintf(b, sizeof b, "be:mriq_q:K%d", d.p.mriq_q.numK); break;
+    case TACKER_BE_FMA_BURN: snprintf(b, sizeof b, "be:fma_burn:it%d", d.p.fma_burn.iters); break;
+    default: snprintf(b, sizeof b, "be:%s", be_kind_name(d.kind)); break;
+  }
+  return b;
+}
+
+static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, int warp_split, tacker_ratio ratio,
+                          tacker_fused_s &F) {
+  memset(&F.P, 0, sizeof F.P);
+  const bool has_lc = lc && lc->kind != TACKER_LC_NONE;
+  const bool has_be = be && be->kind != TACKER_BE_NONE;
+  if (!has_lc) return set_error("tacker_fuse: an LC descriptor is required"), TACKER_EINVAL;
+  if (has_be && (warp_split < 4 || warp_split % 4 || warp_split > kMaxBeWarps))
+    return set_error("warp_split must be a multiple of 4 in [4, %d] (got %d)", kMaxBeWarps, warp_split), TACKER_EUNSUPPORTED;
+  if (!has_be && warp_split != 0) return set_error("warp_split must be 0 without a BE part"), TACKER_EINVAL;
+  const int sms = sm_count();
+  if (sms <= 0) return set_error("no CUDA device"), TACKER_ECUDA;
+
+  LcParams &L = F.P.lc;
+  tacker_status st = lc_view(*lc, L);
+  if (st) return st;
+  const int BN = pick_tile_n(*lc, L);
+  lc_tiles(L, BN);
+  F.BN = BN;
+
+  int64_t be_blocks = 0;
+  int vb = 0;
+  uint32_t be_slice = 0;
+  if (has_be) {
+    if ((st = validate_be(*be, &be_blocks))) return st;
+    vb = warp_split / 4;
+    if (ratio.be && ratio.be != vb)
+      return set_error("block_ratio.be (%d) must equal warp_split/4 (%d)", ratio.be, vb), TACKER_EUNSUPPORTED;
+    if (vb > 15) return set_error("too many BE virtual blocks for named barriers"), TACKER_ERESOURCE;
+    be_slice = (16 + be_smem_bytes(be->kind) + 127) & ~127u;
+    F.P.be = *be;
+  }
+  const int acc = ratio.lc ? ratio.lc : (2 * BN <= kTmemCols ? 2 : 1);
+  if (acc < 1 || acc > 2 || acc * BN > kTmemCols)
+    return set_error("block_ratio.lc (TMEM accumulator stages) %d does not fit %d columns", acc, kTmemCols), TACKER_ERESOURCE;
+  uint32_t cols = 32;
+  while (cols < (uint32_t)(acc * BN)) cols <<= 1;
+
+  // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages, >= 2) that
+  // still leaves room for the requested BE virtual blocks.
+  const uint32_t stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
+  const uint32_t bar_bytes = 256;
+  const uint32_t be_total = (uint32_t)vb * be_slice;
+  int stages = 0;
+  for (int s = 4; s >= 2; --s) {
+    const uint32_t need = 1024 + s * stage_bytes + bar_bytes + be_total;
+    if (need <= (uint32_t)kSmemCap) {
+      stages = s;
+      break;
+    }
+  }
+  if (!stages) {
+    set_error("fused budget exceeds one SM: LC ring %u B x2 + BE %d x %u B > %d B", stage_bytes, vb, be_slice, kSmemCap);
+    return TACKER_ERESOURCE;
+  }
+  const int warps = kLcWarps + warp_split;
+  if (warps > kMaxWarps) return set_error("too many warps"), TACKER_ERESOURCE;
+
+  F.P.stages = stages;
+  F.P.acc_stages = acc;
+  F.P.tmem_cols = cols;
+  F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
+  F.P.be_smem_per_vb = be_slice;
+  F.P.be_vb_per_cta = vb;
+  F.P.be_blocks = be_blocks;
+  F.P.lc_warps = kLcWarps;
+  F.warp_split = warp_split;
+  F.block = 32 * warps;
+  F.smem = 1024 + F.P.lc_smem_bytes + be_total;
+  if (F.smem < kMinLcSmem) F.smem = kMinLcSmem;
+  F.grid = has_be ? sms : (L.num_tiles < sms ? L.num_tiles : sms);
+  if (F.grid < 1) F.grid = 1;
+  F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
+  if (!F.fn) return set_error("no kernel instantiation for BN=%d BE=%d", BN, has_be ? be->kind : 0), TACKER_EUNSUPPORTED;
+
+  // TMA tensor maps
+  if (lc->kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
+    if ((st = encode_conv_x(&F.P.tmap_a, *lc, L))) return st;
+    if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
+  } else {
+    if ((st = encode_2d(&F.P.tmap_a, lc->A, (uint64_t)L.K, (uint64_t)L.M, kBK, kBM))) return st;
+    if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
+  }
+  // registers: the whole CTA must fit the 64K register file
+  cudaFuncAttributes fa{};
+  cudaError_t e = cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(F.fn));
+  if (e != cudaSuccess) return cuda_fail("cudaFuncGetAttributes", e);
+  F.regs = fa.numRegs;
+  if ((int64_t)fa.numRegs * F.block > 65536) {
+    set_error("register budget: %d regs x %d threads > 65536", fa.numRegs, F.block);
+    return TACKER_ERESOURCE;
+  }
+  if ((st = set_smem_attr(reinterpret_cast<const void *>(F.fn), F.smem))) return st;
+  F.lc = *lc;
+  if (has_be) F.be = *be; else memset(&F.be, 0, sizeof F.be);
+  F.lc_key = lc_key_of(*lc, L, BN);
+  F.be_key = has_be ? be_key_of(*be) : "";
+  char pk[512];
+  snprintf(pk, sizeof pk, "pair:%s|%s|ws%d", F.lc_key.c_str(), F.be_key.c_str(), warp_split);
+  F.pair_key = pk;
+  return TACKER_OK;
+}
+
+static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) {
+  void *args[] = {&F.P};
+  cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(F.fn), dim3(F.grid), dim3(F.block), args, F.smem, s);
+  if (e != cudaSuccess) return cuda_fail("launch fused_kernel", e);
+  return TACKER_OK;
+}
+
+// ============================================================================ C ABI
+extern "C" {
+
+const char *tacker_last_error(void) { return g_err.c_str(); }
+const char *tacker_version(void) { return "tacker-b200 0.1 (sm_100a)"; }
+int tacker_device_sm_count(void) { return sm_count(); }
+
+tacker_status tacker_be_num_blocks(const tacker_be_desc *be, int64_t *out) {
+  if (!be || !out) return set_error("null argument"), TACKER_EINVAL;
+  if (!be_num_blocks(*be, out)) return set_error("BE kind %d not supported", be->kind), TACKER_EUNSUPPORTED;
+  return TACKER_OK;
+}
+
+tacker_status tacker_lc_num_tiles(const tacker_lc_desc *lc, int32_t tile_n, int64_t *out) {
+  if (!lc || !out) return set_error("null argument"), TACKER_EINVAL;
+  LcParams L;
+  tacker_status st = lc_view(*lc, L);
+  if (st) return st;
+  int BN = tile_n ? tile_n : pick_tile_n(*lc, L);
+  if (BN != 64 && BN != 128 && BN != 256) return set_error("tile_n must be 64/128/256"), TACKER_EINVAL;
+  lc_tiles(L, BN);
+  *out = L.num_tiles;
+  return TACKER_OK;
+}
+
+tacker_status tacker_fuse(const tacker_lc_desc *lc, const tacker_be_desc *be, int32_t warp_split, tacker_ratio block_ratio,
+                          tacker_fused_t *out) {
+  if (!out) return set_error("null out"), TACKER_EINVAL;
+  *out = nullptr;
+  auto *F = new (std::nothrow) tacker_fused_s();
+  if (!F) return set_error("out of host memory"), TACKER_ENOMEM;
+  tacker_status st = plan(lc, be, warp_split, block_ratio, *F);
+  if (st) {
+    delete F;
+    return st;
+  }
+  cudaError_t e = cudaMalloc(&F->P.work, sizeof(BeWork));
+  if (e == cudaSuccess) e = cudaMemset(F->P.work, 0, sizeof(BeWork));
+  if (e != cudaSuccess) {
+    delete F;
+    return cuda_fail("workspace", e);
+  }
+  *out = F;
+  return TACKER_OK;
+}
+
+tacker_status tacker_fused_destroy(tacker_fused_t f) {
+  if (!f) return TACKER_OK;
+  if (f->P.work) cudaFree(f->P.work);
+  delete f;
+  return TACKER_OK;
+}
+
+tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *o) {
+  if (!f || !o) return set_error("null argument"), TACKER_EINVAL;
+  memset(o, 0, sizeof *o);
+  o->grid = f->grid;
+  o->block_threads = f->block;
+  o->smem_bytes = f->smem;
+  o->lc_warps = f->P.lc_warps;
+  o->be_warps = f->warp_split;
+  o->be_vblocks_per_cta = f->P.be_vb_per_cta;
+  o->lc_tile_m = kBM;
+  o->lc_tile_n = f->BN;
+  o->lc_tile_k = kBK;
+  o->lc_stages = f->P.stages;
+  o->lc_acc_stages = f->P.acc_stages;
+  o->tmem_cols = (int32_t)f->P.tmem_cols;
+  o->lc_tiles = f->P.lc.num_tiles;
+  o->be_blocks = f->P.be_blocks;
+  o->be_smem_per_vblock = (int32_t)f->P.be_smem_per_vb;
+  o->regs_per_thread = f->regs;
+  return TACKER_OK;
+}
+
+tacker_status tacker_fused_keys(tacker_fused_t f, char *lc_key, char *be_key, char *pair_key, size_t n) {
+  if (!f || n == 0) return set_error("null argument"), TACKER_EINVAL;
+  if (lc_key) snprintf(lc_key, n, "%s", f->lc_key.c_str());
+  if (be_key) snprintf(be_key, n, "%s", f->be_key.c_str());
+  if (pair_key) snprintf(pair_key, n, "%s", f->pair_key.c_str());
+  return TACKER_OK;
+}
+
+tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, const tacker_be_desc *be) {
+  if (!f) return set_error("null handle"), TACKER_EINVAL;
+  tacker_fused_s tmp;
+  tacker_lc_desc l = lc ? *lc : f->lc;
+  tacker_be_desc b = be ? *be : f->be;
+  tacker_ratio r{(uint8_t)f->P.acc_stages, (uint8_t)f->P.be_vb_per_cta};
+  l.tile_n = f->BN;
+  tacker_status st = plan(&l, f->be.kind ? &b : nullptr, f->warp_split, r, tmp);
+  if (st) return st;
+  if (tmp.fn != f->fn || tmp.P.stages != f->P.stages || tmp.smem != f->smem)
+    return set_error("rebind changes the plan; call tacker_fuse"), TACKER_EINVAL;
+  BeWork *w = f->P.work;
+  *f = tmp;
+  f->P.work = w;
+  return TACKER_OK;
+}
+
+tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream) {
+  if (!f) return set_error("null handle"), TACKER_EINVAL;
+  return launch_plan(*f, reinterpret_cast<cudaStream_t>(stream));
+}
+
+tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be, tacker_stream_t stream) {
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  tacker_status st;
+  if (lc && lc->kind != TACKER_LC_NONE) {
+    tacker_fused_s F;
+    if ((st = plan(lc, nullptr, 0, tacker_ratio{0, 0}, F))) return st;
+    F.P.work = nullptr;
+    if ((st = launch_plan(F, s))) return st;
+  }
+  if (be && be->kind != TACKER_BE_NONE) {
+    int64_t blocks;
+    if ((st = validate_be(*be, &blocks))) return st;
+    if (blocks == 0) return TACKER_OK;
+    BeFn fn = pick_be_original(be->kind);
+    const int smem = (int)be_smem_bytes(be->kind);
+    if (smem > 48 * 1024 && (st = set_smem_attr(reinterpret_cast<const void *>(fn), smem))) return st;
+    tacker_be_desc d = *be;
+    void *args[] = {&d};
+    if (blocks > 0x7fffffffLL) return set_error("too many blocks"), TACKER_EUNSUPPORTED;
+    cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(fn), dim3((unsigned)blocks), dim3(128), args, smem, s);
+    if (e != cudaSuccess) return cuda_fail("launch be_original_kernel", e);
+  }
+  return TACKER_OK;
+}
+
+}  // extern "C"
+
+// accessors used by the predictor / manager translation units
+namespace tkrt {
+const std::string &fused_lc_key(tacker_fused_t f) { return f->lc_key; }
+const std::string &fused_be_key(tacker_fused_t f) { return f->be_key; }
+const std::string &fused_pair_key(tacker_fused_t f) { return f->pair_key; }
+int64_t fused_lc_tiles(tacker_fused_t f) { return f->P.lc.num_tiles; }
+int64_t fused_be_blocks(tacker_fused_t f) { return f->P.be_blocks; }
+
+// Model-store keys without building a handle (no GPU needed): the manager's predictions.
+bool make_keys(const tacker_lc_desc *lc, const tacker_be_desc *be, int warp_split, std::string *lk, std::string *bk,
+               std::string *pk) {
+  if (lc) {
+    LcParams L;
+    if (lc_view(*lc, L) != TACKER_OK) return false;
+    const int BN = pick_tile_n(*lc, L);
+    *lk = lc_key_of(*lc, L, BN);
+  }
+  if (be) *bk = be_key_of(*be);
+  if (lc && be) {
+    char b[512];
+    snprintf(b, sizeof b, "pair:%s|%s|ws%d", lk->c_str(), bk->c_str(), warp_split);
+    *pk = b;
+  }
+  return true;
+}
+}  // namespace tkrt

@@ -1,0 +1,128 @@
+"""Shared helpers for the -m gpu parity tests (the CUDA path goes through the C ABI)."""
+import numpy as np
+import torch
+
+import synth
+from oracle import be as obe
+
+
+def dev():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return torch.device("cuda:0")
+
+
+def t(a, dtype=None):
+    x = torch.from_numpy(np.ascontiguousarray(a))
+    if dtype is not None:
+        x = x.to(dtype)
+    return x.to(dev())
+
+
+def host(x):
+    torch.cuda.synchronize()
+    return x.cpu().numpy()
+
+
+def be_case(kind, seed=0, size="small"):
+    """Build (desc_builder, outputs, check) for a BE kind: returns dict with
+    'desc' (tacker BeDesc), 'outs' (list of device tensors to compare), 'reset' (callable that
+    restores the inputs/outputs before a launch), 'check' (callable(outs_np) -> None)."""
+    from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
+    from oracle.metrics import max_rel_err
+    g = np.random.default_rng(seed)
+    if kind == tk.BE_SGEMM:
+        M, N, K = (256, 256, 256) if size == "small" else (1024, 1536, 512)
+        A, B = synth.sgemm_inputs(M, N, K, seed)
+        dA, dB = t(A), t(B)
+        dC = torch.zeros(M, N, device=dev())
+        ref, S = obe.sgemm(A, B)
+
+        def check(o):
+            assert max_rel_err(o[0], ref, S) <= 1e-5
+        return dict(desc=tk.be_sgemm(dA, dB, dC), outs=[dC], reset=lambda: dC.zero_(), check=check,
+                    keep=(dA, dB))
+    if kind == tk.BE_STENCIL:
+        nx, ny, nz = (70, 37, 9) if size == "small" else (512, 512, 64)
+        A = synth.stencil_inputs(nx, ny, nz, seed)
+        dA = t(A)
+        dN = torch.zeros_like(dA)
+        c0, c1 = np.float32(1 / 6), np.float32(1 / 36)
+        ref, S = obe.stencil(A, c0, c1)
+
+        def check(o):
+            assert max_rel_err(o[0], ref, S) <= 1e-5
+        return dict(desc=tk.be_stencil(dA, dN, float(c0), float(c1)), outs=[dN], reset=lambda: dN.zero_(),
+                    check=check, keep=(dA,))
+    if kind == tk.BE_MRIQ_Q:
+        N, nk = (12, 700) if size == "small" else (32, 1024)
+        d = synth.mriq_inputs(N, nk, seed)
+        pm = (d["phiR"].astype(np.float32) ** 2 + d["phiI"].astype(np.float32) ** 2).astype(np.float32)
+        dd = {k: t(v) for k, v in d.items()}
+        dpm = t(pm)
+        Qr = torch.zeros(N ** 3, device=dev())
+        Qi = torch.zeros(N ** 3, device=dev())
+        rr, ri, sr, si = obe.mriq_q(d["x"], d["y"], d["z"], d["kx"], d["ky"], d["kz"], pm)
+
+        def check(o):
+            assert max_rel_err(o[0], rr, sr) <= 1e-5
+            assert max_rel_err(o[1], ri, si) <= 1e-5
+
+        def reset():
+            Qr.zero_()
+            Qi.zero_()
+        desc = tk.be_mriq_q(dd["x"], dd["y"], dd["z"], dd["kx"], dd["ky"], dd["kz"], dpm, Qr, Qi)
+        return dict(desc=desc, outs=[Qr, Qi], reset=reset, check=check, keep=(dd, dpm))
+    if kind == tk.BE_MRIQ_PHIMAG:
+        nk = 3000
+        d = synth.mriq_inputs(4, nk, seed)
+        r, i = t(d["phiR"]), t(d["phiI"])
+        out = torch.zeros(nk, device=dev())
+        ref, S = obe.mriq_phimag(d["phiR"], d["phiI"])
+
+        def check(o):
+            assert max_rel_err(o[0], ref, S) <= 1e-5
+        return dict(desc=tk.be_mriq_phimag(r, i, out), outs=[out], reset=lambda: out.zero_(), check=check,
+                    keep=(r, i))
+    if kind == tk.BE_LBM:
+        nx, ny, nz = (20, 14, 11) if size == "small" else (120, 120, 150)
+        f, fl = synth.lbm_inputs(nx, ny, nz, seed)
+        df, dfl = t(f), t(fl.astype(np.uint32).view(np.int32))
+        dst = torch.zeros_like(df)
+        ref, S = obe.lbm_step(f, fl, np.zeros_like(f))
+        mask = obe.lbm_written_mask(nx, ny, nz)
+
+        def check(o):
+            assert max_rel_err(o[0][mask], ref[mask], S[mask]) <= 1e-5
+            assert np.all(o[0][~mask] == 0)
+        return dict(desc=tk.be_lbm(df, dst, dfl), outs=[dst], reset=lambda: dst.zero_(), check=check, keep=(df, dfl))
+    if kind == tk.BE_SPMV_JDS:
+        R = 3000 if size == "small" else 1 << 16
+        rp, cols, vals, x = synth.spmv_inputs(R, seed, mean_len=16)
+        perm, rl, jp, jc, jv = obe.jds_build(rp, cols, vals)
+        ds = [t(a) for a in (perm, rl, jp, jc, jv, x)]
+        y = torch.zeros(R, device=dev())
+        ref, S = obe.spmv_jds(perm, rl, jp, jc, jv, x)
+
+        def check(o):
+            assert max_rel_err(o[0], ref, S) <= 1e-5
+        return dict(desc=tk.be_spmv(*ds, y), outs=[y], reset=lambda: y.zero_(), check=check, keep=ds)
+    if kind == tk.BE_HISTO:
+        n = 1035840 if size == "small" else 1 << 24
+        v = synth.histo_inputs(n, 4096, seed, "skewed")
+        dv = t(v.view(np.int32))
+        cnt = torch.zeros(4096, dtype=torch.int32, device=dev())
+        ref = obe.histo(v, 4096)
+
+        def check(o):
+            assert np.array_equal(o[0].view(np.uint32), ref)
+            assert int(o[0].astype(np.int64).sum()) == n
+        return dict(desc=tk.be_histo(dv, cnt, 4096), outs=[cnt], reset=lambda: cnt.zero_(), check=check, keep=(dv,))
+    if kind == tk.BE_FMA_BURN:
+        n, iters = 128 * 300, 1000
+        out = torch.zeros(n, device=dev())
+        ref = obe.fma_burn(n, iters)
+
+        def check(o):
+            assert max_rel_err(o[0], ref) <= 1e-5
+        return dict(desc=tk.be_fma_burn(out, iters), outs=[out], reset=lambda: out.zero_(), check=check, keep=())
+    raise ValueError(kind)

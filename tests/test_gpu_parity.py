@@ -1,0 +1,180 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element,
+and fused launches bit-identical to the original launches (BASELINE correctness gates)."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import be as obe, lc as olc
+from oracle.metrics import max_rel_err
+
+pytestmark = pytest.mark.gpu
+
+from tests.gpu_helpers import be_case, dev, host, t  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def tk():
+    from paper_conf_hpca_zhaocczlllg22_b200 import tacker
+    assert torch.cuda.is_available()
+    return tacker
+
+
+# ------------------------------------------------------------------ LC GEMM (c1)
+@pytest.mark.parametrize("M,N,K,bn", [(256, 256, 256, 0), (256, 256, 256, 64), (256, 256, 256, 256),
+                                      (300, 136, 200, 128), (1, 8, 8, 64), (129, 264, 72, 256), (1000, 512, 1024, 128)])
+def test_lc_gemm_vs_oracle(tk, M, N, K, bn):
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=M + N + K)
+    D = torch.full((M, N), float("nan"), device=dev())
+    tk.tacker_launch_original(tk.lc_gemm(t(A), t(B), D, tile_n=bn), None)
+    ref, S = olc.lc_gemm(A, B)
+    assert max_rel_err(host(D), ref, S) <= 1e-2
+    assert max_rel_err(host(D), ref, S) <= 1e-5   # fp32 accumulation: far inside the gate
+
+
+@pytest.mark.parametrize("variant", ["int", "identity", "onehot"])
+def test_lc_gemm_exact_variants(tk, variant):
+    M, N, K = 256, 256, 256
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=7, variant=variant)
+    D = torch.zeros(M, N, device=dev())
+    tk.tacker_launch_original(tk.lc_gemm(t(A), t(B), D), None)
+    ref, _ = olc.lc_gemm(A, B)
+    assert np.array_equal(host(D).astype(np.float64), ref)
+
+
+def test_lc_gemm_f16_epilogue(tk):
+    M, N, K = 200, 192, 128
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=9)
+    bias = np.random.default_rng(0).uniform(-0.5, 0.5, N).astype(np.float32)
+    res = np.random.default_rng(1).uniform(-1, 1, (M, N)).astype(np.float16)
+    D = torch.zeros(M, N, dtype=torch.float16, device=dev())
+    tk.tacker_launch_original(tk.lc_gemm(t(A), t(B), D, bias=t(bias), relu=True, residual=t(res)), None)
+    ref, S = olc.lc_gemm(A, B, bias=bias, relu=True, residual=res)
+    got = host(D).astype(np.float64)
+    assert max_rel_err(got, ref, S + 1e-3) <= 1e-2
+
+
+# ------------------------------------------------------------------ LC conv (c2)
+CONV_CASES = [synth.ConvShape("3x3s1", 1, 14, 14, 64, 64, 3, 3, 1, 1),
+              synth.ConvShape("3x3s2", 1, 28, 28, 128, 128, 3, 3, 2, 1),
+              synth.ConvShape("1x1s1", 1, 28, 28, 256, 128, 1, 1, 1, 0),
+              synth.ConvShape("1x1s2", 1, 56, 56, 64, 256, 1, 1, 2, 0),
+              synth.ConvShape("7x7", 1, 7, 7, 512, 512, 3, 3, 1, 1),
+              synth.ConvShape("b2", 2, 9, 11, 64, 72, 3, 3, 1, 1)]
+
+
+@pytest.mark.parametrize("cs", CONV_CASES, ids=lambda c: c.name)
+def test_lc_conv_vs_oracle(tk, cs):
+    x, w, b = synth.conv_inputs(cs, seed=3)
+    out = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    tk.tacker_launch_original(tk.lc_conv(t(x), t(w), out, cs.stride, cs.pad, bias=t(b), relu=True), None)
+    ref, S = olc.lc_conv(x, w, cs.stride, cs.pad, bias=b, relu=True)
+    assert max_rel_err(host(out).astype(np.float64), ref, S) <= 1e-2
+
+
+# ------------------------------------------------------------------ BE originals (c3-c10)
+BE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_MRIQ_PHIMAG", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN"]
+
+
+@pytest.mark.parametrize("kind", BE_KINDS)
+def test_be_original_vs_oracle(tk, kind):
+    c = be_case(getattr(tk, kind))
+    c["reset"]()
+    tk.tacker_launch_original(None, c["desc"])
+    c["check"]([host(o) for o in c["outs"]])
+
+
+def test_bfs_levels_vs_oracle(tk):
+    V = 1 << 14
+    rp, col = synth.bfs_inputs(V, seed=5)
+    drp, dcol = t(rp), t(col)
+    level = torch.full((V,), -1, dtype=torch.int32, device=dev())
+    level[0] = 0
+    mask = torch.zeros(V, dtype=torch.uint8, device=dev())
+    mask[0] = 1
+    visited = mask.clone()
+    upd = torch.zeros_like(mask)
+    over = torch.zeros(1, dtype=torch.int32, device=dev())
+    e = tk.be_bfs_expand(drp, dcol, level, mask, visited, upd)
+    cm = tk.be_bfs_commit(mask, visited, upd, over)
+    for _ in range(V):
+        over.zero_()
+        tk.tacker_launch_original(None, e)
+        tk.tacker_launch_original(None, cm)
+        if int(over.item()) == 0:
+            break
+    assert np.array_equal(host(level), obe.bfs_levels(rp, col))
+
+
+# ------------------------------------------------------------------ fused (a1-a8)
+FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN"]
+
+
+@pytest.mark.parametrize("kind", FUSE_KINDS)
+@pytest.mark.parametrize("ws", [4, 16])
+def test_fused_bit_identical_to_original(tk, kind, ws):
+    M, N, K = 256, 256, 256
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=1)
+    dA, dB = t(A), t(B)
+    D0 = torch.zeros(M, N, device=dev())
+    D1 = torch.zeros(M, N, device=dev())
+    c = be_case(getattr(tk, kind), seed=2)
+    # original launches
+    c["reset"]()
+    tk.tacker_launch_original(tk.lc_gemm(dA, dB, D0), c["desc"])
+    orig = [host(o).copy() for o in c["outs"]]
+    c["check"](orig)
+    # fused launch, twice (the BE ticket must self-reset)
+    f = tk.tacker_fuse(tk.lc_gemm(dA, dB, D1), c["desc"], ws)
+    for _ in range(2):
+        c["reset"]()
+        D1.zero_()
+        f.launch()
+        fused = [host(o) for o in c["outs"]]
+        for a, b in zip(orig, fused):
+            assert a.tobytes() == b.tobytes()
+        assert host(D1).tobytes() == host(D0).tobytes()
+    ref, S = olc.lc_gemm(A, B)
+    assert max_rel_err(host(D1), ref, S) <= 1e-2
+
+
+def test_fused_large_lc_many_tiles(tk):
+    # more LC tiles than CTAs (persistent tile loop, TMEM double buffer) + sgemm BE
+    M, N, K = 4096, 1024, 512
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=4)
+    D = torch.zeros(M, N, device=dev())
+    c = be_case(tk.BE_SGEMM, seed=3, size="large")
+    c["reset"]()
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], 8)
+    assert f.info().lc_tiles > f.info().grid
+    f.launch()
+    ref, S = olc.lc_gemm(A, B)
+    assert max_rel_err(host(D), ref, S) <= 1e-5
+    c["check"]([host(o) for o in c["outs"]])
+
+
+def test_fused_conv_stencil(tk):
+    cs = synth.ConvShape("c", 1, 28, 28, 128, 128, 3, 3, 1, 1)
+    x, w, b = synth.conv_inputs(cs, seed=6)
+    out = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    c = be_case(tk.BE_STENCIL, seed=8)
+    c["reset"]()
+    f = tk.tacker_fuse(tk.lc_conv(t(x), t(w), out, 1, 1, bias=t(b), relu=True), c["desc"], 8)
+    f.launch()
+    ref, S = olc.lc_conv(x, w, 1, 1, bias=b, relu=True)
+    assert max_rel_err(host(out).astype(np.float64), ref, S) <= 1e-2
+    c["check"]([host(o) for o in c["outs"]])
+
+
+def test_ptb_orig_blocks_prefix(tk):
+    # orig_blocks < whole problem: only the first blocks run (PTB runtime argument, Fig. 7)
+    n, iters = 128 * 64, 10
+    out = torch.zeros(n, device=dev())
+    A, B = synth.lc_gemm_inputs(128, 128, 64, seed=0)
+    D = torch.zeros(128, 128, device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), tk.be_fma_burn(out, iters, orig_blocks=10), 4)
+    f.launch()
+    o = host(out)
+    ref = obe.fma_burn(n, iters)
+    assert max_rel_err(o[:1280], ref[:1280]) <= 1e-5
+    assert np.all(o[1280:] == 0)
