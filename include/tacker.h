@@ -102,7 +102,9 @@ typedef enum {
   TACKER_BE_BFS_EXPAND = 9,   /* Rodinia BFS kernel 1; block = 128 nodes                   */
   TACKER_BE_BFS_COMMIT = 10,  /* Rodinia BFS kernel 2; block = 128 nodes                   */
   TACKER_BE_FMA_BURN = 11,    /* register-only FMA chains (Kc, §III-B); block = 128 thr.   */
-  TACKER_BE_KIND_COUNT = 12
+  TACKER_BE_IM2COL = 12,      /* LC CUDA-core helper: explicit im2col (cudnnIm2col, §VIII-H
+                                 P:3350-3381) NHWC fp16 -> [M, Kpad] fp16; block = 1024x8 el. */
+  TACKER_BE_KIND_COUNT = 13
 } tacker_be_kind;
 
 typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
@@ -124,6 +126,13 @@ typedef struct { int32_t n, nbins; const uint32_t *in; uint32_t *count; } tacker
 typedef struct { int32_t V; const int32_t *row_ptr, *col; int32_t *level; uint8_t *mask; const uint8_t *visited; uint8_t *upd; } tacker_be_bfs_expand;
 typedef struct { int32_t V; uint8_t *mask, *visited, *upd; int32_t *over; } tacker_be_bfs_commit;
 typedef struct { int32_t n_threads, iters; float a; float b; float *out; } tacker_be_fma_burn;
+/* out[m, kk] = x[n, p*stride-pad+r, q*stride-pad+s, c] with m = (n*P+p)*Q+q, kk = (r*S+s)*C+c,
+ * 0 outside the image and for kk >= R*S*C (row padded to Kpad, a multiple of 8). */
+typedef struct {
+  int32_t n, h, w, c, r, s, stride, pad, Kpad;
+  const void *x;   /* fp16 NHWC */
+  void *out;       /* fp16 [n*P*Q, Kpad] */
+} tacker_be_im2col;
 
 typedef struct {
   int32_t kind;              /* tacker_be_kind */
@@ -140,6 +149,7 @@ typedef struct {
     tacker_be_bfs_expand bfs_expand;
     tacker_be_bfs_commit bfs_commit;
     tacker_be_fma_burn fma_burn;
+    tacker_be_im2col im2col;
     uint8_t _pad[128];
   } p;
 } tacker_be_desc;

@@ -74,6 +74,30 @@ def lc_conv(x, w, stride: int, pad: int, bias=None, relu=False, residual=None):
     return out, S
 
 
+def im2col(x, r, s, stride, pad, Kpad):
+    """Explicit im2col of the paper's conv->GEMM lowering (cudnnIm2col, §VIII-H):
+    out[m, kk] = x[n, p*st-pad+rr, q*st-pad+ss, c], m = (n*P+p)*Q+q, kk = (rr*S+ss)*C+c;
+    0 outside the image and for kk >= R*S*C.  Exact copy (same dtype as x)."""
+    n, h, wd, c = x.shape
+    P = (h + 2 * pad - r) // stride + 1
+    Q = (wd + 2 * pad - s) // stride + 1
+    out = np.zeros((n * P * Q, Kpad), x.dtype)
+    for ni in range(n):
+        for pi in range(P):
+            for qi in range(Q):
+                m = (ni * P + pi) * Q + qi
+                for rr in range(r):
+                    hh = pi * stride - pad + rr
+                    if hh < 0 or hh >= h:
+                        continue
+                    for ss in range(s):
+                        ww = qi * stride - pad + ss
+                        if ww < 0 or ww >= wd:
+                            continue
+                        out[m, (rr * s + ss) * c:(rr * s + ss + 1) * c] = x[ni, hh, ww, :]
+    return out
+
+
 def lc_conv_point(x, w, stride, pad, n, p, q, k):
     """One output element of lc_conv by explicit loops (for sampled full-size checks)."""
     x64 = np.asarray(x, np.float64)

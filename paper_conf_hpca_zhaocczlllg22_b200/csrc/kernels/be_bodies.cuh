@@ -147,47 +147,89 @@ template <> struct BeBody<TACKER_BE_FMA_BURN> {
 };
 
 // ---------------------------------------------------------------- stencil (Parboil)
-// One 7-point Jacobi sweep over A0[nz][ny][nx] (x fastest).  Block = 32x4 (x,y) columns,
-// swept over all z with the column's z-1/z/z+1 values in registers; x+-1, y+-1 neighbours come
-// through L1.  Interior: An = c1*(((((W+E)+S)+N)+B)+T) - c0*A; boundary cells copied.
+// One 7-point Jacobi sweep over A0[nz][ny][nx] (x fastest), HBM-bound.  Block = 128 x 4 x 4
+// (x,y,z) cells: lane l of warp w owns x = 4l..4l+3 (one float4) of row y = w for ZC = 4 planes.
+// The centre column's ZC+2 planes are loaded up front (memory-level parallelism), x+-1 comes
+// from the neighbouring lanes' float4 by shuffle, y+-1 rows through L1/L2.
+//   interior: An = c1*(((((W+E)+S)+N)+B)+T) - c0*A   (S/N = y-1/y+1, B/T = z-1/z+1)
+//   boundary cells (x, y or z on the faces) are copied.
+// nx % 4 != 0 uses the scalar path with the same per-element arithmetic.
 template <> struct BeBody<TACKER_BE_STENCIL> {
   static constexpr uint32_t kSmem = 0;
+  static constexpr int ZC = 4;
   static __host__ __device__ int64_t num_blocks(const tacker_be_stencil &p) {
-    return (int64_t)((p.nx + 31) / 32) * ((p.ny + 3) / 4);
+    return (int64_t)((p.nx + 127) / 128) * ((p.ny + 3) / 4) * ((p.nz + ZC - 1) / ZC);
+  }
+  static __device__ __forceinline__ float point(const tacker_be_stencil &p, float w, float e, float s, float n,
+                                                float b, float t, float c) {
+    float sum = __fadd_rn(w, e);
+    sum = __fadd_rn(sum, s);
+    sum = __fadd_rn(sum, n);
+    sum = __fadd_rn(sum, b);
+    sum = __fadd_rn(sum, t);
+    return __fsub_rn(__fmul_rn(p.c1, sum), __fmul_rn(p.c0, c));
   }
   static __device__ __forceinline__ void run(const tacker_be_stencil &p, int64_t vb, int tid, uint32_t,
                                              uint8_t *) {
-    const int bx = (p.nx + 31) / 32;
-    const int x = (int)(vb % bx) * 32 + (tid & 31);
-    const int y = (int)(vb / bx) * 4 + (tid >> 5);
-    if (x >= p.nx || y >= p.ny) return;
+    const int bx = (p.nx + 127) / 128, by = (p.ny + 3) / 4;
+    const int zb = (int)(vb / ((int64_t)bx * by));
+    const int rem = (int)(vb % ((int64_t)bx * by));
+    const int lane = tid & 31;
+    const int x0 = (rem % bx) * 128 + 4 * lane;
+    const int y = (rem / bx) * 4 + (tid >> 5);
+    const int z0 = zb * ZC;
+    if (y >= p.ny) return;                     // warp-uniform
     const size_t plane = (size_t)p.nx * p.ny;
-    const float *A = p.A0;
-    float *An = p.Anext;
-    const size_t col = (size_t)y * p.nx + x;
-    const bool border = (x == 0) | (x == p.nx - 1) | (y == 0) | (y == p.ny - 1) | (p.nz < 3);
-    if (border) {
-      for (int z = 0; z < p.nz; ++z) An[z * plane + col] = __ldg(A + z * plane + col);
+    const float *__restrict__ A = p.A0;
+    float *__restrict__ An = p.Anext;
+    const bool ybord = (y == 0) | (y == p.ny - 1);
+    if ((p.nx & 3) == 0) {
+      const bool act = x0 < p.nx;
+      const size_t row = (size_t)y * p.nx + x0;
+      float4 c[ZC + 2];
+#pragma unroll
+      for (int i = 0; i < ZC + 2; ++i) {
+        const int z = z0 - 1 + i;
+        c[i] = (act && z >= 0 && z < p.nz) ? __ldg(reinterpret_cast<const float4 *>(A + z * plane + row))
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+#pragma unroll
+      for (int i = 0; i < ZC; ++i) {
+        const int z = z0 + i;
+        if (z >= p.nz) break;                  // warp-uniform
+        const float4 cc = c[i + 1];
+        float wv = __shfl_up_sync(0xffffffffu, cc.w, 1);
+        float ev = __shfl_down_sync(0xffffffffu, cc.x, 1);
+        if (!act) continue;
+        float4 o = cc;
+        const bool zb_ = (z == 0) | (z == p.nz - 1);
+        if (!ybord && !zb_) {
+          if (lane == 0) wv = x0 > 0 ? __ldg(A + z * plane + row - 1) : 0.f;
+          if (lane == 31 || x0 + 4 >= p.nx) ev = x0 + 4 < p.nx ? __ldg(A + z * plane + row + 4) : 0.f;
+          const float4 s = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row - p.nx));
+          const float4 n = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row + p.nx));
+          const float4 b = c[i], t = c[i + 2];
+          if (x0 > 0) o.x = point(p, wv, cc.y, s.x, n.x, b.x, t.x, cc.x);
+          o.y = point(p, cc.x, cc.z, s.y, n.y, b.y, t.y, cc.y);
+          o.z = point(p, cc.y, cc.w, s.z, n.z, b.z, t.z, cc.z);
+          if (x0 + 3 < p.nx - 1) o.w = point(p, cc.z, ev, s.w, n.w, b.w, t.w, cc.w);
+        }
+        *reinterpret_cast<float4 *>(An + z * plane + row) = o;
+      }
       return;
     }
-    float below = __ldg(A + col);
-    float cur = __ldg(A + plane + col);
-    An[col] = below;
-    for (int z = 1; z < p.nz - 1; ++z) {
-      const size_t o = z * plane + col;
-      const float above = __ldg(A + o + plane);
-      const float w = __ldg(A + o - 1), e = __ldg(A + o + 1);
-      const float s = __ldg(A + o - p.nx), n = __ldg(A + o + p.nx);
-      float sum = __fadd_rn(w, e);
-      sum = __fadd_rn(sum, s);
-      sum = __fadd_rn(sum, n);
-      sum = __fadd_rn(sum, below);
-      sum = __fadd_rn(sum, above);
-      An[o] = __fsub_rn(__fmul_rn(p.c1, sum), __fmul_rn(p.c0, cur));
-      below = cur;
-      cur = above;
+    // scalar path (nx % 4 != 0)
+    for (int e = 0; e < 4; ++e) {
+      const int x = x0 + e;
+      if (x >= p.nx) break;
+      const size_t col = (size_t)y * p.nx + x;
+      for (int z = z0; z < min(z0 + ZC, p.nz); ++z) {
+        const size_t o = z * plane + col;
+        const bool bord = ybord | (x == 0) | (x == p.nx - 1) | (z == 0) | (z == p.nz - 1);
+        An[o] = bord ? A[o]
+                     : point(p, A[o - 1], A[o + 1], A[o - p.nx], A[o + p.nx], A[o - plane], A[o + plane], A[o]);
+      }
     }
-    An[(size_t)(p.nz - 1) * plane + col] = cur;
   }
 };
 
@@ -208,21 +250,28 @@ template <> struct BeBody<TACKER_BE_MRIQ_PHIMAG> {
   }
 };
 
-// Q: block = 256 voxels (thread owns tid and tid+128); k staged through shared memory in
+// Q: block = 512 voxels (thread owns tid + 128h, h < 4); k staged through shared memory in
 // chunks of 512 as float4 (kx, ky, kz, phiMag).  Phase in turns t = kx x + ky y + kz z is
-// range-reduced exactly (t - rint(t), Sterbenz) before the MUFU sin/cos of 2*pi*t.
+// range-reduced exactly (t - rint(t), Sterbenz; rint by the 1.5*2^23 magic add so the XU pipe
+// only runs the two MUFU ops) before the MUFU sin/cos of 2*pi*t.
 template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   static constexpr int KC = 512;
+  static constexpr int VPT = 4;   // voxels per thread
   static constexpr uint32_t kSmem = KC * 16;
-  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) { return (p.numX + 255) / 256; }
+  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) {
+    return (p.numX + 128 * VPT - 1) / (128 * VPT);
+  }
   static __device__ __forceinline__ void run(const tacker_be_mriq_q &p, int64_t vb, int tid, uint32_t bar,
                                              uint8_t *smem) {
     float4 *ks = reinterpret_cast<float4 *>(smem);
     const float kTwoPi = 6.2831853071795864769f;
-    int64_t v[2] = {vb * 256 + tid, vb * 256 + 128 + tid};
-    float xs[2], ys[2], zs[2], qr[2], qi[2];
+    const float kMagic = 12582912.0f;   // 1.5 * 2^23: (t + M) - M == rint(t) for |t| < 2^22
+    int64_t v[VPT];
+    float xs[VPT], ys[VPT], zs[VPT], qr[VPT], qi[VPT];
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
+    for (int h = 0; h < VPT; ++h) v[h] = vb * (128 * VPT) + h * 128 + tid;
+#pragma unroll
+    for (int h = 0; h < VPT; ++h) {
       const bool ok = v[h] < p.numX;
       xs[h] = ok ? p.x[v[h]] : 0.f;
       ys[h] = ok ? p.y[v[h]] : 0.f;
@@ -236,13 +285,14 @@ template <> struct BeBody<TACKER_BE_MRIQ_Q> {
       for (int k = tid; k < kn; k += kVbThreads)
         ks[k] = make_float4(p.kx[k0 + k], p.ky[k0 + k], p.kz[k0 + k], p.phiMag[k0 + k]);
       named_bar_sync(bar, kVbThreads);
-#pragma unroll 4
+#pragma unroll 2
       for (int k = 0; k < kn; ++k) {
         const float4 kv = ks[k];
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
+        for (int h = 0; h < VPT; ++h) {
           float t = __fmaf_rn(kv.z, zs[h], __fmaf_rn(kv.y, ys[h], __fmul_rn(kv.x, xs[h])));
-          t = __fsub_rn(t, rintf(t));
+          const float r = __fsub_rn(__fadd_rn(t, kMagic), kMagic);
+          t = __fsub_rn(t, r);
           const float arg = __fmul_rn(kTwoPi, t);
           float s, c;
           __sincosf(arg, &s, &c);
@@ -252,7 +302,7 @@ template <> struct BeBody<TACKER_BE_MRIQ_Q> {
       }
     }
 #pragma unroll
-    for (int h = 0; h < 2; ++h)
+    for (int h = 0; h < VPT; ++h)
       if (v[h] < p.numX) {
         p.Qr[v[h]] = qr[h];
         p.Qi[v[h]] = qi[h];
@@ -427,6 +477,60 @@ template <> struct BeBody<TACKER_BE_BFS_COMMIT> {
   }
 };
 
+// ---------------------------------------------------------------- im2col (LC CUDA-core helper)
+// Explicit im2col as in the paper's conv->GEMM lowering (cudnnIm2col, §VIII-H):
+// block = 1024 groups of 8 consecutive output columns (16 B); with C % 8 == 0 a group is one
+// filter tap's 8 channels, copied as one 16-byte load (zero outside the image / past R*S*C).
+template <> struct BeBody<TACKER_BE_IM2COL> {
+  static constexpr uint32_t kSmem = 0;
+  static __host__ __device__ int64_t rows(const tacker_be_im2col &p) {
+    const int P = (p.h + 2 * p.pad - p.r) / p.stride + 1, Q = (p.w + 2 * p.pad - p.s) / p.stride + 1;
+    return (int64_t)p.n * P * Q;
+  }
+  static __host__ __device__ int64_t num_blocks(const tacker_be_im2col &p) {
+    return (rows(p) * (p.Kpad / 8) + 1023) / 1024;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_im2col &p, int64_t vb, int tid, uint32_t, uint8_t *) {
+    const int P = (p.h + 2 * p.pad - p.r) / p.stride + 1, Q = (p.w + 2 * p.pad - p.s) / p.stride + 1;
+    const int64_t groups_per_row = p.Kpad / 8;
+    const int64_t total = (int64_t)p.n * P * Q * groups_per_row;
+    const int Kreal = p.r * p.s * p.c;
+    const __half *x = reinterpret_cast<const __half *>(p.x);
+    __half *out = reinterpret_cast<__half *>(p.out);
+#pragma unroll 2
+    for (int u = 0; u < 8; ++u) {
+      const int64_t g = vb * 1024 + u * 128 + tid;
+      if (g >= total) return;
+      const int64_t m = g / groups_per_row;
+      const int kk0 = (int)(g % groups_per_row) * 8;
+      const int q = (int)(m % Q), pp = (int)((m / Q) % P), n = (int)(m / ((int64_t)P * Q));
+      uint4 v = make_uint4(0, 0, 0, 0);
+      if ((p.c & 7) == 0) {
+        if (kk0 < Kreal) {
+          const int c = kk0 % p.c, rs = kk0 / p.c, s = rs % p.s, r = rs / p.s;
+          const int hi = pp * p.stride - p.pad + r, wi = q * p.stride - p.pad + s;
+          if (hi >= 0 && hi < p.h && wi >= 0 && wi < p.w)
+            v = __ldg(reinterpret_cast<const uint4 *>(x + (((int64_t)n * p.h + hi) * p.w + wi) * p.c + c));
+        }
+      } else {
+        __align__(16) __half e[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int kk = kk0 + j;
+          e[j] = __float2half(0.f);
+          if (kk < Kreal) {
+            const int c = kk % p.c, rs = kk / p.c, s = rs % p.s, r = rs / p.s;
+            const int hi = pp * p.stride - p.pad + r, wi = q * p.stride - p.pad + s;
+            if (hi >= 0 && hi < p.h && wi >= 0 && wi < p.w) e[j] = x[(((int64_t)n * p.h + hi) * p.w + wi) * p.c + c];
+          }
+        }
+        v = *reinterpret_cast<uint4 *>(e);
+      }
+      *reinterpret_cast<uint4 *>(out + m * p.Kpad + kk0) = v;
+    }
+  }
+};
+
 // ---------------------------------------------------------------- dispatch helpers
 template <int KIND> struct BeSel;
 #define TK_BE_SEL(K, FIELD)                                                            \
@@ -443,6 +547,17 @@ TK_BE_SEL(TACKER_BE_HISTO, histo)
 TK_BE_SEL(TACKER_BE_BFS_EXPAND, bfs_expand)
 TK_BE_SEL(TACKER_BE_BFS_COMMIT, bfs_commit)
 TK_BE_SEL(TACKER_BE_FMA_BURN, fma_burn)
+TK_BE_SEL(TACKER_BE_IM2COL, im2col)
 #undef TK_BE_SEL
+
+// Maximum BE warps per fused CTA: register-heavy bodies (sgemm's 8x4 register tile) keep the
+// CTA at 6+16 warps (80 registers/thread); the others allow 6+24 warps (64 registers/thread).
+__host__ __device__ constexpr int be_max_warps(int kind) { return kind == TACKER_BE_SGEMM ? 16 : 24; }
+
+// Every implemented BE kind (X-macro used by the host dispatch tables).
+#define TK_FOR_EACH_BE(X)                                                                       \
+  X(TACKER_BE_SGEMM) X(TACKER_BE_STENCIL) X(TACKER_BE_MRIQ_PHIMAG) X(TACKER_BE_MRIQ_Q)          \
+  X(TACKER_BE_LBM) X(TACKER_BE_SPMV_JDS) X(TACKER_BE_HISTO) X(TACKER_BE_BFS_EXPAND)             \
+  X(TACKER_BE_BFS_COMMIT) X(TACKER_BE_FMA_BURN) X(TACKER_BE_IM2COL)
 
 }  // namespace tk

@@ -239,17 +239,19 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   volatile uint32_t *s_ticket = reinterpret_cast<volatile uint32_t *>(slice);
   uint8_t *body_smem = slice + 16;
   const auto &bp = BeSel<BE_KIND>::get(P.be);
-  for (;;) {
-    if (tid == 0) *s_ticket = atomicAdd(&P.work->ticket, 1u);
-    named_bar_sync(bar, kVbThreads);
-    const int64_t vb = *s_ticket;
-    named_bar_sync(bar, kVbThreads);
-    if (vb >= P.be_blocks) break;
+  const uint32_t groups = gridDim.x * (uint32_t)P.be_vb_per_cta;
+  // First round static and interleaved across CTAs (slot j of every CTA before slot j+1, so
+  // a short BE kernel spreads over all SMs); afterwards dynamic tickets balance the tail.
+  int64_t vb = (int64_t)j * gridDim.x + blockIdx.x;
+  while (vb < P.be_blocks) {
     BeBody<BE_KIND>::run(bp, vb, tid, bar, body_smem);
+    if (tid == 0) *s_ticket = groups + atomicAdd(&P.work->ticket, 1u);
+    named_bar_sync(bar, kVbThreads);
+    vb = *s_ticket;
+    named_bar_sync(bar, kVbThreads);
   }
   if (tid == 0) {
     __threadfence();
-    const uint32_t groups = gridDim.x * (uint32_t)P.be_vb_per_cta;
     if (atomicAdd(&P.work->done, 1u) == groups - 1) {   // last group: reset for the next launch
       P.work->ticket = 0;
       P.work->done = 0;
@@ -260,7 +262,8 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 
 // ------------------------------------------------------------------------ the fused kernel
 template <int BN, int BE_KIND>
-__global__ void __launch_bounds__(32 * (kLcWarps + 16), 1) fused_kernel(const __grid_constant__ FusedParams P) {
+__global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
+    fused_kernel(const __grid_constant__ FusedParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *lc = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *be_smem = lc + P.lc_smem_bytes;

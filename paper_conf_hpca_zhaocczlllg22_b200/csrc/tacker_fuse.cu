@@ -54,7 +54,8 @@ int sm_count() {
 
 const char *be_kind_name(int kind) {
   static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
-                                "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn"};
+                                "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn",
+                                "im2col"};
   return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
 }
 
@@ -65,7 +66,6 @@ using namespace tkrt;
 // ============================================================================ constants
 static constexpr int kSmemCap = 232448;      // max dynamic SMEM per CTA on sm_100 (227 KB)
 static constexpr int kTmemCols = 512;
-static constexpr int kMaxBeWarps = 16;       // fused_kernel __launch_bounds__ sizing
 static constexpr int kMaxWarps = 32;
 static constexpr int kMinLcSmem = 120 * 1024;  // forces one LC CTA per SM (TMEM ownership)
 
@@ -79,16 +79,7 @@ static bool be_num_blocks(const tacker_be_desc &d, int64_t *out) {
   switch (d.kind) {
 #define C(K) \
   case K: *out = be_blocks_t<K>(d); return true;
-    C(TACKER_BE_SGEMM)
-    C(TACKER_BE_STENCIL)
-    C(TACKER_BE_MRIQ_PHIMAG)
-    C(TACKER_BE_MRIQ_Q)
-    C(TACKER_BE_LBM)
-    C(TACKER_BE_SPMV_JDS)
-    C(TACKER_BE_HISTO)
-    C(TACKER_BE_BFS_EXPAND)
-    C(TACKER_BE_BFS_COMMIT)
-    C(TACKER_BE_FMA_BURN)
+    TK_FOR_EACH_BE(C)
 #undef C
     default: return false;
   }
@@ -98,16 +89,7 @@ static uint32_t be_smem_bytes(int kind) {
   switch (kind) {
 #define C(K) \
   case K: return BeBody<K>::kSmem;
-    C(TACKER_BE_SGEMM)
-    C(TACKER_BE_STENCIL)
-    C(TACKER_BE_MRIQ_PHIMAG)
-    C(TACKER_BE_MRIQ_Q)
-    C(TACKER_BE_LBM)
-    C(TACKER_BE_SPMV_JDS)
-    C(TACKER_BE_HISTO)
-    C(TACKER_BE_BFS_EXPAND)
-    C(TACKER_BE_BFS_COMMIT)
-    C(TACKER_BE_FMA_BURN)
+    TK_FOR_EACH_BE(C)
 #undef C
     default: return 0;
   }
@@ -151,6 +133,14 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
     case TACKER_BE_BFS_EXPAND:
     case TACKER_BE_BFS_COMMIT:
       break;
+    case TACKER_BE_IM2COL: {
+      const auto &p = d.p.im2col;
+      if (p.n <= 0 || p.h <= 0 || p.w <= 0 || p.c <= 0 || p.r <= 0 || p.s <= 0 || p.stride <= 0 || p.pad < 0 ||
+          !p.x || !p.out)
+        return set_error("im2col: bad args"), TACKER_EINVAL;
+      if (p.Kpad % 8 || p.Kpad < p.r * p.s * p.c) return set_error("im2col: Kpad must be a multiple of 8 >= R*S*C"), TACKER_EINVAL;
+      break;
+    }
     case TACKER_BE_FMA_BURN:
       if (d.p.fma_burn.n_threads < 0 || d.p.fma_burn.iters < 0 || !d.p.fma_burn.out)
         return set_error("fma_burn: bad args"), TACKER_EINVAL;
@@ -283,16 +273,7 @@ static KernelFn fused_fn(int be_kind) {
     case TACKER_BE_NONE: return fused_kernel<BN, TACKER_BE_NONE>;
 #define C(K) \
   case K: return fused_kernel<BN, K>;
-    C(TACKER_BE_SGEMM)
-    C(TACKER_BE_STENCIL)
-    C(TACKER_BE_MRIQ_PHIMAG)
-    C(TACKER_BE_MRIQ_Q)
-    C(TACKER_BE_LBM)
-    C(TACKER_BE_SPMV_JDS)
-    C(TACKER_BE_HISTO)
-    C(TACKER_BE_BFS_EXPAND)
-    C(TACKER_BE_BFS_COMMIT)
-    C(TACKER_BE_FMA_BURN)
+    TK_FOR_EACH_BE(C)
 #undef C
     default: return nullptr;
   }
@@ -309,16 +290,7 @@ static BeFn pick_be_original(int kind) {
   switch (kind) {
 #define C(K) \
   case K: return be_original_kernel<K>;
-    C(TACKER_BE_SGEMM)
-    C(TACKER_BE_STENCIL)
-    C(TACKER_BE_MRIQ_PHIMAG)
-    C(TACKER_BE_MRIQ_Q)
-    C(TACKER_BE_LBM)
-    C(TACKER_BE_SPMV_JDS)
-    C(TACKER_BE_HISTO)
-    C(TACKER_BE_BFS_EXPAND)
-    C(TACKER_BE_BFS_COMMIT)
-    C(TACKER_BE_FMA_BURN)
+    TK_FOR_EACH_BE(C)
 #undef C
     default: return nullptr;
   }
@@ -370,8 +342,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   const bool has_lc = lc && lc->kind != TACKER_LC_NONE;
   const bool has_be = be && be->kind != TACKER_BE_NONE;
   if (!has_lc) return set_error("tacker_fuse: an LC descriptor is required"), TACKER_EINVAL;
-  if (has_be && (warp_split < 4 || warp_split % 4 || warp_split > kMaxBeWarps))
-    return set_error("warp_split must be a multiple of 4 in [4, %d] (got %d)", kMaxBeWarps, warp_split), TACKER_EUNSUPPORTED;
+  if (has_be && (warp_split < 4 || warp_split % 4 || warp_split > be_max_warps(be->kind)))
+    return set_error("warp_split must be a multiple of 4 in [4, %d] for BE kind %d (got %d)", be_max_warps(be->kind),
+                     be->kind, warp_split),
+           TACKER_EUNSUPPORTED;
   if (!has_be && warp_split != 0) return set_error("warp_split must be 0 without a BE part"), TACKER_EINVAL;
   const int sms = sm_count();
   if (sms <= 0) return set_error("no CUDA device"), TACKER_ECUDA;

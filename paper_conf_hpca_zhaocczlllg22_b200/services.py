@@ -1,0 +1,164 @@
+"""LC services and BE applications as device-resident kernel lists for the bench and tests.
+
+An LC query is the ordered kernel list of one DNN inference: here the
+convolutions of ResNet-50 / VGG-16 at a given batch (BASELINE configs 2, 4, 5) and BERT-base
+GEMMs (config 3), with synthetic seeded inputs and random weights (no datasets or trained
+weights exist on the box).  conv1 (C=3 padded to 8) runs as the paper's im2col + GEMM
+(§VIII-H): an LC CUDA-core kernel followed by an LC tensor-core kernel; every
+other convolution is an implicit-GEMM tensor-core kernel.  A BE application (Table II)
+is a cyclic list of CUDA-core kernels on its own buffers.
+
+PyTorch allocates device memory only; every kernel is launched through libtacker.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import numpy as np
+import torch
+
+import synth
+from . import tacker as tk
+
+
+@dataclass
+class LcKernelSpec:
+    name: str
+    is_tc: bool
+    lc: object = None       # tk.LcDesc when is_tc
+    cd: object = None       # tk.BeDesc when not is_tc
+    flops: int = 0
+    bytes: int = 0
+    conv: synth.ConvShape | None = None
+
+
+@dataclass
+class LcService:
+    name: str
+    kernels: list
+    buffers: list = field(default_factory=list)   # keeps device tensors alive
+    inputs: list = field(default_factory=list)    # per-query input activations (H2D in e2e)
+    outputs: list = field(default_factory=list)   # per-query results (D2H in e2e)
+
+    def tc_kernels(self):
+        return [k for k in self.kernels if k.is_tc]
+
+
+def _dev(a, dtype=None):
+    t = torch.from_numpy(np.ascontiguousarray(a))
+    if dtype is not None:
+        t = t.to(dtype)
+    return t.cuda()
+
+
+def resnet50_service(batch: int = 1, seed: int = 2022, convs=None) -> LcService:
+    convs = convs if convs is not None else synth.resnet50_convs(batch)
+    ks, bufs, ins, outs = [], [], [], []
+    for i, cs in enumerate(convs):
+        x, w, b = synth.conv_inputs(cs, seed + i, real_c=3 if cs.name == "conv1" else None)
+        dx, dw, db = _dev(x), _dev(w), _dev(b)
+        out = torch.empty(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device="cuda")
+        ins.append(dx)
+        outs.append(out)
+        M, N, K = cs.gemm_mnk
+        byt = 2 * x.size + 2 * w.size + 2 * out.numel()
+        if cs.c % 64 == 0 or (cs.r == 1 and cs.s == 1 and cs.stride == 1):
+            ks.append(LcKernelSpec(cs.name, True, lc=tk.lc_conv(dx, dw, out, cs.stride, cs.pad, bias=db, relu=True),
+                                   flops=2 * M * N * K, bytes=byt, conv=cs))
+            bufs += [dx, dw, db, out]
+        else:   # conv1: explicit im2col (LC CD kernel) + GEMM (LC TC kernel)
+            Kpad = ((K + 63) // 64) * 64
+            cols = torch.empty(M, Kpad, dtype=torch.float16, device="cuda")
+            wf = np.zeros((cs.k, Kpad), np.float16)
+            wf[:, :K] = w.reshape(cs.k, -1)
+            dwf = _dev(wf)
+            ks.append(LcKernelSpec(cs.name + ".im2col", False,
+                                   cd=tk.be_im2col(dx, cols, cs.r, cs.s, cs.stride, cs.pad, Kpad),
+                                   bytes=2 * x.size + 2 * M * Kpad, conv=cs))
+            ks.append(LcKernelSpec(cs.name + ".gemm", True,
+                                   lc=tk.lc_gemm(cols, dwf, out.view(M, cs.k), M=M, N=cs.k, K=Kpad, bias=db, relu=True),
+                                   flops=2 * M * N * K, bytes=2 * M * Kpad + 2 * wf.size + 2 * out.numel(), conv=cs))
+            bufs += [dx, dw, db, out, cols, dwf]
+    return LcService(f"resnet50_b{batch}", ks, bufs, ins, outs[-1:])
+
+
+def vgg16_service(batch: int = 1, seed: int = 2023) -> LcService:
+    return _named(resnet50_service(batch, seed, convs=synth.vgg16_convs(batch)), f"vgg16_b{batch}")
+
+
+def _named(s: LcService, name: str) -> LcService:
+    s.name = name
+    return s
+
+
+def bert_service(seq: int = 128, seed: int = 2024, layers: int = 1) -> LcService:
+    ks, bufs = [], []
+    g = np.random.default_rng(seed)
+    for li in range(layers):
+        for name, M, N, K in synth.bert_base_gemms(seq):
+            A, B = synth.lc_gemm_inputs(M, N, K, seed + li * 10 + N)
+            B = (B.astype(np.float32) / np.sqrt(K)).astype(np.float16)
+            dA, dB = _dev(A), _dev(B)
+            D = torch.empty(M, N, dtype=torch.float16, device="cuda")
+            ks.append(LcKernelSpec(f"l{li}.{name}", True, lc=tk.lc_gemm(dA, dB, D), flops=2 * M * N * K,
+                                   bytes=2 * (M * K + N * K + M * N)))
+            bufs += [dA, dB, D]
+    return LcService(f"bert_base_s{seq}", ks, bufs)
+
+
+# ----------------------------------------------------------------------------- BE applications
+@dataclass
+class BeKernelSpec:
+    name: str
+    desc: object
+    flops: float = 0.0      # FP32 flops (algorithmic)
+    mufu: float = 0.0       # MUFU ops
+    bytes: float = 0.0      # algorithmic DRAM bytes
+    bound: str = "hbm"
+
+
+@dataclass
+class BeAppSpec:
+    name: str
+    kernels: list
+    buffers: list = field(default_factory=list)
+
+
+def stencil_app(nx=512, ny=512, nz=64, seed=2022) -> BeAppSpec:
+    """Parboil stencil: ping-pong sweeps between two buffers (one kernel = one sweep)."""
+    A = synth.stencil_inputs(nx, ny, nz, seed)
+    a0 = _dev(A)
+    a1 = a0.clone()
+    cells = nx * ny * nz
+    inner = (nx - 2) * (ny - 2) * (nz - 2)
+    ks = [BeKernelSpec("stencil.even", tk.be_stencil(a0, a1), flops=8 * inner, bytes=8 * cells),
+          BeKernelSpec("stencil.odd", tk.be_stencil(a1, a0), flops=8 * inner, bytes=8 * cells)]
+    return BeAppSpec(f"stencil_{nx}x{ny}x{nz}", ks, [a0, a1])
+
+
+def mriq_app(N=64, numK=2048, chunk=1024, seed=2022) -> BeAppSpec:
+    """Parboil mri-q: ComputePhiMag then ComputeQ per k chunk (accumulating into Qr/Qi)."""
+    d = synth.mriq_inputs(N, numK, seed)
+    dd = {k: _dev(v) for k, v in d.items()}
+    phimag = torch.empty(numK, device="cuda")
+    Qr = torch.zeros(N ** 3, device="cuda")
+    Qi = torch.zeros(N ** 3, device="cuda")
+    ks = [BeKernelSpec("mriq.phimag", tk.be_mriq_phimag(dd["phiR"], dd["phiI"], phimag), flops=3 * numK,
+                       bytes=12 * numK)]
+    nx = N ** 3
+    for c0 in range(0, numK, chunk):
+        kn = min(chunk, numK - c0)
+        desc = tk.be_mriq_q(dd["x"], dd["y"], dd["z"], dd["kx"][c0:c0 + kn], dd["ky"][c0:c0 + kn],
+                            dd["kz"][c0:c0 + kn], phimag[c0:c0 + kn], Qr, Qi)
+        ks.append(BeKernelSpec(f"mriq.q{c0 // chunk}", desc, flops=10.0 * nx * kn, mufu=2.0 * nx * kn,
+                               bytes=20.0 * nx + 16.0 * kn, bound="mufu"))
+    return BeAppSpec(f"mriq_{N}^3x{numK}", ks, [dd, phimag, Qr, Qi])
+
+
+def sgemm_app(M=2048, N=2048, K=2048, seed=2022) -> BeAppSpec:
+    A, B = synth.sgemm_inputs(M, N, K, seed)
+    dA, dB = _dev(A), _dev(B)
+    Cm = torch.empty(M, N, device="cuda")
+    return BeAppSpec(f"sgemm_{M}x{N}x{K}", [BeKernelSpec("sgemm", tk.be_sgemm(dA, dB, Cm), flops=2.0 * M * N * K,
+                                                          bytes=4.0 * (M * K + K * N + M * N), bound="fma")],
+                     [dA, dB, Cm])

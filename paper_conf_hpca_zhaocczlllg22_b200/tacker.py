@@ -26,7 +26,7 @@ LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
 EPI_BIAS, EPI_RELU, EPI_RESIDUAL = 1, 2, 4
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
- BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN) = range(12)
+ BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL) = range(13)
 POLICY_TACKER, POLICY_BAYMAX = 0, 1
 DEC_FUSED, DEC_ORIGINAL_LC, DEC_REORDER_BE, DEC_IDLE_BE, DEC_NOTHING = range(5)
 MAX_APPS = 64
@@ -111,11 +111,17 @@ class BeFmaBurn(C.Structure):
                 ("out", C.c_void_p)]
 
 
+class BeIm2col(C.Structure):
+    _fields_ = [("n", C.c_int32), ("h", C.c_int32), ("w", C.c_int32), ("c", C.c_int32), ("r", C.c_int32),
+                ("s", C.c_int32), ("stride", C.c_int32), ("pad", C.c_int32), ("Kpad", C.c_int32),
+                ("x", C.c_void_p), ("out", C.c_void_p)]
+
+
 class _BeUnion(C.Union):
     _fields_ = [("sgemm", BeSgemm), ("stencil", BeStencil), ("mriq_phimag", BeMriqPhimag), ("mriq_q", BeMriqQ),
                 ("cutcp", BeCutcp), ("lbm", BeLbm), ("spmv", BeSpmv), ("histo", BeHisto),
                 ("bfs_expand", BeBfsExpand), ("bfs_commit", BeBfsCommit), ("fma_burn", BeFmaBurn),
-                ("_pad", C.c_uint8 * 128)]
+                ("im2col", BeIm2col), ("_pad", C.c_uint8 * 128)]
 
 
 class BeDesc(C.Structure):
@@ -319,6 +325,13 @@ def be_bfs_commit(mask, visited, upd, over, orig_blocks=0) -> BeDesc:
 def be_fma_burn(out, iters, n_threads=None, a=0.5, b=0.125, orig_blocks=0) -> BeDesc:
     d = BeDesc(kind=BE_FMA_BURN, orig_blocks=orig_blocks)
     d.p.fma_burn = BeFmaBurn(out.numel() if n_threads is None else n_threads, iters, a, b, _ptr(out))
+    return d
+
+
+def be_im2col(x, out, r, s, stride, pad, Kpad=None, orig_blocks=0) -> BeDesc:
+    n, h, w, c = x.shape
+    d = BeDesc(kind=BE_IM2COL, orig_blocks=orig_blocks)
+    d.p.im2col = BeIm2col(n, h, w, c, r, s, stride, pad, out.shape[1] if Kpad is None else Kpad, _ptr(x), _ptr(out))
     return d
 
 

@@ -1,0 +1,212 @@
+"""CPU tests of the C ABI boundary (no GPU): the library loads and exports every symbol the
+header declares, ctypes struct layouts equal the C compiler's, host-only calls (predictor,
+simulated manager) agree with the oracle, and GPU-needing calls fail loudly without a GPU."""
+import ctypes as C
+import math
+import os
+import re
+import subprocess
+import tempfile
+
+import numpy as np
+import pytest
+
+from oracle import manager_ref as mr, predictor as op
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HDR = os.path.join(ROOT, "include", "tacker.h")
+
+
+@pytest.fixture(scope="module")
+def tk():
+    from paper_conf_hpca_zhaocczlllg22_b200 import build, tacker
+    build.build()
+    return tacker
+
+
+def header_functions():
+    src = open(HDR).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(tacker_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol(tk):
+    lib = C.CDLL(tk.LIB_PATH)
+    funcs = header_functions()
+    assert len(funcs) >= 30
+    for f in funcs:
+        assert hasattr(lib, f), f"{f} declared in tacker.h but not exported"
+    assert set(funcs) == set(tk.EXPORTED)
+
+
+STRUCTS = {
+    "tacker_lc_desc": "LcDesc", "tacker_be_desc": "BeDesc", "tacker_be_sgemm": "BeSgemm",
+    "tacker_be_stencil": "BeStencil", "tacker_be_mriq_q": "BeMriqQ", "tacker_be_cutcp": "BeCutcp",
+    "tacker_be_lbm": "BeLbm", "tacker_be_spmv": "BeSpmv", "tacker_be_histo": "BeHisto",
+    "tacker_be_bfs_expand": "BeBfsExpand", "tacker_be_bfs_commit": "BeBfsCommit",
+    "tacker_be_fma_burn": "BeFmaBurn", "tacker_be_im2col": "BeIm2col", "tacker_fused_info_t": "FusedInfo",
+    "tacker_lc_kernel": "LcKernel", "tacker_be_kernel": "BeKernel", "tacker_decision": "Decision",
+    "tacker_manager_params": "ManagerParams", "tacker_manager_stats": "ManagerStats", "tacker_ratio": "Ratio",
+}
+
+
+def test_struct_layouts_match_c(tk):
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "tacker.h"', "int main(void){"]
+    for cs, py in STRUCTS.items():
+        lines.append(f'printf("{py} %zu\\n", sizeof({cs}));')
+    lines.append('printf("be.p %zu\\n", offsetof(tacker_be_desc, p));')
+    lines.append('printf("lc.A %zu\\n", offsetof(tacker_lc_desc, A));')
+    lines.append('printf("lk.cd %zu\\n", offsetof(tacker_lc_kernel, cd));')
+    lines.append("return 0;}")
+    with tempfile.TemporaryDirectory() as d:
+        src = os.path.join(d, "l.c")
+        exe = os.path.join(d, "l")
+        open(src, "w").write("\n".join(lines))
+        subprocess.check_call(["gcc", "-I", os.path.dirname(HDR), src, "-o", exe])
+        out = subprocess.check_output([exe], text=True).split("\n")
+    got = dict(l.split() for l in out if l.strip())
+    for cs, py in STRUCTS.items():
+        assert int(got[py]) == C.sizeof(getattr(tk, py)), (cs, got[py], C.sizeof(getattr(tk, py)))
+    assert int(got["be.p"]) == tk.BeDesc.p.offset
+    assert int(got["lc.A"]) == tk.LcDesc.A.offset
+    assert int(got["lk.cd"]) == tk.LcKernel.cd.offset
+
+
+def test_errors_without_gpu(tk):
+    assert tk.tacker_device_sm_count() == 0 or tk.tacker_device_sm_count() >= 100
+    with pytest.raises(tk.TackerError) as e:
+        tk.tacker_fuse(tk.LcDesc(), None, 0)
+    assert e.value.status in (tk.EINVAL, tk.EUNSUPPORTED, tk.ECUDA)
+    # BE block counts are pure host arithmetic (PTB "original_block_num", Fig. 7)
+    d = tk.BeDesc(kind=tk.BE_SGEMM)
+    d.p.sgemm = tk.BeSgemm(256, 256, 256, 1.0, 0.0, 1, 1, 1)
+    assert tk.tacker_be_num_blocks(d) == 16
+    lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=300, N=136, K=200, A=1, B=1, D=1)
+    assert tk.tacker_lc_num_tiles(lc, 64) == 3 * 3
+    assert tk.tacker_lc_num_tiles(lc, 128) == 3 * 2
+    bad = tk.LcDesc(kind=tk.LC_GEMM_F16, M=16, N=12, K=16, A=1, B=1, D=1)
+    with pytest.raises(tk.TackerError) as e:
+        tk.tacker_lc_num_tiles(bad, 64)
+    assert e.value.status == tk.EUNSUPPORTED   # N % 8 != 0
+
+
+# ------------------------------------------------------------------ predictor: C vs oracle
+def test_kernel_lr_c_matches_oracle(tk):
+    tk.tacker_model_clear()
+    rng = np.random.default_rng(5)
+    m = op.KernelLR()
+    for blocks in (16, 48, 100, 333, 512, 1024):
+        ms = 0.0031 * blocks + 0.02 + rng.normal(0, 1e-3)
+        tk.tacker_model_add_sample("k1", blocks, ms)
+        m.add(blocks, ms)
+    a, b = tk.tacker_model_fit("k1")
+    ra, rb = m.fit()
+    assert abs(a - ra) < 1e-12 and abs(b - rb) < 1e-12
+    assert abs(tk.tacker_model_predict("k1", 700) - m.predict(700)) < 1e-12
+
+
+def test_two_stage_c_matches_oracle_and_refits(tk):
+    tk.tacker_model_clear()
+    m = op.TwoStage()
+    rng = np.random.default_rng(6)
+    for r in (0.1, 0.2, 1.8, 1.9, 0.05, 2.5):
+        xtc = rng.uniform(0.5, 3)
+        tau = max(1 + 0.3 * r, 0.55 + 1.0 * r) * (1 + rng.normal(0, 0.01))
+        tk.tacker_pair_add_sample("p", xtc, r * xtc, tau * xtc)
+        m.add(xtc, r * xtc, tau * xtc)
+    c = tk.tacker_pair_fit("p")
+    (a1, b1), (a2, b2) = m.fit()
+    assert np.allclose(c, (a1, b1, a2, b2), rtol=0, atol=1e-12)
+    for r in (0.0, 0.3, 0.7, 1.2, 3.0):
+        assert abs(tk.tacker_pair_predict("p", 2.0, 2.0 * r) - m.predict(2.0, 2.0 * r)) < 1e-12
+    assert tk.tacker_pair_observe("p", 1.0, 0.5, m.predict(1.0, 0.5) * 1.3) == m.observe(1.0, 0.5, m.predict(1.0, 0.5) * 1.3)
+    assert abs(tk.tacker_pair_predict("p", 1.0, 1.0) - m.predict(1.0, 1.0)) < 1e-12
+
+
+def test_model_save_load_roundtrip(tk, tmp_path):
+    tk.tacker_model_clear()
+    for x in (1, 2, 3):
+        tk.tacker_model_add_sample("a", x, 2 * x + 1)
+    tk.tacker_model_fit("a")
+    for r in (0.1, 0.2, 1.8, 1.9):
+        tk.tacker_pair_add_sample("b", 1.0, r, max(1 + 0.1 * r, r))
+    tk.tacker_pair_fit("b")
+    p = str(tmp_path / "models.txt")
+    tk.tacker_model_save(p)
+    before = (tk.tacker_model_predict("a", 10), tk.tacker_pair_predict("b", 1.0, 0.7))
+    tk.tacker_model_clear()
+    with pytest.raises(tk.TackerError):
+        tk.tacker_model_predict("a", 10)
+    tk.tacker_model_load(p)
+    assert (tk.tacker_model_predict("a", 10), tk.tacker_pair_predict("b", 1.0, 0.7)) == before
+
+
+# ------------------------------------------------------------------ manager: C (simulated) vs oracle
+FAKE = 0x10000
+
+
+def lc_kernel(tk, is_tc, t):
+    k = tk.LcKernel(is_tc=1 if is_tc else 0, t_pred_ms=t)
+    if is_tc:
+        k.lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=1024, N=1024, K=1024, A=FAKE, B=FAKE, D=FAKE)
+    else:
+        k.cd.kind = tk.BE_FMA_BURN
+        k.cd.p.fma_burn = tk.BeFmaBurn(128, 10, 0.5, 0.125, FAKE)
+    return k
+
+
+def be_kernel(tk, t, ws=16):
+    b = tk.BeKernel(is_cd=1, t_pred_ms=t, warp_split=ws)
+    b.be.kind = tk.BE_STENCIL
+    b.be.p.stencil = tk.BeStencil(64, 64, 8, 1 / 6, 1 / 36, FAKE, FAKE)
+    return b
+
+
+def fit_pair_closed_form(tk, tau):
+    # the pair key of (gemm 1024^3, stencil nz=8, ws16), fitted exactly to tau(r) = max(l1, l2)
+    key = "pair:lc:gemm:N1024:K1024:bn128:f32|be:stencil:nz8|ws16"
+    for r in (0.1, 0.2, 1.8, 1.9):
+        tk.tacker_pair_add_sample(key, 1.0, r, tau(r))
+    tk.tacker_pair_fit(key)
+    return key
+
+
+@pytest.mark.parametrize("policy", ["tacker", "baymax"])
+def test_manager_simulation_matches_reference(tk, policy):
+    tk.tacker_model_clear()
+    # stage-2 slope != 1 so that Tgain depends on Tcd (with slope 1 every stage-2 pair has the
+    # same gain (1 - a2) * Ttc and ties would be decided by rounding noise)
+    tau = lambda r: max(1 + 0.25 * r, 0.4 + 0.93 * r)
+    fit_pair_closed_form(tk, tau)
+    fuse_pred = lambda ttc, tcd: ttc * tau(tcd / ttc)
+    rng = np.random.default_rng(11)
+    arrivals = np.cumsum(rng.exponential(6.0, 60))
+    shapes = [[(True, 1.21), (False, 0.3), (True, 0.83), (True, 1.97)], [(True, 0.52), (True, 0.49)]]
+    app_ts = [[1.53, 0.71], [3.07], [0.43, 0.37, 2.51]]
+    pol = tk.POLICY_TACKER if policy == "tacker" else tk.POLICY_BAYMAX
+    m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0)
+    qs = []
+    for i, t in enumerate(arrivals):
+        sh = shapes[i % 2]
+        m.submit_lc([lc_kernel(tk, tc, d) for tc, d in sh], float(t))
+        qs.append(mr.Query(i, float(t), list(sh)))
+    apps = []
+    for ts in app_ts:
+        m.submit_be([be_kernel(tk, d) for d in ts])
+        apps.append(mr.App([(True, d) for d in ts]))
+    ref = mr.simulate(qs, apps, 50.0, mr.TACKER if policy == "tacker" else mr.BAYMAX, fuse_pred, idle_cap=2.0)
+    got = []
+    for _ in range(100000):
+        st = m.stats()
+        if st.lc_queries_done == len(arrivals):
+            break
+        d = m.step(50.0)
+        if d.action in (tk.DEC_FUSED, tk.DEC_ORIGINAL_LC, tk.DEC_REORDER_BE, tk.DEC_IDLE_BE):
+            got.append((d.action, d.fused_app, tuple(d.reorder_apps[:d.n_reorder])))
+    exp = [(x.action, x.fused_app, tuple(x.reorder)) for x in ref["decisions"]]
+    assert got == exp
+    for i in range(len(arrivals)):
+        assert abs(m.latency(i) - ref["latency"][i]) < 1e-9
+    assert max(ref["latency"].values()) <= 50.0
+    if policy == "tacker":
+        assert m.stats().fused_launches > 0

@@ -140,3 +140,16 @@ def test_resnet50_table():
     # ~4.09 GMAC of convolutions per ResNet-50 forward at 224x224 (conv1 with its real C=3)
     assert 8.1 < gflop < 8.25
     assert len(synth.vgg16_convs(1)) == 13
+
+
+def test_im2col_times_filter_is_conv():
+    cs = synth.ConvShape("t", 1, 11, 11, 8, 6, 7, 7, 2, 3)
+    x, w, _ = synth.conv_inputs(cs, seed=8, variant="int")
+    cols = lc.im2col(x, 7, 7, 2, 3, 400)
+    assert cols.shape == (cs.p * cs.q, 400) and np.all(cols[:, 392:] == 0)
+    wf = np.zeros((6, 400), np.float16)
+    wf[:, :392] = w.reshape(6, -1)
+    D, _ = lc.lc_gemm(cols, wf)
+    assert np.array_equal(D.reshape(1, cs.p, cs.q, 6), brute_conv(x, w, 2, 3))
+    # corner element: padding rows/cols of the window are zero
+    assert np.all(cols[0, :3 * 7 * 8] == 0)
