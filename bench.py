@@ -160,7 +160,14 @@ class Workload:
         for k in self.svc.kernels:
             if k.is_tc:
                 be = st_k[(ti // 2) % 2] if ti % 2 == 0 else mq_k[(ti // 2) % len(mq_k)]
-                f = tk.tacker_fuse(k.lc, be.desc, warp_split)
+                f = None
+                for ws in range(warp_split, 3, -4):   # LC-first budget: shrink the BE if it does not fit
+                    try:
+                        f = tk.tacker_fuse(k.lc, be.desc, ws)
+                        break
+                    except tk.TackerError as e:
+                        if e.status != tk.ERESOURCE:
+                            raise
                 self.plan.append((k, be, f))
                 ti += 1
             else:

@@ -50,6 +50,7 @@ struct BeWork {
 struct alignas(64) FusedParams {
   CUtensorMap tmap_a;      // A / x operand
   CUtensorMap tmap_b;      // B / w operand
+  CUtensorMap tmap_be;     // BE input tensor map (stencil), unused otherwise
   LcParams lc;
   tacker_be_desc be;
   int64_t be_blocks;       // original blocks to run (PTB original_block_num)
@@ -237,15 +238,16 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   const int tid = threadIdx.x - kVbThreads * j;     // thread_step rebase (Fig. 5)
   const uint32_t bar = 1 + j;                       // named barrier id (0 is reserved)
   uint8_t *slice = be_smem + (size_t)j * P.be_smem_per_vb;
-  volatile uint32_t *s_ticket = reinterpret_cast<volatile uint32_t *>(slice);
-  uint8_t *body_smem = slice + 16;
-  const auto &bp = BeSel<BE_KIND>::get(P.be);
+  // body scratch first (128-byte aligned: TMA destinations), the ticket slot in the last 16 B
+  uint8_t *body_smem = slice;
+  volatile uint32_t *s_ticket = reinterpret_cast<volatile uint32_t *>(slice + P.be_smem_per_vb - 16);
   const uint32_t groups = gridDim.x * (uint32_t)P.be_vb_per_cta;
   // First round static and interleaved across CTAs (slot j of every CTA before slot j+1, so
   // a short BE kernel spreads over all SMs); afterwards dynamic tickets balance the tail.
   int64_t vb = (int64_t)j * gridDim.x + blockIdx.x;
+  be_init<BE_KIND>(body_smem, tid, bar);
   while (vb < P.be_blocks) {
-    BeBody<BE_KIND>::run(bp, vb, tid, bar, body_smem);
+    be_run<BE_KIND>(P.be, vb, tid, bar, body_smem, &P.tmap_be);
     if (tid == 0) *s_ticket = groups + atomicAdd(&P.work->ticket, 1u);
     named_bar_sync(bar, kVbThreads);
     vb = *s_ticket;
@@ -321,10 +323,16 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
 
 // ------------------------------------------------------------------------ BE original kernel
 // The non-persistent "CD_kernel" of Fig. 7: one CTA of 128 threads per original block.
+struct alignas(64) BeOrigParams {
+  CUtensorMap tmap;        // BE input tensor map (stencil), unused otherwise
+  tacker_be_desc d;
+};
+
 template <int BE_KIND>
-__global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ tacker_be_desc D) {
+__global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ BeOrigParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  BeBody<BE_KIND>::run(BeSel<BE_KIND>::get(D), (int64_t)blockIdx.x, threadIdx.x, 1u, smem_raw);
+  be_init<BE_KIND>(smem_raw, threadIdx.x, 1u);
+  be_run<BE_KIND>(P.d, (int64_t)blockIdx.x, threadIdx.x, 1u, smem_raw, &P.tmap);
 }
 
 }  // namespace tk

@@ -264,6 +264,26 @@ static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, cons
   return TACKER_OK;
 }
 
+// BE tensor maps: the stencil stages plane tiles with one 3-D TMA box each
+// ({TX+8, TY+2, 1} fp32, halo out of the grid zero-filled).  Other kinds need none.
+static tacker_status encode_be_tmap(const tacker_be_desc &d, CUtensorMap *m) {
+  memset(m, 0, sizeof *m);
+  if (d.kind != TACKER_BE_STENCIL || (d.p.stencil.nx & 3)) return TACKER_OK;
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  using SB = BeBody<TACKER_BE_STENCIL>;
+  const auto &p = d.p.stencil;
+  cuuint64_t dims[3] = {(cuuint64_t)p.nx, (cuuint64_t)p.ny, (cuuint64_t)p.nz};
+  cuuint64_t strides[2] = {(cuuint64_t)p.nx * 4, (cuuint64_t)p.nx * p.ny * 4};
+  cuuint32_t box[3] = {(cuuint32_t)SB::ROWF, (cuuint32_t)(SB::TY + 2), 1};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float *>(p.A0), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(stencil) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
 // ============================================================================ kernel table
 using KernelFn = void (*)(FusedParams);
 
@@ -285,7 +305,7 @@ static KernelFn pick_fused(int BN, int be_kind) {
   return nullptr;
 }
 
-using BeFn = void (*)(tacker_be_desc);
+using BeFn = void (*)(BeOrigParams);
 static BeFn pick_be_original(int kind) {
   switch (kind) {
 #define C(K) \
@@ -420,6 +440,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     if ((st = encode_2d(&F.P.tmap_a, lc->A, (uint64_t)L.K, (uint64_t)L.M, kBK, kBM))) return st;
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   }
+  if (has_be && (st = encode_be_tmap(*be, &F.P.tmap_be))) return st;
   // registers: the whole CTA must fit the 64K register file
   cudaFuncAttributes fa{};
   cudaError_t e = cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(F.fn));
@@ -568,8 +589,10 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
     BeFn fn = pick_be_original(be->kind);
     const int smem = (int)be_smem_bytes(be->kind);
     if (smem > 48 * 1024 && (st = set_smem_attr(reinterpret_cast<const void *>(fn), smem))) return st;
-    tacker_be_desc d = *be;
-    void *args[] = {&d};
+    BeOrigParams op;
+    op.d = *be;
+    if ((st = encode_be_tmap(*be, &op.tmap))) return st;
+    void *args[] = {&op};
     if (blocks > 0x7fffffffLL) return set_error("too many blocks"), TACKER_EUNSUPPORTED;
     cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(fn), dim3((unsigned)blocks), dim3(128), args, smem, s);
     if (e != cudaSuccess) return cuda_fail("launch be_original_kernel", e);

@@ -369,7 +369,8 @@ class Fused:
 
     def __del__(self):
         if getattr(self, "h", None):
-            _lib.tacker_fused_destroy(self.h)
+            if _lib is not None:   # None during interpreter shutdown
+                _lib.tacker_fused_destroy(self.h)
             self.h = None
 
     def info(self) -> FusedInfo:
@@ -478,7 +479,8 @@ class Manager:
 
     def __del__(self):
         if getattr(self, "h", None):
-            _lib.tacker_manager_destroy(self.h)
+            if _lib is not None:
+                _lib.tacker_manager_destroy(self.h)
             self.h = None
 
     def submit_lc(self, kernels, arrival_ms) -> int:

@@ -178,3 +178,20 @@ def test_ptb_orig_blocks_prefix(tk):
     ref = obe.fma_burn(n, iters)
     assert max_rel_err(o[:1280], ref[:1280]) <= 1e-5
     assert np.all(o[1280:] == 0)
+
+
+@pytest.mark.parametrize("ws", [4, 20])
+def test_stencil_scalar_path_and_large(tk, ws):
+    # nx % 4 != 0 (scalar path) and the full bench grid (TMA path, 2048 blocks), fused vs original
+    for size in ("scalar", "large"):
+        c = be_case(tk.BE_STENCIL, seed=5, size=size)
+        c["reset"]()
+        tk.tacker_launch_original(None, c["desc"])
+        orig = host(c["outs"][0]).copy()
+        c["check"]([orig])
+        A, B = synth.lc_gemm_inputs(256, 128, 64, seed=0)
+        D = torch.zeros(256, 128, device=dev())
+        f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], ws)
+        c["reset"]()
+        f.launch()
+        assert host(c["outs"][0]).tobytes() == orig.tobytes()
