@@ -18,9 +18,6 @@
 namespace tk {
 
 constexpr int kVbThreads = 128;
-#ifndef TK_MRIQ_VPT
-#define TK_MRIQ_VPT 1
-#endif
 
 template <int KIND> struct BeBody;
 
@@ -150,23 +147,18 @@ template <> struct BeBody<TACKER_BE_FMA_BURN> {
 };
 
 // ---------------------------------------------------------------- stencil (Parboil)
-// One 7-point Jacobi sweep over A0[nz][ny][nx] (x fastest), HBM-bound.
-//   interior: An = c1*(((((W+E)+S)+N)+B)+T) - c0*A   (W/E = x-1/x+1, S/N = y-1/y+1, B/T = z-1/z+1)
+// One 7-point Jacobi sweep over A0[nz][ny][nx] (x fastest), HBM-bound.  Block = 128 x 4 x 4
+// (x,y,z) cells: lane l of warp w owns x = 4l..4l+3 (one float4) of row y = w for ZC = 4 planes.
+// The centre column's ZC+2 planes are loaded up front (memory-level parallelism), x+-1 comes
+// from the neighbouring lanes' float4 by shuffle, y+-1 rows through L1/L2.
+//   interior: An = c1*(((((W+E)+S)+N)+B)+T) - c0*A   (S/N = y-1/y+1, B/T = z-1/z+1)
 //   boundary cells (x, y or z on the faces) are copied.
-// Block = TX x TY x ZR = 128 x 8 x 8 cells, 2.5-D blocked: the block marches through its z range
-// with a ring of NS plane tiles ((TY+2) rows x (TX+8) floats) in shared memory, each tile one
-// 3-D TMA box (cp.async.bulk.tensor, completion on an mbarrier, halo zero-filled out of the
-// grid), so the bytes in flight sit in shared memory instead of registers.  Lane l of warp w
-// computes x = 4l..4l+3 (float4) of rows 2w, 2w+1; x+-1 comes from the neighbouring lanes by
-// shuffle.  nx % 4 != 0 uses a scalar path over the same tile with the same arithmetic.
+// nx % 4 != 0 uses the scalar path with the same per-element arithmetic.
 template <> struct BeBody<TACKER_BE_STENCIL> {
-  static constexpr int TX = 128, TY = 8, ZR = 8, NS = 5;
-  static constexpr int ROWF = TX + 8;                          // x0-4 .. x0+TX+3
-  static constexpr uint32_t kBoxBytes = (TY + 2) * ROWF * 4;   // one TMA box {ROWF, TY+2, 1}
-  static constexpr uint32_t kPlaneBytes = (kBoxBytes + 127) & ~127u;
-  static constexpr uint32_t kSmem = NS * kPlaneBytes + NS * 8 + 16;
+  static constexpr uint32_t kSmem = 0;
+  static constexpr int ZC = 4;
   static __host__ __device__ int64_t num_blocks(const tacker_be_stencil &p) {
-    return (int64_t)((p.nx + TX - 1) / TX) * ((p.ny + TY - 1) / TY) * ((p.nz + ZR - 1) / ZR);
+    return (int64_t)((p.nx + 127) / 128) * ((p.ny + 3) / 4) * ((p.nz + ZC - 1) / ZC);
   }
   static __device__ __forceinline__ float point(const tacker_be_stencil &p, float w, float e, float s, float n,
                                                 float b, float t, float c) {
@@ -177,99 +169,67 @@ template <> struct BeBody<TACKER_BE_STENCIL> {
     sum = __fadd_rn(sum, t);
     return __fsub_rn(__fmul_rn(p.c1, sum), __fmul_rn(p.c0, c));
   }
-  static __device__ __forceinline__ void run(const tacker_be_stencil &p, int64_t vb, int tid, uint32_t bar,
-                                             uint8_t *smem, const CUtensorMap *tm) {
-    const int bxn = (p.nx + TX - 1) / TX, byn = (p.ny + TY - 1) / TY;
-    const int zb = (int)(vb / ((int64_t)bxn * byn));
-    const int rem = (int)(vb % ((int64_t)bxn * byn));
-    const int x0 = (rem % bxn) * TX, y0 = (rem / bxn) * TY, z0 = zb * ZR;
-    const int z1 = min(z0 + ZR, p.nz);
+  static __device__ __forceinline__ void run(const tacker_be_stencil &p, int64_t vb, int tid, uint32_t,
+                                             uint8_t *) {
+    const int bx = (p.nx + 127) / 128, by = (p.ny + 3) / 4;
+    const int zb = (int)(vb / ((int64_t)bx * by));
+    const int rem = (int)(vb % ((int64_t)bx * by));
+    const int lane = tid & 31;
+    const int x0 = (rem % bx) * 128 + 4 * lane;
+    const int y = (rem / bx) * 4 + (tid >> 5);
+    const int z0 = zb * ZC;
+    if (y >= p.ny) return;                     // warp-uniform
     const size_t plane = (size_t)p.nx * p.ny;
     const float *__restrict__ A = p.A0;
     float *__restrict__ An = p.Anext;
-    const int lane = tid & 31, w = tid >> 5;
-    if (p.nx & 3) {   // scalar path
-      for (int r = 0; r < 2; ++r) {
-        const int y = y0 + 2 * w + r;
-        if (y >= p.ny) break;
-        for (int x = x0 + lane; x < min(x0 + TX, p.nx); x += 32)
-          for (int z = z0; z < z1; ++z) {
-            const size_t o = z * plane + (size_t)y * p.nx + x;
-            const bool bord = (y == 0) | (y == p.ny - 1) | (x == 0) | (x == p.nx - 1) | (z == 0) | (z == p.nz - 1);
-            An[o] = bord ? A[o]
-                         : point(p, A[o - 1], A[o + 1], A[o - p.nx], A[o + p.nx], A[o - plane], A[o + plane], A[o]);
-          }
+    const bool ybord = (y == 0) | (y == p.ny - 1);
+    if ((p.nx & 3) == 0) {
+      const bool act = x0 < p.nx;
+      const size_t row = (size_t)y * p.nx + x0;
+      float4 c[ZC + 2];
+#pragma unroll
+      for (int i = 0; i < ZC + 2; ++i) {
+        const int z = z0 - 1 + i;
+        c[i] = (act && z >= 0 && z < p.nz) ? __ldg(reinterpret_cast<const float4 *>(A + z * plane + row))
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+#pragma unroll
+      for (int i = 0; i < ZC; ++i) {
+        const int z = z0 + i;
+        if (z >= p.nz) break;                  // warp-uniform
+        const float4 cc = c[i + 1];
+        float wv = __shfl_up_sync(0xffffffffu, cc.w, 1);
+        float ev = __shfl_down_sync(0xffffffffu, cc.x, 1);
+        if (!act) continue;
+        float4 o = cc;
+        const bool zb_ = (z == 0) | (z == p.nz - 1);
+        if (!ybord && !zb_) {
+          if (lane == 0) wv = x0 > 0 ? __ldg(A + z * plane + row - 1) : 0.f;
+          if (lane == 31 || x0 + 4 >= p.nx) ev = x0 + 4 < p.nx ? __ldg(A + z * plane + row + 4) : 0.f;
+          const float4 s = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row - p.nx));
+          const float4 n = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row + p.nx));
+          const float4 b = c[i], t = c[i + 2];
+          if (x0 > 0) o.x = point(p, wv, cc.y, s.x, n.x, b.x, t.x, cc.x);
+          o.y = point(p, cc.x, cc.z, s.y, n.y, b.y, t.y, cc.y);
+          o.z = point(p, cc.y, cc.w, s.z, n.z, b.z, t.z, cc.z);
+          if (x0 + 3 < p.nx - 1) o.w = point(p, cc.z, ev, s.w, n.w, b.w, t.w, cc.w);
+        }
+        *reinterpret_cast<float4 *>(An + z * plane + row) = o;
       }
       return;
     }
-    float *tiles = reinterpret_cast<float *>(smem);
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + NS * kPlaneBytes);
-    volatile uint32_t *seq = reinterpret_cast<volatile uint32_t *>(bars + NS);
-    const int zlo = max(z0 - 1, 0), zhi = min(z1, p.nz - 1);
-    const int np = zhi - zlo + 1;
-    // The ring and its mbarriers persist across the blocks a virtual-block slot runs (init()
-    // once per slot); plane i of this block is the (base+i)-th plane through the ring.
-    named_bar_sync(bar, kVbThreads);   // the previous block is done with the ring and seq
-    const uint32_t base = *seq;
-    auto slot = [&](int i) { return (base + (uint32_t)i) % NS; };
-    auto parity = [&](int i) { return ((base + (uint32_t)i) / NS) & 1u; };
-    auto tile = [&](int i) { return tiles + (size_t)slot(i) * (kPlaneBytes / 4); };
-    // one 3-D TMA box per plane: x0-4 .. x0+TX+3, y0-1 .. y0+TY, out-of-grid elements zero-filled
-    auto issue = [&](int i) {
-      uint64_t *b = &bars[slot(i)];
-      mbar_arrive_expect_tx(b, kBoxBytes);
-      tma_load_3d(tm, b, tile(i), x0 - 4, y0 - 1, zlo + i);
-    };
-    if (tid == 0)
-      for (int i = 0; i < min(NS, np); ++i) issue(i);
-    const int xl = 4 + 4 * lane;   // this lane's float4 within a staged row
-    const int xg = x0 + 4 * lane;
-    const bool act = xg < p.nx;
-    for (int z = z0; z < z1; ++z) {
-      const int i = z - zlo;
-      const bool zint = (z > 0) & (z < p.nz - 1);
-      if (zint) mbar_wait(&bars[slot(i - 1)], parity(i - 1));
-      mbar_wait(&bars[slot(i)], parity(i));
-      if (zint) mbar_wait(&bars[slot(i + 1)], parity(i + 1));
-      const float *tc = tile(i);
-#pragma unroll
-      for (int r = 0; r < 2; ++r) {
-        const int yr = 2 * w + r, y = y0 + yr;
-        if (y >= p.ny) break;                       // warp-uniform
-        const float *row = tc + (yr + 1) * ROWF;
-        const float4 c = *reinterpret_cast<const float4 *>(row + xl);
-        float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
-        float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
-        if (lane == 0) wv = row[3];
-        if (lane == 31) ev = row[xl + 4];
-        if (!act) continue;
-        float4 o = c;
-        if (zint && y > 0 && y < p.ny - 1) {
-          const float4 s = *reinterpret_cast<const float4 *>(row - ROWF + xl);
-          const float4 n = *reinterpret_cast<const float4 *>(row + ROWF + xl);
-          const float4 b = *reinterpret_cast<const float4 *>(tile(i - 1) + (yr + 1) * ROWF + xl);
-          const float4 t = *reinterpret_cast<const float4 *>(tile(i + 1) + (yr + 1) * ROWF + xl);
-          if (xg > 0) o.x = point(p, wv, c.y, s.x, n.x, b.x, t.x, c.x);
-          if (xg + 1 < p.nx - 1) o.y = point(p, c.x, c.z, s.y, n.y, b.y, t.y, c.y);
-          if (xg + 2 < p.nx - 1) o.z = point(p, c.y, c.w, s.z, n.z, b.z, t.z, c.z);
-          if (xg + 3 < p.nx - 1) o.w = point(p, c.z, ev, s.w, n.w, b.w, t.w, c.w);
-        }
-        *reinterpret_cast<float4 *>(An + z * plane + (size_t)y * p.nx + xg) = o;
+    // scalar path (nx % 4 != 0)
+    for (int e = 0; e < 4; ++e) {
+      const int x = x0 + e;
+      if (x >= p.nx) break;
+      const size_t col = (size_t)y * p.nx + x;
+      for (int z = z0; z < min(z0 + ZC, p.nz); ++z) {
+        const size_t o = z * plane + col;
+        const bool bord = ybord | (x == 0) | (x == p.nx - 1) | (z == 0) | (z == p.nz - 1);
+        An[o] = bord ? A[o]
+                     : point(p, A[o - 1], A[o + 1], A[o - p.nx], A[o + p.nx], A[o - plane], A[o + plane], A[o]);
       }
-      named_bar_sync(bar, kVbThreads);               // plane i-1 is dead for every thread
-      if (tid == 0 && i >= 1 && i - 1 + NS < np) issue(i - 1 + NS);
     }
-    if (tid == 0) *seq = base + (uint32_t)np;      // read by the next block after its first bar.sync
-  }
-  // once per virtual-block slot, before its first block
-  static __device__ __forceinline__ void init(uint8_t *smem, int tid, uint32_t bar) {
-    if (tid == 0) {
-      uint64_t *bars = reinterpret_cast<uint64_t *>(smem + NS * kPlaneBytes);
-      for (int s = 0; s < NS; ++s) mbar_init(&bars[s], 1);
-      *reinterpret_cast<volatile uint32_t *>(bars + NS) = 0;
-      fence_barrier_init();
-    }
-    named_bar_sync(bar, kVbThreads);
   }
 };
 
@@ -296,20 +256,31 @@ template <> struct BeBody<TACKER_BE_MRIQ_PHIMAG> {
 // only runs the two MUFU ops) before the MUFU sin/cos of 2*pi*t.
 template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   static constexpr int KC = 512;
-  static constexpr int VPT = TK_MRIQ_VPT;   // voxels per thread
+  static constexpr int kCoarsen = 4;       // original blocks one fused virtual block runs at once
   static constexpr uint32_t kSmem = KC * 16;
-  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) {
-    return (p.numX + 128 * VPT - 1) / (128 * VPT);
-  }
+  static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) { return (p.numX + 127) / 128; }
+  // original block = 128 voxels, one per thread
   static __device__ __forceinline__ void run(const tacker_be_mriq_q &p, int64_t vb, int tid, uint32_t bar,
                                              uint8_t *smem) {
+    run_v<1>(p, vb, 1, tid, bar, smem);
+  }
+  // fused virtual block = up to kCoarsen consecutive original blocks, thread owns one voxel of
+  // each (more independent MUFU chains per thread where the fused CTA has few BE warps); each
+  // voxel's k-ordered accumulation is unchanged, so results stay bit-identical.
+  static __device__ __forceinline__ void run_coarse(const tacker_be_mriq_q &p, int64_t vb, int nb, int tid,
+                                                    uint32_t bar, uint8_t *smem) {
+    run_v<kCoarsen>(p, vb, nb, tid, bar, smem);
+  }
+  template <int VPT>
+  static __device__ __forceinline__ void run_v(const tacker_be_mriq_q &p, int64_t vb, int nb, int tid, uint32_t bar,
+                                               uint8_t *smem) {
     float4 *ks = reinterpret_cast<float4 *>(smem);
     const float kTwoPi = 6.2831853071795864769f;
     const float kMagic = 12582912.0f;   // 1.5 * 2^23: (t + M) - M == rint(t) for |t| < 2^22
     int64_t v[VPT];
     float xs[VPT], ys[VPT], zs[VPT], qr[VPT], qi[VPT];
 #pragma unroll
-    for (int h = 0; h < VPT; ++h) v[h] = vb * (128 * VPT) + h * 128 + tid;
+    for (int h = 0; h < VPT; ++h) v[h] = h < nb ? (vb + h) * 128 + tid : (int64_t)p.numX;
 #pragma unroll
     for (int h = 0; h < VPT; ++h) {
       const bool ok = v[h] < p.numX;
@@ -598,16 +569,23 @@ __host__ __device__ constexpr int be_max_warps(int kind) { return kind == TACKER
 template <int KIND>
 __device__ __forceinline__ void be_run(const tacker_be_desc &d, int64_t vb, int tid, uint32_t bar, uint8_t *smem,
                                        const CUtensorMap *tm) {
-  if constexpr (KIND == TACKER_BE_STENCIL)
-    BeBody<KIND>::run(BeSel<KIND>::get(d), vb, tid, bar, smem, tm);
-  else
-    BeBody<KIND>::run(BeSel<KIND>::get(d), vb, tid, bar, smem);
+  (void)tm;
+  BeBody<KIND>::run(BeSel<KIND>::get(d), vb, tid, bar, smem);
 }
-// One-time per-slot setup (persistent mbarriers of the stencil's plane ring).
+// Thread coarsening of the fused PTB loop: one ticket covers BeCoarsen original blocks.
+template <int KIND> struct BeCoarsen { static constexpr int value = 1; };
+template <> struct BeCoarsen<TACKER_BE_MRIQ_Q> { static constexpr int value = BeBody<TACKER_BE_MRIQ_Q>::kCoarsen; };
 template <int KIND>
-__device__ __forceinline__ void be_init(uint8_t *smem, int tid, uint32_t bar) {
-  if constexpr (KIND == TACKER_BE_STENCIL) BeBody<KIND>::init(smem, tid, bar);
+__device__ __forceinline__ void be_run_coarse(const tacker_be_desc &d, int64_t vb, int nb, int tid, uint32_t bar,
+                                              uint8_t *smem, const CUtensorMap *tm) {
+  if constexpr (BeCoarsen<KIND>::value > 1)
+    BeBody<KIND>::run_coarse(BeSel<KIND>::get(d), vb, nb, tid, bar, smem);
+  else
+    be_run<KIND>(d, vb, tid, bar, smem, tm);
 }
+// One-time per-slot setup hook (persistent shared-memory state of a body; none at present).
+template <int KIND>
+__device__ __forceinline__ void be_init(uint8_t *, int, uint32_t) {}
 
 // Every implemented BE kind (X-macro used by the host dispatch tables).
 #define TK_FOR_EACH_BE(X)                                                                       \

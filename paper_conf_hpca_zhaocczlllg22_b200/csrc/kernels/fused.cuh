@@ -244,10 +244,13 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   const uint32_t groups = gridDim.x * (uint32_t)P.be_vb_per_cta;
   // First round static and interleaved across CTAs (slot j of every CTA before slot j+1, so
   // a short BE kernel spreads over all SMs); afterwards dynamic tickets balance the tail.
+  constexpr int kC = BeCoarsen<BE_KIND>::value;    // original blocks per ticket
+  const int64_t units = (P.be_blocks + kC - 1) / kC;
   int64_t vb = (int64_t)j * gridDim.x + blockIdx.x;
   be_init<BE_KIND>(body_smem, tid, bar);
-  while (vb < P.be_blocks) {
-    be_run<BE_KIND>(P.be, vb, tid, bar, body_smem, &P.tmap_be);
+  while (vb < units) {
+    const int64_t b0 = vb * kC;
+    be_run_coarse<BE_KIND>(P.be, b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem, &P.tmap_be);
     if (tid == 0) *s_ticket = groups + atomicAdd(&P.work->ticket, 1u);
     named_bar_sync(bar, kVbThreads);
     vb = *s_ticket;

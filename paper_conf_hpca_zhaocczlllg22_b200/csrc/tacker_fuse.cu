@@ -264,23 +264,10 @@ static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, cons
   return TACKER_OK;
 }
 
-// BE tensor maps: the stencil stages plane tiles with one 3-D TMA box each
-// ({TX+8, TY+2, 1} fp32, halo out of the grid zero-filled).  Other kinds need none.
-static tacker_status encode_be_tmap(const tacker_be_desc &d, CUtensorMap *m) {
+// BE tensor-map hook: a body that stages its input with TMA gets its tensor map encoded here
+// (the stencil's TMA plane-ring variant used it; the current bodies load through L1/L2).
+static tacker_status encode_be_tmap(const tacker_be_desc &, CUtensorMap *m) {
   memset(m, 0, sizeof *m);
-  if (d.kind != TACKER_BE_STENCIL || (d.p.stencil.nx & 3)) return TACKER_OK;
-  auto enc = get_encode();
-  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
-  using SB = BeBody<TACKER_BE_STENCIL>;
-  const auto &p = d.p.stencil;
-  cuuint64_t dims[3] = {(cuuint64_t)p.nx, (cuuint64_t)p.ny, (cuuint64_t)p.nz};
-  cuuint64_t strides[2] = {(cuuint64_t)p.nx * 4, (cuuint64_t)p.nx * p.ny * 4};
-  cuuint32_t box[3] = {(cuuint32_t)SB::ROWF, (cuuint32_t)(SB::TY + 2), 1};
-  cuuint32_t es[3] = {1, 1, 1};
-  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float *>(p.A0), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(stencil) failed: %d", (int)r), TACKER_ECUDA;
   return TACKER_OK;
 }
 
