@@ -104,22 +104,41 @@ typedef enum {
   TACKER_BE_FMA_BURN = 11,    /* register-only FMA chains (Kc, §III-B); block = 128 thr.   */
   TACKER_BE_IM2COL = 12,      /* LC CUDA-core helper: explicit im2col (cudnnIm2col, §VIII-H
                                  P:3350-3381) NHWC fp16 -> [M, Kpad] fp16; block = 1024x8 el. */
-  TACKER_BE_KIND_COUNT = 13
+  TACKER_BE_CUTCP_BIN = 13,   /* cutcp atom binning (deterministic, index order); block = 128 bins */
+  TACKER_BE_KIND_COUNT = 14
 } tacker_be_kind;
 
 typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
 typedef struct { int32_t nx, ny, nz; float c0, c1; const float *A0; float *Anext; } tacker_be_stencil;
 typedef struct { int32_t numK; const float *phiR, *phiI; float *phiMag; } tacker_be_mriq_phimag;
 typedef struct { int32_t numX, numK; const float *x, *y, *z, *kx, *ky, *kz, *phiMag; float *Qr, *Qi; } tacker_be_mriq_q;
+/* cutcp: V[p] = sum_{a: d^2 < cutoff^2} q_a / d * (1 - d^2/cutoff^2)^2, V[p] = 0 if any atom has
+ * d < excl.  Atoms come binned (TACKER_BE_CUTCP_BIN): bin side = 8*h, so one block (8x8x8
+ * lattice points) is one bin and its atoms within the cutoff lie in the bins within
+ * ceil(cutoff / bin side) bins in each direction; bins are visited and atoms summed in a fixed
+ * order (bit-identical fused vs original). */
 typedef struct {
   int32_t nx, ny, nz;        /* lattice points per axis, point (i,j,k) at h*(i,j,k) */
   float h, cutoff, excl;     /* spacing, cutoff radius, exclusion radius (Angstrom) */
-  int32_t bdim_x, bdim_y, bdim_z; /* atom bin grid (bin side = bin_size) */
-  float bin_size;
+  int32_t bdim_x, bdim_y, bdim_z; /* atom bin grid: bdim_* = ceil(n* / 8) */
+  float bin_size;            /* must equal 8*h */
   int32_t bin_depth;         /* atom slots per bin; unused slots have q == 0 and far coords */
   const float *bins;         /* float4 (x,y,z,q) [bdim_z][bdim_y][bdim_x][bin_depth] */
   float *V;                  /* [nz][ny][nx] */
 } tacker_be_cutcp;
+/* Binning: bin b = (floor(z/bs)*bdim_y + floor(y/bs))*bdim_x + floor(x/bs) (clamped into the grid)
+ * receives its atoms in atom-index order; unused slots get (1e30,1e30,1e30,0); count[b] = atoms
+ * in bin b, *overflow set to 1 if any bin holds more than bin_depth atoms (the caller re-bins
+ * with a larger depth; no atom is dropped silently). */
+typedef struct {
+  int32_t natoms;
+  const float *atoms;        /* float4 (x,y,z,q) [natoms] */
+  int32_t bdim_x, bdim_y, bdim_z, bin_depth;
+  float bin_size;
+  float *bins;               /* out: float4 [bdim_z*bdim_y*bdim_x*bin_depth] */
+  int32_t *count;            /* out: [bins] */
+  int32_t *overflow;         /* out: flag */
+} tacker_be_cutcp_bin;
 typedef struct { int32_t nx, ny, nz; const float *src; float *dst; const uint32_t *flags; } tacker_be_lbm;
 typedef struct { int32_t rows; const int32_t *perm, *row_len, *jds_ptr, *col; const float *val, *x; float *y; } tacker_be_spmv;
 typedef struct { int32_t n, nbins; const uint32_t *in; uint32_t *count; } tacker_be_histo;
@@ -150,6 +169,7 @@ typedef struct {
     tacker_be_bfs_commit bfs_commit;
     tacker_be_fma_burn fma_burn;
     tacker_be_im2col im2col;
+    tacker_be_cutcp_bin cutcp_bin;
     uint8_t _pad[128];
   } p;
 } tacker_be_desc;

@@ -132,6 +132,25 @@ def cutcp(atoms, nx, ny, nz, h, cutoff=CUTCP_CUTOFF, excl=CUTCP_EXCL, points=Non
     return V, S
 
 
+def cutcp_bins(atoms, bdim, bin_size, depth):
+    """Atom binning feeding the GPU cutcp (a data layout): bin
+    b = (floor(z/bs)*by + floor(y/bs))*bx + floor(x/bs), clamped into the grid, holds its atoms
+    in atom-index order; unused slots (1e30, 1e30, 1e30, 0).  Returns (bins, count)."""
+    bx, by, bz = bdim
+    at = np.asarray(atoms, np.float32)
+    bins = np.tile(np.array([1e30, 1e30, 1e30, 0.0], np.float32), (bx * by * bz, depth, 1))
+    count = np.zeros(bx * by * bz, np.int64)
+    for a in range(at.shape[0]):
+        ix = min(max(int(np.floor(at[a, 0] / bin_size)), 0), bx - 1)
+        iy = min(max(int(np.floor(at[a, 1] / bin_size)), 0), by - 1)
+        iz = min(max(int(np.floor(at[a, 2] / bin_size)), 0), bz - 1)
+        b = (iz * by + iy) * bx + ix
+        if count[b] < depth:
+            bins[b, count[b]] = at[a]
+        count[b] += 1
+    return bins, count
+
+
 # ----------------------------------------------------------------------------- c7 lbm
 import synth as _synth  # direction table only (data, not arithmetic)
 

@@ -321,6 +321,119 @@ template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   }
 };
 
+// ---------------------------------------------------------------- cutcp (Parboil)
+// Cutoff Coulomb potential.  Block = one atom bin = an 8x8x8 lattice region; thread t owns the
+// points (x = t%8, y = (t/8)%8, z = t/64 + 2m), m < 4, sharing dx, dy across its 4 points.
+// Neighbour bins within ceil(cutoff / bin side) are visited in (z, y, x) order, their atom slots
+// staged through shared memory 512 at a time, summed in slot order (deterministic):
+//   r2 = dz^2 + (dy^2 + dx^2);  e = ((q * rsqrt(r2)) * s) * s,  s = 1 - r2/c^2;  for r2 < c^2
+//   V = 0 if any r2 < excl^2.
+template <> struct BeBody<TACKER_BE_CUTCP> {
+  static constexpr int kStage = 512;
+  static constexpr uint32_t kSmem = kStage * 16;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_cutcp &p) {
+    return (int64_t)p.bdim_x * p.bdim_y * p.bdim_z;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_cutcp &p, int64_t vb, int tid, uint32_t bar,
+                                             uint8_t *smem) {
+    float4 *st = reinterpret_cast<float4 *>(smem);
+    const int rbx = (int)(vb % p.bdim_x), rby = (int)((vb / p.bdim_x) % p.bdim_y);
+    const int rbz = (int)(vb / ((int64_t)p.bdim_x * p.bdim_y));
+    const int i = rbx * 8 + (tid & 7), j = rby * 8 + ((tid >> 3) & 7), k0 = rbz * 8 + (tid >> 6);
+    const float px = (float)i * p.h, py = (float)j * p.h;
+    float pz[4], acc[4] = {0.f, 0.f, 0.f, 0.f};
+    bool ex[4] = {false, false, false, false};
+#pragma unroll
+    for (int m = 0; m < 4; ++m) pz[m] = (float)(k0 + 2 * m) * p.h;
+    const float c2 = __fmul_rn(p.cutoff, p.cutoff), e2 = __fmul_rn(p.excl, p.excl);
+    const float inv_c2 = __fdiv_rn(1.f, c2);
+    const int reach = (int)ceilf(p.cutoff / p.bin_size);
+    const int bx0 = max(rbx - reach, 0), bx1 = min(rbx + reach, p.bdim_x - 1);
+    const int by0 = max(rby - reach, 0), by1 = min(rby + reach, p.bdim_y - 1);
+    const int bz0 = max(rbz - reach, 0), bz1 = min(rbz + reach, p.bdim_z - 1);
+    const int nxr = bx1 - bx0 + 1, nyr = by1 - by0 + 1, nzr = bz1 - bz0 + 1;
+    const int64_t total = (int64_t)nxr * nyr * nzr * p.bin_depth;
+    const float4 *bins = reinterpret_cast<const float4 *>(p.bins);
+    for (int64_t c = 0; c < total; c += kStage) {
+      const int n = (int)min((int64_t)kStage, total - c);
+      for (int a = tid; a < n; a += kVbThreads) {
+        const int64_t g = c + a;
+        const int slot = (int)(g % p.bin_depth);
+        const int64_t lb = g / p.bin_depth;
+        const int lx = (int)(lb % nxr), ly = (int)((lb / nxr) % nyr), lz = (int)(lb / ((int64_t)nxr * nyr));
+        const int64_t b = ((int64_t)(bz0 + lz) * p.bdim_y + (by0 + ly)) * p.bdim_x + (bx0 + lx);
+        st[a] = __ldg(bins + b * p.bin_depth + slot);
+      }
+      named_bar_sync(bar, kVbThreads);
+#pragma unroll 4
+      for (int a = 0; a < n; ++a) {
+        const float4 at = st[a];
+        const float dx = __fsub_rn(at.x, px), dy = __fsub_rn(at.y, py);
+        const float dxy2 = __fmaf_rn(dy, dy, __fmul_rn(dx, dx));
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          const float dz = __fsub_rn(at.z, pz[m]);
+          const float r2 = __fmaf_rn(dz, dz, dxy2);
+          const float s = __fmaf_rn(-r2, inv_c2, 1.f);
+          const float e = __fmul_rn(__fmul_rn(__fmul_rn(at.w, rsqrtf(r2)), s), s);
+          acc[m] = r2 < c2 ? __fadd_rn(acc[m], e) : acc[m];
+          ex[m] = ex[m] | (r2 < e2);
+        }
+      }
+      named_bar_sync(bar, kVbThreads);
+    }
+    if (i < p.nx && j < p.ny) {
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+        const int k = k0 + 2 * m;
+        if (k < p.nz) p.V[((int64_t)k * p.ny + j) * p.nx + i] = ex[m] ? 0.f : acc[m];
+      }
+    }
+  }
+};
+
+// Deterministic binning for cutcp: thread = bin; atoms scanned in index order through shared
+// memory, an atom goes to bin (floor(z/bs), floor(y/bs), floor(x/bs)) clamped into the grid.
+template <> struct BeBody<TACKER_BE_CUTCP_BIN> {
+  static constexpr int kStage = 1024;
+  static constexpr uint32_t kSmem = kStage * 16;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_cutcp_bin &p) {
+    return ((int64_t)p.bdim_x * p.bdim_y * p.bdim_z + 127) / 128;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_cutcp_bin &p, int64_t vb, int tid, uint32_t bar,
+                                             uint8_t *smem) {
+    float4 *st = reinterpret_cast<float4 *>(smem);
+    const int64_t nb = (int64_t)p.bdim_x * p.bdim_y * p.bdim_z;
+    const int64_t b = vb * 128 + tid;
+    const float4 *atoms = reinterpret_cast<const float4 *>(p.atoms);
+    float4 *bins = reinterpret_cast<float4 *>(p.bins);
+    int cnt = 0;
+    for (int c = 0; c < p.natoms; c += kStage) {
+      const int n = min(kStage, p.natoms - c);
+      named_bar_sync(bar, kVbThreads);
+      for (int a = tid; a < n; a += kVbThreads) st[a] = __ldg(atoms + c + a);
+      named_bar_sync(bar, kVbThreads);
+      if (b < nb) {
+        for (int a = 0; a < n; ++a) {
+          const float4 at = st[a];
+          const int ix = min(max((int)floorf(__fdiv_rn(at.x, p.bin_size)), 0), p.bdim_x - 1);
+          const int iy = min(max((int)floorf(__fdiv_rn(at.y, p.bin_size)), 0), p.bdim_y - 1);
+          const int iz = min(max((int)floorf(__fdiv_rn(at.z, p.bin_size)), 0), p.bdim_z - 1);
+          if (((int64_t)iz * p.bdim_y + iy) * p.bdim_x + ix == b) {
+            if (cnt < p.bin_depth) bins[b * p.bin_depth + cnt] = at;
+            ++cnt;
+          }
+        }
+      }
+    }
+    if (b < nb) {
+      for (int s = cnt; s < p.bin_depth; ++s) bins[b * p.bin_depth + s] = make_float4(1e30f, 1e30f, 1e30f, 0.f);
+      p.count[b] = cnt;
+      if (cnt > p.bin_depth) *p.overflow = 1;
+    }
+  }
+};
+
 // ---------------------------------------------------------------- lbm (Parboil)
 // D3Q19 BGK push step, SoA src/dst [19][cells], block = 128 consecutive cells (x fastest).
 // Direction order C N S E W T B NE NW SE SW NT NB ST SB ET EB WT WB.
@@ -559,6 +672,8 @@ TK_BE_SEL(TACKER_BE_BFS_EXPAND, bfs_expand)
 TK_BE_SEL(TACKER_BE_BFS_COMMIT, bfs_commit)
 TK_BE_SEL(TACKER_BE_FMA_BURN, fma_burn)
 TK_BE_SEL(TACKER_BE_IM2COL, im2col)
+TK_BE_SEL(TACKER_BE_CUTCP, cutcp)
+TK_BE_SEL(TACKER_BE_CUTCP_BIN, cutcp_bin)
 #undef TK_BE_SEL
 
 // Maximum BE warps per fused CTA: register-heavy bodies (sgemm's 8x4 register tile) keep the
@@ -591,6 +706,6 @@ __device__ __forceinline__ void be_init(uint8_t *, int, uint32_t) {}
 #define TK_FOR_EACH_BE(X)                                                                       \
   X(TACKER_BE_SGEMM) X(TACKER_BE_STENCIL) X(TACKER_BE_MRIQ_PHIMAG) X(TACKER_BE_MRIQ_Q)          \
   X(TACKER_BE_LBM) X(TACKER_BE_SPMV_JDS) X(TACKER_BE_HISTO) X(TACKER_BE_BFS_EXPAND)             \
-  X(TACKER_BE_BFS_COMMIT) X(TACKER_BE_FMA_BURN) X(TACKER_BE_IM2COL)
+  X(TACKER_BE_BFS_COMMIT) X(TACKER_BE_FMA_BURN) X(TACKER_BE_IM2COL) X(TACKER_BE_CUTCP) X(TACKER_BE_CUTCP_BIN)
 
 }  // namespace tk

@@ -55,7 +55,7 @@ int sm_count() {
 const char *be_kind_name(int kind) {
   static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
                                 "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn",
-                                "im2col"};
+                                "im2col", "cutcp_bin"};
   return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
 }
 
@@ -133,6 +133,22 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
     case TACKER_BE_BFS_EXPAND:
     case TACKER_BE_BFS_COMMIT:
       break;
+    case TACKER_BE_CUTCP: {
+      const auto &p = d.p.cutcp;
+      if (p.nx <= 0 || p.ny <= 0 || p.nz <= 0 || !(p.h > 0) || !(p.cutoff > 0) || p.bin_depth <= 0 || !p.bins || !p.V)
+        return set_error("cutcp: bad args"), TACKER_EINVAL;
+      if (p.bin_size != 8.f * p.h || p.bdim_x != (p.nx + 7) / 8 || p.bdim_y != (p.ny + 7) / 8 || p.bdim_z != (p.nz + 7) / 8)
+        return set_error("cutcp: bins must be 8 lattice spacings wide covering the lattice"), TACKER_EUNSUPPORTED;
+      if (p.cutoff > 3.f * p.bin_size) return set_error("cutcp: cutoff > 3 bins"), TACKER_EUNSUPPORTED;
+      break;
+    }
+    case TACKER_BE_CUTCP_BIN: {
+      const auto &p = d.p.cutcp_bin;
+      if (p.natoms < 0 || p.bdim_x <= 0 || p.bdim_y <= 0 || p.bdim_z <= 0 || p.bin_depth <= 0 || !(p.bin_size > 0) ||
+          !p.bins || !p.count || !p.overflow || (p.natoms > 0 && !p.atoms))
+        return set_error("cutcp_bin: bad args"), TACKER_EINVAL;
+      break;
+    }
     case TACKER_BE_IM2COL: {
       const auto &p = d.p.im2col;
       if (p.n <= 0 || p.h <= 0 || p.w <= 0 || p.c <= 0 || p.r <= 0 || p.s <= 0 || p.stride <= 0 || p.pad < 0 ||

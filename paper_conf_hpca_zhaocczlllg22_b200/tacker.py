@@ -26,7 +26,7 @@ LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
 EPI_BIAS, EPI_RELU, EPI_RESIDUAL = 1, 2, 4
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
- BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL) = range(13)
+ BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN) = range(14)
 POLICY_TACKER, POLICY_BAYMAX = 0, 1
 DEC_FUSED, DEC_ORIGINAL_LC, DEC_REORDER_BE, DEC_IDLE_BE, DEC_NOTHING = range(5)
 MAX_APPS = 64
@@ -117,11 +117,17 @@ class BeIm2col(C.Structure):
                 ("x", C.c_void_p), ("out", C.c_void_p)]
 
 
+class BeCutcpBin(C.Structure):
+    _fields_ = [("natoms", C.c_int32), ("atoms", C.c_void_p), ("bdim_x", C.c_int32), ("bdim_y", C.c_int32),
+                ("bdim_z", C.c_int32), ("bin_depth", C.c_int32), ("bin_size", C.c_float), ("bins", C.c_void_p),
+                ("count", C.c_void_p), ("overflow", C.c_void_p)]
+
+
 class _BeUnion(C.Union):
     _fields_ = [("sgemm", BeSgemm), ("stencil", BeStencil), ("mriq_phimag", BeMriqPhimag), ("mriq_q", BeMriqQ),
                 ("cutcp", BeCutcp), ("lbm", BeLbm), ("spmv", BeSpmv), ("histo", BeHisto),
                 ("bfs_expand", BeBfsExpand), ("bfs_commit", BeBfsCommit), ("fma_burn", BeFmaBurn),
-                ("im2col", BeIm2col), ("_pad", C.c_uint8 * 128)]
+                ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("_pad", C.c_uint8 * 128)]
 
 
 class BeDesc(C.Structure):
@@ -332,6 +338,26 @@ def be_im2col(x, out, r, s, stride, pad, Kpad=None, orig_blocks=0) -> BeDesc:
     n, h, w, c = x.shape
     d = BeDesc(kind=BE_IM2COL, orig_blocks=orig_blocks)
     d.p.im2col = BeIm2col(n, h, w, c, r, s, stride, pad, out.shape[1] if Kpad is None else Kpad, _ptr(x), _ptr(out))
+    return d
+
+
+def cutcp_bin_dims(nx, ny, nz):
+    return (nx + 7) // 8, (ny + 7) // 8, (nz + 7) // 8
+
+
+def be_cutcp_bin(atoms, bins, count, overflow, nx, ny, nz, h, depth, orig_blocks=0) -> BeDesc:
+    """Bin atoms (float4 rows) for cutcp: bin side 8*h over the lattice (nx, ny, nz)."""
+    bx, by, bz = cutcp_bin_dims(nx, ny, nz)
+    d = BeDesc(kind=BE_CUTCP_BIN, orig_blocks=orig_blocks)
+    d.p.cutcp_bin = BeCutcpBin(atoms.shape[0], _ptr(atoms), bx, by, bz, depth, 8.0 * h, _ptr(bins), _ptr(count),
+                               _ptr(overflow))
+    return d
+
+
+def be_cutcp(bins, V, nx, ny, nz, h, depth, cutoff=12.0, excl=1.0, orig_blocks=0) -> BeDesc:
+    bx, by, bz = cutcp_bin_dims(nx, ny, nz)
+    d = BeDesc(kind=BE_CUTCP, orig_blocks=orig_blocks)
+    d.p.cutcp = BeCutcp(nx, ny, nz, h, cutoff, excl, bx, by, bz, 8.0 * h, depth, _ptr(bins), _ptr(V))
     return d
 
 

@@ -119,6 +119,29 @@ def be_case(kind, seed=0, size="small"):
             assert np.array_equal(o[0].view(np.uint32), ref)
             assert int(o[0].astype(np.int64).sum()) == n
         return dict(desc=tk.be_histo(dv, cnt, 4096), outs=[cnt], reset=lambda: cnt.zero_(), check=check, keep=(dv,))
+    if kind == tk.BE_CUTCP:
+        L = 16.0 if size == "small" else 48.0
+        d = synth.cutcp_inputs(L, seed)
+        nx = d["nx"]
+        depth = 32
+        bdim = tk.cutcp_bin_dims(nx, nx, nx)
+        datoms = t(d["atoms"])
+        bins = torch.zeros(bdim[0] * bdim[1] * bdim[2] * depth * 4, device=dev())
+        count = torch.zeros(bdim[0] * bdim[1] * bdim[2], dtype=torch.int32, device=dev())
+        ovf = torch.zeros(1, dtype=torch.int32, device=dev())
+        tk.tacker_launch_original(None, tk.be_cutcp_bin(datoms, bins, count, ovf, nx, nx, nx, 0.5, depth))
+        rb, rc = obe.cutcp_bins(d["atoms"], bdim, 4.0, depth)
+        assert int(host(ovf)[0]) == 0
+        assert np.array_equal(host(count), rc) and host(bins).tobytes() == rb.tobytes()
+        V = torch.zeros(nx ** 3, device=dev())
+        pts = None if size == "small" else np.random.default_rng(seed).choice(nx ** 3, 4096, replace=False)
+        ref, S = obe.cutcp(d["atoms"], nx, nx, nx, 0.5, points=pts)
+
+        def check(o):
+            g = o[0] if pts is None else o[0][pts]
+            assert max_rel_err(g, ref, S) <= 1e-5
+        return dict(desc=tk.be_cutcp(bins, V, nx, nx, nx, 0.5, depth), outs=[V], reset=lambda: V.zero_(),
+                    check=check, keep=(datoms, bins, count, ovf))
     if kind == tk.BE_FMA_BURN:
         n, iters = 128 * 300, 1000
         out = torch.zeros(n, device=dev())

@@ -73,7 +73,8 @@ def test_lc_conv_vs_oracle(tk, cs):
 
 
 # ------------------------------------------------------------------ BE originals (c3-c10)
-BE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_MRIQ_PHIMAG", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN"]
+BE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_MRIQ_PHIMAG", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN",
+            "BE_CUTCP"]
 
 
 @pytest.mark.parametrize("kind", BE_KINDS)
@@ -107,7 +108,7 @@ def test_bfs_levels_vs_oracle(tk):
 
 
 # ------------------------------------------------------------------ fused (a1-a8)
-FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN"]
+FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN", "BE_CUTCP"]
 
 
 @pytest.mark.parametrize("kind", FUSE_KINDS)

@@ -329,3 +329,23 @@ def test_fma_burn_closed_form_matches_iteration():
                 x = x * 0.5 + 0.125 * (j + 1)
             s += x
         assert abs(out[g] - s) < 1e-14
+
+
+def test_cutcp_bins_partition_atoms_in_index_order():
+    d = synth.cutcp_inputs(9.0, seed=20)
+    at = d["atoms"]
+    bdim = ((d["nx"] + 7) // 8, (d["ny"] + 7) // 8, (d["nz"] + 7) // 8)
+    bins, count = be.cutcp_bins(at, bdim, 4.0, 64)
+    assert count.sum() == at.shape[0] and count.max() <= 64
+    seen = []
+    for b in range(bins.shape[0]):
+        rows = bins[b, :count[b]]
+        for r in rows:
+            # every atom lies inside its bin's box
+            ix, iy, iz = (int(np.floor(r[c] / 4.0)) for c in range(3))
+            assert (iz * bdim[1] + iy) * bdim[0] + ix == b
+        idx = [int(np.nonzero(np.all(at == r, axis=1))[0][0]) for r in rows]
+        assert idx == sorted(idx)           # index order within a bin
+        seen += idx
+        assert np.all(bins[b, count[b]:, 3] == 0)
+    assert sorted(seen) == list(range(at.shape[0]))
