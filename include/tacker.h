@@ -124,6 +124,7 @@ typedef struct {
   float bin_size;            /* must equal 8*h */
   int32_t bin_depth;         /* atom slots per bin; unused slots have q == 0 and far coords */
   const float *bins;         /* float4 (x,y,z,q) [bdim_z][bdim_y][bdim_x][bin_depth] */
+  const int32_t *count;      /* atoms per bin (from the binning kernel); only these slots are read */
   float *V;                  /* [nz][ny][nx] */
 } tacker_be_cutcp;
 /* Binning: bin b = (floor(z/bs)*bdim_y + floor(y/bs))*bdim_x + floor(x/bs) (clamped into the grid)

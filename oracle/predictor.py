@@ -65,12 +65,17 @@ class TwoStage:
     def add(self, x_tc, x_cd, t_fused):
         self.samples.append((x_cd / x_tc, t_fused / x_tc))
 
-    def fit(self, split=1.0, iters=16):
+    def fit(self, split=None, iters=16):
+        """split=None: the lower half of the samples (by r) starts as stage 1 (for the training
+        ratios {0.1, 0.2, 1.8, 1.9}: {0.1, 0.2} vs {1.8, 1.9}); a split leaving one side empty
+        falls back to that median split."""
         pts = sorted(self.samples)
-        lo = [p for p in pts if p[0] <= split]
-        hi = [p for p in pts if p[0] > split]
+        if len(pts) < 2:
+            raise ValueError("need at least 2 samples")
+        lo = [p for p in pts if split is not None and p[0] <= split]
+        hi = [p for p in pts if split is not None and p[0] > split]
         if not lo or not hi:
-            raise ValueError("need samples on both sides of the split")
+            lo, hi = pts[:len(pts) // 2], pts[len(pts) // 2:]
         for _ in range(iters):
             b1, a1 = ols([p[0] for p in lo], [p[1] for p in lo])
             b2, a2 = ols([p[0] for p in hi], [p[1] for p in hi])
@@ -104,6 +109,6 @@ class TwoStage:
         if abs(pred - t_meas) / t_meas > REFIT_THRESHOLD:
             self.add(x_tc, x_cd, t_meas)
             rs = self.inflection()
-            self.fit(split=rs if rs is not None and rs > 0 else 1.0)
+            self.fit(split=rs if rs is not None and rs > 0 else None)
             return True
         return False

@@ -351,18 +351,25 @@ template <> struct BeBody<TACKER_BE_CUTCP> {
     const int bx0 = max(rbx - reach, 0), bx1 = min(rbx + reach, p.bdim_x - 1);
     const int by0 = max(rby - reach, 0), by1 = min(rby + reach, p.bdim_y - 1);
     const int bz0 = max(rbz - reach, 0), bz1 = min(rbz + reach, p.bdim_z - 1);
-    const int nxr = bx1 - bx0 + 1, nyr = by1 - by0 + 1, nzr = bz1 - bz0 + 1;
-    const int64_t total = (int64_t)nxr * nyr * nzr * p.bin_depth;
+    const int nxr = bx1 - bx0 + 1;
     const float4 *bins = reinterpret_cast<const float4 *>(p.bins);
-    for (int64_t c = 0; c < total; c += kStage) {
-      const int n = (int)min((int64_t)kStage, total - c);
+    // one x-row of neighbour bins (<= 7 bins) per round, only their occupied slots, compacted in
+    // (bin, slot) order
+    for (int bz = bz0; bz <= bz1; ++bz)
+    for (int by = by0; by <= by1; ++by) {
+      const int64_t row = ((int64_t)bz * p.bdim_y + by) * p.bdim_x;
+      int cnt[7], off[7], n = 0;
+#pragma unroll
+      for (int q = 0; q < 7; ++q) {
+        cnt[q] = q < nxr ? min(__ldg(p.count + row + bx0 + q), p.bin_depth) : 0;
+        off[q] = n;
+        n += cnt[q];
+      }
       for (int a = tid; a < n; a += kVbThreads) {
-        const int64_t g = c + a;
-        const int slot = (int)(g % p.bin_depth);
-        const int64_t lb = g / p.bin_depth;
-        const int lx = (int)(lb % nxr), ly = (int)((lb / nxr) % nyr), lz = (int)(lb / ((int64_t)nxr * nyr));
-        const int64_t b = ((int64_t)(bz0 + lz) * p.bdim_y + (by0 + ly)) * p.bdim_x + (bx0 + lx);
-        st[a] = __ldg(bins + b * p.bin_depth + slot);
+        int q = 0;
+#pragma unroll
+        for (int u = 1; u < 7; ++u) q += (a >= off[u] && u < nxr) ? 1 : 0;
+        st[a] = __ldg(bins + (row + bx0 + q) * p.bin_depth + (a - off[q]));
       }
       named_bar_sync(bar, kVbThreads);
 #pragma unroll 4

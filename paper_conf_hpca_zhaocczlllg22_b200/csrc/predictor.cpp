@@ -57,11 +57,19 @@ void ols(const std::vector<std::pair<double, double>> &p, double &slope, double 
   icpt = my - slope * mx;
 }
 
+// split < 0: the lower half of the samples (by r) starts as stage 1 — for the paper's training
+// ratios {0.1, 0.2, 1.8, 1.9} that is {0.1, 0.2} vs {1.8, 1.9}, and it still works
+// when coarse BE blocks shift every measured ratio to one side of 1.
 bool fit_pair(Pair &P, double split) {
   std::vector<std::pair<double, double>> pts = P.pts, lo, hi;
   std::sort(pts.begin(), pts.end());
-  for (auto &q : pts) (q.first <= split ? lo : hi).push_back(q);
-  if (lo.empty() || hi.empty()) return false;
+  if (pts.size() < 2) return false;
+  if (split >= 0)
+    for (auto &q : pts) (q.first <= split ? lo : hi).push_back(q);
+  if (lo.empty() || hi.empty()) {   // median split (also the fallback for a one-sided split)
+    lo.assign(pts.begin(), pts.begin() + pts.size() / 2);
+    hi.assign(pts.begin() + pts.size() / 2, pts.end());
+  }
   for (int it = 0; it < 16; ++it) {
     ols(lo, P.b1, P.a1);
     ols(hi, P.b2, P.a2);
@@ -143,8 +151,8 @@ tacker_status tacker_pair_fit(const char *key, double coef_out[4]) {
   if (!key_ok(key)) return set_error("bad key"), TACKER_EINVAL;
   std::lock_guard<std::mutex> g(g_mu);
   auto it = g_pair.find(key);
-  if (it == g_pair.end() || !fit_pair(it->second, 1.0))
-    return set_error("pair %s needs samples on both sides of r = 1", key), TACKER_ENOMODEL;
+  if (it == g_pair.end() || !fit_pair(it->second, -1.0))
+    return set_error("pair %s needs at least 2 samples", key), TACKER_ENOMODEL;
   if (coef_out) {
     coef_out[0] = it->second.a1;
     coef_out[1] = it->second.b1;
@@ -170,7 +178,7 @@ tacker_status tacker_pair_observe(const char *key, double x_tc, double x_cd, dou
   int32_t refit = 0;
   if (std::fabs(pred - t_meas) / t_meas > 0.10) {
     P.pts.emplace_back(x_cd / x_tc, t_meas / x_tc);
-    double split = 1.0;
+    double split = -1.0;
     if (P.b1 != P.b2) {
       const double rs = (P.a2 - P.a1) / (P.b1 - P.b2);
       if (rs > 0) split = rs;
@@ -231,7 +239,7 @@ tacker_status tacker_model_load(const char *path) {
     } else {
       Pair &P = g_pair[key];
       P.pts = pts;
-      fit_pair(P, 1.0);
+      fit_pair(P, -1.0);
     }
   }
   fclose(f);

@@ -135,8 +135,11 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
       break;
     case TACKER_BE_CUTCP: {
       const auto &p = d.p.cutcp;
-      if (p.nx <= 0 || p.ny <= 0 || p.nz <= 0 || !(p.h > 0) || !(p.cutoff > 0) || p.bin_depth <= 0 || !p.bins || !p.V)
+      if (p.nx <= 0 || p.ny <= 0 || p.nz <= 0 || !(p.h > 0) || !(p.cutoff > 0) || p.bin_depth <= 0 || !p.bins ||
+          !p.count || !p.V)
         return set_error("cutcp: bad args"), TACKER_EINVAL;
+      if (7 * p.bin_depth > BeBody<TACKER_BE_CUTCP>::kStage)
+        return set_error("cutcp: bin_depth must be <= %d", BeBody<TACKER_BE_CUTCP>::kStage / 7), TACKER_EUNSUPPORTED;
       if (p.bin_size != 8.f * p.h || p.bdim_x != (p.nx + 7) / 8 || p.bdim_y != (p.ny + 7) / 8 || p.bdim_z != (p.nz + 7) / 8)
         return set_error("cutcp: bins must be 8 lattice spacings wide covering the lattice"), TACKER_EUNSUPPORTED;
       if (p.cutoff > 3.f * p.bin_size) return set_error("cutcp: cutoff > 3 bins"), TACKER_EUNSUPPORTED;

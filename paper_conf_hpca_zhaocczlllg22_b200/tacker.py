@@ -79,7 +79,8 @@ class BeMriqQ(C.Structure):
 class BeCutcp(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32), ("h", C.c_float), ("cutoff", C.c_float),
                 ("excl", C.c_float), ("bdim_x", C.c_int32), ("bdim_y", C.c_int32), ("bdim_z", C.c_int32),
-                ("bin_size", C.c_float), ("bin_depth", C.c_int32), ("bins", C.c_void_p), ("V", C.c_void_p)]
+                ("bin_size", C.c_float), ("bin_depth", C.c_int32), ("bins", C.c_void_p), ("count", C.c_void_p),
+                ("V", C.c_void_p)]
 
 
 class BeLbm(C.Structure):
@@ -354,10 +355,10 @@ def be_cutcp_bin(atoms, bins, count, overflow, nx, ny, nz, h, depth, orig_blocks
     return d
 
 
-def be_cutcp(bins, V, nx, ny, nz, h, depth, cutoff=12.0, excl=1.0, orig_blocks=0) -> BeDesc:
+def be_cutcp(bins, count, V, nx, ny, nz, h, depth, cutoff=12.0, excl=1.0, orig_blocks=0) -> BeDesc:
     bx, by, bz = cutcp_bin_dims(nx, ny, nz)
     d = BeDesc(kind=BE_CUTCP, orig_blocks=orig_blocks)
-    d.p.cutcp = BeCutcp(nx, ny, nz, h, cutoff, excl, bx, by, bz, 8.0 * h, depth, _ptr(bins), _ptr(V))
+    d.p.cutcp = BeCutcp(nx, ny, nz, h, cutoff, excl, bx, by, bz, 8.0 * h, depth, _ptr(bins), _ptr(count), _ptr(V))
     return d
 
 

@@ -140,7 +140,7 @@ def be_case(kind, seed=0, size="small"):
         def check(o):
             g = o[0] if pts is None else o[0][pts]
             assert max_rel_err(g, ref, S) <= 1e-5
-        return dict(desc=tk.be_cutcp(bins, V, nx, nx, nx, 0.5, depth), outs=[V], reset=lambda: V.zero_(),
+        return dict(desc=tk.be_cutcp(bins, count, V, nx, nx, nx, 0.5, depth), outs=[V], reset=lambda: V.zero_(),
                     check=check, keep=(datoms, bins, count, ovf))
     if kind == tk.BE_FMA_BURN:
         n, iters = 128 * 300, 1000
