@@ -320,9 +320,14 @@ tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms);
  * headroom, or NAN to use the manager's Eq. 9 value; on output the updated headroom. */
 tacker_status tacker_manager_step(tacker_manager_t m, double qos_target_ms, double *headroom_ms,
                                   tacker_decision *out);
+/* Native run loop: steps the manager (launching in GPU mode) until its clock has passed
+ * t_end_ms and every submitted query has completed, or max_decisions decisions were taken
+ * (<= 0: unbounded).  The host thread spins between decisions (no Python in the loop). */
+tacker_status tacker_manager_run(tacker_manager_t m, double qos_target_ms, double t_end_ms, int64_t max_decisions);
 typedef struct {
   int64_t lc_queries_done, be_kernels_done, fused_launches, original_lc, reordered_be, idle_be;
   double now_ms;
+  int64_t model_refits;      /* GPU mode: two-stage refits triggered by measured fused runs */
 } tacker_manager_stats;
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
 /* Completion time (manager clock) of a finished query, or -1 if unfinished. */

@@ -13,8 +13,11 @@ Rules, in the paper's order:
     fused prediction Tk_fuse: admissible iff Ttc + Tcd > Tk_fuse and Tk_fuse - Ttc < Thr.
     Pick the max Tgain = Tcd - (Tk_fuse - Ttc); ties -> lowest app index.
     Then Thr -= Tk_fuse - Ttc.
-  * Reorder: if no fusion happened, launch ready BE heads (app index order)
-    whose Ttmp < Thr, Thr -= Ttmp.
+  * Reorder: after the LC kernel (fused or not), launch the other ready BE heads
+    (app index order) whose Ttmp < Thr, Thr -= Ttmp.  Reading: the text applies
+    reorder when no fusion is possible; Tacker is described as using "both adaptive kernel
+    fusion and kernel reorder", so reordering also follows a fused launch and
+    Tacker never reorders less than Baymax.
   * Only the head kernel of each BE app is a candidate; the next kernel of an app
     becomes ready when the previous one completes.
   * Baymax mode = the same manager with fusion disabled ("static scheduling").
@@ -59,8 +62,10 @@ def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True):
     reorder = []
     if fused >= 0:
         thr -= tf_best - ttc
-    elif allow:
+    if allow:
         for app, tcd, _ in heads:
+            if app == fused:
+                continue
             if tcd < thr:
                 reorder.append(app)
                 thr -= tcd
@@ -137,7 +142,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 apps[fused].pos += 1
                 apps[fused].completed += 1
                 apps[fused].ready_at = start + dur
-                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, [], q.thr, gain))
+                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), q.thr, gain))
             else:
                 dur = ttc
                 timeline.append(("lc", q.qid, q.pos, -1, start, start + dur))

@@ -79,6 +79,14 @@ struct tacker_manager_s {
   std::map<std::string, tacker_fused_t> cache;
   std::deque<cudaEvent_t> inflight;
   std::vector<cudaEvent_t> free_events;
+  std::map<cudaEvent_t, int> refs;
+  struct Observed {
+    cudaEvent_t start, end;
+    std::string pair_key;
+    double x_tc, x_cd;
+  };
+  std::deque<Observed> observed;   // fused launches awaiting their measured duration
+  int64_t refits = 0;
 
   bool sim() const { return prm.simulate != 0; }
 };
@@ -106,18 +114,49 @@ static double event_time(tacker_manager_s *m, cudaEvent_t e) {
   return (double)ms;
 }
 
+// Events are reference counted (in flight / an app's pending kernel / a query's last kernel)
+// and recycled when the last reference drops.
+static cudaEvent_t ref(tacker_manager_s *m, cudaEvent_t e) {
+  m->refs[e]++;
+  return e;
+}
+static void unref(tacker_manager_s *m, cudaEvent_t e) {
+  auto it = m->refs.find(e);
+  if (it != m->refs.end() && --it->second == 0) {
+    m->refs.erase(it);
+    m->free_events.push_back(e);
+  }
+}
+
 static void poll(tacker_manager_s *m) {
   if (m->sim()) return;
-  while (!m->inflight.empty() && cudaEventQuery(m->inflight.front()) == cudaSuccess) m->inflight.pop_front();
+  while (!m->inflight.empty() && cudaEventQuery(m->inflight.front()) == cudaSuccess) {
+    unref(m, m->inflight.front());
+    m->inflight.pop_front();
+  }
   for (auto &a : m->apps)
     if (a.pending && cudaEventQuery(a.pending) == cudaSuccess) {
       a.ready_at = event_time(m, a.pending);
+      unref(m, a.pending);
       a.pending = nullptr;
     }
+  while (!m->observed.empty() && cudaEventQuery(m->observed.front().end) == cudaSuccess) {
+    auto &o = m->observed.front();
+    float ms = 0;
+    cudaEventElapsedTime(&ms, o.start, o.end);
+    int32_t refit = 0;
+    if (ms > 0 && tacker_pair_observe(o.pair_key.c_str(), o.x_tc, o.x_cd, ms, &refit) == TACKER_OK && refit)
+      m->refits++;
+    unref(m, o.start);
+    unref(m, o.end);
+    m->observed.pop_front();
+  }
   for (int id : m->active) {
     Query &q = m->queries[id];
     if (q.pos == q.ks.size() && q.done_at < 0 && q.last_ev && cudaEventQuery(q.last_ev) == cudaSuccess) {
       q.done_at = event_time(m, q.last_ev);
+      unref(m, q.last_ev);
+      q.last_ev = nullptr;
       m->st.lc_queries_done++;
     }
   }
@@ -164,7 +203,7 @@ static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k
 static cudaEvent_t record(tacker_manager_s *m) {
   cudaEvent_t e = get_event(m);
   cudaEventRecord(e, m->stream);
-  m->inflight.push_back(e);
+  m->inflight.push_back(ref(m, e));
   return e;
 }
 
@@ -286,7 +325,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       } else {
         tacker_status s = launch_be(m, b);
         if (s) return s;
-        A.pending = record(m);
+        A.pending = ref(m, record(m));
       }
       A.pos++;
       A.completed++;
@@ -344,10 +383,13 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
     }
   }
   std::vector<int> reorder;
-  if (fused >= 0) {
-    thr -= best_tf - ttc;
-  } else if (allow) {
+  if (fused >= 0) thr -= best_tf - ttc;
+  // Reorder the remaining ready heads after the LC kernel, fused or not (reading:
+  // Tacker = fusion on top of Baymax's reordering, "both adaptive kernel fusion and kernel
+  // reorder").
+  if (allow) {
     for (int a : heads) {
+      if (a == fused) continue;
       const double tt = m->apps[a].head().t_pred_ms;
       if (tt < thr) {
         reorder.push_back(a);
@@ -370,11 +412,17 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       m->now += best_tf;
       A.ready_at = m->now;
     } else {
+      cudaEvent_t e0 = get_event(m);
+      cudaEventRecord(e0, m->stream);
       tacker_status s = launch_fused(m, k, A.head());
       if (s) return s;
       cudaEvent_t e = record(m);
-      A.pending = e;
-      if (q.pos + 1 == q.ks.size()) q.last_ev = e;
+      A.pending = ref(m, e);
+      if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
+      // online model update from the measured co-run
+      std::string lk, bk, pk;
+      make_keys(&k.lc, &A.head().be, A.head().warp_split ? A.head().warp_split : 16, &lk, &bk, &pk);
+      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, A.head().t_pred_ms});
     }
     A.pos++;
     A.completed++;
@@ -388,7 +436,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       tacker_status s = launch_lc(m, k);
       if (s) return s;
       cudaEvent_t e = record(m);
-      if (q.pos + 1 == q.ks.size()) q.last_ev = e;
+      if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
     }
     m->st.original_lc++;
     out->action = reorder.empty() ? TACKER_DEC_ORIGINAL_LC : TACKER_DEC_REORDER_BE;
@@ -407,7 +455,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
     } else {
       tacker_status s = launch_be(m, b);
       if (s) return s;
-      A.pending = record(m);
+      A.pending = ref(m, record(m));
     }
     A.pos++;
     A.completed++;
@@ -419,11 +467,36 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   return TACKER_OK;
 }
 
+tacker_status tacker_manager_run(tacker_manager_t m, double qos, double t_end_ms, int64_t max_decisions) {
+  if (!m) return set_error("null manager"), TACKER_EINVAL;
+  int64_t n = 0;
+  tacker_decision d;
+  for (;;) {
+    double thr = NAN;
+    tacker_status s = tacker_manager_step(m, qos, &thr, &d);
+    if (s) return s;
+    if (d.action != TACKER_DEC_NOTHING && max_decisions > 0 && ++n >= max_decisions) break;
+    if (d.action == TACKER_DEC_NOTHING) {
+      poll(m);
+      const bool all_done = m->st.lc_queries_done == (int64_t)m->queries.size();
+      if (all_done && m->now >= t_end_ms) break;
+      if (m->sim() && all_done && m->next_pending >= m->pending.size()) break;
+    }
+  }
+  if (!m->sim()) {
+    cudaError_t e = cudaStreamSynchronize(m->stream);
+    if (e != cudaSuccess) return cuda_fail("manager run sync", e);
+    poll(m);
+  }
+  return TACKER_OK;
+}
+
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *o) {
   if (!m || !o) return set_error("null argument"), TACKER_EINVAL;
   poll(m);
   *o = m->st;
   o->now_ms = m->sim() ? m->now : host_now(m);
+  o->model_refits = m->refits;
   return TACKER_OK;
 }
 

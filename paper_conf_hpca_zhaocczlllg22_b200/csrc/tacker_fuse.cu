@@ -13,7 +13,9 @@
 #include <cstdio>
 #include <cstring>
 #include <mutex>
+#include <memory>
 #include <string>
+#include <unordered_map>
 
 #include "kernels/fused.cuh"
 #include "runtime.h"
@@ -583,10 +585,26 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   tacker_status st;
   if (lc && lc->kind != TACKER_LC_NONE) {
-    tacker_fused_s F;
-    if ((st = plan(lc, nullptr, 0, tacker_ratio{0, 0}, F))) return st;
-    F.P.work = nullptr;
-    if ((st = launch_plan(F, s))) return st;
+    // LC-only plans (tensor maps, smem attribute) are cached by descriptor bytes: the manager
+    // re-launches the same LC kernels every query.
+    static std::mutex mu;
+    static std::unordered_map<std::string, std::unique_ptr<tacker_fused_s>> cache;
+    const std::string key(reinterpret_cast<const char *>(lc), sizeof *lc);
+    tacker_fused_s *F = nullptr;
+    {
+      std::lock_guard<std::mutex> g(mu);
+      auto it = cache.find(key);
+      if (it != cache.end()) F = it->second.get();
+    }
+    if (!F) {
+      auto P = std::make_unique<tacker_fused_s>();
+      if ((st = plan(lc, nullptr, 0, tacker_ratio{0, 0}, *P))) return st;
+      P->P.work = nullptr;
+      std::lock_guard<std::mutex> g(mu);
+      if (cache.size() > 4096) cache.clear();
+      F = (cache[key] = std::move(P)).get();
+    }
+    if ((st = launch_plan(*F, s))) return st;
   }
   if (be && be->kind != TACKER_BE_NONE) {
     int64_t blocks;

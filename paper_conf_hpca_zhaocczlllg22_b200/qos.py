@@ -1,0 +1,176 @@
+"""QoS-managed co-location run (a12; BASELINE configs 2/4/5; paper §VIII-B).
+
+LC queries of a service (ResNet-50 / VGG-16 / ...) arrive as a Poisson process at a fraction of
+the service's peak rate; a BE queue of Parboil-style applications fills the rest of the GPU; the
+native manager (tacker_manager_run) decides fused / original / reorder per LC kernel from each
+query's QoS headroom (§VII).  Before the run, the predictor is calibrated the paper's way
+(§VI-C): standalone durations of every LC and BE kernel (history), and per (LC kernel class, BE
+kernel class, warp split) a two-stage model from fused runs at the training load ratios
+{0.1, 0.2, 1.8, 1.9}, the BE sized through its PTB block prefix.
+
+Reported: BE kernels/s, LC latency p50/p99 vs the QoS target, fused / reordered / idle BE
+counts; the same trace under the Baymax policy (fusion disabled) gives the Eq. 10 improvement.
+"""
+from __future__ import annotations
+
+import math
+import statistics
+
+import numpy as np
+import torch
+
+from . import tacker as tk
+
+
+def _time(fn, reps=10, stream=None):
+    s = stream or torch.cuda.current_stream()
+    fn()
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        fn()
+        e1.record(s)
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    return statistics.median(ts)
+
+
+class QosRun:
+    def __init__(self, svc, apps, warp_split=24, qos_ms=50.0):
+        self.svc, self.apps, self.ws, self.qos = svc, apps, warp_split, qos_ms
+        self.t_lc = []           # standalone ms per LC kernel
+        self.t_be = {}           # (app index, kernel index) -> ms
+        self.pairs = {}          # pair key -> fitted coefficients
+        self.ws_of = {}          # (app, kernel) -> warp split that fits the budget
+        self.pair_err = []       # |pred - meas| / meas of the fused model on the real pairs
+
+    # ------------------------------------------------------------------ calibration (§VI-C)
+    def calibrate(self, reps=8, pair_reps=5):
+        for k in self.svc.kernels:
+            if k.is_tc:
+                self.t_lc.append(_time(lambda: tk.tacker_launch_original(k.lc, None), reps))
+            else:
+                self.t_lc.append(_time(lambda: tk.tacker_launch_original(None, k.cd), reps))
+        for a, app in enumerate(self.apps):
+            for j, bk in enumerate(app.kernels):
+                self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(None, bk.desc), reps)
+        # two-stage models per (LC class, BE class, ws), trained on block prefixes
+        for i, k in enumerate(self.svc.kernels):
+            if not k.is_tc:
+                continue
+            for a, app in enumerate(self.apps):
+                for j, bk in enumerate(app.kernels):
+                    if bk.name.endswith("phimag"):
+                        continue
+                    f = None
+                    for ws in range(self.ws, 3, -4):
+                        try:
+                            f = tk.tacker_fuse(k.lc, bk.desc, ws)
+                            break
+                        except tk.TackerError as e:
+                            if e.status != tk.ERESOURCE:
+                                raise
+                    if f is None:
+                        continue
+                    self.ws_of[(a, j)] = ws
+                    pkey = f.keys()[2]
+                    if pkey not in self.pairs:
+                        self.pairs[pkey] = self._fit_pair(k, bk, ws, self.t_lc[i], pkey, pair_reps)
+                    # accuracy of the fitted model on the actual whole-kernel pair
+                    t_meas = _time(lambda: f.launch(), 3)
+                    t_pred = tk.tacker_pair_predict(pkey, self.t_lc[i], self.t_be[(a, j)])
+                    self.pair_err.append(abs(t_pred - t_meas) / t_meas)
+
+    def _fit_pair(self, k, bk, ws, x_tc, pkey, reps):
+        full = tk.tacker_be_num_blocks(bk.desc)
+
+        def prefix(n):
+            d = tk.BeDesc()
+            C_copy = bytes(bk.desc)
+            import ctypes
+            ctypes.memmove(ctypes.addressof(d), C_copy, ctypes.sizeof(d))
+            d.orig_blocks = n
+            return d
+        t_full = self.t_be_of(bk)
+        # BE duration is ~ linear in blocks above its one-block floor (PTB LR)
+        t_one = _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)
+        a = (t_full - t_one) / max(full - 1, 1)
+        r_floor = t_one / x_tc
+        shift = max(0.0, 1.25 * r_floor - 0.1)
+        for r in (0.1 + shift, 0.2 + shift, 1.8 + shift, 1.9 + shift):
+            n = int(round((r * x_tc - t_one) / a)) + 1 if a > 0 else full
+            n = min(max(n, 1), full)
+            d = prefix(n)
+            f = tk.tacker_fuse(k.lc, d, ws)
+            t_f = _time(lambda: f.launch(), reps)
+            x_cd = _time(lambda: tk.tacker_launch_original(None, d), reps)
+            tk.tacker_pair_add_sample(pkey, x_tc, x_cd, t_f)
+        return tk.tacker_pair_fit(pkey)
+
+    def t_be_of(self, bk):
+        for a, app in enumerate(self.apps):
+            for j, b in enumerate(app.kernels):
+                if b is bk:
+                    return self.t_be[(a, j)]
+        raise KeyError(bk.name)
+
+    # ------------------------------------------------------------------ structs for the manager
+    def lc_kernels(self):
+        out = []
+        for k, t in zip(self.svc.kernels, self.t_lc):
+            lk = tk.LcKernel(is_tc=1 if k.is_tc else 0, t_pred_ms=t)
+            if k.is_tc:
+                lk.lc = k.lc
+            else:
+                lk.cd = k.cd
+            out.append(lk)
+        return out
+
+    def be_apps(self):
+        out = []
+        for a, app in enumerate(self.apps):
+            ks = []
+            for j, bk in enumerate(app.kernels):
+                ks.append(tk.BeKernel(is_cd=1, t_pred_ms=self.t_be[(a, j)],
+                                      be=bk.desc, warp_split=self.ws_of.get((a, j), self.ws)))
+            out.append(ks)
+        return out
+
+    def query_solo_ms(self):
+        return sum(self.t_lc)
+
+    # ------------------------------------------------------------------ one managed run
+    def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None):
+        """Poisson arrivals at `load` x the service's peak rate (1 / standalone query time; the
+        paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
+        stream = torch.cuda.current_stream()
+        torch.cuda.synchronize()
+        lam = load / self.query_solo_ms()                       # queries per ms
+        rng = np.random.default_rng(seed)
+        gaps = rng.exponential(1.0 / lam, n_queries + warmup)
+        cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
+        m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight)
+        for ks in self.be_apps():
+            m.submit_be(ks)
+        kernels = self.lc_kernels()
+        t0 = m.stats().now_ms + 2.0
+        arr = t0 + np.cumsum(gaps)
+        qids = [m.submit_lc(kernels, float(t)) for t in arr]
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        m.run(self.qos, float(arr[-1]))
+        e1.record(stream)
+        e1.synchronize()
+        st = m.stats()
+        lat = np.array([m.latency(q) for q in qids[warmup:]])
+        gpu_ms = e0.elapsed_time(e1)
+        lat_sorted = np.sort(lat)
+        p99 = float(lat_sorted[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)])
+        return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "queries": int(len(lat)),
+                "lambda_per_s": lam * 1e3, "load": load, "elapsed_ms": gpu_ms,
+                "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
+                "fused": int(st.fused_launches), "reordered": int(st.reordered_be), "idle_be": int(st.idle_be),
+                "model_refits": int(st.model_refits),
+                "lc_p50_ms": float(np.median(lat)), "lc_p99_ms": p99, "lc_max_ms": float(lat.max()),
+                "qos_ms": self.qos, "qos_met": bool(p99 <= self.qos), "query_solo_ms": self.query_solo_ms()}

@@ -178,7 +178,7 @@ class ManagerParams(C.Structure):
 class ManagerStats(C.Structure):
     _fields_ = [("lc_queries_done", C.c_int64), ("be_kernels_done", C.c_int64), ("fused_launches", C.c_int64),
                 ("original_lc", C.c_int64), ("reordered_be", C.c_int64), ("idle_be", C.c_int64),
-                ("now_ms", C.c_double)]
+                ("now_ms", C.c_double), ("model_refits", C.c_int64)]
 
 
 # ----------------------------------------------------------------------------- prototypes
@@ -211,6 +211,7 @@ _PROTOS = {
     "tacker_manager_set_clock": ([_V, _D], C.c_int),
     "tacker_manager_step": ([_V, _D, C.POINTER(_D), C.POINTER(Decision)], C.c_int),
     "tacker_manager_stats_get": ([_V, C.POINTER(ManagerStats)], C.c_int),
+    "tacker_manager_run": ([_V, _D, _D, _I64], C.c_int),
     "tacker_manager_query_latency": ([_V, _I32, C.POINTER(_D)], C.c_int),
 }
 for _name, (_args, _res) in _PROTOS.items():
@@ -532,6 +533,10 @@ class Manager:
         thr = C.c_double(headroom)
         _chk(_lib.tacker_manager_step(self.h, qos_ms, C.byref(thr), C.byref(d)))
         return d
+
+    def run(self, qos_ms, t_end_ms=0.0, max_decisions=0):
+        """Native loop: decide + launch until t_end_ms has passed and all queries completed."""
+        _chk(_lib.tacker_manager_run(self.h, qos_ms, t_end_ms, max_decisions))
 
     def stats(self) -> ManagerStats:
         s = ManagerStats()

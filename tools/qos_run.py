@@ -1,0 +1,61 @@
+"""QoS-managed co-location (BASELINE configs 2/4): LC service + BE queue under the Tacker and the
+Baymax policy on the same Poisson trace.  Prints one JSON line.
+
+  python tools/qos_run.py [--service resnet50|vgg16] [--batch 1] [--queries 400] [--load 0.8]
+                          [--be stencil,mriq] [--ws 24]
+"""
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_hpca_zhaocczlllg22_b200 import qos, services as sv, tacker as tk  # noqa: E402
+
+
+def build_apps(names):
+    apps = []
+    for n in names:
+        if n == "stencil":
+            apps.append(sv.stencil_app(512, 512, 64))
+        elif n == "mriq":
+            apps.append(sv.mriq_app(64, 2048, 1024))
+        elif n == "sgemm":
+            apps.append(sv.sgemm_app(2048, 2048, 2048))
+        else:
+            raise ValueError(n)
+    return apps
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--service", default="resnet50")
+    ap.add_argument("--batch", type=int, default=1)
+    ap.add_argument("--queries", type=int, default=400)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--load", type=float, default=0.8)
+    ap.add_argument("--be", default="stencil,mriq")
+    ap.add_argument("--ws", type=int, default=24)
+    ap.add_argument("--qos", type=float, default=50.0)
+    args = ap.parse_args()
+    svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
+    apps = build_apps(args.be.split(","))
+    tk.tacker_model_clear()
+    q = qos.QosRun(svc, apps, warp_split=args.ws, qos_ms=args.qos)
+    q.calibrate()
+    res = {}
+    for pol in (tk.POLICY_BAYMAX, tk.POLICY_TACKER):
+        r = q.run(pol, args.queries, load=args.load, warmup=args.warmup)
+        res[r["policy"]] = r
+    res["improvement_eq10"] = res["tacker"]["be_kernels_per_s"] / res["baymax"]["be_kernels_per_s"] - 1.0
+    res["pairs_fitted"] = len(q.pairs)
+    res["pair_pred_err"] = {"max": max(q.pair_err), "mean": sum(q.pair_err) / len(q.pair_err), "n": len(q.pair_err)}
+    print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    main()
