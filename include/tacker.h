@@ -105,7 +105,9 @@ typedef enum {
   TACKER_BE_IM2COL = 12,      /* LC CUDA-core helper: explicit im2col (cudnnIm2col, §VIII-H
                                  P:3350-3381) NHWC fp16 -> [M, Kpad] fp16; block = 1024x8 el. */
   TACKER_BE_CUTCP_BIN = 13,   /* cutcp atom binning (deterministic, index order); block = 128 bins */
-  TACKER_BE_KIND_COUNT = 14
+  TACKER_BE_COPY = 14,        /* byte copy, e.g. a query's H2D/D2H through host-mapped pinned
+                                 memory (UVA); block = 16 KiB */
+  TACKER_BE_KIND_COUNT = 15
 } tacker_be_kind;
 
 typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
@@ -153,6 +155,9 @@ typedef struct {
   const void *x;   /* fp16 NHWC */
   void *out;       /* fp16 [n*P*Q, Kpad] */
 } tacker_be_im2col;
+/* dst[0:bytes) = src[0:bytes); both 16-byte aligned, bytes % 16 == 0; either side may be pinned
+ * host memory (device-accessible through UVA). */
+typedef struct { int64_t bytes; const void *src; void *dst; } tacker_be_copy;
 
 typedef struct {
   int32_t kind;              /* tacker_be_kind */
@@ -171,6 +176,7 @@ typedef struct {
     tacker_be_fma_burn fma_burn;
     tacker_be_im2col im2col;
     tacker_be_cutcp_bin cutcp_bin;
+    tacker_be_copy copy;
     uint8_t _pad[128];
   } p;
 } tacker_be_desc;

@@ -662,6 +662,33 @@ template <> struct BeBody<TACKER_BE_IM2COL> {
   }
 };
 
+// ---------------------------------------------------------------- copy (query I/O)
+// 16 KiB per block, 16-byte vectors, 8 independent loads in flight per thread.
+template <> struct BeBody<TACKER_BE_COPY> {
+  static constexpr uint32_t kSmem = 0;
+  static constexpr int64_t kBlockBytes = 16384;
+  static __host__ __device__ int64_t num_blocks(const tacker_be_copy &p) {
+    return (p.bytes + kBlockBytes - 1) / kBlockBytes;
+  }
+  static __device__ __forceinline__ void run(const tacker_be_copy &p, int64_t vb, int tid, uint32_t, uint8_t *) {
+    const uint4 *src = reinterpret_cast<const uint4 *>(p.src);
+    uint4 *dst = reinterpret_cast<uint4 *>(p.dst);
+    const int64_t n16 = p.bytes / 16;
+    const int64_t base = vb * (kBlockBytes / 16);
+    uint4 v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int64_t i = base + u * 128 + tid;
+      if (i < n16) v[u] = src[i];
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int64_t i = base + u * 128 + tid;
+      if (i < n16) dst[i] = v[u];
+    }
+  }
+};
+
 // ---------------------------------------------------------------- dispatch helpers
 template <int KIND> struct BeSel;
 #define TK_BE_SEL(K, FIELD)                                                            \
@@ -681,6 +708,7 @@ TK_BE_SEL(TACKER_BE_FMA_BURN, fma_burn)
 TK_BE_SEL(TACKER_BE_IM2COL, im2col)
 TK_BE_SEL(TACKER_BE_CUTCP, cutcp)
 TK_BE_SEL(TACKER_BE_CUTCP_BIN, cutcp_bin)
+TK_BE_SEL(TACKER_BE_COPY, copy)
 #undef TK_BE_SEL
 
 // Maximum BE warps per fused CTA: register-heavy bodies (sgemm's 8x4 register tile) keep the
@@ -713,6 +741,7 @@ __device__ __forceinline__ void be_init(uint8_t *, int, uint32_t) {}
 #define TK_FOR_EACH_BE(X)                                                                       \
   X(TACKER_BE_SGEMM) X(TACKER_BE_STENCIL) X(TACKER_BE_MRIQ_PHIMAG) X(TACKER_BE_MRIQ_Q)          \
   X(TACKER_BE_LBM) X(TACKER_BE_SPMV_JDS) X(TACKER_BE_HISTO) X(TACKER_BE_BFS_EXPAND)             \
-  X(TACKER_BE_BFS_COMMIT) X(TACKER_BE_FMA_BURN) X(TACKER_BE_IM2COL) X(TACKER_BE_CUTCP) X(TACKER_BE_CUTCP_BIN)
+  X(TACKER_BE_BFS_COMMIT) X(TACKER_BE_FMA_BURN) X(TACKER_BE_IM2COL) X(TACKER_BE_CUTCP) X(TACKER_BE_CUTCP_BIN)        \
+  X(TACKER_BE_COPY)
 
 }  // namespace tk

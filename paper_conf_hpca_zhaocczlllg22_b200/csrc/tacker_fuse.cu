@@ -57,7 +57,7 @@ int sm_count() {
 const char *be_kind_name(int kind) {
   static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
                                 "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn",
-                                "im2col", "cutcp_bin"};
+                                "im2col", "cutcp_bin", "copy"};
   return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
 }
 
@@ -152,6 +152,13 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
       if (p.natoms < 0 || p.bdim_x <= 0 || p.bdim_y <= 0 || p.bdim_z <= 0 || p.bin_depth <= 0 || !(p.bin_size > 0) ||
           !p.bins || !p.count || !p.overflow || (p.natoms > 0 && !p.atoms))
         return set_error("cutcp_bin: bad args"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_COPY: {
+      const auto &p = d.p.copy;
+      if (p.bytes < 0 || (p.bytes && (!p.src || !p.dst)) || (p.bytes & 15) ||
+          ((reinterpret_cast<uintptr_t>(p.src) | reinterpret_cast<uintptr_t>(p.dst)) & 15))
+        return set_error("copy: 16-byte aligned pointers and sizes required"), TACKER_EINVAL;
       break;
     }
     case TACKER_BE_IM2COL: {

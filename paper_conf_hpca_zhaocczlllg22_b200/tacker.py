@@ -26,7 +26,7 @@ LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
 EPI_BIAS, EPI_RELU, EPI_RESIDUAL = 1, 2, 4
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
- BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN) = range(14)
+ BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY) = range(15)
 POLICY_TACKER, POLICY_BAYMAX = 0, 1
 DEC_FUSED, DEC_ORIGINAL_LC, DEC_REORDER_BE, DEC_IDLE_BE, DEC_NOTHING = range(5)
 MAX_APPS = 64
@@ -124,11 +124,15 @@ class BeCutcpBin(C.Structure):
                 ("count", C.c_void_p), ("overflow", C.c_void_p)]
 
 
+class BeCopy(C.Structure):
+    _fields_ = [("bytes", C.c_int64), ("src", C.c_void_p), ("dst", C.c_void_p)]
+
+
 class _BeUnion(C.Union):
     _fields_ = [("sgemm", BeSgemm), ("stencil", BeStencil), ("mriq_phimag", BeMriqPhimag), ("mriq_q", BeMriqQ),
                 ("cutcp", BeCutcp), ("lbm", BeLbm), ("spmv", BeSpmv), ("histo", BeHisto),
                 ("bfs_expand", BeBfsExpand), ("bfs_commit", BeBfsCommit), ("fma_burn", BeFmaBurn),
-                ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("_pad", C.c_uint8 * 128)]
+                ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("copy", BeCopy), ("_pad", C.c_uint8 * 128)]
 
 
 class BeDesc(C.Structure):
@@ -340,6 +344,14 @@ def be_im2col(x, out, r, s, stride, pad, Kpad=None, orig_blocks=0) -> BeDesc:
     n, h, w, c = x.shape
     d = BeDesc(kind=BE_IM2COL, orig_blocks=orig_blocks)
     d.p.im2col = BeIm2col(n, h, w, c, r, s, stride, pad, out.shape[1] if Kpad is None else Kpad, _ptr(x), _ptr(out))
+    return d
+
+
+def be_copy(src, dst, nbytes=None, orig_blocks=0) -> BeDesc:
+    """dst <- src (either may be pinned host memory: the kernel reads/writes it through UVA)."""
+    n = nbytes if nbytes is not None else src.numel() * src.element_size()
+    d = BeDesc(kind=BE_COPY, orig_blocks=orig_blocks)
+    d.p.copy = BeCopy(n, _ptr(src), _ptr(dst))
     return d
 
 
