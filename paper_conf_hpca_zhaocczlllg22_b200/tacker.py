@@ -13,7 +13,7 @@ import math
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtacker.so")
+LIB_PATH = os.environ.get("TACKER_LIB") or os.path.join(_HERE, "libtacker.so")   # TACKER_LIB: tuning variants
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libtacker.so not built at {LIB_PATH}; run `python -m paper_conf_hpca_zhaocczlllg22_b200.build`")

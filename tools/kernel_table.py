@@ -1,5 +1,6 @@
-"""Per-kernel diagnostic: original LC / original BE / fused durations for the bench workload's
-pairs (CUDA events, L2 flushed before each measurement).  Prints one JSON object."""
+"""Per-kernel diagnostic: original LC / original BE / fused durations for the bench's fused-step
+pairs (CUDA events, L2 flushed before each measurement).  Prints a table and one JSON line.
+Usage: python tools/kernel_table.py [warp_split]"""
 import json
 import os
 import statistics
@@ -11,6 +12,7 @@ sys.path.insert(0, ROOT)
 import torch  # noqa: E402
 
 import bench  # noqa: E402
+from paper_conf_hpca_zhaocczlllg22_b200 import services as sv, tacker as tk  # noqa: E402
 
 
 def timeit(fn, reps=5, flush=None):
@@ -29,13 +31,15 @@ def timeit(fn, reps=5, flush=None):
 
 
 def main():
-    ws = int(sys.argv[1]) if len(sys.argv) > 1 else 16
-    wl = bench.Workload(warp_split=ws)
-    tk = wl.tk
+    ws = int(sys.argv[1]) if len(sys.argv) > 1 else 24
+    svc = sv.resnet50_service(1, 2022)
+    stencil, mriq = sv.stencil_app(), sv.mriq_app()
+    tk.tacker_launch_original(None, mriq.kernels[0].desc)
+    step = bench.FusedStep(svc, stencil, mriq, ws)
     buf = torch.empty(64 * 1024 * 1024, device="cuda")
     flush = lambda: buf.fill_(1.0)
     rows = []
-    for k, be, f in wl.plan:
+    for k, be, f in step.plan:
         if f is None:
             continue
         t_lc = timeit(lambda: tk.tacker_launch_original(k.lc, None), flush=flush)
@@ -44,11 +48,11 @@ def main():
         i = f.info()
         rows.append(dict(lc=k.name, be=be.name, t_lc=t_lc, t_be=t_be, t_fused=t_f, seq=t_lc + t_be,
                          gain=(t_lc + t_be) / t_f, tiles=i.lc_tiles, bn=i.lc_tile_n, stages=i.lc_stages,
-                         regs=i.regs_per_thread, smem=i.smem_bytes))
+                         regs=i.regs_per_thread, smem=i.smem_bytes, be_warps=i.be_warps))
     for r in rows:
         print(f"{r['lc']:28s} {r['be']:14s} lc {r['t_lc']*1e3:7.1f}us be {r['t_be']*1e3:7.1f}us "
               f"fused {r['t_fused']*1e3:7.1f}us seq/fused {r['gain']:.2f} tiles {r['tiles']} bn {r['bn']} "
-              f"st {r['stages']} regs {r['regs']}")
+              f"st {r['stages']} regs {r['regs']} bew {r['be_warps']}")
     print(json.dumps({"warp_split": ws, "rows": rows}))
 
 
