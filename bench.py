@@ -47,16 +47,26 @@ WORKLOAD = "resnet50_b1 LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[
 
 
 # ----------------------------------------------------------------------------- helpers
-def dist_setup():
+_BACKEND = "nccl"
+
+
+def dist_setup(simulate=False):
+    """One process per GPU (replicas: no data-path collective).  The process group only carries
+    the barrier and the max/sum reductions of the timing; --simulate uses gloo on CPU."""
+    global _BACKEND
     import torch
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    _BACKEND = "gloo" if simulate else "nccl"
     if ws > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    elif torch.cuda.is_available():
+        if simulate:
+            dist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif not simulate and torch.cuda.is_available():
         torch.cuda.set_device(0)
     return ws, rank, local
 
@@ -72,7 +82,7 @@ def reduce_ranks(ws, v, op="max"):
         return v
     import torch
     import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    t = torch.tensor([v], dtype=torch.float64, device="cpu" if _BACKEND == "gloo" else "cuda")
     dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
     return float(t.item())
 
@@ -424,6 +434,52 @@ def run_tacker(args, ws, rank, local):
         print(json.dumps(line))
 
 
+def run_simulated(args, ws, rank):
+    """--simulate: the same managed run on the manager's simulated GPU (kernels take their
+    predicted time; no CUDA), for CPU tests of the multi-rank path (gloo).  Kernel durations are
+    a fixed table shaped like the B200 measurements of the ResNet-50 b1 / stencil / mri-q run."""
+    from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
+    tk.tacker_model_clear()
+    fake = 0x10000
+    lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=1024, N=256, K=256, A=fake, B=fake, D=fake)
+    ks = [tk.LcKernel(is_tc=1, t_pred_ms=0.010 + 0.0005 * (i % 7), lc=lc) for i in range(53)]
+    st = tk.BeDesc(kind=tk.BE_STENCIL)
+    st.p.stencil = tk.BeStencil(512, 512, 64, 1 / 6, 1 / 36, fake, fake)
+    key = f"pair:lc:gemm:N256:K256:bn128:f32|be:stencil:nz64|ws{args.warp_split}"
+    for r in (0.1, 0.2, 1.8, 1.9):      # tau(r) = max(1 + 0.3 r, 0.45 + 0.95 r)
+        tk.tacker_pair_add_sample(key, 1.0, r, max(1 + 0.3 * r, 0.45 + 0.95 * r))
+    tk.tacker_pair_fit(key)
+    apps = [[tk.BeKernel(is_cd=1, t_pred_ms=0.035, be=st, warp_split=args.warp_split)] * 2,
+            [tk.BeKernel(is_cd=1, t_pred_ms=0.147, be=st, warp_split=args.warp_split)] * 2]
+    rng = np.random.default_rng(2000 + rank)
+    solo = sum(k.t_pred_ms for k in ks)
+    gaps = rng.exponential(solo / LOAD, args.steps)
+    out = {}
+    for pol in (tk.POLICY_BAYMAX, tk.POLICY_TACKER):
+        m = tk.Manager(pol, simulate=True, idle_cap_ms=0.5 * (QOS_MS - solo))
+        for a in apps:
+            m.submit_be(a)
+        arr = np.cumsum(gaps)
+        q = [m.submit_lc(ks, float(t)) for t in arr]
+        barrier(ws)
+        m.run(QOS_MS, float(arr[-1]))
+        s = m.stats()
+        lat = np.sort([m.latency(i) for i in q])
+        out[pol] = (s.be_kernels_done, s.now_ms, float(lat[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)]))
+    be, el, p99 = out[tk.POLICY_TACKER]
+    elapsed = reduce_ranks(ws, el, "max")
+    value = reduce_ranks(ws, be, "sum") / (elapsed / 1e3)
+    bay = reduce_ranks(ws, out[tk.POLICY_BAYMAX][0], "sum") / (reduce_ranks(ws, out[tk.POLICY_BAYMAX][1], "max") / 1e3)
+    line = {"metric": METRIC, "value": value, "unit": "BE kernels/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": elapsed / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "n/a (simulated GPU)", "data": "synthetic",
+            "config": {"workload": WORKLOAD + " [simulated durations]", "parallelism": f"replicas x{ws}"},
+            "lc_p99_ms": reduce_ranks(ws, p99, "max"), "baymax": {"value": bay},
+            "improvement_vs_baymax_eq10": value / bay - 1.0, "simulated": True}
+    if rank == 0:
+        print(json.dumps(line))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -432,12 +488,16 @@ def main():
     ap.add_argument("--impl", default="tacker", choices=["tacker", "reference"])
     ap.add_argument("--warp-split", type=int, default=24)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--simulate", action="store_true", help="CPU-only: manager on its simulated GPU (gloo)")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args, int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")))
         return
-    ws, rank, local = dist_setup()
-    run_tacker(args, ws, rank, local)
+    ws, rank, local = dist_setup(simulate=args.simulate)
+    if args.simulate:
+        run_simulated(args, ws, rank)
+    else:
+        run_tacker(args, ws, rank, local)
     if ws > 1:
         import torch.distributed as dist
         dist.destroy_process_group()

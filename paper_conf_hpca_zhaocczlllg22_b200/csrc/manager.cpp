@@ -476,12 +476,10 @@ tacker_status tacker_manager_run(tacker_manager_t m, double qos, double t_end_ms
     tacker_status s = tacker_manager_step(m, qos, &thr, &d);
     if (s) return s;
     if (d.action != TACKER_DEC_NOTHING && max_decisions > 0 && ++n >= max_decisions) break;
-    if (d.action == TACKER_DEC_NOTHING) {
-      poll(m);
-      const bool all_done = m->st.lc_queries_done == (int64_t)m->queries.size();
-      if (all_done && m->now >= t_end_ms) break;
-      if (m->sim() && all_done && m->next_pending >= m->pending.size()) break;
-    }
+    poll(m);
+    const bool all_done = m->st.lc_queries_done == (int64_t)m->queries.size();
+    if (all_done && m->now >= t_end_ms) break;
+    if (m->sim() && all_done && m->next_pending >= m->pending.size()) break;
   }
   if (!m->sim()) {
     cudaError_t e = cudaStreamSynchronize(m->stream);
