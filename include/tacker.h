@@ -107,7 +107,13 @@ typedef enum {
   TACKER_BE_CUTCP_BIN = 13,   /* cutcp atom binning (deterministic, index order); block = 128 bins */
   TACKER_BE_COPY = 14,        /* byte copy, e.g. a query's H2D/D2H through host-mapped pinned
                                  memory (UVA); block = 16 KiB */
-  TACKER_BE_KIND_COUNT = 15
+  /* CSR -> JDS (spmv's input format) as a stable counting sort by row length, descending,
+   * ties by row index: four kernels run in this order (all deterministic, integer-exact). */
+  TACKER_BE_JDS_COUNT = 15,   /* per 1024-row block: row-length counts; block = 1024 rows */
+  TACKER_BE_JDS_SCAN = 16,    /* prefix over blocks per length, start offsets, jds_ptr; 1 block */
+  TACKER_BE_JDS_PERM = 17,    /* perm / row_len placement; block = 1024 rows */
+  TACKER_BE_JDS_FILL = 18,    /* column / value scatter, diagonal-major; block = 128 JDS rows */
+  TACKER_BE_KIND_COUNT = 19
 } tacker_be_kind;
 
 typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
@@ -158,6 +164,21 @@ typedef struct {
 /* dst[0:bytes) = src[0:bytes); both 16-byte aligned, bytes % 16 == 0; either side may be pinned
  * host memory (device-accessible through UVA). */
 typedef struct { int64_t bytes; const void *src; void *dst; } tacker_be_copy;
+/* JDS build (one struct for the four kinds).  Outputs follow oracle/be.py jds_build: perm[i] =
+ * i-th row by (length desc, index asc); row_len[i] = its length; jds_ptr[d] = start of jagged
+ * diagonal d (jds_ptr[0] = 0, jds_ptr[d+1]-jds_ptr[d] = #rows longer than d), sized max_len+1;
+ * element (d, i) of the JDS arrays is the d-th nonzero of row perm[i].  *overflow = 1 if a row
+ * is longer than max_len (outputs then invalid). */
+typedef struct {
+  int32_t rows, max_len;
+  const int32_t *row_ptr, *col;   /* CSR input, columns sorted within a row */
+  const float *val;
+  int32_t *blk_count;             /* workspace [ceil(rows/1024)][max_len+1] */
+  int32_t *start;                 /* workspace [max_len+2] */
+  int32_t *perm, *row_len, *jds_ptr, *jds_col;
+  float *jds_val;
+  int32_t *overflow;
+} tacker_be_jds;
 
 typedef struct {
   int32_t kind;              /* tacker_be_kind */
@@ -177,6 +198,7 @@ typedef struct {
     tacker_be_im2col im2col;
     tacker_be_cutcp_bin cutcp_bin;
     tacker_be_copy copy;
+    tacker_be_jds jds;
     uint8_t _pad[128];
   } p;
 } tacker_be_desc;

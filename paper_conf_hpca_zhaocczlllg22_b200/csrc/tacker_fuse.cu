@@ -57,7 +57,7 @@ int sm_count() {
 const char *be_kind_name(int kind) {
   static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
                                 "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn",
-                                "im2col", "cutcp_bin", "copy"};
+                                "im2col", "cutcp_bin", "copy", "jds_count", "jds_scan", "jds_perm", "jds_fill"};
   return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
 }
 
@@ -152,6 +152,17 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
       if (p.natoms < 0 || p.bdim_x <= 0 || p.bdim_y <= 0 || p.bdim_z <= 0 || p.bin_depth <= 0 || !(p.bin_size > 0) ||
           !p.bins || !p.count || !p.overflow || (p.natoms > 0 && !p.atoms))
         return set_error("cutcp_bin: bad args"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_JDS_COUNT:
+    case TACKER_BE_JDS_SCAN:
+    case TACKER_BE_JDS_PERM:
+    case TACKER_BE_JDS_FILL: {
+      const auto &p = d.p.jds;
+      if (p.rows < 0 || p.max_len < 1 || p.max_len > kJdsMaxLen || !p.row_ptr || !p.blk_count || !p.start ||
+          !p.perm || !p.row_len || !p.jds_ptr || !p.overflow || (d.kind == TACKER_BE_JDS_FILL && (!p.col || !p.val ||
+                                                                                          !p.jds_col || !p.jds_val)))
+        return set_error("jds: bad args (max_len in [1, %d])", kJdsMaxLen), TACKER_EINVAL;
       break;
     }
     case TACKER_BE_COPY: {

@@ -82,7 +82,7 @@ class QosRun:
                 continue
             for a, app in enumerate(self.apps):
                 for j, bk in enumerate(app.kernels):
-                    if bk.name.endswith("phimag"):
+                    if self.t_be[(a, j)] < 0.01:   # < 10 us (phiMag, binning, bfs levels): reorder only
                         continue
                     f = None
                     for ws in range(self.ws, 3, -4):
@@ -90,7 +90,7 @@ class QosRun:
                             f = tk.tacker_fuse(k.lc, bk.desc, ws)
                             break
                         except tk.TackerError as e:
-                            if e.status != tk.ERESOURCE:
+                            if e.status not in (tk.ERESOURCE, tk.EUNSUPPORTED):   # budget / per-kind warp cap
                                 raise
                     if f is None:
                         continue

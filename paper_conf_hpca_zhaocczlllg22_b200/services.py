@@ -155,6 +155,72 @@ def mriq_app(N=64, numK=2048, chunk=1024, seed=2022) -> BeAppSpec:
     return BeAppSpec(f"mriq_{N}^3x{numK}", ks, [dd, phimag, Qr, Qi])
 
 
+def lbm_app(nx=120, ny=120, nz=150, seed=2022) -> BeAppSpec:
+    """Parboil lbm: ping-pong stream-collide steps (one kernel = one step)."""
+    f, fl = synth.lbm_inputs(nx, ny, nz, seed)
+    a, flags = _dev(f), _dev(fl.astype(np.uint32).view(np.int32))
+    b = a.clone()
+    cells = nx * ny * nz
+    ks = [BeKernelSpec("lbm.even", tk.be_lbm(a, b, flags), flops=210.0 * cells, bytes=156.0 * cells),
+          BeKernelSpec("lbm.odd", tk.be_lbm(b, a, flags), flops=210.0 * cells, bytes=156.0 * cells)]
+    return BeAppSpec(f"lbm_{nx}x{ny}x{nz}", ks, [a, b, flags])
+
+
+def cutcp_app(L=48.0, seed=2022, depth=32) -> BeAppSpec:
+    """Parboil cutcp: binning (once per app iteration) + the potential kernel."""
+    d = synth.cutcp_inputs(L, seed)
+    nx = d["nx"]
+    bd = tk.cutcp_bin_dims(nx, nx, nx)
+    atoms = _dev(d["atoms"])
+    nb = bd[0] * bd[1] * bd[2]
+    bins = torch.zeros(nb * depth * 4, device="cuda")
+    cnt = torch.zeros(nb, dtype=torch.int32, device="cuda")
+    ovf = torch.zeros(1, dtype=torch.int32, device="cuda")
+    V = torch.zeros(nx ** 3, device="cuda")
+    ks = [BeKernelSpec("cutcp.bin", tk.be_cutcp_bin(atoms, bins, cnt, ovf, nx, nx, nx, float(d["h"]), depth),
+                       bytes=16.0 * atoms.shape[0] * 2),
+          BeKernelSpec("cutcp.potential", tk.be_cutcp(bins, cnt, V, nx, nx, nx, float(d["h"]), depth),
+                       bytes=4.0 * nx ** 3, bound="fma")]
+    return BeAppSpec(f"cutcp_{L:g}A", ks, [atoms, bins, cnt, ovf, V])
+
+
+def spmv_app(R=1 << 20, seed=2022) -> BeAppSpec:
+    """Parboil spmv: the CSR input is converted to JDS on the GPU once (the four JDS kernels),
+    then the app cycles the JDS spmv kernel."""
+    rp, cols, vals, x = synth.spmv_inputs(R, seed)
+    csr = [_dev(rp), _dev(cols), _dev(vals)]
+    jb = tk.JdsBuffers(*csr, max_len=1023).build()
+    dx = _dev(x)
+    y = torch.zeros(R, device="cuda")
+    nnz = int(rp[-1])
+    desc = tk.be_spmv(jb.perm, jb.row_len, jb.jds_ptr, jb.jds_col, jb.jds_val, dx, y)
+    return BeAppSpec(f"spmv_{R}", [BeKernelSpec("spmv", desc, flops=2.0 * nnz, bytes=8.0 * nnz + 16.0 * R)],
+                     csr + [jb, dx, y])
+
+
+def histo_app(N=1 << 26, nbins=4096, seed=2022) -> BeAppSpec:
+    v = synth.histo_inputs(N, nbins, seed, "skewed")
+    dv = _dev(v.view(np.int32))
+    cnt = torch.zeros(nbins, dtype=torch.int32, device="cuda")
+    return BeAppSpec(f"histo_{N}", [BeKernelSpec("histo", tk.be_histo(dv, cnt, nbins), bytes=4.0 * N)], [dv, cnt])
+
+
+def bfs_app(V=1 << 20, seed=2022) -> BeAppSpec:
+    """Rodinia bfs level step (expand + commit), cycled over a fixed number of levels."""
+    rp, col = synth.bfs_inputs(V, seed)
+    drp, dcol = _dev(rp), _dev(col)
+    level = torch.full((V,), -1, dtype=torch.int32, device="cuda")
+    level[0] = 0
+    mask = torch.zeros(V, dtype=torch.uint8, device="cuda")
+    mask[0] = 1
+    visited = mask.clone()
+    upd = torch.zeros_like(mask)
+    over = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ks = [BeKernelSpec("bfs.expand", tk.be_bfs_expand(drp, dcol, level, mask, visited, upd), bytes=8.0 * V),
+          BeKernelSpec("bfs.commit", tk.be_bfs_commit(mask, visited, upd, over), bytes=3.0 * V)]
+    return BeAppSpec(f"bfs_{V}", ks, [drp, dcol, level, mask, visited, upd, over])
+
+
 def sgemm_app(M=2048, N=2048, K=2048, seed=2022) -> BeAppSpec:
     A, B = synth.sgemm_inputs(M, N, K, seed)
     dA, dB = _dev(A), _dev(B)

@@ -26,7 +26,8 @@ LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
 EPI_BIAS, EPI_RELU, EPI_RESIDUAL = 1, 2, 4
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
- BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY) = range(15)
+ BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY, BE_JDS_COUNT, BE_JDS_SCAN,
+ BE_JDS_PERM, BE_JDS_FILL) = range(19)
 POLICY_TACKER, POLICY_BAYMAX = 0, 1
 DEC_FUSED, DEC_ORIGINAL_LC, DEC_REORDER_BE, DEC_IDLE_BE, DEC_NOTHING = range(5)
 MAX_APPS = 64
@@ -128,11 +129,19 @@ class BeCopy(C.Structure):
     _fields_ = [("bytes", C.c_int64), ("src", C.c_void_p), ("dst", C.c_void_p)]
 
 
+class BeJds(C.Structure):
+    _fields_ = [("rows", C.c_int32), ("max_len", C.c_int32), ("row_ptr", C.c_void_p), ("col", C.c_void_p),
+                ("val", C.c_void_p), ("blk_count", C.c_void_p), ("start", C.c_void_p), ("perm", C.c_void_p),
+                ("row_len", C.c_void_p), ("jds_ptr", C.c_void_p), ("jds_col", C.c_void_p), ("jds_val", C.c_void_p),
+                ("overflow", C.c_void_p)]
+
+
 class _BeUnion(C.Union):
     _fields_ = [("sgemm", BeSgemm), ("stencil", BeStencil), ("mriq_phimag", BeMriqPhimag), ("mriq_q", BeMriqQ),
                 ("cutcp", BeCutcp), ("lbm", BeLbm), ("spmv", BeSpmv), ("histo", BeHisto),
                 ("bfs_expand", BeBfsExpand), ("bfs_commit", BeBfsCommit), ("fma_burn", BeFmaBurn),
-                ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("copy", BeCopy), ("_pad", C.c_uint8 * 128)]
+                ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("copy", BeCopy), ("jds", BeJds),
+                ("_pad", C.c_uint8 * 128)]
 
 
 class BeDesc(C.Structure):
@@ -353,6 +362,43 @@ def be_copy(src, dst, nbytes=None, orig_blocks=0) -> BeDesc:
     d = BeDesc(kind=BE_COPY, orig_blocks=orig_blocks)
     d.p.copy = BeCopy(n, _ptr(src), _ptr(dst))
     return d
+
+
+class JdsBuffers:
+    """Device buffers of a CSR -> JDS build (outputs + workspace); `descs()` returns the four
+    BE kernel descriptors (COUNT, SCAN, PERM, FILL) to launch in order."""
+
+    def __init__(self, row_ptr, col, val, max_len=1023):
+        import torch
+        rows = row_ptr.numel() - 1
+        nnz = col.numel()
+        dev = row_ptr.device
+        i32 = dict(dtype=torch.int32, device=dev)
+        self.src = (row_ptr, col, val)
+        self.rows, self.max_len = rows, max_len
+        self.blk_count = torch.zeros(((rows + 1023) // 1024) * (max_len + 1), **i32)
+        self.start = torch.zeros(max_len + 2, **i32)
+        self.perm = torch.zeros(max(rows, 1), **i32)
+        self.row_len = torch.zeros(max(rows, 1), **i32)
+        self.jds_ptr = torch.zeros(max_len + 1, **i32)
+        self.jds_col = torch.zeros(max(nnz, 1), **i32)
+        self.jds_val = torch.zeros(max(nnz, 1), dtype=torch.float32, device=dev)
+        self.overflow = torch.zeros(1, **i32)
+
+    def descs(self):
+        out = []
+        for kind in (BE_JDS_COUNT, BE_JDS_SCAN, BE_JDS_PERM, BE_JDS_FILL):
+            d = BeDesc(kind=kind)
+            d.p.jds = BeJds(self.rows, self.max_len, _ptr(self.src[0]), _ptr(self.src[1]), _ptr(self.src[2]),
+                            _ptr(self.blk_count), _ptr(self.start), _ptr(self.perm), _ptr(self.row_len),
+                            _ptr(self.jds_ptr), _ptr(self.jds_col), _ptr(self.jds_val), _ptr(self.overflow))
+            out.append(d)
+        return out
+
+    def build(self, stream=None):
+        for d in self.descs():
+            tacker_launch_original(None, d, stream)
+        return self
 
 
 def cutcp_bin_dims(nx, ny, nz):

@@ -62,28 +62,15 @@ def be_kernels():
     src, flags = dev(f), dev(fl.astype(np.uint32).view(np.int32))
     dst = torch.zeros_like(src)
     out["lbm"] = (lambda n=0: tk.be_lbm(src, dst, flags, orig_blocks=n), [src, dst, flags])
-    # spmv 2^20 rows: JDS arrays built from the generator's CSR with a host counting sort (input
-    # layout preparation, like Parboil's driver; GPU jds_build is future work)
+    # spmv 2^20 rows: JDS built on the GPU (TACKER_BE_JDS_* kernels)
     R = 1 << 20
     rp, cols, vals, x = synth.spmv_inputs(R, 2022)
-    lens = np.diff(rp)
-    perm = np.lexsort((np.arange(R), -lens)).astype(np.int32)
-    rl = lens[perm].astype(np.int32)
-    maxlen = int(rl[0])
-    cnt_d = np.array([(lens > dd).sum() for dd in range(maxlen)], np.int64)
-    jptr = np.zeros(maxlen + 1, np.int64)
-    jptr[1:] = np.cumsum(cnt_d)
-    nnz = int(jptr[-1])
-    jc = np.zeros(nnz, np.int32)
-    jv = np.zeros(nnz, np.float32)
-    starts = rp[perm]
-    for dd in range(maxlen):
-        m = int(cnt_d[dd])
-        jc[jptr[dd]:jptr[dd] + m] = cols[starts[:m] + dd]
-        jv[jptr[dd]:jptr[dd] + m] = vals[starts[:m] + dd]
-    ds = [dev(a) for a in (perm, rl, jptr.astype(np.int32), jc, jv, x)]
+    csr = [dev(rp), dev(cols), dev(vals)]
+    jb = tk.JdsBuffers(*csr, max_len=1023).build()
+    dx = dev(x)
     y = torch.zeros(R, device="cuda")
-    out["spmv"] = (lambda n=0: tk.be_spmv(*ds, y, orig_blocks=n), ds + [y])
+    out["spmv"] = (lambda n=0: tk.be_spmv(jb.perm, jb.row_len, jb.jds_ptr, jb.jds_col, jb.jds_val, dx, y,
+                                          orig_blocks=n), csr + [jb, dx, y])
     return out
 
 

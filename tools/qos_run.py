@@ -26,6 +26,16 @@ def build_apps(names):
             apps.append(sv.mriq_app(64, 2048, 1024))
         elif n == "sgemm":
             apps.append(sv.sgemm_app(2048, 2048, 2048))
+        elif n == "lbm":
+            apps.append(sv.lbm_app())
+        elif n == "cutcp":
+            apps.append(sv.cutcp_app())
+        elif n == "spmv":
+            apps.append(sv.spmv_app())
+        elif n == "histo":
+            apps.append(sv.histo_app())
+        elif n == "bfs":
+            apps.append(sv.bfs_app())
         else:
             raise ValueError(n)
     return apps
