@@ -22,7 +22,7 @@ constexpr int kVbThreads = 128;
 #define TK_STENCIL_ZC 4
 #endif
 #ifndef TK_MRIQ_COARSEN
-#define TK_MRIQ_COARSEN 3
+#define TK_MRIQ_COARSEN 4
 #endif
 #ifndef TK_MRIQ_REDUCE
 #define TK_MRIQ_REDUCE 0
@@ -265,8 +265,8 @@ template <> struct BeBody<TACKER_BE_MRIQ_PHIMAG> {
 // only runs the two MUFU ops) before the MUFU sin/cos of 2*pi*t.
 template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   static constexpr int KC = 512;
-  // original blocks one fused virtual block runs at once: 3 balances 2048 blocks (64^3 voxels)
-  // over 148 CTAs x 6 slots better than 4 (683 units: max 5 vs mean 4.6 per CTA)
+  // original blocks one fused virtual block runs at once (measured sweep 2/3/4/6 on the bench
+  // grid: 4 is fastest; per-thread MUFU ILP outweighs the 86 % unit balance of 512 units)
   static constexpr int kCoarsen = TK_MRIQ_COARSEN;
   static constexpr uint32_t kSmem = KC * 16;
   static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) { return (p.numX + 127) / 128; }
