@@ -452,7 +452,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.warp_split = warp_split;
   F.block = 32 * warps;
   F.smem = 1024 + F.P.lc_smem_bytes + be_total;
-  if (F.smem < kMinLcSmem) F.smem = kMinLcSmem;
+  // An LC-only CTA (6 warps) could otherwise share an SM with a second one (both allocating
+  // TMEM); a fused CTA is already alone on its SM through its registers (>= 16 warps x 64
+  // regs... a second CTA would exceed 64K), so it keeps the unused shared memory as L1.
+  if (!has_be && F.smem < kMinLcSmem) F.smem = kMinLcSmem;
   F.grid = has_be ? sms : (L.num_tiles < sms ? L.num_tiles : sms);
   if (F.grid < 1) F.grid = 1;
   F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
