@@ -1,0 +1,23 @@
+// be_common.cuh — shared definitions of the BE bodies (see be_bodies.cuh).
+#pragma once
+#include <cuda_fp16.h>
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "tacker.h"
+
+namespace tk {
+constexpr int kVbThreads = 128;
+#ifndef TK_STENCIL_ZC
+#define TK_STENCIL_ZC 4
+#endif
+#ifndef TK_MRIQ_COARSEN
+#define TK_MRIQ_COARSEN 4
+#endif
+#ifndef TK_MRIQ_REDUCE
+#define TK_MRIQ_REDUCE 0
+#endif
+
+template <int KIND> struct BeBody;
+
+}  // namespace tk
