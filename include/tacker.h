@@ -352,10 +352,21 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos_target_ms, doub
  * t_end_ms and every submitted query has completed, or max_decisions decisions were taken
  * (<= 0: unbounded).  The host thread spins between decisions (no Python in the loop). */
 tacker_status tacker_manager_run(tacker_manager_t m, double qos_target_ms, double t_end_ms, int64_t max_decisions);
+enum { TACKER_CLASS_LC_TC = 0, TACKER_CLASS_LC_CD = 1, TACKER_CLASS_FUSED = 2, TACKER_CLASS_BE = 3 };
 typedef struct {
   int64_t lc_queries_done, be_kernels_done, fused_launches, original_lc, reordered_be, idle_be;
   double now_ms;
   int64_t model_refits;      /* GPU mode: two-stage refits triggered by measured fused runs */
+  /* GPU mode: device time per launch class (LC tensor-core original, LC CUDA-core original,
+   * fused, BE original).  class_launches counts every launch; class_ms is estimated from CUDA
+   * events (manager stream) around one launch in 8 of each class (every fused launch), scaled
+   * to the count. */
+  double class_ms[4];
+  int64_t class_launches[4];
+  /* GPU mode: sum of |predicted - measured| / measured of the fused duration over pred_err_n
+   * timed fused launches (the pair model as it stood when the manager decided) */
+  double pred_err_sum;
+  int64_t pred_err_n;
 } tacker_manager_stats;
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
 /* Completion time (manager clock) of a finished query, or -1 if unfinished. */

@@ -27,8 +27,8 @@ template <> struct BeBody<TACKER_BE_MRIQ_PHIMAG> {
 // only runs the two MUFU ops) before the MUFU sin/cos of 2*pi*t.
 template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   static constexpr int KC = 512;
-  // original blocks one fused virtual block runs at once (measured sweep 2/3/4/6 on the bench
-  // grid: 4 is fastest; per-thread MUFU ILP outweighs the 86 % unit balance of 512 units)
+  // at most this many original blocks per fused virtual block at once (independent MUFU chains
+  // per thread; the fused PTB loop gives every CTA an even share, see be_ptb_loop)
   static constexpr int kCoarsen = TK_MRIQ_COARSEN;
   static constexpr uint32_t kSmem = KC * 16;
   static __host__ __device__ int64_t num_blocks(const tacker_be_mriq_q &p) { return (p.numX + 127) / 128; }
@@ -42,7 +42,12 @@ template <> struct BeBody<TACKER_BE_MRIQ_Q> {
   // voxel's k-ordered accumulation is unchanged, so results stay bit-identical.
   static __device__ __forceinline__ void run_coarse(const tacker_be_mriq_q &p, int64_t vb, int nb, int tid,
                                                     uint32_t bar, uint8_t *smem) {
-    run_v<kCoarsen>(p, vb, nb, tid, bar, smem);
+    // exact chain count (a masked voxel would still spend its MUFU slots)
+    static_assert(kCoarsen <= 4, "run_coarse dispatches 1..4 voxels per thread");
+    if (nb >= 4) run_v<4>(p, vb, 4, tid, bar, smem);
+    else if (nb == 3) run_v<3>(p, vb, 3, tid, bar, smem);
+    else if (nb == 2) run_v<2>(p, vb, 2, tid, bar, smem);
+    else run_v<1>(p, vb, 1, tid, bar, smem);
   }
   template <int VPT>
   static __device__ __forceinline__ void run_v(const tacker_be_mriq_q &p, int64_t vb, int nb, int tid, uint32_t bar,

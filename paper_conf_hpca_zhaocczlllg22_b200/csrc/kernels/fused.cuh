@@ -245,9 +245,23 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   // First round static and interleaved across CTAs (slot j of every CTA before slot j+1, so
   // a short BE kernel spreads over all SMs); afterwards dynamic tickets balance the tail.
   constexpr int kC = BeCoarsen<BE_KIND>::value;    // original blocks per ticket
-  const int64_t units = (P.be_blocks + kC - 1) / kC;
-  int64_t vb = (int64_t)j * gridDim.x + blockIdx.x;
+  // LC tiles sit on the lowest CTA indices (tile t on CTA t mod grid): hand them the smaller BE
+  // shares by numbering CTAs from the top.
+  const int64_t cta = (int64_t)gridDim.x - 1 - blockIdx.x;
   be_init<BE_KIND>(body_smem, tid, bar);
+  if constexpr (kC > 1) {
+    // Coarsened (compute-bound, uniform-cost) bodies: static even split.  CTA c owns original
+    // blocks [B c / G, B (c+1) / G), its slot j a contiguous part of that, run kC at a time
+    // with exactly as many per-thread chains as blocks; per-SM work differs by <= 1 block, so
+    // the SMs finish together without a ticket tail.
+    const int64_t lo = P.be_blocks * cta / gridDim.x, hi = P.be_blocks * (cta + 1) / gridDim.x;
+    const int S = P.be_vb_per_cta;
+    for (int64_t b = lo + (hi - lo) * j / S, e = lo + (hi - lo) * (j + 1) / S; b < e; b += kC)
+      be_run_coarse<BE_KIND>(P.be, b, (int)min((int64_t)kC, e - b), tid, bar, body_smem, &P.tmap_be);
+    return;
+  }
+  const int64_t units = (P.be_blocks + kC - 1) / kC;
+  int64_t vb = (int64_t)j * gridDim.x + cta;
   while (vb < units) {
     const int64_t b0 = vb * kC;
     be_run_coarse<BE_KIND>(P.be, b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem, &P.tmap_be);

@@ -83,10 +83,20 @@ struct tacker_manager_s {
   struct Observed {
     cudaEvent_t start, end;
     std::string pair_key;
-    double x_tc, x_cd;
+    double x_tc, x_cd, t_pred;
   };
   std::deque<Observed> observed;   // fused launches awaiting their measured duration
   int64_t refits = 0;
+  double pred_err_sum = 0;         // sum |predicted - measured| / measured over fused launches
+  int64_t pred_err_n = 0;
+  struct Timed {
+    cudaEvent_t start, end;
+    int cls;
+  };
+  std::deque<Timed> timed;         // sampled launches: device time per class
+  double class_ms[4] = {0, 0, 0, 0};   // summed over the timed sample
+  int64_t class_timed[4] = {0, 0, 0, 0};
+  int64_t class_n[4] = {0, 0, 0, 0};   // every launch
 
   bool sim() const { return prm.simulate != 0; }
 };
@@ -140,11 +150,25 @@ static void poll(tacker_manager_s *m) {
       unref(m, a.pending);
       a.pending = nullptr;
     }
+  while (!m->timed.empty() && cudaEventQuery(m->timed.front().end) == cudaSuccess) {
+    auto &t = m->timed.front();
+    float ms = 0;
+    cudaEventElapsedTime(&ms, t.start, t.end);
+    m->class_ms[t.cls] += ms;
+    m->class_timed[t.cls]++;
+    unref(m, t.start);
+    unref(m, t.end);
+    m->timed.pop_front();
+  }
   while (!m->observed.empty() && cudaEventQuery(m->observed.front().end) == cudaSuccess) {
     auto &o = m->observed.front();
     float ms = 0;
     cudaEventElapsedTime(&ms, o.start, o.end);
     int32_t refit = 0;
+    if (ms > 0) {
+      m->pred_err_sum += std::fabs(o.t_pred - ms) / ms;
+      m->pred_err_n++;
+    }
     if (ms > 0 && tacker_pair_observe(o.pair_key.c_str(), o.x_tc, o.x_cd, ms, &refit) == TACKER_OK && refit)
       m->refits++;
     unref(m, o.start);
@@ -162,9 +186,17 @@ static void poll(tacker_manager_s *m) {
   }
 }
 
+// A BE application's head kernel is ready once its predecessor has been issued: in GPU mode the
+// manager's single stream orders an app's kernels, so the next one may be fused or reordered
+// right away (as on the simulator's serial virtual stream, where ready_at is the issue end);
+// the in-flight cap bounds how far the host runs ahead.
 static bool app_ready(tacker_manager_s *m, const App &a, double t) {
   if (m->sim()) return a.ready_at <= t;
-  return a.pending == nullptr;
+  return true;
+}
+static void set_pending(tacker_manager_s *m, App &a, cudaEvent_t e) {
+  if (a.pending) unref(m, a.pending);
+  a.pending = ref(m, e);
 }
 
 static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, double *tf) {
@@ -205,6 +237,23 @@ static cudaEvent_t record(tacker_manager_s *m) {
   cudaEventRecord(e, m->stream);
   m->inflight.push_back(ref(m, e));
   return e;
+}
+// Per-class device time (stats.class_ms): every launch is counted, one launch in kTimeEvery of
+// each class is bracketed by events (a start event costs a host API call per launch, and the
+// manager loop of a 53-kernel query is host-latency sensitive); the class total is the sampled
+// mean x the count.  Fused launches are always timed: the online refit needs each one.
+static constexpr int64_t kTimeEvery = 8;
+// start event of a launch (the stream reaches it when the previous kernel has finished), or
+// nullptr when this launch is not in the timed sample
+static cudaEvent_t begin(tacker_manager_s *m, int cls, bool always = false) {
+  if (!always && m->class_n[cls]++ % kTimeEvery != 0) return nullptr;
+  if (always) m->class_n[cls]++;
+  cudaEvent_t e = get_event(m);
+  cudaEventRecord(e, m->stream);
+  return e;
+}
+static void track(tacker_manager_s *m, cudaEvent_t start, cudaEvent_t end, int cls) {
+  if (start) m->timed.push_back(tacker_manager_s::Timed{ref(m, start), ref(m, end), cls});
 }
 
 extern "C" {
@@ -323,9 +372,11 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
         m->now += b.t_pred_ms;
         A.ready_at = m->now;
       } else {
+        cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
         tacker_status s = launch_be(m, b);
         if (s) return s;
-        A.pending = ref(m, record(m));
+        set_pending(m, A, record(m));
+        track(m, e0, A.pending, TACKER_CLASS_BE);
       }
       A.pos++;
       A.completed++;
@@ -412,17 +463,17 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       m->now += best_tf;
       A.ready_at = m->now;
     } else {
-      cudaEvent_t e0 = get_event(m);
-      cudaEventRecord(e0, m->stream);
+      cudaEvent_t e0 = begin(m, TACKER_CLASS_FUSED, true);
       tacker_status s = launch_fused(m, k, A.head());
       if (s) return s;
       cudaEvent_t e = record(m);
-      A.pending = ref(m, e);
+      track(m, e0, e, TACKER_CLASS_FUSED);
+      set_pending(m, A, e);
       if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
       // online model update from the measured co-run
       std::string lk, bk, pk;
       make_keys(&k.lc, &A.head().be, A.head().warp_split ? A.head().warp_split : 16, &lk, &bk, &pk);
-      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, A.head().t_pred_ms});
+      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, A.head().t_pred_ms, best_tf});
     }
     A.pos++;
     A.completed++;
@@ -433,9 +484,11 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
     if (m->sim()) {
       m->now += ttc;
     } else {
+      cudaEvent_t e0 = begin(m, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
       tacker_status s = launch_lc(m, k);
       if (s) return s;
       cudaEvent_t e = record(m);
+      track(m, e0, e, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
       if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
     }
     m->st.original_lc++;
@@ -453,9 +506,11 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       m->now += b.t_pred_ms;
       A.ready_at = m->now;
     } else {
+      cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
       tacker_status s = launch_be(m, b);
       if (s) return s;
-      A.pending = ref(m, record(m));
+      set_pending(m, A, record(m));
+      track(m, e0, A.pending, TACKER_CLASS_BE);
     }
     A.pos++;
     A.completed++;
@@ -495,6 +550,12 @@ tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats 
   *o = m->st;
   o->now_ms = m->sim() ? m->now : host_now(m);
   o->model_refits = m->refits;
+  o->pred_err_sum = m->pred_err_sum;
+  o->pred_err_n = m->pred_err_n;
+  for (int c = 0; c < 4; ++c) {
+    o->class_ms[c] = m->class_timed[c] ? m->class_ms[c] / (double)m->class_timed[c] * (double)m->class_n[c] : 0.0;
+    o->class_launches[c] = m->class_n[c];
+  }
   return TACKER_OK;
 }
 

@@ -199,5 +199,8 @@ class QosRun:
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
                 "fused": int(st.fused_launches), "reordered": int(st.reordered_be), "idle_be": int(st.idle_be),
                 "model_refits": int(st.model_refits),
+                "fused_pred_err_mean": st.pred_err_sum / st.pred_err_n if st.pred_err_n else None,
+                "class_ms": {n: float(st.class_ms[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
+                "class_launches": {n: int(st.class_launches[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
                 "lc_p50_ms": float(np.median(lat)), "lc_p99_ms": p99, "lc_max_ms": float(lat.max()),
                 "qos_ms": self.qos, "qos_met": bool(p99 <= self.qos), "query_solo_ms": self.query_solo_ms()}

@@ -51,11 +51,14 @@ def main():
     ap.add_argument("--be", default="stencil,mriq")
     ap.add_argument("--ws", type=int, default=24)
     ap.add_argument("--qos", type=float, default=50.0)
+    ap.add_argument("--io", action="store_true", help="each query copies its input H2D and result D2H")
     args = ap.parse_args()
     svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
     apps = build_apps(args.be.split(","))
     tk.tacker_model_clear()
     q = qos.QosRun(svc, apps, warp_split=args.ws, qos_ms=args.qos)
+    if args.io:
+        q.with_io()
     q.calibrate()
     res = {}
     for pol in (tk.POLICY_BAYMAX, tk.POLICY_TACKER):
