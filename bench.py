@@ -525,7 +525,7 @@ def run_simulated(args, ws, rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300, help="timed LC queries")
+    ap.add_argument("--steps", type=int, default=1000, help="timed LC queries")
     ap.add_argument("--warmup", type=int, default=20, help="untimed warm-up LC queries")
     ap.add_argument("--impl", default="tacker", choices=["tacker", "reference"])
     ap.add_argument("--warp-split", type=int, default=24)

@@ -348,6 +348,13 @@ tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms);
  * headroom, or NAN to use the manager's Eq. 9 value; on output the updated headroom. */
 tacker_status tacker_manager_step(tacker_manager_t m, double qos_target_ms, double *headroom_ms,
                                   tacker_decision *out);
+/* GPU mode, Tacker policy: build (and cache in the manager) the fused handle of every (TC
+ * kernel, BE kernel) pair with a fitted pair model, so no handle is built (tensor maps, a small
+ * cudaMalloc) inside a timed run.  q = NULL: the kernels of every submitted query; else the
+ * kernels of *q (not submitted; e.g. before arrival times are fixed).  BE apps must be
+ * submitted first.  Handles are keyed by the LC operand pointers and the BE kernel.
+ * tacker_manager_run calls it with NULL. */
+tacker_status tacker_manager_prepare(tacker_manager_t m, const tacker_lc_query *q);
 /* Native run loop: steps the manager (launching in GPU mode) until its clock has passed
  * t_end_ms and every submitted query has completed, or max_decisions decisions were taken
  * (<= 0: unbounded).  The host thread spins between decisions (no Python in the loop). */

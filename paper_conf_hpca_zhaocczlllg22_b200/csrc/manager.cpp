@@ -20,7 +20,9 @@
 #include <cmath>
 #include <cstring>
 #include <deque>
+#include <array>
 #include <map>
+#include <set>
 #include <string>
 #include <vector>
 
@@ -87,6 +89,8 @@ struct tacker_manager_s {
   };
   std::deque<Observed> observed;   // fused launches awaiting their measured duration
   int64_t refits = 0;
+  size_t prepared = 0;                                   // queries visited by tacker_manager_prepare
+  std::set<std::array<const void *, 3>> prepared_lc;     // LC operand triples already prepared
   double pred_err_sum = 0;         // sum |predicted - measured| / measured over fused launches
   int64_t pred_err_n = 0;
   struct Timed {
@@ -216,19 +220,26 @@ static tacker_status launch_be(tacker_manager_s *m, const tacker_be_kernel &b) {
   return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
-static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b) {
+// Fused handle of (LC kernel, BE kernel) from the manager's cache, built on first use.
+static tacker_status fused_handle(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b,
+                                  tacker_fused_t *out) {
   const int ws = b.warp_split ? b.warp_split : 16;
   char key[256];
   snprintf(key, sizeof key, "%p/%p/%p/%p/%d/%d", k.lc.A, k.lc.B, k.lc.D, (const void *)&b, ws, b.be.orig_blocks);
   auto it = m->cache.find(key);
-  tacker_fused_t f = nullptr;
-  if (it == m->cache.end()) {
-    tacker_status s = tacker_fuse(&k.lc, &b.be, ws, tacker_ratio{0, 0}, &f);
-    if (s) return s;
-    m->cache[key] = f;
-  } else {
-    f = it->second;
+  if (it != m->cache.end()) {
+    *out = it->second;
+    return TACKER_OK;
   }
+  tacker_status s = tacker_fuse(&k.lc, &b.be, ws, tacker_ratio{0, 0}, out);
+  if (s == TACKER_OK) m->cache[key] = *out;
+  return s;
+}
+
+static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b) {
+  tacker_fused_t f = nullptr;
+  tacker_status s = fused_handle(m, k, b, &f);
+  if (s) return s;
   return tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
@@ -522,8 +533,43 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   return TACKER_OK;
 }
 
+// Fused handles of every (TC kernel in ks, CUDA-core kernel of a BE app) pair the predictor has
+// a model for: the only pairs Eq. 8 can admit.  Queries of one service share their kernels, so
+// only LC operand triples not seen before are visited.
+static tacker_status prepare_kernels(tacker_manager_s *m, const tacker_lc_kernel *ks, size_t n) {
+  for (size_t i = 0; i < n; ++i) {
+    const tacker_lc_kernel &k = ks[i];
+    if (!k.is_tc) continue;
+    if (!m->prepared_lc.insert({k.lc.A, k.lc.B, k.lc.D}).second) continue;
+    for (const App &A : m->apps)
+      for (const tacker_be_kernel &b : A.ks) {
+        double tf;
+        if (!b.is_cd || !pair_time(k, b, &tf)) continue;
+        tacker_fused_t f = nullptr;
+        tacker_status s = fused_handle(m, k, b, &f);
+        if (s != TACKER_OK && s != TACKER_ERESOURCE && s != TACKER_EUNSUPPORTED) return s;
+      }
+  }
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_prepare(tacker_manager_t m, const tacker_lc_query *q) {
+  if (!m) return set_error("null manager"), TACKER_EINVAL;
+  if (m->sim() || m->policy != TACKER_POLICY_TACKER) return TACKER_OK;
+  if (q) {
+    if (q->n_kernels < 0 || (q->n_kernels > 0 && !q->kernels)) return set_error("bad query"), TACKER_EINVAL;
+    return prepare_kernels(m, q->kernels, (size_t)q->n_kernels);
+  }
+  for (; m->prepared < m->queries.size(); ++m->prepared) {
+    const Query &Q = m->queries[m->prepared];
+    if (tacker_status s = prepare_kernels(m, Q.ks.data(), Q.ks.size())) return s;
+  }
+  return TACKER_OK;
+}
+
 tacker_status tacker_manager_run(tacker_manager_t m, double qos, double t_end_ms, int64_t max_decisions) {
   if (!m) return set_error("null manager"), TACKER_EINVAL;
+  if (tacker_status s = tacker_manager_prepare(m, nullptr)) return s;
   int64_t n = 0;
   tacker_decision d;
   for (;;) {

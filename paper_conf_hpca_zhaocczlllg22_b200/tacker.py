@@ -229,6 +229,7 @@ _PROTOS = {
     "tacker_manager_step": ([_V, _D, C.POINTER(_D), C.POINTER(Decision)], C.c_int),
     "tacker_manager_stats_get": ([_V, C.POINTER(ManagerStats)], C.c_int),
     "tacker_manager_run": ([_V, _D, _D, _I64], C.c_int),
+    "tacker_manager_prepare": ([_V, _V], C.c_int),
     "tacker_manager_query_latency": ([_V, _I32, C.POINTER(_D)], C.c_int),
 }
 for _name, (_args, _res) in _PROTOS.items():
@@ -595,6 +596,16 @@ class Manager:
         thr = C.c_double(headroom)
         _chk(_lib.tacker_manager_step(self.h, qos_ms, C.byref(thr), C.byref(d)))
         return d
+
+    def prepare(self, kernels=None):
+        """Build the fused handles of every admissible (TC kernel, BE kernel) pair up front: of
+        `kernels` (a query's kernel list, not submitted) or of every submitted query."""
+        if kernels is None:
+            _chk(_lib.tacker_manager_prepare(self.h, None))
+            return
+        arr = (LcKernel * len(kernels))(*kernels)
+        q = LcQuery(len(kernels), arr)
+        _chk(_lib.tacker_manager_prepare(self.h, C.byref(q)))
 
     def run(self, qos_ms, t_end_ms=0.0, max_decisions=0):
         """Native loop: decide + launch until t_end_ms has passed and all queries completed."""
