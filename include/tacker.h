@@ -374,6 +374,9 @@ typedef struct {
    * timed fused launches (the pair model as it stood when the manager decided) */
   double pred_err_sum;
   int64_t pred_err_n;
+  /* sum of the standalone (predicted) durations of the BE kernels issued: BE work in original-
+   * kernel milliseconds, so throughput can be normalised across BE apps of different length */
+  double be_work_ms;
 } tacker_manager_stats;
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
 /* Completion time (manager clock) of a finished query, or -1 if unfinished. */

@@ -91,6 +91,7 @@ struct tacker_manager_s {
   int64_t refits = 0;
   size_t prepared = 0;                                   // queries visited by tacker_manager_prepare
   std::set<std::array<const void *, 3>> prepared_lc;     // LC operand triples already prepared
+  double be_work_ms = 0;           // sum of standalone (predicted) times of issued BE kernels
   double pred_err_sum = 0;         // sum |predicted - measured| / measured over fused launches
   int64_t pred_err_n = 0;
   struct Timed {
@@ -389,6 +390,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
         set_pending(m, A, record(m));
         track(m, e0, A.pending, TACKER_CLASS_BE);
       }
+      m->be_work_ms += A.head().t_pred_ms;
       A.pos++;
       A.completed++;
       m->st.be_kernels_done++;
@@ -486,6 +488,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       make_keys(&k.lc, &A.head().be, A.head().warp_split ? A.head().warp_split : 16, &lk, &bk, &pk);
       m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, A.head().t_pred_ms, best_tf});
     }
+    m->be_work_ms += A.head().t_pred_ms;
     A.pos++;
     A.completed++;
     m->st.fused_launches++;
@@ -523,6 +526,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       set_pending(m, A, record(m));
       track(m, e0, A.pending, TACKER_CLASS_BE);
     }
+    m->be_work_ms += A.head().t_pred_ms;
     A.pos++;
     A.completed++;
     m->st.be_kernels_done++;
@@ -597,6 +601,7 @@ tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats 
   o->now_ms = m->sim() ? m->now : host_now(m);
   o->model_refits = m->refits;
   o->pred_err_sum = m->pred_err_sum;
+  o->be_work_ms = m->be_work_ms;
   o->pred_err_n = m->pred_err_n;
   for (int c = 0; c < 4; ++c) {
     o->class_ms[c] = m->class_timed[c] ? m->class_ms[c] / (double)m->class_timed[c] * (double)m->class_n[c] : 0.0;

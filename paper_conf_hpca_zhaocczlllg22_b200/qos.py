@@ -216,6 +216,8 @@ class QosRun:
         return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "queries": int(len(lat)),
                 "lambda_per_s": lam * 1e3, "load": load, "elapsed_ms": gpu_ms,
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
+                # normalised BE throughput: standalone-milliseconds of BE work per wall millisecond
+                "be_work_ms": st.be_work_ms, "be_norm_thpt": st.be_work_ms / gpu_ms,
                 "fused": int(st.fused_launches), "reordered": int(st.reordered_be), "idle_be": int(st.idle_be),
                 "model_refits": int(st.model_refits),
                 "fused_pred_err_mean": st.pred_err_sum / st.pred_err_n if st.pred_err_n else None,

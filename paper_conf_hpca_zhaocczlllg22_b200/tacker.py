@@ -192,7 +192,8 @@ class ManagerStats(C.Structure):
     _fields_ = [("lc_queries_done", C.c_int64), ("be_kernels_done", C.c_int64), ("fused_launches", C.c_int64),
                 ("original_lc", C.c_int64), ("reordered_be", C.c_int64), ("idle_be", C.c_int64),
                 ("now_ms", C.c_double), ("model_refits", C.c_int64), ("class_ms", C.c_double * 4),
-                ("class_launches", C.c_int64 * 4), ("pred_err_sum", C.c_double), ("pred_err_n", C.c_int64)]
+                ("class_launches", C.c_int64 * 4), ("pred_err_sum", C.c_double), ("pred_err_n", C.c_int64),
+                ("be_work_ms", C.c_double)]
 
 
 CLASS_LC_TC, CLASS_LC_CD, CLASS_FUSED, CLASS_BE = range(4)

@@ -65,6 +65,7 @@ def main():
         r = q.run(pol, args.queries, load=args.load, warmup=args.warmup)
         res[r["policy"]] = r
     res["improvement_eq10"] = res["tacker"]["be_kernels_per_s"] / res["baymax"]["be_kernels_per_s"] - 1.0
+    res["improvement_eq10_normalised"] = res["tacker"]["be_norm_thpt"] / res["baymax"]["be_norm_thpt"] - 1.0
     res["pairs_fitted"] = len(q.pairs)
     res["pair_pred_err"] = {"max": max(q.pair_err), "mean": sum(q.pair_err) / len(q.pair_err), "n": len(q.pair_err)}
     print(json.dumps(res))
