@@ -212,3 +212,12 @@ def test_manager_simulation_matches_reference(tk, policy):
     assert max(ref["latency"].values()) <= 50.0
     if policy == "tacker":
         assert m.stats().fused_launches > 0
+    # be_work_ms = standalone time of every BE kernel issued, app heads cycling in order
+    work, pos = 0.0, [0] * len(app_ts)
+    for _, fa, ra in exp:
+        for a in ([fa] if fa >= 0 else []) + list(ra):
+            work += app_ts[a][pos[a] % len(app_ts[a])]
+            pos[a] += 1
+    assert abs(m.stats().be_work_ms - work) < 1e-9
+    m.prepare()            # no-op on the simulated GPU
+    m.prepare([lc_kernel(tk, True, 1.0)])

@@ -196,3 +196,32 @@ def test_stencil_scalar_path_and_large(tk, ws):
         c["reset"]()
         f.launch()
         assert host(c["outs"][0]).tobytes() == orig.tobytes()
+
+
+@pytest.mark.parametrize("ws", [4, 12, 24])
+@pytest.mark.parametrize("orig_blocks", [0, 301])
+def test_mriq_static_split_chunks(tk, ws, orig_blocks):
+    # fused mri-q Q uses the static even split with up to 4 blocks per thread (BeCoarsen): 666
+    # blocks over 148 CTAs gives 4-5 per CTA, so at ws=4 a slot runs a 4-chunk plus a 1-chunk,
+    # at ws=24 slots get 0 or 1; orig_blocks = 301 exercises the PTB prefix on the same split
+    N, nk = 44, 256
+    d = synth.mriq_inputs(N, nk, 11)
+    pm = (d["phiR"].astype(np.float32) ** 2 + d["phiI"].astype(np.float32) ** 2).astype(np.float32)
+    dd = {k: t(v) for k, v in d.items()}
+    dpm = t(pm)
+    outs = [torch.zeros(N ** 3, device=dev()) for _ in range(4)]
+    desc_o = tk.be_mriq_q(dd["x"], dd["y"], dd["z"], dd["kx"], dd["ky"], dd["kz"], dpm, outs[0], outs[1],
+                          orig_blocks=orig_blocks)
+    desc_f = tk.be_mriq_q(dd["x"], dd["y"], dd["z"], dd["kx"], dd["ky"], dd["kz"], dpm, outs[2], outs[3],
+                          orig_blocks=orig_blocks)
+    tk.tacker_launch_original(None, desc_o)
+    A, B = synth.lc_gemm_inputs(256, 128, 64, seed=0)
+    D = torch.zeros(256, 128, device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), desc_f, ws)
+    f.launch()
+    qr_o, qi_o, qr_f, qi_f = (host(o) for o in outs)
+    assert qr_f.tobytes() == qr_o.tobytes() and qi_f.tobytes() == qi_o.tobytes()
+    n = N ** 3 if orig_blocks == 0 else orig_blocks * 128
+    rr, ri, sr, si = obe.mriq_q(d["x"][:n], d["y"][:n], d["z"][:n], d["kx"], d["ky"], d["kz"], pm)
+    assert max_rel_err(qr_o[:n], rr, sr) <= 1e-5 and max_rel_err(qi_o[:n], ri, si) <= 1e-5
+    assert np.all(qr_o[n:] == 0) and np.all(qi_o[n:] == 0)
