@@ -88,13 +88,19 @@ typedef struct {
  * PTB runtime argument of Fig. 7: 0 = the whole problem, else only blocks
  * [0, orig_blocks) run (must not exceed the whole-problem count).  Bodies use fixed
  * per-element arithmetic order, so a fused launch is bit-identical to the original one.
+ * `block_offset` shifts the PTB range to [block_offset, block_offset + orig_blocks) (orig_blocks
+ * 0 = to the end): a launch runs a SLICE of the original kernel.  Running the slices of a
+ * partition of [0, blocks) in order on one stream is bit-identical to the whole kernel for every
+ * kind whose blocks write disjoint outputs or commutative integer counts (all kinds except
+ * TACKER_BE_JDS_SCAN, whose single block reads every count).  The manager sizes the BE slice of
+ * a fused launch to the pair's opportune load ratio (DESIGN.md §2 reading 13).
  */
 typedef enum {
   TACKER_BE_NONE = 0,
   TACKER_BE_SGEMM = 1,        /* C = alpha A.B + beta C; block = 64x64 tile of C          */
   TACKER_BE_STENCIL = 2,      /* 7-point Jacobi sweep; block = 32x4 columns, all z        */
   TACKER_BE_MRIQ_PHIMAG = 3,  /* phiMag = phiR^2 + phiI^2; block = 512 k                   */
-  TACKER_BE_MRIQ_Q = 4,       /* Qr/Qi += sum_k phiMag cos/sin(2pi k.x); block = 256 voxels */
+  TACKER_BE_MRIQ_Q = 4,       /* Qr/Qi += sum_k phiMag cos/sin(2pi k.x); block = 32 voxels x 4 k-lanes */
   TACKER_BE_CUTCP = 5,        /* cutoff Coulomb potential; block = 4x4x8 lattice points    */
   TACKER_BE_LBM = 6,          /* D3Q19 BGK push step; block = 128 cells along x            */
   TACKER_BE_SPMV_JDS = 7,     /* y[perm[i]] = sum_d val*x[col]; block = 128 rows           */
@@ -182,7 +188,8 @@ typedef struct {
 
 typedef struct {
   int32_t kind;              /* tacker_be_kind */
-  int32_t orig_blocks;       /* PTB original block count (0 = whole problem) */
+  int32_t orig_blocks;       /* PTB original block count (0 = whole problem / rest) */
+  int32_t block_offset;      /* first original block of this launch (0 = from the start) */
   union {
     tacker_be_sgemm sgemm;
     tacker_be_stencil stencil;
@@ -253,6 +260,11 @@ tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, co
 tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream);
 tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be,
                                      tacker_stream_t stream);
+/* One fused launch of handle f whose BE part runs only the PTB slice [block_offset,
+ * block_offset + n_blocks) of the handle's BE kernel (the LC part is unchanged; n_blocks 0 = no
+ * BE work).  The handle is not modified.  EINVAL if the slice leaves the whole-problem range. */
+tacker_status tacker_launch_fused_slice(tacker_fused_t f, int64_t block_offset, int64_t n_blocks,
+                                        tacker_stream_t stream);
 
 /* ======================================================================== predictor (a9, a10)
  * Per-kernel LR (§VI-C): X = a * blocks + b, keyed by kernel class.
@@ -305,9 +317,15 @@ typedef struct {
 
 typedef struct {
   int32_t is_cd;             /* 1: CUDA-core kernel (fusable as BE) */
-  double t_pred_ms;
+  double t_pred_ms;          /* predicted standalone duration of the whole kernel */
   tacker_be_desc be;
   int32_t warp_split;        /* fusion plan for this kernel (0 = library default 16) */
+  /* PTB slicing (params.slice_be): the kernel's original blocks [be.block_offset,
+   * be.block_offset + n_blocks) may run as several launches.  Per-kernel LR of a slice of n
+   * blocks (§VI-C): X_cd(n) = t_floor_ms + t_block_ms * n.  n_blocks <= 1 or
+   * t_block_ms <= 0: never sliced. */
+  int32_t n_blocks;
+  double t_block_ms, t_floor_ms;
 } tacker_be_kernel;
 
 typedef struct {
@@ -324,6 +342,7 @@ typedef struct {
   double thr_ms;             /* headroom after the decision */
   double gain_ms;            /* Tgain of the fused pair */
   double t_start_ms, t_end_ms; /* manager clock: predicted (sim) or issue time (GPU) */
+  int64_t fused_blocks;      /* BE blocks in the fused launch: a PTB slice, or -1 = the whole rest */
 } tacker_decision;
 
 typedef struct {
@@ -331,6 +350,15 @@ typedef struct {
   double idle_cap_ms;        /* idle GPU: launch BE heads no longer than this (<=0: any) */
   int32_t max_inflight;      /* GPU mode: kernels allowed in flight on the stream (>=1) */
   int32_t simulate;          /* 1: no GPU, durations = predictions */
+  /* Tacker policy, B200 reading 13: the BE part of a fused launch is the slice
+   * of the head kernel's remaining blocks whose predicted X_cd puts the pair at its opportune
+   * load ratio r* (the two-stage model's inflection), or at slice_ratio when > 0.
+   * 0: whole BE kernels only (the paper's fusion unit). */
+  int32_t slice_be;
+  double slice_ratio;
+  /* 0 (default): after every LC kernel, fused or not, reorder the other ready BE heads with
+   * Ttmp < Thr (reading 6); 1: reorder only after an LC kernel that was not fused. */
+  int32_t reorder_only_unfused;
 } tacker_manager_params;
 
 typedef struct tacker_manager_s *tacker_manager_t;

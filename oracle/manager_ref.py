@@ -23,8 +23,20 @@ Rules, in the paper's order:
   * Baymax mode = the same manager with fusion disabled ("static scheduling").
   * Idle GPU (no active LC query; the paper is silent): launch one ready BE head whose
     duration <= idle_cap, round robin over apps.
+  * PTB slicing (B200 reading 13 in DESIGN.md §2; off by default): with slice_be, the BE part of
+    a fused launch is a slice of n of the head kernel's N original blocks (PTB, Fig. 7), with
+    predicted standalone time X_cd(n) = t_floor + t_block * n (the kernel's LR, §VI-C
+    P:1839-1851); n is the smallest block count with X_cd(n) >= r * Ttc, r = the pair's opportune
+    ratio (Fig. 10) or a fixed slice_ratio, clamped to [1, remaining]; a slice that
+    would take every remaining block is the whole rest.  The head kernel stays the head until
+    its last block is issued; reorder and idle launches issue the whole rest, whose predicted
+    time is X_cd(remaining) once a slice of it has run.  BE work = n/N of the kernel's
+    standalone time per slice.
+  * reorder_only_unfused: reorder only after an LC kernel that was not fused (P:2035 literally).
 """
 from __future__ import annotations
+
+import math
 
 from dataclasses import dataclass, field
 
@@ -40,18 +52,23 @@ class Decision:
     reorder: list = field(default_factory=list)   # app ids launched after the LC kernel
     thr: float = 0.0
     gain: float = 0.0
+    blocks: int = -1              # BE blocks of the fused launch (PTB slice), -1 = whole rest
 
 
-def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True):
+def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=None, reorder_only_unfused=False):
     """Pure decision for one LC kernel.
 
-    heads: list of (app, Tcd, be_is_cd) for READY BE head kernels, in app order.
-    fuse_pred(app) -> Tk_fuse or None.  Returns (fused_app, reorder_apps, thr, gain)."""
+    heads: list of (app, Tcd, be_is_cd) for READY BE head kernels, in app order (Tcd = the
+    predicted time of what is left of the head kernel).  fuse_tcd(app) -> the BE time a fused
+    launch would carry (a PTB slice; default Tcd).  fuse_pred(app) -> Tk_fuse or None.
+    Returns (fused_app, reorder_apps, thr, gain)."""
     fused, gain_best, tf_best = -1, None, None
     if allow and policy == TACKER and lc_is_tc:
         for app, tcd, be_cd in heads:
             if not be_cd:
                 continue
+            if fuse_tcd is not None:
+                tcd = fuse_tcd(app)
             tf = fuse_pred(app)
             if tf is None:
                 continue
@@ -62,7 +79,7 @@ def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True):
     reorder = []
     if fused >= 0:
         thr -= tf_best - ttc
-    if allow:
+    if allow and not (reorder_only_unfused and fused >= 0):
         for app, tcd, _ in heads:
             if app == fused:
                 continue
@@ -89,20 +106,61 @@ class Query:
 
 @dataclass
 class App:
-    kernels: list          # [(is_cd, T_pred)], cycled forever
+    kernels: list          # [(is_cd, T_pred[, N_blocks, t_block, t_floor])], cycled forever
     pos: int = 0
     ready_at: float = 0.0
     completed: int = 0
+    done: int = 0          # blocks of the head kernel already issued (PTB slices)
+    work: float = 0.0      # standalone-time of the BE work issued
 
     def head(self):
         return self.kernels[self.pos % len(self.kernels)]
 
+    def lr(self):
+        """(N, t_block, t_floor) of the head kernel; N = 0 when it has no slicing data."""
+        h = self.head()
+        return (h[2], h[3], h[4]) if len(h) >= 5 else (0, 0.0, 0.0)
 
-def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=None, t_end=None):
+    def rem(self):
+        """Predicted standalone time of what is left of the head kernel."""
+        N, a, b = self.lr()
+        return self.head()[1] if self.done == 0 else b + a * (N - self.done)
+
+    def issue(self, n):
+        """n blocks of the head kernel issued (n < 0: the whole rest, completing it)."""
+        N, _, _ = self.lr()
+        T = self.head()[1]
+        if n >= 0 and N > 1 and self.done + n < N:
+            self.work += T * n / N
+            self.done += n
+            return
+        self.work += T if self.done == 0 else T * (N - self.done) / N
+        self.done = 0
+        self.pos += 1
+        self.completed += 1
+
+
+def slice_blocks(app, ttc, r_opp, slice_be, slice_ratio):
+    """Blocks of app's head kernel for a fused launch with a TC kernel of time ttc, or -1 for
+    the whole rest (reading 13)."""
+    N, a, b = app.lr()
+    if not (slice_be and N > 1 and a > 0):
+        return -1
+    rt = slice_ratio if slice_ratio > 0 else r_opp
+    if rt is None:
+        return -1
+    R = N - app.done
+    n = max(1, min(math.ceil((rt * ttc - b) / a - 1e-9), R))
+    return n if n < R else -1
+
+
+def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=None, t_end=None,
+             slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_only_unfused=False):
     """Serial single-stream GPU whose kernels take exactly their predicted time.
 
-    fuse_pred(lc_T, be_T) -> Tk_fuse or None.  The manager acts whenever the stream drains.
-    Returns dict(latency per query, be_completed, timeline, decisions)."""
+    fuse_pred(lc_T, be_T) -> Tk_fuse or None; opp_ratio(app) -> the pair's opportune ratio or
+    None (slicing).  The manager acts whenever the stream drains.
+    Returns dict(latency per query, be_completed, be_work, timeline, decisions)."""
     t = 0.0
     active: list[Query] = []
     pending = sorted(queries, key=lambda q: q.arrival)
@@ -117,7 +175,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
             break
         if t_end is not None and t >= t_end:
             break
-        heads = [(a, app.head()[1], app.head()[0]) for a, app in enumerate(apps) if app.ready_at <= t]
+        heads = [(a, app.rem(), app.head()[0]) for a, app in enumerate(apps) if app.ready_at <= t]
         if active:
             q = active[0]
             newest = active[-1]
@@ -130,19 +188,29 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
             is_tc, ttc = q.kernels[q.pos]
             allow = (q is newest) and not q.direct and q.thr is not None
             thr = q.thr if q.thr is not None else 0.0
+            nblk = {a: slice_blocks(apps[a], ttc, opp_ratio(a) if opp_ratio else None, slice_be, slice_ratio)
+                    for a, _, _ in heads}
+
+            def tcd_of(a):
+                n = nblk[a]
+                if n < 0:
+                    return apps[a].rem()
+                N, sa, sb = apps[a].lr()
+                return sb + sa * n
+
             fused, reorder, thr2, gain = decide(
                 ttc, is_tc, thr, heads, policy,
-                lambda a: fuse_pred(ttc, apps[a].head()[1]), allow)
+                lambda a: fuse_pred(ttc, tcd_of(a)), allow, fuse_tcd=tcd_of,
+                reorder_only_unfused=reorder_only_unfused)
             if allow:
                 q.thr = thr2
             start = t
             if fused >= 0:
-                dur = fuse_pred(ttc, apps[fused].head()[1])
+                dur = fuse_pred(ttc, tcd_of(fused))
                 timeline.append(("fused", q.qid, q.pos, fused, start, start + dur))
-                apps[fused].pos += 1
-                apps[fused].completed += 1
+                apps[fused].issue(nblk[fused])
                 apps[fused].ready_at = start + dur
-                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), q.thr, gain))
+                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), q.thr, gain, nblk[fused]))
             else:
                 dur = ttc
                 timeline.append(("lc", q.qid, q.pos, -1, start, start + dur))
@@ -153,10 +221,9 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
             if q.pos == len(q.kernels):
                 q.done_at = t
             for a in reorder:
-                d = apps[a].head()[1]
+                d = apps[a].rem()
                 timeline.append(("be", -1, -1, a, t, t + d))
-                apps[a].pos += 1
-                apps[a].completed += 1
+                apps[a].issue(-1)
                 t += d
                 apps[a].ready_at = t
         else:
@@ -166,8 +233,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 a, d = cands[0]
                 timeline.append(("be", -1, -1, a, t, t + d))
                 decisions.append(Decision(IDLE_BE, None, -1, [a], 0.0))
-                apps[a].pos += 1
-                apps[a].completed += 1
+                apps[a].issue(-1)
                 t += d
                 apps[a].ready_at = t
             else:
@@ -177,5 +243,5 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                     break
                 t = min(cand)
     lat = {q.qid: (q.done_at - q.arrival) for q in queries if q.done_at is not None}
-    return dict(latency=lat, be_completed=[a.completed for a in apps], timeline=timeline,
-                decisions=decisions, t=t)
+    return dict(latency=lat, be_completed=[a.completed for a in apps], be_work=sum(a.work for a in apps),
+                timeline=timeline, decisions=decisions, t=t)

@@ -12,7 +12,7 @@ constexpr int kVbThreads = 128;
 #define TK_STENCIL_ZC 4
 #endif
 #ifndef TK_MRIQ_COARSEN
-#define TK_MRIQ_COARSEN 4
+#define TK_MRIQ_COARSEN 2
 #endif
 #ifndef TK_MRIQ_REDUCE
 #define TK_MRIQ_REDUCE 0

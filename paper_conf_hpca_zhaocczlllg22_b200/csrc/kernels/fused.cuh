@@ -54,6 +54,7 @@ struct alignas(64) FusedParams {
   LcParams lc;
   tacker_be_desc be;
   int64_t be_blocks;       // original blocks to run (PTB original_block_num)
+  int64_t be_offset;       // first original block (a slice [be_offset, be_offset + be_blocks))
   BeWork *work;            // device workspace for the BE ticket
   int32_t be_vb_per_cta;   // virtual blocks per CTA
   int32_t lc_warps;        // 6 or 0
@@ -257,14 +258,15 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
     const int64_t lo = P.be_blocks * cta / gridDim.x, hi = P.be_blocks * (cta + 1) / gridDim.x;
     const int S = P.be_vb_per_cta;
     for (int64_t b = lo + (hi - lo) * j / S, e = lo + (hi - lo) * (j + 1) / S; b < e; b += kC)
-      be_run_coarse<BE_KIND>(P.be, b, (int)min((int64_t)kC, e - b), tid, bar, body_smem, &P.tmap_be);
+      be_run_coarse<BE_KIND>(P.be, P.be_offset + b, (int)min((int64_t)kC, e - b), tid, bar, body_smem, &P.tmap_be);
     return;
   }
   const int64_t units = (P.be_blocks + kC - 1) / kC;
   int64_t vb = (int64_t)j * gridDim.x + cta;
   while (vb < units) {
     const int64_t b0 = vb * kC;
-    be_run_coarse<BE_KIND>(P.be, b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem, &P.tmap_be);
+    be_run_coarse<BE_KIND>(P.be, P.be_offset + b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem,
+                           &P.tmap_be);
     if (tid == 0) *s_ticket = groups + atomicAdd(&P.work->ticket, 1u);
     named_bar_sync(bar, kVbThreads);
     vb = *s_ticket;
@@ -339,7 +341,8 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
 }
 
 // ------------------------------------------------------------------------ BE original kernel
-// The non-persistent "CD_kernel" of Fig. 7: one CTA of 128 threads per original block.
+// The non-persistent "CD_kernel" of Fig. 7: one CTA of 128 threads per original block (of the
+// slice starting at block_offset).
 struct alignas(64) BeOrigParams {
   CUtensorMap tmap;        // BE input tensor map (stencil), unused otherwise
   tacker_be_desc d;
@@ -349,7 +352,7 @@ template <int BE_KIND>
 __global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ BeOrigParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   be_init<BE_KIND>(smem_raw, threadIdx.x, 1u);
-  be_run<BE_KIND>(P.d, (int64_t)blockIdx.x, threadIdx.x, 1u, smem_raw, &P.tmap);
+  be_run<BE_KIND>(P.d, (int64_t)P.d.block_offset + blockIdx.x, threadIdx.x, 1u, smem_raw, &P.tmap);
 }
 
 }  // namespace tk

@@ -11,6 +11,10 @@
 //   * No fusion: original launch, then reorder ready BE heads with Ttmp < Thr.
 //   * Baymax policy: identical with fusion disabled ("static scheduling").
 //   * Idle GPU (paper silent): one ready BE head no longer than idle_cap.
+//   * PTB slicing (params.slice_be, reading 13): a fused launch may carry only a slice of the BE
+//     head kernel's remaining blocks, sized so that X_cd(n) = t_floor + t_block n (the kernel's
+//     LR, §VI-C) puts the pair at its opportune ratio r* (Fig. 10); the head stays
+//     the head until its last block is issued.  Reorder / idle launches issue the whole rest.
 // In simulation mode every kernel takes its predicted time on a serial virtual stream (the
 // discrete-event reference oracle/manager_ref.py follows the same rules); in GPU mode the
 // manager launches on its stream and observes completion with CUDA events.
@@ -58,9 +62,18 @@ struct App {
   size_t pos = 0;
   double ready_at = 0;
   int64_t completed = 0;
+  int64_t done = 0;                // blocks of the head kernel already issued (PTB slices)
   cudaEvent_t pending = nullptr;   // GPU mode: last launched kernel of this app
   const tacker_be_kernel &head() const { return ks[pos % ks.size()]; }
 };
+
+// Per-kernel LR of a PTB slice of n blocks (§VI-C)
+double slice_ms(const tacker_be_kernel &b, int64_t n) { return b.t_floor_ms + b.t_block_ms * (double)n; }
+// predicted standalone time of what is left of an app's head kernel
+double rem_ms(const App &A) {
+  const tacker_be_kernel &b = A.head();
+  return A.done == 0 ? b.t_pred_ms : slice_ms(b, b.n_blocks - A.done);
+}
 
 }  // namespace
 
@@ -105,6 +118,27 @@ struct tacker_manager_s {
 
   bool sim() const { return prm.simulate != 0; }
 };
+
+static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b) {
+  return m->policy == TACKER_POLICY_TACKER && m->prm.slice_be && b.n_blocks > 1 && b.t_block_ms > 0;
+}
+
+// Bookkeeping of n issued blocks of app A's head kernel (n < 0: the whole rest, which completes
+// the kernel).  BE work is counted in standalone milliseconds: a slice of n of N blocks is
+// n/N of the kernel's standalone time, so the slices of a kernel add up to the whole kernel.
+static void issue_be(tacker_manager_s *m, App &A, int64_t n) {
+  const tacker_be_kernel &b = A.head();
+  if (n >= 0 && b.n_blocks > 1 && A.done + n < b.n_blocks) {
+    m->be_work_ms += b.t_pred_ms * (double)n / (double)b.n_blocks;
+    A.done += n;
+    return;
+  }
+  m->be_work_ms += A.done == 0 ? b.t_pred_ms : b.t_pred_ms * (double)(b.n_blocks - A.done) / (double)b.n_blocks;
+  A.done = 0;
+  A.pos++;
+  A.completed++;
+  m->st.be_kernels_done++;
+}
 
 static double host_now(tacker_manager_s *m) {
   if (m->external_clock || m->sim()) return m->now;
@@ -204,11 +238,31 @@ static void set_pending(tacker_manager_s *m, App &a, cudaEvent_t e) {
   a.pending = ref(m, e);
 }
 
-static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, double *tf) {
-  std::string lk, bk, pk;
+static bool pair_key(const tacker_lc_kernel &k, const tacker_be_kernel &b, std::string *pk) {
+  std::string lk, bk;
   const int ws = b.warp_split ? b.warp_split : 16;
-  if (!make_keys(&k.lc, &b.be, ws, &lk, &bk, &pk)) return false;
+  return make_keys(&k.lc, &b.be, ws, &lk, &bk, pk);
+}
+static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, double *tf) {
+  std::string pk;
+  if (!pair_key(k, b, &pk)) return false;
   return pair_predict(pk, k.t_pred_ms, b.t_pred_ms, tf);
+}
+
+static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b);
+
+// Blocks of the head kernel of A that a fused launch with TC kernel k should carry: the
+// smallest n with X_cd(n) >= r* X_tc (clamped to the remaining blocks), or -1 = the whole rest
+// (slicing off, kernel not sliceable, or no opportune ratio for the pair).
+static int64_t slice_blocks(const tacker_manager_s *m, const App &A, const std::string &pk, double ttc) {
+  const tacker_be_kernel &b = A.head();
+  if (!sliceable(m, b)) return -1;
+  double rt = m->prm.slice_ratio;
+  if (!(rt > 0) && !pair_opportune(pk, &rt)) return -1;
+  const int64_t R = b.n_blocks - A.done;
+  int64_t n = (int64_t)std::ceil((rt * ttc - b.t_floor_ms) / b.t_block_ms - 1e-9);
+  n = std::max<int64_t>(1, std::min<int64_t>(n, R));
+  return n < R ? n : -1;
 }
 
 // ---------------------------------------------------------------- GPU launches
@@ -217,8 +271,14 @@ static tacker_status launch_lc(tacker_manager_s *m, const tacker_lc_kernel &k) {
   return tacker_launch_original(nullptr, &k.cd, reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
-static tacker_status launch_be(tacker_manager_s *m, const tacker_be_kernel &b) {
-  return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
+// the rest of app A's head kernel (the whole kernel when no slice of it was issued yet)
+static tacker_status launch_be(tacker_manager_s *m, const App &A) {
+  const tacker_be_kernel &b = A.head();
+  if (A.done == 0) return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
+  tacker_be_desc d = b.be;
+  d.block_offset = b.be.block_offset + (int32_t)A.done;
+  d.orig_blocks = (int32_t)(b.n_blocks - A.done);
+  return tacker_launch_original(nullptr, &d, reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
 // Fused handle of (LC kernel, BE kernel) from the manager's cache, built on first use.
@@ -237,11 +297,15 @@ static tacker_status fused_handle(tacker_manager_s *m, const tacker_lc_kernel &k
   return s;
 }
 
-static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b) {
+// TC kernel k fused with n blocks of app A's head kernel (n < 0: the whole rest)
+static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const App &A, int64_t n) {
+  const tacker_be_kernel &b = A.head();
   tacker_fused_t f = nullptr;
   tacker_status s = fused_handle(m, k, b, &f);
   if (s) return s;
-  return tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
+  if (A.done == 0 && n < 0) return tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
+  return tacker_launch_fused_slice(f, (int64_t)b.be.block_offset + A.done, n < 0 ? b.n_blocks - A.done : n,
+                                   reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
 static cudaEvent_t record(tacker_manager_s *m) {
@@ -373,27 +437,24 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   if (qid < 0) {
     // idle GPU (or only tails of earlier queries still running): one bounded BE kernel
     for (int a : heads) {
-      const tacker_be_kernel &b = m->apps[a].head();
-      if (m->prm.idle_cap_ms > 0 && b.t_pred_ms > m->prm.idle_cap_ms) continue;
+      const double tt = rem_ms(m->apps[a]);
+      if (m->prm.idle_cap_ms > 0 && tt > m->prm.idle_cap_ms) continue;
       if (!m->active.empty()) break;   // do not delay a running query's completion
       out->action = TACKER_DEC_IDLE_BE;
       out->n_reorder = 1;
       out->reorder_apps[0] = a;
       App &A = m->apps[a];
       if (m->sim()) {
-        m->now += b.t_pred_ms;
+        m->now += tt;
         A.ready_at = m->now;
       } else {
         cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
-        tacker_status s = launch_be(m, b);
+        tacker_status s = launch_be(m, A);
         if (s) return s;
         set_pending(m, A, record(m));
         track(m, e0, A.pending, TACKER_CLASS_BE);
       }
-      m->be_work_ms += A.head().t_pred_ms;
-      A.pos++;
-      A.completed++;
-      m->st.be_kernels_done++;
+      issue_be(m, A, -1);
       m->st.idle_be++;
       out->t_end_ms = m->now;
       return TACKER_OK;
@@ -429,19 +490,27 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   const double ttc = k.t_pred_ms;
 
   int fused = -1;
-  double best_gain = 0, best_tf = 0;
+  int64_t best_n = -1;
+  double best_gain = 0, best_tf = 0, best_tcd = 0;
   if (allow && m->policy == TACKER_POLICY_TACKER && k.is_tc) {
     for (int a : heads) {
-      const tacker_be_kernel &b = m->apps[a].head();
+      const App &A = m->apps[a];
+      const tacker_be_kernel &b = A.head();
       if (!b.is_cd) continue;
+      std::string pk;
+      if (!pair_key(k, b, &pk)) continue;
+      const int64_t n = slice_blocks(m, A, pk, ttc);
+      const double tcd = n < 0 ? rem_ms(A) : slice_ms(b, n);
       double tf;
-      if (!pair_time(k, b, &tf)) continue;
-      if (ttc + b.t_pred_ms > tf && tf - ttc < thr) {   // Eq. 8
-        const double gain = b.t_pred_ms - (tf - ttc);
+      if (!pair_predict(pk, ttc, tcd, &tf)) continue;
+      if (ttc + tcd > tf && tf - ttc < thr) {   // Eq. 8
+        const double gain = tcd - (tf - ttc);
         if (fused < 0 || gain > best_gain) {
           fused = a;
           best_gain = gain;
           best_tf = tf;
+          best_tcd = tcd;
+          best_n = n;
         }
       }
     }
@@ -450,11 +519,11 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   if (fused >= 0) thr -= best_tf - ttc;
   // Reorder the remaining ready heads after the LC kernel, fused or not (reading:
   // Tacker = fusion on top of Baymax's reordering, "both adaptive kernel fusion and kernel
-  // reorder").
-  if (allow) {
+  // reorder"); reorder_only_unfused = the literal P:2035 rule.
+  if (allow && !(m->prm.reorder_only_unfused && fused >= 0)) {
     for (int a : heads) {
       if (a == fused) continue;
-      const double tt = m->apps[a].head().t_pred_ms;
+      const double tt = rem_ms(m->apps[a]);
       if (tt < thr) {
         reorder.push_back(a);
         thr -= tt;
@@ -467,6 +536,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   out->query = qid;
   out->lc_index = (int)q.pos;
   out->fused_app = fused;
+  out->fused_blocks = fused >= 0 ? best_n : 0;
   out->gain_ms = fused >= 0 ? best_gain : 0;
   out->thr_ms = thr;
   if (headroom) *headroom = thr;
@@ -477,7 +547,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       A.ready_at = m->now;
     } else {
       cudaEvent_t e0 = begin(m, TACKER_CLASS_FUSED, true);
-      tacker_status s = launch_fused(m, k, A.head());
+      tacker_status s = launch_fused(m, k, A, best_n);
       if (s) return s;
       cudaEvent_t e = record(m);
       track(m, e0, e, TACKER_CLASS_FUSED);
@@ -486,13 +556,10 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       // online model update from the measured co-run
       std::string lk, bk, pk;
       make_keys(&k.lc, &A.head().be, A.head().warp_split ? A.head().warp_split : 16, &lk, &bk, &pk);
-      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, A.head().t_pred_ms, best_tf});
+      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, best_tcd, best_tf});
     }
-    m->be_work_ms += A.head().t_pred_ms;
-    A.pos++;
-    A.completed++;
+    issue_be(m, A, best_n);
     m->st.fused_launches++;
-    m->st.be_kernels_done++;
     out->action = TACKER_DEC_FUSED;
   } else {
     if (m->sim()) {
@@ -515,21 +582,17 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   }
   for (int a : reorder) {
     App &A = m->apps[a];
-    const tacker_be_kernel &b = A.head();
     if (m->sim()) {
-      m->now += b.t_pred_ms;
+      m->now += rem_ms(A);
       A.ready_at = m->now;
     } else {
       cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
-      tacker_status s = launch_be(m, b);
+      tacker_status s = launch_be(m, A);
       if (s) return s;
       set_pending(m, A, record(m));
       track(m, e0, A.pending, TACKER_CLASS_BE);
     }
-    m->be_work_ms += A.head().t_pred_ms;
-    A.pos++;
-    A.completed++;
-    m->st.be_kernels_done++;
+    issue_be(m, A, -1);
     m->st.reordered_be++;
     if (out->n_reorder < TACKER_MAX_REORDER) out->reorder_apps[out->n_reorder++] = a;
   }

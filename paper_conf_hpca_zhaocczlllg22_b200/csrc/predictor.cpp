@@ -106,6 +106,20 @@ bool pair_predict(const std::string &key, double x_tc, double x_cd, double *y) {
   *y = x_tc * pair_tau(it->second, x_cd / x_tc);
   return true;
 }
+// Opportune load ratio of a pair (Fig. 10): the inflection r* = (a2 - a1) / (b1 - b2)
+// of the two-stage model, where stage 1 (co-run, slope b1) meets stage 2 (CD solo, slope b2).
+// False when the fitted stages do not form a convex two-stage curve (b1 >= b2) or r* <= 0.
+bool pair_opportune(const std::string &key, double *r) {
+  std::lock_guard<std::mutex> g(g_mu);
+  auto it = g_pair.find(key);
+  if (it == g_pair.end() || !it->second.fitted) return false;
+  const Pair &P = it->second;
+  if (!(P.b1 < P.b2)) return false;
+  const double rs = (P.a2 - P.a1) / (P.b1 - P.b2);
+  if (!(rs > 0) || !std::isfinite(rs)) return false;
+  *r = rs;
+  return true;
+}
 const std::string &fused_lc_key(tacker_fused_t f);
 const std::string &fused_be_key(tacker_fused_t f);
 const std::string &fused_pair_key(tacker_fused_t f);

@@ -13,6 +13,7 @@ int sm_count();
 // model store (predictor.cpp)
 bool model_predict(const std::string &key, double x, double *y);
 bool pair_predict(const std::string &key, double x_tc, double x_cd, double *y);
+bool pair_opportune(const std::string &key, double *r);
 
 // kind names
 const char *be_kind_name(int kind);

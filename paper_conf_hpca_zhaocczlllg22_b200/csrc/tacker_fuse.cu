@@ -185,11 +185,15 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
         return set_error("fma_burn: bad args"), TACKER_EINVAL;
       break;
   }
-  if (d.orig_blocks < 0 || d.orig_blocks > full) {
-    set_error("orig_blocks %d outside [0, %lld]", d.orig_blocks, (long long)full);
+  if (d.block_offset < 0 || d.block_offset > full || d.orig_blocks < 0 ||
+      (int64_t)d.orig_blocks > full - d.block_offset) {
+    set_error("PTB slice [%d, %d + %d) outside [0, %lld]", d.block_offset, d.block_offset, d.orig_blocks,
+              (long long)full);
     return TACKER_EINVAL;
   }
-  *blocks = d.orig_blocks ? d.orig_blocks : full;
+  if (d.block_offset && d.kind == TACKER_BE_JDS_SCAN)
+    return set_error("jds_scan runs as one block and cannot be sliced"), TACKER_EUNSUPPORTED;
+  *blocks = d.orig_blocks ? d.orig_blocks : full - d.block_offset;
   return TACKER_OK;
 }
 
@@ -358,6 +362,7 @@ struct tacker_fused_s {
   int grid, block, smem;
   int BN;
   int regs;
+  int64_t be_full;         // whole-problem BE block count (slice bound)
   std::string lc_key, be_key, pair_key;
 };
 
@@ -406,8 +411,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   int64_t be_blocks = 0;
   int vb = 0;
   uint32_t be_slice = 0;
+  F.be_full = 0;
   if (has_be) {
     if ((st = validate_be(*be, &be_blocks))) return st;
+    be_num_blocks(*be, &F.be_full);
     vb = warp_split / 4;
     if (ratio.be && ratio.be != vb)
       return set_error("block_ratio.be (%d) must equal warp_split/4 (%d)", ratio.be, vb), TACKER_EUNSUPPORTED;
@@ -448,6 +455,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.P.be_smem_per_vb = be_slice;
   F.P.be_vb_per_cta = vb;
   F.P.be_blocks = be_blocks;
+  F.P.be_offset = has_be ? be->block_offset : 0;
   F.P.lc_warps = kLcWarps;
   F.warp_split = warp_split;
   F.block = 32 * warps;
@@ -490,12 +498,13 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   return TACKER_OK;
 }
 
-static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) {
-  void *args[] = {&F.P};
+static tacker_status launch_params(const tacker_fused_s &F, FusedParams &P, cudaStream_t s) {
+  void *args[] = {&P};
   cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(F.fn), dim3(F.grid), dim3(F.block), args, F.smem, s);
   if (e != cudaSuccess) return cuda_fail("launch fused_kernel", e);
   return TACKER_OK;
 }
+static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) { return launch_params(F, F.P, s); }
 
 // ============================================================================ C ABI
 extern "C" {
@@ -600,6 +609,23 @@ tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, co
 tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream) {
   if (!f) return set_error("null handle"), TACKER_EINVAL;
   return launch_plan(*f, reinterpret_cast<cudaStream_t>(stream));
+}
+
+tacker_status tacker_launch_fused_slice(tacker_fused_t f, int64_t block_offset, int64_t n_blocks, tacker_stream_t stream) {
+  if (!f) return set_error("null handle"), TACKER_EINVAL;
+  if (!f->be.kind) return set_error("handle has no BE part"), TACKER_EINVAL;
+  if (f->be.kind == TACKER_BE_JDS_SCAN && (block_offset || n_blocks != f->be_full))
+    return set_error("jds_scan runs as one block and cannot be sliced"), TACKER_EUNSUPPORTED;
+  if (block_offset < 0 || n_blocks < 0 || block_offset > f->be_full || n_blocks > f->be_full - block_offset)
+    return set_error("PTB slice [%lld, +%lld) outside [0, %lld]", (long long)block_offset, (long long)n_blocks,
+                     (long long)f->be_full),
+           TACKER_EINVAL;
+  FusedParams P = f->P;    // by value: the handle itself is not modified (launchable from any thread)
+  P.be_offset = block_offset;
+  P.be_blocks = n_blocks;
+  P.be.block_offset = (int32_t)block_offset;
+  P.be.orig_blocks = (int32_t)n_blocks;
+  return launch_params(*f, P, reinterpret_cast<cudaStream_t>(stream));
 }
 
 tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be, tacker_stream_t stream) {

@@ -22,6 +22,15 @@ import torch
 from . import tacker as tk
 
 
+def _prefix(desc, n):
+    """Copy of a BE descriptor restricted to its first n original blocks (PTB, Fig. 7)."""
+    import ctypes
+    d = tk.BeDesc()
+    ctypes.memmove(ctypes.addressof(d), ctypes.addressof(desc), ctypes.sizeof(d))
+    d.orig_blocks = n
+    return d
+
+
 def _time(fn, reps=10, stream=None):
     s = stream or torch.cuda.current_stream()
     fn()
@@ -44,6 +53,7 @@ class QosRun:
         self.pairs = {}          # pair key -> fitted coefficients
         self.ws_of = {}          # (app, kernel) -> warp split that fits the budget
         self.pair_err = []       # |pred - meas| / meas of the fused model on the real pairs
+        self.lr_be = {}          # (app, kernel) -> (n_blocks, t_block_ms, t_floor_ms): slice LR
 
     # ------------------------------------------------------------------ calibration (§VI-C)
     def with_io(self):
@@ -73,6 +83,8 @@ class QosRun:
         for a, app in enumerate(self.apps):
             for j, bk in enumerate(app.kernels):
                 self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(None, bk.desc), reps)
+                if self.t_be[(a, j)] >= 0.01 and bk.desc.kind != tk.BE_JDS_SCAN:
+                    self.lr_be[(a, j)] = self._fit_slice_lr(a, j, bk, reps)
         # warp split per BE kernel (NEXT-1): the fastest fused launch with a
         # representative LC kernel among the splits that fit the budget
         tcs = [k for k in self.svc.kernels if k.is_tc]
@@ -127,24 +139,38 @@ class QosRun:
         for pkey in refit:
             self.pairs[pkey] = tk.tacker_pair_fit(pkey)
 
+    def _fit_slice_lr(self, a, j, bk, reps):
+        """Per-kernel LR over PTB slices (§VI-C): standalone time of the first n
+        original blocks, X_cd(n) = t_floor + t_block n, OLS over n in {N/16, N/8, N/4, N/2, N}
+        (the regime a fused slice runs in; one block alone sits on the latency floor)."""
+        full = tk.tacker_be_num_blocks(bk.desc)
+        key = f"be:slice:app{a}:k{j}"
+        ns = sorted({max(1, full // d) for d in (16, 8, 4, 2, 1)})
+        for n in ns:
+            d = _prefix(bk.desc, n)
+            t = self.t_be[(a, j)] if n == full else _time(lambda: tk.tacker_launch_original(None, d), reps)
+            tk.tacker_model_add_sample(key, n, t)
+        slope, icpt = tk.tacker_model_fit(key)
+        return (full, max(slope, 0.0), max(icpt, 0.0))
+
     def _fit_pair(self, k, bk, ws, x_tc, pkey, reps):
         full = tk.tacker_be_num_blocks(bk.desc)
-
-        def prefix(n):
-            d = tk.BeDesc()
-            C_copy = bytes(bk.desc)
-            import ctypes
-            ctypes.memmove(ctypes.addressof(d), C_copy, ctypes.sizeof(d))
-            d.orig_blocks = n
-            return d
+        prefix = lambda n: _prefix(bk.desc, n)
         t_full = self.t_be_of(bk)
-        # BE duration is ~ linear in blocks above its one-block floor (PTB LR)
-        t_one = _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)
-        a = (t_full - t_one) / max(full - 1, 1)
+        # BE duration is ~ linear in blocks above its one-block floor (PTB LR, P:1839-1851): the
+        # slice LR when the kernel has one, else the line through one block and the whole kernel
+        lr = next((v for (a_, j_), v in self.lr_be.items() if self.apps[a_].kernels[j_] is bk), None)
+        if lr is not None and lr[1] > 0:
+            _, a, t0 = lr
+            t_one = t0 + a
+        else:
+            t_one = _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)
+            a = (t_full - t_one) / max(full - 1, 1)
+            t0 = t_one - a
         r_floor = t_one / x_tc
         shift = max(0.0, 1.25 * r_floor - 0.1)
         for r in (0.1 + shift, 0.2 + shift, 1.8 + shift, 1.9 + shift):
-            n = int(round((r * x_tc - t_one) / a)) + 1 if a > 0 else full
+            n = int(round((r * x_tc - t0) / a)) if a > 0 else full
             n = min(max(n, 1), full)
             d = prefix(n)
             f = tk.tacker_fuse(k.lc, d, ws)
@@ -177,8 +203,10 @@ class QosRun:
         for a, app in enumerate(self.apps):
             ks = []
             for j, bk in enumerate(app.kernels):
-                ks.append(tk.BeKernel(is_cd=1, t_pred_ms=self.t_be[(a, j)],
-                                      be=bk.desc, warp_split=self.ws_of.get((a, j), self.ws)))
+                n, tb, tf = self.lr_be.get((a, j), (0, 0.0, 0.0))
+                ks.append(tk.BeKernel(is_cd=1, t_pred_ms=self.t_be[(a, j)], be=bk.desc,
+                                      warp_split=self.ws_of.get((a, j), self.ws),
+                                      n_blocks=n, t_block_ms=tb, t_floor_ms=tf))
             out.append(ks)
         return out
 
@@ -186,7 +214,8 @@ class QosRun:
         return sum(self.t_lc)
 
     # ------------------------------------------------------------------ one managed run
-    def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None):
+    def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None,
+            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False):
         """Poisson arrivals at `load` x the service's peak rate (1 / standalone query time; the
         paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
         stream = torch.cuda.current_stream()
@@ -195,7 +224,8 @@ class QosRun:
         rng = np.random.default_rng(seed)
         gaps = rng.exponential(1.0 / lam, n_queries + warmup)
         cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
-        m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight)
+        m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
+                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused)
         for ks in self.be_apps():
             m.submit_be(ks)
         kernels = self.lc_kernels()
@@ -213,7 +243,8 @@ class QosRun:
         gpu_ms = e0.elapsed_time(e1)
         lat_sorted = np.sort(lat)
         p99 = float(lat_sorted[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)])
-        return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "queries": int(len(lat)),
+        return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "slice_be": bool(slice_be),
+                "reorder_only_unfused": bool(reorder_only_unfused), "queries": int(len(lat)),
                 "lambda_per_s": lam * 1e3, "load": load, "elapsed_ms": gpu_ms,
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
                 # normalised BE throughput: standalone-milliseconds of BE work per wall millisecond

@@ -145,7 +145,7 @@ class _BeUnion(C.Union):
 
 
 class BeDesc(C.Structure):
-    _fields_ = [("kind", C.c_int32), ("orig_blocks", C.c_int32), ("p", _BeUnion)]
+    _fields_ = [("kind", C.c_int32), ("orig_blocks", C.c_int32), ("block_offset", C.c_int32), ("p", _BeUnion)]
 
 
 class Ratio(C.Structure):
@@ -170,7 +170,8 @@ class LcQuery(C.Structure):
 
 
 class BeKernel(C.Structure):
-    _fields_ = [("is_cd", C.c_int32), ("t_pred_ms", C.c_double), ("be", BeDesc), ("warp_split", C.c_int32)]
+    _fields_ = [("is_cd", C.c_int32), ("t_pred_ms", C.c_double), ("be", BeDesc), ("warp_split", C.c_int32),
+                ("n_blocks", C.c_int32), ("t_block_ms", C.c_double), ("t_floor_ms", C.c_double)]
 
 
 class BeApp(C.Structure):
@@ -180,12 +181,14 @@ class BeApp(C.Structure):
 class Decision(C.Structure):
     _fields_ = [("action", C.c_int32), ("query", C.c_int32), ("lc_index", C.c_int32), ("fused_app", C.c_int32),
                 ("n_reorder", C.c_int32), ("reorder_apps", C.c_int32 * MAX_REORDER), ("thr_ms", C.c_double),
-                ("gain_ms", C.c_double), ("t_start_ms", C.c_double), ("t_end_ms", C.c_double)]
+                ("gain_ms", C.c_double), ("t_start_ms", C.c_double), ("t_end_ms", C.c_double),
+                ("fused_blocks", C.c_int64)]
 
 
 class ManagerParams(C.Structure):
     _fields_ = [("direct_eps_ms", C.c_double), ("idle_cap_ms", C.c_double), ("max_inflight", C.c_int32),
-                ("simulate", C.c_int32)]
+                ("simulate", C.c_int32), ("slice_be", C.c_int32), ("slice_ratio", C.c_double),
+                ("reorder_only_unfused", C.c_int32)]
 
 
 class ManagerStats(C.Structure):
@@ -211,6 +214,7 @@ _PROTOS = {
     "tacker_fused_keys": ([_V, C.c_char_p, C.c_char_p, C.c_char_p, C.c_size_t], C.c_int),
     "tacker_fused_rebind": ([_V, C.POINTER(LcDesc), C.POINTER(BeDesc)], C.c_int),
     "tacker_launch_fused": ([_V, _V], C.c_int),
+    "tacker_launch_fused_slice": ([_V, _I64, _I64, _V], C.c_int),
     "tacker_launch_original": ([C.POINTER(LcDesc), C.POINTER(BeDesc), _V], C.c_int),
     "tacker_model_add_sample": ([_S, _D, _D], C.c_int),
     "tacker_model_fit": ([_S, C.POINTER(_D), C.POINTER(_D)], C.c_int),
@@ -478,6 +482,10 @@ class Fused:
     def launch(self, stream=None):
         _chk(_lib.tacker_launch_fused(self.h, _stream(stream)))
 
+    def launch_slice(self, block_offset, n_blocks, stream=None):
+        """The LC part plus BE original blocks [block_offset, block_offset + n_blocks) only."""
+        _chk(_lib.tacker_launch_fused_slice(self.h, block_offset, n_blocks, _stream(stream)))
+
     def rebind(self, lc=None, be=None):
         _chk(_lib.tacker_fused_rebind(self.h, C.byref(lc) if lc is not None else None,
                                       C.byref(be) if be is not None else None))
@@ -498,6 +506,10 @@ def tacker_fuse(lc: LcDesc, be: BeDesc | None, warp_split: int, block_ratio=(0, 
 
 def tacker_launch_fused(f: Fused, stream=None):
     f.launch(stream)
+
+
+def tacker_launch_fused_slice(f: Fused, block_offset: int, n_blocks: int, stream=None):
+    f.launch_slice(block_offset, n_blocks, stream)
 
 
 def tacker_launch_original(lc: LcDesc | None, be: BeDesc | None, stream=None):
@@ -563,9 +575,10 @@ class Manager:
     """Owning wrapper of tacker_manager_t."""
 
     def __init__(self, policy=POLICY_TACKER, stream=None, simulate=False, direct_eps_ms=0.0, idle_cap_ms=0.0,
-                 max_inflight=2):
+                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False):
         self.h = C.c_void_p()
-        self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0)
+        self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0,
+                                    1 if slice_be else 0, slice_ratio, 1 if reorder_only_unfused else 0)
         _chk(_lib.tacker_manager_create(policy, C.byref(self.params), _stream(stream), C.byref(self.h)))
         self._keep = []
 

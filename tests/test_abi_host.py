@@ -221,3 +221,63 @@ def test_manager_simulation_matches_reference(tk, policy):
     assert abs(m.stats().be_work_ms - work) < 1e-9
     m.prepare()            # no-op on the simulated GPU
     m.prepare([lc_kernel(tk, True, 1.0)])
+
+
+def be_kernel_sliced(tk, t, n, floor, ws=16):
+    b = be_kernel(tk, t, ws)
+    b.n_blocks, b.t_floor_ms, b.t_block_ms = n, floor, (t - floor) / n
+    return b
+
+
+@pytest.mark.parametrize("mode", ["opportune", "fixed", "opportune_literal"])
+def test_manager_slicing_matches_reference(tk, mode):
+    """PTB slicing (reading 13): the C manager's decisions (incl. slice sizes), latencies and BE
+    work equal the discrete-event reference's."""
+    tk.tacker_model_clear()
+    tau = lambda r: max(1 + 0.25 * r, 0.4 + 0.93 * r)     # r* = 0.6 / 0.68
+    fit_pair_closed_form(tk, tau)
+    fuse_pred = lambda ttc, tcd: ttc * tau(tcd / ttc)
+    ratio = 1.3 if mode == "fixed" else 0.0
+    literal = mode == "opportune_literal"
+    rng = np.random.default_rng(5)
+    arrivals = np.cumsum(rng.exponential(7.0, 50))
+    shapes = [[(True, 1.21), (False, 0.3), (True, 0.83), (True, 1.97)], [(True, 0.52), (True, 0.49)]]
+    app_ts = [[(1.53, 64, 0.05), (0.71, 0, 0.0)], [(3.07, 200, 0.11)], [(0.43, 1, 0.4), (2.51, 37, 0.2)]]
+    m = tk.Manager(tk.POLICY_TACKER, simulate=True, idle_cap_ms=2.0, slice_be=True, slice_ratio=ratio,
+                   reorder_only_unfused=literal)
+    qs = []
+    for i, tt in enumerate(arrivals):
+        sh = shapes[i % 2]
+        m.submit_lc([lc_kernel(tk, tc, d) for tc, d in sh], float(tt))
+        qs.append(mr.Query(i, float(tt), list(sh)))
+    apps = []
+    for ts in app_ts:
+        ks, rk = [], []
+        for T, n, fl in ts:
+            if n > 1:
+                ks.append(be_kernel_sliced(tk, T, n, fl))
+                rk.append((True, T, n, (T - fl) / n, fl))
+            else:
+                ks.append(be_kernel(tk, T))
+                rk.append((True, T))
+        m.submit_be(ks)
+        apps.append(mr.App(rk))
+    r_opp = 0.6 / 0.68
+    ref = mr.simulate(qs, apps, 50.0, mr.TACKER, fuse_pred, idle_cap=2.0, slice_be=True, slice_ratio=ratio,
+                      opp_ratio=lambda a: r_opp, reorder_only_unfused=literal)
+    got = []
+    for _ in range(100000):
+        if m.stats().lc_queries_done == len(arrivals):
+            break
+        d = m.step(50.0)
+        if d.action in (tk.DEC_FUSED, tk.DEC_ORIGINAL_LC, tk.DEC_REORDER_BE, tk.DEC_IDLE_BE):
+            got.append((d.action, d.fused_app, d.fused_blocks if d.action == tk.DEC_FUSED else -1,
+                        tuple(d.reorder_apps[:d.n_reorder])))
+    exp = [(x.action, x.fused_app, x.blocks if x.action == mr.FUSED else -1, tuple(x.reorder))
+           for x in ref["decisions"]]
+    assert got == exp
+    assert any(x[0] == mr.FUSED and x[2] > 0 for x in exp), "no slice was fused"
+    for i in range(len(arrivals)):
+        assert abs(m.latency(i) - ref["latency"][i]) < 1e-9
+    assert abs(m.stats().be_work_ms - ref["be_work"]) < 1e-9
+    assert m.stats().be_kernels_done == sum(ref["be_completed"])

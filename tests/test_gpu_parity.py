@@ -201,9 +201,10 @@ def test_stencil_scalar_path_and_large(tk, ws):
 @pytest.mark.parametrize("ws", [4, 12, 24])
 @pytest.mark.parametrize("orig_blocks", [0, 301])
 def test_mriq_static_split_chunks(tk, ws, orig_blocks):
-    # fused mri-q Q uses the static even split with up to 4 blocks per thread (BeCoarsen): 666
-    # blocks over 148 CTAs gives 4-5 per CTA, so at ws=4 a slot runs a 4-chunk plus a 1-chunk,
-    # at ws=24 slots get 0 or 1; orig_blocks = 301 exercises the PTB prefix on the same split
+    # fused mri-q Q uses the static even split with up to kCoarsen blocks per thread: 2662 blocks
+    # of 32 voxels over 148 CTAs gives 17-18 per CTA, several per slot at every split, with
+    # coarsened chunks and 1-block tails; orig_blocks = 301 exercises the PTB prefix (2 per CTA,
+    # slots with 0 or 1 block)
     N, nk = 44, 256
     d = synth.mriq_inputs(N, nk, 11)
     pm = (d["phiR"].astype(np.float32) ** 2 + d["phiI"].astype(np.float32) ** 2).astype(np.float32)
@@ -221,7 +222,39 @@ def test_mriq_static_split_chunks(tk, ws, orig_blocks):
     f.launch()
     qr_o, qi_o, qr_f, qi_f = (host(o) for o in outs)
     assert qr_f.tobytes() == qr_o.tobytes() and qi_f.tobytes() == qi_o.tobytes()
-    n = N ** 3 if orig_blocks == 0 else orig_blocks * 128
+    n = N ** 3 if orig_blocks == 0 else orig_blocks * 32     # 32 voxels per original block
     rr, ri, sr, si = obe.mriq_q(d["x"][:n], d["y"][:n], d["z"][:n], d["kx"], d["ky"], d["kz"], pm)
     assert max_rel_err(qr_o[:n], rr, sr) <= 1e-5 and max_rel_err(qi_o[:n], ri, si) <= 1e-5
     assert np.all(qr_o[n:] == 0) and np.all(qi_o[n:] == 0)
+
+
+@pytest.mark.parametrize("kind", FUSE_KINDS)
+def test_ptb_slices_compose_to_whole_kernel(tk, kind):
+    # PTB slices (reading 13): a fused slice, an original slice and a fused slice that partition
+    # [0, N) give the whole original kernel's bytes; every slice run once
+    import ctypes
+    c = be_case(getattr(tk, kind), seed=3)
+    c["reset"]()
+    tk.tacker_launch_original(None, c["desc"])
+    whole = [host(o).copy() for o in c["outs"]]
+    c["check"](whole)
+    N = tk.tacker_be_num_blocks(c["desc"])
+    a, b = max(1, N // 3), max(1, N // 3) + max(1, N // 4)
+    assert 0 < a < b < N, (N, a, b)
+    A, B = synth.lc_gemm_inputs(256, 256, 128, seed=1)
+    D = torch.zeros(256, 256, device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], 8)
+    mid = tk.BeDesc()
+    ctypes.memmove(ctypes.addressof(mid), ctypes.addressof(c["desc"]), ctypes.sizeof(mid))
+    mid.block_offset, mid.orig_blocks = a, b - a
+    for _ in range(2):
+        c["reset"]()
+        f.launch_slice(0, a)
+        tk.tacker_launch_original(None, mid)
+        f.launch_slice(b, N - b)
+        for w, o in zip(whole, c["outs"]):
+            assert host(o).tobytes() == w.tobytes()
+    with pytest.raises(tk.TackerError):
+        f.launch_slice(b, N - b + 1)
+    ref, S = olc.lc_gemm(A, B)
+    assert max_rel_err(host(D), ref, S) <= 1e-2

@@ -174,6 +174,34 @@ def test_manager_qos_holds_and_tacker_beats_baymax():
     assert out[mr.TACKER] > out[mr.BAYMAX]
 
 
+def test_manager_slice_to_opportune_ratio():
+    """Reading 13, hand-computed: TC kernel 2 ms; BE head 10 ms = 100 blocks,
+    X_cd(n) = 0.1 n; tau(r) = max(1 + 0.1 r, 0.5 + r) -> r* = 0.5/0.9 = 5/9 (Fig. 10 inflection).
+    Slice n = ceil(r* 2 / 0.1) = ceil(11.1) = 12 blocks: Tcd = 1.2, Tk_fuse = 2 tau(0.6) = 2.2,
+    Tgain = 1.2 - 0.2 = 1.0 (Eq. 8 holds), Thr 48 -> 47.8; the query ends at 2.2 and the idle GPU
+    then runs the other 88 blocks (X_cd(88) = 8.8 ms, ending at 11.0) before a second query
+    arrives at 20 (one 1 ms CUDA-core kernel, behind which the app's next 30 ms kernel is
+    reordered).  Whole-kernel fusion has the same Tgain (Tk_fuse = 2 tau(5) = 11, Tgain =
+    10 - 9 = 1) but costs 9 ms of headroom and an 11 ms query."""
+    tau = lambda r: max(1 + 0.1 * r, 0.5 + r)
+    fp = lambda ttc, tcd: ttc * tau(tcd / ttc)
+    for sliced, lat, thr_after, blocks in ((True, 2.2, 47.8, 12), (False, 11.0, 39.0, -1)):
+        qs = [mr.Query(0, 0.0, [(True, 2.0)]), mr.Query(1, 20.0, [(False, 1.0)])]
+        app = mr.App([(True, 10.0, 100, 0.1, 0.0), (True, 30.0)])
+        res = mr.simulate(qs, [app], 50.0, mr.TACKER, fp, slice_be=sliced, opp_ratio=lambda a: 5 / 9,
+                          idle_cap=9.0)
+        d0 = res["decisions"][0]
+        assert d0.action == mr.FUSED and d0.blocks == blocks
+        assert abs(d0.gain - 1.0) < 1e-12 and abs(d0.thr - thr_after) < 1e-12
+        assert abs(res["latency"][0] - lat) < 1e-12
+        if sliced:
+            d1 = res["decisions"][1]
+            assert d1.action == mr.IDLE_BE and d1.reorder == [0]
+            assert [e for e in res["timeline"] if e[0] == "be"][0][4:] == (2.2, 2.2 + 8.8)
+        # both kernels complete (the 30 ms one is reordered behind query 1): 10 + 30 ms of work
+        assert abs(res["be_work"] - 40.0) < 1e-12 and res["be_completed"] == [2]
+
+
 # ------------------------------------------------------------------ metrics
 def test_overlap_rate_bounds():
     assert metrics.overlap_rate(1.0, 1.0, 1.0) == 0.5      # perfect overlap

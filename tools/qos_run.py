@@ -52,6 +52,8 @@ def main():
     ap.add_argument("--ws", type=int, default=24)
     ap.add_argument("--qos", type=float, default=50.0)
     ap.add_argument("--io", action="store_true", help="each query copies its input H2D and result D2H")
+    ap.add_argument("--variants", default="baymax,tacker,tacker_slice,tacker_slice_literal")
+    ap.add_argument("--slice-ratio", type=float, default=0.0, help="fixed slice load ratio (0: opportune r*)")
     args = ap.parse_args()
     svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
     apps = build_apps(args.be.split(","))
@@ -61,11 +63,19 @@ def main():
         q.with_io()
     q.calibrate()
     res = {}
-    for pol in (tk.POLICY_BAYMAX, tk.POLICY_TACKER):
-        r = q.run(pol, args.queries, load=args.load, warmup=args.warmup)
-        res[r["policy"]] = r
-    res["improvement_eq10"] = res["tacker"]["be_kernels_per_s"] / res["baymax"]["be_kernels_per_s"] - 1.0
-    res["improvement_eq10_normalised"] = res["tacker"]["be_norm_thpt"] / res["baymax"]["be_norm_thpt"] - 1.0
+    variants = {"baymax": (tk.POLICY_BAYMAX, {}), "tacker": (tk.POLICY_TACKER, {}),
+                "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
+                "tacker_slice_literal": (tk.POLICY_TACKER, {"slice_be": True, "reorder_only_unfused": True})}
+    for name in args.variants.split(","):
+        pol, kw = variants[name]
+        if args.slice_ratio > 0 and kw.get("slice_be"):
+            kw = dict(kw, slice_ratio=args.slice_ratio)
+        res[name] = q.run(pol, args.queries, load=args.load, warmup=args.warmup, **kw)
+    for name in res:
+        if name != "baymax" and "baymax" in res:
+            res[name]["improvement_eq10"] = res[name]["be_kernels_per_s"] / res["baymax"]["be_kernels_per_s"] - 1.0
+            res[name]["improvement_eq10_normalised"] = res[name]["be_norm_thpt"] / res["baymax"]["be_norm_thpt"] - 1.0
+    res["slice_lr"] = {f"{a}.{j}": v for (a, j), v in q.lr_be.items()}
     res["pairs_fitted"] = len(q.pairs)
     res["pair_pred_err"] = {"max": max(q.pair_err), "mean": sum(q.pair_err) / len(q.pair_err), "n": len(q.pair_err)}
     print(json.dumps(res))
