@@ -66,7 +66,10 @@ int tacker_device_sm_count(void);
  */
 typedef enum { TACKER_LC_NONE = 0, TACKER_LC_GEMM_F16 = 1, TACKER_LC_CONV_F16 = 2 } tacker_lc_kind;
 enum { TACKER_F32 = 0, TACKER_F16 = 1 };
-enum { TACKER_EPI_BIAS = 1, TACKER_EPI_RELU = 2, TACKER_EPI_RESIDUAL = 4 };
+enum { TACKER_EPI_BIAS = 1, TACKER_EPI_RELU = 2, TACKER_EPI_RESIDUAL = 4,
+       /* B (weights) is not written by any kernel on the stream: a launch may fetch its first
+        * B k-blocks before waiting for the stream predecessor (programmatic dependent launch) */
+       TACKER_LC_B_CONST = 8 };
 
 typedef struct {
   int32_t kind;                       /* tacker_lc_kind */
@@ -260,6 +263,13 @@ tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, co
 tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream);
 tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be,
                                      tacker_stream_t stream);
+/* Programmatic dependent launch (default on): every launch of this library may begin its
+ * prologue (CTA scheduling, barrier / TMEM setup, TACKER_LC_B_CONST weight fetches) while the
+ * previous kernel on the stream is still running; each kernel waits for its predecessor
+ * (griddepcontrol.wait) before touching any other global memory, so stream order semantics are
+ * unchanged.  0 disables it (plain stream serialization).  Process-wide. */
+tacker_status tacker_set_launch_overlap(int32_t enable);
+
 /* One fused launch of handle f whose BE part runs only the PTB slice [block_offset,
  * block_offset + n_blocks) of the handle's BE kernel (the LC part is unchanged; n_blocks 0 = no
  * BE work).  The handle is not modified.  EINVAL if the slice leaves the whole-problem range. */

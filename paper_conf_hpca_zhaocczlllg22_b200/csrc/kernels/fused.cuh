@@ -88,33 +88,68 @@ struct LcGemm {
     nt = t % L.tiles_n;
   }
 
+  static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
+    return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
+  }
+  // B (weights) k-block kb of N-tile nt
+  static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
+    const LcParams &L = P.lc;
+    if (implicit_conv(L)) {
+      // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
+      const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
+      tma_load_2d(&P.tmap_b, bar, sb, rs * L.c + cb * kBK, nt * BN);
+    } else {
+      tma_load_2d(&P.tmap_b, bar, sb, kb * kBK, nt * BN);
+    }
+  }
+  // A (activations) k-block kb of M-tile mt
+  static __device__ __forceinline__ void load_a(const FusedParams &P, uint64_t *bar, uint8_t *sa, int kb, int mt) {
+    const LcParams &L = P.lc;
+    if (implicit_conv(L)) {
+      // k-block -> (filter tap r,s ; channel block cb); A = shifted NHWC window (implicit im2col)
+      const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
+      const int rr = rs / L.s, ss = rs % L.s;
+      const int img = mt / (L.tiles_p * L.tiles_q);
+      const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
+      const int h0 = pt * L.tp * L.stride - L.pad + rr;
+      const int w0 = qt * L.tq * L.stride - L.pad + ss;
+      tma_load_4d(&P.tmap_a, bar, sa, cb * kBK, w0, h0, img);
+    } else {
+      tma_load_2d(&P.tmap_a, bar, sa, kb * kBK, mt * kBM);
+    }
+  }
+
   static __device__ __forceinline__ void producer(const FusedParams &P, uint8_t *lc, const Bars &bb) {
     const LcParams &L = P.lc;
+    // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
+    // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
+    int pre = 0;
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_tiles) {
+      int mt, nt;
+      tile_coords(L, blockIdx.x, mt, nt);
+      pre = min(P.stages, L.num_kb);
+      for (int kb = 0; kb < pre; ++kb) {
+        mbar_arrive_expect_tx(&bb.full[kb], kStage);
+        load_b(P, &bb.full[kb], lc + kb * kStage + kStageA, kb, nt);
+      }
+    }
+    griddep_wait();
     int stage = 0;
     uint32_t phase = 0;
     for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
       int mt, nt;
       tile_coords(L, t, mt, nt);
       for (int kb = 0; kb < L.num_kb; ++kb) {
-        mbar_wait(&bb.empty[stage], phase ^ 1);
         uint8_t *sa = lc + stage * kStage;
         uint8_t *sb = sa + kStageA;
-        mbar_arrive_expect_tx(&bb.full[stage], kStage);
-        if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-          // k-block -> (filter tap r,s ; channel block cb); A = shifted NHWC window (implicit im2col)
-          const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
-          const int rr = rs / L.s, ss = rs % L.s;
-          const int img = mt / (L.tiles_p * L.tiles_q);
-          const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
-          const int h0 = pt * L.tp * L.stride - L.pad + rr;
-          const int w0 = qt * L.tq * L.stride - L.pad + ss;
-          tma_load_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, w0, h0, img);
-          // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
-          tma_load_2d(&P.tmap_b, &bb.full[stage], sb, rs * L.c + cb * kBK, nt * BN);
+        if (pre > 0) {
+          --pre;              // first tile, stage == kb: B already in flight, its bytes expected
         } else {
-          tma_load_2d(&P.tmap_a, &bb.full[stage], sa, kb * kBK, mt * kBM);
-          tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);
+          mbar_wait(&bb.empty[stage], phase ^ 1);
+          mbar_arrive_expect_tx(&bb.full[stage], kStage);
+          load_b(P, &bb.full[stage], sb, kb, nt);
         }
+        load_a(P, &bb.full[stage], sa, kb, mt);
         if (++stage == P.stages) {
           stage = 0;
           phase ^= 1;
@@ -159,6 +194,7 @@ struct LcGemm {
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;          // TMEM lanes 32*quarter .. +31
     const int row_in_tile = quarter * 32 + lane_id();
+    griddep_wait();                             // residual / D of earlier kernels
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
@@ -249,6 +285,7 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   // LC tiles sit on the lowest CTA indices (tile t on CTA t mod grid): hand them the smaller BE
   // shares by numbering CTAs from the top.
   const int64_t cta = (int64_t)gridDim.x - 1 - blockIdx.x;
+  griddep_wait();
   be_init<BE_KIND>(body_smem, tid, bar);
   if constexpr (kC > 1) {
     // Coarsened (compute-bound, uniform-cost) bodies: static even split.  CTA c owns original
@@ -287,6 +324,7 @@ template <int BN, int BE_KIND>
 __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  griddep_launch_dependents();   // the next kernel on the stream may start its prologue
   uint8_t *lc = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *be_smem = lc + P.lc_smem_bytes;
   // BE warps come first and the LC warps last: the B200 warp arbiter issues highest-warp-id
@@ -351,6 +389,8 @@ struct alignas(64) BeOrigParams {
 template <int BE_KIND>
 __global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ BeOrigParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  griddep_launch_dependents();
+  griddep_wait();
   be_init<BE_KIND>(smem_raw, threadIdx.x, 1u);
   be_run<BE_KIND>(P.d, (int64_t)P.d.block_offset + blockIdx.x, threadIdx.x, 1u, smem_raw, &P.tmap);
 }

@@ -19,6 +19,17 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t cnt) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(cnt) : "memory");
 }
 
+// ---------------------------------------------------------------- programmatic dependent launch
+// A kernel launched with programmatic stream serialization may start while its stream
+// predecessor is still running: launch_dependents lets the NEXT kernel's CTAs be scheduled,
+// wait blocks until every prerequisite grid has completed and its memory is visible.  Every
+// thread calls wait before it touches global memory that an earlier kernel may write or read
+// (no-ops for a normally launched kernel).
+__device__ __forceinline__ void griddep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // ---------------------------------------------------------------- mbarrier
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");

@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -498,9 +499,26 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   return TACKER_OK;
 }
 
+static std::atomic<int> g_overlap{1};
+
+// cudaLaunchKernelEx with programmatic stream serialization (PDL) unless disabled
+template <typename Param>
+static cudaError_t launch_ex(void (*fn)(Param), dim3 grid, dim3 block, int smem, cudaStream_t s, const Param &p) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = g_overlap.load(std::memory_order_relaxed) ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, fn, p);
+}
+
 static tacker_status launch_params(const tacker_fused_s &F, FusedParams &P, cudaStream_t s) {
-  void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(F.fn), dim3(F.grid), dim3(F.block), args, F.smem, s);
+  cudaError_t e = launch_ex(F.fn, dim3(F.grid), dim3(F.block), F.smem, s, P);
   if (e != cudaSuccess) return cuda_fail("launch fused_kernel", e);
   return TACKER_OK;
 }
@@ -510,6 +528,11 @@ static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) { return lau
 extern "C" {
 
 const char *tacker_last_error(void) { return g_err.c_str(); }
+
+tacker_status tacker_set_launch_overlap(int32_t enable) {
+  g_overlap.store(enable ? 1 : 0);
+  return TACKER_OK;
+}
 const char *tacker_version(void) { return "tacker-b200 0.1 (sm_100a)"; }
 int tacker_device_sm_count(void) { return sm_count(); }
 
@@ -663,9 +686,8 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
     BeOrigParams op;
     op.d = *be;
     if ((st = encode_be_tmap(*be, &op.tmap))) return st;
-    void *args[] = {&op};
     if (blocks > 0x7fffffffLL) return set_error("too many blocks"), TACKER_EUNSUPPORTED;
-    cudaError_t e = cudaLaunchKernel(reinterpret_cast<const void *>(fn), dim3((unsigned)blocks), dim3(128), args, smem, s);
+    cudaError_t e = launch_ex(fn, dim3((unsigned)blocks), dim3(128), smem, s, op);
     if (e != cudaSuccess) return cuda_fail("launch be_original_kernel", e);
   }
   return TACKER_OK;

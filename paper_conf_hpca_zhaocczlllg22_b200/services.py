@@ -63,7 +63,8 @@ def resnet50_service(batch: int = 1, seed: int = 2022, convs=None) -> LcService:
         M, N, K = cs.gemm_mnk
         byt = 2 * x.size + 2 * w.size + 2 * out.numel()
         if cs.c % 64 == 0 or (cs.r == 1 and cs.s == 1 and cs.stride == 1):
-            ks.append(LcKernelSpec(cs.name, True, lc=tk.lc_conv(dx, dw, out, cs.stride, cs.pad, bias=db, relu=True),
+            lc = tk.lc_conv(dx, dw, out, cs.stride, cs.pad, bias=db, relu=True, b_const=True)
+            ks.append(LcKernelSpec(cs.name, True, lc=lc,
                                    flops=2 * M * N * K, bytes=byt, conv=cs))
             bufs += [dx, dw, db, out]
         else:   # conv1: explicit im2col (LC CD kernel) + GEMM (LC TC kernel)
@@ -76,7 +77,8 @@ def resnet50_service(batch: int = 1, seed: int = 2022, convs=None) -> LcService:
                                    cd=tk.be_im2col(dx, cols, cs.r, cs.s, cs.stride, cs.pad, Kpad),
                                    bytes=2 * x.size + 2 * M * Kpad, conv=cs))
             ks.append(LcKernelSpec(cs.name + ".gemm", True,
-                                   lc=tk.lc_gemm(cols, dwf, out.view(M, cs.k), M=M, N=cs.k, K=Kpad, bias=db, relu=True),
+                                   lc=tk.lc_gemm(cols, dwf, out.view(M, cs.k), M=M, N=cs.k, K=Kpad, bias=db, relu=True,
+                                                 b_const=True),
                                    flops=2 * M * N * K, bytes=2 * M * Kpad + 2 * wf.size + 2 * out.numel(), conv=cs))
             bufs += [dx, dw, db, out, cols, dwf]
     return LcService(f"resnet50_b{batch}", ks, bufs, ins, outs[-1:])
@@ -100,7 +102,7 @@ def bert_service(seq: int = 128, seed: int = 2024, layers: int = 1) -> LcService
             B = (B.astype(np.float32) / np.sqrt(K)).astype(np.float16)
             dA, dB = _dev(A), _dev(B)
             D = torch.empty(M, N, dtype=torch.float16, device="cuda")
-            ks.append(LcKernelSpec(f"l{li}.{name}", True, lc=tk.lc_gemm(dA, dB, D), flops=2 * M * N * K,
+            ks.append(LcKernelSpec(f"l{li}.{name}", True, lc=tk.lc_gemm(dA, dB, D, b_const=True), flops=2 * M * N * K,
                                    bytes=2 * (M * K + N * K + M * N)))
             bufs += [dA, dB, D]
     return LcService(f"bert_base_s{seq}", ks, bufs)

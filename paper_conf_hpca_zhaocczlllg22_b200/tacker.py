@@ -24,7 +24,7 @@ OK, EINVAL, ERESOURCE, EUNSUPPORTED, ECUDA, ENOMODEL, ENOMEM = 0, -1, -2, -3, -4
 STATUS_NAMES = {0: "OK", -1: "EINVAL", -2: "ERESOURCE", -3: "EUNSUPPORTED", -4: "ECUDA", -5: "ENOMODEL", -6: "ENOMEM"}
 LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
-EPI_BIAS, EPI_RELU, EPI_RESIDUAL = 1, 2, 4
+EPI_BIAS, EPI_RELU, EPI_RESIDUAL, LC_B_CONST = 1, 2, 4, 8
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
  BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY, BE_JDS_COUNT, BE_JDS_SCAN,
  BE_JDS_PERM, BE_JDS_FILL) = range(19)
@@ -215,6 +215,7 @@ _PROTOS = {
     "tacker_fused_rebind": ([_V, C.POINTER(LcDesc), C.POINTER(BeDesc)], C.c_int),
     "tacker_launch_fused": ([_V, _V], C.c_int),
     "tacker_launch_fused_slice": ([_V, _I64, _I64, _V], C.c_int),
+    "tacker_set_launch_overlap": ([_I32], C.c_int),
     "tacker_launch_original": ([C.POINTER(LcDesc), C.POINTER(BeDesc), _V], C.c_int),
     "tacker_model_add_sample": ([_S, _D, _D], C.c_int),
     "tacker_model_fit": ([_S, C.POINTER(_D), C.POINTER(_D)], C.c_int),
@@ -259,31 +260,33 @@ def _stream(s):
 
 
 # ----------------------------------------------------------------------------- descriptor builders
-def lc_gemm(A, B, D, M=None, N=None, K=None, bias=None, relu=False, residual=None, tile_n=0) -> LcDesc:
-    """D[M,N] = A[M,K] . B[N,K]^T (+bias)(+residual)(relu); A, B fp16; D fp32 or fp16."""
+def lc_gemm(A, B, D, M=None, N=None, K=None, bias=None, relu=False, residual=None, tile_n=0,
+            b_const=False) -> LcDesc:
+    """D[M,N] = A[M,K] . B[N,K]^T (+bias)(+residual)(relu); A, B fp16; D fp32 or fp16.
+    b_const: B is never written by a kernel on the stream (weights; TACKER_LC_B_CONST)."""
     import torch
     M = A.shape[0] if M is None else M
     K = A.shape[1] if K is None else K
     N = B.shape[0] if N is None else N
     d = LcDesc(kind=LC_GEMM_F16, M=M, N=N, K=K, A=_ptr(A), B=_ptr(B), D=_ptr(D),
                d_dtype=F16 if D.dtype == torch.float16 else F32, tile_n=tile_n)
-    _epi(d, bias, relu, residual)
+    _epi(d, bias, relu, residual, b_const)
     return d
 
 
-def lc_conv(x, w, out, stride, pad, bias=None, relu=False, residual=None, tile_n=0) -> LcDesc:
+def lc_conv(x, w, out, stride, pad, bias=None, relu=False, residual=None, tile_n=0, b_const=False) -> LcDesc:
     """NHWC x [n,h,w,c] fp16, KRSC w [k,r,s,c] fp16 -> NHWC out [n,p,q,k]."""
     import torch
     n, h, wd, c = x.shape
     k, r, s, _ = w.shape
     d = LcDesc(kind=LC_CONV_F16, n=n, h=h, w=wd, c=c, k=k, r=r, s=s, stride=stride, pad=pad, A=_ptr(x), B=_ptr(w),
                D=_ptr(out), d_dtype=F16 if out.dtype == torch.float16 else F32, tile_n=tile_n)
-    _epi(d, bias, relu, residual)
+    _epi(d, bias, relu, residual, b_const)
     return d
 
 
-def _epi(d, bias, relu, residual):
-    f = 0
+def _epi(d, bias, relu, residual, b_const=False):
+    f = LC_B_CONST if b_const else 0
     if bias is not None:
         d.bias = _ptr(bias)
         f |= EPI_BIAS
@@ -506,6 +509,11 @@ def tacker_fuse(lc: LcDesc, be: BeDesc | None, warp_split: int, block_ratio=(0, 
 
 def tacker_launch_fused(f: Fused, stream=None):
     f.launch(stream)
+
+
+def tacker_set_launch_overlap(enable: bool):
+    """Programmatic dependent launch for every launch of the library (default on)."""
+    _chk(_lib.tacker_set_launch_overlap(1 if enable else 0))
 
 
 def tacker_launch_fused_slice(f: Fused, block_offset: int, n_blocks: int, stream=None):

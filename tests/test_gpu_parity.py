@@ -258,3 +258,38 @@ def test_ptb_slices_compose_to_whole_kernel(tk, kind):
         f.launch_slice(b, N - b + 1)
     ref, S = olc.lc_gemm(A, B)
     assert max_rel_err(host(D), ref, S) <= 1e-2
+
+
+def test_launch_overlap_keeps_stream_order(tk):
+    """Programmatic dependent launch: a chain where every kernel reads its predecessor's output
+    (LC GEMM -> LC GEMM on the fp16 result, stencil ping-pong sweeps fused with them, an original
+    BE sweep in between) gives the same bytes with overlap on and off."""
+    M = N = K = 512
+    A, B1 = synth.lc_gemm_inputs(M, N, K, seed=21)
+    _, B2 = synth.lc_gemm_inputs(M, N, K, seed=22)
+    S = synth.stencil_inputs(132, 64, 40, 23)
+
+    def run():
+        dA, dB1, dB2 = t(A), t(B1), t(B2)
+        D1 = torch.zeros(M, N, dtype=torch.float16, device=dev())
+        D2 = torch.zeros(M, N, dtype=torch.float16, device=dev())
+        s0, s1 = t(S), torch.zeros(S.shape, device=dev())
+        st01, st10 = tk.be_stencil(s0, s1), tk.be_stencil(s1, s0)
+        g1 = tk.lc_gemm(dA, dB1, D1, b_const=True)
+        g2 = tk.lc_gemm(D1, dB2, D2, b_const=True)
+        f1, f2 = tk.tacker_fuse(g1, st01, 8), tk.tacker_fuse(g2, st10, 8)
+        torch.cuda.synchronize()
+        for _ in range(5):
+            f1.launch()                                   # D1 = A B1 ; s1 = sweep(s0)
+            f2.launch()                                   # D2 = D1 B2 ; s0 = sweep(s1)
+            tk.tacker_launch_original(None, st01)         # s1 = sweep(s0)
+            tk.tacker_launch_original(g2, st10)           # D2 again ; s0 = sweep(s1)
+        return host(D2).tobytes(), host(s0).tobytes()
+
+    tk.tacker_set_launch_overlap(False)
+    try:
+        ref = run()
+    finally:
+        tk.tacker_set_launch_overlap(True)
+    for _ in range(3):
+        assert run() == ref
