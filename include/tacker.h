@@ -69,7 +69,10 @@ enum { TACKER_F32 = 0, TACKER_F16 = 1 };
 enum { TACKER_EPI_BIAS = 1, TACKER_EPI_RELU = 2, TACKER_EPI_RESIDUAL = 4,
        /* B (weights) is not written by any kernel on the stream: a launch may fetch its first
         * B k-blocks before waiting for the stream predecessor (programmatic dependent launch) */
-       TACKER_LC_B_CONST = 8 };
+       TACKER_LC_B_CONST = 8,
+       /* never split K (by default a GEMM with <= #SMs/2 tiles and >= 4 k-blocks is split
+        * into <= #SMs units with an in-kernel deterministic fixup, see tacker_fused_info) */
+       TACKER_LC_NO_SPLIT = 16 };
 
 typedef struct {
   int32_t kind;                       /* tacker_lc_kind */
@@ -244,6 +247,7 @@ typedef struct {
   int32_t lc_tile_m, lc_tile_n, lc_tile_k, lc_stages, lc_acc_stages, tmem_cols;
   int64_t lc_tiles, be_blocks;
   int32_t be_smem_per_vblock, regs_per_thread;
+  int32_t lc_splits;         /* split-K factor of the LC part (1 = none) */
 } tacker_fused_info_t;
 tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *out);
 /* Model-store keys of the handle's LC kernel, BE kernel and fused pair (for the predictor). */
@@ -415,6 +419,10 @@ typedef struct {
   /* sum of the standalone (predicted) durations of the BE kernels issued: BE work in original-
    * kernel milliseconds, so throughput can be normalised across BE apps of different length */
   double be_work_ms;
+  /* GPU mode: host time of the manager loop (ms): event polling, CUDA launch + event-record
+   * calls, and everything else in tacker_manager_step (decisions, bookkeeping) */
+  double host_poll_ms, host_launch_ms, host_decide_ms;
+  int64_t host_steps;        /* tacker_manager_step calls */
 } tacker_manager_stats;
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
 /* Completion time (manager clock) of a finished query, or -1 if unfinished. */

@@ -25,6 +25,7 @@ constexpr int kLcWarps = 6;
 constexpr int kBM = 128;   // UMMA M
 constexpr int kBK = 64;    // one 128-byte swizzle row of fp16
 constexpr int kUK = 16;    // UMMA K for kind::f16
+constexpr uint32_t kLcEpiBar = 15;   // named barrier of the 4 LC epilogue warps (BE uses 1..14)
 
 struct LcParams {
   int32_t kind;            // tacker_lc_kind (0 = no LC part)
@@ -40,6 +41,13 @@ struct LcParams {
   int32_t tp, tq;          // output tile = tp x tq positions (tp*tq == 128)
   int32_t tiles_p, tiles_q, c_blocks;
   int32_t conv_direct_gemm;  // 1x1 stride-1 conv handled as a plain GEMM over [n*h*w, c]
+  // split-K: work unit u = (tile u / splits, k-blocks [s kb_per_split, (s+1) kb_per_split) of split
+  // s = u % splits).  splits > 1 only when every unit has its own CTA (num_units <= grid): the
+  // splits of a tile write fp32 partials, meet on a counter, then each reduces 1/splits of the tile
+  // in split order (deterministic) and runs the epilogue on it.
+  int32_t splits, kb_per_split, num_units;
+  float *part;             // [num_tiles * splits][kBM][BN] fp32 partial tiles
+  uint32_t *cnt;           // [2 * num_tiles]: arrivals, finished reductions (self-resetting)
 };
 
 struct BeWork {
@@ -77,6 +85,9 @@ struct LcGemm {
     uint64_t *full, *empty, *tfull, *tempty;
     uint32_t *tmem_holder;
   };
+  static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
+    return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
+  }
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * kStage);
     return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4)};
@@ -87,10 +98,49 @@ struct LcGemm {
     mt = t / L.tiles_n;
     nt = t % L.tiles_n;
   }
-
-  static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
-    return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
+  // work unit -> tile, split and its k-block range
+  static __device__ __forceinline__ void unit_coords(const LcParams &L, int u, int &t, int &sp, int &kb0, int &kb1) {
+    t = u / L.splits;
+    sp = u % L.splits;
+    kb0 = sp * L.kb_per_split;
+    kb1 = min(L.num_kb, kb0 + L.kb_per_split);
   }
+  // output row (GEMM row of D) of row r of M-tile mt, or -1 outside the problem
+  static __device__ __forceinline__ int64_t out_row(const LcParams &L, int mt, int r) {
+    if (implicit_conv(L)) {
+      const int img = mt / (L.tiles_p * L.tiles_q);
+      const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
+      const int pp = pt * L.tp + r / L.tq, qq = qt * L.tq + r % L.tq;
+      return (pp < L.p && qq < L.q) ? ((int64_t)img * L.p + pp) * L.q + qq : -1;
+    }
+    const int m = mt * kBM + r;
+    return m < L.M ? m : -1;
+  }
+  // epilogue of 4 consecutive columns n..n+3 of output row orow: bias, residual, ReLU, store
+  static __device__ __forceinline__ void store4(const LcParams &L, int64_t orow, int n, float f0, float f1, float f2,
+                                                float f3) {
+    float f[4] = {f0, f1, f2, f3};
+    if (L.epi & TACKER_EPI_BIAS) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) f[j] = __fadd_rn(f[j], __ldg(L.bias + n + j));
+    }
+    if (L.epi & TACKER_EPI_RESIDUAL) {
+      const __half *rp = L.residual + orow * L.N + n;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) f[j] = __fadd_rn(f[j], __half2float(rp[j]));
+    }
+    if (L.epi & TACKER_EPI_RELU) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) f[j] = fmaxf(f[j], 0.f);
+    }
+    if (L.d_f16) {
+      __align__(8) __half2 hv[2] = {__floats2half2_rn(f[0], f[1]), __floats2half2_rn(f[2], f[3])};
+      *reinterpret_cast<uint2 *>(reinterpret_cast<__half *>(L.D) + orow * L.N + n) = *reinterpret_cast<uint2 *>(hv);
+    } else {
+      *reinterpret_cast<float4 *>(reinterpret_cast<float *>(L.D) + orow * L.N + n) = make_float4(f[0], f[1], f[2], f[3]);
+    }
+  }
+
   // B (weights) k-block kb of N-tile nt
   static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
     const LcParams &L = P.lc;
@@ -124,22 +174,24 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_tiles) {
-      int mt, nt;
-      tile_coords(L, blockIdx.x, mt, nt);
-      pre = min(P.stages, L.num_kb);
-      for (int kb = 0; kb < pre; ++kb) {
-        mbar_arrive_expect_tx(&bb.full[kb], kStage);
-        load_b(P, &bb.full[kb], lc + kb * kStage + kStageA, kb, nt);
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units) {
+      int t, sp, kb0, kb1, mt, nt;
+      unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
+      tile_coords(L, t, mt, nt);
+      pre = min(P.stages, kb1 - kb0);
+      for (int i = 0; i < pre; ++i) {
+        mbar_arrive_expect_tx(&bb.full[i], kStage);
+        load_b(P, &bb.full[i], lc + i * kStage + kStageA, kb0 + i, nt);
       }
     }
     griddep_wait();
     int stage = 0;
     uint32_t phase = 0;
-    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
-      int mt, nt;
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+      int t, sp, kb0, kb1, mt, nt;
+      unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
-      for (int kb = 0; kb < L.num_kb; ++kb) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         uint8_t *sa = lc + stage * kStage;
         uint8_t *sb = sa + kStageA;
         if (pre > 0) {
@@ -162,11 +214,13 @@ struct LcGemm {
     const LcParams &L = P.lc;
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
-    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+      int t, sp, kb0, kb1;
+      unit_coords(L, u, t, sp, kb0, kb1);
       mbar_wait(&bb.tempty[acc], acc_phase ^ 1);
       tc_fence_after();
       const uint32_t d = tmem + acc * BN;
-      for (int kb = 0; kb < L.num_kb; ++kb) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&bb.full[stage], phase);
         tc_fence_after();
         const uint32_t sa = smem_u32(lc + stage * kStage);
@@ -174,7 +228,7 @@ struct LcGemm {
 #pragma unroll
         for (int k = 0; k < kBK / kUK; ++k) {
           umma_f16(d, umma_desc_sw128(sa + k * kUK * 2), umma_desc_sw128(sb + k * kUK * 2), kIdesc,
-                   (kb | k) != 0);
+                   (kb != kb0 || k != 0));
         }
         umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
         if (++stage == P.stages) {
@@ -197,65 +251,33 @@ struct LcGemm {
     griddep_wait();                             // residual / D of earlier kernels
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int t = blockIdx.x; t < L.num_tiles; t += gridDim.x) {
-      int mt, nt;
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+      int t, sp, kb0, kb1, mt, nt;
+      unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
       mbar_wait(&bb.tfull[acc], acc_phase);
       tc_fence_after();
-      // output row of this thread
-      int64_t orow = -1;
-      if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-        const int img = mt / (L.tiles_p * L.tiles_q);
-        const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
-        const int pp = pt * L.tp + row_in_tile / L.tq, qq = qt * L.tq + row_in_tile % L.tq;
-        if (pp < L.p && qq < L.q) orow = ((int64_t)img * L.p + pp) * L.q + qq;
-      } else {
-        const int m = mt * kBM + row_in_tile;
-        if (m < L.M) orow = m;
-      }
+      const int64_t orow = out_row(L, mt, row_in_tile);
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
+      float *prow = L.splits > 1 ? L.part + ((size_t)u * kBM + row_in_tile) * BN : nullptr;
 #pragma unroll 1
       for (int c0 = 0; c0 < BN; c0 += 32) {
         uint32_t v[32];
         tmem_ld_32x32b_x32(tbase + c0, v);
         tmem_ld_wait();
         const int n0 = nt * BN + c0;
-        if (orow >= 0 && n0 < L.N) {
-          float f[32];
+        if (orow < 0 || n0 >= L.N) continue;
+        if (prow) {   // split-K partial, fp32
 #pragma unroll
-          for (int j = 0; j < 32; ++j) f[j] = __uint_as_float(v[j]);
-          if (L.epi & TACKER_EPI_BIAS) {
+          for (int j = 0; j < 32; j += 4)
+            *reinterpret_cast<float4 *>(prow + c0 + j) = make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]),
+                                                                    __uint_as_float(v[j + 2]), __uint_as_float(v[j + 3]));
+        } else {
 #pragma unroll
-            for (int j = 0; j < 32; ++j)
-              if (n0 + j < L.N) f[j] = __fadd_rn(f[j], __ldg(L.bias + n0 + j));
-          }
-          if (L.epi & TACKER_EPI_RESIDUAL) {
-            const __half *rp = L.residual + orow * L.N + n0;
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-              if (n0 + j < L.N) f[j] = __fadd_rn(f[j], __half2float(rp[j]));
-          }
-          if (L.epi & TACKER_EPI_RELU) {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) f[j] = fmaxf(f[j], 0.f);
-          }
-          if (L.d_f16) {
-            __half *dp = reinterpret_cast<__half *>(L.D) + orow * L.N + n0;
-#pragma unroll
-            for (int j = 0; j < 32; j += 8) {
-              if (n0 + j < L.N) {  // N % 8 == 0: a group of 8 is all in or all out
-                __align__(16) __half2 hv[4];
-#pragma unroll
-                for (int u = 0; u < 4; ++u) hv[u] = __floats2half2_rn(f[j + 2 * u], f[j + 2 * u + 1]);
-                *reinterpret_cast<uint4 *>(dp + j) = *reinterpret_cast<uint4 *>(hv);
-              }
-            }
-          } else {
-            float *dp = reinterpret_cast<float *>(L.D) + orow * L.N + n0;
-#pragma unroll
-            for (int j = 0; j < 32; j += 4)
-              if (n0 + j < L.N) *reinterpret_cast<float4 *>(dp + j) = make_float4(f[j], f[j + 1], f[j + 2], f[j + 3]);
-          }
+          for (int j = 0; j < 32; j += 4)   // N % 8 == 0: a group of 4 is all in or all out
+            if (n0 + j < L.N)
+              store4(L, orow, n0 + j, __uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
+                     __uint_as_float(v[j + 3]));
         }
       }
       tc_fence_before();
@@ -264,6 +286,49 @@ struct LcGemm {
         acc = 0;
         acc_phase ^= 1;
       }
+      if (L.splits > 1) reduce_split(L, t, sp, mt, nt);
+    }
+  }
+
+  // Split-K fixup of tile t by split sp (all splits of the tile run concurrently, one per CTA):
+  // wait until every split has written its partial, then reduce elements [sp E/S, (sp+1) E/S) of
+  // the tile (E = kBM x BN, in groups of 4 columns) over the splits in order 0..S-1 and store them.
+  static __device__ __forceinline__ void reduce_split(const LcParams &L, int t, int sp, int mt, int nt) {
+    const int S = L.splits;
+    const int et = (int)threadIdx.x % 128;      // the 4 epilogue warps are 128 consecutive threads
+    uint32_t *arrive = L.cnt + 2 * t, *finish = arrive + 1;
+    __threadfence();                            // partial visible before the arrival
+    named_bar_sync(kLcEpiBar, 128);
+    if (et == 0) {
+      atomicAdd(arrive, 1u);
+      while (ld_acquire_gpu(arrive) < (uint32_t)S) {
+      }
+    }
+    named_bar_sync(kLcEpiBar, 128);
+    constexpr int G = BN / 4;                   // column groups per row
+    const int E = kBM * G;
+    const float *base = L.part + (size_t)t * S * kBM * BN;
+    for (int g = E * sp / S + et; g < E * (sp + 1) / S; g += 128) {
+      const int r = g / G, c = (g % G) * 4;
+      const int64_t orow = out_row(L, mt, r);
+      const int n = nt * BN + c;
+      if (orow < 0 || n >= L.N) continue;
+      const float *q = base + (size_t)r * BN + c;
+      float4 a = __ldcg(reinterpret_cast<const float4 *>(q));
+      for (int k = 1; k < S; ++k) {
+        const float4 b = __ldcg(reinterpret_cast<const float4 *>(q + (size_t)k * kBM * BN));
+        a.x = __fadd_rn(a.x, b.x);
+        a.y = __fadd_rn(a.y, b.y);
+        a.z = __fadd_rn(a.z, b.z);
+        a.w = __fadd_rn(a.w, b.w);
+      }
+      store4(L, orow, n, a.x, a.y, a.z, a.w);
+    }
+    named_bar_sync(kLcEpiBar, 128);
+    if (et == 0 && atomicAdd(finish, 1u) == (uint32_t)S - 1) {   // last reducer: reset for the next launch
+      *arrive = 0;
+      *finish = 0;
+      __threadfence();
     }
   }
 };
@@ -332,7 +397,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
   // (TMA issue, MMA issue, TMEM drain) win every issue slot they compete for.
   const int be_warps = 4 * P.be_vb_per_cta;
   const int warp = (int)warp_id() - be_warps;       // LC role index (< 0: BE warp)
-  const bool has_lc = P.lc_warps > 0 && P.lc.num_tiles > 0;
+  const bool has_lc = P.lc_warps > 0 && P.lc.num_units > 0;
   typename LcGemm<BN>::Bars bb{};
   if (P.lc_warps > 0) {
     bb = LcGemm<BN>::bars(lc, P.stages);

@@ -28,6 +28,7 @@
 #include <map>
 #include <set>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "runtime.h"
@@ -63,7 +64,6 @@ struct App {
   double ready_at = 0;
   int64_t completed = 0;
   int64_t done = 0;                // blocks of the head kernel already issued (PTB slices)
-  cudaEvent_t pending = nullptr;   // GPU mode: last launched kernel of this app
   const tacker_be_kernel &head() const { return ks[pos % ks.size()]; }
 };
 
@@ -91,8 +91,24 @@ struct tacker_manager_s {
   std::deque<int> active;
   std::vector<App> apps;
   tacker_manager_stats st{};
-  std::map<std::string, tacker_fused_t> cache;
-  std::deque<cudaEvent_t> inflight;
+  std::vector<tacker_fused_t> owned;      // fused handles built by the manager
+  // per (LC operands, BE kernel) pair: model-store key and fused handle, so a decision does no
+  // string formatting / handle lookup (the manager loop is host-latency bound for 10 us kernels)
+  struct PairEntry {
+    bool keyed = false;
+    std::string pk;
+    tacker_fused_t f = nullptr;
+  };
+  std::map<std::tuple<const void *, const void *, const void *, int, size_t>, PairEntry> pairs;
+  // in-flight cap: launches issued vs launches known complete, observed through stream events
+  // recorded every ev_every launches (and after launches whose completion is needed), so the
+  // stream is not cut by an event after every ~10 us kernel (events block launch overlap)
+  struct Mark {
+    cudaEvent_t e;
+    int64_t upto;
+  };
+  std::deque<Mark> marks;
+  int64_t launched = 0, marked_upto = 0, completed_upto = 0, ev_every = 1;
   std::vector<cudaEvent_t> free_events;
   std::map<cudaEvent_t, int> refs;
   struct Observed {
@@ -116,8 +132,21 @@ struct tacker_manager_s {
   int64_t class_timed[4] = {0, 0, 0, 0};
   int64_t class_n[4] = {0, 0, 0, 0};   // every launch
 
+  double host_ns[3] = {0, 0, 0};   // poll, launch + event calls, whole step
+  int64_t host_steps = 0;
+
   bool sim() const { return prm.simulate != 0; }
 };
+
+namespace {
+// accumulates the wall time of a scope into a manager counter (GPU mode host profile)
+struct HostTimer {
+  double &acc;
+  std::chrono::steady_clock::time_point t0;
+  explicit HostTimer(double &a) : acc(a), t0(std::chrono::steady_clock::now()) {}
+  ~HostTimer() { acc += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count(); }
+};
+}  // namespace
 
 static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b) {
   return m->policy == TACKER_POLICY_TACKER && m->prm.slice_be && b.n_blocks > 1 && b.t_block_ms > 0;
@@ -179,16 +208,12 @@ static void unref(tacker_manager_s *m, cudaEvent_t e) {
 
 static void poll(tacker_manager_s *m) {
   if (m->sim()) return;
-  while (!m->inflight.empty() && cudaEventQuery(m->inflight.front()) == cudaSuccess) {
-    unref(m, m->inflight.front());
-    m->inflight.pop_front();
+  HostTimer ht(m->host_ns[0]);
+  while (!m->marks.empty() && cudaEventQuery(m->marks.front().e) == cudaSuccess) {
+    m->completed_upto = m->marks.front().upto;
+    unref(m, m->marks.front().e);
+    m->marks.pop_front();
   }
-  for (auto &a : m->apps)
-    if (a.pending && cudaEventQuery(a.pending) == cudaSuccess) {
-      a.ready_at = event_time(m, a.pending);
-      unref(m, a.pending);
-      a.pending = nullptr;
-    }
   while (!m->timed.empty() && cudaEventQuery(m->timed.front().end) == cudaSuccess) {
     auto &t = m->timed.front();
     float ms = 0;
@@ -233,10 +258,6 @@ static bool app_ready(tacker_manager_s *m, const App &a, double t) {
   if (m->sim()) return a.ready_at <= t;
   return true;
 }
-static void set_pending(tacker_manager_s *m, App &a, cudaEvent_t e) {
-  if (a.pending) unref(m, a.pending);
-  a.pending = ref(m, e);
-}
 
 static bool pair_key(const tacker_lc_kernel &k, const tacker_be_kernel &b, std::string *pk) {
   std::string lk, bk;
@@ -250,6 +271,17 @@ static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, doub
 }
 
 static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b);
+
+// keyed by the LC operands and (app, kernel index): stable across reallocation of the app list
+static tacker_manager_s::PairEntry &pair_entry(tacker_manager_s *m, const tacker_lc_kernel &k, int app, size_t kidx) {
+  const tacker_be_kernel &b = m->apps[app].ks[kidx];
+  auto &e = m->pairs[std::make_tuple(k.lc.A, k.lc.B, k.lc.D, app, kidx)];
+  if (!e.keyed) {
+    e.keyed = true;
+    if (!pair_key(k, b, &e.pk)) e.pk.clear();
+  }
+  return e;
+}
 
 // Blocks of the head kernel of A that a fused launch with TC kernel k should carry: the
 // smallest n with X_cd(n) >= r* X_tc (clamped to the remaining blocks), or -1 = the whole rest
@@ -267,12 +299,14 @@ static int64_t slice_blocks(const tacker_manager_s *m, const App &A, const std::
 
 // ---------------------------------------------------------------- GPU launches
 static tacker_status launch_lc(tacker_manager_s *m, const tacker_lc_kernel &k) {
+  HostTimer ht(m->host_ns[1]);
   if (k.is_tc) return tacker_launch_original(&k.lc, nullptr, reinterpret_cast<tacker_stream_t>(m->stream));
   return tacker_launch_original(nullptr, &k.cd, reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
 // the rest of app A's head kernel (the whole kernel when no slice of it was issued yet)
 static tacker_status launch_be(tacker_manager_s *m, const App &A) {
+  HostTimer ht(m->host_ns[1]);
   const tacker_be_kernel &b = A.head();
   if (A.done == 0) return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
   tacker_be_desc d = b.be;
@@ -282,48 +316,59 @@ static tacker_status launch_be(tacker_manager_s *m, const App &A) {
 }
 
 // Fused handle of (LC kernel, BE kernel) from the manager's cache, built on first use.
-static tacker_status fused_handle(tacker_manager_s *m, const tacker_lc_kernel &k, const tacker_be_kernel &b,
+static tacker_status fused_handle(tacker_manager_s *m, const tacker_lc_kernel &k, int app, size_t kidx,
                                   tacker_fused_t *out) {
-  const int ws = b.warp_split ? b.warp_split : 16;
-  char key[256];
-  snprintf(key, sizeof key, "%p/%p/%p/%p/%d/%d", k.lc.A, k.lc.B, k.lc.D, (const void *)&b, ws, b.be.orig_blocks);
-  auto it = m->cache.find(key);
-  if (it != m->cache.end()) {
-    *out = it->second;
+  auto &pe = pair_entry(m, k, app, kidx);
+  if (pe.f) {
+    *out = pe.f;
     return TACKER_OK;
   }
+  const tacker_be_kernel &b = m->apps[app].ks[kidx];
+  const int ws = b.warp_split ? b.warp_split : 16;
   tacker_status s = tacker_fuse(&k.lc, &b.be, ws, tacker_ratio{0, 0}, out);
-  if (s == TACKER_OK) m->cache[key] = *out;
+  if (s == TACKER_OK) {
+    pe.f = *out;
+    m->owned.push_back(*out);
+  }
   return s;
 }
 
 // TC kernel k fused with n blocks of app A's head kernel (n < 0: the whole rest)
-static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, const App &A, int64_t n) {
+static tacker_status launch_fused(tacker_manager_s *m, const tacker_lc_kernel &k, int app, int64_t n) {
+  HostTimer ht(m->host_ns[1]);
+  const App &A = m->apps[app];
   const tacker_be_kernel &b = A.head();
   tacker_fused_t f = nullptr;
-  tacker_status s = fused_handle(m, k, b, &f);
+  tacker_status s = fused_handle(m, k, app, A.pos % A.ks.size(), &f);
   if (s) return s;
   if (A.done == 0 && n < 0) return tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
   return tacker_launch_fused_slice(f, (int64_t)b.be.block_offset + A.done, n < 0 ? b.n_blocks - A.done : n,
                                    reinterpret_cast<tacker_stream_t>(m->stream));
 }
 
-static cudaEvent_t record(tacker_manager_s *m) {
+// After a launch: count it, and record a stream event when one is needed at this point (force:
+// the launch is timed, observed or ends a query) or ev_every launches have gone unmarked.
+static cudaEvent_t mark(tacker_manager_s *m, bool force) {
+  m->launched++;
+  if (!force && m->launched - m->marked_upto < m->ev_every) return nullptr;
+  HostTimer ht(m->host_ns[1]);
   cudaEvent_t e = get_event(m);
   cudaEventRecord(e, m->stream);
-  m->inflight.push_back(ref(m, e));
+  m->marks.push_back(tacker_manager_s::Mark{ref(m, e), m->launched});
+  m->marked_upto = m->launched;
   return e;
 }
 // Per-class device time (stats.class_ms): every launch is counted, one launch in kTimeEvery of
 // each class is bracketed by events (a start event costs a host API call per launch, and the
 // manager loop of a 53-kernel query is host-latency sensitive); the class total is the sampled
 // mean x the count.  Fused launches are always timed: the online refit needs each one.
-static constexpr int64_t kTimeEvery = 8;
+static constexpr int64_t kTimeEvery = 16;
 // start event of a launch (the stream reaches it when the previous kernel has finished), or
 // nullptr when this launch is not in the timed sample
 static cudaEvent_t begin(tacker_manager_s *m, int cls, bool always = false) {
   if (!always && m->class_n[cls]++ % kTimeEvery != 0) return nullptr;
   if (always) m->class_n[cls]++;
+  HostTimer ht(m->host_ns[1]);
   cudaEvent_t e = get_event(m);
   cudaEventRecord(e, m->stream);
   return e;
@@ -343,6 +388,7 @@ tacker_status tacker_manager_create(int32_t policy, const tacker_manager_params 
   m->policy = policy;
   m->prm = *params;
   if (m->prm.max_inflight < 1) m->prm.max_inflight = 1;
+  m->ev_every = std::max(1, m->prm.max_inflight / 2);
   m->stream = reinterpret_cast<cudaStream_t>(stream);
   m->t0 = std::chrono::steady_clock::now();
   if (!m->sim()) {
@@ -361,8 +407,8 @@ tacker_status tacker_manager_destroy(tacker_manager_t m) {
   if (!m) return TACKER_OK;
   if (!m->sim()) {
     cudaStreamSynchronize(m->stream);
-    for (auto &kv : m->cache) tacker_fused_destroy(kv.second);
-    for (auto e : m->inflight) cudaEventDestroy(e);
+    for (auto f : m->owned) tacker_fused_destroy(f);
+    for (auto &mk : m->marks) cudaEventDestroy(mk.e);
     for (auto e : m->free_events) cudaEventDestroy(e);
     if (m->base_ev) cudaEventDestroy(m->base_ev);
   }
@@ -405,6 +451,8 @@ tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms) {
 
 tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headroom, tacker_decision *out) {
   if (!m || !out) return set_error("null argument"), TACKER_EINVAL;
+  HostTimer ht(m->host_ns[2]);
+  m->host_steps++;
   memset(out, 0, sizeof *out);
   out->action = TACKER_DEC_NOTHING;
   out->query = out->lc_index = out->fused_app = -1;
@@ -421,7 +469,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
     if (m->sim() || q.done_at >= 0) m->active.pop_front();
     else break;
   }
-  if (!m->sim() && (int)m->inflight.size() >= m->prm.max_inflight) return TACKER_OK;   // stream is busy
+  if (!m->sim() && m->launched - m->completed_upto >= m->prm.max_inflight) return TACKER_OK;   // stream is busy
 
   // oldest query with kernels still to issue
   int qid = -1;
@@ -451,8 +499,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
         cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
         tacker_status s = launch_be(m, A);
         if (s) return s;
-        set_pending(m, A, record(m));
-        track(m, e0, A.pending, TACKER_CLASS_BE);
+        track(m, e0, mark(m, e0 != nullptr), TACKER_CLASS_BE);
       }
       issue_be(m, A, -1);
       m->st.idle_be++;
@@ -497,8 +544,8 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       const App &A = m->apps[a];
       const tacker_be_kernel &b = A.head();
       if (!b.is_cd) continue;
-      std::string pk;
-      if (!pair_key(k, b, &pk)) continue;
+      const std::string &pk = pair_entry(m, k, a, A.pos % A.ks.size()).pk;
+      if (pk.empty()) continue;
       const int64_t n = slice_blocks(m, A, pk, ttc);
       const double tcd = n < 0 ? rem_ms(A) : slice_ms(b, n);
       double tf;
@@ -547,15 +594,13 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       A.ready_at = m->now;
     } else {
       cudaEvent_t e0 = begin(m, TACKER_CLASS_FUSED, true);
-      tacker_status s = launch_fused(m, k, A, best_n);
+      tacker_status s = launch_fused(m, k, fused, best_n);
       if (s) return s;
-      cudaEvent_t e = record(m);
+      cudaEvent_t e = mark(m, true);
       track(m, e0, e, TACKER_CLASS_FUSED);
-      set_pending(m, A, e);
       if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
       // online model update from the measured co-run
-      std::string lk, bk, pk;
-      make_keys(&k.lc, &A.head().be, A.head().warp_split ? A.head().warp_split : 16, &lk, &bk, &pk);
+      const std::string &pk = pair_entry(m, k, fused, A.pos % A.ks.size()).pk;
       m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, best_tcd, best_tf});
     }
     issue_be(m, A, best_n);
@@ -568,9 +613,10 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       cudaEvent_t e0 = begin(m, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
       tacker_status s = launch_lc(m, k);
       if (s) return s;
-      cudaEvent_t e = record(m);
+      const bool last = q.pos + 1 == q.ks.size();
+      cudaEvent_t e = mark(m, e0 != nullptr || last);
       track(m, e0, e, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
-      if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
+      if (last) q.last_ev = ref(m, e);
     }
     m->st.original_lc++;
     out->action = reorder.empty() ? TACKER_DEC_ORIGINAL_LC : TACKER_DEC_REORDER_BE;
@@ -589,8 +635,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       cudaEvent_t e0 = begin(m, TACKER_CLASS_BE);
       tacker_status s = launch_be(m, A);
       if (s) return s;
-      set_pending(m, A, record(m));
-      track(m, e0, A.pending, TACKER_CLASS_BE);
+      track(m, e0, mark(m, e0 != nullptr), TACKER_CLASS_BE);
     }
     issue_be(m, A, -1);
     m->st.reordered_be++;
@@ -608,12 +653,13 @@ static tacker_status prepare_kernels(tacker_manager_s *m, const tacker_lc_kernel
     const tacker_lc_kernel &k = ks[i];
     if (!k.is_tc) continue;
     if (!m->prepared_lc.insert({k.lc.A, k.lc.B, k.lc.D}).second) continue;
-    for (const App &A : m->apps)
-      for (const tacker_be_kernel &b : A.ks) {
+    for (size_t a = 0; a < m->apps.size(); ++a)
+      for (size_t j = 0; j < m->apps[a].ks.size(); ++j) {
+        const tacker_be_kernel &b = m->apps[a].ks[j];
         double tf;
         if (!b.is_cd || !pair_time(k, b, &tf)) continue;
         tacker_fused_t f = nullptr;
-        tacker_status s = fused_handle(m, k, b, &f);
+        tacker_status s = fused_handle(m, k, (int)a, j, &f);
         if (s != TACKER_OK && s != TACKER_ERESOURCE && s != TACKER_EUNSUPPORTED) return s;
       }
   }
@@ -666,6 +712,10 @@ tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats 
   o->pred_err_sum = m->pred_err_sum;
   o->be_work_ms = m->be_work_ms;
   o->pred_err_n = m->pred_err_n;
+  o->host_poll_ms = m->host_ns[0] * 1e-6;
+  o->host_launch_ms = m->host_ns[1] * 1e-6;
+  o->host_decide_ms = m->host_ns[2] * 1e-6;   // whole step (includes its poll and launches)
+  o->host_steps = m->host_steps;
   for (int c = 0; c < 4; ++c) {
     o->class_ms[c] = m->class_timed[c] ? m->class_ms[c] / (double)m->class_timed[c] * (double)m->class_n[c] : 0.0;
     o->class_launches[c] = m->class_n[c];

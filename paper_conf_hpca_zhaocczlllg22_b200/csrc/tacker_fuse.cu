@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
@@ -263,6 +264,24 @@ static void lc_tiles(LcParams &L, int BN) {
     L.num_kb = (L.K + kBK - 1) / kBK;
   }
   L.num_tiles = L.tiles_m * L.tiles_n;
+  L.splits = 1;
+  L.kb_per_split = L.num_kb;
+  L.num_units = L.num_tiles;
+}
+
+// Split-K for GEMMs with few tiles and a deep K (batch-1 layer3/4 convs: 4-16 tiles of 16-72
+// k-blocks would leave >= 132 SMs idle and serialise the k-loop): S splits of >= 2 k-blocks so
+// that tiles x S <= #SMs -- every unit gets its own CTA, which the in-kernel fixup requires.
+static void lc_split(LcParams &L, int sms) {
+  if (L.num_tiles * 2 > sms || L.num_kb < 4) return;
+  int S = std::min(sms / L.num_tiles, L.num_kb / 2);
+  if (S < 2) return;
+  const int kbs = (L.num_kb + S - 1) / S;
+  S = (L.num_kb + kbs - 1) / kbs;
+  if (S < 2) return;
+  L.splits = S;
+  L.kb_per_split = kbs;
+  L.num_units = L.num_tiles * S;
 }
 
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -407,6 +426,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   if (st) return st;
   const int BN = pick_tile_n(*lc, L);
   lc_tiles(L, BN);
+  if (!(lc->epi_flags & TACKER_LC_NO_SPLIT)) lc_split(L, sms);
   F.BN = BN;
 
   int64_t be_blocks = 0;
@@ -419,7 +439,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     vb = warp_split / 4;
     if (ratio.be && ratio.be != vb)
       return set_error("block_ratio.be (%d) must equal warp_split/4 (%d)", ratio.be, vb), TACKER_EUNSUPPORTED;
-    if (vb > 15) return set_error("too many BE virtual blocks for named barriers"), TACKER_ERESOURCE;
+    if (vb > 14) return set_error("too many BE virtual blocks for named barriers (1..14)"), TACKER_ERESOURCE;
     be_slice = (16 + be_smem_bytes(be->kind) + 127) & ~127u;
     F.P.be = *be;
   }
@@ -465,7 +485,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // TMEM); a fused CTA is already alone on its SM through its registers (>= 16 warps x 64
   // regs... a second CTA would exceed 64K), so it keeps the unused shared memory as L1.
   if (!has_be && F.smem < kMinLcSmem) F.smem = kMinLcSmem;
-  F.grid = has_be ? sms : (L.num_tiles < sms ? L.num_tiles : sms);
+  F.grid = has_be ? sms : (L.num_units < sms ? L.num_units : sms);
   if (F.grid < 1) F.grid = 1;
   F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
   if (!F.fn) return set_error("no kernel instantiation for BN=%d BE=%d", BN, has_be ? be->kind : 0), TACKER_EUNSUPPORTED;
@@ -515,6 +535,25 @@ static cudaError_t launch_ex(void (*fn)(Param), dim3 grid, dim3 block, int smem,
   cfg.attrs = attr;
   cfg.numAttrs = g_overlap.load(std::memory_order_relaxed) ? 1 : 0;
   return cudaLaunchKernelEx(&cfg, fn, p);
+}
+
+// Split-K workspace (partial tiles + counters) of a plan, owned by its handle.
+static tacker_status alloc_lc_workspace(tacker_fused_s &F) {
+  LcParams &L = F.P.lc;
+  L.part = nullptr;
+  L.cnt = nullptr;
+  if (L.splits <= 1) return TACKER_OK;
+  const size_t part = (size_t)L.num_units * kBM * F.BN * sizeof(float);
+  void *p = nullptr;
+  cudaError_t e = cudaMalloc(&p, part + 2 * (size_t)L.num_tiles * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMemset(static_cast<char *>(p) + part, 0, 2 * (size_t)L.num_tiles * sizeof(uint32_t));
+  if (e != cudaSuccess) {
+    if (p) cudaFree(p);
+    return cuda_fail("split-K workspace", e);
+  }
+  L.part = static_cast<float *>(p);
+  L.cnt = reinterpret_cast<uint32_t *>(static_cast<char *>(p) + part);
+  return TACKER_OK;
 }
 
 static tacker_status launch_params(const tacker_fused_s &F, FusedParams &P, cudaStream_t s) {
@@ -571,6 +610,11 @@ tacker_status tacker_fuse(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     delete F;
     return cuda_fail("workspace", e);
   }
+  if ((st = alloc_lc_workspace(*F))) {
+    cudaFree(F->P.work);
+    delete F;
+    return st;
+  }
   *out = F;
   return TACKER_OK;
 }
@@ -578,6 +622,7 @@ tacker_status tacker_fuse(const tacker_lc_desc *lc, const tacker_be_desc *be, in
 tacker_status tacker_fused_destroy(tacker_fused_t f) {
   if (!f) return TACKER_OK;
   if (f->P.work) cudaFree(f->P.work);
+  if (f->P.lc.part) cudaFree(f->P.lc.part);
   delete f;
   return TACKER_OK;
 }
@@ -598,6 +643,7 @@ tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *o) {
   o->lc_acc_stages = f->P.acc_stages;
   o->tmem_cols = (int32_t)f->P.tmem_cols;
   o->lc_tiles = f->P.lc.num_tiles;
+  o->lc_splits = f->P.lc.splits;
   o->be_blocks = f->P.be_blocks;
   o->be_smem_per_vblock = (int32_t)f->P.be_smem_per_vb;
   o->regs_per_thread = f->regs;
@@ -623,9 +669,15 @@ tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, co
   if (st) return st;
   if (tmp.fn != f->fn || tmp.P.stages != f->P.stages || tmp.smem != f->smem)
     return set_error("rebind changes the plan; call tacker_fuse"), TACKER_EINVAL;
+  if (tmp.P.lc.splits != f->P.lc.splits || tmp.P.lc.num_units != f->P.lc.num_units)
+    return set_error("rebind changes the split-K plan; call tacker_fuse"), TACKER_EINVAL;
   BeWork *w = f->P.work;
+  float *part = f->P.lc.part;
+  uint32_t *cnt = f->P.lc.cnt;
   *f = tmp;
   f->P.work = w;
+  f->P.lc.part = part;
+  f->P.lc.cnt = cnt;
   return TACKER_OK;
 }
 
@@ -670,6 +722,7 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
       auto P = std::make_unique<tacker_fused_s>();
       if ((st = plan(lc, nullptr, 0, tacker_ratio{0, 0}, *P))) return st;
       P->P.work = nullptr;
+      if ((st = alloc_lc_workspace(*P))) return st;
       std::lock_guard<std::mutex> g(mu);
       if (cache.size() > 4096) cache.clear();
       F = (cache[key] = std::move(P)).get();

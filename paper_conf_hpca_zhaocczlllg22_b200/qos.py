@@ -31,17 +31,22 @@ def _prefix(desc, n):
     return d
 
 
-def _time(fn, reps=10, stream=None):
+def _time(fn, reps=10, stream=None, inner=8):
+    """Device time per launch in a pipelined stream (the manager's regime): median over `reps`
+    rounds of `inner` back-to-back launches between two events, divided by `inner`.  A single
+    launch between two events would add the host's launch latency (Python here) to a 10 us
+    kernel."""
     s = stream or torch.cuda.current_stream()
     fn()
     ts = []
     for _ in range(reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
-        fn()
+        for _ in range(inner):
+            fn()
         e1.record(s)
         e1.synchronize()
-        ts.append(e0.elapsed_time(e1))
+        ts.append(e0.elapsed_time(e1) / inner)
     return statistics.median(ts)
 
 
@@ -213,6 +218,26 @@ class QosRun:
     def query_solo_ms(self):
         return sum(self.t_lc)
 
+    def measure_service(self, n=200, max_inflight=4):
+        """Peak LC load: the manager's service rate for LC-only queries -- n
+        queries all arriving at once, run back to back through the manager (no BE apps); with a
+        50 ms target and ~1 ms queries the QoS-safe peak rate is this service rate.  Returns and
+        stores the mean service time per query (ms)."""
+        stream = torch.cuda.current_stream()
+        torch.cuda.synchronize()
+        m = tk.Manager(tk.POLICY_BAYMAX, stream=stream, simulate=False, max_inflight=max_inflight)
+        kernels = self.lc_kernels()
+        t0 = m.stats().now_ms + 1.0
+        for _ in range(n):
+            m.submit_lc(kernels, t0)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        m.run(self.qos, t0)
+        e1.record(stream)
+        e1.synchronize()
+        self.service_ms = e0.elapsed_time(e1) / n
+        return self.service_ms
+
     # ------------------------------------------------------------------ one managed run
     def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None,
             slice_be=False, slice_ratio=0.0, reorder_only_unfused=False):
@@ -220,7 +245,9 @@ class QosRun:
         paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
         stream = torch.cuda.current_stream()
         torch.cuda.synchronize()
-        lam = load / self.query_solo_ms()                       # queries per ms
+        # peak rate = the measured LC-only service rate through the manager (measure_service), else
+        # 1 / the standalone query time
+        lam = load / getattr(self, "service_ms", self.query_solo_ms())     # queries per ms
         rng = np.random.default_rng(seed)
         gaps = rng.exponential(1.0 / lam, n_queries + warmup)
         cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
@@ -255,4 +282,5 @@ class QosRun:
                 "class_ms": {n: float(st.class_ms[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
                 "class_launches": {n: int(st.class_launches[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
                 "lc_p50_ms": float(np.median(lat)), "lc_p99_ms": p99, "lc_max_ms": float(lat.max()),
-                "qos_ms": self.qos, "qos_met": bool(p99 <= self.qos), "query_solo_ms": self.query_solo_ms()}
+                "qos_ms": self.qos, "qos_met": bool(p99 <= self.qos), "query_solo_ms": self.query_solo_ms(),
+                "service_ms": getattr(self, "service_ms", None), "max_inflight": max_inflight}

@@ -24,7 +24,7 @@ OK, EINVAL, ERESOURCE, EUNSUPPORTED, ECUDA, ENOMODEL, ENOMEM = 0, -1, -2, -3, -4
 STATUS_NAMES = {0: "OK", -1: "EINVAL", -2: "ERESOURCE", -3: "EUNSUPPORTED", -4: "ECUDA", -5: "ENOMODEL", -6: "ENOMEM"}
 LC_NONE, LC_GEMM_F16, LC_CONV_F16 = 0, 1, 2
 F32, F16 = 0, 1
-EPI_BIAS, EPI_RELU, EPI_RESIDUAL, LC_B_CONST = 1, 2, 4, 8
+EPI_BIAS, EPI_RELU, EPI_RESIDUAL, LC_B_CONST, LC_NO_SPLIT = 1, 2, 4, 8, 16
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
  BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY, BE_JDS_COUNT, BE_JDS_SCAN,
  BE_JDS_PERM, BE_JDS_FILL) = range(19)
@@ -158,7 +158,7 @@ class FusedInfo(C.Structure):
                 ("lc_tile_m", C.c_int32), ("lc_tile_n", C.c_int32), ("lc_tile_k", C.c_int32),
                 ("lc_stages", C.c_int32), ("lc_acc_stages", C.c_int32), ("tmem_cols", C.c_int32),
                 ("lc_tiles", C.c_int64), ("be_blocks", C.c_int64), ("be_smem_per_vblock", C.c_int32),
-                ("regs_per_thread", C.c_int32)]
+                ("regs_per_thread", C.c_int32), ("lc_splits", C.c_int32)]
 
 
 class LcKernel(C.Structure):
@@ -196,7 +196,8 @@ class ManagerStats(C.Structure):
                 ("original_lc", C.c_int64), ("reordered_be", C.c_int64), ("idle_be", C.c_int64),
                 ("now_ms", C.c_double), ("model_refits", C.c_int64), ("class_ms", C.c_double * 4),
                 ("class_launches", C.c_int64 * 4), ("pred_err_sum", C.c_double), ("pred_err_n", C.c_int64),
-                ("be_work_ms", C.c_double)]
+                ("be_work_ms", C.c_double), ("host_poll_ms", C.c_double), ("host_launch_ms", C.c_double),
+                ("host_decide_ms", C.c_double), ("host_steps", C.c_int64)]
 
 
 CLASS_LC_TC, CLASS_LC_CD, CLASS_FUSED, CLASS_BE = range(4)

@@ -293,3 +293,51 @@ def test_launch_overlap_keeps_stream_order(tk):
         tk.tacker_set_launch_overlap(True)
     for _ in range(3):
         assert run() == ref
+
+
+@pytest.mark.parametrize("M,N,K", [(128, 256, 4096), (130, 264, 4104), (49, 512, 4608)])
+def test_lc_split_k_vs_oracle(tk, M, N, K):
+    """Split-K (few tiles, deep K): every unit on its own CTA, deterministic in-kernel fixup.
+    Against the oracle, against the unsplit kernel, and repeatable (self-resetting counters)."""
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=K)
+    dA, dB = t(A), t(B)
+    D = torch.full((M, N), float("nan"), device=dev())
+    D1 = torch.full((M, N), float("nan"), device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(dA, dB, D, b_const=True), None, 0)
+    assert f.info().lc_splits > 1 and f.info().grid == f.info().lc_tiles * f.info().lc_splits
+    ref, S = olc.lc_gemm(A, B)
+    outs = []
+    for _ in range(3):
+        D.fill_(float("nan"))
+        f.launch()
+        outs.append(host(D).tobytes())
+        assert max_rel_err(host(D), ref, S) <= 1e-5
+    assert outs[0] == outs[1] == outs[2]
+    nd = tk.lc_gemm(dA, dB, D1)
+    nd.epi_flags |= tk.LC_NO_SPLIT
+    tk.tacker_launch_original(nd, None)
+    assert max_rel_err(host(D1), ref, S) <= 1e-5
+
+
+def test_fused_split_k_conv_bit_identical(tk):
+    # layer4-like 3x3 conv (7x7 output, 4 tiles x 72 k-blocks -> 36 splits) fused with histo
+    cs = synth.ConvShape("l4", 1, 7, 7, 512, 512, 3, 3, 1, 1)
+    x, w, b = synth.conv_inputs(cs, seed=12)
+    dx, dw, db = t(x), t(w), t(b)
+    o0 = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    o1 = torch.zeros_like(o0)
+    c = be_case(tk.BE_HISTO, seed=4)
+    c["reset"]()
+    tk.tacker_launch_original(tk.lc_conv(dx, dw, o0, 1, 1, bias=db, relu=True, b_const=True), c["desc"])
+    orig = [host(o).copy() for o in c["outs"]]
+    f = tk.tacker_fuse(tk.lc_conv(dx, dw, o1, 1, 1, bias=db, relu=True, b_const=True), c["desc"], 16)
+    assert f.info().lc_splits == 36
+    for _ in range(2):
+        c["reset"]()
+        o1.zero_()
+        f.launch()
+        assert host(o1).tobytes() == host(o0).tobytes()
+        for a, g in zip(orig, c["outs"]):
+            assert host(g).tobytes() == a.tobytes()
+    ref, S = olc.lc_conv(x, w, 1, 1, bias=b, relu=True)
+    assert max_rel_err(host(o1).astype(np.float64), ref, S) <= 1e-2

@@ -68,6 +68,9 @@ def main():
         "managed_overhead_p50_ms": float(np.median(lat)) - solo,
         "class_ms": {n: float(st.class_ms[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
         "class_launches": {n: int(st.class_launches[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},
+        "host_ms_per_query": {"poll": st.host_poll_ms / args.queries, "launch_and_events": st.host_launch_ms / args.queries,
+                              "step_total": st.host_decide_ms / args.queries, "steps": st.host_steps / args.queries},
+        "saturated_service_ms": q.measure_service(200),
         "wall_s": wall}))
 
 

@@ -52,6 +52,7 @@ def main():
     ap.add_argument("--ws", type=int, default=24)
     ap.add_argument("--qos", type=float, default=50.0)
     ap.add_argument("--io", action="store_true", help="each query copies its input H2D and result D2H")
+    ap.add_argument("--inflight", type=int, default=4)
     ap.add_argument("--variants", default="baymax,tacker,tacker_slice,tacker_slice_literal")
     ap.add_argument("--slice-ratio", type=float, default=0.0, help="fixed slice load ratio (0: opportune r*)")
     args = ap.parse_args()
@@ -62,6 +63,7 @@ def main():
     if args.io:
         q.with_io()
     q.calibrate()
+    q.measure_service(max_inflight=args.inflight)
     res = {}
     variants = {"baymax": (tk.POLICY_BAYMAX, {}), "tacker": (tk.POLICY_TACKER, {}),
                 "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
@@ -70,7 +72,7 @@ def main():
         pol, kw = variants[name]
         if args.slice_ratio > 0 and kw.get("slice_be"):
             kw = dict(kw, slice_ratio=args.slice_ratio)
-        res[name] = q.run(pol, args.queries, load=args.load, warmup=args.warmup, **kw)
+        res[name] = q.run(pol, args.queries, load=args.load, warmup=args.warmup, max_inflight=args.inflight, **kw)
     for name in res:
         if name != "baymax" and "baymax" in res:
             res[name]["improvement_eq10"] = res[name]["be_kernels_per_s"] / res["baymax"]["be_kernels_per_s"] - 1.0
