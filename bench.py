@@ -2,26 +2,28 @@
 """Bench for the B200-native Tacker hot path (BASELINE.json metric:
 "BE kernels/sec at LC p99 <= QoS target; fused time vs overlap roofline").
 
-Workload (N=1, BASELINE configs[1]): ResNet-50 batch-1 inference as the LC service (53 convs as
-implicit-GEMM tcgen05 kernels; conv1 = im2col + GEMM) co-located with a BE queue of two
-Parboil applications, stencil (512x512x64 sweeps) and mri-q (64^3 voxels, 2048 k in two 1024-k
-ComputeQ chunks).
+Workload (N=1): BASELINE configs[3] (SURVEY config 4), QoS-managed co-location -- ResNet-50 at
+the paper's batch 32 (Table II) as the LC service (53 convs as implicit-GEMM tcgen05
+kernels, split-K where few tiles; conv1 = im2col + GEMM) with a BE queue of two Parboil
+applications, stencil (512x512x64 sweeps) and mri-q (64^3 voxels, 2048 k in two 1024-k chunks).
 
 * Headline (`value`): the QoS-managed run.  One step = one LC query; queries arrive as a
-  Poisson process at 80 % of the service's peak rate, the native manager
-  (tacker_manager_run, Tacker policy) launches fused / original / reordered kernels from each
-  query's headroom under a 50 ms QoS target.  value = BE kernels completed per second over the
-  K timed queries (CUDA events on the manager stream), with the queries' p99 latency checked
-  against the target.  The same trace under the Baymax policy (fusion off) gives Eq. 10.
+  Poisson process at 80 % of the peak LC load (peak = the manager's LC-only
+  service rate, measured), the native manager (tacker_manager_run, Tacker policy) launches
+  fused / original / reordered kernels from each query's headroom under a 50 ms QoS target.
+  value = BE kernels completed per second over the K timed queries (CUDA events on the manager
+  stream), with the queries' p99 latency checked against the target.  The same trace under the
+  Baymax policy (fusion off) gives Eq. 10; a PTB-sliced Tacker run (reading 13) is reported too.
 * `e2e`: the same managed run through the public API where every query also moves its input
-  image host->device and its result device->host (pinned host memory, UVA copy kernels inside
+  images host->device and its result device->host (pinned host memory, UVA copy kernels inside
   the managed stream).
-* `fused_step` + `roofline`: the kernel-level view — every LC tensor-core kernel of one query
-  fused with the next BE kernel (the fused kernels' time vs their overlap roofline and vs the
-  sequential original launches); `roofline` is the dominant fused kernel class.
+* `roofline`: the dominant launch class of the timed run (LC convs: achieved vs tensor / HBM
+  peak).  `fused_step` + `roofline_fused`: BASELINE configs[1] -- every LC tensor-core kernel of a
+  ResNet-50 batch-1 query fused with the next BE kernel (fused time vs overlap roofline and vs
+  the sequential original launches); `config1_resnet50_b1` = the managed protocol at batch 1.
 * `cpu_baseline`: the CPU oracle on a bounded sample.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tacker|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--batch 32] [--impl tacker|reference]
 """
 from __future__ import annotations
 
@@ -43,7 +45,7 @@ sys.path.insert(0, ROOT)
 QOS_MS = 50.0
 LOAD = 0.8
 METRIC = "BE kernels/sec at LC p99 <= QoS target"
-WORKLOAD = "resnet50_b1 LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[1])"
+WORKLOAD = "resnet50_b{b} LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[3])"
 
 
 # ----------------------------------------------------------------------------- helpers
@@ -285,11 +287,12 @@ def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
 
 
 # ----------------------------------------------------------------------------- CPU oracle baseline
-def cpu_oracle_sample(small=False):
+def cpu_oracle_sample(small=False, batch=32):
     """The oracle as it stands on a bounded sample of the same workload: oracle conv of two
-    ResNet-50 layers + one stencil sweep (512x512x64, or an 8-plane slab scaled x8 when small)
-    + one mri-q 1024-k chunk on 4096 (small: 256) of the 64^3 voxels, time scaled to the full
-    kernel.  Returns BE kernels/s = 1 / mean (LC conv + BE kernel) pair time."""
+    ResNet-50 layers on one image (time x batch: the conv is linear in the batch) + one stencil
+    sweep (512x512x64, or an 8-plane slab scaled x8 when small) + one mri-q 1024-k chunk on 4096
+    (small: 256) of the 64^3 voxels, time scaled to the full kernel.  Returns BE kernels/s =
+    1 / mean (LC conv + BE kernel) pair time."""
     import synth
     from oracle import be as obe, lc as olc
     convs = synth.resnet50_convs(1)
@@ -299,7 +302,7 @@ def cpu_oracle_sample(small=False):
     cs = convs[5]
     x, w, _ = synth.conv_inputs(cs, 1)
     olc.lc_conv(x, w, cs.stride, cs.pad)
-    tc = time.perf_counter() - t0
+    tc = (time.perf_counter() - t0) * batch
     A = synth.stencil_inputs(512, 512, nz, 2022)
     t0 = time.perf_counter()
     obe.stencil(A, np.float32(1 / 6), np.float32(1 / 36))
@@ -308,7 +311,7 @@ def cpu_oracle_sample(small=False):
     cs = convs[20]
     x, w, _ = synth.conv_inputs(cs, 2)
     olc.lc_conv(x, w, cs.stride, cs.pad)
-    tc = time.perf_counter() - t0
+    tc = (time.perf_counter() - t0) * batch
     d = synth.mriq_inputs(64, 1024, 2022)
     pm, _ = obe.mriq_phimag(d["phiR"], d["phiI"])
     sub = 256 if small else 4096
@@ -316,7 +319,7 @@ def cpu_oracle_sample(small=False):
     obe.mriq_q(d["x"][:sub], d["y"][:sub], d["z"][:sub], d["kx"], d["ky"], d["kz"], pm)
     t_pairs.append(tc + (time.perf_counter() - t0) * (64 ** 3 / sub))
     per = sum(t_pairs) / len(t_pairs)
-    desc = (f"oracle conv (2 ResNet-50 b1 layers) + 1 stencil 512x512x64 sweep ({'8-plane slab x8' if small else 'full'})"
+    desc = (f"oracle conv (2 ResNet-50 layers, 1 image, time x{batch}) + 1 stencil 512x512x64 sweep ({'8-plane slab x8' if small else 'full'})"
             f" + 1 mri-q 1024-k chunk on {sub} of 64^3 voxels (time scaled x{64 ** 3 // sub}); "
             "BE kernels/s = 1 / mean pair time")
     return {"value": 1.0 / per, "unit": "BE kernels/s", "cores": _oracle_threads(), "kind": "oracle",
@@ -340,7 +343,7 @@ def run_reference(args, ws, rank):
     t0 = time.perf_counter()
     vals, r = [], None
     for _ in range(args.steps):
-        r = cpu_oracle_sample(small=True)
+        r = cpu_oracle_sample(small=True, batch=args.batch)
         vals.append(r["seconds_per_be_kernel"])
         if time.perf_counter() - t0 > 120.0:
             break
@@ -349,11 +352,53 @@ def run_reference(args, ws, rank):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "BE kernels/s", "n_gpus": ws,
             "steps": len(vals), "warmup": args.warmup, "ms_per_step": el * 1000 / len(vals),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": WORKLOAD, "l2": "n/a (CPU)"},
+            "config": {"workload": WORKLOAD.format(b=args.batch), "l2": "n/a (CPU)"},
             "cpu_baseline": {"value": v, "unit": "BE kernels/s", "cores": r["cores"], "kind": "oracle",
                              "sample": "per step: " + r["sample"]},
             "e2e": {"value": v, "unit": "BE kernels/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
+
+
+def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "tacker_slice")):
+    """The same Poisson trace under each policy (the headline Tacker run first, timed by the
+    caller's window); returns {variant: result}."""
+    out = {}
+    kw = {"tacker": (tk.POLICY_TACKER, {}), "baymax": (tk.POLICY_BAYMAX, {}),
+          "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True})}
+    for v in variants:
+        pol, extra = kw[v]
+        out[v] = q.run(pol, steps, load=LOAD, seed=seed, max_inflight=inflight, **extra)
+    return out
+
+
+def lc_class_roofline(q, peaks, peak_kind, svc):
+    """Roofline of the LC tensor-core kernels (the dominant launch class of the managed run):
+    per kernel the algorithmic flops (2 NPQ K CRS) and bytes (x, w, out once), timed back to back
+    with CUDA events on the launching stream (QosRun.calibrate).  The bound is the one that gives
+    the larger roofline time summed over the query."""
+    off = 1 if getattr(q, "io", None) else 0
+    tc = [(k, q.t_lc[i + off]) for i, k in enumerate(svc.kernels) if k.is_tc]
+    p_t, bw = peaks["bf16_tflops"] * 1e12, peaks["hbm_gbs"] * 1e9
+    fl = sum(k.flops for k, _ in tc)
+    by = sum(k.bytes for k, _ in tc)
+    t_ms = sum(t for _, t in tc)
+    t_roof = sum(max(k.flops / p_t, k.bytes / bw) for k, _ in tc)
+    n = len(tc)
+    if fl / p_t >= by / bw:
+        ach = fl / n / (t_ms / n / 1e3) / 1e12
+        roof = {"bound": "tensor", "achieved": ach, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
+                "frac": ach / peaks["bf16_tflops"], "per_launch_work": "mean 2*NPQ*K*CRS of the TC convs",
+                "peak_source": f"MEASURED_PEAKS.json bf16_tflops burst ({peak_kind}); fp16 = bf16 rate"}
+    else:
+        ach = by / n / (t_ms / n / 1e3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": ach / peaks["hbm_gbs"], "per_launch_work": "mean 2*(NHWC + KRSC + NPQK) bytes of the TC convs",
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
+    roof.update(traffic=None, kernel=f"LC tensor-core convs of {svc.name} (implicit GEMM tcgen05, split-K where few tiles)",
+                avg_launch_ms=t_ms / n, launches_per_query=n,
+                per_kernel_roofline_frac=t_roof * 1e3 / t_ms,
+                stream="launching stream, back-to-back launches (CUDA events)")
+    return roof
 
 
 def run_tacker(args, ws, rank, local):
@@ -362,7 +407,7 @@ def run_tacker(args, ws, rank, local):
 
     peaks, peak_kind = measured_peaks()
     seed = 2022 + rank
-    svc = sv.resnet50_service(1, seed)
+    svc = sv.resnet50_service(args.batch, seed)
     stencil = sv.stencil_app(512, 512, 64, seed)
     mriq = sv.mriq_app(64, 2048, 1024, seed)
     tk.tacker_launch_original(None, mriq.kernels[0].desc)       # phiMag ready for the Q chunks
@@ -371,12 +416,13 @@ def run_tacker(args, ws, rank, local):
     def flush():
         flush_buf.fill_(1.0)
 
-    # ---- calibration (predictor, §VI-C) -- untimed
+    # ---- calibration (predictor, §VI-C) and the peak LC load -- untimed
     tk.tacker_model_clear()
     q = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
     q.calibrate()
+    q.measure_service(max_inflight=args.inflight)
     # ---- warm-up queries (untimed)
-    q.run(tk.POLICY_TACKER, max(args.warmup, 3), load=LOAD, seed=1000 + rank)
+    q.run(tk.POLICY_TACKER, max(args.warmup, 3), load=LOAD, seed=1000 + rank, max_inflight=args.inflight)
     torch.cuda.synchronize()
 
     # ---- timed region: K queries under the Tacker policy
@@ -385,7 +431,7 @@ def run_tacker(args, ws, rank, local):
     barrier(ws)
     torch.cuda.synchronize()
     torch.cuda.nvtx.range_push("timed")      # ncu --nvtx --nvtx-include "timed/" selects these launches
-    res = q.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank)
+    res = q.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank, max_inflight=args.inflight)
     torch.cuda.nvtx.range_pop()
     torch.cuda.synchronize()
     barrier(ws)
@@ -395,71 +441,60 @@ def run_tacker(args, ws, rank, local):
     value = be_total / (elapsed_ms / 1e3)
     p99 = reduce_ranks(ws, res["lc_p99_ms"], "max")
 
-    # ---- Baymax on the same trace (Eq. 10)
-    bay = q.run(tk.POLICY_BAYMAX, args.steps, load=LOAD, seed=2000 + rank)
+    # ---- Baymax (Eq. 10) and PTB-sliced Tacker on the same trace
+    other = managed_runs(q, tk, args.steps, 2000 + rank, args.inflight, ("baymax", "tacker_slice"))
+    bay, slc = other["baymax"], other["tacker_slice"]
 
     # ---- e2e: the same managed run, each query with its H2D input + D2H result
     qi = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS).with_io()
-    qi.pairs, qi.ws_of = q.pairs, q.ws_of
-    qi.t_be = q.t_be
+    qi.pairs, qi.ws_of, qi.t_be, qi.lr_be = q.pairs, q.ws_of, q.t_be, q.lr_be
     qi.t_lc = []
     for is_tc, d in qi._kernel_list():
         qi.t_lc.append(qos._time(lambda: tk.tacker_launch_original(d, None) if is_tc
                                   else tk.tacker_launch_original(None, d), 5))
-    e2e = qi.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank)
+    qi.measure_service(max_inflight=args.inflight)
+    e2e = qi.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank, max_inflight=args.inflight)
     e2e_value = reduce_ranks(ws, e2e["be_kernels"], "sum") / (reduce_ranks(ws, e2e["elapsed_ms"], "max") / 1e3)
 
-    # ---- kernel-level fused step + roofline of the dominant fused kernel
-    step = FusedStep(svc, stencil, mriq, args.warp_split)
-    for _ in range(3):
-        step.fused()
-    torch.cuda.synchronize()
-    fstep, roof_fused = kernel_level(torch, step, flush, peaks, peak_kind, clocks, max(5, min(args.steps, 20)))
-
-    # ---- roofline of the dominant launch class of the timed managed run (CUDA events around every
-    #      launch on the manager stream, accumulated by the manager per class)
+    # ---- roofline of the dominant launch class of the timed run (class shares from the manager's
+    #      sampled CUDA events on its stream)
     cms, cn = res["class_ms"], res["class_launches"]
     tot_ms = sum(cms.values()) or 1.0
     shares = {c: {"ms": cms[c], "launches": cn[c], "share": cms[c] / tot_ms} for c in cms}
     dom = max(cms, key=cms.get)
-    if dom == "lc_tc":
-        tc = [k for k in svc.kernels if k.is_tc]
-        avg_flops = sum(k.flops for k in tc) / len(tc)
-        avg_ms = cms[dom] / max(cn[dom], 1)
-        achieved = avg_flops / (avg_ms / 1e3) / 1e12
-        peak = peaks["bf16_tflops"]
-        roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-                "traffic": None, "kernel": "LC tensor-core original launches (ResNet-50 b1 implicit-GEMM convs)",
-                "avg_launch_ms": avg_ms, "launches": cn[dom],
-                "per_launch_work": "mean 2*NPQ*K*CRS of the 53 convs (conv1 as GEMM)",
-                "peak_source": f"MEASURED_PEAKS.json bf16_tflops burst ({peak_kind}); fp16 = bf16 rate"}
+
+    # ---- BASELINE configs[1]: ResNet-50 batch-1 convs fused with stencil / mri-q -- the kernel-
+    #      level fused step (fused time vs overlap roofline) and the same managed protocol
+    svc1 = sv.resnet50_service(1, seed)
+    step = FusedStep(svc1, stencil, mriq, args.warp_split)
+    for _ in range(3):
+        step.fused()
+    torch.cuda.synchronize()
+    fstep, roof_fused = kernel_level(torch, step, flush, peaks, peak_kind, clocks, max(5, min(args.steps, 20)))
+    b1 = None
+    if not args.no_extra:
+        tk.tacker_model_clear()
+        q1 = qos.QosRun(svc1, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
+        q1.calibrate()
+        q1.measure_service(max_inflight=args.inflight)
+        q1.run(tk.POLICY_TACKER, 20, load=LOAD, seed=1000 + rank, max_inflight=args.inflight)
+        r1 = managed_runs(q1, tk, 1000, 3000 + rank, args.inflight)
+        b1 = {"workload": "resnet50_b1 LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[1], config-4 protocol)",
+              "queries": 1000, "service_ms": q1.service_ms, "lc_roofline": lc_class_roofline(q1, peaks, peak_kind, svc1)}
+        for v, r in r1.items():
+            b1[v] = {k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p50_ms", "lc_p99_ms", "qos_met",
+                                        "fused", "reordered", "idle_be")}
+        for v in ("tacker", "tacker_slice"):
+            b1[v]["improvement_vs_baymax_eq10"] = r1[v]["be_kernels_per_s"] / r1["baymax"]["be_kernels_per_s"] - 1
+            b1[v]["improvement_vs_baymax_eq10_normalised"] = r1[v]["be_norm_thpt"] / r1["baymax"]["be_norm_thpt"] - 1
+
+    if dom in ("lc_tc", "lc_cd"):
+        roof = lc_class_roofline(q, peaks, peak_kind, svc)
     else:
         roof = dict(roof_fused)
     roof["class_shares"] = shares
-    roof["stream"] = "manager stream (CUDA events around each launch)"
 
-    # ---- config 4: the same BE queue beside ResNet-50 batch 32 (Table II's
-    #      batch), where every conv spans all SMs -- reported beside the headline, not in it
-    extra = None
-    if not args.no_extra:
-        svc32 = sv.resnet50_service(32, seed)
-        tk.tacker_model_clear()
-        q32 = qos.QosRun(svc32, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
-        q32.calibrate()
-        q32.run(tk.POLICY_TACKER, 10, load=LOAD, seed=1000 + rank)
-        n32 = max(50, args.steps // 3)
-        t32 = q32.run(tk.POLICY_TACKER, n32, load=LOAD, seed=3000 + rank)
-        b32 = q32.run(tk.POLICY_BAYMAX, n32, load=LOAD, seed=3000 + rank)
-        extra = {"workload": "resnet50_b32 LC + stencil/mriq BE queue, QoS 50 ms (SURVEY config 4)",
-                 "queries": n32, "query_solo_ms": t32["query_solo_ms"],
-                 "tacker": {k: t32[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p50_ms", "lc_p99_ms",
-                                                 "qos_met", "fused", "reordered", "fused_pred_err_mean")},
-                 "baymax": {k: b32[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p50_ms", "lc_p99_ms",
-                                                 "qos_met", "reordered")},
-                 "improvement_vs_baymax_eq10": t32["be_kernels_per_s"] / b32["be_kernels_per_s"] - 1.0,
-                 "improvement_vs_baymax_eq10_normalised": t32["be_norm_thpt"] / b32["be_norm_thpt"] - 1.0}
-
-    cpu = cpu_oracle_sample() if (rank == 0 and ws == 1 and not args.no_cpu) else None
+    cpu = cpu_oracle_sample(batch=args.batch) if (rank == 0 and ws == 1 and not args.no_cpu) else None
     if cpu is not None:
         cpu.pop("seconds_per_be_kernel", None)
 
@@ -468,14 +503,16 @@ def run_tacker(args, ws, rank, local):
         "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "f16xf16->f32 (LC tcgen05) + f32 (BE CUDA cores)",
         "data": "synthetic (seeded inputs, random weights)",
-        "config": {"workload": WORKLOAD, "lc": "ResNet-50 batch-1, 53 convs, fp16 NHWC, implicit GEMM tcgen05",
+        "config": {"workload": WORKLOAD.format(b=args.batch),
+                   "lc": f"ResNet-50 batch-{args.batch} (Table II), 53 convs, fp16 NHWC, implicit GEMM tcgen05",
                    "be": "stencil 512x512x64 sweeps | mri-q 64^3 x (phiMag + 2 x 1024-k chunks)",
-                   "arrivals": f"Poisson at {LOAD:.0%} of the peak rate (1 / standalone query time)",
-                   "qos_ms": QOS_MS, "policy": "tacker", "warp_split": args.warp_split,
+                   "arrivals": f"Poisson at {LOAD:.0%} of the peak rate (the manager's LC-only service rate)",
+                   "qos_ms": QOS_MS, "policy": "tacker", "warp_split": args.warp_split, "max_inflight": args.inflight,
                    "step": "one LC query", "parallelism": f"replicas x{ws}",
-                   "l2": "inputs larger than L2 (stencil 2 x 64 MiB ping-pong + ResNet-50 weights 50 MB)"},
+                   "l2": "inputs larger than L2 (stencil 2 x 64 MiB ping-pong + activations and weights > 1 GB)"},
         "lc_p99_ms": p99, "lc_p50_ms": res["lc_p50_ms"], "lc_qos_ms": QOS_MS, "qos_met": p99 <= QOS_MS,
-        "lambda_per_s": res["lambda_per_s"], "fused_launches": res["fused"], "reordered_be": res["reordered"],
+        "lambda_per_s": res["lambda_per_s"], "service_ms": q.service_ms, "query_solo_ms": q.query_solo_ms(),
+        "fused_launches": res["fused"], "reordered_be": res["reordered"],
         "idle_be": res["idle_be"], "model_refits": res["model_refits"],
         "baymax": {"value": bay["be_kernels_per_s"], "lc_p99_ms": bay["lc_p99_ms"], "qos_met": bay["qos_met"],
                    "be_norm_thpt": bay["be_norm_thpt"]},
@@ -483,11 +520,14 @@ def run_tacker(args, ws, rank, local):
         # BE work in standalone-kernel milliseconds per wall millisecond (app-length independent)
         "be_norm_thpt": res["be_norm_thpt"],
         "improvement_vs_baymax_eq10_normalised": res["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0,
+        "tacker_slice": {"value": slc["be_kernels_per_s"], "be_norm_thpt": slc["be_norm_thpt"],
+                         "lc_p99_ms": slc["lc_p99_ms"], "fused": slc["fused"],
+                         "improvement_vs_baymax_eq10_normalised": slc["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0},
         "fused_pred_err_mean": res["fused_pred_err_mean"],
         "pair_pred_err_mean": statistics.mean(q.pair_err) if q.pair_err else None,
-        "fused_step": fstep,
         "roofline": roof,
         "roofline_fused": roof_fused,
+        "fused_step": fstep,
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": "BE kernels/s", "h2d_bytes_per_step": qi.h2d_bytes,
                 "d2h_bytes_per_step": qi.d2h_bytes, "lc_p99_ms": e2e["lc_p99_ms"],
@@ -497,7 +537,7 @@ def run_tacker(args, ws, rank, local):
         # reordered and idle-time BE launches
         "gpu_launches": int(sum(res["class_launches"].values())),
         "clocks": clocks,
-        "config4_resnet50_b32": extra,
+        "config1_resnet50_b1": b1,
     }
     if rank == 0:
         print(json.dumps(line))
@@ -542,7 +582,7 @@ def run_simulated(args, ws, rank):
     line = {"metric": METRIC, "value": value, "unit": "BE kernels/s", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "n/a (simulated GPU)", "data": "synthetic",
-            "config": {"workload": WORKLOAD + " [simulated durations]", "parallelism": f"replicas x{ws}"},
+            "config": {"workload": WORKLOAD.format(b=1) + " [simulated durations]", "parallelism": f"replicas x{ws}"},
             "lc_p99_ms": reduce_ranks(ws, p99, "max"), "baymax": {"value": bay},
             "improvement_vs_baymax_eq10": value / bay - 1.0, "simulated": True}
     if rank == 0:
@@ -552,12 +592,14 @@ def run_simulated(args, ws, rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=1000, help="timed LC queries")
+    ap.add_argument("--steps", type=int, default=300, help="timed LC queries")
+    ap.add_argument("--batch", type=int, default=32, help="LC batch (Table II: ResNet-50 at 32)")
+    ap.add_argument("--inflight", type=int, default=16, help="manager: launches in flight on its stream")
     ap.add_argument("--warmup", type=int, default=20, help="untimed warm-up LC queries")
     ap.add_argument("--impl", default="tacker", choices=["tacker", "reference"])
     ap.add_argument("--warp-split", type=int, default=24)
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--no-extra", action="store_true", help="skip the ResNet-50 b32 (config 4) side run")
+    ap.add_argument("--no-extra", action="store_true", help="skip the ResNet-50 b1 (configs[1]) managed side run")
     ap.add_argument("--simulate", action="store_true", help="CPU-only: manager on its simulated GPU (gloo)")
     args = ap.parse_args()
     if args.impl == "reference":

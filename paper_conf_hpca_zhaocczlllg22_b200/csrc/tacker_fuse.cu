@@ -366,9 +366,17 @@ static BeFn pick_be_original(int kind) {
   }
 }
 
+// The dynamic-SMEM limit is a per-function attribute shared by every plan of that instantiation:
+// only ever raise it (a later, smaller plan must not invalidate the launches of an earlier one).
 static tacker_status set_smem_attr(const void *fn, int bytes) {
+  static std::mutex mu;
+  static std::unordered_map<const void *, int> limit;
+  std::lock_guard<std::mutex> g(mu);
+  int &cur = limit[fn];
+  if (bytes <= cur) return TACKER_OK;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   if (e != cudaSuccess) return cuda_fail("cudaFuncSetAttribute", e);
+  cur = bytes;
   return TACKER_OK;
 }
 

@@ -341,3 +341,18 @@ def test_fused_split_k_conv_bit_identical(tk):
             assert host(g).tobytes() == a.tobytes()
     ref, S = olc.lc_conv(x, w, 1, 1, bias=b, relu=True)
     assert max_rel_err(host(o1).astype(np.float64), ref, S) <= 1e-2
+
+
+def test_plans_of_one_instantiation_keep_their_smem(tk):
+    # two plans of the same fused_kernel<BN, BE> with different SMEM sizes: building the smaller
+    # one after the larger must not lower the function's dynamic-SMEM limit under the larger one
+    A, B = synth.lc_gemm_inputs(256, 256, 128, seed=2)
+    D = torch.zeros(256, 256, device=dev())
+    c = be_case(tk.BE_STENCIL, seed=1)
+    big = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], 24)
+    small = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], 4)
+    assert big.info().smem_bytes > small.info().smem_bytes
+    c["reset"]()
+    big.launch()
+    small.launch()
+    torch.cuda.synchronize()
