@@ -62,7 +62,7 @@ int tacker_device_sm_count(void);
  *        M = n*p*q, N = k, K = c*r*s.  Constraints: c % 64 == 0 or (r == s == 1 and c % 8 == 0)
  *        or c == 8 (conv1 padded); k % 8 == 0.
  * Epilogue (both): D = act(acc + bias[j] + residual[i,j]) with optional fp32 bias [N], fp16
- *        residual with D's layout, ReLU.
+ *        residual with D's layout, ReLU.  D, bias and residual 16-byte aligned (EINVAL).
  */
 typedef enum { TACKER_LC_NONE = 0, TACKER_LC_GEMM_F16 = 1, TACKER_LC_CONV_F16 = 2 } tacker_lc_kind;
 enum { TACKER_F32 = 0, TACKER_F16 = 1 };

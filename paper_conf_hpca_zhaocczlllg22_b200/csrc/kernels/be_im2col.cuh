@@ -18,42 +18,53 @@ template <> struct BeBody<TACKER_BE_IM2COL> {
     return (rows(p) * (p.Kpad / 8) + 1023) / 1024;
   }
   static __device__ __forceinline__ void run(const tacker_be_im2col &p, int64_t vb, int tid, uint32_t, uint8_t *) {
-    const int P = (p.h + 2 * p.pad - p.r) / p.stride + 1, Q = (p.w + 2 * p.pad - p.s) / p.stride + 1;
-    const int64_t groups_per_row = p.Kpad / 8;
-    const int64_t total = (int64_t)p.n * P * Q * groups_per_row;
+    // 32-bit index math (the host bounds rows * Kpad / 8 < 2^31); (r, s, c) of a group's 8
+    // columns is stepped incrementally instead of divided per element
+    const uint32_t P = (uint32_t)((p.h + 2 * p.pad - p.r) / p.stride + 1);
+    const uint32_t Q = (uint32_t)((p.w + 2 * p.pad - p.s) / p.stride + 1);
+    const uint32_t gpr = (uint32_t)(p.Kpad / 8);
+    const uint32_t total = (uint32_t)p.n * P * Q * gpr;
     const int Kreal = p.r * p.s * p.c;
     const __half *x = reinterpret_cast<const __half *>(p.x);
     __half *out = reinterpret_cast<__half *>(p.out);
 #pragma unroll 2
     for (int u = 0; u < 8; ++u) {
-      const int64_t g = vb * 1024 + u * 128 + tid;
+      const uint32_t g = (uint32_t)vb * 1024u + (uint32_t)(u * 128 + tid);
       if (g >= total) return;
-      const int64_t m = g / groups_per_row;
-      const int kk0 = (int)(g % groups_per_row) * 8;
-      const int q = (int)(m % Q), pp = (int)((m / Q) % P), n = (int)(m / ((int64_t)P * Q));
+      const uint32_t m = g / gpr;
+      const int kk0 = (int)(g - m * gpr) * 8;
+      const uint32_t mq = m / Q;
+      const int q = (int)(m - mq * Q), pp = (int)(mq % P), n = (int)(mq / P);
+      const int h0 = pp * p.stride - p.pad, w0 = q * p.stride - p.pad;
+      const __half *xn = x + (int64_t)n * p.h * p.w * p.c;
       uint4 v = make_uint4(0, 0, 0, 0);
       if ((p.c & 7) == 0) {
         if (kk0 < Kreal) {
           const int c = kk0 % p.c, rs = kk0 / p.c, s = rs % p.s, r = rs / p.s;
-          const int hi = pp * p.stride - p.pad + r, wi = q * p.stride - p.pad + s;
+          const int hi = h0 + r, wi = w0 + s;
           if (hi >= 0 && hi < p.h && wi >= 0 && wi < p.w)
-            v = __ldg(reinterpret_cast<const uint4 *>(x + (((int64_t)n * p.h + hi) * p.w + wi) * p.c + c));
+            v = __ldg(reinterpret_cast<const uint4 *>(xn + ((int64_t)hi * p.w + wi) * p.c + c));
         }
       } else {
         __align__(16) __half e[8];
+        int c = kk0 % p.c, rs = kk0 / p.c;
+        int s = rs % p.s, r = rs / p.s;
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          const int kk = kk0 + j;
           e[j] = __float2half(0.f);
-          if (kk < Kreal) {
-            const int c = kk % p.c, rs = kk / p.c, s = rs % p.s, r = rs / p.s;
-            const int hi = pp * p.stride - p.pad + r, wi = q * p.stride - p.pad + s;
-            if (hi >= 0 && hi < p.h && wi >= 0 && wi < p.w) e[j] = x[(((int64_t)n * p.h + hi) * p.w + wi) * p.c + c];
+          const int hi = h0 + r, wi = w0 + s;
+          if (kk0 + j < Kreal && hi >= 0 && hi < p.h && wi >= 0 && wi < p.w) e[j] = xn[((int64_t)hi * p.w + wi) * p.c + c];
+          if (++c == p.c) {
+            c = 0;
+            if (++s == p.s) {
+              s = 0;
+              ++r;
+            }
           }
         }
         v = *reinterpret_cast<uint4 *>(e);
       }
-      *reinterpret_cast<uint4 *>(out + m * p.Kpad + kk0) = v;
+      *reinterpret_cast<uint4 *>(out + (int64_t)m * p.Kpad + kk0) = v;
     }
   }
 };

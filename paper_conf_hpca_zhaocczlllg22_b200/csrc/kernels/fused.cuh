@@ -84,13 +84,15 @@ struct LcGemm {
   struct Bars {
     uint64_t *full, *empty, *tfull, *tempty;
     uint32_t *tmem_holder;
+    float *bias;             // the current tile's BN bias values (epilogue warps)
   };
   static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
     return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
   }
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * kStage);
-    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4)};
+    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4),
+                reinterpret_cast<float *>(b + 2 * stages + 6)};
   }
 
   static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
@@ -116,31 +118,40 @@ struct LcGemm {
     const int m = mt * kBM + r;
     return m < L.M ? m : -1;
   }
-  // epilogue of 4 consecutive columns n..n+3 of output row orow: bias, residual, ReLU, store
-  static __device__ __forceinline__ void store4(const LcParams &L, int64_t orow, int n, float f0, float f1, float f2,
-                                                float f3) {
-    float f[4] = {f0, f1, f2, f3};
+  // epilogue of 8 consecutive columns n..n+7 of output row orow (N % 8 == 0: a group is all in or
+  // all out): + bias (preloaded, bias8 = bias[n..n+7]), + residual, ReLU, one 16-byte (fp16) or
+  // two 16-byte (fp32) stores
+  static __device__ __forceinline__ void store8(const LcParams &L, int64_t orow, int n, float (&f)[8],
+                                                const float *bias8) {
     if (L.epi & TACKER_EPI_BIAS) {
 #pragma unroll
-      for (int j = 0; j < 4; ++j) f[j] = __fadd_rn(f[j], __ldg(L.bias + n + j));
+      for (int j = 0; j < 8; ++j) f[j] = __fadd_rn(f[j], bias8[j]);
     }
     if (L.epi & TACKER_EPI_RESIDUAL) {
-      const __half *rp = L.residual + orow * L.N + n;
+      const uint4 rv = *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n);
+      const __half2 *rh = reinterpret_cast<const __half2 *>(&rv);
 #pragma unroll
-      for (int j = 0; j < 4; ++j) f[j] = __fadd_rn(f[j], __half2float(rp[j]));
+      for (int j = 0; j < 4; ++j) {
+        const float2 r2 = __half22float2(rh[j]);
+        f[2 * j] = __fadd_rn(f[2 * j], r2.x);
+        f[2 * j + 1] = __fadd_rn(f[2 * j + 1], r2.y);
+      }
     }
     if (L.epi & TACKER_EPI_RELU) {
 #pragma unroll
-      for (int j = 0; j < 4; ++j) f[j] = fmaxf(f[j], 0.f);
+      for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.f);
     }
     if (L.d_f16) {
-      __align__(8) __half2 hv[2] = {__floats2half2_rn(f[0], f[1]), __floats2half2_rn(f[2], f[3])};
-      *reinterpret_cast<uint2 *>(reinterpret_cast<__half *>(L.D) + orow * L.N + n) = *reinterpret_cast<uint2 *>(hv);
+      __align__(16) __half2 hv[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) hv[j] = __floats2half2_rn(f[2 * j], f[2 * j + 1]);
+      *reinterpret_cast<uint4 *>(reinterpret_cast<__half *>(L.D) + orow * L.N + n) = *reinterpret_cast<uint4 *>(hv);
     } else {
-      *reinterpret_cast<float4 *>(reinterpret_cast<float *>(L.D) + orow * L.N + n) = make_float4(f[0], f[1], f[2], f[3]);
+      float4 *dp = reinterpret_cast<float4 *>(reinterpret_cast<float *>(L.D) + orow * L.N + n);
+      dp[0] = make_float4(f[0], f[1], f[2], f[3]);
+      dp[1] = make_float4(f[4], f[5], f[6], f[7]);
     }
   }
-
   // B (weights) k-block kb of N-tile nt
   static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
     const LcParams &L = P.lc;
@@ -260,24 +271,34 @@ struct LcGemm {
       const int64_t orow = out_row(L, mt, row_in_tile);
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
       float *prow = L.splits > 1 ? L.part + ((size_t)u * kBM + row_in_tile) * BN : nullptr;
+      const bool bias = !prow && (L.epi & TACKER_EPI_BIAS);
+      if (bias) {   // stage this tile's bias in shared memory (read as a broadcast per column)
+        const int et = (int)threadIdx.x % 128;
+        named_bar_sync(kLcEpiBar, 128);           // the previous tile's readers are done
+        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(kLcEpiBar, 128);
+      }
 #pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 32) {
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tbase + c0, v);
+      for (int c0 = 0; c0 < BN; c0 += 16) {
+        uint32_t v[16];
+        tmem_ld_32x32b_x16(tbase + c0, v);
         tmem_ld_wait();
         const int n0 = nt * BN + c0;
         if (orow < 0 || n0 >= L.N) continue;
         if (prow) {   // split-K partial, fp32
 #pragma unroll
-          for (int j = 0; j < 32; j += 4)
+          for (int j = 0; j < 16; j += 4)
             *reinterpret_cast<float4 *>(prow + c0 + j) = make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]),
                                                                     __uint_as_float(v[j + 2]), __uint_as_float(v[j + 3]));
         } else {
 #pragma unroll
-          for (int j = 0; j < 32; j += 4)   // N % 8 == 0: a group of 4 is all in or all out
-            if (n0 + j < L.N)
-              store4(L, orow, n0 + j, __uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
-                     __uint_as_float(v[j + 3]));
+          for (int j = 0; j < 16; j += 8)
+            if (n0 + j < L.N) {
+              float f[8];
+#pragma unroll
+              for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j + u]);
+              store8(L, orow, n0 + j, f, bb.bias + c0 + j);
+            }
         }
       }
       tc_fence_before();
@@ -305,24 +326,29 @@ struct LcGemm {
       }
     }
     named_bar_sync(kLcEpiBar, 128);
-    constexpr int G = BN / 4;                   // column groups per row
+    constexpr int G = BN / 8;                   // 8-column groups per row
     const int E = kBM * G;
     const float *base = L.part + (size_t)t * S * kBM * BN;
     for (int g = E * sp / S + et; g < E * (sp + 1) / S; g += 128) {
-      const int r = g / G, c = (g % G) * 4;
+      const int r = g / G, c = (g % G) * 8;
       const int64_t orow = out_row(L, mt, r);
       const int n = nt * BN + c;
       if (orow < 0 || n >= L.N) continue;
       const float *q = base + (size_t)r * BN + c;
-      float4 a = __ldcg(reinterpret_cast<const float4 *>(q));
+      float4 a0 = __ldcg(reinterpret_cast<const float4 *>(q)), a1 = __ldcg(reinterpret_cast<const float4 *>(q + 4));
       for (int k = 1; k < S; ++k) {
-        const float4 b = __ldcg(reinterpret_cast<const float4 *>(q + (size_t)k * kBM * BN));
-        a.x = __fadd_rn(a.x, b.x);
-        a.y = __fadd_rn(a.y, b.y);
-        a.z = __fadd_rn(a.z, b.z);
-        a.w = __fadd_rn(a.w, b.w);
+        const float4 b0 = __ldcg(reinterpret_cast<const float4 *>(q + (size_t)k * kBM * BN));
+        const float4 b1 = __ldcg(reinterpret_cast<const float4 *>(q + (size_t)k * kBM * BN + 4));
+        a0 = make_float4(__fadd_rn(a0.x, b0.x), __fadd_rn(a0.y, b0.y), __fadd_rn(a0.z, b0.z), __fadd_rn(a0.w, b0.w));
+        a1 = make_float4(__fadd_rn(a1.x, b1.x), __fadd_rn(a1.y, b1.y), __fadd_rn(a1.z, b1.z), __fadd_rn(a1.w, b1.w));
       }
-      store4(L, orow, n, a.x, a.y, a.z, a.w);
+      float f[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+      __align__(16) float bias[8];
+      if (L.epi & TACKER_EPI_BIAS) {
+        *reinterpret_cast<float4 *>(bias) = __ldg(reinterpret_cast<const float4 *>(L.bias + n));
+        *reinterpret_cast<float4 *>(bias + 4) = __ldg(reinterpret_cast<const float4 *>(L.bias + n + 4));
+      }
+      store8(L, orow, n, f, bias);
     }
     named_bar_sync(kLcEpiBar, 128);
     if (et == 0 && atomicAdd(finish, 1u) == (uint32_t)S - 1) {   // last reducer: reset for the next launch

@@ -180,6 +180,8 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
           !p.x || !p.out)
         return set_error("im2col: bad args"), TACKER_EINVAL;
       if (p.Kpad % 8 || p.Kpad < p.r * p.s * p.c) return set_error("im2col: Kpad must be a multiple of 8 >= R*S*C"), TACKER_EINVAL;
+      if (BeBody<TACKER_BE_IM2COL>::rows(p) * (p.Kpad / 8) >= (int64_t)1 << 31)
+        return set_error("im2col: rows * Kpad / 8 must be < 2^31"), TACKER_EUNSUPPORTED;
       break;
     }
     case TACKER_BE_FMA_BURN:
@@ -229,6 +231,9 @@ static tacker_status lc_view(const tacker_lc_desc &d, LcParams &L) {
   if ((d.epi_flags & TACKER_EPI_BIAS) && !d.bias) return set_error("LC: bias flag without bias"), TACKER_EINVAL;
   if ((d.epi_flags & TACKER_EPI_RESIDUAL) && !d.residual) return set_error("LC: residual flag without residual"), TACKER_EINVAL;
   if (d.d_dtype != TACKER_F32 && d.d_dtype != TACKER_F16) return set_error("LC: bad d_dtype"), TACKER_EINVAL;
+  // the epilogue moves 8 columns at a time with 16-byte accesses
+  if (((uintptr_t)d.D | (uintptr_t)d.bias | (uintptr_t)d.residual) & 15)
+    return set_error("LC: D, bias and residual must be 16-byte aligned"), TACKER_EINVAL;
   L.D = d.D;
   L.d_f16 = d.d_dtype == TACKER_F16;
   L.epi = d.epi_flags;
@@ -457,13 +462,15 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   uint32_t cols = 32;
   while (cols < (uint32_t)(acc * BN)) cols <<= 1;
 
-  // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages, >= 2) that
-  // still leaves room for the requested BE virtual blocks.
+  // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
+  // >= 2) that still leaves room for the requested BE virtual blocks.
   const uint32_t stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
-  const uint32_t bar_bytes = 256;
+  const uint32_t bar_bytes = 256 + 4 * 256;   // mbarriers + TMEM address + one tile's bias (BN <= 256)
   const uint32_t be_total = (uint32_t)vb * be_slice;
+  // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
+  // SM for the latency-bound implicit-GEMM loads); fused plans stop at 4 so the BE keeps L1
   int stages = 0;
-  for (int s = 4; s >= 2; --s) {
+  for (int s = has_be ? 4 : 8; s >= 2; --s) {
     const uint32_t need = 1024 + s * stage_bytes + bar_bytes + be_total;
     if (need <= (uint32_t)kSmemCap) {
       stages = s;
