@@ -83,7 +83,11 @@ def test_errors_without_gpu(tk):
     d = tk.BeDesc(kind=tk.BE_SGEMM)
     d.p.sgemm = tk.BeSgemm(256, 256, 256, 1.0, 0.0, 1, 1, 1)
     assert tk.tacker_be_num_blocks(d) == 16
-    lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=300, N=136, K=200, A=1, B=1, D=1)
+    lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=300, N=136, K=200, A=16, B=16, D=8)
+    with pytest.raises(tk.TackerError) as e:      # the epilogue's 16-byte stores need an aligned D
+        tk.tacker_lc_num_tiles(lc, 64)
+    assert e.value.status == tk.EINVAL
+    lc.D = 16
     assert tk.tacker_lc_num_tiles(lc, 64) == 3 * 3
     assert tk.tacker_lc_num_tiles(lc, 128) == 3 * 2
     bad = tk.LcDesc(kind=tk.LC_GEMM_F16, M=16, N=12, K=16, A=1, B=1, D=1)
