@@ -196,6 +196,24 @@ class FusedStep:
             if be is not None:
                 self.tk.tacker_launch_original(None, be.desc)
 
+    def two_streams(self):
+        """Co-running baseline (NEXT-4, the paper's Stream co-location of Fig. 20): the LC
+        kernels in order on one stream, the BE kernels in order on another, original kernels,
+        the hardware scheduler interleaving their CTAs; joined back into the current stream."""
+        import torch
+        cur = torch.cuda.current_stream()
+        if not hasattr(self, "_streams"):
+            self._streams = (torch.cuda.Stream(), torch.cuda.Stream())
+        s_lc, s_be = self._streams
+        s_lc.wait_stream(cur)
+        s_be.wait_stream(cur)
+        for k, be, f in self.plan:
+            self.tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd, stream=s_lc)
+            if be is not None:
+                self.tk.tacker_launch_original(None, be.desc, stream=s_be)
+        cur.wait_stream(s_lc)
+        cur.wait_stream(s_be)
+
 
 def time_steps(torch, fn, steps, flush):
     s = torch.cuda.current_stream()
@@ -232,13 +250,15 @@ def per_launch_times(torch, step, reps=3):
 
 
 def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
-    from oracle.metrics import overlap_rate   # Eq. 11 definition only (no oracle compute)
+    from paper_conf_hpca_zhaocczlllg22_b200.qos import overlap_rate   # Eq. 11
     fused_ms = time_steps(torch, step.fused, steps, flush)
     orig_ms = time_steps(torch, step.original, max(3, steps // 2), flush)
     lc_ms = time_steps(torch, step.lc_only, 3, flush)
     be_ms = time_steps(torch, step.be_only, 3, flush)
+    st_ms = time_steps(torch, step.two_streams, max(3, steps // 2), flush)
     t_f, t_s = statistics.median(fused_ms), statistics.median(orig_ms)
     t_lc, t_be = statistics.median(lc_ms), statistics.median(be_ms)
+    t_st = statistics.median(st_ms)
     flush()
     pl = per_launch_times(torch, step)
     dom = max(pl, key=lambda c: sum(x[0] for x in pl[c]))
@@ -277,6 +297,7 @@ def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
         t_roof += max(k.flops / p_tensor, t_be_roof, (k.bytes + be.bytes) / bw)
     fs = {"fused_step_ms": t_f, "sequential_step_ms": t_s, "lc_only_ms": t_lc, "be_only_ms": t_be,
           "speedup_vs_sequential": t_s / t_f, "overlap_rate_eq11": overlap_rate(t_lc, t_be, t_f),
+          "two_streams_step_ms": t_st, "overlap_rate_eq11_two_streams": overlap_rate(t_lc, t_be, t_st),
           "overlap_roofline_ms": t_roof * 1e3, "overlap_roofline_frac": t_roof * 1e3 / t_f,
           "be_kernels_per_s": step.n_fused / (t_f / 1e3), "launches_per_step": len(step.plan)}
     # LC convolutions alone against the tensor peak (batch 1: latency-bound, few tiles)

@@ -11,8 +11,11 @@ constexpr int kVbThreads = 128;
 #ifndef TK_STENCIL_ZC
 #define TK_STENCIL_ZC 4
 #endif
+#ifndef TK_STENCIL_HOIST
+#define TK_STENCIL_HOIST 0
+#endif
 #ifndef TK_MRIQ_COARSEN
-#define TK_MRIQ_COARSEN 2
+#define TK_MRIQ_COARSEN 4
 #endif
 #ifndef TK_MRIQ_REDUCE
 #define TK_MRIQ_REDUCE 0

@@ -51,6 +51,19 @@ template <> struct BeBody<TACKER_BE_STENCIL> {
         c[i] = (act && z >= 0 && z < p.nz) ? __ldg(reinterpret_cast<const float4 *>(A + z * plane + row))
                                            : make_float4(0.f, 0.f, 0.f, 0.f);
       }
+#if TK_STENCIL_HOIST
+      // y-1 / y+1 rows of every plane requested up front too: all of the block's loads in flight
+      // at once (memory-level parallelism for a CTA with few warps, e.g. the fused one)
+      float4 sv[ZC], nv[ZC];
+      const bool inner = act && !ybord;
+#pragma unroll
+      for (int i = 0; i < ZC; ++i) {
+        const int z = z0 + i;
+        const bool ok = inner && z > 0 && z < p.nz - 1;
+        sv[i] = ok ? __ldg(reinterpret_cast<const float4 *>(A + z * plane + row - p.nx)) : make_float4(0.f, 0.f, 0.f, 0.f);
+        nv[i] = ok ? __ldg(reinterpret_cast<const float4 *>(A + z * plane + row + p.nx)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+#endif
 #pragma unroll
       for (int i = 0; i < ZC; ++i) {
         const int z = z0 + i;
@@ -64,8 +77,12 @@ template <> struct BeBody<TACKER_BE_STENCIL> {
         if (!ybord && !zb_) {
           if (lane == 0) wv = x0 > 0 ? __ldg(A + z * plane + row - 1) : 0.f;
           if (lane == 31 || x0 + 4 >= p.nx) ev = x0 + 4 < p.nx ? __ldg(A + z * plane + row + 4) : 0.f;
+#if TK_STENCIL_HOIST
+          const float4 s = sv[i], n = nv[i];
+#else
           const float4 s = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row - p.nx));
           const float4 n = __ldg(reinterpret_cast<const float4 *>(A + z * plane + row + p.nx));
+#endif
           const float4 b = c[i], t = c[i + 2];
           if (x0 > 0) o.x = point(p, wv, cc.y, s.x, n.x, b.x, t.x, cc.x);
           o.y = point(p, cc.x, cc.z, s.y, n.y, b.y, t.y, cc.y);

@@ -22,6 +22,12 @@ import torch
 from . import tacker as tk
 
 
+def overlap_rate(t_tc, t_cd, t_corun):
+    """Eq. 11 (P:3315-3320): (T_TC + T_CD - T_corun) / (T_TC + T_CD) -- 0 for sequential
+    execution, 0.5 for perfect overlap of equal parts."""
+    return (t_tc + t_cd - t_corun) / (t_tc + t_cd)
+
+
 def _prefix(desc, n):
     """Copy of a BE descriptor restricted to its first n original blocks (PTB, Fig. 7)."""
     import ctypes
