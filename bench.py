@@ -415,7 +415,12 @@ def lc_class_roofline(q, peaks, peak_kind, svc):
         roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": ach / peaks["hbm_gbs"], "per_launch_work": "mean 2*(NHWC + KRSC + NPQK) bytes of the TC convs",
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
-    roof.update(traffic=None, kernel=f"LC tensor-core convs of {svc.name} (implicit GEMM tcgen05, split-K where few tiles)",
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp) and svc.name == "resnet50_b32":
+        with open(tp) as f:
+            traffic = json.load(f).get("lc_tc")
+    roof.update(traffic=traffic, kernel=f"LC tensor-core convs of {svc.name} (implicit GEMM tcgen05, split-K where few tiles)",
                 avg_launch_ms=t_ms / n, launches_per_query=n,
                 per_kernel_roofline_frac=t_roof * 1e3 / t_ms,
                 stream="launching stream, back-to-back launches (CUDA events)")
