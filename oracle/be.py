@@ -95,6 +95,66 @@ def mriq_q(x, y, z, kx, ky, kz, phiMag, Qr_in=None, Qi_in=None):
     return Qr, Qi, Sr, Si
 
 
+# ----------------------------------------------------------------------------- NEXT-3 mri-fhd
+def mrifhd_rhophi(phiR, phiI, dR, dI):
+    """ComputeRhoPhi (Parboil mri-fhd, Table II; not defined in the paper, DESIGN.md
+    §2 reading 14): rRhoPhi = phiR*dR + phiI*dI, iRhoPhi = phiR*dI - phiI*dR.  Returns
+    (rRhoPhi, iRhoPhi, abs-sum of the r terms, abs-sum of the i terms)."""
+    pr, pi, r, i = (np.asarray(a, np.float64) for a in (phiR, phiI, dR, dI))
+    return pr * r + pi * i, pr * i - pi * r, np.abs(pr * r) + np.abs(pi * i), np.abs(pr * i) + np.abs(pi * r)
+
+
+def mrifhd_fh(x, y, z, kx, ky, kz, rRhoPhi, iRhoPhi, rF_in=None, iF_in=None):
+    """ComputeFH over one k chunk (accumulating into rF_in / iF_in when given):
+
+        arg = 2*pi*(kx[k]*x[v] + ky[k]*y[v] + kz[k]*z[v])
+        rFhD[v] += sum_k rRhoPhi[k]*cos(arg) - iRhoPhi[k]*sin(arg)
+        iFhD[v] += sum_k iRhoPhi[k]*cos(arg) + rRhoPhi[k]*sin(arg)
+
+    fp64 with 2*pi = Parboil's fp32 PIx2 (as mri-q).  Returns (rFhD, iFhD, Sr, Si), S = abs-sums."""
+    x, y, z = (np.asarray(a, np.float64) for a in (x, y, z))
+    nv = x.size
+    rF = np.zeros(nv) if rF_in is None else np.asarray(rF_in, np.float64).copy()
+    iF = np.zeros(nv) if iF_in is None else np.asarray(iF_in, np.float64).copy()
+    Sr, Si = np.abs(rF).copy(), np.abs(iF).copy()
+    kx, ky, kz, rr, ri = (np.asarray(a, np.float64) for a in (kx, ky, kz, rRhoPhi, iRhoPhi))
+    step = 256
+    for k0 in range(0, kx.size, step):
+        sl = slice(k0, k0 + step)
+        arg = TWO_PI_F32 * (np.outer(x, kx[sl]) + np.outer(y, ky[sl]) + np.outer(z, kz[sl]))
+        c, s_ = np.cos(arg), np.sin(arg)
+        t1, t2 = c * rr[None, sl], s_ * ri[None, sl]      # rF terms
+        t3, t4 = c * ri[None, sl], s_ * rr[None, sl]      # iF terms
+        rF += (t1 - t2).sum(axis=1)
+        iF += (t3 + t4).sum(axis=1)
+        Sr += (np.abs(t1) + np.abs(t2)).sum(axis=1)
+        Si += (np.abs(t3) + np.abs(t4)).sum(axis=1)
+    return rF, iF, Sr, Si
+
+
+# ----------------------------------------------------------------------------- NEXT-3 cp
+def cp(atoms, nx, ny, h, z, V_in=None):
+    """Direct Coulomb summation on one lattice slice (Parboil cp, Table II; not
+    defined in the paper, DESIGN.md §2 reading 14), accumulating into V_in when given:
+
+        V[j, i] += sum_a q_a / sqrt((i*h - x_a)^2 + (j*h - y_a)^2 + (z - z_a)^2)
+
+    lattice point (i, j) at (i*h, j*h, z), flat index j*nx + i.  Returns (V, abs-sum)."""
+    at = np.asarray(atoms, np.float64)
+    px = np.arange(nx, dtype=np.float64) * h
+    py = np.arange(ny, dtype=np.float64) * h
+    V = np.zeros(ny * nx) if V_in is None else np.asarray(V_in, np.float64).ravel().copy()
+    S = np.abs(V).copy()
+    gx, gy = np.meshgrid(px, py)                 # [ny, nx]
+    gx, gy = gx.ravel(), gy.ravel()
+    for a in range(at.shape[0]):
+        ax, ay, az, q = at[a]
+        e = q / np.sqrt((gx - ax) ** 2 + (gy - ay) ** 2 + (z - az) ** 2)
+        V += e
+        S += np.abs(e)
+    return V, S
+
+
 # ----------------------------------------------------------------------------- c6 cutcp
 CUTCP_CUTOFF = 12.0
 CUTCP_EXCL = 1.0

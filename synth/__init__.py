@@ -170,6 +170,36 @@ def mriq_inputs(N: int, numK: int, seed: int):
                 kx=kx, ky=ky, kz=kz, phiR=phiR, phiI=phiI)
 
 
+def mrifhd_inputs(N: int, numK: int, seed: int):
+    """mri-q's voxel grid and k-space trajectory plus the data samples dR, dI ~ U[-1,1)."""
+    d = mriq_inputs(N, numK, seed)
+    g = rng(seed + 7919)
+    d["dR"] = g.uniform(-1, 1, size=numK).astype(np.float32)
+    d["dI"] = g.uniform(-1, 1, size=numK).astype(np.float32)
+    return d
+
+
+def cp_inputs(natoms: int, nx: int, ny: int, h: float, seed: int, z: float | None = None):
+    """Parboil cp-like: natoms atoms U[0, L)^3 over the lattice box L = max(nx, ny)*h (z range
+    the same), charges U[-1, 1); the slice height z defaults to L/2.  Atoms within 1e-3 of a
+    lattice point of the slice are re-drawn (the potential there would be a near-singularity;
+    only coordinates are compared).  Returns (atoms float32 [natoms, 4], z)."""
+    g = rng(seed)
+    L = max(nx, ny) * h
+    z = L / 2 if z is None else z
+    at = np.empty((natoms, 4), np.float32)
+    for a in range(natoms):
+        while True:
+            p = g.uniform(0, L, size=3)
+            far_x = abs(p[0] / h - round(p[0] / h)) * h > 1e-3
+            far_y = abs(p[1] / h - round(p[1] / h)) * h > 1e-3
+            if abs(p[2] - z) > 1e-3 or far_x or far_y:
+                break
+        at[a, :3] = p
+        at[a, 3] = g.uniform(-1, 1)
+    return at, float(np.float32(z))
+
+
 def cutcp_inputs(L: float, seed: int, h: float = 0.5, density: float = 0.1, excl: float = 1.0):
     """Water-like box of side L (Angstrom): round(density*L^3) atoms U[0,L)^3, charges cycle
     (-0.834, +0.417, +0.417); lattice origin 0, ceil(L/h) points per axis, spacing h.

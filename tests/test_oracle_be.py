@@ -349,3 +349,78 @@ def test_cutcp_bins_partition_atoms_in_index_order():
         seen += idx
         assert np.all(bins[b, count[b]:, 3] == 0)
     assert sorted(seen) == list(range(at.shape[0]))
+
+
+# ------------------------------------------------------------------ NEXT-3 mri-fhd (reading 14)
+def test_mrifhd_rhophi_is_conj_phi_times_d():
+    # RhoPhi = conj(phi) * d as a complex product (an independent formulation)
+    g = np.random.default_rng(3)
+    pr, pi, dr, di = (g.uniform(-1, 1, 50) for _ in range(4))
+    rr, ri, sr, si = be.mrifhd_rhophi(pr, pi, dr, di)
+    ref = np.conj(pr + 1j * pi) * (dr + 1j * di)
+    assert np.allclose(rr, ref.real, rtol=0, atol=1e-15) and np.allclose(ri, ref.imag, rtol=0, atol=1e-15)
+    assert np.all(sr >= np.abs(rr)) and np.all(si >= np.abs(ri))
+
+
+def test_mrifhd_fh_complex_exponential_closed_form():
+    # rF + i iF = sum_k RhoPhi_k exp(i arg_k)  (complex arithmetic, not the real expansion)
+    d = synth.mrifhd_inputs(4, 97, 5)
+    rr, ri, _, _ = be.mrifhd_rhophi(d["phiR"], d["phiI"], d["dR"], d["dI"])
+    rF, iF, Sr, Si = be.mrifhd_fh(d["x"], d["y"], d["z"], d["kx"], d["ky"], d["kz"], rr, ri)
+    f64 = {k: v.astype(np.float64) for k, v in d.items()}
+    arg = be.TWO_PI_F32 * (np.outer(f64["x"], f64["kx"]) + np.outer(f64["y"], f64["ky"]) + np.outer(f64["z"], f64["kz"]))
+    ref = (np.exp(1j * arg) * (rr + 1j * ri)[None, :]).sum(axis=1)
+    assert np.max(np.abs(rF - ref.real) / Sr) < 1e-12 and np.max(np.abs(iF - ref.imag) / Si) < 1e-12
+
+
+def test_mrifhd_origin_voxel_and_real_rhophi_reduces_to_mriq():
+    g = np.random.default_rng(9)
+    kx, ky, kz = (g.uniform(-8, 8, 40) for _ in range(3))
+    rr, ri = g.uniform(-1, 1, 40), g.uniform(-1, 1, 40)
+    zero = np.zeros(1)
+    rF, iF, _, _ = be.mrifhd_fh(zero, zero, zero, kx, ky, kz, rr, ri)     # arg = 0: sums of RhoPhi
+    assert abs(rF[0] - rr.sum()) < 1e-12 and abs(iF[0] - ri.sum()) < 1e-12
+    # iRhoPhi = 0: (rFhD, iFhD) is mri-q's (Qr, Qi) with phiMag = rRhoPhi (mri-q is pinned above)
+    d = synth.mriq_inputs(4, 40, 2)
+    rF, iF, _, _ = be.mrifhd_fh(d["x"], d["y"], d["z"], kx, ky, kz, rr, np.zeros(40))
+    qr, qi, _, _ = be.mriq_q(d["x"], d["y"], d["z"], kx, ky, kz, rr)
+    assert np.allclose(rF, qr, rtol=0, atol=1e-12) and np.allclose(iF, qi, rtol=0, atol=1e-12)
+
+
+def test_mrifhd_chunks_accumulate():
+    d = synth.mrifhd_inputs(4, 64, 1)
+    rr, ri, _, _ = be.mrifhd_rhophi(d["phiR"], d["phiI"], d["dR"], d["dI"])
+    args = (d["x"], d["y"], d["z"])
+    full = be.mrifhd_fh(*args, d["kx"], d["ky"], d["kz"], rr, ri)
+    a = be.mrifhd_fh(*args, d["kx"][:30], d["ky"][:30], d["kz"][:30], rr[:30], ri[:30])
+    b = be.mrifhd_fh(*args, d["kx"][30:], d["ky"][30:], d["kz"][30:], rr[30:], ri[30:], a[0], a[1])
+    assert np.allclose(b[0], full[0], rtol=0, atol=1e-12) and np.allclose(b[1], full[1], rtol=0, atol=1e-12)
+
+
+# ------------------------------------------------------------------ NEXT-3 cp (reading 14)
+def test_cp_single_atom_closed_form():
+    # q = 2 at (0, 0, z + 1), h = 1: V(0,0) = 2/1, V(3,4) = 2/sqrt(9 + 16 + 1)
+    z = 5.0
+    V, S = be.cp(np.array([[0.0, 0.0, z + 1.0, 2.0]]), 6, 6, 1.0, z)
+    assert V[0] == 2.0
+    assert abs(V[4 * 6 + 3] - 2.0 / math.sqrt(26.0)) < 1e-15
+    assert np.array_equal(np.abs(V), S)
+
+
+def test_cp_bruteforce_loops_linearity_accumulate():
+    at, z = synth.cp_inputs(13, 5, 4, 0.7, seed=3)
+    V, S = be.cp(at, 5, 4, 0.7, z)
+    for j in range(4):
+        for i in range(5):
+            e = 0.0
+            for a in at.astype(np.float64):
+                e += a[3] / math.sqrt((i * 0.7 - a[0]) ** 2 + (j * 0.7 - a[1]) ** 2 + (z - a[2]) ** 2)
+            assert abs(V[j * 5 + i] - e) <= 1e-12 * S[j * 5 + i]
+    # linearity in the charges and accumulation over atom chunks
+    at2 = at.copy()
+    at2[:, 3] *= -3.0
+    V2, _ = be.cp(at2, 5, 4, 0.7, z)
+    assert np.allclose(V2, -3.0 * V, rtol=1e-12, atol=0)
+    Va, _ = be.cp(at[:6], 5, 4, 0.7, z)
+    Vb, _ = be.cp(at[6:], 5, 4, 0.7, z, V_in=Va)
+    assert np.allclose(Vb, V, rtol=1e-12, atol=0)
