@@ -417,7 +417,7 @@ def test_cp_bruteforce_loops_linearity_accumulate():
                 e += a[3] / math.sqrt((i * 0.7 - a[0]) ** 2 + (j * 0.7 - a[1]) ** 2 + (z - a[2]) ** 2)
             assert abs(V[j * 5 + i] - e) <= 1e-12 * S[j * 5 + i]
     # linearity in the charges and accumulation over atom chunks
-    at2 = at.copy()
+    at2 = at.astype(np.float64)
     at2[:, 3] *= -3.0
     V2, _ = be.cp(at2, 5, 4, 0.7, z)
     assert np.allclose(V2, -3.0 * V, rtol=1e-12, atol=0)
