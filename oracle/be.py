@@ -405,3 +405,63 @@ def fma_burn(n_threads, iters, a=0.5, b_scale=0.125):
         an = a ** iters
         out += an * x + bj * (1.0 - an) / (1.0 - a)
     return out
+
+
+# ----------------------------------------------------------------------------- NEXT-3 fft
+def fft(x):
+    """Batched forward complex DFT (Parboil fft, Table II; the GEMM-fft pair of Fig. 10
+    P:1417-1419; not defined in the paper, DESIGN.md §2 reading 15), written out as the definition:
+
+        X[b, k] = sum_j x[b, j] * exp(-2 pi i (j k mod n) / n),   0 <= j, k < n
+
+    x: complex [batch, n].  fp64 (complex128) with the twiddle of each (j k mod n) evaluated by
+    numpy's exp.  Returns (X, S) with S[b, k] = sum_j |x[b, j]| (every term has modulus |x[b, j]|;
+    the abs-sum of metrics.max_rel_err for both the real and the imaginary part)."""
+    x = np.asarray(x, np.complex128)
+    n = x.shape[-1]
+    jk = np.mod(np.outer(np.arange(n), np.arange(n)), n)
+    W = np.exp(-2j * np.pi * jk / n)
+    X = x @ W
+    S = np.repeat(np.abs(x).sum(axis=-1, keepdims=True), n, axis=-1)
+    return X, S
+
+
+# ----------------------------------------------------------------------------- NEXT-3 tpacf
+def tpacf_dot_f32(a, b):
+    """The pair's cosine as the kernel computes it, in fp32 with every product and sum rounded
+    (no FMA): ((ax*bx + ay*by) + az*bz).  Integer counts are decided from this value, so both
+    sides take the decision in the same precision (DESIGN.md §2 reading 16)."""
+    a = np.asarray(a, np.float32)
+    b = np.asarray(b, np.float32)
+    return ((a[..., 0] * b[..., 0]) + (a[..., 1] * b[..., 1])) + (a[..., 2] * b[..., 2])
+
+
+def tpacf_bin(dot, edges):
+    """bin(dot) = #{k : dot < edges[k]} for the strictly decreasing fp32 cosines of increasing
+    angular bin edges: 0 = closer than edges[0], len(edges) = wider than the last edge."""
+    dot = np.asarray(dot, np.float32)
+    e = np.asarray(edges, np.float32)
+    return (dot[..., None] < e).sum(axis=-1)
+
+
+def tpacf(A, B, edges, self_pairs):
+    """Two-point angular correlation histogram (Parboil tpacf, Table II; reading 16):
+
+        count[b] = #{pairs (i, j) : bin(dot_f32(A[i], B[j])) == b},  b in [0, len(edges)]
+
+    over all pairs i, j (cross correlation, DR) or over i < j with B = A (self correlation, DD /
+    RR when self_pairs).  A, B: unit vectors float32 [n, 3].  Returns int64 [len(edges) + 1]."""
+    A = np.asarray(A, np.float32)
+    B = np.asarray(B, np.float32)
+    nb = len(edges) + 1
+    cnt = np.zeros(nb, np.int64)
+    step = 256
+    for i0 in range(0, A.shape[0], step):
+        a = A[i0:i0 + step]
+        bins = tpacf_bin(tpacf_dot_f32(a[:, None, :], B[None, :, :]), edges)
+        if self_pairs:
+            ii = np.arange(i0, i0 + a.shape[0])[:, None]
+            jj = np.arange(B.shape[0])[None, :]
+            bins = bins[jj > ii]
+        cnt += np.bincount(bins.ravel(), minlength=nb)
+    return cnt

@@ -340,3 +340,59 @@ def bfs_inputs(V: int, seed: int, variant: str = "random"):
     np.add.at(row_ptr, s + 1, 1)
     row_ptr = np.cumsum(row_ptr)
     return row_ptr.astype(np.int32), d.astype(np.int32)
+
+
+# --------------------------------------------------------------------------- NEXT-3 fft
+def fft_inputs(batch: int, n: int, seed: int, variant: str = "uniform"):
+    """Complex fp32 signals [batch, n, 2] (re, im interleaved), Parboil-fft-like batches of 1-D
+    transforms.  'uniform': re, im ~ U[-1,1); 'impulse': x[b, b % n] = 1; 'tone': x[b, j] =
+    exp(2 pi i m j / n) with m = b % n (rounded to fp32)."""
+    g = rng(seed)
+    if variant == "uniform":
+        x = g.uniform(-1, 1, size=(batch, n, 2))
+    elif variant == "impulse":
+        x = np.zeros((batch, n, 2))
+        x[np.arange(batch), np.arange(batch) % n, 0] = 1.0
+    elif variant == "tone":
+        m = (np.arange(batch) % n)[:, None]
+        ph = 2 * np.pi * np.mod(m * np.arange(n)[None, :], n) / n
+        x = np.stack([np.cos(ph), np.sin(ph)], axis=-1)
+    else:
+        raise ValueError(variant)
+    return np.ascontiguousarray(x.astype(np.float32))
+
+
+# --------------------------------------------------------------------------- NEXT-3 tpacf
+def tpacf_edges(bins_per_dec: int = 5, min_arcmin: float = 1.0, max_arcmin: float = 10000.0):
+    """Parboil tpacf's bin boundaries as fp32 cosines, strictly decreasing: the angles
+    10^(log10(min) + k / bins_per_dec) arcmin, k = 0 .. decades * bins_per_dec (21 edges ->
+    22 counters with the two open ends)."""
+    nb = int(round(math.log10(max_arcmin / min_arcmin) * bins_per_dec))
+    ang = 10.0 ** (math.log10(min_arcmin) + np.arange(nb + 1) / bins_per_dec) / 60.0 * math.pi / 180.0
+    e = np.cos(ang).astype(np.float32)
+    assert np.all(np.diff(e) < 0)
+    return e
+
+
+def tpacf_inputs(n: int, seed: int, variant: str = "clustered"):
+    """Unit vectors float32 [n, 3] (a sky catalogue as Cartesian points, Parboil tpacf's input
+    after its ra/dec conversion).  'clustered': 60 % of the points in 64 Gaussian clumps of
+    0.5-5 degrees on the sphere, 40 % uniform (galaxy-catalogue-like: every angular scale of the
+    bins is populated); 'uniform'.  Normalised in fp64, then rounded to fp32."""
+    g = rng(seed)
+    def sphere(m):
+        v = g.normal(size=(m, 3))
+        return v / np.linalg.norm(v, axis=1, keepdims=True)
+    if variant == "uniform":
+        p = sphere(n)
+    elif variant == "clustered":
+        nc = int(0.6 * n)
+        centres = sphere(64)
+        which = g.integers(0, 64, size=nc)
+        sig = g.uniform(0.5, 5.0, size=64)[which] * math.pi / 180.0
+        p = np.concatenate([centres[which] + g.normal(size=(nc, 3)) * sig[:, None], sphere(n - nc)])
+        p = p[g.permutation(n)]
+        p /= np.linalg.norm(p, axis=1, keepdims=True)
+    else:
+        raise ValueError(variant)
+    return np.ascontiguousarray(p.astype(np.float32))

@@ -1,5 +1,6 @@
 """Pins for oracle/be.py (c3-c10): closed forms, invariants, special cases and brute force on
 tiny inputs, chosen so a dropped term / wrong sign / wrong index fails one of them."""
+import cmath
 import math
 
 import numpy as np
@@ -424,3 +425,89 @@ def test_cp_bruteforce_loops_linearity_accumulate():
     Va, _ = be.cp(at[:6], 5, 4, 0.7, z)
     Vb, _ = be.cp(at[6:], 5, 4, 0.7, z, V_in=Va)
     assert np.allclose(Vb, V, rtol=1e-12, atol=0)
+
+
+# ------------------------------------------------------------------ NEXT-3 fft (reading 15)
+def test_fft_matches_library_fft():
+    # second opinion: numpy's FFT (a different algorithm) on a ragged batch of several lengths
+    for n in (2, 8, 64, 256):
+        x = synth.fft_inputs(5, n, seed=n)
+        xc = x[..., 0].astype(np.float64) + 1j * x[..., 1]
+        X, S = be.fft(xc)
+        assert np.max(np.abs(X - np.fft.fft(xc, axis=-1)) / S) < 1e-13
+
+
+def test_fft_bruteforce_loops():
+    x = synth.fft_inputs(2, 8, seed=3)
+    xc = x[..., 0].astype(np.float64) + 1j * x[..., 1]
+    X, _ = be.fft(xc)
+    for b in range(2):
+        for k in range(8):
+            s = sum(complex(xc[b, j]) * cmath.exp(-2j * math.pi * j * k / 8) for j in range(8))
+            assert abs(X[b, k] - s) < 1e-13
+
+
+def test_fft_closed_forms():
+    n = 64
+    # impulse at m -> X[k] = exp(-2 pi i m k / n); tone m -> n delta_{k, m}; constant -> n c delta_k0
+    imp = synth.fft_inputs(n, n, 0, "impulse")
+    X, _ = be.fft(imp[..., 0] + 1j * imp[..., 1])
+    m, k = np.meshgrid(np.arange(n), np.arange(n), indexing="ij")
+    assert np.max(np.abs(X - np.exp(-2j * np.pi * m * k / n))) < 1e-13
+    tone = synth.fft_inputs(n, n, 0, "tone").astype(np.float64)
+    X, _ = be.fft(tone[..., 0] + 1j * tone[..., 1])
+    assert np.max(np.abs(X - n * np.eye(n))) < 1e-4            # the tone itself is fp32-rounded
+    X, S = be.fft(np.full((1, n), 0.25 - 0.5j))
+    assert abs(X[0, 0] - n * (0.25 - 0.5j)) < 1e-13 and np.max(np.abs(X[0, 1:])) < 1e-13
+    assert np.allclose(S, n * abs(0.25 - 0.5j))
+
+
+def test_fft_parseval_linearity_shift():
+    n = 128
+    x = synth.fft_inputs(3, n, seed=11)
+    xc = x[..., 0].astype(np.float64) + 1j * x[..., 1]
+    X, _ = be.fft(xc)
+    assert np.allclose((np.abs(X) ** 2).sum(-1), n * (np.abs(xc) ** 2).sum(-1), rtol=1e-12)
+    Y, _ = be.fft(2.5 * xc + 1j * xc[::-1])
+    assert np.allclose(Y, 2.5 * X + 1j * X[::-1], rtol=0, atol=1e-11)
+    Z, _ = be.fft(np.roll(xc, 3, axis=-1))                      # x[j - 3] -> X[k] exp(-2 pi i 3 k / n)
+    assert np.allclose(Z, X * np.exp(-2j * np.pi * 3 * np.arange(n) / n), rtol=0, atol=1e-11)
+
+
+# ------------------------------------------------------------------ NEXT-3 tpacf (reading 16)
+def test_tpacf_bruteforce_loops():
+    e = synth.tpacf_edges()
+    A = synth.tpacf_inputs(40, 1)
+    B = synth.tpacf_inputs(23, 2)
+    f = np.float32
+    for self_pairs, X, Y in ((True, A, A), (False, A, B)):
+        cnt = [0] * (len(e) + 1)
+        for i in range(X.shape[0]):
+            for j in range(Y.shape[0]):
+                if self_pairs and j <= i:
+                    continue
+                d = f(f(f(X[i, 0]) * f(Y[j, 0])) + f(f(X[i, 1]) * f(Y[j, 1])))
+                d = f(d + f(f(X[i, 2]) * f(Y[j, 2])))
+                b = 0
+                for k in range(len(e)):
+                    if d < e[k]:
+                        b += 1
+                cnt[b] += 1
+        assert list(be.tpacf(X, Y, e, self_pairs)) == cnt
+
+
+def test_tpacf_counts_and_exact_geometry():
+    e = synth.tpacf_edges()
+    nb = len(e) + 1
+    A = synth.tpacf_inputs(700, 5)
+    B = synth.tpacf_inputs(300, 6, "uniform")
+    assert be.tpacf(A, A, e, True).sum() == 700 * 699 // 2
+    assert be.tpacf(A, B, e, False).sum() == 700 * 300
+    # cross is symmetric; cross(A, A) = 2 self(A) + the i == j pairs
+    assert np.array_equal(be.tpacf(A, B, e, False), be.tpacf(B, A, e, False))
+    diag = np.bincount(be.tpacf_bin(be.tpacf_dot_f32(A, A), e), minlength=nb)
+    assert np.array_equal(be.tpacf(A, A, e, False), 2 * be.tpacf(A, A, e, True) + diag)
+    # axis points: identical -> dot 1 (bin 0), orthogonal -> dot 0, antipodal -> dot -1 (last bin)
+    ax = np.array([[1, 0, 0], [0, 1, 0], [-1, 0, 0]], np.float32)
+    c = be.tpacf(ax[:1], ax, e, False)
+    assert c[0] == 1 and c[nb - 1] == 1 and c[int((e > 0).sum())] == 1
