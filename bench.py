@@ -627,6 +627,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-extra", action="store_true", help="skip the ResNet-50 b1 (configs[1]) managed side run")
     ap.add_argument("--simulate", action="store_true", help="CPU-only: manager on its simulated GPU (gloo)")
+    ap.add_argument("--overlap", type=int, default=None,
+                    help="programmatic dependent launch mode (tacker_set_launch_overlap: 0, 1, 2)")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args, int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")))
@@ -635,6 +637,9 @@ def main():
     if args.simulate:
         run_simulated(args, ws, rank)
     else:
+        if args.overlap is not None:
+            from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
+            tk.tacker_set_launch_overlap(args.overlap)
         run_tacker(args, ws, rank, local)
     if ws > 1:
         import torch.distributed as dist

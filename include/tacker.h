@@ -125,13 +125,44 @@ typedef enum {
   TACKER_BE_JDS_SCAN = 16,    /* prefix over blocks per length, start offsets, jds_ptr; 1 block */
   TACKER_BE_JDS_PERM = 17,    /* perm / row_len placement; block = 1024 rows */
   TACKER_BE_JDS_FILL = 18,    /* column / value scatter, diagonal-major; block = 128 JDS rows */
-  TACKER_BE_KIND_COUNT = 19
+  /* NEXT-3: the remaining Parboil BE apps of Table II */
+  TACKER_BE_MRIFHD_RHOPHI = 19, /* mri-fhd ComputeRhoPhi: rho*phi = conj(phi) d; block = 512 k      */
+  TACKER_BE_MRIFHD_FH = 20,   /* mri-fhd ComputeFH: F^H d over one k chunk; block = 32 voxels x 4 k-lanes */
+  TACKER_BE_CP = 21,          /* cp direct Coulomb summation on one lattice slice; block = 128x4 points */
+  TACKER_BE_FFT_TWIDDLE = 22, /* fft plan: twiddle table w[m] = exp(-2 pi i m / n); block = 128 entries */
+  TACKER_BE_FFT = 23,         /* batched forward complex DFT, length n <= 2048; block = 1 transform */
+  TACKER_BE_TPACF = 24,       /* angular correlation histogram; block = 128 points of a      */
+  TACKER_BE_KIND_COUNT = 25
 } tacker_be_kind;
 
 typedef struct { int32_t M, N, K; float alpha, beta; const float *A, *B; float *C; } tacker_be_sgemm;
 typedef struct { int32_t nx, ny, nz; float c0, c1; const float *A0; float *Anext; } tacker_be_stencil;
 typedef struct { int32_t numK; const float *phiR, *phiI; float *phiMag; } tacker_be_mriq_phimag;
 typedef struct { int32_t numX, numK; const float *x, *y, *z, *kx, *ky, *kz, *phiMag; float *Qr, *Qi; } tacker_be_mriq_q;
+/* mri-fhd (Parboil; Table II, not defined in the paper: DESIGN.md §2 reading 14).
+ * RhoPhi: rRhoPhi[k] = phiR dR + phiI dI, iRhoPhi[k] = phiR dI - phiI dR (all fp32 [numK]).
+ * FH:     arg = 2pi (kx x + ky y + kz z);
+ *         rFhD[v] += sum_k rRhoPhi cos(arg) - iRhoPhi sin(arg),
+ *         iFhD[v] += sum_k iRhoPhi cos(arg) + rRhoPhi sin(arg)   (fp32 [numX], accumulated).
+ * Same thread mapping, k staging and fixed per-voxel order as TACKER_BE_MRIQ_Q. */
+typedef struct { int32_t numK; const float *phiR, *phiI, *dR, *dI; float *rRhoPhi, *iRhoPhi; } tacker_be_mrifhd_rhophi;
+typedef struct { int32_t numX, numK; const float *x, *y, *z, *kx, *ky, *kz, *rRhoPhi, *iRhoPhi; float *rFhD, *iFhD; } tacker_be_mrifhd_fh;
+/* cp (Parboil; Table II; reading 14): direct Coulomb summation on one lattice slice,
+ *   V[j*nx + i] += sum_a q_a * rsqrt((i h - x_a)^2 + (j h - y_a)^2 + (z - z_a)^2)
+ * atoms float4 (x, y, z, q) [natoms]; V fp32 [ny][nx] accumulated (one launch per atom chunk, as
+ * Parboil's constant-memory chunks).  An atom ON a lattice point gives inf (caller's concern). */
+typedef struct { int32_t natoms, nx, ny; float h, z; const float *atoms; float *V; } tacker_be_cp;
+/* fft (Parboil; Fig. 10's GEMM-fft pair P:1417-1419; reading 15): y[b, k] = sum_j x[b, j]
+ * exp(-2 pi i j k / n), b < batch, complex fp32 interleaved (re, im) [batch][n][2], out of place,
+ * x, y 16-byte aligned; n a power of two in [2, 2048].  twiddle [n][2] fp32 is written by
+ * TACKER_BE_FFT_TWIDDLE (w[m] = (cos, -sin)(2 pi m / n), accurate sincospi) and read by
+ * TACKER_BE_FFT (Stockham radix-4/2 in shared memory). */
+typedef struct { int32_t n, batch; float *twiddle; const float *x; float *y; } tacker_be_fft;
+/* tpacf (Parboil; reading 16): count[bin(a_i . b_j)] += 1 over all (i, j) (self_pairs = 0) or
+ * over i < j with b == a (self_pairs = 1); bin(d) = #{k : d < edges[k]}, edges strictly
+ * decreasing fp32 cosines, nedges <= 31; d = ((ax bx + ay by) + az bz) in fp32 without FMA;
+ * a, b unit vectors fp32 [n][3]; count u32 [nedges + 1], accumulated. */
+typedef struct { int32_t na, nb, nedges, self_pairs; const float *a, *b, *edges; uint32_t *count; } tacker_be_tpacf;
 /* cutcp: V[p] = sum_{a: d^2 < cutoff^2} q_a / d * (1 - d^2/cutoff^2)^2, V[p] = 0 if any atom has
  * d < excl.  Atoms come binned (TACKER_BE_CUTCP_BIN): bin side = 8*h, so one block (8x8x8
  * lattice points) is one bin and its atoms within the cutoff lie in the bins within
@@ -212,6 +243,11 @@ typedef struct {
     tacker_be_cutcp_bin cutcp_bin;
     tacker_be_copy copy;
     tacker_be_jds jds;
+    tacker_be_mrifhd_rhophi mrifhd_rhophi;
+    tacker_be_mrifhd_fh mrifhd_fh;
+    tacker_be_cp cp;
+    tacker_be_fft fft;
+    tacker_be_tpacf tpacf;
     uint8_t _pad[128];
   } p;
 } tacker_be_desc;
@@ -267,11 +303,13 @@ tacker_status tacker_fused_rebind(tacker_fused_t f, const tacker_lc_desc *lc, co
 tacker_status tacker_launch_fused(tacker_fused_t f, tacker_stream_t stream);
 tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_desc *be,
                                      tacker_stream_t stream);
-/* Programmatic dependent launch (default on): every launch of this library may begin its
+/* Programmatic dependent launch (default mode 2): every launch of this library may begin its
  * prologue (CTA scheduling, barrier / TMEM setup, TACKER_LC_B_CONST weight fetches) while the
  * previous kernel on the stream is still running; each kernel waits for its predecessor
  * (griddepcontrol.wait) before touching any other global memory, so stream order semantics are
- * unchanged.  0 disables it (plain stream serialization).  Process-wide. */
+ * unchanged.  0 disables it (plain stream serialization); 1 = every launch; 2 (default) = every
+ * launch except original BE kernels (their non-persistent grid is then distributed over an
+ * idle GPU instead of being parked behind the running kernel).  Process-wide.  EINVAL else. */
 tacker_status tacker_set_launch_overlap(int32_t enable);
 
 /* One fused launch of handle f whose BE part runs only the PTB slice [block_offset,

@@ -65,7 +65,7 @@ template <> struct BeBody<TACKER_BE_CUTCP> {
           const float dz = __fsub_rn(at.z, pz[m]);
           const float r2 = __fmaf_rn(dz, dz, dxy2);
           const float s = __fmaf_rn(-r2, inv_c2, 1.f);
-          const float e = __fmul_rn(__fmul_rn(__fmul_rn(at.w, rsqrtf(r2)), s), s);
+          const float e = __fmul_rn(__fmul_rn(__fmul_rn(at.w, rsqrt_ftz(r2)), s), s);
           acc[m] = r2 < c2 ? __fadd_rn(acc[m], e) : acc[m];
           ex[m] = ex[m] | (r2 < e2);
         }

@@ -478,7 +478,7 @@ struct alignas(64) BeOrigParams {
 };
 
 template <int BE_KIND>
-__global__ void __launch_bounds__(128) be_original_kernel(const __grid_constant__ BeOrigParams P) {
+__global__ void __launch_bounds__(128, be_orig_min_blocks(BE_KIND)) be_original_kernel(const __grid_constant__ BeOrigParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();
   griddep_wait();

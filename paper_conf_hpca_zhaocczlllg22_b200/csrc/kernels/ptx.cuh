@@ -10,6 +10,14 @@ namespace tk {
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+// MUFU reciprocal square root without rsqrtf's subnormal rescaling (FSETP + 2 predicated FMULs
+// per call): the cp / cutcp distances are >= 1e-3 A, so r^2 is never subnormal and the result
+// is the same MUFU.RSQ value.
+__device__ __forceinline__ float rsqrt_ftz(float x) {
+  float y;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 __device__ __forceinline__ uint32_t warp_id() { return threadIdx.x >> 5; }
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 

@@ -59,7 +59,8 @@ int sm_count() {
 const char *be_kind_name(int kind) {
   static const char *names[] = {"none",   "sgemm", "stencil", "mriq_phimag", "mriq_q",   "cutcp",
                                 "lbm",    "spmv",  "histo",   "bfs_expand",  "bfs_commit", "fma_burn",
-                                "im2col", "cutcp_bin", "copy", "jds_count", "jds_scan", "jds_perm", "jds_fill"};
+                                "im2col", "cutcp_bin", "copy", "jds_count", "jds_scan", "jds_perm", "jds_fill",
+                                "mrifhd_rhophi", "mrifhd_fh", "cp", "fft_twiddle", "fft", "tpacf"};
   return (kind >= 0 && kind < TACKER_BE_KIND_COUNT) ? names[kind] : "?";
 }
 
@@ -68,6 +69,9 @@ const char *be_kind_name(int kind) {
 using namespace tkrt;
 
 // ============================================================================ constants
+#ifndef TACKER_OVERLAP_DEFAULT
+#define TACKER_OVERLAP_DEFAULT 2
+#endif
 static constexpr int kSmemCap = 232448;      // max dynamic SMEM per CTA on sm_100 (227 KB)
 static constexpr int kTmemCols = 512;
 static constexpr int kMaxWarps = 32;
@@ -123,6 +127,47 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
     case TACKER_BE_MRIQ_Q:
       if (d.p.mriq_q.numX < 0 || d.p.mriq_q.numK < 0 || !d.p.mriq_q.Qr) return set_error("mriq_q: bad args"), TACKER_EINVAL;
       break;
+    case TACKER_BE_MRIFHD_RHOPHI: {
+      const auto &p = d.p.mrifhd_rhophi;
+      if (p.numK < 0 || (p.numK && (!p.phiR || !p.phiI || !p.dR || !p.dI || !p.rRhoPhi || !p.iRhoPhi)))
+        return set_error("mrifhd_rhophi: bad args"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_MRIFHD_FH: {
+      const auto &p = d.p.mrifhd_fh;
+      if (p.numX < 0 || p.numK < 0 ||
+          (p.numX && (!p.x || !p.y || !p.z || !p.rFhD || !p.iFhD)) ||
+          (p.numX && p.numK && (!p.kx || !p.ky || !p.kz || !p.rRhoPhi || !p.iRhoPhi)))
+        return set_error("mrifhd_fh: bad args"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_CP: {
+      const auto &p = d.p.cp;
+      if (p.natoms < 0 || p.nx < 0 || p.ny < 0 || !(p.h > 0) || (p.nx && p.ny && !p.V) || (p.natoms && !p.atoms))
+        return set_error("cp: bad args"), TACKER_EINVAL;
+      if (reinterpret_cast<uintptr_t>(p.atoms) & 15) return set_error("cp: atoms must be 16-byte aligned float4"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_FFT_TWIDDLE:
+    case TACKER_BE_FFT: {
+      const auto &p = d.p.fft;
+      if (p.n < 2 || p.n > BeBody<TACKER_BE_FFT>::kMaxN || (p.n & (p.n - 1)))
+        return set_error("fft: n must be a power of two in [2, %d]", BeBody<TACKER_BE_FFT>::kMaxN), TACKER_EUNSUPPORTED;
+      if (!p.twiddle || (d.kind == TACKER_BE_FFT && (p.batch < 0 || (p.batch && (!p.x || !p.y)))))
+        return set_error("fft: bad args"), TACKER_EINVAL;
+      if (d.kind == TACKER_BE_FFT && ((reinterpret_cast<uintptr_t>(p.x) | reinterpret_cast<uintptr_t>(p.y)) & 15))
+        return set_error("fft: x and y must be 16-byte aligned"), TACKER_EINVAL;
+      break;
+    }
+    case TACKER_BE_TPACF: {
+      const auto &p = d.p.tpacf;
+      if (p.na < 0 || p.nb < 0 || !p.count || !p.edges || (p.na && !p.a) || (p.nb && !p.b) ||
+          (p.self_pairs && (p.a != p.b || p.na != p.nb)))
+        return set_error("tpacf: bad args (self_pairs needs b == a)"), TACKER_EINVAL;
+      if (p.nedges < 1 || p.nedges > BeBody<TACKER_BE_TPACF>::kMaxEdges)
+        return set_error("tpacf: nedges must be in [1, %d]", BeBody<TACKER_BE_TPACF>::kMaxEdges), TACKER_EUNSUPPORTED;
+      break;
+    }
     case TACKER_BE_LBM:
       if (d.p.lbm.nx <= 0 || !d.p.lbm.src || !d.p.lbm.dst || !d.p.lbm.flags || d.p.lbm.src == d.p.lbm.dst)
         return set_error("lbm: bad args (src and dst must differ)"), TACKER_EINVAL;
@@ -414,6 +459,10 @@ static std::string be_key_of(const tacker_be_desc &d) {
     case TACKER_BE_SGEMM: snprintf(b, sizeof b, "be:sgemm:N%d:K%d", d.p.sgemm.N, d.p.sgemm.K); break;
     case TACKER_BE_STENCIL: snprintf(b, sizeof b, "be:stencil:nz%d", d.p.stencil.nz); break;
     case TACKER_BE_MRIQ_Q: snprintf(b, sizeof b, "be:mriq_q:K%d", d.p.mriq_q.numK); break;
+    case TACKER_BE_MRIFHD_FH: snprintf(b, sizeof b, "be:mrifhd_fh:K%d", d.p.mrifhd_fh.numK); break;
+    case TACKER_BE_CP: snprintf(b, sizeof b, "be:cp:A%d", d.p.cp.natoms); break;
+    case TACKER_BE_FFT: snprintf(b, sizeof b, "be:fft:n%d", d.p.fft.n); break;
+    case TACKER_BE_TPACF: snprintf(b, sizeof b, "be:tpacf:nb%d:s%d", d.p.tpacf.nb, d.p.tpacf.self_pairs); break;
     case TACKER_BE_FMA_BURN: snprintf(b, sizeof b, "be:fma_burn:it%d", d.p.fma_burn.iters); break;
     default: snprintf(b, sizeof b, "be:%s", be_kind_name(d.kind)); break;
   }
@@ -534,11 +583,13 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   return TACKER_OK;
 }
 
-static std::atomic<int> g_overlap{1};
+static std::atomic<int> g_overlap{TACKER_OVERLAP_DEFAULT};
 
-// cudaLaunchKernelEx with programmatic stream serialization (PDL) unless disabled
+// cudaLaunchKernelEx with programmatic stream serialization (PDL) unless disabled for this
+// launch class (be_original: a non-persistent BE grid)
 template <typename Param>
-static cudaError_t launch_ex(void (*fn)(Param), dim3 grid, dim3 block, int smem, cudaStream_t s, const Param &p) {
+static cudaError_t launch_ex(void (*fn)(Param), dim3 grid, dim3 block, int smem, cudaStream_t s, const Param &p,
+                             bool be_original = false) {
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
   cfg.blockDim = block;
@@ -548,7 +599,8 @@ static cudaError_t launch_ex(void (*fn)(Param), dim3 grid, dim3 block, int smem,
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = g_overlap.load(std::memory_order_relaxed) ? 1 : 0;
+  const int ov = g_overlap.load(std::memory_order_relaxed);
+  cfg.numAttrs = (ov == 1 || (ov == 2 && !be_original)) ? 1 : 0;
   return cudaLaunchKernelEx(&cfg, fn, p);
 }
 
@@ -584,7 +636,8 @@ extern "C" {
 const char *tacker_last_error(void) { return g_err.c_str(); }
 
 tacker_status tacker_set_launch_overlap(int32_t enable) {
-  g_overlap.store(enable ? 1 : 0);
+  if (enable < 0 || enable > 2) return set_error("launch overlap mode must be 0, 1 or 2"), TACKER_EINVAL;
+  g_overlap.store(enable);
   return TACKER_OK;
 }
 const char *tacker_version(void) { return "tacker-b200 0.1 (sm_100a)"; }
@@ -755,7 +808,7 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
     op.d = *be;
     if ((st = encode_be_tmap(*be, &op.tmap))) return st;
     if (blocks > 0x7fffffffLL) return set_error("too many blocks"), TACKER_EUNSUPPORTED;
-    cudaError_t e = launch_ex(fn, dim3((unsigned)blocks), dim3(128), smem, s, op);
+    cudaError_t e = launch_ex(fn, dim3((unsigned)blocks), dim3(128), smem, s, op, true);
     if (e != cudaSuccess) return cuda_fail("launch be_original_kernel", e);
   }
   return TACKER_OK;

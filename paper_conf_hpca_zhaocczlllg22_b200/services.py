@@ -14,6 +14,8 @@ from __future__ import annotations
 
 from dataclasses import dataclass, field
 
+import math
+
 import numpy as np
 import torch
 
@@ -155,6 +157,62 @@ def mriq_app(N=64, numK=2048, chunk=1024, seed=2022) -> BeAppSpec:
         ks.append(BeKernelSpec(f"mriq.q{c0 // chunk}", desc, flops=10.0 * nx * kn, mufu=2.0 * nx * kn,
                                bytes=20.0 * nx + 16.0 * kn, bound="mufu"))
     return BeAppSpec(f"mriq_{N}^3x{numK}", ks, [dd, phimag, Qr, Qi])
+
+
+def mrifhd_app(N=64, numK=2048, chunk=1024, seed=2022) -> BeAppSpec:
+    """Parboil mri-fhd (NEXT-3): ComputeRhoPhi then ComputeFH per k chunk (accumulating)."""
+    d = synth.mrifhd_inputs(N, numK, seed)
+    dd = {k: _dev(v) for k, v in d.items()}
+    rr, ri = torch.empty(numK, device="cuda"), torch.empty(numK, device="cuda")
+    Fr, Fi = torch.zeros(N ** 3, device="cuda"), torch.zeros(N ** 3, device="cuda")
+    ks = [BeKernelSpec("mrifhd.rhophi", tk.be_mrifhd_rhophi(dd["phiR"], dd["phiI"], dd["dR"], dd["dI"], rr, ri),
+                       flops=6 * numK, bytes=24 * numK)]
+    nx = N ** 3
+    for c0 in range(0, numK, chunk):
+        kn = min(chunk, numK - c0)
+        sl = slice(c0, c0 + kn)
+        desc = tk.be_mrifhd_fh(dd["x"], dd["y"], dd["z"], dd["kx"][sl], dd["ky"][sl], dd["kz"][sl], rr[sl], ri[sl],
+                               Fr, Fi)
+        ks.append(BeKernelSpec(f"mrifhd.fh{c0 // chunk}", desc, flops=14.0 * nx * kn, mufu=2.0 * nx * kn,
+                               bytes=20.0 * nx + 20.0 * kn, bound="mufu"))
+    return BeAppSpec(f"mrifhd_{N}^3x{numK}", ks, [dd, rr, ri, Fr, Fi])
+
+
+def cp_app(natoms=4000, nx=512, ny=512, h=0.1, seed=2022) -> BeAppSpec:
+    """Parboil cp (NEXT-3): one kernel = one chunk of natoms atoms summed into a 512x512 slice."""
+    at, z = synth.cp_inputs(natoms, nx, ny, h, seed)
+    dat = _dev(at)
+    V = torch.zeros(ny, nx, device="cuda")
+    pairs = float(natoms) * nx * ny
+    return BeAppSpec(f"cp_{nx}x{ny}x{natoms}", [BeKernelSpec("cp", tk.be_cp(dat, V, h, z), flops=6.0 * pairs,
+                                                             mufu=pairs, bytes=16.0 * natoms + 8.0 * nx * ny,
+                                                             bound="mufu")], [dat, V])
+
+
+def fft_app(batch=1 << 14, n=1024, seed=2022) -> BeAppSpec:
+    """Parboil fft (NEXT-3): the twiddle plan once, then forward transforms ping-ponging between
+    two buffers (one kernel = one batched transform of batch x n complex fp32)."""
+    x = _dev(synth.fft_inputs(batch, n, seed))
+    y = torch.empty_like(x)
+    tw = torch.empty(n, 2, device="cuda")
+    tk.tacker_launch_original(None, tk.be_fft_twiddle(tw, n))
+    flops = 5.0 * batch * n * math.log2(n)
+    ks = [BeKernelSpec("fft.even", tk.be_fft(x, y, tw), flops=flops, bytes=16.0 * batch * n),
+          BeKernelSpec("fft.odd", tk.be_fft(y, x, tw), flops=flops, bytes=16.0 * batch * n)]
+    return BeAppSpec(f"fft_{batch}x{n}", ks, [x, y, tw])
+
+
+def tpacf_app(n=16384, seed=2022) -> BeAppSpec:
+    """Parboil tpacf (NEXT-3): DD (self) and DR (cross) angular histograms of a clustered
+    catalogue against a uniform random one (one kernel = one correlation)."""
+    e = _dev(synth.tpacf_edges())
+    d = _dev(synth.tpacf_inputs(n, seed))
+    r = _dev(synth.tpacf_inputs(n, seed + 1, "uniform"))
+    dd = torch.zeros(e.numel() + 1, dtype=torch.int32, device="cuda")
+    dr = torch.zeros_like(dd)
+    ks = [BeKernelSpec("tpacf.dd", tk.be_tpacf(d, d, e, dd, self_pairs=True), bytes=12.0 * n, bound="alu"),
+          BeKernelSpec("tpacf.dr", tk.be_tpacf(d, r, e, dr), bytes=24.0 * n, bound="alu")]
+    return BeAppSpec(f"tpacf_{n}", ks, [e, d, r, dd, dr])
 
 
 def lbm_app(nx=120, ny=120, nz=150, seed=2022) -> BeAppSpec:

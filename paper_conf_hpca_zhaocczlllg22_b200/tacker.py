@@ -27,7 +27,7 @@ F32, F16 = 0, 1
 EPI_BIAS, EPI_RELU, EPI_RESIDUAL, LC_B_CONST, LC_NO_SPLIT = 1, 2, 4, 8, 16
 (BE_NONE, BE_SGEMM, BE_STENCIL, BE_MRIQ_PHIMAG, BE_MRIQ_Q, BE_CUTCP, BE_LBM, BE_SPMV_JDS, BE_HISTO,
  BE_BFS_EXPAND, BE_BFS_COMMIT, BE_FMA_BURN, BE_IM2COL, BE_CUTCP_BIN, BE_COPY, BE_JDS_COUNT, BE_JDS_SCAN,
- BE_JDS_PERM, BE_JDS_FILL) = range(19)
+ BE_JDS_PERM, BE_JDS_FILL, BE_MRIFHD_RHOPHI, BE_MRIFHD_FH, BE_CP, BE_FFT_TWIDDLE, BE_FFT, BE_TPACF) = range(25)
 POLICY_TACKER, POLICY_BAYMAX = 0, 1
 DEC_FUSED, DEC_ORIGINAL_LC, DEC_REORDER_BE, DEC_IDLE_BE, DEC_NOTHING = range(5)
 MAX_APPS = 64
@@ -136,11 +136,38 @@ class BeJds(C.Structure):
                 ("overflow", C.c_void_p)]
 
 
+class BeMrifhdRhophi(C.Structure):
+    _fields_ = [("numK", C.c_int32), ("phiR", C.c_void_p), ("phiI", C.c_void_p), ("dR", C.c_void_p),
+                ("dI", C.c_void_p), ("rRhoPhi", C.c_void_p), ("iRhoPhi", C.c_void_p)]
+
+
+class BeMrifhdFh(C.Structure):
+    _fields_ = [("numX", C.c_int32), ("numK", C.c_int32), ("x", C.c_void_p), ("y", C.c_void_p), ("z", C.c_void_p),
+                ("kx", C.c_void_p), ("ky", C.c_void_p), ("kz", C.c_void_p), ("rRhoPhi", C.c_void_p),
+                ("iRhoPhi", C.c_void_p), ("rFhD", C.c_void_p), ("iFhD", C.c_void_p)]
+
+
+class BeCp(C.Structure):
+    _fields_ = [("natoms", C.c_int32), ("nx", C.c_int32), ("ny", C.c_int32), ("h", C.c_float), ("z", C.c_float),
+                ("atoms", C.c_void_p), ("V", C.c_void_p)]
+
+
+class BeFft(C.Structure):
+    _fields_ = [("n", C.c_int32), ("batch", C.c_int32), ("twiddle", C.c_void_p), ("x", C.c_void_p), ("y", C.c_void_p)]
+
+
+class BeTpacf(C.Structure):
+    _fields_ = [("na", C.c_int32), ("nb", C.c_int32), ("nedges", C.c_int32), ("self_pairs", C.c_int32),
+                ("a", C.c_void_p), ("b", C.c_void_p), ("edges", C.c_void_p), ("count", C.c_void_p)]
+
+
 class _BeUnion(C.Union):
     _fields_ = [("sgemm", BeSgemm), ("stencil", BeStencil), ("mriq_phimag", BeMriqPhimag), ("mriq_q", BeMriqQ),
                 ("cutcp", BeCutcp), ("lbm", BeLbm), ("spmv", BeSpmv), ("histo", BeHisto),
                 ("bfs_expand", BeBfsExpand), ("bfs_commit", BeBfsCommit), ("fma_burn", BeFmaBurn),
                 ("im2col", BeIm2col), ("cutcp_bin", BeCutcpBin), ("copy", BeCopy), ("jds", BeJds),
+                ("mrifhd_rhophi", BeMrifhdRhophi), ("mrifhd_fh", BeMrifhdFh), ("cp", BeCp), ("fft", BeFft),
+                ("tpacf", BeTpacf),
                 ("_pad", C.c_uint8 * 128)]
 
 
@@ -322,6 +349,51 @@ def be_mriq_q(x, y, z, kx, ky, kz, phiMag, Qr, Qi, orig_blocks=0) -> BeDesc:
     d = BeDesc(kind=BE_MRIQ_Q, orig_blocks=orig_blocks)
     d.p.mriq_q = BeMriqQ(x.numel(), kx.numel(), _ptr(x), _ptr(y), _ptr(z), _ptr(kx), _ptr(ky), _ptr(kz),
                          _ptr(phiMag), _ptr(Qr), _ptr(Qi))
+    return d
+
+
+def be_mrifhd_rhophi(phiR, phiI, dR, dI, rRhoPhi, iRhoPhi, orig_blocks=0) -> BeDesc:
+    d = BeDesc(kind=BE_MRIFHD_RHOPHI, orig_blocks=orig_blocks)
+    d.p.mrifhd_rhophi = BeMrifhdRhophi(phiR.numel(), _ptr(phiR), _ptr(phiI), _ptr(dR), _ptr(dI), _ptr(rRhoPhi),
+                                       _ptr(iRhoPhi))
+    return d
+
+
+def be_mrifhd_fh(x, y, z, kx, ky, kz, rRhoPhi, iRhoPhi, rFhD, iFhD, orig_blocks=0) -> BeDesc:
+    d = BeDesc(kind=BE_MRIFHD_FH, orig_blocks=orig_blocks)
+    d.p.mrifhd_fh = BeMrifhdFh(x.numel(), kx.numel(), _ptr(x), _ptr(y), _ptr(z), _ptr(kx), _ptr(ky), _ptr(kz),
+                               _ptr(rRhoPhi), _ptr(iRhoPhi), _ptr(rFhD), _ptr(iFhD))
+    return d
+
+
+def be_cp(atoms, V, h, z, orig_blocks=0) -> BeDesc:
+    """atoms: float32 [natoms, 4] (x, y, z, q) device tensor; V: float32 [ny, nx] (accumulated)."""
+    ny, nx = V.shape
+    d = BeDesc(kind=BE_CP, orig_blocks=orig_blocks)
+    d.p.cp = BeCp(atoms.shape[0], nx, ny, h, z, _ptr(atoms), _ptr(V))
+    return d
+
+
+def be_fft_twiddle(twiddle, n, orig_blocks=0) -> BeDesc:
+    """twiddle: float32 [n, 2] device tensor (written)."""
+    d = BeDesc(kind=BE_FFT_TWIDDLE, orig_blocks=orig_blocks)
+    d.p.fft = BeFft(n, 0, _ptr(twiddle), None, None)
+    return d
+
+
+def be_fft(x, y, twiddle, orig_blocks=0) -> BeDesc:
+    """x, y: float32 [batch, n, 2] (complex interleaved); twiddle from be_fft_twiddle."""
+    batch, n = x.shape[0], x.shape[1]
+    d = BeDesc(kind=BE_FFT, orig_blocks=orig_blocks)
+    d.p.fft = BeFft(n, batch, _ptr(twiddle), _ptr(x), _ptr(y))
+    return d
+
+
+def be_tpacf(a, b, edges, count, self_pairs=False, orig_blocks=0) -> BeDesc:
+    """a, b: float32 [n, 3] unit vectors; edges float32 decreasing; count int32/uint32 [len(edges)+1]."""
+    d = BeDesc(kind=BE_TPACF, orig_blocks=orig_blocks)
+    d.p.tpacf = BeTpacf(a.shape[0], b.shape[0], edges.numel(), int(bool(self_pairs)), _ptr(a), _ptr(b), _ptr(edges),
+                        _ptr(count))
     return d
 
 
@@ -512,9 +584,10 @@ def tacker_launch_fused(f: Fused, stream=None):
     f.launch(stream)
 
 
-def tacker_set_launch_overlap(enable: bool):
-    """Programmatic dependent launch for every launch of the library (default on)."""
-    _chk(_lib.tacker_set_launch_overlap(1 if enable else 0))
+def tacker_set_launch_overlap(enable):
+    """Programmatic dependent launch: False/0 off, True/1 every launch, 2 (the library default)
+    every launch except original BE kernels."""
+    _chk(_lib.tacker_set_launch_overlap(int(enable)))
 
 
 def tacker_launch_fused_slice(f: Fused, block_offset: int, n_blocks: int, stream=None):

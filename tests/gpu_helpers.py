@@ -142,6 +142,89 @@ def be_case(kind, seed=0, size="small"):
             assert max_rel_err(g, ref, S) <= 1e-5
         return dict(desc=tk.be_cutcp(bins, count, V, nx, nx, nx, 0.5, depth), outs=[V], reset=lambda: V.zero_(),
                     check=check, keep=(datoms, bins, count, ovf))
+    if kind == tk.BE_MRIFHD_RHOPHI:
+        nk = 3000
+        d = synth.mrifhd_inputs(4, nk, seed)
+        ins = [t(d[k]) for k in ("phiR", "phiI", "dR", "dI")]
+        rr, ri = torch.zeros(nk, device=dev()), torch.zeros(nk, device=dev())
+        ref_r, ref_i, sr, si = obe.mrifhd_rhophi(d["phiR"], d["phiI"], d["dR"], d["dI"])
+
+        def check(o):
+            assert max_rel_err(o[0], ref_r, sr) <= 1e-5
+            assert max_rel_err(o[1], ref_i, si) <= 1e-5
+
+        def reset():
+            rr.zero_()
+            ri.zero_()
+        return dict(desc=tk.be_mrifhd_rhophi(*ins, rr, ri), outs=[rr, ri], reset=reset, check=check, keep=ins)
+    if kind == tk.BE_MRIFHD_FH:
+        N, nk = (12, 700) if size == "small" else (32, 1024)
+        d = synth.mrifhd_inputs(N, nk, seed)
+        # the FH inputs are fp32 RhoPhi values; both sides take the same fp32 array
+        r64, i64, _, _ = obe.mrifhd_rhophi(d["phiR"], d["phiI"], d["dR"], d["dI"])
+        rr, ri = r64.astype(np.float32), i64.astype(np.float32)
+        dd = {k: t(d[k]) for k in ("x", "y", "z", "kx", "ky", "kz")}
+        drr, dri = t(rr), t(ri)
+        Fr, Fi = torch.zeros(N ** 3, device=dev()), torch.zeros(N ** 3, device=dev())
+        ref_r, ref_i, sr, si = obe.mrifhd_fh(d["x"], d["y"], d["z"], d["kx"], d["ky"], d["kz"], rr, ri)
+
+        def check(o):
+            assert max_rel_err(o[0], ref_r, sr) <= 1e-5
+            assert max_rel_err(o[1], ref_i, si) <= 1e-5
+
+        def reset():
+            Fr.zero_()
+            Fi.zero_()
+        desc = tk.be_mrifhd_fh(dd["x"], dd["y"], dd["z"], dd["kx"], dd["ky"], dd["kz"], drr, dri, Fr, Fi)
+        return dict(desc=desc, outs=[Fr, Fi], reset=reset, check=check, keep=(dd, drr, dri))
+    if kind == tk.BE_CP:
+        # small: 2 x-tiles (ragged), 4 row blocks (ragged), 2 atom stages (ragged)
+        natoms, nx, ny, h = (700, 200, 13, 0.5) if size == "small" else (4000, 256, 256, 0.5)
+        at, z = synth.cp_inputs(natoms, nx, ny, h, seed)
+        dat = t(at)
+        V = torch.zeros(ny, nx, device=dev())
+        ref, S = obe.cp(at, nx, ny, h, z)
+
+        def check(o):
+            assert max_rel_err(o[0].ravel(), ref, S) <= 1e-5
+        return dict(desc=tk.be_cp(dat, V, h, z), outs=[V], reset=lambda: V.zero_(), check=check, keep=(dat,))
+    if kind in (tk.BE_FFT, tk.BE_FFT_TWIDDLE):
+        # small: a ragged batch at n = 256 (radix-4 only); "odd": n = 2048 (final radix-2 pass);
+        # large: the bench shape on sampled rows
+        batch, n = {"small": (37, 256), "odd": (5, 2048), "tiny": (3, 2), "large": (1 << 14, 1024)}[size]
+        x = synth.fft_inputs(batch, n, seed)
+        dx = t(x)
+        tw = torch.zeros(n, 2, device=dev())
+        y = torch.zeros_like(dx)
+        if kind == tk.BE_FFT_TWIDDLE:
+            # the twiddles are the DFT of impulses at 1: pinned through the oracle's DFT
+            X, _ = obe.fft(np.eye(n)[1:2])
+
+            def check(o):
+                assert np.max(np.abs(o[0][:, 0] - X[0].real)) <= 2e-7 and np.max(np.abs(o[0][:, 1] - X[0].imag)) <= 2e-7
+            return dict(desc=tk.be_fft_twiddle(tw, n), outs=[tw], reset=lambda: tw.zero_(), check=check, keep=())
+        tk.tacker_launch_original(None, tk.be_fft_twiddle(tw, n))
+        rows = np.arange(batch) if size != "large" else np.random.default_rng(seed).choice(batch, 64, replace=False)
+        X, S = obe.fft(x[rows, :, 0].astype(np.float64) + 1j * x[rows, :, 1])
+
+        def check(o):
+            g = o[0][rows]
+            assert max_rel_err(g[..., 0], X.real, S) <= 1e-5
+            assert max_rel_err(g[..., 1], X.imag, S) <= 1e-5
+        return dict(desc=tk.be_fft(dx, y, tw), outs=[y], reset=lambda: y.zero_(), check=check, keep=(dx, tw))
+    if kind == tk.BE_TPACF:
+        # small: self pairs over a ragged point count (3 b stages, 5 blocks); cross pairs below
+        n = 600 if size == "small" else 8192
+        e = synth.tpacf_edges()
+        A = synth.tpacf_inputs(n, seed)
+        dA, de = t(A), t(e)
+        cnt = torch.zeros(len(e) + 1, dtype=torch.int32, device=dev())
+        ref = obe.tpacf(A, A, e, True)
+
+        def check(o):
+            assert np.array_equal(o[0].view(np.uint32).astype(np.int64), ref)
+        return dict(desc=tk.be_tpacf(dA, dA, de, cnt, self_pairs=True), outs=[cnt], reset=lambda: cnt.zero_(),
+                    check=check, keep=(dA, de))
     if kind == tk.BE_FMA_BURN:
         n, iters = 128 * 300, 1000
         out = torch.zeros(n, device=dev())

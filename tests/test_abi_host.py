@@ -45,7 +45,8 @@ STRUCTS = {
     "tacker_be_lbm": "BeLbm", "tacker_be_spmv": "BeSpmv", "tacker_be_histo": "BeHisto",
     "tacker_be_bfs_expand": "BeBfsExpand", "tacker_be_bfs_commit": "BeBfsCommit",
     "tacker_be_fma_burn": "BeFmaBurn", "tacker_be_im2col": "BeIm2col", "tacker_be_cutcp_bin": "BeCutcpBin",
-    "tacker_be_copy": "BeCopy", "tacker_be_jds": "BeJds",
+    "tacker_be_copy": "BeCopy", "tacker_be_jds": "BeJds", "tacker_be_mrifhd_rhophi": "BeMrifhdRhophi",
+    "tacker_be_mrifhd_fh": "BeMrifhdFh", "tacker_be_cp": "BeCp", "tacker_be_fft": "BeFft", "tacker_be_tpacf": "BeTpacf",
     "tacker_fused_info_t": "FusedInfo",
     "tacker_lc_kernel": "LcKernel", "tacker_be_kernel": "BeKernel", "tacker_decision": "Decision",
     "tacker_manager_params": "ManagerParams", "tacker_manager_stats": "ManagerStats", "tacker_ratio": "Ratio",

@@ -15,7 +15,7 @@ def tk():
     return tacker
 
 
-@pytest.mark.parametrize("kind", ["BE_CUTCP", "BE_MRIQ_Q", "BE_STENCIL", "BE_LBM"])
+@pytest.mark.parametrize("kind", ["BE_CUTCP", "BE_MRIQ_Q", "BE_STENCIL", "BE_LBM", "BE_MRIFHD_FH", "BE_CP", "BE_FFT", "BE_TPACF"])
 def test_full_size_original_and_fused(tk, kind):
     import synth
     from tests.gpu_helpers import dev, t

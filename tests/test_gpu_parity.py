@@ -74,7 +74,7 @@ def test_lc_conv_vs_oracle(tk, cs):
 
 # ------------------------------------------------------------------ BE originals (c3-c10)
 BE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_MRIQ_PHIMAG", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN",
-            "BE_CUTCP"]
+            "BE_CUTCP", "BE_MRIFHD_RHOPHI", "BE_MRIFHD_FH", "BE_CP", "BE_FFT_TWIDDLE", "BE_FFT", "BE_TPACF"]
 
 
 @pytest.mark.parametrize("kind", BE_KINDS)
@@ -83,6 +83,41 @@ def test_be_original_vs_oracle(tk, kind):
     c["reset"]()
     tk.tacker_launch_original(None, c["desc"])
     c["check"]([host(o) for o in c["outs"]])
+
+
+@pytest.mark.parametrize("size", ["odd", "tiny"])
+def test_fft_lengths_vs_oracle(tk, size):
+    c = be_case(tk.BE_FFT, seed=4, size=size)
+    c["reset"]()
+    tk.tacker_launch_original(None, c["desc"])
+    c["check"]([host(o) for o in c["outs"]])
+
+
+@pytest.mark.parametrize("variant", ["impulse", "tone"])
+def test_fft_closed_form_inputs(tk, variant):
+    # impulse -> pure twiddle rows, tone -> n at one bin: vs the oracle's DFT of the same fp32 input
+    batch, n = 40, 512
+    x = synth.fft_inputs(batch, n, 0, variant)
+    tw = torch.zeros(n, 2, device=dev())
+    y = torch.zeros(batch, n, 2, device=dev())
+    tk.tacker_launch_original(None, tk.be_fft_twiddle(tw, n))
+    tk.tacker_launch_original(None, tk.be_fft(t(x), y, tw))
+    X, S = obe.fft(x[..., 0].astype(np.float64) + 1j * x[..., 1])
+    g = host(y)
+    assert max_rel_err(g[..., 0], X.real, S) <= 1e-5 and max_rel_err(g[..., 1], X.imag, S) <= 1e-5
+
+
+def test_tpacf_cross_and_axis_points(tk):
+    e = synth.tpacf_edges()
+    A = synth.tpacf_inputs(777, 3)
+    B = synth.tpacf_inputs(1500, 4, "uniform")
+    cnt = torch.zeros(len(e) + 1, dtype=torch.int32, device=dev())
+    tk.tacker_launch_original(None, tk.be_tpacf(t(A), t(B), t(e), cnt))
+    assert np.array_equal(host(cnt).astype(np.int64), obe.tpacf(A, B, e, False))
+    ax = np.array([[1, 0, 0], [0, 1, 0], [-1, 0, 0]], np.float32)
+    cnt.zero_()
+    tk.tacker_launch_original(None, tk.be_tpacf(t(ax[:1]), t(ax), t(e), cnt))
+    assert np.array_equal(host(cnt).astype(np.int64), obe.tpacf(ax[:1], ax, e, False))
 
 
 def test_bfs_levels_vs_oracle(tk):
@@ -108,7 +143,8 @@ def test_bfs_levels_vs_oracle(tk):
 
 
 # ------------------------------------------------------------------ fused (a1-a8)
-FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN", "BE_CUTCP"]
+FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "BE_HISTO", "BE_FMA_BURN", "BE_CUTCP",
+              "BE_MRIFHD_RHOPHI", "BE_MRIFHD_FH", "BE_CP", "BE_FFT", "BE_TPACF"]
 
 
 @pytest.mark.parametrize("kind", FUSE_KINDS)
@@ -290,9 +326,14 @@ def test_launch_overlap_keeps_stream_order(tk):
     try:
         ref = run()
     finally:
-        tk.tacker_set_launch_overlap(True)
+        tk.tacker_set_launch_overlap(2)
     for _ in range(3):
-        assert run() == ref
+        assert run() == ref                               # default: PDL except original BE launches
+    tk.tacker_set_launch_overlap(True)
+    try:
+        assert run() == ref                               # PDL on every launch
+    finally:
+        tk.tacker_set_launch_overlap(2)
 
 
 @pytest.mark.parametrize("M,N,K", [(128, 256, 4096), (130, 264, 4104), (49, 512, 4608)])

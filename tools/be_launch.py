@@ -31,10 +31,17 @@ def main():
         elif k == "sgemm":
             app = sv.sgemm_app(2048, 2048, 2048)
             d = app.kernels[0].desc
+        elif k == "mrifhd":
+            app = sv.mrifhd_app()
+            tk.tacker_launch_original(None, app.kernels[0].desc)
+            d = app.kernels[1].desc
+        elif k in ("cp", "fft", "tpacf", "lbm", "spmv", "histo", "cutcp"):
+            app = getattr(sv, k + "_app")()
+            d = app.kernels[-1].desc
         else:
             raise ValueError(k)
         keep.append(app)
-        f = tk.tacker_fuse(lc, d, 24 if k != "sgemm" else 16)
+        f = tk.tacker_fuse(lc, d, 24 if k not in ("sgemm", "fft", "tpacf") else 16)
         for _ in range(reps):
             tk.tacker_launch_original(None, d)
         for _ in range(reps):

@@ -49,7 +49,7 @@ def main():
         tk.tacker_set_launch_overlap(on)
         res["overlap" if on else "serial"] = {"query_ms": timed(lambda: query(svc), args.reps)}
     per = []
-    tk.tacker_set_launch_overlap(True)
+    tk.tacker_set_launch_overlap(2)
     for k in svc.kernels:
         f = (lambda k=k: tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd))
         us = timed(lambda: [f() for _ in range(8)], 5) * 1e3 / 8     # back to back
