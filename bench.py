@@ -385,7 +385,8 @@ def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "ta
     caller's window); returns {variant: result}."""
     out = {}
     kw = {"tacker": (tk.POLICY_TACKER, {}), "baymax": (tk.POLICY_BAYMAX, {}),
-          "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True})}
+          "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
+          "tacker_no_reverse": (tk.POLICY_TACKER, {"reverse_fusion": False})}
     for v in variants:
         pol, extra = kw[v]
         out[v] = q.run(pol, steps, load=LOAD, seed=seed, max_inflight=inflight, **extra)
@@ -482,6 +483,26 @@ def run_tacker(args, ws, rank, local):
     e2e = qi.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank, max_inflight=args.inflight)
     e2e_value = reduce_ranks(ws, e2e["be_kernels"], "sum") / (reduce_ranks(ws, e2e["elapsed_ms"], "max") / 1e3)
 
+    # ---- NEXT-2 reverse fusion side run: the same service with a tensor-core training BE app added
+    #      (Table II's DNN-training BE jobs); conv1's im2col (an LC CUDA-core kernel) may now fuse
+    #      with a BE GEMM.  The b32 calibration is reused; only the new pairs are fitted.
+    reverse = None
+    if not args.no_extra:
+        train = sv.gemm_train_app(4096, 4096, 4096, n=2, seed=seed + 3)
+        qr = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
+        qr.t_lc, qr.t_be, qr.pairs, qr.ws_of, qr.lr_be = q.t_lc, dict(q.t_be), dict(q.pairs), q.ws_of, q.lr_be
+        qr.service_ms = q.service_ms
+        qr.add_tc_apps([train])
+        rr = managed_runs(qr, tk, args.steps, 2000 + rank, args.inflight, ("tacker", "tacker_no_reverse", "baymax"))
+        reverse = {"workload": "resnet50_b%d LC + stencil / mri-q / train-GEMM (2 x 4096^3 fp16) BE queue" % args.batch,
+                   "train_gemm_ms": [qr.t_be[(2, j)] for j in range(len(train.kernels))],
+                   "im2col_ms": qr.t_lc[0]}
+        for v, r in rr.items():
+            reverse[v] = {k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms", "qos_met", "fused",
+                                            "reverse_fused", "reordered")}
+        for v in ("tacker", "tacker_no_reverse"):
+            reverse[v]["improvement_vs_baymax_eq10_normalised"] = rr[v]["be_norm_thpt"] / rr["baymax"]["be_norm_thpt"] - 1
+
     # ---- roofline of the dominant launch class of the timed run (class shares from the manager's
     #      sampled CUDA events on its stream)
     cms, cn = res["class_ms"], res["class_launches"]
@@ -549,6 +570,7 @@ def run_tacker(args, ws, rank, local):
         "tacker_slice": {"value": slc["be_kernels_per_s"], "be_norm_thpt": slc["be_norm_thpt"],
                          "lc_p99_ms": slc["lc_p99_ms"], "fused": slc["fused"],
                          "improvement_vs_baymax_eq10_normalised": slc["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0},
+        "reverse_fusion": reverse,
         "fused_pred_err_mean": res["fused_pred_err_mean"],
         "pair_pred_err_mean": statistics.mean(q.pair_err) if q.pair_err else None,
         "roofline": roof,

@@ -359,7 +359,9 @@ typedef struct {
   int32_t is_tc;             /* 1: tensor-core kernel (fusable as LC); 0: CUDA-core kernel */
   double t_pred_ms;          /* predicted standalone duration */
   tacker_lc_desc lc;         /* used when is_tc */
-  tacker_be_desc cd;         /* used when !is_tc (an LC CUDA-core kernel launched original) */
+  tacker_be_desc cd;         /* used when !is_tc (an LC CUDA-core kernel: launched original, or
+                                fused as the CUDA-core part with a BE tensor-core kernel) */
+  int32_t warp_split;        /* !is_tc: CUDA-core warps of a reverse-fused launch (0 = 16) */
 } tacker_lc_kernel;
 
 typedef struct {
@@ -378,6 +380,13 @@ typedef struct {
    * t_block_ms <= 0: never sliced. */
   int32_t n_blocks;
   double t_block_ms, t_floor_ms;
+  /* NEXT-2 reverse fusion ("LC and BE kernels are not limited to a specified type";
+   * DNN-training BE apps, Table II): is_tc = 1 makes this BE kernel the tensor-core
+   * GEMM / conv `tc` (is_cd must be 0).  The manager fuses it with an LC CUDA-core kernel under
+   * the same Eq. 8 (LC and BE solo times swap roles in the predictor: X_tc = this kernel,
+   * X_cd = the LC kernel); it is never sliced. */
+  int32_t is_tc;
+  tacker_lc_desc tc;
 } tacker_be_kernel;
 
 typedef struct {
@@ -388,13 +397,15 @@ typedef struct {
 typedef struct {
   int32_t action;            /* tacker_action */
   int32_t query, lc_index;   /* LC kernel decided (-1 if none) */
-  int32_t fused_app;         /* BE app fused with it (-1 if none) */
+  int32_t fused_app;         /* BE app fused with it (-1 if none); a reverse fusion (LC CUDA-core
+                                kernel + BE tensor-core kernel) is FUSED with reverse = 1 */
   int32_t n_reorder;
   int32_t reorder_apps[TACKER_MAX_REORDER];
   double thr_ms;             /* headroom after the decision */
   double gain_ms;            /* Tgain of the fused pair */
   double t_start_ms, t_end_ms; /* manager clock: predicted (sim) or issue time (GPU) */
   int64_t fused_blocks;      /* BE blocks in the fused launch: a PTB slice, or -1 = the whole rest */
+  int32_t reverse;           /* FUSED: 1 = LC CUDA-core kernel + BE tensor-core kernel (NEXT-2) */
 } tacker_decision;
 
 typedef struct {
@@ -411,6 +422,8 @@ typedef struct {
   /* 0 (default): after every LC kernel, fused or not, reorder the other ready BE heads with
    * Ttmp < Thr (reading 6); 1: reorder only after an LC kernel that was not fused. */
   int32_t reorder_only_unfused;
+  /* 1: never fuse an LC CUDA-core kernel with a BE tensor-core kernel (NEXT-2 off) */
+  int32_t no_reverse_fusion;
 } tacker_manager_params;
 
 typedef struct tacker_manager_s *tacker_manager_t;
@@ -461,6 +474,7 @@ typedef struct {
    * calls, and everything else in tacker_manager_step (decisions, bookkeeping) */
   double host_poll_ms, host_launch_ms, host_decide_ms;
   int64_t host_steps;        /* tacker_manager_step calls */
+  int64_t reverse_fused;     /* fused launches that were reverse fusions (included in fused_launches) */
 } tacker_manager_stats;
 tacker_status tacker_manager_stats_get(tacker_manager_t m, tacker_manager_stats *out);
 /* Completion time (manager clock) of a finished query, or -1 if unfinished. */

@@ -33,6 +33,17 @@ Rules, in the paper's order:
     time is X_cd(remaining) once a slice of it has run.  BE work = n/N of the kernel's
     standalone time per slice.
   * reorder_only_unfused: reorder only after an LC kernel that was not fused (P:2035 literally).
+  * Reverse fusion (NEXT-2; "LC and BE kernels are not limited to a specified type",
+    P:924-926; DNN-training BE apps, Table II): when the LC kernel is a CUDA-core
+    kernel (T_lc) and a ready BE head is a tensor-core kernel (T_be; kind 2 below), the same
+    Eq. 8 applies with the roles of the two solo times exchanged in the predictor,
+    Tk_fuse = fuse_pred(x_tc = T_be, x_cd = T_lc): admissible iff T_lc + T_be > Tk_fuse and
+    Tk_fuse - T_lc < Thr; Tgain = T_be - (Tk_fuse - T_lc); Thr -= Tk_fuse - T_lc.  Tensor-core
+    BE kernels are never sliced.
+
+BE kernel kinds (first tuple element of an App kernel): 1 (True) = CUDA-core kernel (fusable with
+an LC tensor-core kernel), 2 = tensor-core kernel (fusable with an LC CUDA-core kernel), 0 (False)
+= never fused (reorder / idle only).
 """
 from __future__ import annotations
 
@@ -41,6 +52,7 @@ import math
 from dataclasses import dataclass, field
 
 TACKER, BAYMAX = 0, 1
+BE_OTHER, BE_CD, BE_TC = 0, 1, 2
 FUSED, ORIGINAL_LC, REORDER_BE, IDLE_BE, NOTHING = 0, 1, 2, 3, 4
 
 
@@ -53,19 +65,33 @@ class Decision:
     thr: float = 0.0
     gain: float = 0.0
     blocks: int = -1              # BE blocks of the fused launch (PTB slice), -1 = whole rest
+    reverse: bool = False         # fused: LC CUDA-core kernel + BE tensor-core kernel (NEXT-2)
 
 
-def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=None, reorder_only_unfused=False):
+def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=None, reorder_only_unfused=False,
+           reverse=True, with_reverse_flag=False):
     """Pure decision for one LC kernel.
 
-    heads: list of (app, Tcd, be_is_cd) for READY BE head kernels, in app order (Tcd = the
-    predicted time of what is left of the head kernel).  fuse_tcd(app) -> the BE time a fused
-    launch would carry (a PTB slice; default Tcd).  fuse_pred(app) -> Tk_fuse or None.
-    Returns (fused_app, reorder_apps, thr, gain)."""
-    fused, gain_best, tf_best = -1, None, None
+    heads: list of (app, Tcd, be_kind) for READY BE head kernels, in app order (Tcd = the
+    predicted time of what is left of the head kernel; be_kind as in the module doc).
+    fuse_tcd(app) -> the BE time a fused launch would carry (a PTB slice; default Tcd).
+    fuse_pred(app) -> Tk_fuse or None (for a reverse pair: the model at x_tc = the BE kernel,
+    x_cd = the LC kernel).  Returns (fused_app, reorder_apps, thr, gain[, reversed])."""
+    fused, gain_best, tf_best, rev = -1, None, None, False
+    if allow and policy == TACKER and not lc_is_tc and reverse:
+        for app, tbe, kind in heads:
+            if kind != BE_TC:
+                continue
+            tf = fuse_pred(app)
+            if tf is None:
+                continue
+            if ttc + tbe > tf and tf - ttc < thr:                   # Eq. 8, roles exchanged
+                gain = tbe - (tf - ttc)
+                if gain_best is None or gain > gain_best:
+                    fused, gain_best, tf_best, rev = app, gain, tf, True
     if allow and policy == TACKER and lc_is_tc:
         for app, tcd, be_cd in heads:
-            if not be_cd:
+            if be_cd != BE_CD:
                 continue
             if fuse_tcd is not None:
                 tcd = fuse_tcd(app)
@@ -86,6 +112,8 @@ def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=No
             if tcd < thr:
                 reorder.append(app)
                 thr -= tcd
+    if with_reverse_flag:
+        return fused, reorder, thr, (gain_best or 0.0), rev
     return fused, reorder, thr, (gain_best or 0.0)
 
 
@@ -117,9 +145,10 @@ class App:
         return self.kernels[self.pos % len(self.kernels)]
 
     def lr(self):
-        """(N, t_block, t_floor) of the head kernel; N = 0 when it has no slicing data."""
+        """(N, t_block, t_floor) of the head kernel; N = 0 when it has no slicing data (and for
+        tensor-core kernels, which are never sliced)."""
         h = self.head()
-        return (h[2], h[3], h[4]) if len(h) >= 5 else (0, 0.0, 0.0)
+        return (h[2], h[3], h[4]) if len(h) >= 5 and h[0] != BE_TC else (0, 0.0, 0.0)
 
     def rem(self):
         """Predicted standalone time of what is left of the head kernel."""
@@ -155,11 +184,13 @@ def slice_blocks(app, ttc, r_opp, slice_be, slice_ratio):
 
 
 def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=None, t_end=None,
-             slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_only_unfused=False):
+             slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_only_unfused=False, reverse=True,
+             rfuse_pred=None):
     """Serial single-stream GPU whose kernels take exactly their predicted time.
 
     fuse_pred(lc_T, be_T) -> Tk_fuse or None; opp_ratio(app) -> the pair's opportune ratio or
-    None (slicing).  The manager acts whenever the stream drains.
+    None (slicing); rfuse_pred(x_tc = BE tensor-core T, x_cd = LC CUDA-core T) -> Tk_fuse or None
+    for reverse pairs (default fuse_pred).  The manager acts whenever the stream drains.
     Returns dict(latency per query, be_completed, be_work, timeline, decisions)."""
     t = 0.0
     active: list[Query] = []
@@ -198,19 +229,27 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 N, sa, sb = apps[a].lr()
                 return sb + sa * n
 
-            fused, reorder, thr2, gain = decide(
-                ttc, is_tc, thr, heads, policy,
-                lambda a: fuse_pred(ttc, tcd_of(a)), allow, fuse_tcd=tcd_of,
-                reorder_only_unfused=reorder_only_unfused)
+            rpred = rfuse_pred or fuse_pred
+            kind_of = {a: k for a, _, k in heads}
+
+            def pred(a):
+                if not is_tc and kind_of[a] == BE_TC:
+                    return rpred(apps[a].rem(), ttc)
+                return fuse_pred(ttc, tcd_of(a))
+
+            fused, reorder, thr2, gain, rev = decide(
+                ttc, is_tc, thr, heads, policy, pred, allow, fuse_tcd=tcd_of,
+                reorder_only_unfused=reorder_only_unfused, reverse=reverse, with_reverse_flag=True)
             if allow:
                 q.thr = thr2
             start = t
             if fused >= 0:
-                dur = fuse_pred(ttc, tcd_of(fused))
+                dur = pred(fused)
                 timeline.append(("fused", q.qid, q.pos, fused, start, start + dur))
-                apps[fused].issue(nblk[fused])
+                apps[fused].issue(-1 if rev else nblk[fused])
                 apps[fused].ready_at = start + dur
-                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), q.thr, gain, nblk[fused]))
+                decisions.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), q.thr, gain,
+                                          -1 if rev else nblk[fused], rev))
             else:
                 dur = ttc
                 timeline.append(("lc", q.qid, q.pos, -1, start, start + dur))

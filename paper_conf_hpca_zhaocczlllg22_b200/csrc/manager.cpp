@@ -100,6 +100,9 @@ struct tacker_manager_s {
     tacker_fused_t f = nullptr;
   };
   std::map<std::tuple<const void *, const void *, const void *, int, size_t>, PairEntry> pairs;
+  // reverse fusion (NEXT-2): keyed by the LC CUDA-core descriptor's bytes and (app, kernel)
+  std::map<std::tuple<std::string, int, size_t>, PairEntry> rpairs;
+  std::set<std::string> prepared_cd;   // LC CUDA-core descriptors already prepared
   // in-flight cap: launches issued vs launches known complete, observed through stream events
   // recorded every ev_every launches (and after launches whose completion is needed), so the
   // stream is not cut by an event after every ~10 us kernel (events block launch overlap)
@@ -149,7 +152,7 @@ struct HostTimer {
 }  // namespace
 
 static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b) {
-  return m->policy == TACKER_POLICY_TACKER && m->prm.slice_be && b.n_blocks > 1 && b.t_block_ms > 0;
+  return m->policy == TACKER_POLICY_TACKER && m->prm.slice_be && !b.is_tc && b.n_blocks > 1 && b.t_block_ms > 0;
 }
 
 // Bookkeeping of n issued blocks of app A's head kernel (n < 0: the whole rest, which completes
@@ -272,6 +275,41 @@ static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, doub
 
 static bool sliceable(const tacker_manager_s *m, const tacker_be_kernel &b);
 
+// ---- reverse fusion (NEXT-2): LC CUDA-core kernel k (the fused kernel's CUDA-core part) with
+// BE tensor-core kernel b (its tcgen05 part); the pair model takes X_tc = b, X_cd = k.
+static int rev_ws(const tacker_lc_kernel &k) { return k.warp_split ? k.warp_split : 16; }
+static bool rpair_key(const tacker_lc_kernel &k, const tacker_be_kernel &b, std::string *pk) {
+  std::string lk, bk;
+  return make_keys(&b.tc, &k.cd, rev_ws(k), &lk, &bk, pk);
+}
+static std::string cd_bytes(const tacker_be_desc &d) {
+  return std::string(reinterpret_cast<const char *>(&d), sizeof d);
+}
+static tacker_manager_s::PairEntry &rpair_entry(tacker_manager_s *m, const tacker_lc_kernel &k, int app, size_t kidx) {
+  const tacker_be_kernel &b = m->apps[app].ks[kidx];
+  auto &e = m->rpairs[std::make_tuple(cd_bytes(k.cd), app, kidx)];
+  if (!e.keyed) {
+    e.keyed = true;
+    if (!rpair_key(k, b, &e.pk)) e.pk.clear();
+  }
+  return e;
+}
+static tacker_status rfused_handle(tacker_manager_s *m, const tacker_lc_kernel &k, int app, size_t kidx,
+                                   tacker_fused_t *out) {
+  auto &pe = rpair_entry(m, k, app, kidx);
+  if (pe.f) {
+    *out = pe.f;
+    return TACKER_OK;
+  }
+  const tacker_be_kernel &b = m->apps[app].ks[kidx];
+  tacker_status s = tacker_fuse(&b.tc, &k.cd, rev_ws(k), tacker_ratio{0, 0}, out);
+  if (s == TACKER_OK) {
+    pe.f = *out;
+    m->owned.push_back(*out);
+  }
+  return s;
+}
+
 // keyed by the LC operands and (app, kernel index): stable across reallocation of the app list
 static tacker_manager_s::PairEntry &pair_entry(tacker_manager_s *m, const tacker_lc_kernel &k, int app, size_t kidx) {
   const tacker_be_kernel &b = m->apps[app].ks[kidx];
@@ -308,6 +346,7 @@ static tacker_status launch_lc(tacker_manager_s *m, const tacker_lc_kernel &k) {
 static tacker_status launch_be(tacker_manager_s *m, const App &A) {
   HostTimer ht(m->host_ns[1]);
   const tacker_be_kernel &b = A.head();
+  if (b.is_tc) return tacker_launch_original(&b.tc, nullptr, reinterpret_cast<tacker_stream_t>(m->stream));
   if (A.done == 0) return tacker_launch_original(nullptr, &b.be, reinterpret_cast<tacker_stream_t>(m->stream));
   tacker_be_desc d = b.be;
   d.block_offset = b.be.block_offset + (int32_t)A.done;
@@ -434,6 +473,11 @@ tacker_status tacker_manager_submit_lc(tacker_manager_t m, const tacker_lc_query
 tacker_status tacker_manager_submit_be(tacker_manager_t m, const tacker_be_app *app, int32_t *id) {
   if (!m || !app || app->n_kernels <= 0 || !app->kernels) return set_error("bad BE app"), TACKER_EINVAL;
   if (m->apps.size() >= TACKER_MAX_APPS) return set_error("too many BE apps"), TACKER_ERESOURCE;
+  for (int32_t i = 0; i < app->n_kernels; ++i) {
+    const tacker_be_kernel &b = app->kernels[i];
+    if (b.is_tc && (b.is_cd || b.tc.kind == TACKER_LC_NONE))
+      return set_error("BE kernel %d: is_tc needs is_cd == 0 and a tensor-core descriptor", i), TACKER_EINVAL;
+  }
   App A;
   A.ks.assign(app->kernels, app->kernels + app->n_kernels);
   A.ready_at = m->now;
@@ -562,6 +606,32 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       }
     }
   }
+  // NEXT-2 reverse fusion: the LC kernel is a CUDA-core kernel and a ready BE head a tensor-core
+  // kernel; Eq. 8 unchanged with t_lc = ttc, t_be = the BE kernel's time (the model's X_tc)
+  bool reverse = false;
+  if (allow && m->policy == TACKER_POLICY_TACKER && !k.is_tc && !m->prm.no_reverse_fusion) {
+    for (int a : heads) {
+      const App &A = m->apps[a];
+      const tacker_be_kernel &b = A.head();
+      if (!b.is_tc) continue;
+      const std::string &pk = rpair_entry(m, k, a, A.pos % A.ks.size()).pk;
+      if (pk.empty()) continue;
+      const double tbe = b.t_pred_ms;
+      double tf;
+      if (!pair_predict(pk, tbe, ttc, &tf)) continue;
+      if (ttc + tbe > tf && tf - ttc < thr) {   // Eq. 8
+        const double gain = tbe - (tf - ttc);
+        if (fused < 0 || gain > best_gain) {
+          fused = a;
+          best_gain = gain;
+          best_tf = tf;
+          best_tcd = tbe;
+          best_n = -1;
+          reverse = true;
+        }
+      }
+    }
+  }
   std::vector<int> reorder;
   if (fused >= 0) thr -= best_tf - ttc;
   // Reorder the remaining ready heads after the LC kernel, fused or not (reading:
@@ -586,6 +656,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   out->fused_blocks = fused >= 0 ? best_n : 0;
   out->gain_ms = fused >= 0 ? best_gain : 0;
   out->thr_ms = thr;
+  out->reverse = reverse ? 1 : 0;
   if (headroom) *headroom = thr;
   if (fused >= 0) {
     App &A = m->apps[fused];
@@ -594,17 +665,31 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       A.ready_at = m->now;
     } else {
       cudaEvent_t e0 = begin(m, TACKER_CLASS_FUSED, true);
-      tacker_status s = launch_fused(m, k, fused, best_n);
+      tacker_status s;
+      if (reverse) {
+        HostTimer ht(m->host_ns[1]);
+        tacker_fused_t f = nullptr;
+        s = rfused_handle(m, k, fused, A.pos % A.ks.size(), &f);
+        if (s == TACKER_OK) s = tacker_launch_fused(f, reinterpret_cast<tacker_stream_t>(m->stream));
+      } else {
+        s = launch_fused(m, k, fused, best_n);
+      }
       if (s) return s;
       cudaEvent_t e = mark(m, true);
       track(m, e0, e, TACKER_CLASS_FUSED);
       if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
-      // online model update from the measured co-run
-      const std::string &pk = pair_entry(m, k, fused, A.pos % A.ks.size()).pk;
-      m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, best_tcd, best_tf});
+      // online model update from the measured co-run: (X_tc, X_cd) of the pair
+      if (reverse) {
+        const std::string &pk = rpair_entry(m, k, fused, A.pos % A.ks.size()).pk;
+        m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, best_tcd, ttc, best_tf});
+      } else {
+        const std::string &pk = pair_entry(m, k, fused, A.pos % A.ks.size()).pk;
+        m->observed.push_back(tacker_manager_s::Observed{ref(m, e0), ref(m, e), pk, ttc, best_tcd, best_tf});
+      }
     }
     issue_be(m, A, best_n);
     m->st.fused_launches++;
+    if (reverse) m->st.reverse_fused++;
     out->action = TACKER_DEC_FUSED;
   } else {
     if (m->sim()) {
@@ -651,7 +736,21 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
 static tacker_status prepare_kernels(tacker_manager_s *m, const tacker_lc_kernel *ks, size_t n) {
   for (size_t i = 0; i < n; ++i) {
     const tacker_lc_kernel &k = ks[i];
-    if (!k.is_tc) continue;
+    if (!k.is_tc) {
+      // reverse pairs (NEXT-2): this CUDA-core kernel with every BE tensor-core kernel
+      if (m->prm.no_reverse_fusion || !m->prepared_cd.insert(cd_bytes(k.cd)).second) continue;
+      for (size_t a = 0; a < m->apps.size(); ++a)
+        for (size_t j = 0; j < m->apps[a].ks.size(); ++j) {
+          const tacker_be_kernel &b = m->apps[a].ks[j];
+          std::string pk;
+          double tf;
+          if (!b.is_tc || !rpair_key(k, b, &pk) || !pair_predict(pk, b.t_pred_ms, k.t_pred_ms, &tf)) continue;
+          tacker_fused_t f = nullptr;
+          tacker_status s = rfused_handle(m, k, (int)a, j, &f);
+          if (s != TACKER_OK && s != TACKER_ERESOURCE && s != TACKER_EUNSUPPORTED) return s;
+        }
+      continue;
+    }
     if (!m->prepared_lc.insert({k.lc.A, k.lc.B, k.lc.D}).second) continue;
     for (size_t a = 0; a < m->apps.size(); ++a)
       for (size_t j = 0; j < m->apps[a].ks.size(); ++j) {

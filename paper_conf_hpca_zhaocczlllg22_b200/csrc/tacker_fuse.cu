@@ -225,6 +225,8 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
           !p.x || !p.out)
         return set_error("im2col: bad args"), TACKER_EINVAL;
       if (p.Kpad % 8 || p.Kpad < p.r * p.s * p.c) return set_error("im2col: Kpad must be a multiple of 8 >= R*S*C"), TACKER_EINVAL;
+      if (p.Kpad > 8 * BeBody<TACKER_BE_IM2COL>::kMaxGroups || p.r > 255 || p.s > 255)
+        return set_error("im2col: Kpad <= %d and R, S <= 255", 8 * BeBody<TACKER_BE_IM2COL>::kMaxGroups), TACKER_EUNSUPPORTED;
       if (BeBody<TACKER_BE_IM2COL>::rows(p) * (p.Kpad / 8) >= (int64_t)1 << 31)
         return set_error("im2col: rows * Kpad / 8 must be < 2^31"), TACKER_EUNSUPPORTED;
       break;

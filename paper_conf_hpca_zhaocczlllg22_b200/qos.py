@@ -93,6 +93,9 @@ class QosRun:
                 self.t_lc.append(_time(lambda: tk.tacker_launch_original(None, d), reps))
         for a, app in enumerate(self.apps):
             for j, bk in enumerate(app.kernels):
+                if bk.is_tc:       # NEXT-2: tensor-core BE kernel (never sliced)
+                    self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(bk.desc, None), reps)
+                    continue
                 self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(None, bk.desc), reps)
                 if self.t_be[(a, j)] >= 0.01 and bk.desc.kind != tk.BE_JDS_SCAN:
                     self.lr_be[(a, j)] = self._fit_slice_lr(a, j, bk, reps)
@@ -101,7 +104,7 @@ class QosRun:
         tcs = [k for k in self.svc.kernels if k.is_tc]
         for a, app in enumerate(self.apps):
             for j, bk in enumerate(app.kernels):
-                if self.t_be[(a, j)] < 0.01:
+                if self.t_be[(a, j)] < 0.01 or bk.is_tc:
                     continue
                 best = None
                 for ws in range(self.ws, 3, -4):
@@ -125,7 +128,7 @@ class QosRun:
                 continue
             for a, app in enumerate(self.apps):
                 for j, bk in enumerate(app.kernels):
-                    if self.t_be[(a, j)] < 0.01:   # < 10 us (phiMag, binning, bfs levels): reorder only
+                    if self.t_be[(a, j)] < 0.01 or bk.is_tc:   # < 10 us (phiMag, binning, bfs levels): reorder only
                         continue
                     if (a, j) not in self.ws_of:
                         continue
@@ -147,8 +150,75 @@ class QosRun:
                     self.pair_err.append(abs(t_pred - t_meas) / t_meas)
                     tk.tacker_pair_add_sample(pkey, self.t_lc[i], self.t_be[(a, j)], t_meas)
                     refit.add(pkey)
+        self._calibrate_reverse(range(len(self.apps)), pair_reps, refit)
         for pkey in refit:
             self.pairs[pkey] = tk.tacker_pair_fit(pkey)
+
+    def _calibrate_reverse(self, app_ids, pair_reps, refit):
+        """NEXT-2 reverse pairs: every LC CUDA-core kernel (the fused kernel's CUDA-core part) with
+        every tensor-core kernel of the BE apps `app_ids` (its tcgen05 part), at REV_WS warps."""
+        for i, (is_tc, d) in enumerate(self._kernel_list()):
+            if is_tc or self.t_lc[i] < 0.01 or d.kind == tk.BE_COPY:
+                continue
+            for a in app_ids:
+                for j, bk in enumerate(self.apps[a].kernels):
+                    if not bk.is_tc:
+                        continue
+                    try:
+                        f = tk.tacker_fuse(bk.desc, d, self.REV_WS)
+                    except tk.TackerError as e:
+                        if e.status not in (tk.ERESOURCE, tk.EUNSUPPORTED):
+                            raise
+                        continue
+                    pkey = f.keys()[2]
+                    if pkey not in self.pairs:
+                        self.pairs[pkey] = self._fit_pair_rev(bk.desc, d, self.t_be[(a, j)], self.t_lc[i], pkey,
+                                                              pair_reps)
+                    t_meas = _time(lambda: f.launch(), 3)
+                    t_pred = tk.tacker_pair_predict(pkey, self.t_be[(a, j)], self.t_lc[i])
+                    self.pair_err.append(abs(t_pred - t_meas) / t_meas)
+                    tk.tacker_pair_add_sample(pkey, self.t_be[(a, j)], self.t_lc[i], t_meas)
+                    refit.add(pkey)
+
+    def add_tc_apps(self, apps, reps=8, pair_reps=5):
+        """Append tensor-core BE apps (NEXT-2) to a calibrated run: time their kernels and fit the
+        reverse pairs with the LC CUDA-core kernels (the existing calibration is kept)."""
+        first = len(self.apps)
+        self.apps = list(self.apps) + list(apps)
+        for a in range(first, len(self.apps)):
+            for j, bk in enumerate(self.apps[a].kernels):
+                assert bk.is_tc, "add_tc_apps takes tensor-core BE apps only"
+                self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(bk.desc, None), reps)
+        refit = set()
+        self._calibrate_reverse(range(first, len(self.apps)), pair_reps, refit)
+        for pkey in refit:
+            self.pairs[pkey] = tk.tacker_pair_fit(pkey)
+        return self
+
+    REV_WS = 24    # CUDA-core warps of a reverse-fused LC kernel (tools/reverse_pair.py: im2col needs 24)
+
+    def _fit_pair_rev(self, tc, cd, x_tc, x_cd, pkey, reps):
+        """Reverse pair (NEXT-2) at the training ratios r = X_cd / X_tc in {0.1, 0.2, 1.8, 1.9}
+        (P:1852-1858): below the whole pair's ratio the CUDA-core kernel runs a PTB block prefix
+        (Fig. 7); above it the tensor-core GEMM runs a prefix of its rows (fewer M tiles)."""
+        import ctypes
+        full = tk.tacker_be_num_blocks(cd)
+        r_full = x_cd / x_tc
+        for r in (0.1, 0.2, 1.8, 1.9):
+            if r <= r_full:
+                n = min(max(int(round(full * r / r_full)), 1), full)
+                c, t = _prefix(cd, n), tc
+            else:
+                t = tk.LcDesc()
+                ctypes.memmove(ctypes.addressof(t), ctypes.addressof(tc), ctypes.sizeof(t))
+                t.M = max(128, int(round(tc.M * r_full / r / 128)) * 128)
+                c = cd
+            f = tk.tacker_fuse(t, c, self.REV_WS)
+            t_f = _time(lambda: f.launch(), reps)
+            xt = _time(lambda: tk.tacker_launch_original(t, None), reps)
+            xc = _time(lambda: tk.tacker_launch_original(None, c), reps)
+            tk.tacker_pair_add_sample(pkey, xt, xc, t_f)
+        return tk.tacker_pair_fit(pkey)
 
     def _fit_slice_lr(self, a, j, bk, reps):
         """Per-kernel LR over PTB slices (§VI-C): standalone time of the first n
@@ -201,7 +271,7 @@ class QosRun:
     def lc_kernels(self):
         out = []
         for (is_tc, d), t in zip(self._kernel_list(), self.t_lc):
-            lk = tk.LcKernel(is_tc=1 if is_tc else 0, t_pred_ms=t)
+            lk = tk.LcKernel(is_tc=1 if is_tc else 0, t_pred_ms=t, warp_split=0 if is_tc else self.REV_WS)
             if is_tc:
                 lk.lc = d
             else:
@@ -214,6 +284,9 @@ class QosRun:
         for a, app in enumerate(self.apps):
             ks = []
             for j, bk in enumerate(app.kernels):
+                if bk.is_tc:
+                    ks.append(tk.BeKernel(is_cd=0, is_tc=1, t_pred_ms=self.t_be[(a, j)], tc=bk.desc))
+                    continue
                 n, tb, tf = self.lr_be.get((a, j), (0, 0.0, 0.0))
                 ks.append(tk.BeKernel(is_cd=1, t_pred_ms=self.t_be[(a, j)], be=bk.desc,
                                       warp_split=self.ws_of.get((a, j), self.ws),
@@ -246,7 +319,7 @@ class QosRun:
 
     # ------------------------------------------------------------------ one managed run
     def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None,
-            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False):
+            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True):
         """Poisson arrivals at `load` x the service's peak rate (1 / standalone query time; the
         paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
         stream = torch.cuda.current_stream()
@@ -258,7 +331,8 @@ class QosRun:
         gaps = rng.exponential(1.0 / lam, n_queries + warmup)
         cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
         m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
-                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused)
+                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused,
+                       reverse_fusion=reverse_fusion)
         for ks in self.be_apps():
             m.submit_be(ks)
         kernels = self.lc_kernels()
@@ -282,7 +356,8 @@ class QosRun:
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
                 # normalised BE throughput: standalone-milliseconds of BE work per wall millisecond
                 "be_work_ms": st.be_work_ms, "be_norm_thpt": st.be_work_ms / gpu_ms,
-                "fused": int(st.fused_launches), "reordered": int(st.reordered_be), "idle_be": int(st.idle_be),
+                "fused": int(st.fused_launches), "reverse_fused": int(st.reverse_fused),
+                "reordered": int(st.reordered_be), "idle_be": int(st.idle_be),
                 "model_refits": int(st.model_refits),
                 "fused_pred_err_mean": st.pred_err_sum / st.pred_err_n if st.pred_err_n else None,
                 "class_ms": {n: float(st.class_ms[c]) for c, n in enumerate(("lc_tc", "lc_cd", "fused", "be"))},

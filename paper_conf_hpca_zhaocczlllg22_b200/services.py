@@ -119,6 +119,7 @@ class BeKernelSpec:
     mufu: float = 0.0       # MUFU ops
     bytes: float = 0.0      # algorithmic DRAM bytes
     bound: str = "hbm"
+    is_tc: bool = False     # NEXT-2: a tensor-core BE kernel (desc is a tk.LcDesc)
 
 
 @dataclass
@@ -213,6 +214,24 @@ def tpacf_app(n=16384, seed=2022) -> BeAppSpec:
     ks = [BeKernelSpec("tpacf.dd", tk.be_tpacf(d, d, e, dd, self_pairs=True), bytes=12.0 * n, bound="alu"),
           BeKernelSpec("tpacf.dr", tk.be_tpacf(d, r, e, dr), bytes=24.0 * n, bound="alu")]
     return BeAppSpec(f"tpacf_{n}", ks, [e, d, r, dd, dr])
+
+
+def gemm_train_app(M=4096, N=4096, K=4096, n=2, seed=2025) -> BeAppSpec:
+    """NEXT-2 reverse fusion: a DNN-training-like BE job of tensor-core kernels (Table II's
+    Res-T / VGG-T are training jobs): n fp16 GEMMs D = A B^T (fp32 accumulate, fp16
+    out) chained through their outputs, cycled forever."""
+    bufs, ks = [], []
+    A, B = synth.lc_gemm_inputs(M, N, K, seed)
+    dA = _dev(A)
+    for i in range(n):
+        _, Bi = synth.lc_gemm_inputs(8, N, K, seed + 1 + i)
+        dB = _dev((Bi.astype(np.float32) / np.sqrt(K)).astype(np.float16))
+        D = torch.empty(M, N, dtype=torch.float16, device="cuda")
+        ks.append(BeKernelSpec(f"train.gemm{i}", tk.lc_gemm(dA, dB, D, b_const=True), flops=2.0 * M * N * K,
+                               bytes=2.0 * (M * K + N * K + M * N), bound="tensor", is_tc=True))
+        bufs += [dB, D]
+        dA = D if N == K else dA
+    return BeAppSpec(f"train_gemm_{M}x{N}x{K}", ks, [dA] + bufs)
 
 
 def lbm_app(nx=120, ny=120, nz=150, seed=2022) -> BeAppSpec:

@@ -189,7 +189,8 @@ class FusedInfo(C.Structure):
 
 
 class LcKernel(C.Structure):
-    _fields_ = [("is_tc", C.c_int32), ("t_pred_ms", C.c_double), ("lc", LcDesc), ("cd", BeDesc)]
+    _fields_ = [("is_tc", C.c_int32), ("t_pred_ms", C.c_double), ("lc", LcDesc), ("cd", BeDesc),
+                ("warp_split", C.c_int32)]
 
 
 class LcQuery(C.Structure):
@@ -198,7 +199,8 @@ class LcQuery(C.Structure):
 
 class BeKernel(C.Structure):
     _fields_ = [("is_cd", C.c_int32), ("t_pred_ms", C.c_double), ("be", BeDesc), ("warp_split", C.c_int32),
-                ("n_blocks", C.c_int32), ("t_block_ms", C.c_double), ("t_floor_ms", C.c_double)]
+                ("n_blocks", C.c_int32), ("t_block_ms", C.c_double), ("t_floor_ms", C.c_double),
+                ("is_tc", C.c_int32), ("tc", LcDesc)]
 
 
 class BeApp(C.Structure):
@@ -209,13 +211,13 @@ class Decision(C.Structure):
     _fields_ = [("action", C.c_int32), ("query", C.c_int32), ("lc_index", C.c_int32), ("fused_app", C.c_int32),
                 ("n_reorder", C.c_int32), ("reorder_apps", C.c_int32 * MAX_REORDER), ("thr_ms", C.c_double),
                 ("gain_ms", C.c_double), ("t_start_ms", C.c_double), ("t_end_ms", C.c_double),
-                ("fused_blocks", C.c_int64)]
+                ("fused_blocks", C.c_int64), ("reverse", C.c_int32)]
 
 
 class ManagerParams(C.Structure):
     _fields_ = [("direct_eps_ms", C.c_double), ("idle_cap_ms", C.c_double), ("max_inflight", C.c_int32),
                 ("simulate", C.c_int32), ("slice_be", C.c_int32), ("slice_ratio", C.c_double),
-                ("reorder_only_unfused", C.c_int32)]
+                ("reorder_only_unfused", C.c_int32), ("no_reverse_fusion", C.c_int32)]
 
 
 class ManagerStats(C.Structure):
@@ -224,7 +226,7 @@ class ManagerStats(C.Structure):
                 ("now_ms", C.c_double), ("model_refits", C.c_int64), ("class_ms", C.c_double * 4),
                 ("class_launches", C.c_int64 * 4), ("pred_err_sum", C.c_double), ("pred_err_n", C.c_int64),
                 ("be_work_ms", C.c_double), ("host_poll_ms", C.c_double), ("host_launch_ms", C.c_double),
-                ("host_decide_ms", C.c_double), ("host_steps", C.c_int64)]
+                ("host_decide_ms", C.c_double), ("host_steps", C.c_int64), ("reverse_fused", C.c_int64)]
 
 
 CLASS_LC_TC, CLASS_LC_CD, CLASS_FUSED, CLASS_BE = range(4)
@@ -657,10 +659,11 @@ class Manager:
     """Owning wrapper of tacker_manager_t."""
 
     def __init__(self, policy=POLICY_TACKER, stream=None, simulate=False, direct_eps_ms=0.0, idle_cap_ms=0.0,
-                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False):
+                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True):
         self.h = C.c_void_p()
         self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0,
-                                    1 if slice_be else 0, slice_ratio, 1 if reorder_only_unfused else 0)
+                                    1 if slice_be else 0, slice_ratio, 1 if reorder_only_unfused else 0,
+                                    0 if reverse_fusion else 1)
         _chk(_lib.tacker_manager_create(policy, C.byref(self.params), _stream(stream), C.byref(self.h)))
         self._keep = []
 

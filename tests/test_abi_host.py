@@ -169,6 +169,22 @@ def be_kernel(tk, t, ws=16):
     return b
 
 
+def be_kernel_tc(tk, t):
+    b = tk.BeKernel(is_cd=0, is_tc=1, t_pred_ms=t)
+    b.tc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=512, N=512, K=512, A=FAKE, B=FAKE, D=FAKE)
+    return b
+
+
+def fit_reverse_pair_closed_form(tk, tau):
+    # reverse pair (NEXT-2): BE gemm 512^3 as the tcgen05 part, the LC fma_burn (it10) as the
+    # CUDA-core part, the LC kernel's default 16 warps
+    key = "pair:lc:gemm:N512:K512:bn128:f32|be:fma_burn:it10|ws16"
+    for r in (0.1, 0.2, 1.8, 1.9):
+        tk.tacker_pair_add_sample(key, 1.0, r, tau(r))
+    tk.tacker_pair_fit(key)
+    return key
+
+
 def fit_pair_closed_form(tk, tau):
     # the pair key of (gemm 1024^3, stencil nz=8, ws16), fitted exactly to tau(r) = max(l1, l2)
     key = "pair:lc:gemm:N1024:K1024:bn128:f32|be:stencil:nz8|ws16"
@@ -178,7 +194,7 @@ def fit_pair_closed_form(tk, tau):
     return key
 
 
-@pytest.mark.parametrize("policy", ["tacker", "baymax"])
+@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse"])
 def test_manager_simulation_matches_reference(tk, policy):
     tk.tacker_model_clear()
     # stage-2 slope != 1 so that Tgain depends on Tcd (with slope 1 every stage-2 pair has the
@@ -186,11 +202,18 @@ def test_manager_simulation_matches_reference(tk, policy):
     tau = lambda r: max(1 + 0.25 * r, 0.4 + 0.93 * r)
     fit_pair_closed_form(tk, tau)
     fuse_pred = lambda ttc, tcd: ttc * tau(tcd / ttc)
+    reverse = policy == "tacker_reverse"
+    tau_r = lambda r: max(1 + 0.35 * r, 0.3 + 0.97 * r)
+    fit_reverse_pair_closed_form(tk, tau_r)
+    rfuse_pred = lambda xtc, xcd: xtc * tau_r(xcd / xtc)
     rng = np.random.default_rng(11)
     arrivals = np.cumsum(rng.exponential(6.0, 60))
     shapes = [[(True, 1.21), (False, 0.3), (True, 0.83), (True, 1.97)], [(True, 0.52), (True, 0.49)]]
+    if reverse:   # LC CUDA-core kernels long enough to hide a BE tensor-core kernel
+        shapes = [[(True, 1.21), (False, 1.3), (True, 0.83), (False, 0.61)], [(False, 0.92), (True, 0.49)]]
     app_ts = [[1.53, 0.71], [3.07], [0.43, 0.37, 2.51]]
-    pol = tk.POLICY_TACKER if policy == "tacker" else tk.POLICY_BAYMAX
+    tc_apps = [[0.47, 1.12], [0.81]] if reverse else []
+    pol = tk.POLICY_BAYMAX if policy == "baymax" else tk.POLICY_TACKER
     m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0)
     qs = []
     for i, t in enumerate(arrivals):
@@ -201,7 +224,11 @@ def test_manager_simulation_matches_reference(tk, policy):
     for ts in app_ts:
         m.submit_be([be_kernel(tk, d) for d in ts])
         apps.append(mr.App([(True, d) for d in ts]))
-    ref = mr.simulate(qs, apps, 50.0, mr.TACKER if policy == "tacker" else mr.BAYMAX, fuse_pred, idle_cap=2.0)
+    for ts in tc_apps:
+        m.submit_be([be_kernel_tc(tk, d) for d in ts])
+        apps.append(mr.App([(mr.BE_TC, d) for d in ts]))
+    ref = mr.simulate(qs, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER, fuse_pred, idle_cap=2.0,
+                      rfuse_pred=rfuse_pred)
     got = []
     for _ in range(100000):
         st = m.stats()
@@ -209,17 +236,21 @@ def test_manager_simulation_matches_reference(tk, policy):
             break
         d = m.step(50.0)
         if d.action in (tk.DEC_FUSED, tk.DEC_ORIGINAL_LC, tk.DEC_REORDER_BE, tk.DEC_IDLE_BE):
-            got.append((d.action, d.fused_app, tuple(d.reorder_apps[:d.n_reorder])))
-    exp = [(x.action, x.fused_app, tuple(x.reorder)) for x in ref["decisions"]]
+            got.append((d.action, d.fused_app, tuple(d.reorder_apps[:d.n_reorder]), bool(d.reverse)))
+    exp = [(x.action, x.fused_app, tuple(x.reorder), bool(x.reverse)) for x in ref["decisions"]]
     assert got == exp
     for i in range(len(arrivals)):
         assert abs(m.latency(i) - ref["latency"][i]) < 1e-9
     assert max(ref["latency"].values()) <= 50.0
-    if policy == "tacker":
+    if policy != "baymax":
         assert m.stats().fused_launches > 0
+    assert m.stats().reverse_fused == sum(1 for x in exp if x[3])
+    if reverse:
+        assert m.stats().reverse_fused > 0 and any(x[0] == mr.FUSED and not x[3] for x in exp)
     # be_work_ms = standalone time of every BE kernel issued, app heads cycling in order
+    app_ts = app_ts + tc_apps
     work, pos = 0.0, [0] * len(app_ts)
-    for _, fa, ra in exp:
+    for _, fa, ra, _ in exp:
         for a in ([fa] if fa >= 0 else []) + list(ra):
             work += app_ts[a][pos[a] % len(app_ts[a])]
             pos[a] += 1

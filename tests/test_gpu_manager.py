@@ -1,0 +1,67 @@
+"""GPU: NEXT-2 reverse fusion (LC CUDA-core kernel + BE tensor-core kernel) through the
+C ABI -- the fused kernel against the oracle and bit-identical to the original launches, and a
+short managed run whose reverse-fused queries produce the same bytes as standalone queries."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import lc as olc
+from oracle.metrics import max_rel_err
+
+pytestmark = pytest.mark.gpu
+
+from tests.gpu_helpers import dev, host, t  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def tk():
+    from paper_conf_hpca_zhaocczlllg22_b200 import tacker
+    assert torch.cuda.is_available()
+    return tacker
+
+
+def test_reverse_fused_im2col_with_be_gemm(tk):
+    # LC CUDA-core part: conv1's explicit im2col (b2, ragged last block); BE tensor-core part: a
+    # training-like fp16 GEMM
+    cs = synth.ConvShape("conv1", 2, 64, 60, 8, 64, 7, 7, 2, 3)
+    x, _, _ = synth.conv_inputs(cs, seed=4, real_c=3)
+    M, _, K = cs.gemm_mnk
+    Kpad = ((K + 63) // 64) * 64
+    dx = t(x)
+    cols0 = torch.zeros(M, Kpad, dtype=torch.float16, device=dev())
+    cols1 = torch.zeros_like(cols0)
+    A, B = synth.lc_gemm_inputs(512, 384, 1024, seed=5)
+    dA, dB = t(A), t(B)
+    D0 = torch.zeros(512, 384, device=dev())
+    D1 = torch.zeros_like(D0)
+    tk.tacker_launch_original(tk.lc_gemm(dA, dB, D0), tk.be_im2col(dx, cols0, 7, 7, 2, 3, Kpad))
+    f = tk.tacker_fuse(tk.lc_gemm(dA, dB, D1), tk.be_im2col(dx, cols1, 7, 7, 2, 3, Kpad), 16)
+    f.launch()
+    assert host(cols1).tobytes() == host(cols0).tobytes()
+    assert host(D1).tobytes() == host(D0).tobytes()
+    assert np.array_equal(host(cols1), olc.im2col(x, 7, 7, 2, 3, Kpad))
+    ref, S = olc.lc_gemm(A, B)
+    assert max_rel_err(host(D1), ref, S) <= 1e-2
+
+
+def test_managed_reverse_fusion_outputs_match_standalone(tk):
+    from paper_conf_hpca_zhaocczlllg22_b200 import qos, services as sv
+    # LC service = ResNet-50 conv1 at batch 32 (im2col on the CUDA cores + GEMM) and the next conv;
+    # BE queue = one tensor-core training GEMM app (tools/reverse_pair.py: this pair overlaps)
+    convs = synth.resnet50_convs(32)[:2]
+    svc = sv.resnet50_service(32, convs=convs)
+    app = sv.gemm_train_app(4096, 4096, 4096, n=1)
+    # reference bytes: one standalone query
+    for k in svc.kernels:
+        tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd)
+    ref = host(svc.outputs[-1]).tobytes()
+    run = qos.QosRun(svc, [app], warp_split=16)
+    run.calibrate(reps=3, pair_reps=3)
+    assert any("be:im2col" in k for k in run.pairs), run.pairs.keys()
+    run.measure_service(n=20)
+    svc.outputs[-1].zero_()
+    res = run.run(tk.POLICY_TACKER, 40, load=0.8)
+    assert res["qos_met"]
+    assert res["reverse_fused"] > 0, res
+    assert host(svc.outputs[-1]).tobytes() == ref

@@ -202,6 +202,36 @@ def test_manager_slice_to_opportune_ratio():
         assert abs(res["be_work"] - 40.0) < 1e-12 and res["be_completed"] == [2]
 
 
+def test_manager_reverse_fusion_scenarios():
+    """NEXT-2, hand-computed (Thr 40 as in S1-S7): LC CUDA-core kernel 2 ms, BE tensor-core head
+    3 ms, Tk_fuse 4 -> Eq. 8 holds (5 > 4, 4 - 2 = 2 < 40): FUSED, Tgain 3 - 2 = 1, Thr 38.
+    Tk_fuse 5 -> not admitted (strict >): the head is reordered (3 < 40), Thr 37.  A CUDA-core
+    head never pairs with a CUDA-core LC kernel, nor a tensor-core head with a tensor-core one."""
+    fp = lambda a: {0: 4.0, 1: 4.5}[a]
+    fused, reorder, thr, gain, rev = mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, fp,
+                                               with_reverse_flag=True)
+    assert (fused, reorder, rev) == (0, [], True) and thr == 38.0 and gain == 1.0
+    fused, reorder, thr, _ = mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, lambda a: 5.0)
+    assert (fused, reorder, thr) == (-1, [0], 37.0)
+    # two tensor-core heads: gains 1 (3 ms, 4.0) and 2.5 - 2.5 = ... (3 ms, 4.5) -> 0.5: the first wins
+    fused, reorder, thr, gain = mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC), (1, 3.0, mr.BE_TC)], mr.TACKER, fp)
+    assert fused == 0 and gain == 1.0 and reorder == [1] and thr == 35.0
+    assert mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_CD)], mr.TACKER, lambda a: 1.0)[0] == -1
+    assert mr.decide(2.0, True, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, lambda a: 1.0)[0] == -1
+    assert mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, fp, reverse=False)[0] == -1
+    assert mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC)], mr.BAYMAX, fp)[0] == -1
+    # in a run: TC kernel (1 ms, no CUDA-core head to fuse) with the 3 ms tensor-core head
+    # reordered behind it (Thr 47); the CUDA-core kernel then fuses with the app's next
+    # tensor-core kernel (Tk_fuse 4): latency 1 + 3 + 4 = 8, two BE kernels (6 ms of work)
+    q = mr.Query(0, 0.0, [(True, 1.0), (False, 2.0)])
+    app = mr.App([(mr.BE_TC, 3.0)])
+    res = mr.simulate([q], [app], 50.0, mr.TACKER, lambda ttc, tcd: None, rfuse_pred=lambda xtc, xcd: 4.0)
+    d0, d1 = res["decisions"][:2]
+    assert d0.action == mr.REORDER_BE and d0.reorder == [0] and abs(d0.thr - 44.0) < 1e-12
+    assert d1.action == mr.FUSED and d1.reverse and d1.fused_app == 0 and abs(d1.thr - 42.0) < 1e-12
+    assert res["latency"][0] == 8.0 and res["be_completed"] == [2] and res["be_work"] == 6.0
+
+
 # ------------------------------------------------------------------ metrics
 def test_overlap_rate_bounds():
     assert metrics.overlap_rate(1.0, 1.0, 1.0) == 0.5      # perfect overlap
