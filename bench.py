@@ -496,7 +496,13 @@ def run_tacker(args, ws, rank, local):
         rr = managed_runs(qr, tk, args.steps, 2000 + rank, args.inflight, ("tacker", "tacker_no_reverse", "baymax"))
         reverse = {"workload": "resnet50_b%d LC + stencil / mri-q / train-GEMM (2 x 4096^3 fp16) BE queue" % args.batch,
                    "train_gemm_ms": [qr.t_be[(2, j)] for j in range(len(train.kernels))],
-                   "im2col_ms": qr.t_lc[0]}
+                   "im2col_ms": qr.t_lc[0], "pairs": {}}
+        for j, bk in enumerate(train.kernels):
+            f = tk.tacker_fuse(bk.desc, svc.kernels[0].cd, qr.REV_WS)
+            pk = f.keys()[2]
+            reverse["pairs"][pk] = {"fused_ms": qos._time(lambda: f.launch(), 5),
+                                    "predicted_ms": tk.tacker_pair_predict(pk, qr.t_be[(2, j)], qr.t_lc[0]),
+                                    "in_model": pk in qr.pairs}
         for v, r in rr.items():
             reverse[v] = {k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms", "qos_met", "fused",
                                             "reverse_fused", "reordered")}

@@ -41,6 +41,8 @@ struct LcParams {
   int32_t tp, tq;          // output tile = tp x tq positions (tp*tq == 128)
   int32_t tiles_p, tiles_q, c_blocks;
   int32_t conv_direct_gemm;  // 1x1 stride-1 conv handled as a plain GEMM over [n*h*w, c]
+  int32_t conv_im2col;       // implicit conv through the TMA im2col mode: M-tile = 128 consecutive
+                             // output pixels (n, p, q linear); else tp x tq windows of one image
   // split-K: work unit u = (tile u / splits, k-blocks [s kb_per_split, (s+1) kb_per_split) of split
   // s = u % splits).  splits > 1 only when every unit has its own CTA (num_units <= grid): the
   // splits of a tile write fp32 partials, meet on a counter, then each reduces 1/splits of the tile
@@ -109,7 +111,7 @@ struct LcGemm {
   }
   // output row (GEMM row of D) of row r of M-tile mt, or -1 outside the problem
   static __device__ __forceinline__ int64_t out_row(const LcParams &L, int mt, int r) {
-    if (implicit_conv(L)) {
+    if (implicit_conv(L) && !L.conv_im2col) {
       const int img = mt / (L.tiles_p * L.tiles_q);
       const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
       const int pp = pt * L.tp + r / L.tq, qq = qt * L.tq + r % L.tq;
@@ -166,7 +168,17 @@ struct LcGemm {
   // A (activations) k-block kb of M-tile mt
   static __device__ __forceinline__ void load_a(const FusedParams &P, uint64_t *bar, uint8_t *sa, int kb, int mt) {
     const LcParams &L = P.lc;
-    if (implicit_conv(L)) {
+    if (implicit_conv(L) && L.conv_im2col) {
+      // k-block -> (filter tap r,s ; channel block cb); A = 128 output pixels from m0 = 128 mt,
+      // first pixel (n0, p0, q0) -> input corner (q0 stride - pad, p0 stride - pad), tap offset (s, r)
+      const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
+      const int rr = rs / L.s, ss = rs % L.s;
+      const int pq = L.p * L.q, m0 = mt * kBM;
+      const int n0 = m0 / pq, rem = m0 - n0 * pq;
+      const int p0 = rem / L.q, q0 = rem - p0 * L.q;
+      tma_load_im2col_4d(&P.tmap_a, bar, sa, cb * kBK, q0 * L.stride - L.pad, p0 * L.stride - L.pad, n0,
+                         (uint16_t)ss, (uint16_t)rr);
+    } else if (implicit_conv(L)) {
       // k-block -> (filter tap r,s ; channel block cb); A = shifted NHWC window (implicit im2col)
       const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
       const int rr = rs / L.s, ss = rs % L.s;

@@ -94,6 +94,18 @@ __device__ __forceinline__ void tma_load_4d(const void *tmap, uint64_t *bar, voi
       : "memory");
 }
 
+// im2col mode (convolution A operand): 128 output pixels walked from (c0, w0, h0, n0) in the
+// tensor map's bounding box (traversal stride = conv stride), each reading its channel range at
+// the filter-tap offset (ow, oh); out-of-image pixels are zero-filled.
+__device__ __forceinline__ void tma_load_im2col_4d(const void *tmap, uint64_t *bar, void *dst, int32_t c0, int32_t w0,
+                                                   int32_t h0, int32_t n0, uint16_t ow, uint16_t oh) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+      "[%2], {%7, %8};" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(tmap)), "r"(smem_u32(bar)), "r"(c0), "r"(w0), "r"(h0), "r"(n0), "h"(ow), "h"(oh)
+      : "memory");
+}
+
 __device__ __forceinline__ void tma_load_3d(const void *tmap, uint64_t *bar, void *dst, int32_t c0, int32_t c1,
                                             int32_t c2) {
   asm volatile(

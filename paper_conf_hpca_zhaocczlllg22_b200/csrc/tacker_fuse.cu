@@ -13,6 +13,7 @@
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <memory>
@@ -297,9 +298,24 @@ static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
   return 128;
 }
 
+// Implicit convs load A through the TMA im2col mode (linear 128-pixel M-tiles, no padding of a
+// small image to a 128-position window) unless TACKER_CONV_TILED=1 selects the tiled 4-D windows.
+static bool conv_im2col_mode() {
+  static const bool tiled = [] {
+    const char *e = getenv("TACKER_CONV_TILED");
+    return e && e[0] == '1';
+  }();
+  return !tiled;
+}
+
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
-  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
+  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && conv_im2col_mode()) {
+    L.conv_im2col = 1;
+    L.tiles_m = (L.M + kBM - 1) / kBM;
+    L.c_blocks = L.c / kBK;
+    L.num_kb = L.r * L.s * L.c_blocks;
+  } else if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
     // output tile of 128 positions: tq along q (power of two <= 32 covering q), tp = 128/tq
     int tq = 1;
     while (tq < L.q && tq < 32) tq <<= 1;
@@ -376,6 +392,49 @@ static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, cons
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv x) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+using PFN_encodeIm2col = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                       const cuuint64_t *, const int *, const int *, cuuint32_t, cuuint32_t,
+                                       const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                       CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static PFN_encodeIm2col get_encode_im2col() {
+  static PFN_encodeIm2col fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeIm2col>(p);
+  });
+  return fn;
+}
+
+// A of an implicit conv in im2col mode: NHWC as (C, W, H, N); the pixel bounding box of every
+// image is [-pad, W - 1 + pad - (S - 1)] x [-pad, H - 1 + pad - (R - 1)] walked with the conv
+// stride, i.e. exactly the P x Q output positions; 64 channels (128 B, SW128) per pixel, 128
+// pixels per load.
+static tacker_status encode_conv_im2col(CUtensorMap *m, const tacker_lc_desc &d) {
+  auto enc = get_encode_im2col();
+  if (!enc) return set_error("cuTensorMapEncodeIm2col unavailable"), TACKER_ECUDA;
+  if (d.pad > 127 || d.pad - (d.s - 1) < -128 || d.pad - (d.r - 1) < -128 || d.r > 256 || d.s > 256)
+    return set_error("conv: padding / filter outside the im2col corner range"), TACKER_EUNSUPPORTED;
+  cuuint64_t dims[4] = {(cuuint64_t)d.c, (cuuint64_t)d.w, (cuuint64_t)d.h, (cuuint64_t)d.n};
+  cuuint64_t strides[3] = {(cuuint64_t)d.c * 2, (cuuint64_t)d.c * d.w * 2, (cuuint64_t)d.c * d.w * d.h * 2};
+  int lower[2] = {-d.pad, -d.pad};
+  int upper[2] = {d.pad - (d.s - 1), d.pad - (d.r - 1)};
+  cuuint32_t es[4] = {1, (cuuint32_t)d.stride, (cuuint32_t)d.stride, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void *>(d.A), dims, strides, lower, upper,
+                   (cuuint32_t)kBK, (cuuint32_t)kBM, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeIm2col(conv x) failed: %d", (int)r), TACKER_ECUDA;
+  // driver <= 13.1 with a tensor under 128 KiB: clear descriptor bit 85 (as CUTLASS does)
+  int drv = 0;
+  if (cudaDriverGetVersion(&drv) == cudaSuccess && drv <= 13010 &&
+      (uint64_t)d.n * d.h * d.w * d.c * 2 < 131072)
+    reinterpret_cast<uint64_t *>(m)[1] &= ~(1ull << 21);
   return TACKER_OK;
 }
 
@@ -558,7 +617,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
 
   // TMA tensor maps
   if (lc->kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-    if ((st = encode_conv_x(&F.P.tmap_a, *lc, L))) return st;
+    if ((st = L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc) : encode_conv_x(&F.P.tmap_a, *lc, L))) return st;
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   } else {
     if ((st = encode_2d(&F.P.tmap_a, lc->A, (uint64_t)L.K, (uint64_t)L.M, kBK, kBM))) return st;
