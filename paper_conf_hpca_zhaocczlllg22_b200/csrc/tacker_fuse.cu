@@ -295,6 +295,13 @@ static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
   if (L.N <= 64) return 64;
   const int sms = sm_count() > 0 ? sm_count() : 148;
   if (L.N >= 256 && (int64_t)((L.M + 127) / 128) * ((L.N + 255) / 256) >= 2LL * sms) return 256;
+  // deep-K problems (>= kDeepKb k-blocks) with few tiles: 256-wide tiles halve the A traffic per
+  // flop through L2 (the bound of these mainloops); split-K (lc_split) then fills the SMs
+  static const int deep_kb = [] {
+    const char *e = getenv("TACKER_DEEP_KB");
+    return e ? atoi(e) : 1 << 30;
+  }();
+  if (L.N >= 256 && (L.K + kBK - 1) / kBK >= deep_kb) return 256;
   return 128;
 }
 
