@@ -130,7 +130,7 @@ typedef enum {
   TACKER_BE_MRIFHD_FH = 20,   /* mri-fhd ComputeFH: F^H d over one k chunk; block = 32 voxels x 4 k-lanes */
   TACKER_BE_CP = 21,          /* cp direct Coulomb summation on one lattice slice; block = 128x4 points */
   TACKER_BE_FFT_TWIDDLE = 22, /* fft plan: twiddle table w[m] = exp(-2 pi i m / n); block = 128 entries */
-  TACKER_BE_FFT = 23,         /* batched forward complex DFT, length n <= 2048; block = 1 transform */
+  TACKER_BE_FFT = 23,         /* batched forward complex DFT, length n <= 1024; block = 1 transform */
   TACKER_BE_TPACF = 24,       /* angular correlation histogram; block = 128 points of a      */
   TACKER_BE_KIND_COUNT = 25
 } tacker_be_kind;
@@ -154,9 +154,9 @@ typedef struct { int32_t numX, numK; const float *x, *y, *z, *kx, *ky, *kz, *rRh
 typedef struct { int32_t natoms, nx, ny; float h, z; const float *atoms; float *V; } tacker_be_cp;
 /* fft (Parboil; Fig. 10's GEMM-fft pair P:1417-1419; reading 15): y[b, k] = sum_j x[b, j]
  * exp(-2 pi i j k / n), b < batch, complex fp32 interleaved (re, im) [batch][n][2], out of place,
- * x, y 16-byte aligned; n a power of two in [2, 2048].  twiddle [n][2] fp32 is written by
+ * x, y 16-byte aligned; n a power of two in [2, 1024].  twiddle [n][2] fp32 is written by
  * TACKER_BE_FFT_TWIDDLE (w[m] = (cos, -sin)(2 pi m / n), accurate sincospi) and read by
- * TACKER_BE_FFT (Stockham radix-4/2 in shared memory). */
+ * TACKER_BE_FFT (Stockham radix-8/4/2 in shared memory). */
 typedef struct { int32_t n, batch; float *twiddle; const float *x; float *y; } tacker_be_fft;
 /* tpacf (Parboil; reading 16): count[bin(a_i . b_j)] += 1 over all (i, j) (self_pairs = 0) or
  * over i < j with b == a (self_pairs = 1); bin(d) = #{k : d < edges[k]}, edges strictly

@@ -17,6 +17,12 @@ constexpr int kVbThreads = 128;
 #ifndef TK_MRIQ_COARSEN
 #define TK_MRIQ_COARSEN 4
 #endif
+#ifndef TK_FFT_MAXN
+#define TK_FFT_MAXN 1024
+#endif
+#ifndef TK_FFT_MIN_BLOCKS
+#define TK_FFT_MIN_BLOCKS 12
+#endif
 #ifndef TK_MRIQ_REDUCE
 #define TK_MRIQ_REDUCE 0
 #endif

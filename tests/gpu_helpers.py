@@ -189,9 +189,10 @@ def be_case(kind, seed=0, size="small"):
             assert max_rel_err(o[0].ravel(), ref, S) <= 1e-5
         return dict(desc=tk.be_cp(dat, V, h, z), outs=[V], reset=lambda: V.zero_(), check=check, keep=(dat,))
     if kind in (tk.BE_FFT, tk.BE_FFT_TWIDDLE):
-        # small: a ragged batch at n = 256 (radix-4 only); "odd": n = 2048 (final radix-2 pass);
-        # large: the bench shape on sampled rows
-        batch, n = {"small": (37, 256), "odd": (5, 2048), "tiny": (3, 2), "large": (1 << 14, 1024)}[size]
+        # radix passes: small n = 256 (8, 8, 4); "odd" n = 1024 (8, 8, 8, 2); "mid" n = 128 (8, 8, 2);
+        # "tiny" n = 2; large: the bench shape on sampled rows
+        batch, n = {"small": (37, 256), "odd": (7, 1024), "mid": (11, 128), "tiny": (3, 2),
+                    "large": (1 << 14, 1024)}[size]
         x = synth.fft_inputs(batch, n, seed)
         dx = t(x)
         tw = torch.zeros(n, 2, device=dev())
