@@ -54,7 +54,10 @@ TK_BE_SEL(TACKER_BE_TPACF, tpacf)
 
 // Maximum BE warps per fused CTA: register-heavy bodies (sgemm's 8x4 register tile) keep the
 // CTA at 6+16 warps (80 registers/thread); the others allow 6+24 warps (64 registers/thread).
-__host__ __device__ constexpr int be_max_warps(int kind) { return kind == TACKER_BE_SGEMM ? 16 : 24; }
+// LC-only instantiations (kind NONE) have no BE warps: their launch bound is the 6 LC warps.
+__host__ __device__ constexpr int be_max_warps(int kind) {
+  return kind == TACKER_BE_NONE ? 0 : kind == TACKER_BE_SGEMM ? 16 : 24;
+}
 // Minimum resident blocks per SM of an original (standalone) BE launch: caps the registers of
 // bodies whose latency hiding needs many blocks (fft: TK_FFT_MIN_BLOCKS = 12 blocks -> <= 40 registers).
 __host__ __device__ constexpr int be_orig_min_blocks(int kind) { return kind == TACKER_BE_FFT ? TK_FFT_MIN_BLOCKS : 1; }

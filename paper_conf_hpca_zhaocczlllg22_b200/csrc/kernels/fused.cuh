@@ -124,13 +124,12 @@ struct LcGemm {
   // all out): + bias (preloaded, bias8 = bias[n..n+7]), + residual, ReLU, one 16-byte (fp16) or
   // two 16-byte (fp32) stores
   static __device__ __forceinline__ void store8(const LcParams &L, int64_t orow, int n, float (&f)[8],
-                                                const float *bias8) {
+                                                const float *bias8, uint4 rv) {
     if (L.epi & TACKER_EPI_BIAS) {
 #pragma unroll
       for (int j = 0; j < 8; ++j) f[j] = __fadd_rn(f[j], bias8[j]);
     }
     if (L.epi & TACKER_EPI_RESIDUAL) {
-      const uint4 rv = *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n);
       const __half2 *rh = reinterpret_cast<const __half2 *>(&rv);
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -267,7 +266,12 @@ struct LcGemm {
     }
   }
 
+  // EC columns per batch: EC/16 TMEM loads in flight behind one wait, and the batch's residual
+  // rows requested before that wait (LC-only launches: 64 columns; fused CTAs, capped at 64
+  // registers per thread: 16)
+  template <int EC>
   static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem) {
+    static_assert(EC % 16 == 0 && BN % EC == 0, "EC: multiple of 16 dividing BN");
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;          // TMEM lanes 32*quarter .. +31
     const int row_in_tile = quarter * 32 + lane_id();
@@ -290,26 +294,34 @@ struct LcGemm {
         for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
         named_bar_sync(kLcEpiBar, 128);
       }
+      const bool res = !prow && (L.epi & TACKER_EPI_RESIDUAL) && orow >= 0;
 #pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 16) {
-        uint32_t v[16];
-        tmem_ld_32x32b_x16(tbase + c0, v);
-        tmem_ld_wait();
+      for (int c0 = 0; c0 < BN; c0 += EC) {
+        uint32_t v[EC / 16][16];
+#pragma unroll
+        for (int i = 0; i < EC / 16; ++i) tmem_ld_32x32b_x16(tbase + c0 + 16 * i, v[i]);
         const int n0 = nt * BN + c0;
+        uint4 rv[EC / 8];
+#pragma unroll
+        for (int g = 0; g < EC / 8; ++g)
+          rv[g] = (res && n0 + 8 * g < L.N) ? *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n0 + 8 * g)
+                                            : make_uint4(0, 0, 0, 0);
+        tmem_ld_wait();
         if (orow < 0 || n0 >= L.N) continue;
         if (prow) {   // split-K partial, fp32
 #pragma unroll
-          for (int j = 0; j < 16; j += 4)
-            *reinterpret_cast<float4 *>(prow + c0 + j) = make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]),
-                                                                    __uint_as_float(v[j + 2]), __uint_as_float(v[j + 3]));
+          for (int j = 0; j < EC; j += 4)
+            *reinterpret_cast<float4 *>(prow + c0 + j) =
+                make_float4(__uint_as_float(v[j / 16][j % 16]), __uint_as_float(v[j / 16][j % 16 + 1]),
+                            __uint_as_float(v[j / 16][j % 16 + 2]), __uint_as_float(v[j / 16][j % 16 + 3]));
         } else {
 #pragma unroll
-          for (int j = 0; j < 16; j += 8)
+          for (int j = 0; j < EC; j += 8)
             if (n0 + j < L.N) {
               float f[8];
 #pragma unroll
-              for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j + u]);
-              store8(L, orow, n0 + j, f, bb.bias + c0 + j);
+              for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j / 16][j % 16 + u]);
+              store8(L, orow, n0 + j, f, bb.bias + c0 + j, rv[j / 8]);
             }
         }
       }
@@ -360,7 +372,9 @@ struct LcGemm {
         *reinterpret_cast<float4 *>(bias) = __ldg(reinterpret_cast<const float4 *>(L.bias + n));
         *reinterpret_cast<float4 *>(bias + 4) = __ldg(reinterpret_cast<const float4 *>(L.bias + n + 4));
       }
-      store8(L, orow, n, f, bias);
+      const uint4 rv = (L.epi & TACKER_EPI_RESIDUAL) ? *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n)
+                                                     : make_uint4(0, 0, 0, 0);
+      store8(L, orow, n, f, bias, rv);
     }
     named_bar_sync(kLcEpiBar, 128);
     if (et == 0 && atomicAdd(finish, 1u) == (uint32_t)S - 1) {   // last reducer: reset for the next launch
@@ -466,7 +480,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
       } else if (warp == 1) {
         if (lane_id() == 0) LcGemm<BN>::mma(P, lc, bb, tmem);
       } else {
-        LcGemm<BN>::epilogue(P, bb, tmem);
+        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : 16>(P, bb, tmem);
       }
     }
   } else if constexpr (BE_KIND != TACKER_BE_NONE) {
