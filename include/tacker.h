@@ -424,6 +424,13 @@ typedef struct {
   int32_t reorder_only_unfused;
   /* 1: never fuse an LC CUDA-core kernel with a BE tensor-core kernel (NEXT-2 off) */
   int32_t no_reverse_fusion;
+  /* B200 reading 18 (off = the paper's rule: only the newest query fuses / reorders):
+   * 1 = an older query may fuse / reorder too, within the smallest headroom of itself and of every
+   * later active query (Eq. 9 of each at the current time), so no later query is pushed past the
+   * QoS target either; that bound is lowered by older_margin_ms (a guard against the predictor's
+   * error and the host running ahead of the GPU). */
+  int32_t fuse_older;
+  double older_margin_ms;
 } tacker_manager_params;
 
 typedef struct tacker_manager_s *tacker_manager_t;

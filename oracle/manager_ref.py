@@ -41,6 +41,13 @@ Rules, in the paper's order:
     Tk_fuse - T_lc < Thr; Tgain = T_be - (Tk_fuse - T_lc); Thr -= Tk_fuse - T_lc.  Tensor-core
     BE kernels are never sliced.
 
+  * fuse_older (B200 reading 18 in DESIGN.md §2; off by default): an older query (not the
+    newest) also fuses / reorders, spending at most min(its own Thr, Thr_j of every later active
+    query j) with Thr_j = T_qos - (t - arrival_j) - sum of the remaining predicted time of j and
+    of every active query ahead of j (Eq. 9 at time t); its own Thr is then reduced by what the
+    decision spent.  Eq. 9 for a query at its first issue counts only the queries ahead of it.
+    older_margin lowers that bound (a guard against prediction error on the GPU).
+
 BE kernel kinds (first tuple element of an App kernel): 1 (True) = CUDA-core kernel (fusable with
 an LC tensor-core kernel), 2 = tensor-core kernel (fusable with an LC CUDA-core kernel), 0 (False)
 = never fused (reorder / idle only).
@@ -185,7 +192,7 @@ def slice_blocks(app, ttc, r_opp, slice_be, slice_ratio):
 
 def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=None, t_end=None,
              slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_only_unfused=False, reverse=True,
-             rfuse_pred=None):
+             rfuse_pred=None, fuse_older=False, older_margin=0.0):
     """Serial single-stream GPU whose kernels take exactly their predicted time.
 
     fuse_pred(lc_T, be_T) -> Tk_fuse or None; opp_ratio(app) -> the pair's opportune ratio or
@@ -212,13 +219,22 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
             newest = active[-1]
             if q.issue is None:
                 q.issue = t
-                if q is newest:
-                    earlier = sum(o.remaining() for o in active[:-1])
+                if q is newest or fuse_older:
+                    earlier = sum(o.remaining() for o in active[:active.index(q)])
                     q.thr = qos - (t - q.arrival) - q.remaining() - earlier
                     q.direct = q.thr <= direct_eps
             is_tc, ttc = q.kernels[q.pos]
-            allow = (q is newest) and not q.direct and q.thr is not None
+            allow = (q is newest or fuse_older) and not q.direct and q.thr is not None
             thr = q.thr if q.thr is not None else 0.0
+            thr_in = thr
+            if allow and q is not newest:
+                ahead = 0.0
+                for j, o in enumerate(active):
+                    ahead += o.remaining()
+                    if j > active.index(q):
+                        thr = min(thr, qos - (t - o.arrival) - ahead)
+                thr -= older_margin
+            thr_eff = thr
             nblk = {a: slice_blocks(apps[a], ttc, opp_ratio(a) if opp_ratio else None, slice_be, slice_ratio)
                     for a, _, _ in heads}
 
@@ -241,7 +257,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 ttc, is_tc, thr, heads, policy, pred, allow, fuse_tcd=tcd_of,
                 reorder_only_unfused=reorder_only_unfused, reverse=reverse, with_reverse_flag=True)
             if allow:
-                q.thr = thr2
+                q.thr = thr_in - (thr_eff - thr2)
             start = t
             if fused >= 0:
                 dur = pred(fused)

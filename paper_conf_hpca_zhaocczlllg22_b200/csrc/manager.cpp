@@ -563,20 +563,38 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
 
   Query &q = m->queries[qid];
   const bool newest = (qid == m->active.back());
+  const bool older_ok = m->prm.fuse_older != 0;
   if (!q.issued) {
     q.issued = true;
-    if (newest) {
-      double earlier = 0;
-      for (int id : m->active)
-        if (id != qid) earlier += m->queries[id].remaining();
+    if (newest || older_ok) {
+      double earlier = 0;   // remaining predicted time of the active queries ahead of q
+      for (int id : m->active) {
+        if (id == qid) break;
+        earlier += m->queries[id].remaining();
+      }
       q.thr = qos - (t - q.arrival) - q.remaining() - earlier;   // Eq. 9
       q.has_thr = true;
       q.direct = q.thr <= m->prm.direct_eps_ms;
     }
   }
-  const bool allow = newest && q.has_thr && !q.direct;
+  const bool allow = (newest || older_ok) && q.has_thr && !q.direct;
   double thr = q.has_thr ? q.thr : 0.0;
   if (allow && headroom && !std::isnan(*headroom)) thr = *headroom;
+  // reading 18: an older query spends at most the smallest headroom of itself and of every later
+  // active query (Eq. 9 of each at time t)
+  const double thr_in = thr;
+  if (allow && !newest) {
+    double ahead = 0;
+    bool after = false;
+    for (int id : m->active) {
+      const Query &o = m->queries[id];
+      ahead += o.remaining();
+      if (after) thr = std::min(thr, qos - (t - o.arrival) - ahead);
+      if (id == qid) after = true;
+    }
+    thr -= m->prm.older_margin_ms;
+  }
+  const double thr_eff = thr;
   const tacker_lc_kernel &k = q.ks[q.pos];
   const double ttc = k.t_pred_ms;
 
@@ -647,7 +665,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       }
     }
   }
-  if (allow) q.thr = thr;
+  if (allow) q.thr = thr_in - (thr_eff - thr);   // what this decision spent
 
   // execute
   out->query = qid;

@@ -319,7 +319,8 @@ class QosRun:
 
     # ------------------------------------------------------------------ one managed run
     def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None,
-            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True):
+            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True, fuse_older=False,
+            older_margin_ms=None):
         """Poisson arrivals at `load` x the service's peak rate (1 / standalone query time; the
         paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
         stream = torch.cuda.current_stream()
@@ -332,7 +333,8 @@ class QosRun:
         cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
         m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
                        slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused,
-                       reverse_fusion=reverse_fusion)
+                       reverse_fusion=reverse_fusion, fuse_older=fuse_older,
+                       older_margin_ms=0.2 * self.qos if older_margin_ms is None else older_margin_ms)
         for ks in self.be_apps():
             m.submit_be(ks)
         kernels = self.lc_kernels()

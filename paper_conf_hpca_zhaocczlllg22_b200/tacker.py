@@ -217,7 +217,8 @@ class Decision(C.Structure):
 class ManagerParams(C.Structure):
     _fields_ = [("direct_eps_ms", C.c_double), ("idle_cap_ms", C.c_double), ("max_inflight", C.c_int32),
                 ("simulate", C.c_int32), ("slice_be", C.c_int32), ("slice_ratio", C.c_double),
-                ("reorder_only_unfused", C.c_int32), ("no_reverse_fusion", C.c_int32)]
+                ("reorder_only_unfused", C.c_int32), ("no_reverse_fusion", C.c_int32), ("fuse_older", C.c_int32),
+                ("older_margin_ms", C.c_double)]
 
 
 class ManagerStats(C.Structure):
@@ -659,11 +660,12 @@ class Manager:
     """Owning wrapper of tacker_manager_t."""
 
     def __init__(self, policy=POLICY_TACKER, stream=None, simulate=False, direct_eps_ms=0.0, idle_cap_ms=0.0,
-                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True):
+                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True,
+                 fuse_older=False, older_margin_ms=0.0):
         self.h = C.c_void_p()
         self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0,
                                     1 if slice_be else 0, slice_ratio, 1 if reorder_only_unfused else 0,
-                                    0 if reverse_fusion else 1)
+                                    0 if reverse_fusion else 1, 1 if fuse_older else 0, older_margin_ms)
         _chk(_lib.tacker_manager_create(policy, C.byref(self.params), _stream(stream), C.byref(self.h)))
         self._keep = []
 

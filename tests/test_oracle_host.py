@@ -232,6 +232,29 @@ def test_manager_reverse_fusion_scenarios():
     assert res["latency"][0] == 8.0 and res["be_completed"] == [2] and res["be_work"] == 6.0
 
 
+def test_manager_fuse_older_respects_later_headroom():
+    """Reading 18, hand-computed.  Q0 (arrives 0): [TC 2, TC 2]; Q1 arrives at 1: [TC 3].  BE app:
+    CUDA-core kernel 4 ms, Tk_fuse = ttc + 1.5 for any pair (extra 1.5, gain 2.5).
+    At t=0 Q0 is alone (newest): Thr0 = 50 - 4 = 46, fused (Thr0 44.5), ends at 3.5.  At 3.5 Q1
+    has arrived, so Q0 is no longer the newest: paper rule -> Q0's second kernel runs plain;
+    fuse_older -> Thr_eff = min(44.5, 50 - (3.5 - 1) - (2 + 3)) = 42.5 -> fused again, and Q1
+    still has 50 - 2.5 - 3 - 3.5 (extra) >= 0 left."""
+    fp = lambda ttc, tcd: ttc + 1.5
+    for older, n_fused in ((False, 1), (True, 2)):
+        qs = [mr.Query(0, 0.0, [(True, 2.0), (True, 2.0)]), mr.Query(1, 1.0, [(True, 3.0)])]
+        apps = [mr.App([(True, 4.0)])]
+        res = mr.simulate(qs, apps, 50.0, mr.TACKER, fp, fuse_older=older)
+        q0 = [d for d in res["decisions"] if d.lc and d.lc[0] == 0]
+        assert sum(d.action == mr.FUSED for d in q0) == n_fused
+        if older:
+            assert abs(q0[1].thr - (44.5 - 1.5)) < 1e-12   # Q0's own headroom pays the extra
+    # a later query with no headroom left blocks the older query's fusion
+    qs = [mr.Query(0, 0.0, [(True, 2.0), (True, 2.0)]), mr.Query(1, 1.0, [(True, 47.0)])]
+    res = mr.simulate(qs, [mr.App([(True, 4.0)])], 50.0, mr.TACKER, fp, fuse_older=True)
+    q0 = [d for d in res["decisions"] if d.lc and d.lc[0] == 0]
+    assert q0[0].action == mr.FUSED and q0[1].action != mr.FUSED
+
+
 # ------------------------------------------------------------------ metrics
 def test_overlap_rate_bounds():
     assert metrics.overlap_rate(1.0, 1.0, 1.0) == 0.5      # perfect overlap
