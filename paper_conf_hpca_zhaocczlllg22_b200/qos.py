@@ -334,7 +334,7 @@ class QosRun:
         m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
                        slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused,
                        reverse_fusion=reverse_fusion, fuse_older=fuse_older,
-                       older_margin_ms=0.2 * self.qos if older_margin_ms is None else older_margin_ms)
+                       older_margin_ms=0.3 * self.qos if older_margin_ms is None else older_margin_ms)
         for ks in self.be_apps():
             m.submit_be(ks)
         kernels = self.lc_kernels()
