@@ -60,8 +60,21 @@ def test_managed_reverse_fusion_outputs_match_standalone(tk):
     run.calibrate(reps=3, pair_reps=3)
     assert any("be:im2col" in k for k in run.pairs), run.pairs.keys()
     run.measure_service(n=20)
+    pk = next(k for k in run.pairs if "be:im2col" in k)
+    t_be, t_lc = run.t_be[(0, 0)], run.t_lc[0]
+    gain = t_be - (tk.tacker_pair_predict(pk, t_be, t_lc) - t_lc)     # Eq. 8's Tgain for this pair
     svc.outputs[-1].zero_()
     res = run.run(tk.POLICY_TACKER, 40, load=0.8)
     assert res["qos_met"]
+    # the manager fuses exactly when the calibrated model predicts a gain (measured on this box)
+    assert (res["reverse_fused"] > 0) == (gain > 0), (gain, res["reverse_fused"])
+    assert host(svc.outputs[-1]).tobytes() == ref
+    # the GPU reverse-fused launch path, whatever this box measured: a model with a sure gain
+    tk.tacker_model_clear()
+    for r in (0.1, 0.2, 1.8, 1.9):
+        tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0, r) + 0.05)
+    tk.tacker_pair_fit(pk)
+    svc.outputs[-1].zero_()
+    res = run.run(tk.POLICY_TACKER, 40, load=0.8)
     assert res["reverse_fused"] > 0, res
     assert host(svc.outputs[-1]).tobytes() == ref
