@@ -42,7 +42,7 @@ def be_case(kind, seed=0, size="small"):
         return dict(desc=tk.be_sgemm(dA, dB, dC), outs=[dC], reset=lambda: dC.zero_(), check=check,
                     keep=(dA, dB))
     if kind == tk.BE_STENCIL:
-        # small: TMA plane-tile path (nx % 4 == 0) with a partial x tile and partial y / z blocks;
+        # small: float4 path (nx % 4 == 0) with a partial x tile and partial y / z blocks;
         # scalar: nx % 4 != 0 path
         nx, ny, nz = {"small": (132, 21, 19), "scalar": (70, 37, 9), "large": (512, 512, 64)}[size]
         A = synth.stencil_inputs(nx, ny, nz, seed)
