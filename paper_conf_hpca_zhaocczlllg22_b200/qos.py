@@ -56,6 +56,60 @@ def _time(fn, reps=10, stream=None, inner=8):
     return statistics.median(ts)
 
 
+def _interp_n(curve, t_target, full):
+    """Smallest block count whose standalone time reaches t_target, by linear interpolation of the
+    measured (blocks, ms) curve (the BE time is not linear near its one-block latency floor)."""
+    pts = sorted(curve)
+    if t_target <= pts[0][1]:
+        return pts[0][0]
+    for (n0, t0), (n1, t1) in zip(pts, pts[1:]):
+        if t0 <= t_target <= t1:
+            return min(full, max(1, int(round(n0 + (n1 - n0) * (t_target - t0) / max(t1 - t0, 1e-9)))))
+    return full
+
+
+def training_prefixes(prefix, full, x_tc, curve, time_fn, ratios=(0.1, 0.2, 1.8, 1.9), min_gap=0.08,
+                      stage2_to_full=True):
+    """BE block prefixes for the two-stage model's training ratios, realised on the
+    MEASURED BE time: each target r gives the block count whose interpolated standalone time is
+    r X_tc.  Below the one-block floor the targets shift up (as the sweep does); above what the
+    whole kernel reaches the stage-2 pair becomes the whole kernel and a prefix 0.15 below it.
+    The two points of a stage are kept at least min_gap apart in measured r (two prefixes on the
+    latency floor, or a clamp, would otherwise give a degenerate stage line).  stage2_to_full: the
+    second stage-2 sample is the whole kernel (its ratio is the one the manager predicts; 1.8 and
+    1.9 alone left the stage-2 slope to measurement noise over 0.1 of r, extrapolated up to r ~ 18).
+    prefix(n) -> descriptor, time_fn(desc) -> ms, curve = [(blocks, ms)] incl. 1 and full.
+    Returns [(n, x_cd)] (four samples; fewer when the kernel has fewer distinct prefixes)."""
+    pts = sorted(curve)
+    r_floor, r_full = pts[0][1] / x_tc, pts[-1][1] / x_tc
+    shift = max(0.0, 1.25 * r_floor - ratios[0])
+    tr = [r + shift for r in ratios]
+    if stage2_to_full and r_full > tr[2] + min_gap:
+        tr[3] = r_full               # reading 5: stage 2 spans up to the whole kernel's ratio
+    if tr[3] > r_full:
+        tr[3] = r_full
+        tr[2] = max(min(tr[2], r_full - 0.15), tr[1] + min_gap)
+    if tr[2] >= r_full:
+        # the whole BE kernel is short next to this LC kernel: no stage-2 ratio is reachable with
+        # BE prefixes, so the samples spread evenly over what is, [r_floor-ish, r_full]
+        lo = min(tr[0], r_full)
+        tr = [lo + (r_full - lo) * i / 3 for i in range(4)]
+    out = []
+    for i, r in enumerate(tr):
+        n = _interp_n(pts, r * x_tc, full) if r < r_full else full
+        if out and n <= out[-1][0]:
+            if out[-1][0] >= full:
+                break                    # fewer distinct samples than four
+            n = min(full, out[-1][0] + 1)
+        x = time_fn(prefix(n))
+        if i in (1, 3):
+            while (x - out[-1][1]) / x_tc < min_gap and n < full:
+                n = min(full, max(n + 1, int(n * 1.5)))
+                x = time_fn(prefix(n))
+        out.append((n, x))
+    return out
+
+
 class QosRun:
     def __init__(self, svc, apps, warp_split=24, qos_ms=50.0):
         self.svc, self.apps, self.ws, self.qos = svc, apps, warp_split, qos_ms
@@ -65,6 +119,7 @@ class QosRun:
         self.ws_of = {}          # (app, kernel) -> warp split that fits the budget
         self.pair_err = []       # |pred - meas| / meas of the fused model on the real pairs
         self.lr_be = {}          # (app, kernel) -> (n_blocks, t_block_ms, t_floor_ms): slice LR
+        self.curve_be = {}       # (app, kernel) -> [(blocks, ms)] measured prefixes incl. 1 block
 
     # ------------------------------------------------------------------ calibration (§VI-C)
     def with_io(self):
@@ -227,36 +282,34 @@ class QosRun:
         full = tk.tacker_be_num_blocks(bk.desc)
         key = f"be:slice:app{a}:k{j}"
         ns = sorted({max(1, full // d) for d in (16, 8, 4, 2, 1)})
+        curve = []
         for n in ns:
             d = _prefix(bk.desc, n)
             t = self.t_be[(a, j)] if n == full else _time(lambda: tk.tacker_launch_original(None, d), reps)
             tk.tacker_model_add_sample(key, n, t)
+            curve.append((n, t))
+        if ns[0] > 1:     # the one-block floor (not an LR sample: the LR covers the slice regime)
+            d1 = _prefix(bk.desc, 1)
+            curve.append((1, _time(lambda: tk.tacker_launch_original(None, d1), reps)))
+        self.curve_be[(a, j)] = sorted(curve)
         slope, icpt = tk.tacker_model_fit(key)
         return (full, max(slope, 0.0), max(icpt, 0.0))
 
     def _fit_pair(self, k, bk, ws, x_tc, pkey, reps):
+        """Two-stage model of (LC kernel k, BE kernel bk, ws) from fused runs at the training ratios
+        (P:1852-1858), the BE sized by PTB prefixes picked on its measured time curve
+        (training_prefixes)."""
         full = tk.tacker_be_num_blocks(bk.desc)
         prefix = lambda n: _prefix(bk.desc, n)
-        t_full = self.t_be_of(bk)
-        # BE duration is ~ linear in blocks above its one-block floor (PTB LR): the
-        # slice LR when the kernel has one, else the line through one block and the whole kernel
-        lr = next((v for (a_, j_), v in self.lr_be.items() if self.apps[a_].kernels[j_] is bk), None)
-        if lr is not None and lr[1] > 0:
-            _, a, t0 = lr
-            t_one = t0 + a
-        else:
-            t_one = _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)
-            a = (t_full - t_one) / max(full - 1, 1)
-            t0 = t_one - a
-        r_floor = t_one / x_tc
-        shift = max(0.0, 1.25 * r_floor - 0.1)
-        for r in (0.1 + shift, 0.2 + shift, 1.8 + shift, 1.9 + shift):
-            n = int(round((r * x_tc - t0) / a)) if a > 0 else full
-            n = min(max(n, 1), full)
+        aj = next(((a_, j_) for (a_, j_) in self.t_be if self.apps[a_].kernels[j_] is bk), None)
+        curve = self.curve_be.get(aj)
+        if not curve:
+            curve = [(1, _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)), (full, self.t_be_of(bk))]
+        time_fn = lambda d: _time(lambda: tk.tacker_launch_original(None, d), reps)
+        for n, x_cd in training_prefixes(prefix, full, x_tc, curve, time_fn):
             d = prefix(n)
             f = tk.tacker_fuse(k.lc, d, ws)
             t_f = _time(lambda: f.launch(), reps)
-            x_cd = _time(lambda: tk.tacker_launch_original(None, d), reps)
             tk.tacker_pair_add_sample(pkey, x_tc, x_cd, t_f)
         return tk.tacker_pair_fit(pkey)
 

@@ -325,3 +325,22 @@ def test_manager_slicing_matches_reference(tk, mode):
         assert abs(m.latency(i) - ref["latency"][i]) < 1e-9
     assert abs(m.stats().be_work_ms - ref["be_work"]) < 1e-9
     assert m.stats().be_kernels_done == sum(ref["be_completed"])
+
+
+def test_training_prefixes_spread_over_the_latency_floor(tk):
+    """Calibration host logic: the two-stage model's training prefixes are picked on the measured
+    BE time curve; two prefixes on the one-block latency floor (the r01 sweep's degenerate stage-1
+    fits) or a clamp at the whole kernel must not give coincident points."""
+    from paper_conf_hpca_zhaocczlllg22_b200.qos import training_prefixes
+    full = 1000
+    t_of = lambda n: 0.04 + (0.0 if n < 8 else 0.0002 * (n - 8))      # floor 40 us up to 8 blocks
+    curve = [(n, t_of(n)) for n in (1, 50, 125, 250, 500, 1000)]
+    for x_tc in (0.05, 0.2, 1.0):
+        out = training_prefixes(lambda n: n, full, x_tc, curve, t_of)
+        ns = [n for n, _ in out]
+        rs = [x / x_tc for _, x in out]
+        assert ns == sorted(ns) and len(set(ns)) == len(ns) >= 3, ns
+        for i in (1, 3):
+            if i < len(ns):
+                assert rs[i] - rs[i - 1] >= 0.08 - 1e-12 or ns[i] == full
+        assert all(abs(x - t_of(n)) < 1e-12 for n, x in out)

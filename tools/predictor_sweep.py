@@ -4,8 +4,9 @@ LC = BERT-base seq-128 GEMMs (QKV, O, FFN1, FFN2), BE = cutcp / lbm / spmv, warp
 1. Per-kernel LR (P:1839-1851): LC x = tiles (M varied), BE x = original blocks (PTB prefix);
    error of the LR on held-out sizes (paper: <= 3 % max, < 2 % mean).
 2. Two-stage fused model (Eqs. 1-6): trained on r in {0.1, 0.2, 1.8, 1.9} with the
-   BE sized by inverting its LR, evaluated on 12 other ratios in [0.05, 3] with predictions from
-   the LRs (paper: < 8 %).
+   BE sized on its measured time curve (qos.training_prefixes), evaluated on other BE prefixes
+   (3-100 % of the blocks) with predictions from the LRs and from measured X (the model alone)
+   (paper: < 8 %, P:3183-3198).
 Prints one JSON line and writes the fitted model store (tacker_model_save) if a path is given.
 
   python tools/predictor_sweep.py [--ws 8,16,24] [--out profiles/r01/predictor_sweep.json]
@@ -24,6 +25,7 @@ import torch  # noqa: E402
 
 import synth  # noqa: E402
 from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk  # noqa: E402
+from paper_conf_hpca_zhaocczlllg22_b200.qos import training_prefixes  # noqa: E402
 
 
 def timeit(fn, reps=15):
@@ -150,36 +152,43 @@ def main():
                     continue
                 pkey = probe.keys()[2]
 
-                def run_at(r):
-                    n = int(round((r * x_tc - bb) / ba))
-                    n = min(max(n, 1), full)
+                def run_n(n):
                     d = mk(n)
                     f = tk.tacker_fuse(lcd, d, ws)
                     t_f = timeit(lambda: f.launch())
                     x_cd = timeit(lambda: tk.tacker_launch_original(None, d))
-                    return n, x_cd, t_f
-                # A BE kernel cannot run shorter than one original block (its latency floor: e.g.
-                # spmv's longest JDS rows, a cutcp region): ratios below r_floor are not achievable,
-                # so the training and evaluation ratios are shifted above it.
+                    return x_cd, t_f
+
+                # The BE kernel is sized on its measured time curve (qos.training_prefixes): the
+                # training ratios {0.1, 0.2, 1.8, 1.9} shifted above the one-block latency floor,
+                # the two points of each stage kept apart in measured r.
                 x_floor = timeit(lambda: tk.tacker_launch_original(None, mk(1)))
+                curve = sorted(set([(1, x_floor)] + [(n, t) for n, t in res["be_lr"][bname]["samples"]]))
                 r_floor = x_floor / x_tc
                 shift = max(0.0, 1.25 * r_floor - train_r[0])
-                tr = [r + shift for r in train_r]
-                er = [r + shift for r in eval_r]
+                pref = training_prefixes(mk, full, x_tc, curve,
+                                         lambda d: timeit(lambda: tk.tacker_launch_original(None, d)))
                 train = []
-                for r in tr:
-                    n, x_cd, t_f = run_at(r)
+                for n, x_cd in pref:
+                    _, t_f = run_n(n)
                     tk.tacker_pair_add_sample(pkey, x_tc, x_cd, t_f)
-                    train.append((r, n, x_cd, t_f))
+                    train.append((x_cd / x_tc, n, x_cd, t_f))
+                # evaluation: other prefixes spread over the measured range (not the training ones)
+                trained = {n for n, _ in pref}
+                er = []
+                for f_ in (0.03, 0.08, 0.15, 0.25, 0.4, 0.6, 0.8, 1.0):
+                    n = max(1, int(full * f_))
+                    if n not in trained:
+                        er.append(n)
                 coef = tk.tacker_pair_fit(pkey)
                 errs, errs_meas, ev = [], [], []
-                for r in er:
-                    n, x_cd, t_f = run_at(r)
+                for n in er:
+                    x_cd, t_f = run_n(n)
                     pred = tk.tacker_pair_predict(pkey, x_tc_pred, tk.tacker_model_predict(bkey, n))
                     pred_m = tk.tacker_pair_predict(pkey, x_tc, x_cd)   # model error alone
                     errs.append(abs(pred - t_f) / t_f)
                     errs_meas.append(abs(pred_m - t_f) / t_f)
-                    ev.append((r, n, x_cd, t_f, pred))
+                    ev.append((x_cd / x_tc, n, x_cd, t_f, pred))
                 rs = (coef[2] - coef[0]) / (coef[1] - coef[3]) if coef[1] != coef[3] else None
                 res["pairs"].append({"lc": lname, "be": bname, "ws": ws, "x_tc_ms": x_tc, "coef": coef,
                                      "r_floor": r_floor, "ratio_shift": shift,
@@ -190,6 +199,10 @@ def main():
     summary = {"lc_lr_max_err": max(v["max_err"] for v in res["lc_lr"].values()),
                "be_lr_max_err": max(v["max_err"] for v in res["be_lr"].values()),
                "pair_max_err": max(pe), "pair_mean_err": statistics.mean(p["mean_err"] for p in res["pairs"]),
+               # the two-stage model alone (measured X_tc, X_cd), and its median over the pairs
+               "pair_model_max_err": max(p["max_err_measured_x"] for p in res["pairs"]),
+               "pair_model_mean_err": statistics.mean(p["mean_err_measured_x"] for p in res["pairs"]),
+               "pair_model_mean_err_median": statistics.median(p["mean_err_measured_x"] for p in res["pairs"]),
                "pairs": len(pe), "paper": {"per_kernel_max": 0.03, "fused_max": 0.08}}
     res["summary"] = summary
     if args.models:
