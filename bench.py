@@ -392,7 +392,7 @@ def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "ta
     out = {}
     kw = {"tacker": (tk.POLICY_TACKER, dict(HEADLINE)), "baymax": (tk.POLICY_BAYMAX, {}),
           "tacker_paper": (tk.POLICY_TACKER, {}),
-          "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
+          "tacker_slice": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True)),
           "tacker_no_reverse": (tk.POLICY_TACKER, dict(HEADLINE, reverse_fusion=False))}
     for v in variants:
         pol, extra = kw[v]
