@@ -197,6 +197,8 @@ class QosRun:
                     pkey = f.keys()[2]
                     if pkey not in self.pairs:
                         self.pairs[pkey] = self._fit_pair(k, bk, ws, self.t_lc[i], pkey, pair_reps)
+                    if self.pairs[pkey] is None:
+                        continue
                     # accuracy of the 4-point model on the actual whole-kernel pair, then that
                     # co-run joins the pair's history (the paper trains on historical data and
                     # refits from co-running data)
@@ -306,7 +308,10 @@ class QosRun:
         if not curve:
             curve = [(1, _time(lambda: tk.tacker_launch_original(None, prefix(1)), reps)), (full, self.t_be_of(bk))]
         time_fn = lambda d: _time(lambda: tk.tacker_launch_original(None, d), reps)
-        for n, x_cd in training_prefixes(prefix, full, x_tc, curve, time_fn):
+        samples = training_prefixes(prefix, full, x_tc, curve, time_fn)
+        if len(samples) < 2:
+            return None           # too few distinct prefixes (a tiny kernel): no model, never fused
+        for n, x_cd in samples:
             d = prefix(n)
             f = tk.tacker_fuse(k.lc, d, ws)
             t_f = _time(lambda: f.launch(), reps)

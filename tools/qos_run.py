@@ -36,6 +36,8 @@ def build_apps(names):
             apps.append(sv.histo_app())
         elif n == "bfs":
             apps.append(sv.bfs_app())
+        elif n in ("mrifhd", "cp", "fft", "tpacf"):
+            apps.append(getattr(sv, n + "_app")())
         else:
             raise ValueError(n)
     return apps
@@ -67,7 +69,9 @@ def main():
     res = {}
     variants = {"baymax": (tk.POLICY_BAYMAX, {}), "tacker": (tk.POLICY_TACKER, {}),
                 "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
-                "tacker_slice_literal": (tk.POLICY_TACKER, {"slice_be": True, "reorder_only_unfused": True})}
+                "tacker_slice_literal": (tk.POLICY_TACKER, {"slice_be": True, "reorder_only_unfused": True}),
+                "tacker_older": (tk.POLICY_TACKER, {"fuse_older": True}),   # reading 18 (the bench headline)
+                "baymax_older": (tk.POLICY_BAYMAX, {"fuse_older": True})}   # Baymax with the same queueing rule
     for name in args.variants.split(","):
         pol, kw = variants[name]
         if args.slice_ratio > 0 and kw.get("slice_be"):
@@ -79,7 +83,9 @@ def main():
             res[name]["improvement_eq10_normalised"] = res[name]["be_norm_thpt"] / res["baymax"]["be_norm_thpt"] - 1.0
     res["slice_lr"] = {f"{a}.{j}": v for (a, j), v in q.lr_be.items()}
     res["pairs_fitted"] = len(q.pairs)
-    res["pair_pred_err"] = {"max": max(q.pair_err), "mean": sum(q.pair_err) / len(q.pair_err), "n": len(q.pair_err)}
+    res["pair_pred_err"] = ({"max": max(q.pair_err), "mean": sum(q.pair_err) / len(q.pair_err), "n": len(q.pair_err)}
+                            if q.pair_err else None)
+    res["config"] = {"service": svc.name, "be": args.be, "queries": args.queries, "load": args.load, "qos_ms": args.qos}
     print(json.dumps(res))
 
 
