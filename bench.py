@@ -393,6 +393,8 @@ def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "ta
     kw = {"tacker": (tk.POLICY_TACKER, dict(HEADLINE)), "baymax": (tk.POLICY_BAYMAX, {}),
           "tacker_paper": (tk.POLICY_TACKER, {}),
           "baymax_older": (tk.POLICY_BAYMAX, dict(HEADLINE)),
+          "tacker_fuse_first": (tk.POLICY_TACKER, dict(HEADLINE, reorder_only_unfused=True)),
+          "tacker_slice_ff": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True, reorder_only_unfused=True)),
           "tacker_slice": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True)),
           "tacker_no_reverse": (tk.POLICY_TACKER, dict(HEADLINE, reverse_fusion=False))}
     for v in variants:
@@ -478,7 +480,8 @@ def run_tacker(args, ws, rank, local):
 
     # ---- Baymax (Eq. 10) and PTB-sliced Tacker on the same trace
     other = managed_runs(q, tk, args.steps, 2000 + rank, args.inflight,
-                         ("baymax", "tacker_slice", "tacker_paper", "baymax_older"))
+                         ("baymax", "tacker_slice", "tacker_paper", "baymax_older", "tacker_fuse_first",
+                          "tacker_slice_ff"))
     bay, slc, old, bay18 = other["baymax"], other["tacker_slice"], other["tacker_paper"], other["baymax_older"]
 
     # ---- e2e: the same managed run, each query with its H2D input + D2H result
@@ -590,6 +593,11 @@ def run_tacker(args, ws, rank, local):
         "baymax_same_rule": {"value": bay18["be_kernels_per_s"], "be_norm_thpt": bay18["be_norm_thpt"],
                              "lc_p99_ms": bay18["lc_p99_ms"], "qos_met": bay18["qos_met"]},
         "improvement_vs_baymax_same_rule_eq10": res["be_kernels_per_s"] / bay18["be_kernels_per_s"] - 1.0,
+        # reorder only after LC kernels that were not fused (the literal P:2035 rule) on top of reading 18
+        "tacker_fuse_first": {k: other["tacker_fuse_first"][k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms",
+                                                                         "qos_met", "fused", "reordered")},
+        "tacker_slice_ff": {k: other["tacker_slice_ff"][k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms",
+                                                                     "qos_met", "fused", "reordered")},
         "improvement_vs_baymax_same_rule_eq10_normalised": res["be_norm_thpt"] / bay18["be_norm_thpt"] - 1.0,
         # the paper-literal manager rule: only the newest query fuses / reorders
         "tacker_paper": {"value": old["be_kernels_per_s"], "be_norm_thpt": old["be_norm_thpt"],

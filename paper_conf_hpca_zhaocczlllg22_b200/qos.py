@@ -56,6 +56,12 @@ def _time(fn, reps=10, stream=None, inner=8):
     return statistics.median(ts)
 
 
+# Training ratios of the two-stage model: the paper's {0.1, 0.2, 1.8, 1.9} with the
+# middle of the range sampled too (0.6, 1.0: the PTB slices the manager fuses sit near r* ~ 1) and
+# the last point at the whole kernel (training_prefixes) -- DESIGN.md §2 reading 5.
+TRAIN_RATIOS = (0.1, 0.2, 0.6, 1.0, 1.8, 1.9)
+
+
 def _interp_n(curve, t_target, full):
     """Smallest block count whose standalone time reaches t_target, by linear interpolation of the
     measured (blocks, ms) curve (the BE time is not linear near its one-block latency floor)."""
@@ -68,44 +74,41 @@ def _interp_n(curve, t_target, full):
     return full
 
 
-def training_prefixes(prefix, full, x_tc, curve, time_fn, ratios=(0.1, 0.2, 1.8, 1.9), min_gap=0.08,
+def training_prefixes(prefix, full, x_tc, curve, time_fn, ratios=TRAIN_RATIOS, min_gap=0.08,
                       stage2_to_full=True):
-    """BE block prefixes for the two-stage model's training ratios, realised on the
-    MEASURED BE time: each target r gives the block count whose interpolated standalone time is
-    r X_tc.  Below the one-block floor the targets shift up (as the sweep does); above what the
-    whole kernel reaches the stage-2 pair becomes the whole kernel and a prefix 0.15 below it.
-    The two points of a stage are kept at least min_gap apart in measured r (two prefixes on the
-    latency floor, or a clamp, would otherwise give a degenerate stage line).  stage2_to_full: the
-    second stage-2 sample is the whole kernel (its ratio is the one the manager predicts; 1.8 and
-    1.9 alone left the stage-2 slope to measurement noise over 0.1 of r, extrapolated up to r ~ 18).
+    """BE block prefixes for the two-stage model's training ratios, realised on the MEASURED BE
+    time: each target r gives the block count whose interpolated standalone time is r X_tc.
+    Below the one-block floor the targets shift up (as the sweep does); stage2_to_full: the last
+    sample is the whole kernel (the ratio the manager predicts for whole-kernel fusion); targets
+    beyond what the whole kernel reaches fold onto it.  Consecutive samples are kept at least
+    min_gap apart in measured r (prefixes on the latency floor, or a clamp, would otherwise give
+    coincident points); if fewer than three targets are reachable the samples spread evenly over
+    [lowest target, r_full].
     prefix(n) -> descriptor, time_fn(desc) -> ms, curve = [(blocks, ms)] incl. 1 and full.
-    Returns [(n, x_cd)] (four samples; fewer when the kernel has fewer distinct prefixes)."""
+    Returns [(n, x_cd)] (fewer than len(ratios) when the kernel has fewer distinct prefixes)."""
     pts = sorted(curve)
     r_floor, r_full = pts[0][1] / x_tc, pts[-1][1] / x_tc
     shift = max(0.0, 1.25 * r_floor - ratios[0])
     tr = [r + shift for r in ratios]
-    if stage2_to_full and r_full > tr[2] + min_gap:
-        tr[3] = r_full               # reading 5: stage 2 spans up to the whole kernel's ratio
-    if tr[3] > r_full:
-        tr[3] = r_full
-        tr[2] = max(min(tr[2], r_full - 0.15), tr[1] + min_gap)
-    if tr[2] >= r_full:
-        # the whole BE kernel is short next to this LC kernel: no stage-2 ratio is reachable with
-        # BE prefixes, so the samples spread evenly over what is, [r_floor-ish, r_full]
+    if stage2_to_full and r_full > tr[-2] + min_gap:
+        tr[-1] = r_full
+    if sum(1 for r in tr if r < r_full) < 3:
         lo = min(tr[0], r_full)
-        tr = [lo + (r_full - lo) * i / 3 for i in range(4)]
+        tr = [lo + (r_full - lo) * i / (len(ratios) - 1) for i in range(len(ratios))]
+        min_gap = min(min_gap, 0.5 * (r_full - lo) / (len(ratios) - 1))
     out = []
-    for i, r in enumerate(tr):
+    for r in tr:
         n = _interp_n(pts, r * x_tc, full) if r < r_full else full
         if out and n <= out[-1][0]:
             if out[-1][0] >= full:
-                break                    # fewer distinct samples than four
+                break                    # fewer distinct samples than targets
             n = min(full, out[-1][0] + 1)
         x = time_fn(prefix(n))
-        if i in (1, 3):
-            while (x - out[-1][1]) / x_tc < min_gap and n < full:
-                n = min(full, max(n + 1, int(n * 1.5)))
-                x = time_fn(prefix(n))
+        while out and (x - out[-1][1]) / x_tc < min_gap and n < full:
+            n = min(full, max(n + 1, int(n * 1.5)))
+            x = time_fn(prefix(n))
+        if out and n == out[-1][0]:
+            break
         out.append((n, x))
     return out
 
