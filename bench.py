@@ -395,6 +395,7 @@ def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "ta
           "baymax_older": (tk.POLICY_BAYMAX, dict(HEADLINE)),
           "tacker_fuse_first": (tk.POLICY_TACKER, dict(HEADLINE, reorder_only_unfused=True)),
           "tacker_slice_ff": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True, reorder_only_unfused=True)),
+          "tacker_slice_noreorder": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True, reorder_only_unfused=2)),
           "tacker_slice": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True)),
           "tacker_no_reverse": (tk.POLICY_TACKER, dict(HEADLINE, reverse_fusion=False))}
     for v in variants:
@@ -481,7 +482,7 @@ def run_tacker(args, ws, rank, local):
     # ---- Baymax (Eq. 10) and PTB-sliced Tacker on the same trace
     other = managed_runs(q, tk, args.steps, 2000 + rank, args.inflight,
                          ("baymax", "tacker_slice", "tacker_paper", "baymax_older", "tacker_fuse_first",
-                          "tacker_slice_ff"))
+                          "tacker_slice_ff", "tacker_slice_noreorder"))
     bay, slc, old, bay18 = other["baymax"], other["tacker_slice"], other["tacker_paper"], other["baymax_older"]
 
     # ---- e2e: the same managed run, each query with its H2D input + D2H result
@@ -598,6 +599,9 @@ def run_tacker(args, ws, rank, local):
                                                                          "qos_met", "fused", "reordered")},
         "tacker_slice_ff": {k: other["tacker_slice_ff"][k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms",
                                                                      "qos_met", "fused", "reordered")},
+        "tacker_slice_noreorder": {k: other["tacker_slice_noreorder"][k] for k in ("be_kernels_per_s", "be_norm_thpt",
+                                                                                   "lc_p99_ms", "qos_met", "fused",
+                                                                                   "reordered", "idle_be")},
         "improvement_vs_baymax_same_rule_eq10_normalised": res["be_norm_thpt"] / bay18["be_norm_thpt"] - 1.0,
         # the paper-literal manager rule: only the newest query fuses / reorders
         "tacker_paper": {"value": old["be_kernels_per_s"], "be_norm_thpt": old["be_norm_thpt"],

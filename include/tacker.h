@@ -421,7 +421,7 @@ typedef struct {
   double slice_ratio;
   /* 0 (default): after every LC kernel, fused or not, reorder the other ready BE heads with
    * Ttmp < Thr (reading 6); 1: reorder only after an LC kernel that was not fused. */
-  int32_t reorder_only_unfused;
+  int32_t reorder_only_unfused;   /* 2: never reorder (BE work only fused or on an idle GPU) */
   /* 1: never fuse an LC CUDA-core kernel with a BE tensor-core kernel (NEXT-2 off) */
   int32_t no_reverse_fusion;
   /* B200 reading 18 (off = the paper's rule: only the newest query fuses / reorders):

@@ -32,7 +32,8 @@ Rules, in the paper's order:
     its last block is issued; reorder and idle launches issue the whole rest, whose predicted
     time is X_cd(remaining) once a slice of it has run.  BE work = n/N of the kernel's
     standalone time per slice.
-  * reorder_only_unfused: reorder only after an LC kernel that was not fused (P:2035 literally).
+  * reorder_only_unfused: 1 = reorder only after an LC kernel that was not fused (P:2035
+    literally); 2 = never reorder (BE work runs fused or on an idle GPU only).
   * Reverse fusion (NEXT-2; "LC and BE kernels are not limited to a specified type",
     P:924-926; DNN-training BE apps, Table II): when the LC kernel is a CUDA-core
     kernel (T_lc) and a ready BE head is a tensor-core kernel (T_be; kind 2 below), the same
@@ -112,7 +113,7 @@ def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=No
     reorder = []
     if fused >= 0:
         thr -= tf_best - ttc
-    if allow and not (reorder_only_unfused and fused >= 0):
+    if allow and reorder_only_unfused != 2 and not (reorder_only_unfused == 1 and fused >= 0):
         for app, tcd, _ in heads:
             if app == fused:
                 continue

@@ -655,7 +655,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   // Reorder the remaining ready heads after the LC kernel, fused or not (reading:
   // Tacker = fusion on top of Baymax's reordering, "both adaptive kernel fusion and kernel
   // reorder"); reorder_only_unfused = the literal P:2035 rule.
-  if (allow && !(m->prm.reorder_only_unfused && fused >= 0)) {
+  if (allow && m->prm.reorder_only_unfused != 2 && !(m->prm.reorder_only_unfused == 1 && fused >= 0)) {
     for (int a : heads) {
       if (a == fused) continue;
       const double tt = rem_ms(m->apps[a]);

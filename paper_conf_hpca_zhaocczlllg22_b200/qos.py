@@ -414,7 +414,7 @@ class QosRun:
         lat_sorted = np.sort(lat)
         p99 = float(lat_sorted[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)])
         return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "slice_be": bool(slice_be),
-                "reorder_only_unfused": bool(reorder_only_unfused), "queries": int(len(lat)),
+                "reorder_only_unfused": int(reorder_only_unfused), "queries": int(len(lat)),
                 "lambda_per_s": lam * 1e3, "load": load, "elapsed_ms": gpu_ms,
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
                 # normalised BE throughput: standalone-milliseconds of BE work per wall millisecond

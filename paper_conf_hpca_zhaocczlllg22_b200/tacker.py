@@ -664,7 +664,7 @@ class Manager:
                  fuse_older=False, older_margin_ms=0.0):
         self.h = C.c_void_p()
         self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0,
-                                    1 if slice_be else 0, slice_ratio, 1 if reorder_only_unfused else 0,
+                                    1 if slice_be else 0, slice_ratio, int(reorder_only_unfused),
                                     0 if reverse_fusion else 1, 1 if fuse_older else 0, older_margin_ms)
         _chk(_lib.tacker_manager_create(policy, C.byref(self.params), _stream(stream), C.byref(self.h)))
         self._keep = []

@@ -194,7 +194,7 @@ def fit_pair_closed_form(tk, tau):
     return key
 
 
-@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse", "tacker_older"])
+@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse", "tacker_older", "tacker_noreorder"])
 def test_manager_simulation_matches_reference(tk, policy):
     tk.tacker_model_clear()
     # stage-2 slope != 1 so that Tgain depends on Tcd (with slope 1 every stage-2 pair has the
@@ -214,10 +214,12 @@ def test_manager_simulation_matches_reference(tk, policy):
     app_ts = [[1.53, 0.71], [3.07], [0.43, 0.37, 2.51]]
     tc_apps = [[0.47, 1.12], [0.81]] if reverse else []
     pol = tk.POLICY_BAYMAX if policy == "baymax" else tk.POLICY_TACKER
-    older = policy == "tacker_older"
+    older = policy in ("tacker_older", "tacker_noreorder")
+    noreorder = 2 if policy == "tacker_noreorder" else 0
     if older:   # a denser trace so that queries queue behind each other
         arrivals = np.cumsum(rng.exponential(3.3, 60))
-    m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0, fuse_older=older, older_margin_ms=0.7 if older else 0.0)
+    m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0, fuse_older=older, older_margin_ms=0.7 if older else 0.0,
+                   reorder_only_unfused=noreorder)
     qs = []
     for i, t in enumerate(arrivals):
         sh = shapes[i % 2]
@@ -231,8 +233,11 @@ def test_manager_simulation_matches_reference(tk, policy):
         m.submit_be([be_kernel_tc(tk, d) for d in ts])
         apps.append(mr.App([(mr.BE_TC, d) for d in ts]))
     ref = mr.simulate(qs, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER, fuse_pred, idle_cap=2.0,
-                      rfuse_pred=rfuse_pred, fuse_older=older, older_margin=0.7 if older else 0.0)
-    if older:   # older queries did fuse, which the paper-literal rule forbids
+                      rfuse_pred=rfuse_pred, fuse_older=older, older_margin=0.7 if older else 0.0,
+                      reorder_only_unfused=noreorder)
+    if noreorder:
+        assert all(not x.reorder for x in ref["decisions"] if x.action != mr.IDLE_BE)
+    if older and not noreorder:   # older queries did fuse, which the paper-literal rule forbids
         lit = mr.simulate([mr.Query(q.qid, q.arrival, list(q.kernels)) for q in qs],
                           [mr.App(list(a.kernels)) for a in apps], 50.0, mr.TACKER, fuse_pred, idle_cap=2.0,
                           rfuse_pred=rfuse_pred)
