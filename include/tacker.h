@@ -342,7 +342,9 @@ tacker_status tacker_predict_duration(tacker_fused_t f, double *ms_out);
  * QoS-aware kernel manager (§VII).  Rules: Eq. 9 headroom at the first issue of
  * the newest query; per TC kernel Eq. 8 admission over ready BE heads, max Tgain, then
  * Thr -= Tk_fuse - Ttc; otherwise original launch and reorder of ready BE heads with
- * Ttmp < Thr.  Only the newest query fuses/reorders; Baymax policy = fusion disabled.
+ * Ttmp < Thr.  Only the newest query fuses/reorders (params.fuse_older relaxes it, reading 18);
+ * CUDA-core LC kernels may fuse with BE tensor-core kernels (NEXT-2, reading 17); Baymax policy =
+ * fusion disabled.
  * The manager keeps its own clock: in simulation mode (stream == NULL and simulate != 0)
  * kernels take their predicted duration; otherwise launches go to `stream` and completions
  * are observed with CUDA events.

@@ -4,11 +4,15 @@
 //   * Eq. 9: at the first issue of the newest query Q,
 //       Thr = T_qos - T_queue - T_ori_solo(Q) - sum_i T_lc_i(remaining, earlier queries),
 //     T_queue = issue time - arrival (reading).  Thr <= direct_eps -> Q runs direct.
-//   * Only the newest query fuses/reorders.
+//   * Only the newest query fuses/reorders; params.fuse_older (reading 18): an older
+//     query too, within min(its Thr, Eq. 9 of every later active query) - older_margin_ms.
+//   * CUDA-core LC kernel (NEXT-2, reading 17): the same Eq. 8 over ready BE tensor-core heads,
+//     the pair model evaluated with X_tc = the BE kernel, X_cd = the LC kernel.
 //   * TC kernel: Eq. 8 over the ready BE heads with a fitted pair model:
 //       Ttc + Tcd > Tk_fuse  &&  Tk_fuse - Ttc < Thr;  max Tgain = Tcd - (Tk_fuse - Ttc)
 //     (P:2045-2056), ties -> lowest app index; Thr -= Tk_fuse - Ttc.
-//   * No fusion: original launch, then reorder ready BE heads with Ttmp < Thr.
+//   * Original launch (if not fused), then reorder ready BE heads with Ttmp < Thr:
+//     after every LC kernel (reading 6), only unfused ones (reorder_only_unfused 1) or never (2).
 //   * Baymax policy: identical with fusion disabled ("static scheduling").
 //   * Idle GPU (paper silent): one ready BE head no longer than idle_cap.
 //   * PTB slicing (params.slice_be, reading 13): a fused launch may carry only a slice of the BE
