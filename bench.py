@@ -366,6 +366,8 @@ def run_reference(args, ws, rank):
     """--impl reference: the CPU oracle as it stands is this tier's reference arm."""
     if rank != 0:
         return
+    for _ in range(min(args.warmup, 3)):    # untimed warm-up steps (bounded)
+        cpu_oracle_sample(small=True, batch=args.batch)
     # bounded: each step is a small sample (~0.3 s); at most 120 s of steps
     t0 = time.perf_counter()
     vals, r = [], None
