@@ -78,3 +78,34 @@ def test_managed_reverse_fusion_outputs_match_standalone(tk):
     res = run.run(tk.POLICY_TACKER, 40, load=0.8)
     assert res["reverse_fused"] > 0, res
     assert host(svc.outputs[-1]).tobytes() == ref
+
+
+@pytest.mark.parametrize("variant", [dict(fuse_older=True), dict(fuse_older=True, slice_be=True, reorder_only_unfused=2)])
+def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
+    """GPU-mode managed runs with reading 18 (older queries fuse) and with PTB slices and no
+    reorder: every LC query's output bytes equal a standalone query's, QoS holds, kernels fused."""
+    from paper_conf_hpca_zhaocczlllg22_b200 import qos, services as sv
+    convs = [c for c in synth.resnet50_convs(8) if c.name in ("layer1.0.conv1", "layer1.0.conv2", "layer1.0.conv3")]
+    svc = sv.resnet50_service(8, convs=convs)
+    st, mq = sv.stencil_app(512, 512, 64), sv.mriq_app(64, 1024, 1024)   # >= 10 us: fusable kernels
+    tk.tacker_launch_original(None, mq.kernels[0].desc)
+    for k in svc.kernels:
+        tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd)
+    ref = host(svc.outputs[-1]).tobytes()
+    tk.tacker_model_clear()
+    run = qos.QosRun(svc, [st, mq], warp_split=16)
+    run.calibrate(reps=3, pair_reps=3)
+    run.measure_service(n=20)
+    assert run.pairs, "no fusable pair calibrated"
+    # the launch paths under test must run whatever this box measured: pair models with a sure
+    # gain (tau = max(1 + 0.1 r, 0.5 + r), opportune ratio 5/9)
+    tk.tacker_model_clear()
+    for pk in run.pairs:
+        for r in (0.1, 0.2, 1.8, 1.9):
+            tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0 + 0.1 * r, 0.5 + r))
+        tk.tacker_pair_fit(pk)
+    svc.outputs[-1].zero_()
+    res = run.run(tk.POLICY_TACKER, 60, load=0.8, max_inflight=8, **variant)
+    assert res["qos_met"], res
+    assert res["fused"] > 0, res
+    assert host(svc.outputs[-1]).tobytes() == ref
