@@ -448,6 +448,7 @@ def run_tacker(args, ws, rank, local):
     peaks, peak_kind = measured_peaks()
     seed = 2022 + rank
     svc = sv.resnet50_service(args.batch, seed)
+    sv.autotune_tile_n(svc)                                      # LC tile width per conv, measured
     stencil = sv.stencil_app(512, 512, 64, seed)
     mriq = sv.mriq_app(64, 2048, 1024, seed)
     tk.tacker_launch_original(None, mriq.kernels[0].desc)       # phiMag ready for the Q chunks
@@ -534,6 +535,7 @@ def run_tacker(args, ws, rank, local):
     # ---- BASELINE configs[1]: ResNet-50 batch-1 convs fused with stencil / mri-q -- the kernel-
     #      level fused step (fused time vs overlap roofline) and the same managed protocol
     svc1 = sv.resnet50_service(1, seed)
+    sv.autotune_tile_n(svc1)
     step = FusedStep(svc1, stencil, mriq, args.warp_split)
     for _ in range(3):
         step.fused()

@@ -42,9 +42,12 @@ def main():
     ap.add_argument("--service", default="resnet50")
     ap.add_argument("--batch", type=int, default=1)
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--autotune", action="store_true", help="measured LC tile width per conv (services.autotune_tile_n)")
     args = ap.parse_args()
     svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
-    res = {"service": svc.name, "kernels": len(svc.kernels)}
+    if args.autotune:
+        sv.autotune_tile_n(svc)
+    res = {"service": svc.name, "kernels": len(svc.kernels), "autotune": bool(args.autotune)}
     for on in (False, True):
         tk.tacker_set_launch_overlap(on)
         res["overlap" if on else "serial"] = {"query_ms": timed(lambda: query(svc), args.reps)}
