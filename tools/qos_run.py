@@ -57,8 +57,11 @@ def main():
     ap.add_argument("--inflight", type=int, default=4)
     ap.add_argument("--variants", default="baymax,tacker,tacker_slice,tacker_slice_literal")
     ap.add_argument("--slice-ratio", type=float, default=0.0, help="fixed slice load ratio (0: opportune r*)")
+    ap.add_argument("--autotune", action="store_true", help="measured LC tile width per conv (as the bench)")
     args = ap.parse_args()
     svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
+    if args.autotune:
+        sv.autotune_tile_n(svc)
     apps = build_apps(args.be.split(","))
     tk.tacker_model_clear()
     q = qos.QosRun(svc, apps, warp_split=args.ws, qos_ms=args.qos)
