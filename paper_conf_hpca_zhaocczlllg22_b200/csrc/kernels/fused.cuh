@@ -41,6 +41,8 @@ struct LcParams {
   int32_t tp, tq;          // output tile = tp x tq positions (tp*tq == 128)
   int32_t tiles_p, tiles_q, c_blocks;
   int32_t conv_direct_gemm;  // 1x1 stride-1 conv handled as a plain GEMM over [n*h*w, c]
+  int32_t conv_c8;           // im2col mode with C = 8 channels (conv1): a k-block = 8 filter taps of
+                             // 16 B, loaded as 8 unswizzled 128 x 16 B boxes (K-major, no swizzle)
   int32_t conv_im2col;       // implicit conv through the TMA im2col mode: M-tile = 128 consecutive
                              // output pixels (n, p, q linear); else tp x tq windows of one image
   // split-K: work unit u = (tile u / splits, k-blocks [s kb_per_split, (s+1) kb_per_split) of split
@@ -156,7 +158,9 @@ struct LcGemm {
   // B (weights) k-block kb of N-tile nt
   static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
     const LcParams &L = P.lc;
-    if (implicit_conv(L)) {
+    if (implicit_conv(L) && L.conv_c8) {
+      tma_load_2d(&P.tmap_b, bar, sb, kb * kBK, nt * BN);   // K = R*S*8 linear (OOB tail zero-filled)
+    } else if (implicit_conv(L)) {
       // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
       const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
       tma_load_2d(&P.tmap_b, bar, sb, rs * L.c + cb * kBK, nt * BN);
@@ -167,7 +171,21 @@ struct LcGemm {
   // A (activations) k-block kb of M-tile mt
   static __device__ __forceinline__ void load_a(const FusedParams &P, uint64_t *bar, uint8_t *sa, int kb, int mt) {
     const LcParams &L = P.lc;
-    if (implicit_conv(L) && L.conv_im2col) {
+    if (implicit_conv(L) && L.conv_c8) {
+      // k-block kb = filter taps 8 kb .. 8 kb + 7 (K index = tap * 8 + c); tap t lands at sa + 2 KB t
+      // as 128 pixel rows of 16 B; taps past R*S reload tap 0 (their weights are the zero padding)
+      const int pq = L.p * L.q, m0 = mt * kBM;
+      const int n0 = m0 / pq, rem = m0 - n0 * pq;
+      const int p0 = rem / L.q, q0 = rem - p0 * L.q;
+      const int taps = L.r * L.s;
+#pragma unroll 1
+      for (int t = 0; t < 8; ++t) {
+        int tap = kb * 8 + t;
+        if (tap >= taps) tap = 0;
+        tma_load_im2col_4d(&P.tmap_a, bar, sa + t * kBM * 16, 0, q0 * L.stride - L.pad, p0 * L.stride - L.pad, n0,
+                           (uint16_t)(tap % L.s), (uint16_t)(tap / L.s));
+      }
+    } else if (implicit_conv(L) && L.conv_im2col) {
       // k-block -> (filter tap r,s ; channel block cb); A = 128 output pixels from m0 = 128 mt,
       // first pixel (n0, p0, q0) -> input corner (q0 stride - pad, p0 stride - pad), tap offset (s, r)
       const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
@@ -247,10 +265,17 @@ struct LcGemm {
         tc_fence_after();
         const uint32_t sa = smem_u32(lc + stage * kStage);
         const uint32_t sb = sa + kStageA;
+        if (L.conv_c8) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
 #pragma unroll
-        for (int k = 0; k < kBK / kUK; ++k) {
-          umma_f16(d, umma_desc_sw128(sa + k * kUK * 2), umma_desc_sw128(sb + k * kUK * 2), kIdesc,
-                   (kb != kb0 || k != 0));
+          for (int k = 0; k < kBK / kUK; ++k)
+            umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
+                     umma_desc_sw128(sb + k * kUK * 2), kIdesc, (kb != kb0 || k != 0));
+        } else {
+#pragma unroll
+          for (int k = 0; k < kBK / kUK; ++k) {
+            umma_f16(d, umma_desc_sw128(sa + k * kUK * 2), umma_desc_sw128(sb + k * kUK * 2), kIdesc,
+                     (kb != kb0 || k != 0));
+          }
         }
         umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
         if (++stage == P.stages) {

@@ -205,6 +205,16 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t smem_addr) {
   d |= (uint64_t)2 << 61;                              // SWIZZLE_128B    [61,64)
   return d;
 }
+// K-major operand without swizzle (core matrices of 8 rows x 16 B): rows 16 B apart inside a core
+// matrix, SBO between 8-row groups, LBO between the two 8-element K halves of an MMA's K = 16.
+__device__ __forceinline__ uint64_t umma_desc_kmajor_noswz(uint32_t smem_addr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr & 0x3FFFF) >> 4);        // start address  [0,14)
+  d |= (uint64_t)((lbo & 0x3FFFF) >> 4) << 16;         // LBO             [16,30)
+  d |= (uint64_t)((sbo & 0x3FFFF) >> 4) << 32;         // SBO             [32,46)
+  d |= (uint64_t)1 << 46;                              // version = 1     [46,48)
+  return d;                                            // SWIZZLE_NONE    [61,64) = 0
+}
 // Instruction descriptor, kind::f16: D fp32, A/B fp16, both K-major, shape M x N.
 __host__ __device__ constexpr uint32_t umma_idesc_f16(uint32_t M, uint32_t N) {
   return (1u << 4)                 // c_format = F32

@@ -268,8 +268,8 @@ static tacker_status lc_view(const tacker_lc_desc &d, LcParams &L) {
     L.N = d.k;
     L.K = d.c * d.r * d.s;
     L.conv_direct_gemm = (d.r == 1 && d.s == 1 && d.stride == 1 && d.pad == 0);
-    if (!L.conv_direct_gemm && d.c % 64 != 0)
-      return set_error("conv: C must be a multiple of 64 for implicit GEMM (got %d)", d.c), TACKER_EUNSUPPORTED;
+    if (!L.conv_direct_gemm && d.c % 64 != 0 && d.c != 8)
+      return set_error("conv: C must be a multiple of 64 (or 8) for implicit GEMM (got %d)", d.c), TACKER_EUNSUPPORTED;
   } else {
     return set_error("LC kind %d not supported", d.kind), TACKER_EUNSUPPORTED;
   }
@@ -317,7 +317,13 @@ static bool conv_im2col_mode() {
 
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
-  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && conv_im2col_mode()) {
+  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && L.c == 8) {
+    L.conv_im2col = 1;               // C = 8 (conv1 padded): 8 taps per k-block
+    L.conv_c8 = 1;
+    L.tiles_m = (L.M + kBM - 1) / kBM;
+    L.c_blocks = 1;
+    L.num_kb = (L.r * L.s + 7) / 8;
+  } else if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && conv_im2col_mode()) {
     L.conv_im2col = 1;
     L.tiles_m = (L.M + kBM - 1) / kBM;
     L.c_blocks = L.c / kBK;
@@ -423,7 +429,7 @@ static PFN_encodeIm2col get_encode_im2col() {
 // image is [-pad, W - 1 + pad - (S - 1)] x [-pad, H - 1 + pad - (R - 1)] walked with the conv
 // stride, i.e. exactly the P x Q output positions; 64 channels (128 B, SW128) per pixel, 128
 // pixels per load.
-static tacker_status encode_conv_im2col(CUtensorMap *m, const tacker_lc_desc &d) {
+static tacker_status encode_conv_im2col(CUtensorMap *m, const tacker_lc_desc &d, bool c8 = false) {
   auto enc = get_encode_im2col();
   if (!enc) return set_error("cuTensorMapEncodeIm2col unavailable"), TACKER_ECUDA;
   if (d.pad > 127 || d.pad - (d.s - 1) < -128 || d.pad - (d.r - 1) < -128 || d.r > 256 || d.s > 256)
@@ -434,8 +440,9 @@ static tacker_status encode_conv_im2col(CUtensorMap *m, const tacker_lc_desc &d)
   int upper[2] = {d.pad - (d.s - 1), d.pad - (d.r - 1)};
   cuuint32_t es[4] = {1, (cuuint32_t)d.stride, (cuuint32_t)d.stride, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void *>(d.A), dims, strides, lower, upper,
-                   (cuuint32_t)kBK, (cuuint32_t)kBM, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   c8 ? 8u : (cuuint32_t)kBK, (cuuint32_t)kBM, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   c8 ? CU_TENSOR_MAP_SWIZZLE_NONE : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeIm2col(conv x) failed: %d", (int)r), TACKER_ECUDA;
   // driver <= 13.1 with a tensor under 128 KiB: clear descriptor bit 85 (as CUTLASS does)
   int drv = 0;
@@ -624,7 +631,8 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
 
   // TMA tensor maps
   if (lc->kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-    if ((st = L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc) : encode_conv_x(&F.P.tmap_a, *lc, L))) return st;
+    if ((st = L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc, L.conv_c8 != 0) : encode_conv_x(&F.P.tmap_a, *lc, L)))
+      return st;
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   } else {
     if ((st = encode_2d(&F.P.tmap_a, lc->A, (uint64_t)L.K, (uint64_t)L.M, kBK, kBM))) return st;

@@ -53,7 +53,11 @@ def _dev(a, dtype=None):
     return t.cuda()
 
 
-def resnet50_service(batch: int = 1, seed: int = 2022, convs=None) -> LcService:
+def resnet50_service(batch: int = 1, seed: int = 2022, convs=None, conv1_im2col: bool = True) -> LcService:
+    """conv1 (C = 3 padded to 8): the paper's explicit im2col (an LC CUDA-core kernel, §VIII-H
+    P:3350-3381) + GEMM by default; conv1_im2col=False runs it as one implicit GEMM over 8-tap
+    k-blocks (TMA im2col mode, unswizzled A) -- correct, but measured no faster at b32 (189 us vs
+    130 + 66 us: eight 2 KB TMA loads per k-block)."""
     convs = convs if convs is not None else synth.resnet50_convs(batch)
     ks, bufs, ins, outs = [], [], [], []
     for i, cs in enumerate(convs):
@@ -64,7 +68,7 @@ def resnet50_service(batch: int = 1, seed: int = 2022, convs=None) -> LcService:
         outs.append(out)
         M, N, K = cs.gemm_mnk
         byt = 2 * x.size + 2 * w.size + 2 * out.numel()
-        if cs.c % 64 == 0 or (cs.r == 1 and cs.s == 1 and cs.stride == 1):
+        if cs.c % 64 == 0 or (cs.r == 1 and cs.s == 1 and cs.stride == 1) or (cs.c == 8 and not conv1_im2col):
             lc = tk.lc_conv(dx, dw, out, cs.stride, cs.pad, bias=db, relu=True, b_const=True)
             ks.append(LcKernelSpec(cs.name, True, lc=lc,
                                    flops=2 * M * N * K, bytes=byt, conv=cs))

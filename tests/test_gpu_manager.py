@@ -50,7 +50,7 @@ def test_managed_reverse_fusion_outputs_match_standalone(tk):
     # LC service = ResNet-50 conv1 at batch 32 (im2col on the CUDA cores + GEMM) and the next conv;
     # BE queue = one tensor-core training GEMM app (tools/reverse_pair.py: this pair overlaps)
     convs = synth.resnet50_convs(32)[:2]
-    svc = sv.resnet50_service(32, convs=convs)
+    svc = sv.resnet50_service(32, convs=convs, conv1_im2col=True)
     app = sv.gemm_train_app(4096, 4096, 4096, n=1)
     # reference bytes: one standalone query
     for k in svc.kernels:

@@ -60,12 +60,13 @@ CONV_CASES = [synth.ConvShape("3x3s1", 1, 14, 14, 64, 64, 3, 3, 1, 1),
               synth.ConvShape("1x1s1", 1, 28, 28, 256, 128, 1, 1, 1, 0),
               synth.ConvShape("1x1s2", 1, 56, 56, 64, 256, 1, 1, 2, 0),
               synth.ConvShape("7x7", 1, 7, 7, 512, 512, 3, 3, 1, 1),
-              synth.ConvShape("b2", 2, 9, 11, 64, 72, 3, 3, 1, 1)]
+              synth.ConvShape("b2", 2, 9, 11, 64, 72, 3, 3, 1, 1),
+              synth.ConvShape("c8_conv1", 2, 30, 28, 8, 64, 7, 7, 2, 3)]   # 8-tap k-blocks, unswizzled A
 
 
 @pytest.mark.parametrize("cs", CONV_CASES, ids=lambda c: c.name)
 def test_lc_conv_vs_oracle(tk, cs):
-    x, w, b = synth.conv_inputs(cs, seed=3)
+    x, w, b = synth.conv_inputs(cs, seed=3, real_c=3 if cs.c == 8 else None)
     out = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
     tk.tacker_launch_original(tk.lc_conv(t(x), t(w), out, cs.stride, cs.pad, bias=t(b), relu=True), None)
     ref, S = olc.lc_conv(x, w, cs.stride, cs.pad, bias=b, relu=True)

@@ -34,7 +34,7 @@ def main():
         fh, cp, ff, tp = sv.mrifhd_app(), sv.cp_app(), sv.fft_app(), sv.tpacf_app()
         tk.tacker_launch_original(None, fh.kernels[0].desc)
         train = sv.gemm_train_app(4096, 4096, 4096, n=1)
-        c1 = sv.resnet50_service(32, convs=synth.resnet50_convs(32)[:1])
+        c1 = sv.resnet50_service(32, convs=synth.resnet50_convs(32)[:1], conv1_im2col=True)
         extra = [tk.tacker_fuse(k1.lc, fh.kernels[1].desc, 24), tk.tacker_fuse(k1.lc, cp.kernels[0].desc, 24),
                  tk.tacker_fuse(k1.lc, ff.kernels[0].desc, 24), tk.tacker_fuse(k1.lc, tp.kernels[1].desc, 16),
                  tk.tacker_fuse(train.kernels[0].desc, c1.kernels[0].cd, 24)]

@@ -25,7 +25,7 @@ def main():
     kc = tk.be_fma_burn(out, 60000)
     f = tk.tacker_fuse(lc, kc, 24)
     train = sv.gemm_train_app(4096, 4096, 4096, n=1)
-    c1 = sv.resnet50_service(32, convs=synth.resnet50_convs(32)[:1])
+    c1 = sv.resnet50_service(32, convs=synth.resnet50_convs(32)[:1], conv1_im2col=True)
     fr = tk.tacker_fuse(train.kernels[0].desc, c1.kernels[0].cd, 24)
     torch.cuda.synchronize()
     f.launch()

@@ -26,7 +26,7 @@ def main():
     ap.add_argument("--gemm", default="4096,4096,4096;2048,2048,2048;8192,4096,1024")
     ap.add_argument("--ws", default="8,16,24")
     args = ap.parse_args()
-    svc = sv.resnet50_service(args.batch, convs=synth.resnet50_convs(args.batch)[:1])
+    svc = sv.resnet50_service(args.batch, convs=synth.resnet50_convs(args.batch)[:1], conv1_im2col=True)
     cd = svc.kernels[0].cd
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
     cur = torch.cuda.current_stream()
