@@ -156,7 +156,7 @@ typedef struct { int32_t natoms, nx, ny; float h, z; const float *atoms; float *
  * exp(-2 pi i j k / n), b < batch, complex fp32 interleaved (re, im) [batch][n][2], out of place,
  * x, y 16-byte aligned; n a power of two in [2, 1024].  twiddle [n][2] fp32 is written by
  * TACKER_BE_FFT_TWIDDLE (w[m] = (cos, -sin)(2 pi m / n), accurate sincospi) and read by
- * TACKER_BE_FFT (Stockham radix-8/4/2 in shared memory). */
+ * TACKER_BE_FFT (Stockham radix-16/8/4/2; first pass from and last pass to global memory). */
 typedef struct { int32_t n, batch; float *twiddle; const float *x; float *y; } tacker_be_fft;
 /* tpacf (Parboil; reading 16): count[bin(a_i . b_j)] += 1 over all (i, j) (self_pairs = 0) or
  * over i < j with b == a (self_pairs = 1); bin(d) = #{k : d < edges[k]}, edges strictly

@@ -20,6 +20,9 @@ constexpr int kVbThreads = 128;
 #ifndef TK_FFT_MAXN
 #define TK_FFT_MAXN 1024
 #endif
+#ifndef TK_FFT_ODD_FIRST
+#define TK_FFT_ODD_FIRST 1   // fft: the radix-2^f pass first (n = 256: 98.6 -> 90.7 us; equal at 1024)
+#endif
 #ifndef TK_FFT_MIN_BLOCKS
 #define TK_FFT_MIN_BLOCKS 12
 #endif

@@ -10,16 +10,18 @@ namespace tk {
 //
 // Twiddle table (TACKER_BE_FFT_TWIDDLE, the "plan" step, one launch per n):
 //   w[m] = (cospi(2m/n), -sinpi(2m/n)), m < n, with the accurate sincospi (not the MUFU).
-// Transform (TACKER_BE_FFT): one original block = one transform, held in shared memory (8n
-// bytes), Stockham autosort radix-8 passes (a final radix-4 or radix-2 pass), so input
-// and output are both in natural order and every global access is a coalesced 16-byte vector.
+// Transform (TACKER_BE_FFT): one original block = one transform, Stockham autosort: one
+// radix-2/4/8/16 pass, then radix-8 passes (n = 1024: 16, 8, 8), so input and output are both
+// in natural order; the first pass reads x from global memory and the last writes y to it
+// (coalesced 8-byte accesses), intermediate results sit in shared memory (8n bytes).
 // Pass with sub-transform size Ns (1, R, R^2, ...), butterfly j < n/R, k = j mod Ns:
 //   v_r = x[j + r n/R] * w[(r k n / (Ns R)) mod n],  V = DFT_R(v),
 //   out[(j / Ns) Ns R + k + r Ns] = V_r,   r < R.
 // A pass reads all its inputs into registers, synchronises, then writes in place.  The twiddles
 // of a radix-R butterfly are w, w^2, ..., w^(R-1) with w = w[k n / (Ns R)] from the table, the
 // powers formed by complex products (one table load per butterfly; a few ulp, far inside the
-// gate).  DFT_8 = two DFT_4 combined with W8^k (n = 1024: passes 8, 8, 8, 2).
+// gate; radix 16 loads w, w^4, w^8, w^12 and forms the rest with at most two products).
+// DFT_8 = two DFT_4 combined with W8^k; DFT_16 = 4 x 4 with W16^(n2 k1) between the stages.
 template <> struct BeBody<TACKER_BE_FFT_TWIDDLE> {
   static constexpr uint32_t kSmem = 0;
   static __host__ __device__ int64_t num_blocks(const tacker_be_fft &p) { return (p.n + 127) / 128; }
@@ -34,7 +36,7 @@ template <> struct BeBody<TACKER_BE_FFT_TWIDDLE> {
 };
 
 template <> struct BeBody<TACKER_BE_FFT> {
-  static constexpr int kMaxN = TK_FFT_MAXN;   // register arrays of one radix-8 butterfly per thread (1024)
+  static constexpr int kMaxN = TK_FFT_MAXN;   // register arrays of one radix-16 butterfly per thread (1024)
   // shared layout XOR-swizzled in 16-complex (128-byte) rows: index i lives at i ^ ((i >> 4) & 15).
   // Consecutive indices stay within their aligned 16-block (reads and staging conflict-free);
   // the Stockham writes of the first pass (stride 4 complex) spread over all 16 slots instead of
@@ -43,9 +45,9 @@ template <> struct BeBody<TACKER_BE_FFT> {
   static __device__ __forceinline__ int pad(int i) { return i ^ ((i >> 4) & 15); }
   static __host__ __device__ int64_t num_blocks(const tacker_be_fft &p) { return p.batch; }
 
+  // complex product, contracted to two FMUL + two FFMA (the gate is 1e-5 of the signal scale)
   static __device__ __forceinline__ float2 cmul(float2 a, float2 w) {
-    return make_float2(__fsub_rn(__fmul_rn(a.x, w.x), __fmul_rn(a.y, w.y)),
-                       __fadd_rn(__fmul_rn(a.x, w.y), __fmul_rn(a.y, w.x)));
+    return make_float2(fmaf(a.x, w.x, -(a.y * w.y)), fmaf(a.x, w.y, a.y * w.x));
   }
   static __device__ __forceinline__ float2 add(float2 a, float2 b) { return make_float2(__fadd_rn(a.x, b.x), __fadd_rn(a.y, b.y)); }
   static __device__ __forceinline__ float2 sub(float2 a, float2 b) { return make_float2(__fsub_rn(a.x, b.x), __fsub_rn(a.y, b.y)); }
@@ -61,67 +63,135 @@ template <> struct BeBody<TACKER_BE_FFT> {
     y[3] = sub(t1, t3);
   }
 
-  template <int R, int NMAX>
-  static __device__ __forceinline__ void pass(float2 *s, const float2 *tw, int n, int Ns, int tid, uint32_t bar) {
-    constexpr int kMaxBf = NMAX / R / kVbThreads;    // butterflies per thread at n = NMAX
-    const int nbf = n / R, q = n / R;
-    float2 v[kMaxBf > 0 ? kMaxBf : 1][R];
+  // W16^m = exp(-2 pi i m / 16) products used inside DFT_16 (m in {1, 2, 3, 4, 6, 9})
+  static constexpr float kC1 = 0.92387953251128674f, kS1 = 0.38268343236508978f, kH = 0.70710678118654752f;
+  static __device__ __forceinline__ float2 w16_2(float2 a) {   // (h, -h)
+    return make_float2(__fmul_rn(__fadd_rn(a.x, a.y), kH), __fmul_rn(__fsub_rn(a.y, a.x), kH));
+  }
+  static __device__ __forceinline__ float2 w16_6(float2 a) {   // (-h, -h)
+    return make_float2(__fmul_rn(__fsub_rn(a.y, a.x), kH), __fmul_rn(-__fadd_rn(a.x, a.y), kH));
+  }
+
+  // y[r] = sum_m v[m] W_R^(m r) for R in {2, 4, 8, 16}
+  template <int R>
+  static __device__ __forceinline__ void dft(const float2 (&v)[R], float2 (&y)[R]) {
+    if constexpr (R == 16) {
+      // n = 4 n1 + n2, k = k1 + 4 k2:  X[k] = DFT_4 over n2 of W16^(n2 k1) * DFT_4 over n1 of v[4 n1 + n2]
+      float2 a[4][4];
 #pragma unroll
-    for (int u = 0; u < (kMaxBf > 0 ? kMaxBf : 1); ++u) {
+      for (int n2 = 0; n2 < 4; ++n2) dft4(v[n2], v[n2 + 4], v[n2 + 8], v[n2 + 12], a[n2]);
+      a[1][1] = cmul(a[1][1], make_float2(kC1, -kS1));
+      a[1][2] = w16_2(a[1][2]);
+      a[1][3] = cmul(a[1][3], make_float2(kS1, -kC1));
+      a[2][1] = w16_2(a[2][1]);
+      a[2][2] = mul_mi(a[2][2]);
+      a[2][3] = w16_6(a[2][3]);
+      a[3][1] = cmul(a[3][1], make_float2(kS1, -kC1));
+      a[3][2] = w16_6(a[3][2]);
+      a[3][3] = cmul(a[3][3], make_float2(-kC1, kS1));
+#pragma unroll
+      for (int k1 = 0; k1 < 4; ++k1) {
+        float2 z[4];
+        dft4(a[0][k1], a[1][k1], a[2][k1], a[3][k1], z);
+#pragma unroll
+        for (int k2 = 0; k2 < 4; ++k2) y[k1 + 4 * k2] = z[k2];
+      }
+    } else if constexpr (R == 8) {
+      // DFT_8 = two DFT_4 (even / odd inputs) combined with W8^k, W8 = exp(-2 pi i / 8)
+      float2 e[4], d[4];
+      dft4(v[0], v[2], v[4], v[6], e);
+      dft4(v[1], v[3], v[5], v[7], d);
+      const float2 d1 = w16_2(d[1]), d2 = mul_mi(d[2]), d3 = w16_6(d[3]);
+      y[0] = add(e[0], d[0]);
+      y[1] = add(e[1], d1);
+      y[2] = add(e[2], d2);
+      y[3] = add(e[3], d3);
+      y[4] = sub(e[0], d[0]);
+      y[5] = sub(e[1], d1);
+      y[6] = sub(e[2], d2);
+      y[7] = sub(e[3], d3);
+    } else if constexpr (R == 4) {
+      dft4(v[0], v[1], v[2], v[3], y);
+    } else {
+      y[0] = add(v[0], v[1]);
+      y[1] = sub(v[0], v[1]);
+    }
+  }
+
+  // One Stockham pass.  kIn: the first pass (Ns = 1, no twiddles) reads x straight from global
+  // memory (thread j loads x[j + r n/R]: consecutive j, coalesced); kOut: the last pass
+  // (Ns = n/R, o = j) writes y[j + r Ns] straight to global memory.  In-between results live in
+  // shared memory, so a transform moves 16n bytes through shared memory per middle boundary and
+  // none for staging.  The shared buffer is free on entry to a kIn pass (run_n's leading barrier).
+  template <int R, int NMAX, bool kIn, bool kOut>
+  static __device__ __forceinline__ void pass(float2 *s, const float2 *gx, float2 *gy, const float2 *tw, int n,
+                                              int Ns, int tid, uint32_t bar) {
+    constexpr int kMaxBf = NMAX / R / kVbThreads > 0 ? NMAX / R / kVbThreads : 1;   // butterflies per thread
+    // n, Ns, R are powers of two: shifts and masks instead of integer division
+    constexpr int lR = R == 2 ? 1 : R == 4 ? 2 : R == 8 ? 3 : 4;
+    const int ln = __ffs(n) - 1, ls = __ffs(Ns) - 1;
+    const int nbf = n >> lR, q = nbf;
+    float2 v[kMaxBf][R];
+#pragma unroll
+    for (int u = 0; u < kMaxBf; ++u) {
       const int j = tid + u * kVbThreads;
       if (j < nbf) {
-        const int k = j % Ns;
-        const int tstep = k * (n / (Ns * R));            // twiddle index step: k n / (Ns R)
-        // one table load per butterfly: w^r = w^(r-1) w (complex products)
-        const float2 w1 = __ldg(tw + tstep);
-        float2 w = w1;
+        if constexpr (kIn) {
+#pragma unroll
+          for (int r = 0; r < R; ++r) v[u][r] = __ldg(gx + j + r * q);
+        } else {
+          const int k = j & (Ns - 1);
+          const int tstep = k << (ln - ls - lR);           // twiddle index step: k n / (Ns R)
+#pragma unroll
+          for (int r = 0; r < R; ++r) v[u][r] = s[pad(j + r * q)];
+          const float2 w1 = __ldg(tw + tstep);
+          if constexpr (R == 16) {
+            // w^(4a + b) = w^(4a) w^b: table loads of w, w^4, w^8, w^12, at most two products each
+            const float2 w2 = cmul(w1, w1), w3 = cmul(w2, w1);
+#pragma unroll
+            for (int a4 = 0; a4 < 4; ++a4) {
+              const float2 wa = a4 == 0 ? make_float2(1.f, 0.f) : __ldg(tw + 4 * a4 * tstep);
+              if (a4) v[u][4 * a4] = cmul(v[u][4 * a4], wa);
+              v[u][4 * a4 + 1] = cmul(v[u][4 * a4 + 1], a4 ? cmul(wa, w1) : w1);
+              v[u][4 * a4 + 2] = cmul(v[u][4 * a4 + 2], a4 ? cmul(wa, w2) : w2);
+              v[u][4 * a4 + 3] = cmul(v[u][4 * a4 + 3], a4 ? cmul(wa, w3) : w3);
+            }
+          } else {
+            // one table load per butterfly: w^r = w^(r-1) w (complex products)
+            float2 w = w1;
+#pragma unroll
+            for (int r = 1; r < R; ++r) {
+              v[u][r] = cmul(v[u][r], w);
+              w = cmul(w, w1);
+            }
+          }
+        }
+      }
+    }
+    if constexpr (!kIn) named_bar_sync(bar, kVbThreads);   // every read done before the in-place writes
+#pragma unroll
+    for (int u = 0; u < kMaxBf; ++u) {
+      const int j = tid + u * kVbThreads;
+      if (j < nbf) {
+        const int k = j & (Ns - 1);
+        const int o = ((j >> ls) << (ls + lR)) + k;
+        float2 y[R];
+        dft<R>(v[u], y);
 #pragma unroll
         for (int r = 0; r < R; ++r) {
-          const float2 a = s[pad(j + r * q)];
-          v[u][r] = r == 0 ? a : cmul(a, w);
-          if (r >= 1) w = cmul(w, w1);
+          if constexpr (kOut) gy[o + r * Ns] = y[r];
+          else s[pad(o + r * Ns)] = y[r];
         }
       }
     }
-    named_bar_sync(bar, kVbThreads);
-#pragma unroll
-    for (int u = 0; u < (kMaxBf > 0 ? kMaxBf : 1); ++u) {
-      const int j = tid + u * kVbThreads;
-      if (j < nbf) {
-        const int k = j % Ns;
-        const int o = (j / Ns) * Ns * R + k;
-        if constexpr (R == 8) {
-          // DFT_8 = two DFT_4 (even / odd inputs) combined with W8^k, W8 = exp(-2 pi i / 8)
-          float2 e[4], d[4];
-          dft4(v[u][0], v[u][2], v[u][4], v[u][6], e);
-          dft4(v[u][1], v[u][3], v[u][5], v[u][7], d);
-          const float h = 0.70710678118654752f;   // 1/sqrt(2)
-          const float2 d1 = make_float2(__fmul_rn(__fadd_rn(d[1].x, d[1].y), h), __fmul_rn(__fsub_rn(d[1].y, d[1].x), h));
-          const float2 d2 = mul_mi(d[2]);
-          const float2 d3 = make_float2(__fmul_rn(__fsub_rn(d[3].y, d[3].x), h), __fmul_rn(-__fadd_rn(d[3].x, d[3].y), h));
-          s[pad(o)] = add(e[0], d[0]);
-          s[pad(o + Ns)] = add(e[1], d1);
-          s[pad(o + 2 * Ns)] = add(e[2], d2);
-          s[pad(o + 3 * Ns)] = add(e[3], d3);
-          s[pad(o + 4 * Ns)] = sub(e[0], d[0]);
-          s[pad(o + 5 * Ns)] = sub(e[1], d1);
-          s[pad(o + 6 * Ns)] = sub(e[2], d2);
-          s[pad(o + 7 * Ns)] = sub(e[3], d3);
-        } else if constexpr (R == 4) {
-          // DFT_4: X0 = (a0+a2)+(a1+a3), X1 = (a0-a2) - i(a1-a3), X2 = (a0+a2)-(a1+a3), X3 = (a0-a2) + i(a1-a3)
-          const float2 t0 = add(v[u][0], v[u][2]), t1 = sub(v[u][0], v[u][2]);
-          const float2 t2 = add(v[u][1], v[u][3]), t3 = mul_mi(sub(v[u][1], v[u][3]));
-          s[pad(o)] = add(t0, t2);
-          s[pad(o + Ns)] = add(t1, t3);
-          s[pad(o + 2 * Ns)] = sub(t0, t2);
-          s[pad(o + 3 * Ns)] = sub(t1, t3);
-        } else {
-          s[pad(o)] = add(v[u][0], v[u][1]);
-          s[pad(o + Ns)] = sub(v[u][0], v[u][1]);
-        }
-      }
-    }
-    named_bar_sync(bar, kVbThreads);
+    if constexpr (!kOut) named_bar_sync(bar, kVbThreads);
+  }
+
+  template <int R, int NMAX>
+  static __device__ __forceinline__ void last_pass(bool first, float2 *s, const float2 *gx, float2 *gy,
+                                                   const float2 *tw, int n, int Ns, int tid, uint32_t bar) {
+    if (first) pass<R, NMAX, true, true>(s, gx, gy, tw, n, Ns, tid, bar);
+    else pass<R, NMAX, false, true>(s, gx, gy, tw, n, Ns, tid, bar);
   }
 
   static __device__ __forceinline__ void run(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
@@ -130,31 +200,50 @@ template <> struct BeBody<TACKER_BE_FFT> {
     else if (p.n <= 1024) run_n<(kMaxN < 1024 ? kMaxN : 1024)>(p, vb, tid, bar, smem);
     else run_n<kMaxN>(p, vb, tid, bar, smem);
   }
+  // Pass plan for n = 2^L: one radix-2^f pass (f in {1, 2, 3, 4}) and p8 radix-8 passes, the
+  // radix-2^f one first (TK_FFT_ODD_FIRST) or last; n = 1024: 16, 8, 8 — two shared-memory
+  // boundaries (was 8, 8, 8, 2 with staging: 110 -> 68 us for 16384 x 1024, 0.60 of HBM).
   template <int NMAX>
   static __device__ __forceinline__ void run_n(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
                                                uint8_t *smem) {
     float2 *s = reinterpret_cast<float2 *>(smem);
     const float2 *tw = reinterpret_cast<const float2 *>(p.twiddle);
     const int n = p.n;
-    const float4 *x = reinterpret_cast<const float4 *>(p.x) + vb * (n / 2);
-    named_bar_sync(bar, kVbThreads);        // the previous transform of this slot is written out
-    for (int i = tid; i < n / 2; i += kVbThreads) {
-      const float4 v = __ldg(x + i);
-      s[pad(2 * i)] = make_float2(v.x, v.y);
-      s[pad(2 * i + 1)] = make_float2(v.z, v.w);
+    const float2 *gx = reinterpret_cast<const float2 *>(p.x) + vb * n;
+    float2 *gy = reinterpret_cast<float2 *>(p.y) + vb * n;
+    const int L = __ffs(n) - 1;
+    int p8, f;
+    if (L <= 4) p8 = 0, f = L;
+    else if (L % 3 == 0) p8 = L / 3 - 1, f = 3;
+    else if (L % 3 == 1) p8 = (L - 4) / 3, f = 4;
+    else p8 = (L - 2) / 3, f = 2;
+    named_bar_sync(bar, kVbThreads);        // the previous transform of this slot is done with s
+#if TK_FFT_ODD_FIRST
+    if (p8 > 0) {
+      // the radix-2^f pass first (reads global), then the radix-8 passes (the last one writes global)
+      switch (f) {
+        case 1: pass<2, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
+        case 2: pass<4, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
+        case 3: pass<8, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
+        default: pass<16, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
+      }
+      int Ns = 1 << f;
+      for (int i = 0; i < p8 - 1; ++i, Ns *= 8) pass<8, NMAX, false, false>(s, gx, gy, tw, n, Ns, tid, bar);
+      pass<8, NMAX, false, true>(s, gx, gy, tw, n, Ns, tid, bar);
+      return;
     }
-    named_bar_sync(bar, kVbThreads);
+#endif
     int Ns = 1;
-    for (; Ns * 8 <= n; Ns *= 8) pass<8, NMAX>(s, tw, n, Ns, tid, bar);
-    if (Ns * 4 <= n) {
-      pass<4, NMAX>(s, tw, n, Ns, tid, bar);
-      Ns *= 4;
+    for (int i = 0; i < p8; ++i, Ns *= 8) {
+      if (i == 0) pass<8, NMAX, true, false>(s, gx, gy, tw, n, Ns, tid, bar);
+      else pass<8, NMAX, false, false>(s, gx, gy, tw, n, Ns, tid, bar);
     }
-    if (Ns < n) pass<2, NMAX>(s, tw, n, Ns, tid, bar);
-    float4 *y = reinterpret_cast<float4 *>(p.y) + vb * (n / 2);
-    for (int i = tid; i < n / 2; i += kVbThreads) {
-      const float2 a = s[pad(2 * i)], b = s[pad(2 * i + 1)];
-      y[i] = make_float4(a.x, a.y, b.x, b.y);
+    const bool first = p8 == 0;
+    switch (f) {
+      case 1: last_pass<2, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
+      case 2: last_pass<4, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
+      case 3: last_pass<8, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
+      default: last_pass<16, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
     }
   }
 };

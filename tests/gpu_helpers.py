@@ -189,9 +189,12 @@ def be_case(kind, seed=0, size="small"):
             assert max_rel_err(o[0].ravel(), ref, S) <= 1e-5
         return dict(desc=tk.be_cp(dat, V, h, z), outs=[V], reset=lambda: V.zero_(), check=check, keep=(dat,))
     if kind in (tk.BE_FFT, tk.BE_FFT_TWIDDLE):
-        # radix passes: small n = 256 (8, 8, 4); "odd" n = 1024 (8, 8, 8, 2); "mid" n = 128 (8, 8, 2);
-        # "tiny" n = 2; large: the bench shape on sampled rows
+        # radix passes (first pass reads global, last writes global): small n = 256 (4, 8, 8);
+        # "odd" n = 1024 (16, 8, 8); "mid" n = 128 (16, 8); "tiny" n = 2 (2); "single16" n = 16 and
+        # "single8" n = 8 (one pass, global in and out); "two" n = 32 (4, 8); large: the bench shape
+        # on sampled rows
         batch, n = {"small": (37, 256), "odd": (7, 1024), "mid": (11, 128), "tiny": (3, 2),
+                    "single16": (5, 16), "single8": (6, 8), "two": (9, 32),
                     "large": (1 << 14, 1024)}[size]
         x = synth.fft_inputs(batch, n, seed)
         dx = t(x)

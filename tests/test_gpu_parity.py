@@ -86,7 +86,7 @@ def test_be_original_vs_oracle(tk, kind):
     c["check"]([host(o) for o in c["outs"]])
 
 
-@pytest.mark.parametrize("size", ["odd", "mid", "tiny"])
+@pytest.mark.parametrize("size", ["odd", "mid", "tiny", "single16", "single8", "two"])
 def test_fft_lengths_vs_oracle(tk, size):
     c = be_case(tk.BE_FFT, seed=4, size=size)
     c["reset"]()
