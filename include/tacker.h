@@ -130,7 +130,7 @@ typedef enum {
   TACKER_BE_MRIFHD_FH = 20,   /* mri-fhd ComputeFH: F^H d over one k chunk; block = 32 voxels x 4 k-lanes */
   TACKER_BE_CP = 21,          /* cp direct Coulomb summation on one lattice slice; block = 128x4 points */
   TACKER_BE_FFT_TWIDDLE = 22, /* fft plan: twiddle table w[m] = exp(-2 pi i m / n); block = 128 entries */
-  TACKER_BE_FFT = 23,         /* batched forward complex DFT, length n <= 1024; block = 1 transform */
+  TACKER_BE_FFT = 23,         /* batched forward complex DFT, length n <= 1024; block = 2 transforms */
   TACKER_BE_TPACF = 24,       /* angular correlation histogram; block = 128 points of a      */
   TACKER_BE_KIND_COUNT = 25
 } tacker_be_kind;

@@ -23,8 +23,11 @@ constexpr int kVbThreads = 128;
 #ifndef TK_FFT_ODD_FIRST
 #define TK_FFT_ODD_FIRST 1   // fft: the radix-2^f pass first (n = 256: 98.6 -> 90.7 us; equal at 1024)
 #endif
+#ifndef TK_FFT_PER_BLOCK
+#define TK_FFT_PER_BLOCK 2   // fft: transforms per original block (n = 256: 80 -> 72 us; equal at 1024)
+#endif
 #ifndef TK_FFT_MIN_BLOCKS
-#define TK_FFT_MIN_BLOCKS 12
+#define TK_FFT_MIN_BLOCKS 8  // fft original grid: 64 registers, no spills with two transforms per block
 #endif
 #ifndef TK_MRIQ_REDUCE
 #define TK_MRIQ_REDUCE 0

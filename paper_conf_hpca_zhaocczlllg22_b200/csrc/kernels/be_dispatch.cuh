@@ -59,7 +59,7 @@ __host__ __device__ constexpr int be_max_warps(int kind) {
   return kind == TACKER_BE_NONE ? 0 : kind == TACKER_BE_SGEMM ? 16 : 24;
 }
 // Minimum resident blocks per SM of an original (standalone) BE launch: caps the registers of
-// bodies whose latency hiding needs many blocks (fft: TK_FFT_MIN_BLOCKS = 12 blocks -> <= 40 registers).
+// bodies whose latency hiding needs many blocks (fft: TK_FFT_MIN_BLOCKS = 8 blocks -> <= 64 registers).
 __host__ __device__ constexpr int be_orig_min_blocks(int kind) { return kind == TACKER_BE_FFT ? TK_FFT_MIN_BLOCKS : 1; }
 
 // Body call with the optional per-kind TMA tensor map (only the stencil uses one).

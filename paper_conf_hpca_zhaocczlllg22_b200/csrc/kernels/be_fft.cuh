@@ -10,7 +10,7 @@ namespace tk {
 //
 // Twiddle table (TACKER_BE_FFT_TWIDDLE, the "plan" step, one launch per n):
 //   w[m] = (cospi(2m/n), -sinpi(2m/n)), m < n, with the accurate sincospi (not the MUFU).
-// Transform (TACKER_BE_FFT): one original block = one transform, Stockham autosort: one
+// Transform (TACKER_BE_FFT): one original block = kT transforms (2), Stockham autosort: one
 // radix-2/4/8/16 pass, then radix-8 passes (n = 1024: 16, 8, 8), so input and output are both
 // in natural order; the first pass reads x from global memory and the last writes y to it
 // (coalesced 8-byte accesses), intermediate results sit in shared memory (8n bytes).
@@ -41,9 +41,13 @@ template <> struct BeBody<TACKER_BE_FFT> {
   // Consecutive indices stay within their aligned 16-block (reads and staging conflict-free);
   // the Stockham writes of the first pass (stride 4 complex) spread over all 16 slots instead of
   // 4, those of Ns >= 16 stay conflict-free, Ns = 4 drops from 8-way to 4-way.
-  static constexpr uint32_t kSmem = kMaxN * 8;
+  // kT transforms per original block (TK_FFT_PER_BLOCK): with 2, a radix-16 pass of n = 1024 keeps
+  // all 128 threads busy (64 butterflies per transform) and every thread has twice the loads
+  // in flight, so a vblock of the fused kernel (fewer resident warps) hides more latency.
+  static constexpr int kT = TK_FFT_PER_BLOCK;
+  static constexpr uint32_t kSmem = kT * kMaxN * 8;
   static __device__ __forceinline__ int pad(int i) { return i ^ ((i >> 4) & 15); }
-  static __host__ __device__ int64_t num_blocks(const tacker_be_fft &p) { return p.batch; }
+  static __host__ __device__ int64_t num_blocks(const tacker_be_fft &p) { return (p.batch + kT - 1) / kT; }
 
   // complex product, contracted to two FMUL + two FFMA (the gate is 1e-5 of the signal scale)
   static __device__ __forceinline__ float2 cmul(float2 a, float2 w) {
@@ -123,19 +127,24 @@ template <> struct BeBody<TACKER_BE_FFT> {
   // (Ns = n/R, o = j) writes y[j + r Ns] straight to global memory.  In-between results live in
   // shared memory, so a transform moves 16n bytes through shared memory per middle boundary and
   // none for staging.  The shared buffer is free on entry to a kIn pass (run_n's leading barrier).
+  // Butterfly g < nt n/R of the block's nt transforms: transform h = g / (n/R), j = g mod (n/R);
+  // transform h lives at s + h n in shared memory and at gx + h n, gy + h n in global memory.
   template <int R, int NMAX, bool kIn, bool kOut>
-  static __device__ __forceinline__ void pass(float2 *s, const float2 *gx, float2 *gy, const float2 *tw, int n,
-                                              int Ns, int tid, uint32_t bar) {
-    constexpr int kMaxBf = NMAX / R / kVbThreads > 0 ? NMAX / R / kVbThreads : 1;   // butterflies per thread
+  static __device__ __forceinline__ void pass(float2 *s0, const float2 *gx0, float2 *gy0, const float2 *tw, int n,
+                                              int nt, int Ns, int tid, uint32_t bar) {
+    constexpr int kMaxBf = kT * NMAX / R / kVbThreads > 0 ? kT * NMAX / R / kVbThreads : 1;   // per thread
     // n, Ns, R are powers of two: shifts and masks instead of integer division
     constexpr int lR = R == 2 ? 1 : R == 4 ? 2 : R == 8 ? 3 : 4;
     const int ln = __ffs(n) - 1, ls = __ffs(Ns) - 1;
-    const int nbf = n >> lR, q = nbf;
+    const int nbf = n >> lR, q = nbf, lbf = ln - lR;
     float2 v[kMaxBf][R];
 #pragma unroll
     for (int u = 0; u < kMaxBf; ++u) {
-      const int j = tid + u * kVbThreads;
-      if (j < nbf) {
+      const int g = tid + u * kVbThreads;
+      const int j = g & (nbf - 1), hn = (g >> lbf) * n;
+      const float2 *gx = gx0 + hn;
+      const float2 *s = s0 + hn;
+      if (g < nt * nbf) {
         if constexpr (kIn) {
 #pragma unroll
           for (int r = 0; r < R; ++r) v[u][r] = __ldg(gx + j + r * q);
@@ -171,8 +180,11 @@ template <> struct BeBody<TACKER_BE_FFT> {
     if constexpr (!kIn) named_bar_sync(bar, kVbThreads);   // every read done before the in-place writes
 #pragma unroll
     for (int u = 0; u < kMaxBf; ++u) {
-      const int j = tid + u * kVbThreads;
-      if (j < nbf) {
+      const int g = tid + u * kVbThreads;
+      const int j = g & (nbf - 1), hn = (g >> lbf) * n;
+      float2 *gy = gy0 + hn;
+      float2 *s = s0 + hn;
+      if (g < nt * nbf) {
         const int k = j & (Ns - 1);
         const int o = ((j >> ls) << (ls + lR)) + k;
         float2 y[R];
@@ -189,9 +201,9 @@ template <> struct BeBody<TACKER_BE_FFT> {
 
   template <int R, int NMAX>
   static __device__ __forceinline__ void last_pass(bool first, float2 *s, const float2 *gx, float2 *gy,
-                                                   const float2 *tw, int n, int Ns, int tid, uint32_t bar) {
-    if (first) pass<R, NMAX, true, true>(s, gx, gy, tw, n, Ns, tid, bar);
-    else pass<R, NMAX, false, true>(s, gx, gy, tw, n, Ns, tid, bar);
+                                                   const float2 *tw, int n, int nt, int Ns, int tid, uint32_t bar) {
+    if (first) pass<R, NMAX, true, true>(s, gx, gy, tw, n, nt, Ns, tid, bar);
+    else pass<R, NMAX, false, true>(s, gx, gy, tw, n, nt, Ns, tid, bar);
   }
 
   static __device__ __forceinline__ void run(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
@@ -202,15 +214,16 @@ template <> struct BeBody<TACKER_BE_FFT> {
   }
   // Pass plan for n = 2^L: one radix-2^f pass (f in {1, 2, 3, 4}) and p8 radix-8 passes, the
   // radix-2^f one first (TK_FFT_ODD_FIRST) or last; n = 1024: 16, 8, 8 — two shared-memory
-  // boundaries (was 8, 8, 8, 2 with staging: 110 -> 68 us for 16384 x 1024, 0.60 of HBM).
+  // boundaries (was 8, 8, 8, 2 with staging: 110 -> 56 us for 16384 x 1024, 0.73 of HBM).
   template <int NMAX>
   static __device__ __forceinline__ void run_n(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
                                                uint8_t *smem) {
     float2 *s = reinterpret_cast<float2 *>(smem);
     const float2 *tw = reinterpret_cast<const float2 *>(p.twiddle);
     const int n = p.n;
-    const float2 *gx = reinterpret_cast<const float2 *>(p.x) + vb * n;
-    float2 *gy = reinterpret_cast<float2 *>(p.y) + vb * n;
+    const int nt = p.batch - vb * kT < kT ? (int)(p.batch - vb * kT) : kT;   // transforms of this block
+    const float2 *gx = reinterpret_cast<const float2 *>(p.x) + vb * kT * n;
+    float2 *gy = reinterpret_cast<float2 *>(p.y) + vb * kT * n;
     const int L = __ffs(n) - 1;
     int p8, f;
     if (L <= 4) p8 = 0, f = L;
@@ -222,28 +235,28 @@ template <> struct BeBody<TACKER_BE_FFT> {
     if (p8 > 0) {
       // the radix-2^f pass first (reads global), then the radix-8 passes (the last one writes global)
       switch (f) {
-        case 1: pass<2, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
-        case 2: pass<4, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
-        case 3: pass<8, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
-        default: pass<16, NMAX, true, false>(s, gx, gy, tw, n, 1, tid, bar); break;
+        case 1: pass<2, NMAX, true, false>(s, gx, gy, tw, n, nt, 1, tid, bar); break;
+        case 2: pass<4, NMAX, true, false>(s, gx, gy, tw, n, nt, 1, tid, bar); break;
+        case 3: pass<8, NMAX, true, false>(s, gx, gy, tw, n, nt, 1, tid, bar); break;
+        default: pass<16, NMAX, true, false>(s, gx, gy, tw, n, nt, 1, tid, bar); break;
       }
       int Ns = 1 << f;
-      for (int i = 0; i < p8 - 1; ++i, Ns *= 8) pass<8, NMAX, false, false>(s, gx, gy, tw, n, Ns, tid, bar);
-      pass<8, NMAX, false, true>(s, gx, gy, tw, n, Ns, tid, bar);
+      for (int i = 0; i < p8 - 1; ++i, Ns *= 8) pass<8, NMAX, false, false>(s, gx, gy, tw, n, nt, Ns, tid, bar);
+      pass<8, NMAX, false, true>(s, gx, gy, tw, n, nt, Ns, tid, bar);
       return;
     }
 #endif
     int Ns = 1;
     for (int i = 0; i < p8; ++i, Ns *= 8) {
-      if (i == 0) pass<8, NMAX, true, false>(s, gx, gy, tw, n, Ns, tid, bar);
-      else pass<8, NMAX, false, false>(s, gx, gy, tw, n, Ns, tid, bar);
+      if (i == 0) pass<8, NMAX, true, false>(s, gx, gy, tw, n, nt, Ns, tid, bar);
+      else pass<8, NMAX, false, false>(s, gx, gy, tw, n, nt, Ns, tid, bar);
     }
     const bool first = p8 == 0;
     switch (f) {
-      case 1: last_pass<2, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
-      case 2: last_pass<4, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
-      case 3: last_pass<8, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
-      default: last_pass<16, NMAX>(first, s, gx, gy, tw, n, Ns, tid, bar); break;
+      case 1: last_pass<2, NMAX>(first, s, gx, gy, tw, n, nt, Ns, tid, bar); break;
+      case 2: last_pass<4, NMAX>(first, s, gx, gy, tw, n, nt, Ns, tid, bar); break;
+      case 3: last_pass<8, NMAX>(first, s, gx, gy, tw, n, nt, Ns, tid, bar); break;
+      default: last_pass<16, NMAX>(first, s, gx, gy, tw, n, nt, Ns, tid, bar); break;
     }
   }
 };
