@@ -4,28 +4,27 @@
 
 Workload (N=1): BASELINE configs[3] (SURVEY config 4), QoS-managed co-location -- ResNet-50 at
 the paper's batch 32 (Table II) as the LC service (53 convs as implicit-GEMM tcgen05
-kernels, split-K where few tiles; conv1 = im2col + GEMM) with a BE queue of two Parboil
-applications, stencil (512x512x64 sweeps) and mri-q (64^3 voxels, 2048 k in two 1024-k chunks).
+kernels, split-K where few tiles; conv1 = im2col + GEMM) with the paper's mixed BE queue (Table II
+P:2021-2023: mri-q, fft, mri-fhd, cutcp, cp, sgemm, lbm, tpacf; each app resubmitted forever).
 
-* Headline (`value`): the QoS-managed run.  One step = one LC query; queries arrive as a
-  Poisson process at 80 % of the peak LC load (peak = the manager's LC-only
-  service rate, measured), the native manager (tacker_manager_run, Tacker policy) launches
-  fused / original / reordered kernels from each query's headroom under a 50 ms QoS target
-  (with B200 reading 18: an older query may fuse within the headroom of every later query, minus
-  a 15 ms guard; the paper-literal newest-query-only rule is reported as `tacker_paper`).
-  value = BE kernels completed per second over the K timed queries (CUDA events on the manager
-  stream), with the queries' p99 latency checked against the target.  The same trace under the
-  Baymax policy (fusion off) gives Eq. 10; a PTB-sliced Tacker run (reading 13) is reported too.
-* `e2e`: the same managed run through the public API where every query also moves its input
-  images host->device and its result device->host (pinned host memory, UVA copy kernels inside
-  the managed stream).
-* `roofline`: the dominant launch class of the timed run (LC convs: achieved vs tensor / HBM
-  peak).  `fused_step` + `roofline_fused`: BASELINE configs[1] -- every LC tensor-core kernel of a
-  ResNet-50 batch-1 query fused with the next BE kernel (fused time vs overlap roofline and vs
-  the sequential original launches); `config1_resnet50_b1` = the managed protocol at batch 1.
-* `cpu_baseline`: the CPU oracle on a bounded sample.
+Protocol:
+* lambda_peak = the largest LC arrival rate whose LC-only p99 meets the 50 ms QoS target
+  (bisection on LC-only windowed runs); arrivals are Poisson at 0.8 lambda_peak.
+* A STEP is a fixed block of STEP_QUERIES (100) LC queries' worth of arrivals (100 / lambda ms
+  of the trace).  One continuous Poisson run per arm: W warm-up steps, then the timed window of
+  exactly K steps, then a tail (1.5 x QoS of arrivals while the window's last queries finish),
+  then drain.  The window is bracketed by a stream sync + barrier and CUDA events on the manager
+  stream; the ramp-up and drain are outside it, so `value` does not depend on K.
+* value = BE kernels issued inside the window / its device time (sum over replicas / max time);
+  lc_p99 over every query that arrived inside the window (nearest rank) with a bootstrap 95 % CI.
+* Arms on the same trace: `tacker` (the headline; its rules are named in config.policy),
+  `baymax` (fusion off, the paper's queueing rule), `baymax_same_rule` (fusion off, the headline's
+  queueing rule: Eq. 10 against it isolates what fusion adds), `tacker_paper` (every rule as the
+  paper states it).  Each of tacker / baymax_same_rule runs `--seeds` trace seeds.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--batch 32] [--impl tacker|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--seeds S] [--impl tacker|reference]
+  --gpus N (no torchrun): N replica processes, one per GPU (CUDA_VISIBLE_DEVICES=i), no NCCL;
+  under torchrun the replicas coordinate over gloo (CPU), never NCCL.
 """
 from __future__ import annotations
 
@@ -36,6 +35,7 @@ import os
 import statistics
 import subprocess
 import sys
+import tempfile
 import threading
 import time
 
@@ -45,54 +45,80 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 QOS_MS = 50.0
-# Manager options of the headline Tacker run: B200 reading 18 -- an older query may
-# fuse / reorder within the headroom of every later active query, minus a 0.3 x QoS guard (qos.py).
-# The paper-literal rule (only the newest query fuses) is reported as tacker_paper.
-HEADLINE = {"fuse_older": True}
-LOAD = 0.8
+LOAD = 0.8                    # x lambda_peak
+STEP_QUERIES = 100            # LC queries per step
 METRIC = "BE kernels/sec at LC p99 <= QoS target"
-WORKLOAD = "resnet50_b{b} LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[3])"
+WORKLOAD = "resnet50_b{b} LC + Table II mixed BE queue ({be}), QoS 50 ms (BASELINE configs[3])"
+# Manager rules of the headline Tacker arm: the paper's reorder rule and direct rule
+# plus B200 reading 18 (older queries may fuse / reorder within the headroom of
+# every later active query, minus a 0.3 x QoS guard).  `tacker_paper` drops reading 18.
+HEADLINE = {"fuse_older": True}
 
 
-# ----------------------------------------------------------------------------- helpers
-_BACKEND = "nccl"
+# ----------------------------------------------------------------------------- replicas (no NCCL)
+class Comm:
+    """Coordination of replica processes, never a data-path collective: a single
+    process, gloo on CPU (under torchrun), or files (bench.py --gpus N spawns the replicas)."""
 
-
-def dist_setup(simulate=False):
-    """One process per GPU (replicas: no data-path collective).  The process group only carries
-    the barrier and the max/sum reductions of the timing; --simulate uses gloo on CPU."""
-    global _BACKEND
-    import torch
-    ws = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    _BACKEND = "gloo" if simulate else "nccl"
-    if ws > 1:
-        import torch.distributed as dist
-        if simulate:
+    def __init__(self):
+        self.ws = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        self.dir = os.environ.get("TACKER_REPLICA_DIR")
+        self.mode = "single" if self.ws == 1 else ("files" if self.dir else "gloo")
+        self._n = 0
+        if self.mode == "gloo":
+            import torch.distributed as dist
             dist.init_process_group("gloo")
-        else:
-            torch.cuda.set_device(local)
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    elif not simulate and torch.cuda.is_available():
-        torch.cuda.set_device(0)
-    return ws, rank, local
+
+    def reduce(self, v, op="max"):
+        if self.mode == "single":
+            return v
+        if self.mode == "gloo":
+            import torch
+            import torch.distributed as dist
+            t = torch.tensor([float(v)], dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
+            return float(t.item())
+        self._n += 1
+        path = os.path.join(self.dir, f"c{self._n}.r{self.rank}")
+        with open(path + ".tmp", "w") as f:
+            json.dump(float(v), f)
+        os.replace(path + ".tmp", path)
+        vals, t0 = [], time.time()
+        for r in range(self.ws):
+            p = os.path.join(self.dir, f"c{self._n}.r{r}")
+            while not os.path.exists(p):
+                if time.time() - t0 > 3600:
+                    raise TimeoutError(f"replica {r} never reached sync point {self._n}")
+                time.sleep(0.002)
+            with open(p) as f:
+                vals.append(json.load(f))
+        return max(vals) if op == "max" else sum(vals)
+
+    def barrier(self):
+        self.reduce(0.0)
+
+    def close(self):
+        if self.mode == "gloo":
+            import torch.distributed as dist
+            dist.destroy_process_group()
 
 
-def barrier(ws):
-    if ws > 1:
-        import torch.distributed as dist
-        dist.barrier()
-
-
-def reduce_ranks(ws, v, op="max"):
-    if ws == 1:
-        return v
-    import torch
-    import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cpu" if _BACKEND == "gloo" else "cuda")
-    dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
-    return float(t.item())
+def spawn_replicas(n):
+    """bench.py --gpus N without torchrun: N replica processes, replica i pinned to GPU i
+    (CUDA_VISIBLE_DEVICES), own seeds (rank), coordinating through files; rank 0 prints the line."""
+    d = tempfile.mkdtemp(prefix="tacker_replicas_")
+    procs = []
+    for i in range(n):
+        env = dict(os.environ, WORLD_SIZE=str(n), RANK=str(i), LOCAL_RANK="0", TACKER_REPLICA_DIR=d)
+        if "--simulate" not in sys.argv:
+            env["CUDA_VISIBLE_DEVICES"] = str(i)
+        procs.append(subprocess.Popen([sys.executable, os.path.abspath(__file__)] + sys.argv[1:], env=env))
+    rc = 0
+    for p in procs:
+        rc = max(rc, p.wait())
+    sys.exit(rc)
 
 
 class ClockSampler:
@@ -147,17 +173,26 @@ class ClockSampler:
 
 
 def measured_peaks():
+    """MEASURED_PEAKS.json (driver-written: HBM, bf16 burst / sustained) plus this repo's own
+    micro-benchmark peaks (profiles/peaks.json: FFMA, MUFU, fp16 GEMM) when present."""
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         with open(p) as f:
-            return json.load(f), "measured"
-    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+            peaks, kind = json.load(f), "measured"
+    else:
+        peaks, kind = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+    q = os.path.join(ROOT, "profiles", "peaks.json")
+    if os.path.exists(q):
+        with open(q) as f:
+            peaks["micro"] = json.load(f)
+    return peaks, kind
 
 
 # ----------------------------------------------------------------------------- kernel-level step
 class FusedStep:
-    """Every LC tensor-core kernel of one query fused with the next BE kernel (alternating a
-    stencil sweep and a mri-q Q chunk); CUDA-core LC kernels (im2col) launch original."""
+    """BASELINE configs[1]: every LC tensor-core kernel of one ResNet-50 batch-1 query fused with
+    the next BE kernel (alternating a stencil sweep and a mri-q Q chunk); CUDA-core LC kernels
+    (im2col) launch original."""
 
     def __init__(self, svc, stencil, mriq, warp_split):
         from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
@@ -204,8 +239,7 @@ class FusedStep:
 
     def two_streams(self):
         """Co-running baseline (NEXT-4, the paper's Stream co-location of Fig. 20): the LC
-        kernels in order on one stream, the BE kernels in order on another, original kernels,
-        the hardware scheduler interleaving their CTAs; joined back into the current stream."""
+        kernels in order on one stream, the BE kernels in order on another, original kernels."""
         import torch
         cur = torch.cuda.current_stream()
         if not hasattr(self, "_streams"):
@@ -235,27 +269,8 @@ def time_steps(torch, fn, steps, flush):
     return out
 
 
-def per_launch_times(torch, step, reps=3):
-    """Per-fused-launch device time (events between launches on the launching stream)."""
-    s = torch.cuda.current_stream()
-    acc = {}
-    for _ in range(reps):
-        evs = [torch.cuda.Event(enable_timing=True) for _ in range(len(step.plan) + 1)]
-        evs[0].record(s)
-        for i, (k, be, f) in enumerate(step.plan):
-            if f is not None:
-                f.launch()
-            else:
-                step.tk.tacker_launch_original(None, k.cd)
-            evs[i + 1].record(s)
-        evs[-1].synchronize()
-        for i, (k, be, f) in enumerate(step.plan):
-            cls = ("fused:" + be.name.split(".")[0]) if f is not None else ("lc_cd:" + k.name.split(".")[-1])
-            acc.setdefault(cls, []).append((evs[i].elapsed_time(evs[i + 1]), k, be))
-    return acc
-
-
-def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
+def kernel_level(torch, step, flush, peaks, steps):
+    """configs[1] fused step vs the BASELINE overlap roofline and vs sequential / two streams."""
     from paper_conf_hpca_zhaocczlllg22_b200.qos import overlap_rate   # Eq. 11
     fused_ms = time_steps(torch, step.fused, steps, flush)
     orig_ms = time_steps(torch, step.original, max(3, steps // 2), flush)
@@ -265,35 +280,9 @@ def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
     t_f, t_s = statistics.median(fused_ms), statistics.median(orig_ms)
     t_lc, t_be = statistics.median(lc_ms), statistics.median(be_ms)
     t_st = statistics.median(st_ms)
-    flush()
-    pl = per_launch_times(torch, step)
-    dom = max(pl, key=lambda c: sum(x[0] for x in pl[c]))
-    recs = pl[dom]
-    avg_ms = sum(x[0] for x in recs) / len(recs)
-    be0 = recs[0][2]
-    lc_bytes = sum(x[1].bytes for x in recs) / len(recs)
-    if be0 is not None and be0.bound == "mufu":
-        achieved = be0.mufu / (avg_ms / 1e3) / 1e12
-        peak = 148 * 16 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
-        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tops/s (MUFU sin/cos)",
-                "frac": achieved / peak, "traffic": None,
-                "peak_source": "derived: 148 SM x 16 MUFU/clk x sm_max_mhz (DESIGN.md §5)"}
-    else:
-        byts = (be0.bytes if be0 is not None else 0) + lc_bytes
-        achieved = byts / (avg_ms / 1e3) / 1e9
-        peak = peaks["hbm_gbs"]
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": None, "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
-    roof.update(kernel=dom, avg_launch_ms=avg_ms, launches=len(recs), stream="launching stream (torch current)")
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
-        with open(tp) as f:
-            roof["traffic"] = json.load(f).get(dom)
-    # BASELINE's overlap roofline per fused launch: max(F_LC / P_tensor, BE at its roofline,
-    # (B_LC + B_BE) / BW), summed over the step (CUDA-core LC kernels at their HBM time)
     p_tensor = peaks["bf16_tflops"] * 1e12          # fp16 runs at the bf16 rate
     bw = peaks["hbm_gbs"] * 1e9
-    p_mufu = 148 * 16 * peaks.get("sm_max_mhz", 1965.0) * 1e6
+    p_mufu = mufu_peak(peaks)[0] * 1e12
     t_roof = 0.0
     for k, be, f in step.plan:
         if f is None:
@@ -301,16 +290,81 @@ def kernel_level(torch, step, flush, peaks, peak_kind, clocks, steps):
             continue
         t_be_roof = be.mufu / p_mufu if be.bound == "mufu" else be.bytes / bw
         t_roof += max(k.flops / p_tensor, t_be_roof, (k.bytes + be.bytes) / bw)
-    fs = {"fused_step_ms": t_f, "sequential_step_ms": t_s, "lc_only_ms": t_lc, "be_only_ms": t_be,
-          "speedup_vs_sequential": t_s / t_f, "overlap_rate_eq11": overlap_rate(t_lc, t_be, t_f),
-          "two_streams_step_ms": t_st, "overlap_rate_eq11_two_streams": overlap_rate(t_lc, t_be, t_st),
-          "overlap_roofline_ms": t_roof * 1e3, "overlap_roofline_frac": t_roof * 1e3 / t_f,
-          "be_kernels_per_s": step.n_fused / (t_f / 1e3), "launches_per_step": len(step.plan)}
-    # LC convolutions alone against the tensor peak (batch 1: latency-bound, few tiles)
-    lc_flops = sum(k.flops for k, _, _ in step.plan if k.is_tc)
-    fs["lc_only_tflops"] = lc_flops / (t_lc / 1e3) / 1e12
-    fs["lc_only_tensor_frac"] = fs["lc_only_tflops"] * 1e12 / p_tensor
-    return fs, roof
+    return {"workload": "resnet50_b1 TC convs each fused with the next stencil sweep / mri-q chunk (BASELINE configs[1])",
+            "fused_step_ms": t_f, "sequential_step_ms": t_s, "lc_only_ms": t_lc, "be_only_ms": t_be,
+            "speedup_vs_sequential": t_s / t_f, "overlap_rate_eq11": overlap_rate(t_lc, t_be, t_f),
+            "two_streams_step_ms": t_st, "overlap_rate_eq11_two_streams": overlap_rate(t_lc, t_be, t_st),
+            "overlap_roofline_ms": t_roof * 1e3, "overlap_roofline_frac": t_roof * 1e3 / t_f,
+            "launches_per_step": len(step.plan), "l2": "256 MiB fill before every step"}
+
+
+def mufu_peak(peaks):
+    """(Tops/s, source) of the MUFU sin/cos pipe: the repo's micro-benchmark if measured, else
+    148 SMs x 16 /clk x sm_max_mhz (the guide's unit count)."""
+    m = peaks.get("micro", {}).get("mufu_sincos_tops")
+    if m:
+        return m, "measured: profiles/peaks.json (tools/peaks.py MUFU sin+cos micro-benchmark)"
+    return 148 * 16 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12, "derived: 148 SM x 16 MUFU/clk x sm_max_mhz"
+
+
+# ----------------------------------------------------------------------------- rooflines
+def lc_class_roofline(q, peaks, peak_kind, svc, traffic_key=None):
+    """The LC tensor-core convs of the timed run: per kernel the algorithmic flops (2 NPQ K CRS)
+    and bytes (x, w, out once), timed back to back with CUDA events on the launching stream
+    (QosRun.calibrate).  The bound is the one that gives the larger roofline time summed over
+    the query."""
+    off = 1 if getattr(q, "io", None) else 0
+    tc = [(k, q.t_lc[i + off]) for i, k in enumerate(svc.kernels) if k.is_tc]
+    p_t, bw = peaks["bf16_tflops"] * 1e12, peaks["hbm_gbs"] * 1e9
+    fl = sum(k.flops for k, _ in tc)
+    by = sum(k.bytes for k, _ in tc)
+    t_ms = sum(t for _, t in tc)
+    t_roof = sum(max(k.flops / p_t, k.bytes / bw) for k, _ in tc)
+    n = len(tc)
+    if fl / p_t >= by / bw:
+        ach = fl / n / (t_ms / n / 1e3) / 1e12
+        roof = {"bound": "tensor", "achieved": ach, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
+                "frac": ach / peaks["bf16_tflops"], "per_launch_work": "mean 2*NPQ*K*CRS of the TC convs",
+                "peak_source": f"MEASURED_PEAKS.json bf16_tflops burst ({peak_kind}); fp16 = bf16 rate"}
+    else:
+        ach = by / n / (t_ms / n / 1e3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": ach / peaks["hbm_gbs"], "per_launch_work": "mean 2*(NHWC + KRSC + NPQK) bytes of the TC convs",
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
+    roof["traffic"] = _traffic(traffic_key or f"lc_tc:{svc.name}")
+    roof.update(kernel=f"LC tensor-core convs of {svc.name} (implicit GEMM tcgen05, split-K where few tiles)",
+                avg_launch_ms=t_ms / n, launches_per_query=n, algorithmic_flops_per_launch=fl / n,
+                algorithmic_bytes_per_launch=by / n,
+                per_kernel_roofline_frac=t_roof * 1e3 / t_ms,
+                stream="launching stream, back-to-back launches (CUDA events)")
+    return roof
+
+
+def _traffic(key):
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            return json.load(f).get(key)
+    return None
+
+
+def be_class_roofline(q, peaks, apps):
+    """BE kernels of the timed run (original launches): per kernel its roofline time at its own
+    bound (HBM bytes / BW, FP32 flops / P_fp32, MUFU ops / P_mufu) against its measured
+    back-to-back time; aggregated as sum(T_roof) / sum(T_meas) over one cycle of every app."""
+    bw = peaks["hbm_gbs"] * 1e9
+    p_mufu = mufu_peak(peaks)[0] * 1e12
+    p_fma = peaks.get("micro", {}).get("ffma_tflops", 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12) * 1e12
+    rows, t_roof, t_meas = [], 0.0, 0.0
+    for a, app in enumerate(apps):
+        for j, bk in enumerate(app.kernels):
+            t = q.t_be[(a, j)]
+            r = max(bk.bytes / bw, bk.mufu / p_mufu if bk.mufu else 0.0, bk.flops / p_fma if bk.bound == "fma" else 0.0)
+            rows.append({"kernel": bk.name, "ms": t, "roofline_ms": r * 1e3, "frac": r * 1e3 / t if t else None,
+                         "bound": bk.bound})
+            t_roof += r * 1e3
+            t_meas += t
+    return {"frac": t_roof / t_meas if t_meas else None, "kernels": rows}
 
 
 # ----------------------------------------------------------------------------- CPU oracle baseline
@@ -368,7 +422,6 @@ def run_reference(args, ws, rank):
         return
     for _ in range(min(args.warmup, 3)):    # untimed warm-up steps (bounded)
         cpu_oracle_sample(small=True, batch=args.batch)
-    # bounded: each step is a small sample (~0.3 s); at most 120 s of steps
     t0 = time.perf_counter()
     vals, r = [], None
     for _ in range(args.steps):
@@ -381,263 +434,252 @@ def run_reference(args, ws, rank):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "BE kernels/s", "n_gpus": ws,
             "steps": len(vals), "warmup": args.warmup, "ms_per_step": el * 1000 / len(vals),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": WORKLOAD.format(b=args.batch), "l2": "n/a (CPU)"},
+            "config": {"workload": WORKLOAD.format(b=args.batch, be=args.be), "l2": "n/a (CPU)"},
             "cpu_baseline": {"value": v, "unit": "BE kernels/s", "cores": r["cores"], "kind": "oracle",
                              "sample": "per step: " + r["sample"]},
             "e2e": {"value": v, "unit": "BE kernels/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
 
 
-def managed_runs(q, tk, steps, seed, inflight, variants=("tacker", "baymax", "tacker_slice")):
-    """The same Poisson trace under each policy (the headline Tacker run first, timed by the
-    caller's window); returns {variant: result}."""
+ARMS = {   # name -> (policy, manager rules); the rules of each arm are also named in its result
+    "tacker": ("T", dict(HEADLINE)),
+    "baymax": ("B", {}),
+    "baymax_same_rule": ("B", dict(HEADLINE)),
+    "tacker_paper": ("T", {}),
+    "tacker_reorder_always": ("T", dict(HEADLINE, reorder_rule=1)),
+}
+KEEP = ("be_kernels_per_s", "be_norm_thpt", "lc_p50_ms", "lc_p99_ms", "lc_p99_ci95_ms", "qos_met", "violations",
+        "queries", "fused", "reordered", "idle_be", "rules", "elapsed_ms")
+
+
+def arm_result(q, tk, name, window_ms, warm_ms, load, seed, inflight, sync=None):
+    pol, rules = ARMS[name]
+    return q.run_window(tk.POLICY_TACKER if pol == "T" else tk.POLICY_BAYMAX, window_ms, warm_ms, load=load,
+                        seed=seed, max_inflight=inflight, sync=sync, **rules)
+
+
+def calibrated_run(qos, tk, svc, apps, args, comm):
+    q = qos.QosRun(svc, apps, warp_split=args.warp_split, qos_ms=QOS_MS)
+    q.calibrate()
+    q.measure_service(max_inflight=args.inflight)
+    # lambda_peak by bisection on LC-only runs (2000 queries' worth each)
+    q.find_peak_load(window_ms=20 * STEP_QUERIES * q.service_ms, max_inflight=args.inflight)
+    return q
+
+
+def side_runs(q, tk, arms, steps, rank, inflight, seeds=(0,)):
+    """The same protocol on other arms / seeds (not the timed headline)."""
+    load = LOAD * q.peak_load
+    win = steps * STEP_QUERIES * q.service_ms / load
+    warm = 5 * STEP_QUERIES * q.service_ms / load
     out = {}
-    kw = {"tacker": (tk.POLICY_TACKER, dict(HEADLINE)), "baymax": (tk.POLICY_BAYMAX, {}),
-          "tacker_paper": (tk.POLICY_TACKER, {}),
-          "baymax_older": (tk.POLICY_BAYMAX, dict(HEADLINE)),
-          "tacker_fuse_first": (tk.POLICY_TACKER, dict(HEADLINE, reorder_only_unfused=True)),
-          "tacker_slice_ff": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True, reorder_only_unfused=True)),
-          "tacker_slice_noreorder": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True, reorder_only_unfused=2)),
-          "tacker_slice": (tk.POLICY_TACKER, dict(HEADLINE, slice_be=True)),
-          "tacker_no_reverse": (tk.POLICY_TACKER, dict(HEADLINE, reverse_fusion=False))}
-    for v in variants:
-        pol, extra = kw[v]
-        out[v] = q.run(pol, steps, load=LOAD, seed=seed, max_inflight=inflight, **extra)
+    for a in arms:
+        rs = [arm_result(q, tk, a, win, warm, load, 2000 + 100 * s + rank, inflight) for s in seeds]
+        out[a] = {k: rs[0][k] for k in KEEP if k in rs[0]}
+        if len(rs) > 1:
+            out[a]["seeds"] = [{k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms")} for r in rs]
+            out[a]["be_norm_thpt_mean"] = statistics.mean(r["be_norm_thpt"] for r in rs)
+            out[a]["be_kernels_per_s_mean"] = statistics.mean(r["be_kernels_per_s"] for r in rs)
     return out
 
 
-def lc_class_roofline(q, peaks, peak_kind, svc):
-    """Roofline of the LC tensor-core kernels (the dominant launch class of the managed run):
-    per kernel the algorithmic flops (2 NPQ K CRS) and bytes (x, w, out once), timed back to back
-    with CUDA events on the launching stream (QosRun.calibrate).  The bound is the one that gives
-    the larger roofline time summed over the query."""
-    off = 1 if getattr(q, "io", None) else 0
-    tc = [(k, q.t_lc[i + off]) for i, k in enumerate(svc.kernels) if k.is_tc]
-    p_t, bw = peaks["bf16_tflops"] * 1e12, peaks["hbm_gbs"] * 1e9
-    fl = sum(k.flops for k, _ in tc)
-    by = sum(k.bytes for k, _ in tc)
-    t_ms = sum(t for _, t in tc)
-    t_roof = sum(max(k.flops / p_t, k.bytes / bw) for k, _ in tc)
-    n = len(tc)
-    if fl / p_t >= by / bw:
-        ach = fl / n / (t_ms / n / 1e3) / 1e12
-        roof = {"bound": "tensor", "achieved": ach, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
-                "frac": ach / peaks["bf16_tflops"], "per_launch_work": "mean 2*NPQ*K*CRS of the TC convs",
-                "peak_source": f"MEASURED_PEAKS.json bf16_tflops burst ({peak_kind}); fp16 = bf16 rate"}
-    else:
-        ach = by / n / (t_ms / n / 1e3) / 1e9
-        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": ach / peaks["hbm_gbs"], "per_launch_work": "mean 2*(NHWC + KRSC + NPQK) bytes of the TC convs",
-                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp) and svc.name == "resnet50_b32":
-        with open(tp) as f:
-            traffic = json.load(f).get("lc_tc")
-    roof.update(traffic=traffic, kernel=f"LC tensor-core convs of {svc.name} (implicit GEMM tcgen05, split-K where few tiles)",
-                avg_launch_ms=t_ms / n, launches_per_query=n,
-                per_kernel_roofline_frac=t_roof * 1e3 / t_ms,
-                stream="launching stream, back-to-back launches (CUDA events)")
-    return roof
+def eq10(a, b, key):
+    return a[key] / b[key] - 1.0 if a and b and b.get(key) else None
 
 
-def run_tacker(args, ws, rank, local):
+def run_tacker(args, comm):
     import torch
     from paper_conf_hpca_zhaocczlllg22_b200 import qos, services as sv, tacker as tk
 
+    if torch.cuda.is_available():
+        torch.cuda.set_device(comm.local)
+    ws, rank = comm.ws, comm.rank
     peaks, peak_kind = measured_peaks()
     seed = 2022 + rank
     svc = sv.resnet50_service(args.batch, seed)
     sv.autotune_tile_n(svc)                                      # LC tile width per conv, measured
-    stencil = sv.stencil_app(512, 512, 64, seed)
-    mriq = sv.mriq_app(64, 2048, 1024, seed)
-    tk.tacker_launch_original(None, mriq.kernels[0].desc)       # phiMag ready for the Q chunks
+    names = sv.TABLE2_BE if args.be == "table2" else tuple(args.be.split(","))
+    apps = sv.be_apps(names, seed)
+    sv.prime_apps(apps)
     flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
 
     def flush():
         flush_buf.fill_(1.0)
 
-    # ---- calibration (predictor, §VI-C) and the peak LC load (P:2184-2191) -- untimed
+    # ---- calibration (predictor, §VI-C), service rate and lambda_peak (P:2184-2191) -- untimed
     tk.tacker_model_clear()
-    q = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
-    q.calibrate()
-    q.measure_service(max_inflight=args.inflight)
-    # ---- warm-up queries (untimed)
-    q.run(tk.POLICY_TACKER, max(args.warmup, 3), load=LOAD, seed=1000 + rank, max_inflight=args.inflight, **HEADLINE)
-    torch.cuda.synchronize()
+    q = calibrated_run(qos, tk, svc, apps, args, comm)
+    load = LOAD * q.peak_load
+    step_ms = STEP_QUERIES * q.service_ms / load          # one step = 100 queries' worth of arrivals
+    window_ms, warm_ms = args.steps * step_ms, max(args.warmup, 3) * step_ms
 
-    # ---- timed region: K queries under the Tacker policy
-    clk = ClockSampler(local)
+    # ---- timed region: the steady-state window of the headline arm
+    clk = ClockSampler(comm.local)
     clk.start()
-    barrier(ws)
+    comm.barrier()
     torch.cuda.synchronize()
-    torch.cuda.nvtx.range_push("timed")      # ncu --nvtx --nvtx-include "timed/" selects these launches
-    res = q.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank, max_inflight=args.inflight, **HEADLINE)
+    torch.cuda.nvtx.range_push("timed")
+    res = arm_result(q, tk, "tacker", window_ms, warm_ms, load, 2000 + rank, args.inflight, sync=comm.barrier)
     torch.cuda.nvtx.range_pop()
     torch.cuda.synchronize()
-    barrier(ws)
+    comm.barrier()
     clocks = clk.stop()
-    elapsed_ms = reduce_ranks(ws, res["elapsed_ms"], "max")
-    be_total = reduce_ranks(ws, res["be_kernels"], "sum")
+    elapsed_ms = comm.reduce(res["elapsed_ms"], "max")
+    be_total = comm.reduce(res["be_kernels"], "sum")
     value = be_total / (elapsed_ms / 1e3)
-    p99 = reduce_ranks(ws, res["lc_p99_ms"], "max")
+    p99 = comm.reduce(res["lc_p99_ms"], "max")
+    norm = comm.reduce(res["be_work_ms"], "sum") / elapsed_ms
 
-    # ---- Baymax (Eq. 10) and PTB-sliced Tacker on the same trace
-    other = managed_runs(q, tk, args.steps, 2000 + rank, args.inflight,
-                         ("baymax", "tacker_slice", "tacker_paper", "baymax_older", "tacker_fuse_first",
-                          "tacker_slice_ff", "tacker_slice_noreorder"))
-    bay, slc, old, bay18 = other["baymax"], other["tacker_slice"], other["tacker_paper"], other["baymax_older"]
+    # ---- the other arms on the same trace; tacker / baymax_same_rule over --seeds seeds
+    seeds = tuple(range(args.seeds))
+    other = side_runs(q, tk, ("baymax", "baymax_same_rule", "tacker_paper"), args.steps, rank, args.inflight)
+    if args.seeds > 1:
+        more = side_runs(q, tk, ("tacker", "baymax_same_rule"), args.steps, rank, args.inflight, seeds)
+        other["tacker_seeds"] = more["tacker"]
+        other["baymax_same_rule_seeds"] = more["baymax_same_rule"]
+    bay, same, paper = other["baymax"], other["baymax_same_rule"], other["tacker_paper"]
 
-    # ---- e2e: the same managed run, each query with its H2D input + D2H result
-    qi = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS).with_io()
+    # ---- e2e: the same windowed run, each query with its H2D input + D2H result
+    qi = qos.QosRun(svc, apps, warp_split=args.warp_split, qos_ms=QOS_MS).with_io()
     qi.pairs, qi.ws_of, qi.t_be, qi.lr_be = q.pairs, q.ws_of, q.t_be, q.lr_be
     qi.t_lc = []
     for is_tc, d in qi._kernel_list():
         qi.t_lc.append(qos._time(lambda: tk.tacker_launch_original(d, None) if is_tc
                                   else tk.tacker_launch_original(None, d), 5))
     qi.measure_service(max_inflight=args.inflight)
-    e2e = qi.run(tk.POLICY_TACKER, args.steps, load=LOAD, seed=2000 + rank, max_inflight=args.inflight, **HEADLINE)
-    e2e_value = reduce_ranks(ws, e2e["be_kernels"], "sum") / (reduce_ranks(ws, e2e["elapsed_ms"], "max") / 1e3)
+    qi.peak_load = q.peak_load
+    load_io = LOAD * qi.peak_load
+    e2e = arm_result(qi, tk, "tacker", args.steps * STEP_QUERIES * qi.service_ms / load_io,
+                     max(args.warmup, 3) * STEP_QUERIES * qi.service_ms / load_io, load_io, 2000 + rank, args.inflight)
+    e2e_value = comm.reduce(e2e["be_kernels"], "sum") / (comm.reduce(e2e["elapsed_ms"], "max") / 1e3)
 
-    # ---- NEXT-2 reverse fusion side run: the same service with a tensor-core training BE app added
-    #      (Table II's DNN-training BE jobs); conv1's im2col (an LC CUDA-core kernel) may now fuse
-    #      with a BE GEMM.  The b32 calibration is reused; only the new pairs are fitted.
-    reverse = None
-    if not args.no_extra:
-        train = sv.gemm_train_app(4096, 4096, 4096, n=2, seed=seed + 3)
-        qr = qos.QosRun(svc, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
-        qr.t_lc, qr.t_be, qr.pairs, qr.ws_of, qr.lr_be = q.t_lc, dict(q.t_be), dict(q.pairs), q.ws_of, q.lr_be
-        qr.service_ms = q.service_ms
-        qr.add_tc_apps([train])
-        rr = managed_runs(qr, tk, args.steps, 2000 + rank, args.inflight, ("tacker", "tacker_no_reverse", "baymax"))
-        reverse = {"workload": "resnet50_b%d LC + stencil / mri-q / train-GEMM (2 x 4096^3 fp16) BE queue" % args.batch,
-                   "train_gemm_ms": [qr.t_be[(2, j)] for j in range(len(train.kernels))],
-                   "im2col_ms": qr.t_lc[0], "pairs": {}}
-        for j, bk in enumerate(train.kernels):
-            f = tk.tacker_fuse(bk.desc, svc.kernels[0].cd, qr.REV_WS)
-            pk = f.keys()[2]
-            reverse["pairs"][pk] = {"fused_ms": qos._time(lambda: f.launch(), 5),
-                                    "predicted_ms": tk.tacker_pair_predict(pk, qr.t_be[(2, j)], qr.t_lc[0]),
-                                    "in_model": pk in qr.pairs}
-        for v, r in rr.items():
-            reverse[v] = {k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms", "qos_met", "fused",
-                                            "reverse_fused", "reordered")}
-        for v in ("tacker", "tacker_no_reverse"):
-            reverse[v]["improvement_vs_baymax_eq10_normalised"] = rr[v]["be_norm_thpt"] / rr["baymax"]["be_norm_thpt"] - 1
-
-    # ---- roofline of the dominant launch class of the timed run (class shares from the manager's
-    #      sampled CUDA events on its stream)
+    # ---- roofline of the dominant launch class of the timed window
     cms, cn = res["class_ms"], res["class_launches"]
     tot_ms = sum(cms.values()) or 1.0
     shares = {c: {"ms": cms[c], "launches": cn[c], "share": cms[c] / tot_ms} for c in cms}
     dom = max(cms, key=cms.get)
-
-    # ---- BASELINE configs[1]: ResNet-50 batch-1 convs fused with stencil / mri-q -- the kernel-
-    #      level fused step (fused time vs overlap roofline) and the same managed protocol
-    svc1 = sv.resnet50_service(1, seed)
-    sv.autotune_tile_n(svc1)
-    step = FusedStep(svc1, stencil, mriq, args.warp_split)
-    for _ in range(3):
-        step.fused()
-    torch.cuda.synchronize()
-    fstep, roof_fused = kernel_level(torch, step, flush, peaks, peak_kind, clocks, max(5, min(args.steps, 20)))
-    b1 = None
-    if not args.no_extra:
-        tk.tacker_model_clear()
-        q1 = qos.QosRun(svc1, [stencil, mriq], warp_split=args.warp_split, qos_ms=QOS_MS)
-        q1.calibrate()
-        q1.measure_service(max_inflight=args.inflight)
-        q1.run(tk.POLICY_TACKER, 20, load=LOAD, seed=1000 + rank, max_inflight=args.inflight, **HEADLINE)
-        r1 = managed_runs(q1, tk, 1000, 3000 + rank, args.inflight, ("tacker", "baymax", "tacker_slice", "tacker_paper"))
-        b1 = {"workload": "resnet50_b1 LC + stencil/mriq BE queue, QoS 50 ms (BASELINE configs[1], config-4 protocol)",
-              "queries": 1000, "service_ms": q1.service_ms, "lc_roofline": lc_class_roofline(q1, peaks, peak_kind, svc1)}
-        for v, r in r1.items():
-            b1[v] = {k: r[k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p50_ms", "lc_p99_ms", "qos_met",
-                                        "fused", "reordered", "idle_be")}
-        for v in ("tacker", "tacker_slice", "tacker_paper"):
-            b1[v]["improvement_vs_baymax_eq10"] = r1[v]["be_kernels_per_s"] / r1["baymax"]["be_kernels_per_s"] - 1
-            b1[v]["improvement_vs_baymax_eq10_normalised"] = r1[v]["be_norm_thpt"] / r1["baymax"]["be_norm_thpt"] - 1
-
     if dom in ("lc_tc", "lc_cd"):
         roof = lc_class_roofline(q, peaks, peak_kind, svc)
     else:
-        roof = dict(roof_fused)
+        roof = lc_class_roofline(q, peaks, peak_kind, svc)
+        roof["note"] = f"dominant class of the window is {dom}; the LC convs are reported (BE: be_roofline)"
     roof["class_shares"] = shares
+    be_roof = be_class_roofline(q, peaks, apps)
+
+    extra = {}
+    if not args.no_extra:
+        extra = side_workloads(args, comm, peaks, flush, tk, qos, sv, torch)
 
     cpu = cpu_oracle_sample(batch=args.batch) if (rank == 0 and ws == 1 and not args.no_cpu) else None
     if cpu is not None:
         cpu.pop("seconds_per_be_kernel", None)
 
+    tk_line = {k: res[k] for k in KEEP if k in res}
     line = {
         "metric": METRIC, "value": value, "unit": "BE kernels/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "f16xf16->f32 (LC tcgen05) + f32 (BE CUDA cores)",
         "data": "synthetic (seeded inputs, random weights)",
-        "config": {"workload": WORKLOAD.format(b=args.batch),
+        "config": {"workload": WORKLOAD.format(b=args.batch, be=",".join(names)),
                    "lc": f"ResNet-50 batch-{args.batch} (Table II), 53 convs, fp16 NHWC, implicit GEMM tcgen05",
-                   "be": "stencil 512x512x64 sweeps | mri-q 64^3 x (phiMag + 2 x 1024-k chunks)",
-                   "arrivals": f"Poisson at {LOAD:.0%} of the peak rate (the manager's LC-only service rate)",
-                   "qos_ms": QOS_MS, "policy": "tacker (+ reading 18: older queries fuse within later queries' headroom - 15 ms)", "warp_split": args.warp_split, "max_inflight": args.inflight,
-                   "step": "one LC query", "parallelism": f"replicas x{ws}",
-                   "l2": "inputs larger than L2 (stencil 2 x 64 MiB ping-pong + activations and weights > 1 GB)"},
-        "lc_p99_ms": p99, "lc_p50_ms": res["lc_p50_ms"], "lc_qos_ms": QOS_MS, "qos_met": p99 <= QOS_MS,
-        "lambda_per_s": res["lambda_per_s"], "service_ms": q.service_ms, "query_solo_ms": q.query_solo_ms(),
-        "fused_launches": res["fused"], "reordered_be": res["reordered"],
-        "idle_be": res["idle_be"], "model_refits": res["model_refits"],
-        "baymax": {"value": bay["be_kernels_per_s"], "lc_p99_ms": bay["lc_p99_ms"], "qos_met": bay["qos_met"],
-                   "be_norm_thpt": bay["be_norm_thpt"]},
-        "improvement_vs_baymax_eq10": res["be_kernels_per_s"] / bay["be_kernels_per_s"] - 1.0,
-        # BE work in standalone-kernel milliseconds per wall millisecond (app-length independent)
-        "be_norm_thpt": res["be_norm_thpt"],
-        "improvement_vs_baymax_eq10_normalised": res["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0,
-        "tacker_slice": {"value": slc["be_kernels_per_s"], "be_norm_thpt": slc["be_norm_thpt"],
-                         "lc_p99_ms": slc["lc_p99_ms"], "fused": slc["fused"],
-                         "improvement_vs_baymax_eq10_normalised": slc["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0},
-        # Baymax with the same reading-18 queueing rule (older queries reorder within later
-        # queries' headroom): Eq. 10 against it isolates what fusion adds
-        "baymax_same_rule": {"value": bay18["be_kernels_per_s"], "be_norm_thpt": bay18["be_norm_thpt"],
-                             "lc_p99_ms": bay18["lc_p99_ms"], "qos_met": bay18["qos_met"]},
-        "improvement_vs_baymax_same_rule_eq10": res["be_kernels_per_s"] / bay18["be_kernels_per_s"] - 1.0,
-        # reorder only after LC kernels that were not fused (the literal P:2035 rule) on top of reading 18
-        "tacker_fuse_first": {k: other["tacker_fuse_first"][k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms",
-                                                                         "qos_met", "fused", "reordered")},
-        "tacker_slice_ff": {k: other["tacker_slice_ff"][k] for k in ("be_kernels_per_s", "be_norm_thpt", "lc_p99_ms",
-                                                                     "qos_met", "fused", "reordered")},
-        "tacker_slice_noreorder": {k: other["tacker_slice_noreorder"][k] for k in ("be_kernels_per_s", "be_norm_thpt",
-                                                                                   "lc_p99_ms", "qos_met", "fused",
-                                                                                   "reordered", "idle_be")},
-        "improvement_vs_baymax_same_rule_eq10_normalised": res["be_norm_thpt"] / bay18["be_norm_thpt"] - 1.0,
-        # the paper-literal manager rule: only the newest query fuses / reorders (P:2058-2072)
-        "tacker_paper": {"value": old["be_kernels_per_s"], "be_norm_thpt": old["be_norm_thpt"],
-                         "lc_p99_ms": old["lc_p99_ms"], "qos_met": old["qos_met"], "fused": old["fused"],
-                         "improvement_vs_baymax_eq10": old["be_kernels_per_s"] / bay["be_kernels_per_s"] - 1.0,
-                         "improvement_vs_baymax_eq10_normalised": old["be_norm_thpt"] / bay["be_norm_thpt"] - 1.0},
-        "reverse_fusion": reverse,
-        "fused_pred_err_mean": res["fused_pred_err_mean"],
+                   "be": " | ".join(a.name for a in apps),
+                   "arrivals": f"Poisson at {LOAD:.0%} of lambda_peak (LC-only p99 <= QoS, bisection) = "
+                               f"{load:.3f} x the LC-only service rate",
+                   "step": f"{STEP_QUERIES} LC queries' worth of arrivals ({step_ms:.1f} ms); timed window = "
+                           f"{args.steps} steps inside one continuous run after {max(args.warmup, 3)} warm-up steps, "
+                           "followed by a 1.5 x QoS tail",
+                   "qos_ms": QOS_MS, "policy": res["rules"], "warp_split": args.warp_split,
+                   "max_inflight": args.inflight, "parallelism": f"replicas x{ws} ({comm.mode}, no NCCL)",
+                   "l2": "inputs larger than L2 (activations > 1 GB, BE working sets 8-340 MB)"},
+        "be_norm_thpt": norm,
+        "lc_p99_ms": p99, "lc_p99_ci95_ms": res["lc_p99_ci95_ms"], "lc_p50_ms": res["lc_p50_ms"],
+        "lc_qos_ms": QOS_MS, "qos_met": p99 <= QOS_MS, "queries_in_window": res["queries"],
+        "violations": res["violations"],
+        "lambda_peak_load": q.peak_load, "lambda_per_s": res["lambda_per_s"], "service_ms": q.service_ms,
+        "query_solo_ms": q.query_solo_ms(),
+        "fused_launches": res["fused"], "reordered_be": res["reordered"], "idle_be": res["idle_be"],
+        "model_refits": res["model_refits"], "fused_pred_err_mean": res["fused_pred_err_mean"],
         "pair_pred_err_mean": statistics.mean(q.pair_err) if q.pair_err else None,
+        # Eq. 10 (P:2704-2708) on normalised BE throughput (app-length independent) and on kernels/s
+        "improvement_vs_baymax_same_rule_eq10_normalised": eq10(res, same, "be_norm_thpt"),
+        "improvement_vs_baymax_same_rule_eq10": eq10(res, same, "be_kernels_per_s"),
+        "improvement_vs_baymax_eq10_normalised": eq10(res, bay, "be_norm_thpt"),
+        "improvement_vs_baymax_eq10": eq10(res, bay, "be_kernels_per_s"),
+        "tacker_paper_vs_baymax_eq10_normalised": eq10(paper, bay, "be_norm_thpt"),
+        "arms": dict(other, tacker=tk_line),
         "roofline": roof,
-        "roofline_fused": roof_fused,
-        "fused_step": fstep,
+        "be_roofline": be_roof,
         "cpu_baseline": cpu,
-        "e2e": {"value": e2e_value, "unit": "BE kernels/s", "h2d_bytes_per_step": qi.h2d_bytes,
-                "d2h_bytes_per_step": qi.d2h_bytes, "lc_p99_ms": e2e["lc_p99_ms"],
-                "how": "each query copies its input image H2D and its result D2H from/to pinned host memory "
-                       "(UVA copy kernels on the manager stream) inside the timed managed run"},
+        "e2e": {"value": e2e_value, "unit": "BE kernels/s", "h2d_bytes_per_step": qi.h2d_bytes * STEP_QUERIES,
+                "d2h_bytes_per_step": qi.d2h_bytes * STEP_QUERIES, "lc_p99_ms": e2e["lc_p99_ms"],
+                "be_norm_thpt": e2e["be_norm_thpt"],
+                "how": "the same windowed run where each query copies its input image H2D and its result D2H "
+                       "from/to pinned host memory (UVA copy kernels on the manager stream)"},
         # counted by the manager: every LC kernel of every query (fused or original) plus the
-        # reordered and idle-time BE launches
+        # reordered and idle-time BE launches inside the window
         "gpu_launches": int(sum(res["class_launches"].values())),
         "clocks": clocks,
-        "config1_resnet50_b1": b1,
     }
+    line.update(extra)
     if rank == 0:
         print(json.dumps(line))
 
 
-def run_simulated(args, ws, rank):
-    """--simulate: the same managed run on the manager's simulated GPU (kernels take their
-    predicted time; no CUDA), for CPU tests of the multi-rank path (gloo).  Kernel durations are
-    a fixed table shaped like the B200 measurements of the ResNet-50 b1 / stencil / mri-q run."""
-    from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
+def side_workloads(args, comm, peaks, flush, tk, qos, sv, torch):
+    """Beside the headline: VGG-16 b24 with the same mixed queue, ResNet-50 b32 with the round-1
+    stencil / mri-q queue, and BASELINE configs[1] (ResNet-50 b1) as a managed run and as the
+    kernel-level fused step (fused time vs the overlap roofline)."""
+    out = {}
+    rank = comm.rank
+    steps = max(5, min(args.steps, 30))
+    seed = 2022 + rank
+    names = sv.TABLE2_BE if args.be == "table2" else tuple(args.be.split(","))
+    # VGG-16 batch 24 (Table II) + the mixed queue
+    tk.tacker_model_clear()
+    vgg = sv.vgg16_service(24, seed)
+    sv.autotune_tile_n(vgg)
+    apps = sv.be_apps(names, seed)
+    sv.prime_apps(apps)
+    qv = calibrated_run(qos, tk, vgg, apps, args, comm)
+    r = side_runs(qv, tk, ("tacker", "baymax", "baymax_same_rule", "tacker_paper"), steps, rank, args.inflight)
+    out["vgg16_b24"] = dict(workload="vgg16_b24 LC + Table II mixed BE queue, QoS 50 ms (BASELINE configs[3])",
+                            service_ms=qv.service_ms, lambda_peak_load=qv.peak_load, steps=steps, **r,
+                            improvement_vs_baymax_same_rule_eq10_normalised=eq10(r["tacker"], r["baymax_same_rule"], "be_norm_thpt"),
+                            tacker_paper_vs_baymax_eq10_normalised=eq10(r["tacker_paper"], r["baymax"], "be_norm_thpt"))
+    del vgg, apps, qv
+    torch.cuda.empty_cache()
+    # ResNet-50 b32 + stencil / mri-q (round-1 queue) and b1 (configs[1])
+    st, mq = sv.be_apps(("stencil", "mriq"), seed)
+    sv.prime_apps([mq])
+    for b in (32, 1):
+        tk.tacker_model_clear()
+        svc = sv.resnet50_service(b, seed)
+        sv.autotune_tile_n(svc)
+        qb = calibrated_run(qos, tk, svc, [st, mq], args, comm)
+        r = side_runs(qb, tk, ("tacker", "baymax", "baymax_same_rule", "tacker_paper"), steps, rank, args.inflight)
+        out[f"resnet50_b{b}_stencil_mriq"] = dict(
+            workload=f"resnet50_b{b} LC + stencil/mriq BE queue, QoS 50 ms" + (" (BASELINE configs[1])" if b == 1 else ""),
+            service_ms=qb.service_ms, lambda_peak_load=qb.peak_load, steps=steps, **r,
+            lc_roofline=lc_class_roofline(qb, {**peaks}, "measured", svc),
+            improvement_vs_baymax_same_rule_eq10_normalised=eq10(r["tacker"], r["baymax_same_rule"], "be_norm_thpt"),
+            tacker_paper_vs_baymax_eq10_normalised=eq10(r["tacker_paper"], r["baymax"], "be_norm_thpt"))
+        if b == 1:
+            step = FusedStep(svc, st, mq, args.warp_split)
+            for _ in range(3):
+                step.fused()
+            torch.cuda.synchronize()
+            out["fused_step"] = kernel_level(torch, step, flush, peaks, 20)
+        del svc, qb
+        torch.cuda.empty_cache()
+    return out
+
+
+def run_simulated(args, comm):
+    """--simulate: the same windowed protocol on the manager's simulated GPU (kernels take their
+    predicted time; no CUDA), for CPU tests of the replica path.  Kernel durations are a fixed
+    table shaped like the B200 measurements of the ResNet-50 b1 / stencil / mri-q run."""
+    from paper_conf_hpca_zhaocczlllg22_b200 import qos, tacker as tk
+    ws, rank = comm.ws, comm.rank
     tk.tacker_model_clear()
     fake = 0x10000
     lc = tk.LcDesc(kind=tk.LC_GEMM_F16, M=1024, N=256, K=256, A=fake, B=fake, D=fake)
@@ -650,64 +692,78 @@ def run_simulated(args, ws, rank):
     tk.tacker_pair_fit(key)
     apps = [[tk.BeKernel(is_cd=1, t_pred_ms=0.035, be=st, warp_split=args.warp_split)] * 2,
             [tk.BeKernel(is_cd=1, t_pred_ms=0.147, be=st, warp_split=args.warp_split)] * 2]
-    rng = np.random.default_rng(2000 + rank)
     solo = sum(k.t_pred_ms for k in ks)
-    gaps = rng.exponential(solo / LOAD, args.steps)
+    lam = LOAD / solo
+    step_ms = STEP_QUERIES / lam
+    w0, w1 = max(args.warmup, 3) * step_ms, (max(args.warmup, 3) + args.steps) * step_ms
     out = {}
     for pol in (tk.POLICY_BAYMAX, tk.POLICY_TACKER):
-        m = tk.Manager(pol, simulate=True, idle_cap_ms=0.5 * (QOS_MS - solo))
+        rng = np.random.default_rng(2000 + rank)
+        m = tk.Manager(pol, simulate=True, idle_cap_ms=0.5 * (QOS_MS - solo), **HEADLINE)
         for a in apps:
             m.submit_be(a)
-        arr = np.cumsum(gaps)
-        q = [m.submit_lc(ks, float(t)) for t in arr]
-        barrier(ws)
+        arr, t = [], 0.0
+        while t < w1 + 1.5 * QOS_MS:
+            t += rng.exponential(1.0 / lam)
+            arr.append(t)
+        qids = [m.submit_lc(ks, float(a)) for a in arr]
+        m.run_until(QOS_MS, w0)
+        s0 = m.stats()
+        m.run_until(QOS_MS, w1)
+        s1 = m.stats()
         m.run(QOS_MS, float(arr[-1]))
-        s = m.stats()
-        lat = np.sort([m.latency(i) for i in q])
-        out[pol] = (s.be_kernels_done, s.now_ms, float(lat[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)]))
+        lat = [m.latency(i) for i, a in zip(qids, arr) if w0 <= a < w1]
+        out[pol] = (s1.be_kernels_done - s0.be_kernels_done, s1.now_ms - s0.now_ms,
+                    qos.latency_stats(lat, QOS_MS)["lc_p99_ms"])
     be, el, p99 = out[tk.POLICY_TACKER]
-    elapsed = reduce_ranks(ws, el, "max")
-    value = reduce_ranks(ws, be, "sum") / (elapsed / 1e3)
-    bay = reduce_ranks(ws, out[tk.POLICY_BAYMAX][0], "sum") / (reduce_ranks(ws, out[tk.POLICY_BAYMAX][1], "max") / 1e3)
+    comm.barrier()
+    elapsed = comm.reduce(el, "max")
+    value = comm.reduce(be, "sum") / (elapsed / 1e3)
+    bay = comm.reduce(out[tk.POLICY_BAYMAX][0], "sum") / (comm.reduce(out[tk.POLICY_BAYMAX][1], "max") / 1e3)
     line = {"metric": METRIC, "value": value, "unit": "BE kernels/s", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "n/a (simulated GPU)", "data": "synthetic",
-            "config": {"workload": WORKLOAD.format(b=1) + " [simulated durations]", "parallelism": f"replicas x{ws}"},
-            "lc_p99_ms": reduce_ranks(ws, p99, "max"), "baymax": {"value": bay},
+            "config": {"workload": "resnet50_b1-like LC + stencil-like BE [simulated durations]",
+                       "parallelism": f"replicas x{ws} ({comm.mode}, no NCCL)"},
+            "lc_p99_ms": comm.reduce(p99, "max"), "baymax": {"value": bay},
             "improvement_vs_baymax_eq10": value / bay - 1.0, "simulated": True}
-    if rank == 0:
+    if comm.rank == 0:
         print(json.dumps(line))
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300, help="timed LC queries")
+    ap.add_argument("--steps", type=int, default=100, help=f"timed steps ({STEP_QUERIES} LC queries each)")
+    ap.add_argument("--warmup", type=int, default=5, help="untimed warm-up steps (same continuous run)")
+    ap.add_argument("--seeds", type=int, default=3, help="trace seeds for the tacker / baymax_same_rule arms")
     ap.add_argument("--batch", type=int, default=32, help="LC batch (Table II: ResNet-50 at 32)")
+    ap.add_argument("--be", default="table2", help="BE queue: table2 (Table II mixed queue) or app names")
     ap.add_argument("--inflight", type=int, default=16, help="manager: launches in flight on its stream")
-    ap.add_argument("--warmup", type=int, default=20, help="untimed warm-up LC queries")
     ap.add_argument("--impl", default="tacker", choices=["tacker", "reference"])
     ap.add_argument("--warp-split", type=int, default=24)
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--no-extra", action="store_true", help="skip the ResNet-50 b1 (configs[1]) managed side run")
-    ap.add_argument("--simulate", action="store_true", help="CPU-only: manager on its simulated GPU (gloo)")
+    ap.add_argument("--no-extra", action="store_true", help="skip the side workloads (VGG-16, stencil/mri-q, b1)")
+    ap.add_argument("--simulate", action="store_true", help="CPU-only: manager on its simulated GPU")
     ap.add_argument("--overlap", type=int, default=None,
                     help="programmatic dependent launch mode (tacker_set_launch_overlap: 0, 1, 2)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        spawn_replicas(args.gpus)
     if args.impl == "reference":
         run_reference(args, int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")))
         return
-    ws, rank, local = dist_setup(simulate=args.simulate)
-    if args.simulate:
-        run_simulated(args, ws, rank)
-    else:
-        if args.overlap is not None:
-            from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
-            tk.tacker_set_launch_overlap(args.overlap)
-        run_tacker(args, ws, rank, local)
-    if ws > 1:
-        import torch.distributed as dist
-        dist.destroy_process_group()
+    comm = Comm()
+    try:
+        if args.simulate:
+            run_simulated(args, comm)
+        else:
+            if args.overlap is not None:
+                from paper_conf_hpca_zhaocczlllg22_b200 import tacker as tk
+                tk.tacker_set_launch_overlap(args.overlap)
+            run_tacker(args, comm)
+    finally:
+        comm.close()
 
 
 if __name__ == "__main__":

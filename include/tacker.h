@@ -411,7 +411,7 @@ typedef struct {
 } tacker_decision;
 
 typedef struct {
-  double direct_eps_ms;      /* Thr <= this at first issue -> launch the query directly */
+  double direct_eps_ms;      /* Thr <= this at first issue -> launch the query directly (direct_rule) */
   double idle_cap_ms;        /* idle GPU: launch BE heads no longer than this (<=0: any) */
   int32_t max_inflight;      /* GPU mode: kernels allowed in flight on the stream (>=1) */
   int32_t simulate;          /* 1: no GPU, durations = predictions */
@@ -421,9 +421,12 @@ typedef struct {
    * 0: whole BE kernels only (the paper's fusion unit). */
   int32_t slice_be;
   double slice_ratio;
-  /* 0 (default): after every LC kernel, fused or not, reorder the other ready BE heads with
-   * Ttmp < Thr (reading 6); 1: reorder only after an LC kernel that was not fused. */
-  int32_t reorder_only_unfused;   /* 2: never reorder (BE work only fused or on an idle GPU) */
+  /* tacker_reorder_rule.  TACKER_REORDER_UNFUSED (0, default, the paper's rule P:2035-2043: "If
+   * all the ready BE kernels may not be fused with the current kernel of Q", reorder the ready BE
+   * heads with Ttmp < Thr; nothing after a fused launch); TACKER_REORDER_ALWAYS (B200 reading 6,
+   * after every LC kernel, fused or not); TACKER_REORDER_NEVER (BE work only fused
+   * or on an idle GPU). */
+  int32_t reorder_rule;
   /* 1: never fuse an LC CUDA-core kernel with a BE tensor-core kernel (NEXT-2 off) */
   int32_t no_reverse_fusion;
   /* B200 reading 18 (off = the paper's rule: only the newest query fuses / reorders):
@@ -433,7 +436,14 @@ typedef struct {
    * error and the host running ahead of the GPU). */
   int32_t fuse_older;
   double older_margin_ms;
+  /* tacker_direct_rule: "If the Thr of the new query is close to 0, Tacker directly launches all
+   * the kernels".  TACKER_DIRECT_MIN_BE (0, default; SURVEY §8(c) c15 reading):
+   * close to 0 = Thr <= max(direct_eps_ms, the smallest prediction of a ready BE head) at the
+   * query's first issue; TACKER_DIRECT_EPS: Thr <= direct_eps_ms only. */
+  int32_t direct_rule;
 } tacker_manager_params;
+enum { TACKER_REORDER_UNFUSED = 0, TACKER_REORDER_ALWAYS = 1, TACKER_REORDER_NEVER = 2 };
+enum { TACKER_DIRECT_MIN_BE = 0, TACKER_DIRECT_EPS = 1 };
 
 typedef struct tacker_manager_s *tacker_manager_t;
 
@@ -461,6 +471,33 @@ tacker_status tacker_manager_prepare(tacker_manager_t m, const tacker_lc_query *
  * t_end_ms and every submitted query has completed, or max_decisions decisions were taken
  * (<= 0: unbounded).  The host thread spins between decisions (no Python in the loop). */
 tacker_status tacker_manager_run(tacker_manager_t m, double qos_target_ms, double t_end_ms, int64_t max_decisions);
+/* Steady-state windows (§VIII-B): steps the manager like
+ * tacker_manager_run but returns as soon as its clock reaches t_until_ms, WITHOUT draining the
+ * queries or synchronising the stream, so a caller can mark a measurement window (an event on
+ * the manager stream + tacker_manager_stats_get) inside one continuous Poisson run and resume. */
+tacker_status tacker_manager_run_until(tacker_manager_t m, double qos_target_ms, double t_until_ms);
+
+/* Decision trace (for the discrete-event reference's replay of a GPU-mode run, SURVEY §8(c)
+ * c15): one record per decision that launched something, with the observations the decision
+ * was taken on -- the manager clock, the active queries (arrival order) and, per BE app, the
+ * predicted fused duration Tk_fuse Eq. 8 evaluated (NaN where none was evaluated or no model
+ * exists).  Records beyond the capacity are counted in *dropped, not stored. */
+#define TACKER_TRACE_MAX_APPS 16
+#define TACKER_TRACE_MAX_ACTIVE 64
+typedef struct {
+  double t_ms;                                  /* manager clock at the decision */
+  int32_t n_active;                             /* active queries (may exceed the stored ids) */
+  int32_t active[TACKER_TRACE_MAX_ACTIVE];      /* their ids, oldest first */
+  int32_t direct;                               /* the decided query runs direct (Thr close to 0) */
+  int32_t n_apps;
+  uint32_t ready_mask;                          /* bit a: BE app a's head was ready (always, on the GPU) */
+  double tk_fuse_ms[TACKER_TRACE_MAX_APPS];
+  tacker_decision d;                            /* as tacker_manager_step returned it */
+} tacker_trace_rec;
+/* capacity 0 disables tracing (default); enabling clears the trace */
+tacker_status tacker_manager_trace_enable(tacker_manager_t m, int64_t capacity);
+tacker_status tacker_manager_trace_count(tacker_manager_t m, int64_t *stored, int64_t *dropped);
+tacker_status tacker_manager_trace_get(tacker_manager_t m, int64_t index, tacker_trace_rec *out);
 enum { TACKER_CLASS_LC_TC = 0, TACKER_CLASS_LC_CD = 1, TACKER_CLASS_FUSED = 2, TACKER_CLASS_BE = 3 };
 typedef struct {
   int64_t lc_queries_done, be_kernels_done, fused_launches, original_lc, reordered_be, idle_be;

@@ -8,16 +8,21 @@ Rules, in the paper's order:
     over the remaining predicted GPU time of earlier still-active queries.
     T_queue = time Q waited between arrival and the issue of its first kernel (reading).
   * Only the newest query fuses or reorders; earlier queries' kernels launch directly
-    (P:2058-2072).  Thr "close to 0" -> launch directly: reading Thr <= direct_eps.
+    (P:2058-2072).  "If the Thr of the new query is close to 0, Tacker directly launches all the
+    kernels to the GPU".  Reading (direct_rule DIRECT_MIN_BE, the
+    default): close to 0 = Thr <= max(direct_eps, the smallest predicted time of a ready BE head)
+    at the query's first issue, i.e. not even the shortest ready BE kernel fits; DIRECT_EPS: Thr <=
+    direct_eps only.  A direct query's kernels are all launched plain (no fusion, no reorder).
   * Eq. 8: for the current TC kernel (Ttc) and each ready BE head kernel (Tcd) with a
     fused prediction Tk_fuse: admissible iff Ttc + Tcd > Tk_fuse and Tk_fuse - Ttc < Thr.
     Pick the max Tgain = Tcd - (Tk_fuse - Ttc); ties -> lowest app index.
     Then Thr -= Tk_fuse - Ttc.
-  * Reorder: after the LC kernel (fused or not), launch the other ready BE heads
-    (app index order) whose Ttmp < Thr, Thr -= Ttmp.  Reading: the text applies
-    reorder when no fusion is possible; Tacker is described as using "both adaptive kernel
-    fusion and kernel reorder", so reordering also follows a fused launch and
-    Tacker never reorders less than Baymax.
+  * Reorder (literal, the default reorder_rule REORDER_UNFUSED): "If all the ready
+    BE kernels may not be fused with the current kernel of Q", launch the ready BE heads (app
+    index order) whose Ttmp < Thr, Thr -= Ttmp; after a fused launch nothing is reordered.
+    REORDER_ALWAYS (B200 reading 6, a named option): reorder after every LC kernel,
+    fused or not ("both adaptive kernel fusion and kernel reorder", P:2712-2716).
+    REORDER_NEVER: BE work runs fused or on an idle GPU only.
   * Only the head kernel of each BE app is a candidate; the next kernel of an app
     becomes ready when the previous one completes.
   * Baymax mode = the same manager with fusion disabled ("static scheduling").
@@ -32,8 +37,6 @@ Rules, in the paper's order:
     its last block is issued; reorder and idle launches issue the whole rest, whose predicted
     time is X_cd(remaining) once a slice of it has run.  BE work = n/N of the kernel's
     standalone time per slice.
-  * reorder_only_unfused: 1 = reorder only after an LC kernel that was not fused (P:2035
-    literally); 2 = never reorder (BE work runs fused or on an idle GPU only).
   * Reverse fusion (NEXT-2; "LC and BE kernels are not limited to a specified type",
     P:924-926; DNN-training BE apps, Table II): when the LC kernel is a CUDA-core
     kernel (T_lc) and a ready BE head is a tensor-core kernel (T_be; kind 2 below), the same
@@ -60,6 +63,8 @@ import math
 from dataclasses import dataclass, field
 
 TACKER, BAYMAX = 0, 1
+REORDER_UNFUSED, REORDER_ALWAYS, REORDER_NEVER = 0, 1, 2      # reorder_rule
+DIRECT_MIN_BE, DIRECT_EPS = 0, 1                              # direct_rule
 BE_OTHER, BE_CD, BE_TC = 0, 1, 2
 FUSED, ORIGINAL_LC, REORDER_BE, IDLE_BE, NOTHING = 0, 1, 2, 3, 4
 
@@ -76,7 +81,7 @@ class Decision:
     reverse: bool = False         # fused: LC CUDA-core kernel + BE tensor-core kernel (NEXT-2)
 
 
-def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=None, reorder_only_unfused=False,
+def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=None, reorder_rule=REORDER_UNFUSED,
            reverse=True, with_reverse_flag=False):
     """Pure decision for one LC kernel.
 
@@ -113,7 +118,7 @@ def decide(ttc, lc_is_tc, thr, heads, policy, fuse_pred, allow=True, fuse_tcd=No
     reorder = []
     if fused >= 0:
         thr -= tf_best - ttc
-    if allow and reorder_only_unfused != 2 and not (reorder_only_unfused == 1 and fused >= 0):
+    if allow and reorder_rule != REORDER_NEVER and not (reorder_rule == REORDER_UNFUSED and fused >= 0):
         for app, tcd, _ in heads:
             if app == fused:
                 continue
@@ -191,9 +196,47 @@ def slice_blocks(app, ttc, r_opp, slice_be, slice_ratio):
     return n if n < R else -1
 
 
+def _first_issue(q, active, t, qos, heads, direct_eps, direct_rule, fuse_older):
+    """Eq. 9 at the first issue of q and the direct rule."""
+    q.issue = t
+    if q is active[-1] or fuse_older:
+        earlier = sum(o.remaining() for o in active[:active.index(q)])
+        q.thr = qos - (t - q.arrival) - q.remaining() - earlier
+        bound = direct_eps
+        if direct_rule == DIRECT_MIN_BE and heads:
+            bound = max(bound, min(d for _, d, _ in heads))
+        q.direct = q.thr <= bound
+
+
+def _lc_decision(q, active, t, qos, heads, apps, policy, pred, tcd_of, reorder_rule, reverse, fuse_older,
+                 older_margin):
+    """Eq. 8 / Tgain / reorder for the current kernel of q (the oldest query with work), with the
+    older-query bound of reading 18.  pred(a) -> Tk_fuse or None.  Updates q.thr; returns
+    (fused, reorder, thr_after, gain, rev, allow)."""
+    newest = active[-1]
+    is_tc, ttc = q.kernels[q.pos]
+    allow = (q is newest or fuse_older) and not q.direct and q.thr is not None
+    thr = q.thr if q.thr is not None else 0.0
+    thr_in = thr
+    if allow and q is not newest:
+        ahead = 0.0
+        for j, o in enumerate(active):
+            ahead += o.remaining()
+            if j > active.index(q):
+                thr = min(thr, qos - (t - o.arrival) - ahead)
+        thr -= older_margin
+    thr_eff = thr
+    fused, reorder, thr2, gain, rev = decide(
+        ttc, is_tc, thr, heads, policy, pred, allow, fuse_tcd=tcd_of,
+        reorder_rule=reorder_rule, reverse=reverse, with_reverse_flag=True)
+    if allow:
+        q.thr = thr_in - (thr_eff - thr2)
+    return fused, reorder, (thr2 if allow else thr), gain, rev, allow
+
+
 def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=None, t_end=None,
-             slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_only_unfused=False, reverse=True,
-             rfuse_pred=None, fuse_older=False, older_margin=0.0):
+             slice_be=False, slice_ratio=0.0, opp_ratio=None, reorder_rule=REORDER_UNFUSED, reverse=True,
+             rfuse_pred=None, fuse_older=False, older_margin=0.0, direct_rule=DIRECT_MIN_BE):
     """Serial single-stream GPU whose kernels take exactly their predicted time.
 
     fuse_pred(lc_T, be_T) -> Tk_fuse or None; opp_ratio(app) -> the pair's opportune ratio or
@@ -217,25 +260,9 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
         heads = [(a, app.rem(), app.head()[0]) for a, app in enumerate(apps) if app.ready_at <= t]
         if active:
             q = active[0]
-            newest = active[-1]
             if q.issue is None:
-                q.issue = t
-                if q is newest or fuse_older:
-                    earlier = sum(o.remaining() for o in active[:active.index(q)])
-                    q.thr = qos - (t - q.arrival) - q.remaining() - earlier
-                    q.direct = q.thr <= direct_eps
+                _first_issue(q, active, t, qos, heads, direct_eps, direct_rule, fuse_older)
             is_tc, ttc = q.kernels[q.pos]
-            allow = (q is newest or fuse_older) and not q.direct and q.thr is not None
-            thr = q.thr if q.thr is not None else 0.0
-            thr_in = thr
-            if allow and q is not newest:
-                ahead = 0.0
-                for j, o in enumerate(active):
-                    ahead += o.remaining()
-                    if j > active.index(q):
-                        thr = min(thr, qos - (t - o.arrival) - ahead)
-                thr -= older_margin
-            thr_eff = thr
             nblk = {a: slice_blocks(apps[a], ttc, opp_ratio(a) if opp_ratio else None, slice_be, slice_ratio)
                     for a, _, _ in heads}
 
@@ -254,11 +281,9 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                     return rpred(apps[a].rem(), ttc)
                 return fuse_pred(ttc, tcd_of(a))
 
-            fused, reorder, thr2, gain, rev = decide(
-                ttc, is_tc, thr, heads, policy, pred, allow, fuse_tcd=tcd_of,
-                reorder_only_unfused=reorder_only_unfused, reverse=reverse, with_reverse_flag=True)
-            if allow:
-                q.thr = thr_in - (thr_eff - thr2)
+            fused, reorder, thr_after, gain, rev, allow = _lc_decision(
+                q, active, t, qos, heads, apps, policy, pred, tcd_of, reorder_rule, reverse, fuse_older,
+                older_margin)
             start = t
             if fused >= 0:
                 dur = pred(fused)
@@ -271,7 +296,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 dur = ttc
                 timeline.append(("lc", q.qid, q.pos, -1, start, start + dur))
                 decisions.append(Decision(REORDER_BE if reorder else ORIGINAL_LC, (q.qid, q.pos), -1,
-                                          list(reorder), thr2 if allow else thr))
+                                          list(reorder), thr_after))
             t = start + dur
             q.pos += 1
             if q.pos == len(q.kernels):
@@ -301,3 +326,48 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
     lat = {q.qid: (q.done_at - q.arrival) for q in queries if q.done_at is not None}
     return dict(latency=lat, be_completed=[a.completed for a in apps], be_work=sum(a.work for a in apps),
                 timeline=timeline, decisions=decisions, t=t)
+
+
+def replay(trace, queries, apps, qos, policy, direct_eps=0.0, idle_cap=None, reorder_rule=REORDER_UNFUSED,
+           reverse=True, fuse_older=False, older_margin=0.0, direct_rule=DIRECT_MIN_BE):
+    """Trace-driven reference of a GPU-mode run ("the manager is gated by the
+    discrete-event reference on the recorded trace").  On the GPU the clock, the set of active
+    queries, which BE heads are ready and the online-refitted fused predictions come from the
+    hardware, so they are taken as observations from each trace record: (t, active query ids
+    oldest first, ready app ids, {app: Tk_fuse}).
+    Everything the manager DECIDES -- Eq. 9 at first issue, the direct rule, Eq. 8 admission,
+    max Tgain, Thr updates, reorder, the newest-query rule, idle launches -- is recomputed here
+    with the rules above and the query / app state this function tracks itself.  (On the GPU every
+    BE head is ready: the manager's single stream orders an app's kernels.)  Whole-kernel fusion
+    only (no PTB slices).  Returns the list of Decisions (thr = the headroom after the decision as
+    the manager reports it: the effective bound of an older query under reading 18)."""
+    by_id = {q.qid: q for q in queries}
+    out = []
+    for rec in trace:
+        t, act_ids, tf, ready = rec["t"], rec["active"], rec["tk_fuse"], set(rec["ready"])
+        active = [by_id[i] for i in act_ids]
+        heads = [(a, app.rem(), app.head()[0]) for a, app in enumerate(apps) if a in ready]
+        work = [q for q in active if q.pos < len(q.kernels)]
+        if not work:
+            cands = [a for a, d, _ in heads if (idle_cap is None or d <= idle_cap)] if not active else []
+            a = cands[0] if cands else -1
+            out.append(Decision(IDLE_BE, None, -1, [a] if a >= 0 else [], 0.0))
+            if a >= 0:
+                apps[a].issue(-1)
+            continue
+        q = work[0]
+        if q.issue is None:
+            _first_issue(q, active, t, qos, heads, direct_eps, direct_rule, fuse_older)
+        pred = lambda a: tf.get(a)
+        fused, reorder, thr_after, gain, rev, allow = _lc_decision(
+            q, active, t, qos, heads, apps, policy, pred, None, reorder_rule, reverse, fuse_older, older_margin)
+        if fused >= 0:
+            apps[fused].issue(-1)
+            out.append(Decision(FUSED, (q.qid, q.pos), fused, list(reorder), thr_after, gain, -1, rev))
+        else:
+            out.append(Decision(REORDER_BE if reorder else ORIGINAL_LC, (q.qid, q.pos), -1, list(reorder),
+                                thr_after))
+        q.pos += 1
+        for a in reorder:
+            apps[a].issue(-1)
+    return out

@@ -30,7 +30,11 @@ constexpr int kVbThreads = 128;
 #define TK_FFT_MIN_BLOCKS 8  // fft original grid: 64 registers, no spills with two transforms per block
 #endif
 #ifndef TK_MRIQ_REDUCE
-#define TK_MRIQ_REDUCE 0
+// mri-q / mri-fhd: exact range reduction of the phase in turns, t - rint(t), before the MUFU
+// sin/cos of 2 pi t: |2 pi t| <= pi, where sin.approx / cos.approx hold their
+// 2^-20.9 absolute error bound (the bench's k in [-32, 32) puts |t| up to 48 turns).  Two FADDs
+// per term on the FMA pipe beside the MUFU-bound sin/cos.
+#define TK_MRIQ_REDUCE 1
 #endif
 
 template <int KIND> struct BeBody;

@@ -53,7 +53,11 @@ template <> struct BeBody<TACKER_BE_MRIFHD_FH> {
   static __device__ __forceinline__ void term(const float4 kv, float ri, float x, float y, float z, float &fr,
                                               float &fi) {
     const float kTwoPi = 6.2831853071795864769f;
-    const float t = __fmaf_rn(kv.z, z, __fmaf_rn(kv.y, y, __fmul_rn(kv.x, x)));
+    float t = __fmaf_rn(kv.z, z, __fmaf_rn(kv.y, y, __fmul_rn(kv.x, x)));
+#if TK_MRIQ_REDUCE
+    const float kMagic = 12582912.0f;   // 1.5 * 2^23: (t + M) - M == rint(t) for |t| < 2^22
+    t = __fsub_rn(t, __fsub_rn(__fadd_rn(t, kMagic), kMagic));
+#endif
     float s, c;
     __sincosf(__fmul_rn(kTwoPi, t), &s, &c);
     fr = __fmaf_rn(-ri, s, __fmaf_rn(kv.w, c, fr));

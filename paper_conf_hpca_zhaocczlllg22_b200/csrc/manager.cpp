@@ -3,7 +3,8 @@
 // Per LC kernel of the oldest active query:
 //   * Eq. 9: at the first issue of the newest query Q,
 //       Thr = T_qos - T_queue - T_ori_solo(Q) - sum_i T_lc_i(remaining, earlier queries),
-//     T_queue = issue time - arrival (reading).  Thr <= direct_eps -> Q runs direct.
+//     T_queue = issue time - arrival (reading).  "Thr close to 0" ->
+//     Q runs direct: Thr <= max(direct_eps, shortest ready BE head) (direct_rule MIN_BE, default).
 //   * Only the newest query fuses/reorders; params.fuse_older (reading 18): an older
 //     query too, within min(its Thr, Eq. 9 of every later active query) - older_margin_ms.
 //   * CUDA-core LC kernel (NEXT-2, reading 17): the same Eq. 8 over ready BE tensor-core heads,
@@ -12,7 +13,8 @@
 //       Ttc + Tcd > Tk_fuse  &&  Tk_fuse - Ttc < Thr;  max Tgain = Tcd - (Tk_fuse - Ttc)
 //     (P:2045-2056), ties -> lowest app index; Thr -= Tk_fuse - Ttc.
 //   * Original launch (if not fused), then reorder ready BE heads with Ttmp < Thr:
-//     after every LC kernel (reading 6), only unfused ones (reorder_only_unfused 1) or never (2).
+//     only after an unfused LC kernel (the paper's rule, default), after every LC kernel
+//     (reorder_rule ALWAYS, reading 6) or never.
 //   * Baymax policy: identical with fusion disabled ("static scheduling").
 //   * Idle GPU (paper silent): one ready BE head no longer than idle_cap.
 //   * PTB slicing (params.slice_be, reading 13): a fused launch may carry only a slice of the BE
@@ -138,6 +140,11 @@ struct tacker_manager_s {
   double class_ms[4] = {0, 0, 0, 0};   // summed over the timed sample
   int64_t class_timed[4] = {0, 0, 0, 0};
   int64_t class_n[4] = {0, 0, 0, 0};   // every launch
+
+  std::vector<tacker_trace_rec> trace;   // decision trace (tacker_manager_trace_enable)
+  int64_t trace_cap = 0, trace_dropped = 0;
+  double trace_tf[TACKER_TRACE_MAX_APPS];  // Tk_fuse per app evaluated by the current decision
+  uint32_t trace_ready = 0;                // BE apps whose head was ready at the current decision
 
   double host_ns[3] = {0, 0, 0};   // poll, launch + event calls, whole step
   int64_t host_steps = 0;
@@ -497,9 +504,9 @@ tacker_status tacker_manager_set_clock(tacker_manager_t m, double now_ms) {
   return TACKER_OK;
 }
 
-tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headroom, tacker_decision *out) {
-  if (!m || !out) return set_error("null argument"), TACKER_EINVAL;
+static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom, tacker_decision *out) {
   HostTimer ht(m->host_ns[2]);
+  for (double &x : m->trace_tf) x = NAN;
   m->host_steps++;
   memset(out, 0, sizeof *out);
   out->action = TACKER_DEC_NOTHING;
@@ -527,8 +534,12 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       break;
     }
   std::vector<int> heads;
+  m->trace_ready = 0;
   for (size_t a = 0; a < m->apps.size(); ++a)
-    if (app_ready(m, m->apps[a], t)) heads.push_back((int)a);
+    if (app_ready(m, m->apps[a], t)) {
+      heads.push_back((int)a);
+      if (a < TACKER_TRACE_MAX_APPS) m->trace_ready |= 1u << a;
+    }
 
   if (qid < 0) {
     // idle GPU (or only tails of earlier queries still running): one bounded BE kernel
@@ -578,7 +589,15 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       }
       q.thr = qos - (t - q.arrival) - q.remaining() - earlier;   // Eq. 9
       q.has_thr = true;
-      q.direct = q.thr <= m->prm.direct_eps_ms;
+      // "Thr close to 0": reading TACKER_DIRECT_MIN_BE = not even the shortest
+      // ready BE head fits the headroom
+      double bound = m->prm.direct_eps_ms;
+      if (m->prm.direct_rule == TACKER_DIRECT_MIN_BE && !heads.empty()) {
+        double mn = INFINITY;
+        for (int a : heads) mn = std::min(mn, rem_ms(m->apps[a]));
+        bound = std::max(bound, mn);
+      }
+      q.direct = q.thr <= bound;
     }
   }
   const bool allow = (newest || older_ok) && q.has_thr && !q.direct;
@@ -616,6 +635,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       const double tcd = n < 0 ? rem_ms(A) : slice_ms(b, n);
       double tf;
       if (!pair_predict(pk, ttc, tcd, &tf)) continue;
+      if (a < TACKER_TRACE_MAX_APPS) m->trace_tf[a] = tf;
       if (ttc + tcd > tf && tf - ttc < thr) {   // Eq. 8
         const double gain = tcd - (tf - ttc);
         if (fused < 0 || gain > best_gain) {
@@ -641,6 +661,7 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
       const double tbe = b.t_pred_ms;
       double tf;
       if (!pair_predict(pk, tbe, ttc, &tf)) continue;
+      if (a < TACKER_TRACE_MAX_APPS) m->trace_tf[a] = tf;
       if (ttc + tbe > tf && tf - ttc < thr) {   // Eq. 8
         const double gain = tbe - (tf - ttc);
         if (fused < 0 || gain > best_gain) {
@@ -656,10 +677,11 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   }
   std::vector<int> reorder;
   if (fused >= 0) thr -= best_tf - ttc;
-  // Reorder the remaining ready heads after the LC kernel, fused or not (reading:
-  // Tacker = fusion on top of Baymax's reordering, "both adaptive kernel fusion and kernel
-  // reorder"); reorder_only_unfused = the literal P:2035 rule.
-  if (allow && m->prm.reorder_only_unfused != 2 && !(m->prm.reorder_only_unfused == 1 && fused >= 0)) {
+  // Reorder: the ready heads with Ttmp < Thr after an LC kernel that was not fused
+  // (the paper's rule, TACKER_REORDER_UNFUSED); TACKER_REORDER_ALWAYS (reading 6) also after a
+  // fused launch ("both adaptive kernel fusion and kernel reorder").
+  const int32_t rr = m->prm.reorder_rule;
+  if (allow && rr != TACKER_REORDER_NEVER && !(rr == TACKER_REORDER_UNFUSED && fused >= 0)) {
     for (int a : heads) {
       if (a == fused) continue;
       const double tt = rem_ms(m->apps[a]);
@@ -752,6 +774,50 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   return TACKER_OK;
 }
 
+tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headroom, tacker_decision *out) {
+  if (!m || !out) return set_error("null argument"), TACKER_EINVAL;
+  tacker_status s = step_impl(m, qos, headroom, out);
+  if (s != TACKER_OK || m->trace_cap <= 0 || out->action == TACKER_DEC_NOTHING) return s;
+  if ((int64_t)m->trace.size() >= m->trace_cap) {
+    m->trace_dropped++;
+    return s;
+  }
+  tacker_trace_rec r;
+  memset(&r, 0, sizeof r);
+  r.t_ms = out->t_start_ms;
+  r.n_active = (int32_t)m->active.size();
+  for (size_t i = 0; i < m->active.size() && i < TACKER_TRACE_MAX_ACTIVE; ++i) r.active[i] = m->active[i];
+  r.direct = out->query >= 0 && m->queries[out->query].direct ? 1 : 0;
+  r.n_apps = (int32_t)std::min<size_t>(m->apps.size(), TACKER_TRACE_MAX_APPS);
+  r.ready_mask = m->trace_ready;
+  for (int a = 0; a < TACKER_TRACE_MAX_APPS; ++a) r.tk_fuse_ms[a] = m->trace_tf[a];
+  r.d = *out;
+  m->trace.push_back(r);
+  return s;
+}
+
+tacker_status tacker_manager_trace_enable(tacker_manager_t m, int64_t capacity) {
+  if (!m || capacity < 0) return set_error("bad trace capacity"), TACKER_EINVAL;
+  m->trace.clear();
+  m->trace.reserve((size_t)capacity);
+  m->trace_cap = capacity;
+  m->trace_dropped = 0;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_trace_count(tacker_manager_t m, int64_t *stored, int64_t *dropped) {
+  if (!m || !stored || !dropped) return set_error("null argument"), TACKER_EINVAL;
+  *stored = (int64_t)m->trace.size();
+  *dropped = m->trace_dropped;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_trace_get(tacker_manager_t m, int64_t i, tacker_trace_rec *out) {
+  if (!m || !out || i < 0 || i >= (int64_t)m->trace.size()) return set_error("bad trace index"), TACKER_EINVAL;
+  *out = m->trace[(size_t)i];
+  return TACKER_OK;
+}
+
 // Fused handles of every (TC kernel in ks, CUDA-core kernel of a BE app) pair the predictor has
 // a model for: the only pairs Eq. 8 can admit.  Queries of one service share their kernels, so
 // only LC operand triples not seen before are visited.
@@ -819,6 +885,22 @@ tacker_status tacker_manager_run(tacker_manager_t m, double qos, double t_end_ms
   if (!m->sim()) {
     cudaError_t e = cudaStreamSynchronize(m->stream);
     if (e != cudaSuccess) return cuda_fail("manager run sync", e);
+    poll(m);
+  }
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_run_until(tacker_manager_t m, double qos, double t_until_ms) {
+  if (!m) return set_error("null manager"), TACKER_EINVAL;
+  if (tacker_status s = tacker_manager_prepare(m, nullptr)) return s;
+  tacker_decision d;
+  for (;;) {
+    if ((m->sim() ? m->now : host_now(m)) >= t_until_ms) break;
+    double thr = NAN;
+    if (tacker_status s = tacker_manager_step(m, qos, &thr, &d)) return s;
+    if (m->sim() && d.action == TACKER_DEC_NOTHING && m->next_pending >= m->pending.size() &&
+        m->st.lc_queries_done == (int64_t)m->queries.size())
+      break;   // nothing left to simulate
     poll(m);
   }
   return TACKER_OK;

@@ -22,6 +22,40 @@ import torch
 from . import tacker as tk
 
 
+CLASSES = ("lc_tc", "lc_cd", "fused", "be")
+
+
+def _rules_name(policy, rules):
+    """Which manager rules a run used, by name (DESIGN.md §2 readings)."""
+    rr = rules.get("reorder_rule", tk.REORDER_UNFUSED)
+    parts = ["reorder: " + {tk.REORDER_UNFUSED: "only after an unfused LC kernel (P:2035)",
+                            tk.REORDER_ALWAYS: "after every LC kernel (reading 6)",
+                            tk.REORDER_NEVER: "never"}[rr]]
+    parts.append("older queries fuse/reorder within later queries' headroom (reading 18)" if rules.get("fuse_older")
+                 else "only the newest query fuses/reorders (P:2058-2072)")
+    if rules.get("slice_be"):
+        parts.append("PTB slices at r* (reading 13)")
+    parts.append("direct when Thr <= " + ("eps" if rules.get("direct_rule") == tk.DIRECT_EPS
+                                           else "the shortest ready BE head (P:2092-2096, c15)"))
+    return ("Tacker" if policy == tk.POLICY_TACKER else "Baymax (fusion off)") + "; " + "; ".join(parts)
+
+
+def latency_stats(lat, qos, boot=1000, seed=0):
+    """p50 / p99 (nearest rank) of query latencies, with a bootstrap 95 % CI of p99."""
+    lat = np.sort(np.asarray(lat, dtype=np.float64))
+    n = len(lat)
+    if n == 0:
+        return {"lc_p50_ms": None, "lc_p99_ms": None, "lc_p99_ci95_ms": None, "lc_max_ms": None,
+                "qos_met": False, "violations": 0}
+    k = min(n - 1, int(math.ceil(0.99 * n)) - 1)
+    rng = np.random.default_rng(seed)
+    bs = np.sort(lat[rng.integers(0, n, size=(boot, n))], axis=1)[:, k]
+    return {"lc_p50_ms": float(np.median(lat)), "lc_p99_ms": float(lat[k]),
+            "lc_p99_ci95_ms": [float(np.percentile(bs, 2.5)), float(np.percentile(bs, 97.5))],
+            "lc_mean_ms": float(lat.mean()), "lc_max_ms": float(lat[-1]),
+            "qos_met": bool(lat[k] <= qos), "violations": int((lat > qos).sum())}
+
+
 def overlap_rate(t_tc, t_cd, t_corun):
     """Eq. 11 (P:3315-3320): (T_TC + T_CD - T_corun) / (T_TC + T_CD) -- 0 for sequential
     execution, 0.5 for perfect overlap of equal parts."""
@@ -355,6 +389,17 @@ class QosRun:
             out.append(ks)
         return out
 
+    def replay_inputs(self, arrivals):
+        """(queries, apps) in the form tests/trace_check.check_trace takes: the predicted times the
+        manager was given (every query of a run has the same kernels)."""
+        ks = [(bool(k.is_tc), k.t_pred_ms) for k in self.lc_kernels()]
+        queries = [(float(a), list(ks)) for a in arrivals]
+        apps = [[(2 if b.is_tc else (1 if b.is_cd else 0), b.t_pred_ms) for b in app] for app in self.be_apps()]
+        return queries, apps
+
+    def idle_cap(self):
+        return max(0.5 * (self.qos - self.query_solo_ms()), 0.0)
+
     def query_solo_ms(self):
         return sum(self.t_lc)
 
@@ -378,10 +423,121 @@ class QosRun:
         self.service_ms = e0.elapsed_time(e1) / n
         return self.service_ms
 
+    # ------------------------------------------------------------------ steady-state window
+    def _manager(self, policy, stream, max_inflight, idle_cap_ms, slice_be=False, slice_ratio=0.0,
+                 reorder_rule=tk.REORDER_UNFUSED, reverse_fusion=True, fuse_older=False, older_margin_ms=None,
+                 direct_rule=tk.DIRECT_MIN_BE, lc_only=False):
+        cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
+        m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
+                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_rule=reorder_rule,
+                       reverse_fusion=reverse_fusion, fuse_older=fuse_older,
+                       older_margin_ms=0.3 * self.qos if older_margin_ms is None else older_margin_ms,
+                       direct_rule=direct_rule)
+        if not lc_only:
+            for ks in self.be_apps():
+                m.submit_be(ks)
+        return m
+
+    def find_peak_load(self, window_ms, warm_ms=200.0, lo=0.5, hi=1.0, iters=5, seed=4242, max_inflight=4):
+        """lambda_peak ("the peak load that meets QoS"): bisection on the load
+        fraction of the LC-only service rate (1 / service_ms) with LC-only windowed runs (no BE
+        apps), criterion p99 <= QoS.  Rates above the service rate are not sustainable, so the
+        search is capped at it.  Returns (peak load fraction, [(load, p99)])."""
+        hist = []
+
+        def ok(load):
+            r = self.run_window(tk.POLICY_BAYMAX, window_ms, warm_ms, load=load, seed=seed,
+                                max_inflight=max_inflight, lc_only=True)
+            hist.append((load, r["lc_p99_ms"]))
+            return r["qos_met"]
+
+        if ok(hi):
+            self.peak_load = hi
+            return hi, hist
+        for _ in range(iters):
+            mid = 0.5 * (lo + hi)
+            if ok(mid):
+                lo = mid
+            else:
+                hi = mid
+        self.peak_load = lo
+        return lo, hist
+
+    def run_window(self, policy, window_ms, warm_ms, tail_ms=None, load=0.8, seed=1000, max_inflight=4,
+                   idle_cap_ms=None, sync=None, trace=False, lc_only=False, **rules):
+        """Steady-state measurement: ONE continuous Poisson run of
+        warm_ms + window_ms + tail_ms at `load` x the peak rate; the manager runs natively up to
+        the window start (tacker_manager_run_until: no drain, no sync), the window is bracketed by
+        CUDA events on the manager stream (after a stream sync and `sync()`, e.g. a barrier, at its
+        start and end), then the run continues through the tail (arrivals keep coming while the
+        window's last queries finish) and drains.  Reported over the window only: BE kernels and
+        BE work issued inside it / its device time, and the latency of every query that ARRIVED
+        inside it (p50 / p99 nearest rank, bootstrap 95 % CI of p99).  The ramp-up and drain are
+        outside the window, so the result does not depend on the run length."""
+        stream = torch.cuda.current_stream()
+        torch.cuda.synchronize()
+        tail_ms = self.qos * 1.5 if tail_ms is None else tail_ms
+        lam = load / getattr(self, "service_ms", self.query_solo_ms())     # queries per ms
+        rng = np.random.default_rng(seed)
+        m = self._manager(policy, stream, max_inflight, idle_cap_ms, lc_only=lc_only, **rules)
+        if trace:
+            m.trace_enable(4_000_000)
+        kernels = self.lc_kernels()
+        m.prepare(kernels)
+        t0 = m.stats().now_ms + 2.0
+        w0, w1 = t0 + warm_ms, t0 + warm_ms + window_ms
+        t_end = w1 + tail_ms
+        arr, t = [], t0
+        while True:
+            t += rng.exponential(1.0 / lam)
+            if t >= t_end:
+                break
+            arr.append(t)
+        qids = [m.submit_lc(kernels, float(a)) for a in arr]
+        m.run_until(self.qos, w0)
+        torch.cuda.synchronize()
+        if sync:
+            sync()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0 = m.stats()
+        e0.record(stream)
+        m.run_until(self.qos, w1)
+        e1.record(stream)
+        s1 = m.stats()
+        torch.cuda.synchronize()
+        if sync:
+            sync()
+        m.run(self.qos, float(arr[-1]) if arr else w1)
+        gpu_ms = e0.elapsed_time(e1)
+        inwin = [q for q, a in zip(qids, arr) if w0 <= a < w1]
+        lat = np.array([m.latency(q) for q in inwin])
+        st = m.stats()
+        d = lambda f: getattr(s1, f) - getattr(s0, f)
+        be = d("be_kernels_done")
+        out = {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "rules": _rules_name(policy, rules),
+               "queries": int(len(lat)), "lambda_per_s": lam * 1e3, "load": load,
+               "window_ms": window_ms, "warm_ms": warm_ms, "tail_ms": tail_ms, "elapsed_ms": gpu_ms,
+               "be_kernels": int(be), "be_kernels_per_s": be / (gpu_ms / 1e3),
+               "be_work_ms": d("be_work_ms"), "be_norm_thpt": d("be_work_ms") / gpu_ms,
+               "fused": int(d("fused_launches")), "reverse_fused": int(d("reverse_fused")),
+               "reordered": int(d("reordered_be")), "idle_be": int(d("idle_be")),
+               "model_refits": int(st.model_refits),
+               "fused_pred_err_mean": st.pred_err_sum / st.pred_err_n if st.pred_err_n else None,
+               "class_ms": {n: float(s1.class_ms[c] - s0.class_ms[c]) for c, n in enumerate(CLASSES)},
+               "class_launches": {n: int(s1.class_launches[c] - s0.class_launches[c]) for c, n in enumerate(CLASSES)},
+               "qos_ms": self.qos, "query_solo_ms": self.query_solo_ms(),
+               "service_ms": getattr(self, "service_ms", None), "max_inflight": max_inflight,
+               "host_decide_us_per_step": (st.host_decide_ms * 1e3 / st.host_steps) if st.host_steps else None}
+        out.update(latency_stats(lat, self.qos))
+        if trace:
+            out["trace"], out["trace_dropped"] = m.trace_dicts()
+            out["arrivals"] = list(arr)
+        return out
+
     # ------------------------------------------------------------------ one managed run
     def run(self, policy, n_queries, load=0.8, seed=1000, warmup=0, max_inflight=4, idle_cap_ms=None,
-            slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True, fuse_older=False,
-            older_margin_ms=None):
+            slice_be=False, slice_ratio=0.0, reorder_rule=tk.REORDER_UNFUSED, reverse_fusion=True, fuse_older=False,
+            older_margin_ms=None, direct_rule=tk.DIRECT_MIN_BE):
         """Poisson arrivals at `load` x the service's peak rate (1 / standalone query time; the
         paper's 80 % of the peak QoS-safe load).  Returns a result dict."""
         stream = torch.cuda.current_stream()
@@ -393,9 +549,10 @@ class QosRun:
         gaps = rng.exponential(1.0 / lam, n_queries + warmup)
         cap = idle_cap_ms if idle_cap_ms is not None else 0.5 * (self.qos - self.query_solo_ms())
         m = tk.Manager(policy, stream=stream, simulate=False, idle_cap_ms=max(cap, 0.0), max_inflight=max_inflight,
-                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_only_unfused=reorder_only_unfused,
+                       slice_be=slice_be, slice_ratio=slice_ratio, reorder_rule=reorder_rule,
                        reverse_fusion=reverse_fusion, fuse_older=fuse_older,
-                       older_margin_ms=0.3 * self.qos if older_margin_ms is None else older_margin_ms)
+                       older_margin_ms=0.3 * self.qos if older_margin_ms is None else older_margin_ms,
+                       direct_rule=direct_rule)
         for ks in self.be_apps():
             m.submit_be(ks)
         kernels = self.lc_kernels()
@@ -414,7 +571,7 @@ class QosRun:
         lat_sorted = np.sort(lat)
         p99 = float(lat_sorted[min(len(lat) - 1, int(math.ceil(0.99 * len(lat))) - 1)])
         return {"policy": "tacker" if policy == tk.POLICY_TACKER else "baymax", "slice_be": bool(slice_be),
-                "reorder_only_unfused": int(reorder_only_unfused), "queries": int(len(lat)),
+                "reorder_rule": int(reorder_rule), "queries": int(len(lat)),
                 "lambda_per_s": lam * 1e3, "load": load, "elapsed_ms": gpu_ms,
                 "be_kernels": int(st.be_kernels_done), "be_kernels_per_s": st.be_kernels_done / (gpu_ms / 1e3),
                 # normalised BE throughput: standalone-milliseconds of BE work per wall millisecond

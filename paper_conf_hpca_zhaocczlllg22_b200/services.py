@@ -32,6 +32,7 @@ class LcKernelSpec:
     flops: int = 0
     bytes: int = 0
     conv: synth.ConvShape | None = None
+    out: object = None      # the kernel's output tensor (parity tests read it)
 
 
 @dataclass
@@ -71,7 +72,7 @@ def resnet50_service(batch: int = 1, seed: int = 2022, convs=None, conv1_im2col:
         if cs.c % 64 == 0 or (cs.r == 1 and cs.s == 1 and cs.stride == 1) or (cs.c == 8 and not conv1_im2col):
             lc = tk.lc_conv(dx, dw, out, cs.stride, cs.pad, bias=db, relu=True, b_const=True)
             ks.append(LcKernelSpec(cs.name, True, lc=lc,
-                                   flops=2 * M * N * K, bytes=byt, conv=cs))
+                                   flops=2 * M * N * K, bytes=byt, conv=cs, out=out))
             bufs += [dx, dw, db, out]
         else:   # conv1: explicit im2col (LC CD kernel) + GEMM (LC TC kernel)
             Kpad = ((K + 63) // 64) * 64
@@ -81,11 +82,12 @@ def resnet50_service(batch: int = 1, seed: int = 2022, convs=None, conv1_im2col:
             dwf = _dev(wf)
             ks.append(LcKernelSpec(cs.name + ".im2col", False,
                                    cd=tk.be_im2col(dx, cols, cs.r, cs.s, cs.stride, cs.pad, Kpad),
-                                   bytes=2 * x.size + 2 * M * Kpad, conv=cs))
+                                   bytes=2 * x.size + 2 * M * Kpad, conv=cs, out=cols))
             ks.append(LcKernelSpec(cs.name + ".gemm", True,
                                    lc=tk.lc_gemm(cols, dwf, out.view(M, cs.k), M=M, N=cs.k, K=Kpad, bias=db, relu=True,
                                                  b_const=True),
-                                   flops=2 * M * N * K, bytes=2 * M * Kpad + 2 * wf.size + 2 * out.numel(), conv=cs))
+                                   flops=2 * M * N * K, bytes=2 * M * Kpad + 2 * wf.size + 2 * out.numel(), conv=cs,
+                                   out=out))
             bufs += [dx, dw, db, out, cols, dwf]
     return LcService(f"resnet50_b{batch}", ks, bufs, ins, outs[-1:])
 
@@ -339,3 +341,32 @@ def sgemm_app(M=2048, N=2048, K=2048, seed=2022) -> BeAppSpec:
     return BeAppSpec(f"sgemm_{M}x{N}x{K}", [BeKernelSpec("sgemm", tk.be_sgemm(dA, dB, Cm), flops=2.0 * M * N * K,
                                                           bytes=4.0 * (M * K + K * N + M * N), bound="fma")],
                      [dA, dB, Cm])
+
+
+TABLE2_BE = ("mriq", "fft", "mrifhd", "cutcp", "cp", "sgemm", "lbm", "tpacf")
+
+
+def be_apps(names, seed=2022) -> list:
+    """BE applications by name.  TABLE2_BE = the paper's Table II BE set, the mixed
+    queue of BASELINE configs[3]."""
+    make = {"stencil": lambda: stencil_app(512, 512, 64, seed), "mriq": lambda: mriq_app(64, 2048, 1024, seed),
+            "mrifhd": lambda: mrifhd_app(64, 2048, 1024, seed), "cp": lambda: cp_app(seed=seed),
+            "fft": lambda: fft_app(seed=seed), "tpacf": lambda: tpacf_app(seed=seed),
+            "sgemm": lambda: sgemm_app(2048, 2048, 2048, seed), "lbm": lambda: lbm_app(seed=seed),
+            "cutcp": lambda: cutcp_app(seed=seed), "spmv": lambda: spmv_app(seed=seed),
+            "histo": lambda: histo_app(seed=seed), "bfs": lambda: bfs_app(seed=seed)}
+    out = []
+    for n in names:
+        if n not in make:
+            raise ValueError(f"unknown BE app {n!r}")
+        out.append(make[n]())
+    return out
+
+
+def prime_apps(apps) -> None:
+    """Run the one-time setup kernels an app's cycle depends on (mri-q phiMag, mri-fhd RhoPhi) so
+    that its chunk kernels read initialised data from the first launch on."""
+    for a in apps:
+        for k in a.kernels:
+            if k.name in ("mriq.phimag", "mrifhd.rhophi"):
+                tk.tacker_launch_original(None, k.desc)

@@ -217,8 +217,12 @@ class Decision(C.Structure):
 class ManagerParams(C.Structure):
     _fields_ = [("direct_eps_ms", C.c_double), ("idle_cap_ms", C.c_double), ("max_inflight", C.c_int32),
                 ("simulate", C.c_int32), ("slice_be", C.c_int32), ("slice_ratio", C.c_double),
-                ("reorder_only_unfused", C.c_int32), ("no_reverse_fusion", C.c_int32), ("fuse_older", C.c_int32),
-                ("older_margin_ms", C.c_double)]
+                ("reorder_rule", C.c_int32), ("no_reverse_fusion", C.c_int32), ("fuse_older", C.c_int32),
+                ("older_margin_ms", C.c_double), ("direct_rule", C.c_int32)]
+
+
+REORDER_UNFUSED, REORDER_ALWAYS, REORDER_NEVER = 0, 1, 2     # tacker_manager_params.reorder_rule
+DIRECT_MIN_BE, DIRECT_EPS = 0, 1                             # tacker_manager_params.direct_rule
 
 
 class ManagerStats(C.Structure):
@@ -231,6 +235,14 @@ class ManagerStats(C.Structure):
 
 
 CLASS_LC_TC, CLASS_LC_CD, CLASS_FUSED, CLASS_BE = range(4)
+TRACE_MAX_APPS, TRACE_MAX_ACTIVE = 16, 64
+
+
+class TraceRec(C.Structure):
+    _fields_ = [("t_ms", C.c_double), ("n_active", C.c_int32), ("active", C.c_int32 * TRACE_MAX_ACTIVE),
+                ("direct", C.c_int32), ("n_apps", C.c_int32), ("ready_mask", C.c_uint32),
+                ("tk_fuse_ms", C.c_double * TRACE_MAX_APPS),
+                ("d", Decision)]
 
 
 # ----------------------------------------------------------------------------- prototypes
@@ -268,6 +280,10 @@ _PROTOS = {
     "tacker_manager_run": ([_V, _D, _D, _I64], C.c_int),
     "tacker_manager_prepare": ([_V, _V], C.c_int),
     "tacker_manager_query_latency": ([_V, _I32, C.POINTER(_D)], C.c_int),
+    "tacker_manager_run_until": ([_V, _D, _D], C.c_int),
+    "tacker_manager_trace_enable": ([_V, _I64], C.c_int),
+    "tacker_manager_trace_count": ([_V, C.POINTER(_I64), C.POINTER(_I64)], C.c_int),
+    "tacker_manager_trace_get": ([_V, _I64, C.POINTER(TraceRec)], C.c_int),
 }
 for _name, (_args, _res) in _PROTOS.items():
     _f = getattr(_lib, _name)
@@ -660,12 +676,13 @@ class Manager:
     """Owning wrapper of tacker_manager_t."""
 
     def __init__(self, policy=POLICY_TACKER, stream=None, simulate=False, direct_eps_ms=0.0, idle_cap_ms=0.0,
-                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_only_unfused=False, reverse_fusion=True,
-                 fuse_older=False, older_margin_ms=0.0):
+                 max_inflight=2, slice_be=False, slice_ratio=0.0, reorder_rule=REORDER_UNFUSED, reverse_fusion=True,
+                 fuse_older=False, older_margin_ms=0.0, direct_rule=DIRECT_MIN_BE):
         self.h = C.c_void_p()
         self.params = ManagerParams(direct_eps_ms, idle_cap_ms, max_inflight, 1 if simulate else 0,
-                                    1 if slice_be else 0, slice_ratio, int(reorder_only_unfused),
-                                    0 if reverse_fusion else 1, 1 if fuse_older else 0, older_margin_ms)
+                                    1 if slice_be else 0, slice_ratio, int(reorder_rule),
+                                    0 if reverse_fusion else 1, 1 if fuse_older else 0, older_margin_ms,
+                                    int(direct_rule))
         _chk(_lib.tacker_manager_create(policy, C.byref(self.params), _stream(stream), C.byref(self.h)))
         self._keep = []
 
@@ -711,6 +728,41 @@ class Manager:
     def run(self, qos_ms, t_end_ms=0.0, max_decisions=0):
         """Native loop: decide + launch until t_end_ms has passed and all queries completed."""
         _chk(_lib.tacker_manager_run(self.h, qos_ms, t_end_ms, max_decisions))
+
+    def run_until(self, qos_ms, t_until_ms):
+        """Native loop up to manager clock t_until_ms, no drain / no sync (measurement windows)."""
+        _chk(_lib.tacker_manager_run_until(self.h, qos_ms, t_until_ms))
+
+    def trace_enable(self, capacity):
+        _chk(_lib.tacker_manager_trace_enable(self.h, int(capacity)))
+
+    def trace(self):
+        """[TraceRec] recorded decisions and the count dropped beyond the capacity."""
+        n, dropped = C.c_int64(), C.c_int64()
+        _chk(_lib.tacker_manager_trace_count(self.h, C.byref(n), C.byref(dropped)))
+        out = []
+        for i in range(n.value):
+            r = TraceRec()
+            _chk(_lib.tacker_manager_trace_get(self.h, i, C.byref(r)))
+            out.append(r)
+        return out, dropped.value
+
+    def trace_dicts(self):
+        """The trace as plain records for oracle/manager_ref.replay: t, active ids, ready apps,
+        {app: Tk_fuse}, and the decision (action, query, lc_index, fused_app, reorder, thr)."""
+        recs, dropped = self.trace()
+        out = []
+        for r in recs:
+            if r.n_active > TRACE_MAX_ACTIVE:
+                raise TackerError(EINVAL, "trace record with more active queries than stored")
+            tf = {a: r.tk_fuse_ms[a] for a in range(r.n_apps) if not math.isnan(r.tk_fuse_ms[a])}
+            d = r.d
+            out.append({"t": r.t_ms, "active": list(r.active[:r.n_active]),
+                        "ready": [a for a in range(r.n_apps) if (r.ready_mask >> a) & 1], "tk_fuse": tf,
+                        "direct": bool(r.direct), "action": d.action, "query": d.query, "lc_index": d.lc_index,
+                        "fused_app": d.fused_app, "reorder": list(d.reorder_apps[:d.n_reorder]),
+                        "thr": d.thr_ms, "gain": d.gain_ms, "reverse": bool(d.reverse)})
+        return out, dropped
 
     def stats(self) -> ManagerStats:
         s = ManagerStats()

@@ -2,6 +2,7 @@
 header declares, ctypes struct layouts equal the C compiler's, host-only calls (predictor,
 simulated manager) agree with the oracle, and GPU-needing calls fail loudly without a GPU."""
 import ctypes as C
+import json
 import math
 import os
 import re
@@ -50,6 +51,7 @@ STRUCTS = {
     "tacker_fused_info_t": "FusedInfo",
     "tacker_lc_kernel": "LcKernel", "tacker_be_kernel": "BeKernel", "tacker_decision": "Decision",
     "tacker_manager_params": "ManagerParams", "tacker_manager_stats": "ManagerStats", "tacker_ratio": "Ratio",
+    "tacker_trace_rec": "TraceRec",
 }
 
 
@@ -194,7 +196,8 @@ def fit_pair_closed_form(tk, tau):
     return key
 
 
-@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse", "tacker_older", "tacker_noreorder"])
+@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse", "tacker_older", "tacker_noreorder",
+                                    "tacker_reorder_always", "tacker_older_always", "tacker_direct_eps"])
 def test_manager_simulation_matches_reference(tk, policy):
     tk.tacker_model_clear()
     # stage-2 slope != 1 so that Tgain depends on Tcd (with slope 1 every stage-2 pair has the
@@ -214,12 +217,15 @@ def test_manager_simulation_matches_reference(tk, policy):
     app_ts = [[1.53, 0.71], [3.07], [0.43, 0.37, 2.51]]
     tc_apps = [[0.47, 1.12], [0.81]] if reverse else []
     pol = tk.POLICY_BAYMAX if policy == "baymax" else tk.POLICY_TACKER
-    older = policy in ("tacker_older", "tacker_noreorder")
-    noreorder = 2 if policy == "tacker_noreorder" else 0
+    older = policy in ("tacker_older", "tacker_noreorder", "tacker_older_always")
+    rule = {"tacker_noreorder": mr.REORDER_NEVER, "tacker_reorder_always": mr.REORDER_ALWAYS,
+            "tacker_older_always": mr.REORDER_ALWAYS}.get(policy, mr.REORDER_UNFUSED)
+    noreorder = rule == mr.REORDER_NEVER
+    drule = mr.DIRECT_EPS if policy == "tacker_direct_eps" else mr.DIRECT_MIN_BE
     if older:   # a denser trace so that queries queue behind each other
         arrivals = np.cumsum(rng.exponential(3.3, 60))
     m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0, fuse_older=older, older_margin_ms=0.7 if older else 0.0,
-                   reorder_only_unfused=noreorder)
+                   reorder_rule=rule, direct_rule=drule)
     qs = []
     for i, t in enumerate(arrivals):
         sh = shapes[i % 2]
@@ -234,7 +240,7 @@ def test_manager_simulation_matches_reference(tk, policy):
         apps.append(mr.App([(mr.BE_TC, d) for d in ts]))
     ref = mr.simulate(qs, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER, fuse_pred, idle_cap=2.0,
                       rfuse_pred=rfuse_pred, fuse_older=older, older_margin=0.7 if older else 0.0,
-                      reorder_only_unfused=noreorder)
+                      reorder_rule=rule, direct_rule=drule)
     if noreorder:
         assert all(not x.reorder for x in ref["decisions"] if x.action != mr.IDLE_BE)
     if older and not noreorder:   # older queries did fuse, which the paper-literal rule forbids
@@ -278,7 +284,7 @@ def be_kernel_sliced(tk, t, n, floor, ws=16):
     return b
 
 
-@pytest.mark.parametrize("mode", ["opportune", "fixed", "opportune_literal"])
+@pytest.mark.parametrize("mode", ["opportune", "fixed", "opportune_always"])
 def test_manager_slicing_matches_reference(tk, mode):
     """PTB slicing (reading 13): the C manager's decisions (incl. slice sizes), latencies and BE
     work equal the discrete-event reference's."""
@@ -287,13 +293,13 @@ def test_manager_slicing_matches_reference(tk, mode):
     fit_pair_closed_form(tk, tau)
     fuse_pred = lambda ttc, tcd: ttc * tau(tcd / ttc)
     ratio = 1.3 if mode == "fixed" else 0.0
-    literal = mode == "opportune_literal"
+    rule = mr.REORDER_ALWAYS if mode == "opportune_always" else mr.REORDER_UNFUSED
     rng = np.random.default_rng(5)
     arrivals = np.cumsum(rng.exponential(7.0, 50))
     shapes = [[(True, 1.21), (False, 0.3), (True, 0.83), (True, 1.97)], [(True, 0.52), (True, 0.49)]]
     app_ts = [[(1.53, 64, 0.05), (0.71, 0, 0.0)], [(3.07, 200, 0.11)], [(0.43, 1, 0.4), (2.51, 37, 0.2)]]
     m = tk.Manager(tk.POLICY_TACKER, simulate=True, idle_cap_ms=2.0, slice_be=True, slice_ratio=ratio,
-                   reorder_only_unfused=literal)
+                   reorder_rule=rule)
     qs = []
     for i, tt in enumerate(arrivals):
         sh = shapes[i % 2]
@@ -313,7 +319,7 @@ def test_manager_slicing_matches_reference(tk, mode):
         apps.append(mr.App(rk))
     r_opp = 0.6 / 0.68
     ref = mr.simulate(qs, apps, 50.0, mr.TACKER, fuse_pred, idle_cap=2.0, slice_be=True, slice_ratio=ratio,
-                      opp_ratio=lambda a: r_opp, reorder_only_unfused=literal)
+                      opp_ratio=lambda a: r_opp, reorder_rule=rule)
     got = []
     for _ in range(100000):
         if m.stats().lc_queries_done == len(arrivals):
@@ -349,3 +355,85 @@ def test_training_prefixes_spread_over_the_latency_floor(tk):
         for i in range(1, len(ns)):
             assert rs[i] - rs[i - 1] >= gap - 1e-9 or ns[i] == full
         assert all(abs(x - t_of(n)) < 1e-12 for n, x in out)
+
+
+@pytest.mark.parametrize("rule", ["min_be", "eps"])
+def test_manager_s7_direct_launch_c(tk, rule):
+    """S7 (tests/golden/manager_scenarios.json, hand-computed from P:2092-2096) through the C
+    manager: Thr 2.5 <= the 3 ms ready BE head -> the whole query runs direct (min_be, default);
+    with the eps reading the first kernel fuses (Thr 0.5) and the second does not."""
+    s = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "manager_scenarios.json")))["S7"]
+    tk.tacker_model_clear()
+    # tau(r) = 1 + (2/3) r  ->  Tk_fuse = Ttc + (2/3) Tcd = Ttc + 2 for the 3 ms head
+    fit_pair_closed_form(tk, lambda r: 1 + s["extra"] / s["be"] * r)
+    m = tk.Manager(tk.POLICY_TACKER, simulate=True,
+                   direct_rule=tk.DIRECT_MIN_BE if rule == "min_be" else tk.DIRECT_EPS)
+    m.submit_lc([lc_kernel(tk, True, t) for t in s["kernels"]], 0.0)
+    m.submit_be([be_kernel(tk, float(s["be"]))])
+    names = {tk.DEC_FUSED: "FUSED", tk.DEC_ORIGINAL_LC: "ORIGINAL_LC", tk.DEC_REORDER_BE: "REORDER_BE"}
+    got, thr = [], []
+    for _ in range(100):
+        if m.stats().lc_queries_done == 1:
+            break
+        d = m.step(s["qos"])
+        if d.action in names and d.query >= 0:
+            got.append(names[d.action])
+            thr.append(d.thr_ms)
+    assert got == s[rule]["actions"]
+    assert abs(m.latency(0) - s[rule]["latency"]) < 1e-9
+    if rule == "eps":
+        assert abs(thr[0] - s["eps"]["thr_after_first"]) < 1e-9
+
+
+@pytest.mark.parametrize("policy", ["tacker", "baymax", "tacker_reverse", "tacker_older_always", "tacker_noreorder"])
+def test_manager_trace_replay_sim(tk, policy):
+    """The C manager's decision trace (simulated GPU) replayed through manager_ref.replay: every
+    decision, Tgain and headroom recomputed from the recorded observations matches (the same
+    check the GPU-mode test applies to a hardware run)."""
+    from tests.trace_check import check_trace
+    tk.tacker_model_clear()
+    tau = lambda r: max(1 + 0.25 * r, 0.4 + 0.93 * r)
+    fit_pair_closed_form(tk, tau)
+    reverse = policy == "tacker_reverse"
+    fit_reverse_pair_closed_form(tk, lambda r: max(1 + 0.35 * r, 0.3 + 0.97 * r))
+    rng = np.random.default_rng(17)
+    arrivals = np.cumsum(rng.exponential(3.3, 60))
+    shapes = [[(True, 1.21), (False, 0.3), (True, 0.83), (True, 1.97)], [(True, 0.52), (True, 0.49)]]
+    if reverse:
+        shapes = [[(True, 1.21), (False, 1.3), (True, 0.83), (False, 0.61)], [(False, 0.92), (True, 0.49)]]
+    app_ts = [[1.53, 0.71], [3.07], [0.43, 0.37, 2.51]]
+    tc_apps = [[0.47, 1.12], [0.81]] if reverse else []
+    older = policy in ("tacker_older_always", "tacker_noreorder")
+    rules = dict(fuse_older=older, older_margin=0.7 if older else 0.0,
+                 reorder_rule={"tacker_older_always": mr.REORDER_ALWAYS,
+                               "tacker_noreorder": mr.REORDER_NEVER}.get(policy, mr.REORDER_UNFUSED))
+    pol = tk.POLICY_BAYMAX if policy == "baymax" else tk.POLICY_TACKER
+    m = tk.Manager(pol, simulate=True, idle_cap_ms=2.0, fuse_older=older, older_margin_ms=rules["older_margin"],
+                   reorder_rule=rules["reorder_rule"])
+    m.trace_enable(100000)
+    queries = []
+    for i, t in enumerate(arrivals):
+        sh = shapes[i % 2]
+        m.submit_lc([lc_kernel(tk, tc, d) for tc, d in sh], float(t))
+        queries.append((float(t), sh))
+    apps = []
+    for ts in app_ts:
+        m.submit_be([be_kernel(tk, d) for d in ts])
+        apps.append([(mr.BE_CD, d) for d in ts])
+    for ts in tc_apps:
+        m.submit_be([be_kernel_tc(tk, d) for d in ts])
+        apps.append([(mr.BE_TC, d) for d in ts])
+    m.run(50.0, float(arrivals[-1]))
+    trace, dropped = m.trace_dicts()
+    assert dropped == 0 and len(trace) > 100
+    n = check_trace(trace, queries, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER,
+                    idle_cap=2.0, **rules)
+    assert n == len(trace)
+    if policy != "baymax":
+        assert any(d["action"] == tk.DEC_FUSED for d in trace)
+    # a corrupted decision is caught
+    bad = [dict(d) for d in trace]
+    i = next(j for j, d in enumerate(bad) if d["action"] in (tk.DEC_ORIGINAL_LC, tk.DEC_REORDER_BE))
+    bad[i]["thr"] += 0.5
+    with pytest.raises(AssertionError):
+        check_trace(bad, queries, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER, idle_cap=2.0, **rules)

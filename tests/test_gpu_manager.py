@@ -80,7 +80,7 @@ def test_managed_reverse_fusion_outputs_match_standalone(tk):
     assert host(svc.outputs[-1]).tobytes() == ref
 
 
-@pytest.mark.parametrize("variant", [dict(fuse_older=True), dict(fuse_older=True, slice_be=True, reorder_only_unfused=2)])
+@pytest.mark.parametrize("variant", [dict(fuse_older=True), dict(fuse_older=True, slice_be=True, reorder_rule=2)])
 def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
     """GPU-mode managed runs with reading 18 (older queries fuse) and with PTB slices and no
     reorder: every LC query's output bytes equal a standalone query's, QoS holds, kernels fused."""
@@ -109,3 +109,31 @@ def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
     assert res["qos_met"], res
     assert res["fused"] > 0, res
     assert host(svc.outputs[-1]).tobytes() == ref
+
+
+@pytest.mark.parametrize("rules", [dict(), dict(fuse_older=True, reorder_rule=1), dict(fuse_older=True)])
+def test_gpu_manager_trace_replays_through_reference(tk, rules):
+    """a GPU-mode managed run (steady-state window protocol of the bench) records
+    its decision trace; oracle/manager_ref.replay recomputes every decision, Tgain and headroom
+    from the recorded observations (clock, active queries, online Tk_fuse) and must agree."""
+    from oracle import manager_ref as mr
+    from paper_conf_hpca_zhaocczlllg22_b200 import qos, services as sv
+    from tests.trace_check import check_trace
+    convs = [c for c in synth.resnet50_convs(8) if c.name in ("layer1.0.conv1", "layer1.0.conv2", "layer1.0.conv3")]
+    svc = sv.resnet50_service(8, convs=convs)
+    st, mq = sv.stencil_app(512, 512, 64), sv.mriq_app(64, 1024, 1024)
+    tk.tacker_launch_original(None, mq.kernels[0].desc)
+    tk.tacker_model_clear()
+    run = qos.QosRun(svc, [st, mq], warp_split=16)
+    run.calibrate(reps=3, pair_reps=3)
+    run.measure_service(n=20)
+    res = run.run_window(tk.POLICY_TACKER, window_ms=60.0, warm_ms=20.0, tail_ms=20.0, load=0.8, max_inflight=8,
+                         trace=True, **rules)
+    assert res["trace_dropped"] == 0 and len(res["trace"]) > 50
+    queries, apps = run.replay_inputs(res["arrivals"])
+    cap = run.idle_cap()
+    ref_rules = dict(fuse_older=rules.get("fuse_older", False), older_margin=0.3 * run.qos,
+                     reorder_rule=rules.get("reorder_rule", mr.REORDER_UNFUSED))
+    n = check_trace(res["trace"], queries, apps, run.qos, mr.TACKER, idle_cap=cap if cap > 0 else None, **ref_rules)
+    assert n == len(res["trace"])
+    assert res["qos_met"], res

@@ -114,11 +114,12 @@ def heads_and_pred(spec):
     return heads, (lambda a: tf[a])
 
 
-@pytest.mark.parametrize("sid", ["S1", "S2", "S3", "S4", "S6"])
+@pytest.mark.parametrize("sid", ["S1", "S2", "S3", "S4", "S6", "S3_reorder_always", "S6_reorder_always"])
 def test_manager_scenarios(sid):
     s = gold("manager_scenarios.json")[sid]
     heads, fp = heads_and_pred(s)
-    fused, reorder, thr, gain = mr.decide(s["ttc"], True, s["thr"], heads, mr.TACKER, fp)
+    rule = mr.REORDER_ALWAYS if sid.endswith("_reorder_always") else mr.REORDER_UNFUSED
+    fused, reorder, thr, gain = mr.decide(s["ttc"], True, s["thr"], heads, mr.TACKER, fp, reorder_rule=rule)
     assert fused == s["fused"]
     assert reorder == s["reorder"]
     assert abs(thr - s["thr_after"]) < 1e-12
@@ -131,6 +132,24 @@ def test_manager_baymax_never_fuses():
     heads, fp = heads_and_pred(s)
     fused, reorder, thr, _ = mr.decide(s["ttc"], True, s["thr"], heads, mr.BAYMAX, fp)
     assert fused == -1 and reorder == [0] and thr == 37
+
+
+@pytest.mark.parametrize("rule", ["min_be", "eps"])
+def test_manager_s7_direct_launch(rule):
+    """S7 (golden, hand-computed): Thr close to 0 -> every kernel of the query launched directly."""
+    s = gold("manager_scenarios.json")["S7"]
+    q = mr.Query(0, 0.0, [(True, t) for t in s["kernels"]])
+    app = mr.App([(True, float(s["be"]))])
+    fp = lambda ttc, tcd: ttc + s["extra"]
+    res = mr.simulate([q], [app], s["qos"], mr.TACKER, fp,
+                      direct_rule=mr.DIRECT_MIN_BE if rule == "min_be" else mr.DIRECT_EPS)
+    names = {mr.FUSED: "FUSED", mr.ORIGINAL_LC: "ORIGINAL_LC", mr.REORDER_BE: "REORDER_BE"}
+    lc_dec = [d for d in res["decisions"] if d.lc is not None]
+    assert [names[d.action] for d in lc_dec] == s[rule]["actions"]
+    assert res["latency"][0] == s[rule]["latency"]
+    if rule == "eps":
+        assert abs(lc_dec[0].thr - s["eps"]["thr_after_first"]) < 1e-12
+        assert lc_dec[0].reorder == []
 
 
 def test_manager_eq9_headroom_two_queries():
@@ -213,8 +232,12 @@ def test_manager_reverse_fusion_scenarios():
     assert (fused, reorder, rev) == (0, [], True) and thr == 38.0 and gain == 1.0
     fused, reorder, thr, _ = mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, lambda a: 5.0)
     assert (fused, reorder, thr) == (-1, [0], 37.0)
-    # two tensor-core heads: gains 1 (3 ms, 4.0) and 2.5 - 2.5 = ... (3 ms, 4.5) -> 0.5: the first wins
-    fused, reorder, thr, gain = mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_TC), (1, 3.0, mr.BE_TC)], mr.TACKER, fp)
+    # two tensor-core heads: gains 1 (3 ms, 4.0) and 3 - 2.5 = 0.5 (3 ms, 4.5): the first wins;
+    # paper rule: nothing reordered after a fused launch (Thr 38); reading 6: head 1 too (Thr 35)
+    heads2 = [(0, 3.0, mr.BE_TC), (1, 3.0, mr.BE_TC)]
+    fused, reorder, thr, gain = mr.decide(2.0, False, 40.0, heads2, mr.TACKER, fp)
+    assert fused == 0 and gain == 1.0 and reorder == [] and thr == 38.0
+    fused, reorder, thr, gain = mr.decide(2.0, False, 40.0, heads2, mr.TACKER, fp, reorder_rule=mr.REORDER_ALWAYS)
     assert fused == 0 and gain == 1.0 and reorder == [1] and thr == 35.0
     assert mr.decide(2.0, False, 40.0, [(0, 3.0, mr.BE_CD)], mr.TACKER, lambda a: 1.0)[0] == -1
     assert mr.decide(2.0, True, 40.0, [(0, 3.0, mr.BE_TC)], mr.TACKER, lambda a: 1.0)[0] == -1

@@ -72,7 +72,7 @@ def main():
     res = {}
     variants = {"baymax": (tk.POLICY_BAYMAX, {}), "tacker": (tk.POLICY_TACKER, {}),
                 "tacker_slice": (tk.POLICY_TACKER, {"slice_be": True}),
-                "tacker_slice_literal": (tk.POLICY_TACKER, {"slice_be": True, "reorder_only_unfused": True}),
+                "tacker_slice_literal": (tk.POLICY_TACKER, {"slice_be": True}),
                 "tacker_older": (tk.POLICY_TACKER, {"fuse_older": True}),   # reading 18 (the bench headline)
                 "baymax_older": (tk.POLICY_BAYMAX, {"fuse_older": True})}   # Baymax with the same queueing rule
     for name in args.variants.split(","):
