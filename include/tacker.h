@@ -483,11 +483,12 @@ tacker_status tacker_manager_run_until(tacker_manager_t m, double qos_target_ms,
  * predicted fused duration Tk_fuse Eq. 8 evaluated (NaN where none was evaluated or no model
  * exists).  Records beyond the capacity are counted in *dropped, not stored. */
 #define TACKER_TRACE_MAX_APPS 16
-#define TACKER_TRACE_MAX_ACTIVE 64
 typedef struct {
   double t_ms;                                  /* manager clock at the decision */
-  int32_t n_active;                             /* active queries (may exceed the stored ids) */
-  int32_t active[TACKER_TRACE_MAX_ACTIVE];      /* their ids, oldest first */
+  int32_t first_active, n_active;               /* active queries: ids first_active .. + n_active - 1
+                                                   (admitted in arrival order, retired oldest first) */
+  int32_t active_contiguous;                    /* 0 if the active ids were not that range (queries
+                                                   submitted out of arrival order): not replayable */
   int32_t direct;                               /* the decided query runs direct (Thr close to 0) */
   int32_t n_apps;
   uint32_t ready_mask;                          /* bit a: BE app a's head was ready (always, on the GPU) */

@@ -100,10 +100,8 @@ def im2col(x, r, s, stride, pad, Kpad):
 
 def lc_conv_point(x, w, stride, pad, n, p, q, k):
     """One output element of lc_conv by explicit loops (for sampled full-size checks)."""
-    x64 = np.asarray(x, np.float64)
-    w64 = np.asarray(w, np.float64)
-    _, h, wd, c = x64.shape
-    _, r, s, _ = w64.shape
+    _, h, wd, c = x.shape
+    _, r, s, _ = w.shape
     acc = 0.0
     ab = 0.0
     for rr in range(r):
@@ -114,7 +112,7 @@ def lc_conv_point(x, w, stride, pad, n, p, q, k):
             wi = q * stride - pad + ss
             if wi < 0 or wi >= wd:
                 continue
-            t = x64[n, hi, wi, :] * w64[k, rr, ss, :]
+            t = np.asarray(x[n, hi, wi, :], np.float64) * np.asarray(w[k, rr, ss, :], np.float64)
             acc += float(t.sum())
             ab += float(np.abs(t).sum())
     return acc, ab

@@ -786,7 +786,10 @@ tacker_status tacker_manager_step(tacker_manager_t m, double qos, double *headro
   memset(&r, 0, sizeof r);
   r.t_ms = out->t_start_ms;
   r.n_active = (int32_t)m->active.size();
-  for (size_t i = 0; i < m->active.size() && i < TACKER_TRACE_MAX_ACTIVE; ++i) r.active[i] = m->active[i];
+  r.first_active = m->active.empty() ? -1 : m->active.front();
+  r.active_contiguous = 1;
+  for (size_t i = 0; i < m->active.size(); ++i)
+    if (m->active[i] != r.first_active + (int32_t)i) r.active_contiguous = 0;
   r.direct = out->query >= 0 && m->queries[out->query].direct ? 1 : 0;
   r.n_apps = (int32_t)std::min<size_t>(m->apps.size(), TACKER_TRACE_MAX_APPS);
   r.ready_mask = m->trace_ready;

@@ -235,12 +235,12 @@ class ManagerStats(C.Structure):
 
 
 CLASS_LC_TC, CLASS_LC_CD, CLASS_FUSED, CLASS_BE = range(4)
-TRACE_MAX_APPS, TRACE_MAX_ACTIVE = 16, 64
+TRACE_MAX_APPS = 16
 
 
 class TraceRec(C.Structure):
-    _fields_ = [("t_ms", C.c_double), ("n_active", C.c_int32), ("active", C.c_int32 * TRACE_MAX_ACTIVE),
-                ("direct", C.c_int32), ("n_apps", C.c_int32), ("ready_mask", C.c_uint32),
+    _fields_ = [("t_ms", C.c_double), ("first_active", C.c_int32), ("n_active", C.c_int32),
+                ("active_contiguous", C.c_int32), ("direct", C.c_int32), ("n_apps", C.c_int32), ("ready_mask", C.c_uint32),
                 ("tk_fuse_ms", C.c_double * TRACE_MAX_APPS),
                 ("d", Decision)]
 
@@ -753,11 +753,11 @@ class Manager:
         recs, dropped = self.trace()
         out = []
         for r in recs:
-            if r.n_active > TRACE_MAX_ACTIVE:
-                raise TackerError(EINVAL, "trace record with more active queries than stored")
+            if not r.active_contiguous:
+                raise TackerError(EINVAL, "trace record whose active queries are not an id range")
             tf = {a: r.tk_fuse_ms[a] for a in range(r.n_apps) if not math.isnan(r.tk_fuse_ms[a])}
             d = r.d
-            out.append({"t": r.t_ms, "active": list(r.active[:r.n_active]),
+            out.append({"t": r.t_ms, "active": list(range(r.first_active, r.first_active + r.n_active)),
                         "ready": [a for a in range(r.n_apps) if (r.ready_mask >> a) & 1], "tk_fuse": tf,
                         "direct": bool(r.direct), "action": d.action, "query": d.query, "lc_index": d.lc_index,
                         "fused_app": d.fused_app, "reorder": list(d.reorder_apps[:d.n_reorder]),
