@@ -311,6 +311,9 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
  * launch except original BE kernels (their non-persistent grid is then distributed over an
  * idle GPU instead of being parked behind the running kernel).  Process-wide.  EINVAL else. */
 tacker_status tacker_set_launch_overlap(int32_t enable);
+/* Diagnostics: copies the LC role clock64 stamps recorded by plans built with TACKER_LC_DBG bit 3
+ * ([160 CTAs][5 events][16 work units], see fused.cuh) into out (>= 12800 slots). */
+tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n);
 
 /* One fused launch of handle f whose BE part runs only the PTB slice [block_offset,
  * block_offset + n_blocks) of the handle's BE kernel (the LC part is unchanged; n_blocks 0 = no

@@ -50,6 +50,14 @@ struct LcParams {
   // splits of a tile write fp32 partials, meet on a counter, then each reduces 1/splits of the tile
   // in split order (deterministic) and runs the epilogue on it.
   int32_t splits, kb_per_split, num_units;
+  // TMA-store epilogue (LC-only, fp16 D with linear rows, no residual, no split): each epilogue
+  // warp stages its 32 rows x 64 columns (SW128) in shared memory and one lane stores the box
+  // through tmap_d -- full-line global writes instead of 16-byte row-strided stores
+  int32_t tma_store;
+  // diagnostics (TACKER_LC_DBG, never set in production): bit 0 = epilogue drains TMEM without
+  // math or stores; bit 1 = no MMAs (the issuer only releases stages and signals the epilogue);
+  // bit 2 = no TMA loads (the producer arrives on the full barriers without data)
+  int32_t dbg;
   float *part;             // [num_tiles * splits][kBM][BN] fp32 partial tiles
   uint32_t *cnt;           // [2 * num_tiles]: arrivals, finished reductions (self-resetting)
 };
@@ -63,6 +71,7 @@ struct alignas(64) FusedParams {
   CUtensorMap tmap_a;      // A / x operand
   CUtensorMap tmap_b;      // B / w operand
   CUtensorMap tmap_be;     // BE input tensor map (stencil), unused otherwise
+  CUtensorMap tmap_d;      // LC output D [M, N] fp16, box 64 x 32 (TMA-store epilogue)
   LcParams lc;
   tacker_be_desc be;
   int64_t be_blocks;       // original blocks to run (PTB original_block_num)
@@ -75,7 +84,17 @@ struct alignas(64) FusedParams {
   uint32_t tmem_cols;
   uint32_t lc_smem_bytes;  // ring + barriers, 1024-aligned start
   uint32_t be_smem_per_vb; // per-vblock slice (incl. 16 B ticket slot)
+  uint32_t epi_stage_off;  // TMA-store staging (4 warps x 2 x 4 KB, 1024-aligned) from the LC base
 };
+
+// diagnostics (TACKER_LC_DBG bit 3): per-CTA clock64 stamps of the first 16 work units of each LC
+// role -- [0] producer unit start, [1] MMA start (accumulator free), [2] MMA end (tfull commit),
+// [3] epilogue start (tfull seen), [4] epilogue end (tempty arrive); read by
+// tacker_debug_lc_timestamps
+__device__ unsigned long long g_lc_ts[160][5][16];
+__device__ __forceinline__ void lc_stamp(const LcParams &L, int ev, int i) {
+  if ((L.dbg & 8) && i < 16 && blockIdx.x < 160) g_lc_ts[blockIdx.x][ev][i] = clock64();
+}
 
 // ------------------------------------------------------------------------ LC roles
 template <int BN>
@@ -214,34 +233,76 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4)) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
       pre = min(P.stages, kb1 - kb0);
-      for (int i = 0; i < pre; ++i) {
-        mbar_arrive_expect_tx(&bb.full[i], kStage);
-        load_b(P, &bb.full[i], lc + i * kStage + kStageA, kb0 + i, nt);
+      if (elect_one()) {
+        for (int i = 0; i < pre; ++i) {
+          mbar_arrive_expect_tx(&bb.full[i], kStage);
+          load_b(P, &bb.full[i], lc + i * kStage + kStageA, kb0 + i, nt);
+        }
       }
+      __syncwarp();
     }
     griddep_wait();
     int stage = 0;
     uint32_t phase = 0;
-    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+    int ui = 0;
+    // im2col-mode implicit conv (C % 64 == 0): the k-block -> (channel block, filter tap) walk and
+    // the tile's first output pixel are computed once per unit and advanced incrementally, so the
+    // single producer thread does no integer division per k-block (it was the loop's bound)
+    const bool walk = implicit_conv(L) && L.conv_im2col && !L.conv_c8;
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
+      lc_stamp(L, 0, ui);
+      int wc = 0, hc = 0, n0 = 0, cb = 0, ss = 0, rr = 0;
+      if (walk) {
+        const int pq = L.p * L.q, m0 = mt * kBM;
+        n0 = m0 / pq;
+        const int rem = m0 - n0 * pq;
+        const int p0 = rem / L.q, q0 = rem - p0 * L.q;
+        wc = q0 * L.stride - L.pad;
+        hc = p0 * L.stride - L.pad;
+        cb = kb0 % L.c_blocks;
+        const int rs = kb0 / L.c_blocks;
+        rr = rs / L.s;
+        ss = rs - rr * L.s;
+      }
       for (int kb = kb0; kb < kb1; ++kb) {
         uint8_t *sa = lc + stage * kStage;
         uint8_t *sb = sa + kStageA;
-        if (pre > 0) {
-          --pre;              // first tile, stage == kb: B already in flight, its bytes expected
-        } else {
-          mbar_wait(&bb.empty[stage], phase ^ 1);
-          mbar_arrive_expect_tx(&bb.full[stage], kStage);
-          load_b(P, &bb.full[stage], sb, kb, nt);
+        const bool first = pre > 0;   // first tile, stage == kb: B already in flight, its bytes expected
+        if (first) --pre;
+        else mbar_wait(&bb.empty[stage], phase ^ 1);
+        if (elect_one()) {
+          if (L.dbg & 4) {
+            mbar_arrive(&bb.full[stage]);
+          } else if (walk) {
+            if (!first) {
+              mbar_arrive_expect_tx(&bb.full[stage], kStage);
+              tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);   // K index rs*C + cb*64 = 64 kb
+            }
+            tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc, n0, (uint16_t)ss, (uint16_t)rr);
+          } else {
+            if (!first) {
+              mbar_arrive_expect_tx(&bb.full[stage], kStage);
+              load_b(P, &bb.full[stage], sb, kb, nt);
+            }
+            load_a(P, &bb.full[stage], sa, kb, mt);
+          }
         }
-        load_a(P, &bb.full[stage], sa, kb, mt);
+        __syncwarp();
+        if (walk && ++cb == L.c_blocks) {
+          cb = 0;
+          if (++ss == L.s) {
+            ss = 0;
+            ++rr;
+          }
+        }
         if (++stage == P.stages) {
           stage = 0;
           phase ^= 1;
@@ -254,36 +315,44 @@ struct LcGemm {
     const LcParams &L = P.lc;
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
-    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+    int ui = 0;
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1;
       unit_coords(L, u, t, sp, kb0, kb1);
       mbar_wait(&bb.tempty[acc], acc_phase ^ 1);
       tc_fence_after();
+      lc_stamp(L, 1, ui);
       const uint32_t d = tmem + acc * BN;
       for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&bb.full[stage], phase);
         tc_fence_after();
         const uint32_t sa = smem_u32(lc + stage * kStage);
         const uint32_t sb = sa + kStageA;
-        if (L.conv_c8) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
+        if (elect_one()) {
+          if (L.dbg & 2) {
+            // diagnostics: no MMA
+          } else if (L.conv_c8) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
 #pragma unroll
-          for (int k = 0; k < kBK / kUK; ++k)
-            umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
-                     umma_desc_sw128(sb + k * kUK * 2), kIdesc, (kb != kb0 || k != 0));
-        } else {
+            for (int k = 0; k < kBK / kUK; ++k)
+              umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
+                       umma_desc_sw128(sb + k * kUK * 2), kIdesc, (kb != kb0 || k != 0));
+          } else {
+            const uint64_t da = umma_desc_sw128(sa), db = umma_desc_sw128(sb);
 #pragma unroll
-          for (int k = 0; k < kBK / kUK; ++k) {
-            umma_f16(d, umma_desc_sw128(sa + k * kUK * 2), umma_desc_sw128(sb + k * kUK * 2), kIdesc,
-                     (kb != kb0 || k != 0));
+            for (int k = 0; k < kBK / kUK; ++k)   // K step of 16 fp16 = 32 B = +2 in the start-address field
+              umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || k != 0));
           }
+          umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
         }
-        umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
+        __syncwarp();
         if (++stage == P.stages) {
           stage = 0;
           phase ^= 1;
         }
       }
-      umma_commit(&bb.tfull[acc]);        // accumulator ready for the epilogue
+      if (elect_one()) umma_commit(&bb.tfull[acc]);   // accumulator ready for the epilogue
+      __syncwarp();
+      lc_stamp(L, 2, ui);
       if (++acc == P.acc_stages) {
         acc = 0;
         acc_phase ^= 1;
@@ -294,6 +363,109 @@ struct LcGemm {
   // EC columns per batch: EC/16 TMEM loads in flight behind one wait, and the batch's residual
   // rows requested before that wait (LC-only launches: 64 columns; fused CTAs, capped at 64
   // registers per thread: 16)
+  // TMA-store epilogue (L.tma_store): per 64-column batch, a warp converts its 32 rows (bias,
+  // ReLU, fp16 RNE), writes them into one of its two 4 KB SW128 staging boxes (16-byte chunk j of
+  // row r at chunk j ^ (r % 8): conflict-free) and one lane stores the box with TMA; the box is
+  // rewritten only after that store has finished reading it (bulk wait_group.read 1).  The TMEM
+  // loads of batch b+1 are in flight while batch b is converted (two register buffers), and the
+  // batch's 64 bias values come from shared memory as 16 broadcast LDS.128 issued together.
+  static __device__ __forceinline__ void epi_batch(const FusedParams &P, const uint32_t (&v)[64], uint32_t bias_s,
+                                                   bool bias, uint8_t *stg, int &buf, int n0, int row0, int lane) {
+    const LcParams &L = P.lc;
+    float b[64];
+    if (bias) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const float4 q = ld_shared_v4f(bias_s + 16 * i);
+        b[4 * i] = q.x;
+        b[4 * i + 1] = q.y;
+        b[4 * i + 2] = q.z;
+        b[4 * i + 3] = q.w;
+      }
+    }
+    if (lane == 0) bulk_wait_read<1>();   // this box's previous store has read it
+    __syncwarp();
+    const uint32_t box = smem_u32(stg + buf * 4096) + lane * 128;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      float f[8];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        f[e] = __uint_as_float(v[8 * j + e]);
+        if (bias) f[e] = __fadd_rn(f[e], b[8 * j + e]);
+        if (L.epi & TACKER_EPI_RELU) f[e] = fmaxf(f[e], 0.f);
+      }
+      __align__(16) __half2 hv[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) hv[e] = __floats2half2_rn(f[2 * e], f[2 * e + 1]);
+      st_shared_v4(box + ((uint32_t)(j ^ (lane & 7)) << 4), *reinterpret_cast<uint4 *>(hv));
+    }
+    fence_proxy_async();                  // generic-proxy writes visible to the TMA unit
+    __syncwarp();
+    if (lane == 0) {
+      tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, row0);
+      bulk_commit();
+    }
+    buf ^= 1;
+  }
+  static __device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
+    tmem_ld_32x32b_x16(taddr, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+    tmem_ld_32x32b_x16(taddr + 16, *reinterpret_cast<uint32_t(*)[16]>(&v[16]));
+    tmem_ld_32x32b_x16(taddr + 32, *reinterpret_cast<uint32_t(*)[16]>(&v[32]));
+    tmem_ld_32x32b_x16(taddr + 48, *reinterpret_cast<uint32_t(*)[16]>(&v[48]));
+  }
+  static __device__ __forceinline__ void epilogue_tma(const FusedParams &P, const Bars &bb, uint32_t tmem,
+                                                      uint8_t *lc) {
+    static_assert(BN % 64 == 0, "TMA-store epilogue: 64-column batches");
+    constexpr int NB = BN / 64;
+    const LcParams &L = P.lc;
+    const int quarter = warp_id() & 3;
+    const int lane = lane_id();
+    uint8_t *stg = lc + P.epi_stage_off + quarter * 8192;
+    const uint32_t bias_s = smem_u32(bb.bias);
+    int buf = 0;
+    griddep_wait();
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    int ui = 0;
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
+      int t, sp, kb0, kb1, mt, nt;
+      unit_coords(L, u, t, sp, kb0, kb1);
+      tile_coords(L, t, mt, nt);
+      mbar_wait(&bb.tfull[acc], acc_phase);
+      tc_fence_after();
+      if (quarter == 0 && lane == 0) lc_stamp(L, 3, ui);
+      const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
+      const bool bias = (L.epi & TACKER_EPI_BIAS) != 0;
+      if (bias) {
+        const int et = (int)threadIdx.x % 128;
+        named_bar_sync(kLcEpiBar, 128);
+        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(kLcEpiBar, 128);
+      }
+      const bool skip = (L.dbg & 1) != 0;
+      const int row0 = mt * kBM + quarter * 32;
+      uint32_t va[64], vb[64];
+      tmem_ld64(tbase, va);
+#pragma unroll
+      for (int b = 0; b < NB; ++b) {
+        tmem_ld_wait();
+        if (b + 1 < NB) tmem_ld64(tbase + 64 * (b + 1), (b % 2) ? va : vb);
+        const int n0 = nt * BN + 64 * b;
+        if (n0 < L.N && !skip)
+          epi_batch(P, (b % 2) ? vb : va, bias_s + 256 * b, bias, stg, buf, n0, row0, lane);
+      }
+      tc_fence_before();
+      mbar_arrive(&bb.tempty[acc]);
+      if (quarter == 0 && lane == 0) lc_stamp(L, 4, ui);
+      if (++acc == P.acc_stages) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+    if (lane == 0) bulk_wait<0>();            // every store performed before the CTA retires
+  }
+
   template <int EC>
   static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem) {
     static_assert(EC % 16 == 0 && BN % EC == 0, "EC: multiple of 16 dividing BN");
@@ -332,7 +504,7 @@ struct LcGemm {
           rv[g] = (res && n0 + 8 * g < L.N) ? *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n0 + 8 * g)
                                             : make_uint4(0, 0, 0, 0);
         tmem_ld_wait();
-        if (orow < 0 || n0 >= L.N) continue;
+        if (orow < 0 || n0 >= L.N || (L.dbg & 1)) continue;
         if (prow) {   // split-K partial, fp32
 #pragma unroll
           for (int j = 0; j < EC; j += 4)
@@ -346,7 +518,12 @@ struct LcGemm {
               float f[8];
 #pragma unroll
               for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j / 16][j % 16 + u]);
-              store8(L, orow, n0 + j, f, bb.bias + c0 + j, rv[j / 8]);
+              __align__(16) float b8[8];
+              if (bias) {   // shared-space loads (a generic pointer would compile to LD.E)
+                *reinterpret_cast<float4 *>(b8) = ld_shared_v4f(smem_u32(bb.bias + c0 + j));
+                *reinterpret_cast<float4 *>(b8 + 4) = ld_shared_v4f(smem_u32(bb.bias + c0 + j + 4));
+              }
+              store8(L, orow, n0 + j, f, b8, rv[j / 8]);
             }
         }
       }
@@ -501,9 +678,11 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
     if (has_lc) {
       const uint32_t tmem = *bb.tmem_holder;
       if (warp == 0) {
-        if (lane_id() == 0) LcGemm<BN>::producer(P, lc, bb);
+        LcGemm<BN>::producer(P, lc, bb);      // warp-wide loop, elected issue
       } else if (warp == 1) {
-        if (lane_id() == 0) LcGemm<BN>::mma(P, lc, bb, tmem);
+        LcGemm<BN>::mma(P, lc, bb, tmem);
+      } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
+        LcGemm<BN>::epilogue_tma(P, bb, tmem, lc);
       } else {
         LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : 16>(P, bb, tmem);
       }

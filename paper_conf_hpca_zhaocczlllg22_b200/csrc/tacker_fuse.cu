@@ -305,6 +305,23 @@ static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
   return 128;
 }
 
+// TMA-store epilogue for eligible LC-only plans (TACKER_EPI_TMA=0 restores the register path)
+static bool tma_store_enabled() {
+  static const bool on = [] {
+    const char *e = getenv("TACKER_EPI_TMA");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+static int lc_dbg_flags() {
+  static const int f = [] {
+    const char *e = getenv("TACKER_LC_DBG");
+    return e ? atoi(e) : 0;
+  }();
+  return f;
+}
+
 // Implicit convs load A through the TMA im2col mode (linear 128-pixel M-tiles, no padding of a
 // small image to a 128-position window) unless TACKER_CONV_TILED=1 selects the tiled 4-D windows.
 static bool conv_im2col_mode() {
@@ -586,10 +603,17 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   uint32_t cols = 32;
   while (cols < (uint32_t)(acc * BN)) cols <<= 1;
 
+  // TMA-store epilogue: LC-only fp16 outputs whose GEMM rows are linear in D (plain GEMM, 1x1
+  // stride-1 conv, im2col-mode conv), no residual, no split-K; 4 warps x 2 staging boxes of 4 KB
+  L.tma_store = !has_be && tma_store_enabled() && lc->d_dtype == TACKER_F16 &&
+                !(lc->epi_flags & TACKER_EPI_RESIDUAL) && L.splits == 1 && BN >= 64 && L.N >= 64 &&
+                (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col);
+  const uint32_t epi_bytes = L.tma_store ? 4u * 2u * 4096u + 1024u : 0u;
+  L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
   const uint32_t stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
-  const uint32_t bar_bytes = 256 + 4 * 256;   // mbarriers + TMEM address + one tile's bias (BN <= 256)
+  const uint32_t bar_bytes = 256 + 4 * 256 + epi_bytes;   // mbarriers + TMEM address + one tile's bias (BN <= 256) + staging
   const uint32_t be_total = (uint32_t)vb * be_slice;
   // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
   // SM for the latency-bound implicit-GEMM loads); fused plans stop at 4 so the BE keeps L1
@@ -612,6 +636,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.P.acc_stages = acc;
   F.P.tmem_cols = cols;
   F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
+  F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + 256u + 4u * 256u + 1023u) & ~1023u : 0u;
   F.P.be_smem_per_vb = be_slice;
   F.P.be_vb_per_cta = vb;
   F.P.be_blocks = be_blocks;
@@ -639,6 +664,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   }
   if (has_be && (st = encode_be_tmap(*be, &F.P.tmap_be))) return st;
+  if (L.tma_store && (st = encode_2d(&F.P.tmap_d, lc->D, (uint64_t)L.N, (uint64_t)L.M, 64, 32))) return st;
   // registers: the whole CTA must fit the 64K register file
   cudaFuncAttributes fa{};
   cudaError_t e = cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(F.fn));
@@ -710,6 +736,13 @@ static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) { return lau
 extern "C" {
 
 const char *tacker_last_error(void) { return g_err.c_str(); }
+
+tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n) {
+  if (!out || n < 160 * 5 * 16) return set_error("need 12800 uint64 slots"), TACKER_EINVAL;
+  cudaError_t e = cudaMemcpyFromSymbol(out, tk::g_lc_ts, sizeof(tk::g_lc_ts));
+  if (e != cudaSuccess) return cuda_fail("debug timestamps", e);
+  return TACKER_OK;
+}
 
 tacker_status tacker_set_launch_overlap(int32_t enable) {
   if (enable < 0 || enable > 2) return set_error("launch overlap mode must be 0, 1 or 2"), TACKER_EINVAL;

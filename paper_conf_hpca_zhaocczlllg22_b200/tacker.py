@@ -259,6 +259,7 @@ _PROTOS = {
     "tacker_launch_fused": ([_V, _V], C.c_int),
     "tacker_launch_fused_slice": ([_V, _I64, _I64, _V], C.c_int),
     "tacker_set_launch_overlap": ([_I32], C.c_int),
+    "tacker_debug_lc_timestamps": ([C.POINTER(C.c_uint64), _I64], C.c_int),
     "tacker_launch_original": ([C.POINTER(LcDesc), C.POINTER(BeDesc), _V], C.c_int),
     "tacker_model_add_sample": ([_S, _D, _D], C.c_int),
     "tacker_model_fit": ([_S, C.POINTER(_D), C.POINTER(_D)], C.c_int),
@@ -601,6 +602,14 @@ def tacker_fuse(lc: LcDesc, be: BeDesc | None, warp_split: int, block_ratio=(0, 
 
 def tacker_launch_fused(f: Fused, stream=None):
     f.launch(stream)
+
+
+def tacker_debug_lc_timestamps():
+    """[160][5][16] clock64 stamps of the LC roles (plans built with TACKER_LC_DBG bit 3)."""
+    import numpy as np
+    buf = (C.c_uint64 * (160 * 5 * 16))()
+    _chk(_lib.tacker_debug_lc_timestamps(buf, len(buf)))
+    return np.frombuffer(buf, dtype=np.uint64).reshape(160, 5, 16).copy()
 
 
 def tacker_set_launch_overlap(enable):

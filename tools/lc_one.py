@@ -28,10 +28,12 @@ def main():
     else:
         sv.autotune_tile_n(svc)
     torch.cuda.synchronize()
+    torch.cuda.nvtx.range_push("target")     # ncu --nvtx --nvtx-include "target/" selects these launches
     for n in args.names:
         k = ks[n]
         for _ in range(args.reps):
             tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd)
+    torch.cuda.nvtx.range_pop()
     torch.cuda.synchronize()
     print("ok")
 
