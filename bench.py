@@ -458,12 +458,12 @@ def arm_result(q, tk, name, window_ms, warm_ms, load, seed, inflight, sync=None)
                         seed=seed, max_inflight=inflight, sync=sync, **rules)
 
 
-def calibrated_run(qos, tk, svc, apps, args, comm):
+def calibrated_run(qos, tk, svc, apps, args, comm, peak_steps=50):
     q = qos.QosRun(svc, apps, warp_split=args.warp_split, qos_ms=QOS_MS)
     q.calibrate()
     q.measure_service(max_inflight=args.inflight)
-    # lambda_peak by bisection on LC-only runs (2000 queries' worth each)
-    q.find_peak_load(window_ms=20 * STEP_QUERIES * q.service_ms, max_inflight=args.inflight)
+    # lambda_peak by bisection on LC-only runs of peak_steps x 100 queries' worth each
+    q.find_peak_load(window_ms=peak_steps * STEP_QUERIES * q.service_ms, max_inflight=args.inflight)
     return q
 
 
@@ -532,7 +532,8 @@ def run_tacker(args, comm):
 
     # ---- the other arms on the same trace; tacker / baymax_same_rule over --seeds seeds
     seeds = tuple(range(args.seeds))
-    other = side_runs(q, tk, ("baymax", "baymax_same_rule", "tacker_paper"), args.steps, rank, args.inflight)
+    other = side_runs(q, tk, ("baymax", "baymax_same_rule", "tacker_paper", "tacker_reorder_always"), args.steps,
+                      rank, args.inflight)
     if args.seeds > 1:
         more = side_runs(q, tk, ("tacker", "baymax_same_rule"), args.steps, rank, args.inflight, seeds)
         other["tacker_seeds"] = more["tacker"]
@@ -640,7 +641,7 @@ def side_workloads(args, comm, peaks, flush, tk, qos, sv, torch):
     sv.autotune_tile_n(vgg)
     apps = sv.be_apps(names, seed)
     sv.prime_apps(apps)
-    qv = calibrated_run(qos, tk, vgg, apps, args, comm)
+    qv = calibrated_run(qos, tk, vgg, apps, args, comm, peak_steps=20)
     r = side_runs(qv, tk, ("tacker", "baymax", "baymax_same_rule", "tacker_paper"), steps, rank, args.inflight)
     out["vgg16_b24"] = dict(workload="vgg16_b24 LC + Table II mixed BE queue, QoS 50 ms (BASELINE configs[3])",
                             service_ms=qv.service_ms, lambda_peak_load=qv.peak_load, steps=steps, **r,
@@ -655,7 +656,7 @@ def side_workloads(args, comm, peaks, flush, tk, qos, sv, torch):
         tk.tacker_model_clear()
         svc = sv.resnet50_service(b, seed)
         sv.autotune_tile_n(svc)
-        qb = calibrated_run(qos, tk, svc, [st, mq], args, comm)
+        qb = calibrated_run(qos, tk, svc, [st, mq], args, comm, peak_steps=20)
         r = side_runs(qb, tk, ("tacker", "baymax", "baymax_same_rule", "tacker_paper"), steps, rank, args.inflight)
         out[f"resnet50_b{b}_stencil_mriq"] = dict(
             workload=f"resnet50_b{b} LC + stencil/mriq BE queue, QoS 50 ms" + (" (BASELINE configs[1])" if b == 1 else ""),

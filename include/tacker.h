@@ -455,6 +455,11 @@ tacker_status tacker_manager_create(int32_t policy, const tacker_manager_params 
 tacker_status tacker_manager_destroy(tacker_manager_t m);
 tacker_status tacker_manager_submit_lc(tacker_manager_t m, const tacker_lc_query *q, double arrival_ms,
                                        int32_t *query_id_out);
+/* n queries of the same kernels q arriving at arrivals_ms[0..n) (a Poisson trace), ids first_id ..
+ * first_id + n - 1 in submission order; one call instead of n (a long trace is submitted before
+ * its first arrival). */
+tacker_status tacker_manager_submit_lc_batch(tacker_manager_t m, const tacker_lc_query *q, const double *arrivals_ms,
+                                             int64_t n, int32_t *first_id);
 tacker_status tacker_manager_submit_be(tacker_manager_t m, const tacker_be_app *app, int32_t *app_id_out);
 /* Register the predicted fused duration for (LC kernel t_pred class, BE app kernel); the
  * manager asks the model store with the pair key of the fused handle it would build. */

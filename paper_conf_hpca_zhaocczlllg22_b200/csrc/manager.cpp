@@ -30,6 +30,7 @@
 #include <cmath>
 #include <cstring>
 #include <deque>
+#include <memory>
 #include <array>
 #include <map>
 #include <set>
@@ -51,7 +52,10 @@ namespace {
 struct Query {
   int id;
   double arrival;
-  std::vector<tacker_lc_kernel> ks;
+  // the query's kernels, shared by every query of a batch submission (a trace of 10^4 queries of
+  // one service holds one copy)
+  std::shared_ptr<const std::vector<tacker_lc_kernel>> kv;
+  const std::vector<tacker_lc_kernel> &ks() const { return *kv; }
   size_t pos = 0;
   bool issued = false, direct = false, has_thr = false;
   double thr = 0;
@@ -59,7 +63,7 @@ struct Query {
   cudaEvent_t last_ev = nullptr;  // GPU mode: event after its last kernel
   double remaining() const {
     double s = 0;
-    for (size_t i = pos; i < ks.size(); ++i) s += ks[i].t_pred_ms;
+    for (size_t i = pos; i < kv->size(); ++i) s += (*kv)[i].t_pred_ms;
     return s;
   }
 };
@@ -255,7 +259,7 @@ static void poll(tacker_manager_s *m) {
   }
   for (int id : m->active) {
     Query &q = m->queries[id];
-    if (q.pos == q.ks.size() && q.done_at < 0 && q.last_ev && cudaEventQuery(q.last_ev) == cudaSuccess) {
+    if (q.pos == q.ks().size() && q.done_at < 0 && q.last_ev && cudaEventQuery(q.last_ev) == cudaSuccess) {
       q.done_at = event_time(m, q.last_ev);
       unref(m, q.last_ev);
       q.last_ev = nullptr;
@@ -466,18 +470,44 @@ tacker_status tacker_manager_destroy(tacker_manager_t m) {
   return TACKER_OK;
 }
 
+static tacker_status submit_query(tacker_manager_t m, Query &&Q, int32_t *id);
+
 tacker_status tacker_manager_submit_lc(tacker_manager_t m, const tacker_lc_query *q, double arrival_ms, int32_t *id) {
   if (!m || !q || q->n_kernels <= 0 || !q->kernels) return set_error("bad query"), TACKER_EINVAL;
   Query Q;
   Q.id = (int)m->queries.size();
   Q.arrival = arrival_ms;
-  Q.ks.assign(q->kernels, q->kernels + q->n_kernels);
-  m->queries.push_back(Q);
-  // keep pending sorted by arrival (stable)
-  auto pos = m->pending.begin() + (long)m->next_pending;
-  while (pos != m->pending.end() && m->queries[*pos].arrival <= arrival_ms) ++pos;
-  m->pending.insert(pos, Q.id);
-  if (id) *id = Q.id;
+  Q.kv = std::make_shared<const std::vector<tacker_lc_kernel>>(q->kernels, q->kernels + q->n_kernels);
+  return submit_query(m, std::move(Q), id);
+}
+
+static tacker_status submit_query(tacker_manager_t m, Query &&Q, int32_t *id) {
+  const double arrival_ms = Q.arrival;
+  m->queries.push_back(std::move(Q));
+  Query &Qr = m->queries.back();
+  // keep pending sorted by arrival (stable): scan from the back, so queries submitted in arrival
+  // order append in O(1)
+  size_t pos = m->pending.size();
+  while (pos > m->next_pending && m->queries[m->pending[pos - 1]].arrival > arrival_ms) --pos;
+  m->pending.insert(m->pending.begin() + (long)pos, Qr.id);
+  if (id) *id = Qr.id;
+  return TACKER_OK;
+}
+
+tacker_status tacker_manager_submit_lc_batch(tacker_manager_t m, const tacker_lc_query *q, const double *arrivals_ms,
+                                             int64_t n, int32_t *first_id) {
+  if (!m || !q || n < 0 || (n > 0 && !arrivals_ms)) return set_error("bad query batch"), TACKER_EINVAL;
+  if (q->n_kernels <= 0 || !q->kernels) return set_error("bad query"), TACKER_EINVAL;
+  if (first_id) *first_id = (int32_t)m->queries.size();
+  m->queries.reserve(m->queries.size() + (size_t)n);
+  auto kv = std::make_shared<const std::vector<tacker_lc_kernel>>(q->kernels, q->kernels + q->n_kernels);
+  for (int64_t i = 0; i < n; ++i) {
+    Query Q;
+    Q.id = (int)m->queries.size();
+    Q.arrival = arrivals_ms[i];
+    Q.kv = kv;
+    if (tacker_status s = submit_query(m, std::move(Q), nullptr)) return s;
+  }
   return TACKER_OK;
 }
 
@@ -520,7 +550,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
   // retire finished queries
   while (!m->active.empty()) {
     Query &q = m->queries[m->active.front()];
-    if (q.pos < q.ks.size()) break;
+    if (q.pos < q.ks().size()) break;
     if (m->sim() || q.done_at >= 0) m->active.pop_front();
     else break;
   }
@@ -529,7 +559,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
   // oldest query with kernels still to issue
   int qid = -1;
   for (int id : m->active)
-    if (m->queries[id].pos < m->queries[id].ks.size()) {
+    if (m->queries[id].pos < m->queries[id].ks().size()) {
       qid = id;
       break;
     }
@@ -618,7 +648,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
     thr -= m->prm.older_margin_ms;
   }
   const double thr_eff = thr;
-  const tacker_lc_kernel &k = q.ks[q.pos];
+  const tacker_lc_kernel &k = q.ks()[q.pos];
   const double ttc = k.t_pred_ms;
 
   int fused = -1;
@@ -721,7 +751,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
       if (s) return s;
       cudaEvent_t e = mark(m, true);
       track(m, e0, e, TACKER_CLASS_FUSED);
-      if (q.pos + 1 == q.ks.size()) q.last_ev = ref(m, e);
+      if (q.pos + 1 == q.ks().size()) q.last_ev = ref(m, e);
       // online model update from the measured co-run: (X_tc, X_cd) of the pair
       if (reverse) {
         const std::string &pk = rpair_entry(m, k, fused, A.pos % A.ks.size()).pk;
@@ -742,7 +772,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
       cudaEvent_t e0 = begin(m, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
       tacker_status s = launch_lc(m, k);
       if (s) return s;
-      const bool last = q.pos + 1 == q.ks.size();
+      const bool last = q.pos + 1 == q.ks().size();
       cudaEvent_t e = mark(m, e0 != nullptr || last);
       track(m, e0, e, k.is_tc ? TACKER_CLASS_LC_TC : TACKER_CLASS_LC_CD);
       if (last) q.last_ev = ref(m, e);
@@ -751,7 +781,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
     out->action = reorder.empty() ? TACKER_DEC_ORIGINAL_LC : TACKER_DEC_REORDER_BE;
   }
   q.pos++;
-  if (m->sim() && q.pos == q.ks.size()) {
+  if (m->sim() && q.pos == q.ks().size()) {
     q.done_at = m->now;
     m->st.lc_queries_done++;
   }
@@ -863,9 +893,12 @@ tacker_status tacker_manager_prepare(tacker_manager_t m, const tacker_lc_query *
     if (q->n_kernels < 0 || (q->n_kernels > 0 && !q->kernels)) return set_error("bad query"), TACKER_EINVAL;
     return prepare_kernels(m, q->kernels, (size_t)q->n_kernels);
   }
+  const std::vector<tacker_lc_kernel> *last = nullptr;
   for (; m->prepared < m->queries.size(); ++m->prepared) {
     const Query &Q = m->queries[m->prepared];
-    if (tacker_status s = prepare_kernels(m, Q.ks.data(), Q.ks.size())) return s;
+    if (Q.kv.get() == last) continue;   // same kernels as the previous query (a batch submission)
+    last = Q.kv.get();
+    if (tacker_status s = prepare_kernels(m, Q.ks().data(), Q.ks().size())) return s;
   }
   return TACKER_OK;
 }

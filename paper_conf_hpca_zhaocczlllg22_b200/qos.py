@@ -484,16 +484,21 @@ class QosRun:
             m.trace_enable(4_000_000)
         kernels = self.lc_kernels()
         m.prepare(kernels)
-        t0 = m.stats().now_ms + 2.0
-        w0, w1 = t0 + warm_ms, t0 + warm_ms + window_ms
-        t_end = w1 + tail_ms
-        arr, t = [], t0
+        # the whole trace is submitted (one C call) before its first arrival: offsets first, then
+        # t0 a few ms after the submission finishes
+        span = warm_ms + window_ms + tail_ms
+        offs, t = [], 0.0
         while True:
             t += rng.exponential(1.0 / lam)
-            if t >= t_end:
+            if t >= span:
                 break
-            arr.append(t)
-        qids = [m.submit_lc(kernels, float(a)) for a in arr]
+            offs.append(t)
+        t0 = m.stats().now_ms + 20.0 + 1e-3 * len(offs)
+        w0, w1 = t0 + warm_ms, t0 + warm_ms + window_ms
+        arr = [t0 + o for o in offs]
+        qids = m.submit_lc_batch(kernels, arr)
+        if m.stats().now_ms > t0:
+            raise RuntimeError("query submission overran the trace start")
         m.run_until(self.qos, w0)
         torch.cuda.synchronize()
         if sync:
@@ -557,9 +562,9 @@ class QosRun:
             m.submit_be(ks)
         kernels = self.lc_kernels()
         m.prepare(kernels)                          # fused handles built before arrivals are fixed
-        t0 = m.stats().now_ms + 2.0
+        t0 = m.stats().now_ms + 20.0 + 1e-3 * len(gaps)
         arr = t0 + np.cumsum(gaps)
-        qids = [m.submit_lc(kernels, float(t)) for t in arr]
+        qids = m.submit_lc_batch(kernels, arr)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         m.run(self.qos, float(arr[-1]))

@@ -282,6 +282,7 @@ _PROTOS = {
     "tacker_manager_prepare": ([_V, _V], C.c_int),
     "tacker_manager_query_latency": ([_V, _I32, C.POINTER(_D)], C.c_int),
     "tacker_manager_run_until": ([_V, _D, _D], C.c_int),
+    "tacker_manager_submit_lc_batch": ([_V, C.POINTER(LcQuery), C.POINTER(_D), _I64, C.POINTER(_I32)], C.c_int),
     "tacker_manager_trace_enable": ([_V, _I64], C.c_int),
     "tacker_manager_trace_count": ([_V, C.POINTER(_I64), C.POINTER(_I64)], C.c_int),
     "tacker_manager_trace_get": ([_V, _I64, C.POINTER(TraceRec)], C.c_int),
@@ -707,6 +708,15 @@ class Manager:
         qid = C.c_int32()
         _chk(_lib.tacker_manager_submit_lc(self.h, C.byref(q), arrival_ms, C.byref(qid)))
         return qid.value
+
+    def submit_lc_batch(self, kernels, arrivals_ms) -> list:
+        """Queries of the same kernels at each arrival time (one C call); returns their ids."""
+        arr = (LcKernel * len(kernels))(*kernels)
+        q = LcQuery(len(kernels), arr)
+        ts = (C.c_double * len(arrivals_ms))(*[float(a) for a in arrivals_ms])
+        first = C.c_int32()
+        _chk(_lib.tacker_manager_submit_lc_batch(self.h, C.byref(q), ts, len(arrivals_ms), C.byref(first)))
+        return list(range(first.value, first.value + len(arrivals_ms)))
 
     def submit_be(self, kernels) -> int:
         arr = (BeKernel * len(kernels))(*kernels)
