@@ -284,7 +284,11 @@ typedef struct {
   int64_t lc_tiles, be_blocks;
   int32_t be_smem_per_vblock, regs_per_thread;
   int32_t lc_splits;         /* split-K factor of the LC part (1 = none) */
+  int32_t lc_mode;           /* TACKER_LC_MODE_*: how the LC operands are tiled and loaded */
+  int32_t lc_tma_store;      /* 1: TMA-store epilogue (LC-only fp16 plans) */
 } tacker_fused_info_t;
+enum { TACKER_LC_MODE_GEMM = 0, TACKER_LC_MODE_CONV_IM2COL = 1, TACKER_LC_MODE_CONV_TILED = 2,
+       TACKER_LC_MODE_CONV_C8 = 3, TACKER_LC_MODE_CONV_HALO = 4 };
 tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *out);
 /* Model-store keys of the handle's LC kernel, BE kernel and fused pair (for the predictor). */
 tacker_status tacker_fused_keys(tacker_fused_t f, char *lc_key, char *be_key, char *pair_key, size_t buflen);

@@ -45,6 +45,11 @@ struct LcParams {
                              // 16 B, loaded as 8 unswizzled 128 x 16 B boxes (K-major, no swizzle)
   int32_t conv_im2col;       // implicit conv through the TMA im2col mode: M-tile = 128 consecutive
                              // output pixels (n, p, q linear); else tp x tq windows of one image
+  int32_t conv_halo;         // stride-1 conv, C % 64 == 0: M-tile = 16 x 8 output pixels; a k-step =
+                             // (filter row r, channel block cb) loads ONE input halo of 16 x (8+S-1)
+                             // pixels x 64 channels (SW128) and the S taps' weights, and issues S x 4
+                             // MMAs whose A descriptors start s rows into the halo (SBO = (8+S-1) rows)
+  uint32_t stage_a, stage_bytes;   // shared-memory bytes of a ring stage's A part and of the stage
   // split-K: work unit u = (tile u / splits, k-blocks [s kb_per_split, (s+1) kb_per_split) of split
   // s = u % splits).  splits > 1 only when every unit has its own CTA (num_units <= grid): the
   // splits of a tile write fp32 partials, meet on a counter, then each reduces 1/splits of the tile
@@ -112,8 +117,8 @@ struct LcGemm {
   static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
     return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
   }
-  static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages) {
-    uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * kStage);
+  static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages, uint32_t stage_bytes) {
+    uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * stage_bytes);
     return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4),
                 reinterpret_cast<float *>(b + 2 * stages + 6)};
   }
@@ -177,7 +182,12 @@ struct LcGemm {
   // B (weights) k-block kb of N-tile nt
   static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
     const LcParams &L = P.lc;
-    if (implicit_conv(L) && L.conv_c8) {
+    if (L.conv_halo) {
+      // k-step kb = (filter row r, channel block cb): the S taps' weight columns (r S + t) C + 64 cb
+      const int cb = kb % L.c_blocks, r = kb / L.c_blocks;
+      for (int t = 0; t < L.s; ++t)
+        tma_load_2d(&P.tmap_b, bar, sb + t * BN * 128, (r * L.s + t) * L.c + cb * kBK, nt * BN);
+    } else if (implicit_conv(L) && L.conv_c8) {
       tma_load_2d(&P.tmap_b, bar, sb, kb * kBK, nt * BN);   // K = R*S*8 linear (OOB tail zero-filled)
     } else if (implicit_conv(L)) {
       // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
@@ -190,7 +200,14 @@ struct LcGemm {
   // A (activations) k-block kb of M-tile mt
   static __device__ __forceinline__ void load_a(const FusedParams &P, uint64_t *bar, uint8_t *sa, int kb, int mt) {
     const LcParams &L = P.lc;
-    if (implicit_conv(L) && L.conv_c8) {
+    if (L.conv_halo) {
+      // the input rows of filter row r for the tile's 16 output rows, 8 + S - 1 columns, 64 channels
+      // (out-of-image rows / columns zero-filled = the padding)
+      const int cb = kb % L.c_blocks, r = kb / L.c_blocks;
+      const int img = mt / (L.tiles_p * L.tiles_q);
+      const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
+      tma_load_4d(&P.tmap_a, bar, sa, cb * kBK, qt * L.tq - L.pad, pt * L.tp - L.pad + r, img);
+    } else if (implicit_conv(L) && L.conv_c8) {
       // k-block kb = filter taps 8 kb .. 8 kb + 7 (K index = tap * 8 + c); tap t lands at sa + 2 KB t
       // as 128 pixel rows of 16 B; taps past R*S reload tap 0 (their weights are the zero padding)
       const int pq = L.p * L.q, m0 = mt * kBM;
@@ -240,8 +257,8 @@ struct LcGemm {
       pre = min(P.stages, kb1 - kb0);
       if (elect_one()) {
         for (int i = 0; i < pre; ++i) {
-          mbar_arrive_expect_tx(&bb.full[i], kStage);
-          load_b(P, &bb.full[i], lc + i * kStage + kStageA, kb0 + i, nt);
+          mbar_arrive_expect_tx(&bb.full[i], L.stage_bytes);
+          load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a, kb0 + i, nt);
         }
       }
       __syncwarp();
@@ -260,7 +277,15 @@ struct LcGemm {
       tile_coords(L, t, mt, nt);
       lc_stamp(L, 0, ui);
       int wc = 0, hc = 0, n0 = 0, cb = 0, ss = 0, rr = 0;
-      if (walk) {
+      if (L.conv_halo) {   // halo tile origin (input coordinates of output pixel (p0, q0) minus pad)
+        n0 = mt / (L.tiles_p * L.tiles_q);
+        const int rem = mt - n0 * L.tiles_p * L.tiles_q;
+        const int pt = rem / L.tiles_q, qt = rem - pt * L.tiles_q;
+        wc = qt * L.tq - L.pad;
+        hc = pt * L.tp - L.pad;
+        cb = kb0 % L.c_blocks;
+        rr = kb0 / L.c_blocks;
+      } else if (walk) {
         const int pq = L.p * L.q, m0 = mt * kBM;
         n0 = m0 / pq;
         const int rem = m0 - n0 * pq;
@@ -273,30 +298,40 @@ struct LcGemm {
         ss = rs - rr * L.s;
       }
       for (int kb = kb0; kb < kb1; ++kb) {
-        uint8_t *sa = lc + stage * kStage;
-        uint8_t *sb = sa + kStageA;
+        uint8_t *sa = lc + stage * L.stage_bytes;
+        uint8_t *sb = sa + L.stage_a;
         const bool first = pre > 0;   // first tile, stage == kb: B already in flight, its bytes expected
         if (first) --pre;
         else mbar_wait(&bb.empty[stage], phase ^ 1);
         if (elect_one()) {
           if (L.dbg & 4) {
             mbar_arrive(&bb.full[stage]);
+          } else if (L.conv_halo) {
+            if (!first) {
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
+              for (int t = 0; t < L.s; ++t)   // the filter row's S taps: K columns (rr S + t) C + 64 cb
+                tma_load_2d(&P.tmap_b, &bb.full[stage], sb + t * BN * 128, (rr * L.s + t) * L.c + cb * kBK, nt * BN);
+            }
+            tma_load_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc + rr, n0);
           } else if (walk) {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], kStage);
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
               tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);   // K index rs*C + cb*64 = 64 kb
             }
             tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc, n0, (uint16_t)ss, (uint16_t)rr);
           } else {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], kStage);
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
               load_b(P, &bb.full[stage], sb, kb, nt);
             }
             load_a(P, &bb.full[stage], sa, kb, mt);
           }
         }
         __syncwarp();
-        if (walk && ++cb == L.c_blocks) {
+        if (L.conv_halo && ++cb == L.c_blocks) {
+          cb = 0;
+          ++rr;
+        } else if (walk && ++cb == L.c_blocks) {
           cb = 0;
           if (++ss == L.s) {
             ss = 0;
@@ -326,11 +361,22 @@ struct LcGemm {
       for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&bb.full[stage], phase);
         tc_fence_after();
-        const uint32_t sa = smem_u32(lc + stage * kStage);
-        const uint32_t sb = sa + kStageA;
+        const uint32_t sa = smem_u32(lc + stage * L.stage_bytes);
+        const uint32_t sb = sa + L.stage_a;
         if (elect_one()) {
           if (L.dbg & 2) {
             // diagnostics: no MMA
+          } else if (L.conv_halo) {
+            // tap s of this filter row: A = the halo from row s, 8-row groups (one output row of 8
+            // pixels each) (8 + S - 1) rows apart; B = the tap's BN x 64 weight slot
+            const uint32_t sbo = (uint32_t)(8 + L.s - 1) * 128u;
+            for (int t = 0; t < L.s; ++t) {
+              const uint64_t da = umma_desc_sw128_sbo(sa + 128u * t, sbo);
+              const uint64_t db = umma_desc_sw128(sb + (uint32_t)t * BN * 128u);
+#pragma unroll
+              for (int k = 0; k < kBK / kUK; ++k)
+                umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || t != 0 || k != 0));
+            }
           } else if (L.conv_c8) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
 #pragma unroll
             for (int k = 0; k < kBK / kUK; ++k)
@@ -369,8 +415,14 @@ struct LcGemm {
   // rewritten only after that store has finished reading it (bulk wait_group.read 1).  The TMEM
   // loads of batch b+1 are in flight while batch b is converted (two register buffers), and the
   // batch's 64 bias values come from shared memory as 16 broadcast LDS.128 issued together.
+  // store coordinates of a warp's 32-row box: linear rows (2-D map over D [M, N]) or, for a halo
+  // tile, 4 output rows x 8 columns of one image (4-D map over D [n][P][Q][K], box 64 x 8 x 4 x 1)
+  struct BoxAt {
+    int row0;              // 2-D: first GEMM row
+    int q0, p0, img;       // 4-D
+  };
   static __device__ __forceinline__ void epi_batch(const FusedParams &P, const uint32_t (&v)[64], uint32_t bias_s,
-                                                   bool bias, uint8_t *stg, int &buf, int n0, int row0, int lane) {
+                                                   bool bias, uint8_t *stg, int &buf, int n0, BoxAt at, int lane) {
     const LcParams &L = P.lc;
     float b[64];
     if (bias) {
@@ -403,7 +455,8 @@ struct LcGemm {
     fence_proxy_async();                  // generic-proxy writes visible to the TMA unit
     __syncwarp();
     if (lane == 0) {
-      tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, row0);
+      if (L.conv_halo) tma_store_4d(&P.tmap_d, stg + buf * 4096, n0, at.q0, at.p0, at.img);
+      else tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, at.row0);
       bulk_commit();
     }
     buf ^= 1;
@@ -444,7 +497,12 @@ struct LcGemm {
         named_bar_sync(kLcEpiBar, 128);
       }
       const bool skip = (L.dbg & 1) != 0;
-      const int row0 = mt * kBM + quarter * 32;
+      BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
+      if (L.conv_halo) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
+        at.img = mt / (L.tiles_p * L.tiles_q);
+        at.p0 = ((mt / L.tiles_q) % L.tiles_p) * L.tp + 4 * quarter;
+        at.q0 = (mt % L.tiles_q) * L.tq;
+      }
       uint32_t va[64], vb[64];
       tmem_ld64(tbase, va);
 #pragma unroll
@@ -453,7 +511,7 @@ struct LcGemm {
         if (b + 1 < NB) tmem_ld64(tbase + 64 * (b + 1), (b % 2) ? va : vb);
         const int n0 = nt * BN + 64 * b;
         if (n0 < L.N && !skip)
-          epi_batch(P, (b % 2) ? vb : va, bias_s + 256 * b, bias, stg, buf, n0, row0, lane);
+          epi_batch(P, (b % 2) ? vb : va, bias_s + 256 * b, bias, stg, buf, n0, at, lane);
       }
       tc_fence_before();
       mbar_arrive(&bb.tempty[acc]);
@@ -654,7 +712,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
   const bool has_lc = P.lc_warps > 0 && P.lc.num_units > 0;
   typename LcGemm<BN>::Bars bb{};
   if (P.lc_warps > 0) {
-    bb = LcGemm<BN>::bars(lc, P.stages);
+    bb = LcGemm<BN>::bars(lc, P.stages, P.lc.stage_bytes);
     if (warp == 0 && lane_id() == 0) {
       tma_prefetch_desc(&P.tmap_a);
       tma_prefetch_desc(&P.tmap_b);

@@ -129,6 +129,13 @@ __device__ __forceinline__ void tma_store_2d(const void *tmap, const void *src, 
                "r"(smem_u32(src)), "r"(c0), "r"(c1)
                : "memory");
 }
+__device__ __forceinline__ void tma_store_4d(const void *tmap, const void *src, int32_t c0, int32_t c1, int32_t c2,
+                                             int32_t c3) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(tmap)),
+               "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 // at most N bulk groups still reading their shared-memory source
 template <int N>
@@ -239,6 +246,19 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t smem_addr) {
   d |= (uint64_t)(1024 >> 4) << 32;                    // SBO = 1024 B    [32,46)
   d |= (uint64_t)1 << 46;                              // version = 1     [46,48)
   d |= (uint64_t)2 << 61;                              // SWIZZLE_128B    [61,64)
+  return d;
+}
+// SW128 K-major operand with an explicit stride between 8-row groups: the 128-byte swizzle is a
+// function of the shared-memory address (verified: tools/micro/desc_test.cu), so a descriptor may
+// start at any 128-byte row of a TMA-written SW128 buffer and step 8-row groups by any multiple of
+// 128 B -- the tap-shifted window of a conv halo (base offset field 0).
+__device__ __forceinline__ uint64_t umma_desc_sw128_sbo(uint32_t smem_addr, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr & 0x3FFFF) >> 4);
+  d |= (uint64_t)(16 >> 4) << 16;
+  d |= (uint64_t)((sbo & 0x3FFFF) >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
   return d;
 }
 // K-major operand without swizzle (core matrices of 8 rows x 16 B): rows 16 B apart inside a core

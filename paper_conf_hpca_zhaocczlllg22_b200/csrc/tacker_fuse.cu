@@ -332,9 +332,34 @@ static bool conv_im2col_mode() {
   return !tiled;
 }
 
+// Halo mode (stride-1 "same" convs, C % 64 == 0, tiles up to 128 wide): one input halo per
+// (filter row, channel block) instead of one 128-pixel im2col load per filter tap (S x fewer A
+// bytes through L2 and S x 4 MMAs per ring handshake).  TACKER_CONV_HALO=0 disables it.
+static bool conv_halo_ok(const LcParams &L, int BN) {
+  static const bool on = [] {
+    const char *e = getenv("TACKER_CONV_HALO");
+    return !(e && e[0] == '0');
+  }();
+  return on && L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && L.stride == 1 && L.c % 64 == 0 &&
+         L.r == L.s && L.s <= 7 && 2 * L.pad == L.s - 1 && L.p >= 8 && L.q >= 8 && BN <= 128;
+}
+
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
-  if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && L.c == 8) {
+  L.stage_a = kBM * kBK * 2;
+  L.stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
+  if (conv_halo_ok(L, BN)) {
+    L.conv_halo = 1;
+    L.tq = 8;
+    L.tp = kBM / 8;
+    L.tiles_p = (L.p + L.tp - 1) / L.tp;
+    L.tiles_q = (L.q + L.tq - 1) / L.tq;
+    L.tiles_m = L.n * L.tiles_p * L.tiles_q;
+    L.c_blocks = L.c / kBK;
+    L.num_kb = L.r * L.c_blocks;               // k-steps: (filter row, channel block)
+    L.stage_a = ((uint32_t)L.tp * (L.tq + L.s - 1) * 128u + 1023u) & ~1023u;
+    L.stage_bytes = L.stage_a + (uint32_t)L.s * BN * 128u;
+  } else if (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && L.c == 8) {
     L.conv_im2col = 1;               // C = 8 (conv1 padded): 8 taps per k-block
     L.conv_c8 = 1;
     L.tiles_m = (L.M + kBM - 1) / kBM;
@@ -422,6 +447,37 @@ static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, cons
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv x) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+// Halo mode A: NHWC as (C, W, H, N), box 64 channels x (tq + S - 1) columns x tp rows x 1 image,
+// SW128 (one 128-byte row per pixel, pixels in (row, column) order); out-of-image = zero padding.
+static tacker_status encode_conv_halo(CUtensorMap *m, const tacker_lc_desc &d, const LcParams &L) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)d.c, (cuuint64_t)d.w, (cuuint64_t)d.h, (cuuint64_t)d.n};
+  cuuint64_t strides[3] = {(cuuint64_t)d.c * 2, (cuuint64_t)d.c * d.w * 2, (cuuint64_t)d.c * d.w * d.h * 2};
+  cuuint32_t box[4] = {(cuuint32_t)kBK, (cuuint32_t)(L.tq + L.s - 1), (cuuint32_t)L.tp, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void *>(d.A), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv halo) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+// TMA-store map of a halo tile's output: NHWC D as (K, Q, P, N), box 64 channels x 8 columns x 4
+// rows x 1 image = one epilogue warp's 32 TMEM lanes; rows / columns past P / Q are clipped.
+static tacker_status encode_conv_out_4d(CUtensorMap *m, const tacker_lc_desc &d, const LcParams &L) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  cuuint64_t dims[4] = {(cuuint64_t)L.N, (cuuint64_t)L.q, (cuuint64_t)L.p, (cuuint64_t)L.n};
+  cuuint64_t strides[3] = {(cuuint64_t)L.N * 2, (cuuint64_t)L.N * L.q * 2, (cuuint64_t)L.N * L.q * L.p * 2};
+  cuuint32_t box[4] = {64, (cuuint32_t)L.tq, 4, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, d.D, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv out) failed: %d", (int)r), TACKER_ECUDA;
   return TACKER_OK;
 }
 
@@ -607,12 +663,12 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // stride-1 conv, im2col-mode conv), no residual, no split-K; 4 warps x 2 staging boxes of 4 KB
   L.tma_store = !has_be && tma_store_enabled() && lc->d_dtype == TACKER_F16 &&
                 !(lc->epi_flags & TACKER_EPI_RESIDUAL) && L.splits == 1 && BN >= 64 && L.N >= 64 &&
-                (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col);
+                (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col || L.conv_halo);
   const uint32_t epi_bytes = L.tma_store ? 4u * 2u * 4096u + 1024u : 0u;
   L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
-  const uint32_t stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
+  const uint32_t stage_bytes = L.stage_bytes;
   const uint32_t bar_bytes = 256 + 4 * 256 + epi_bytes;   // mbarriers + TMEM address + one tile's bias (BN <= 256) + staging
   const uint32_t be_total = (uint32_t)vb * be_slice;
   // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
@@ -656,7 +712,9 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
 
   // TMA tensor maps
   if (lc->kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-    if ((st = L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc, L.conv_c8 != 0) : encode_conv_x(&F.P.tmap_a, *lc, L)))
+    if ((st = L.conv_halo ? encode_conv_halo(&F.P.tmap_a, *lc, L)
+                          : L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc, L.conv_c8 != 0)
+                                          : encode_conv_x(&F.P.tmap_a, *lc, L)))
       return st;
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   } else {
@@ -664,7 +722,11 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   }
   if (has_be && (st = encode_be_tmap(*be, &F.P.tmap_be))) return st;
-  if (L.tma_store && (st = encode_2d(&F.P.tmap_d, lc->D, (uint64_t)L.N, (uint64_t)L.M, 64, 32))) return st;
+  if (L.tma_store && L.conv_halo) {
+    if ((st = encode_conv_out_4d(&F.P.tmap_d, *lc, L))) return st;
+  } else if (L.tma_store && (st = encode_2d(&F.P.tmap_d, lc->D, (uint64_t)L.N, (uint64_t)L.M, 64, 32))) {
+    return st;
+  }
   // registers: the whole CTA must fit the 64K register file
   cudaFuncAttributes fa{};
   cudaError_t e = cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(F.fn));
@@ -821,6 +883,13 @@ tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *o) {
   o->tmem_cols = (int32_t)f->P.tmem_cols;
   o->lc_tiles = f->P.lc.num_tiles;
   o->lc_splits = f->P.lc.splits;
+  const LcParams &L = f->P.lc;
+  const bool implicit = L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
+  o->lc_mode = !implicit ? TACKER_LC_MODE_GEMM
+               : L.conv_halo ? TACKER_LC_MODE_CONV_HALO
+               : L.conv_c8 ? TACKER_LC_MODE_CONV_C8
+               : L.conv_im2col ? TACKER_LC_MODE_CONV_IM2COL : TACKER_LC_MODE_CONV_TILED;
+  o->lc_tma_store = L.tma_store;
   o->be_blocks = f->P.be_blocks;
   o->be_smem_per_vblock = (int32_t)f->P.be_smem_per_vb;
   o->regs_per_thread = f->regs;

@@ -185,7 +185,11 @@ class FusedInfo(C.Structure):
                 ("lc_tile_m", C.c_int32), ("lc_tile_n", C.c_int32), ("lc_tile_k", C.c_int32),
                 ("lc_stages", C.c_int32), ("lc_acc_stages", C.c_int32), ("tmem_cols", C.c_int32),
                 ("lc_tiles", C.c_int64), ("be_blocks", C.c_int64), ("be_smem_per_vblock", C.c_int32),
-                ("regs_per_thread", C.c_int32), ("lc_splits", C.c_int32)]
+                ("regs_per_thread", C.c_int32), ("lc_splits", C.c_int32), ("lc_mode", C.c_int32),
+                ("lc_tma_store", C.c_int32)]
+
+
+LC_MODE_GEMM, LC_MODE_CONV_IM2COL, LC_MODE_CONV_TILED, LC_MODE_CONV_C8, LC_MODE_CONV_HALO = range(5)
 
 
 class LcKernel(C.Structure):

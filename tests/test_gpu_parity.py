@@ -398,3 +398,48 @@ def test_plans_of_one_instantiation_keep_their_smem(tk):
     big.launch()
     small.launch()
     torch.cuda.synchronize()
+
+
+# ------------------------------------------------------------------ LC conv, halo mode (a5)
+HALO_CASES = [synth.ConvShape("h14", 2, 14, 14, 64, 64, 3, 3, 1, 1),          # 76 % useful tiles, ragged p and q
+              synth.ConvShape("h9x11", 2, 9, 11, 128, 72, 3, 3, 1, 1),        # 2 channel blocks, N % 64 != 0
+              synth.ConvShape("h28", 3, 28, 28, 64, 128, 3, 3, 1, 1),
+              synth.ConvShape("h56", 2, 56, 56, 64, 64, 3, 3, 1, 1),          # layer1 geometry
+              synth.ConvShape("h14c256", 1, 14, 14, 256, 256, 3, 3, 1, 1),    # b1 layer3: split-K
+              synth.ConvShape("h5x5", 1, 20, 17, 64, 64, 5, 5, 1, 2)]         # S = 5: halo 16 x 12
+
+
+@pytest.mark.parametrize("bn", [64, 128])
+@pytest.mark.parametrize("epi", ["bias_relu", "residual"])
+@pytest.mark.parametrize("cs", HALO_CASES, ids=lambda c: c.name)
+def test_lc_conv_halo_vs_oracle(tk, cs, epi, bn):
+    """Halo mode (one input halo per filter row and channel block, tap-shifted UMMA descriptors):
+    TMA-store epilogue (bias + ReLU) and the register epilogue (residual), vs the oracle."""
+    x, w, b = synth.conv_inputs(cs, seed=5)
+    res = np.random.default_rng(2).uniform(-1, 1, size=(cs.n, cs.p, cs.q, cs.k)).astype(np.float16)
+    out = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    lc = tk.lc_conv(t(x), t(w), out, cs.stride, cs.pad, bias=t(b), relu=True,
+                    residual=t(res) if epi == "residual" else None, tile_n=bn)
+    info = tk.tacker_fuse(lc, None, 0).info()
+    assert info.lc_mode == tk.LC_MODE_CONV_HALO
+    assert info.lc_tma_store == (1 if epi == "bias_relu" and info.lc_splits == 1 else 0)
+    tk.tacker_launch_original(lc, None)
+    ref, S = olc.lc_conv(x, w, cs.stride, cs.pad, bias=b, relu=True, residual=res if epi == "residual" else None)
+    assert max_rel_err(host(out).astype(np.float64), ref, S) <= 1e-2
+
+
+def test_lc_conv_halo_fused_bit_identical(tk):
+    """A halo-mode conv fused with a BE kernel (register epilogue, BE warps beside the LC roles)
+    writes the same bytes as its original launch."""
+    cs = HALO_CASES[2]
+    x, w, b = synth.conv_inputs(cs, seed=6)
+    o0 = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    o1 = torch.zeros_like(o0)
+    c = be_case(tk.BE_SGEMM)
+    c["reset"]()
+    tk.tacker_launch_original(tk.lc_conv(t(x), t(w), o0, 1, 1, bias=t(b), relu=True, tile_n=64), None)
+    f = tk.tacker_fuse(tk.lc_conv(t(x), t(w), o1, 1, 1, bias=t(b), relu=True, tile_n=64), c["desc"], 8)
+    assert f.info().lc_mode == tk.LC_MODE_CONV_HALO
+    f.launch()
+    assert torch.equal(o0, o1)
+    c["check"]([host(o) for o in c["outs"]])

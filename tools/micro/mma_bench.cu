@@ -19,7 +19,7 @@ template <int N, int S>
 __global__ void __launch_bounds__(128, 1) mma_kernel(int rounds, unsigned long long *cyc, int a_tmem_mode) {
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t *base = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(sm) + 1023) & ~uintptr_t(1023));
-  constexpr uint32_t kA = 128 * 128, kB = N * 128, kStage = kA + kB;
+  constexpr uint32_t kA = 288 * 128, kB = N * 128, kStage = kA + kB;
   uint64_t *bar = reinterpret_cast<uint64_t *>(base + S * kStage);
   uint64_t *full = bar + 4, *empty = bar + 4 + S;
   uint32_t *holder = reinterpret_cast<uint32_t *>(bar + 4 + 2 * S);
@@ -43,7 +43,7 @@ __global__ void __launch_bounds__(128, 1) mma_kernel(int rounds, unsigned long l
   tc_fence_after();
   const uint32_t tmem = *holder;
   constexpr uint32_t idesc = umma_idesc_f16(128, N);
-  if (a_tmem_mode >= 3 && threadIdx.x >= 32 && threadIdx.x < 64) {   // producer warp: ring handshake only
+  if (a_tmem_mode >= 3 && a_tmem_mode <= 5 && threadIdx.x >= 32 && threadIdx.x < 64) {   // producer warp: ring handshake only
     int st = 0;
     uint32_t ph = 0;
     for (int i = 0; i < rounds * S; ++i) {
@@ -59,7 +59,7 @@ __global__ void __launch_bounds__(128, 1) mma_kernel(int rounds, unsigned long l
       if (++st == S) { st = 0; ph ^= 1; }
     }
   }
-  if (a_tmem_mode >= 3 && threadIdx.x < 32) {
+  if (a_tmem_mode >= 3 && a_tmem_mode <= 5 && threadIdx.x < 32) {
     unsigned long long t0 = clock64();
     int st = 0;
     uint32_t ph = 0;
@@ -85,16 +85,21 @@ __global__ void __launch_bounds__(128, 1) mma_kernel(int rounds, unsigned long l
     unsigned long long t0 = clock64();
     for (int r = 0; r < rounds; ++r) {
       for (int s = 0; s < S; ++s) {
-        if (a_tmem_mode >= 2) {
+        if (a_tmem_mode == 2) {
           mbar_wait(&bar[2], 0);
           tc_fence_after();
         }
         if (elect_one()) {
           const uint32_t sa = smem_u32(base + s * kStage), sb = sa + kA;
-          const uint64_t da = umma_desc_sw128(sa), db = umma_desc_sw128(sb);
+          // mode 6: halo-style A (start s rows in, SBO 1280); mode 7: SBO 2048 (16-pixel pitch), start s rows
+          const uint64_t da = a_tmem_mode == 6 ? umma_desc_sw128_sbo(sa + 128 * (r % 3), 1280)
+                              : a_tmem_mode == 7 ? umma_desc_sw128_sbo(sa + 128 * (r % 3), 2048)
+                              : a_tmem_mode == 8 ? umma_desc_sw128_sbo(sa, 2048)
+                                                 : umma_desc_sw128(sa);
+          const uint64_t db = umma_desc_sw128(sb);
 #pragma unroll
           for (int k = 0; k < 4; ++k) umma_f16(tmem, da + 2 * k, db + 2 * k, idesc, (r | s | k) != 0);
-          if (a_tmem_mode >= 1) umma_commit(&bar[1]);
+          if (a_tmem_mode == 1) umma_commit(&bar[1]);
         }
         __syncwarp();
       }
@@ -115,7 +120,7 @@ __global__ void __launch_bounds__(128, 1) mma_kernel(int rounds, unsigned long l
 
 template <int N, int S>
 void run(int rounds, unsigned long long *d, int mode) {
-  const int smem = S * (128 * 128 + N * 128) + 2048 + 1024;
+  const int smem = S * (288 * 128 + N * 128) + 2048 + 1024;
   cudaFuncSetAttribute(mma_kernel<N, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   mma_kernel<N, S><<<148, 128, smem>>>(rounds, d, mode);
   cudaDeviceSynchronize();
@@ -139,9 +144,10 @@ void run(int rounds, unsigned long long *d, int mode) {
 int main() {
   unsigned long long *d;
   cudaMalloc(&d, 148 * sizeof(unsigned long long));
-  for (int mode = 3; mode < 6; ++mode) {
-    run<64, 4>(4000, d, mode);
-    run<128, 4>(4000, d, mode);
+  for (int mode : {0, 6, 7, 8}) {
+    run<64, 4>(1000, d, mode);
+    run<128, 4>(1000, d, mode);
+    run<256, 2>(500, d, mode);
   }
   return 0;
 }
