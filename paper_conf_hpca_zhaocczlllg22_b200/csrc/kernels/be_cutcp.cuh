@@ -82,44 +82,69 @@ template <> struct BeBody<TACKER_BE_CUTCP> {
   }
 };
 
-// Deterministic binning for cutcp: thread = bin; atoms scanned in index order through shared
-// memory, an atom goes to bin (floor(z/bs), floor(y/bs), floor(x/bs)) clamped into the grid.
+// Deterministic binning for cutcp: an original block owns 32 bins (lane = bin) and its 4 warps
+// split the atoms into 4 contiguous index ranges.  Pass 1 counts each warp's atoms per bin; the
+// per-warp counts give every warp its write offset inside each bin (warp w after warps < w), so
+// pass 2 stores the atoms of every bin in atom-index order without atomics.  An atom's bin
+// (floor(z/bs), floor(y/bs), floor(x/bs)) clamped into the grid is computed once per 32 atoms (one
+// per lane) and broadcast with shuffles.  Bins past the depth count the overflow; the rest of a
+// bin is padded with far-away zero-charge atoms.
 template <> struct BeBody<TACKER_BE_CUTCP_BIN> {
-  static constexpr int kStage = 1024;
-  static constexpr uint32_t kSmem = kStage * 16;
+  static constexpr uint32_t kSmem = 4 * 32 * 4;
   static __host__ __device__ int64_t num_blocks(const tacker_be_cutcp_bin &p) {
-    return ((int64_t)p.bdim_x * p.bdim_y * p.bdim_z + 127) / 128;
+    return ((int64_t)p.bdim_x * p.bdim_y * p.bdim_z + 31) / 32;
+  }
+  static __device__ __forceinline__ int bin_of(const tacker_be_cutcp_bin &p, float4 at) {
+    const int ix = min(max((int)floorf(__fdiv_rn(at.x, p.bin_size)), 0), p.bdim_x - 1);
+    const int iy = min(max((int)floorf(__fdiv_rn(at.y, p.bin_size)), 0), p.bdim_y - 1);
+    const int iz = min(max((int)floorf(__fdiv_rn(at.z, p.bin_size)), 0), p.bdim_z - 1);
+    return (iz * p.bdim_y + iy) * p.bdim_x + ix;
   }
   static __device__ __forceinline__ void run(const tacker_be_cutcp_bin &p, int64_t vb, int tid, uint32_t bar,
                                              uint8_t *smem) {
-    float4 *st = reinterpret_cast<float4 *>(smem);
-    const int64_t nb = (int64_t)p.bdim_x * p.bdim_y * p.bdim_z;
-    const int64_t b = vb * 128 + tid;
+    int *s_cnt = reinterpret_cast<int *>(smem);   // [4 warps][32 bins]
+    const int w = tid >> 5, lane = tid & 31;
+    const int nb = p.bdim_x * p.bdim_y * p.bdim_z;
+    const int b = (int)(vb * 32) + lane;
     const float4 *atoms = reinterpret_cast<const float4 *>(p.atoms);
     float4 *bins = reinterpret_cast<float4 *>(p.bins);
+    const int a0 = (int)((int64_t)p.natoms * w / 4), a1 = (int)((int64_t)p.natoms * (w + 1) / 4);
     int cnt = 0;
-    for (int c = 0; c < p.natoms; c += kStage) {
-      const int n = min(kStage, p.natoms - c);
-      named_bar_sync(bar, kVbThreads);
-      for (int a = tid; a < n; a += kVbThreads) st[a] = __ldg(atoms + c + a);
-      named_bar_sync(bar, kVbThreads);
-      if (b < nb) {
-        for (int a = 0; a < n; ++a) {
-          const float4 at = st[a];
-          const int ix = min(max((int)floorf(__fdiv_rn(at.x, p.bin_size)), 0), p.bdim_x - 1);
-          const int iy = min(max((int)floorf(__fdiv_rn(at.y, p.bin_size)), 0), p.bdim_y - 1);
-          const int iz = min(max((int)floorf(__fdiv_rn(at.z, p.bin_size)), 0), p.bdim_z - 1);
-          if (((int64_t)iz * p.bdim_y + iy) * p.bdim_x + ix == b) {
-            if (cnt < p.bin_depth) bins[b * p.bin_depth + cnt] = at;
-            ++cnt;
-          }
+    for (int a = a0; a < a1; a += 32) {
+      const int n = min(32, a1 - a);
+      const int mine = lane < n ? bin_of(p, __ldg(atoms + a + lane)) : -1;
+      for (int j = 0; j < n; ++j) cnt += __shfl_sync(0xffffffffu, mine, j) == b ? 1 : 0;
+    }
+    named_bar_sync(bar, kVbThreads);          // previous block's readers of s_cnt are done
+    s_cnt[w * 32 + lane] = cnt;
+    named_bar_sync(bar, kVbThreads);
+    int k = 0, total = 0;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int c = s_cnt[u * 32 + lane];
+      if (u < w) k += c;
+      total += c;
+    }
+    for (int a = a0; a < a1; a += 32) {
+      const int n = min(32, a1 - a);
+      const float4 at = lane < n ? __ldg(atoms + a + lane) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const int mine = lane < n ? bin_of(p, at) : -1;
+      for (int j = 0; j < n; ++j) {
+        const int bj = __shfl_sync(0xffffffffu, mine, j);
+        if ((unsigned)(bj - (int)(vb * 32)) >= 32u) continue;   // warp-uniform: not one of this block's bins
+        const float x = __shfl_sync(0xffffffffu, at.x, j), y = __shfl_sync(0xffffffffu, at.y, j);
+        const float z = __shfl_sync(0xffffffffu, at.z, j), q = __shfl_sync(0xffffffffu, at.w, j);
+        if (bj == b) {
+          if (k < p.bin_depth) bins[(int64_t)b * p.bin_depth + k] = make_float4(x, y, z, q);
+          ++k;
         }
       }
     }
-    if (b < nb) {
-      for (int s = cnt; s < p.bin_depth; ++s) bins[b * p.bin_depth + s] = make_float4(1e30f, 1e30f, 1e30f, 0.f);
-      p.count[b] = cnt;
-      if (cnt > p.bin_depth) *p.overflow = 1;
+    if (w == 0 && b < nb) {
+      for (int t = min(total, p.bin_depth); t < p.bin_depth; ++t)
+        bins[(int64_t)b * p.bin_depth + t] = make_float4(1e30f, 1e30f, 1e30f, 0.f);
+      p.count[b] = total;
+      if (total > p.bin_depth) *p.overflow = 1;
     }
   }
 };

@@ -245,8 +245,11 @@ def tpacf_app(n=16384, seed=2022) -> BeAppSpec:
     r = _dev(synth.tpacf_inputs(n, seed + 1, "uniform"))
     dd = torch.zeros(e.numel() + 1, dtype=torch.int32, device="cuda")
     dr = torch.zeros_like(dd)
-    ks = [BeKernelSpec("tpacf.dd", tk.be_tpacf(d, d, e, dd, self_pairs=True), bytes=12.0 * n, bound="alu"),
-          BeKernelSpec("tpacf.dr", tk.be_tpacf(d, r, e, dr), bytes=24.0 * n, bound="alu")]
+    # per pair the dot product is 5 FP32 pipe instructions (3 FMUL + 2 FADD), counted as 10 FMA-
+    # equivalent flops against the FFMA peak (2 flops per pipe slot); the bin search is extra
+    ks = [BeKernelSpec("tpacf.dd", tk.be_tpacf(d, d, e, dd, self_pairs=True), flops=10.0 * n * (n - 1) / 2,
+                       bytes=12.0 * n, bound="fma"),
+          BeKernelSpec("tpacf.dr", tk.be_tpacf(d, r, e, dr), flops=10.0 * n * n, bytes=24.0 * n, bound="fma")]
     return BeAppSpec(f"tpacf_{n}", ks, [e, d, r, dd, dr])
 
 
@@ -279,6 +282,29 @@ def lbm_app(nx=120, ny=120, nz=150, seed=2022) -> BeAppSpec:
     return BeAppSpec(f"lbm_{nx}x{ny}x{nz}", ks, [a, b, flags])
 
 
+def _cutcp_pairs(atoms, n, h, cutoff):
+    """Number of (lattice point, atom) pairs closer than the cutoff: per atom and lattice plane z and
+    row y, the count of integer x with (x h - ax)^2 < c^2 - dy^2 - dz^2 (vectorised over atoms)."""
+    a = np.asarray(atoms, np.float64)[:, :3]
+    r = int(np.ceil(cutoff / h)) + 1
+    total = 0
+    cz = np.floor(a[:, 2] / h).astype(np.int64)
+    cy = np.floor(a[:, 1] / h).astype(np.int64)
+    for oz in range(-r, r + 2):
+        iz = cz + oz
+        dz2 = (iz * h - a[:, 2]) ** 2
+        okz = (iz >= 0) & (iz < n) & (dz2 < cutoff * cutoff)
+        for oy in range(-r, r + 2):
+            iy = cy + oy
+            rem = cutoff * cutoff - dz2 - (iy * h - a[:, 1]) ** 2
+            ok = okz & (iy >= 0) & (iy < n) & (rem > 0)
+            w = np.sqrt(np.where(ok, rem, 0.0))
+            lo = np.maximum(np.floor((a[:, 0] - w) / h).astype(np.int64) + 1, 0)
+            hi = np.minimum(np.ceil((a[:, 0] + w) / h).astype(np.int64) - 1, n - 1)
+            total += int(np.where(ok, np.maximum(hi - lo + 1, 0), 0).sum())
+    return total
+
+
 def cutcp_app(L=48.0, seed=2022, depth=32) -> BeAppSpec:
     """Parboil cutcp: binning (once per app iteration) + the potential kernel."""
     d = synth.cutcp_inputs(L, seed)
@@ -290,10 +316,13 @@ def cutcp_app(L=48.0, seed=2022, depth=32) -> BeAppSpec:
     cnt = torch.zeros(nb, dtype=torch.int32, device="cuda")
     ovf = torch.zeros(1, dtype=torch.int32, device="cuda")
     V = torch.zeros(nx ** 3, device="cuda")
+    # algorithmic work of the potential: the (lattice point, atom) pairs inside the cutoff (the
+    # kernel also tests the pairs of neighbour bins beyond it), ~14 FP32 ops + 1 rsqrt each
+    pairs = _cutcp_pairs(d["atoms"], nx, float(d["h"]), 12.0)
     ks = [BeKernelSpec("cutcp.bin", tk.be_cutcp_bin(atoms, bins, cnt, ovf, nx, nx, nx, float(d["h"]), depth),
-                       bytes=16.0 * atoms.shape[0] * 2),
+                       bytes=16.0 * atoms.shape[0] * 2 + 16.0 * nb * depth),
           BeKernelSpec("cutcp.potential", tk.be_cutcp(bins, cnt, V, nx, nx, nx, float(d["h"]), depth),
-                       bytes=4.0 * nx ** 3, bound="fma")]
+                       flops=14.0 * pairs, mufu=float(pairs), bytes=4.0 * nx ** 3, bound="mufu")]
     return BeAppSpec(f"cutcp_{L:g}A", ks, [atoms, bins, cnt, ovf, V])
 
 
