@@ -315,6 +315,26 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
  * launch except original BE kernels (their non-persistent grid is then distributed over an
  * idle GPU instead of being parked behind the running kernel).  Process-wide.  EINVAL else. */
 tacker_status tacker_set_launch_overlap(int32_t enable);
+/* NEXT-1 fusion selection (§V-C): "create all possible fused kernels for two kernels,
+ * measure these candidates' performance and two kernels' sequential performance, and choose the
+ * best one among them.  If the sequential case shows the best performance, we do not fuse the two
+ * kernels."  Candidates are the BE warp splits in splits[0..n) (a split the budget rejects is
+ * skipped, fused_ms = NAN); each is timed over `reps` back-to-back launches on stream s (CUDA
+ * events, mean), after one warm-up, as is the sequential pair of original launches.  Out:
+ * *best_ws = the fastest split, or 0 when sequential is fastest -- the BE kernel is then also
+ * blacklisted ("if a CD kernel could not benefit from kernel fusion with one TC
+ * kernel, this CD kernel would not be considered for fusion"); *best_ms its time; *seq_ms;
+ * fused_ms[i] (nullable) per candidate.  Synchronises the stream (calibration, not the hot path).
+ * Buffers: the descriptors' device memory is written by the timed launches. */
+tacker_status tacker_select_fusion(const tacker_lc_desc *lc, const tacker_be_desc *be, const int32_t *splits,
+                                   int32_t n_splits, int32_t reps, tacker_stream_t s, int32_t *best_ws,
+                                   double *best_ms, double *seq_ms, double *fused_ms);
+/* The BE-kernel blacklist (keyed by the BE model-store key, see tacker_fused_keys): op 1 adds, 0
+ * removes, -1 only queries; *listed (nullable) = membership after the op.  The manager never fuses
+ * a blacklisted BE kernel (it is still reordered / run on an idle GPU). */
+tacker_status tacker_blacklist(const char *be_key, int32_t op, int32_t *listed);
+tacker_status tacker_blacklist_clear(void);
+
 /* Diagnostics: copies the LC role clock64 stamps recorded by plans built with TACKER_LC_DBG bit 3
  * ([160 CTAs][5 events][16 work units], see fused.cuh) into out (>= 12800 slots). */
 tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n);

@@ -44,6 +44,7 @@
 namespace tkrt {
 bool make_keys(const tacker_lc_desc *lc, const tacker_be_desc *be, int warp_split, std::string *lk, std::string *bk,
                std::string *pk);
+bool blacklist_op(const std::string &be_key, int op);
 }
 using namespace tkrt;
 
@@ -277,10 +278,13 @@ static bool app_ready(tacker_manager_s *m, const App &a, double t) {
   return true;
 }
 
+// pair-model key of (TC kernel k, BE CUDA-core kernel b); false for a blacklisted BE kernel (NEXT-1,
+// never considered for fusion)
 static bool pair_key(const tacker_lc_kernel &k, const tacker_be_kernel &b, std::string *pk) {
   std::string lk, bk;
   const int ws = b.warp_split ? b.warp_split : 16;
-  return make_keys(&k.lc, &b.be, ws, &lk, &bk, pk);
+  if (!make_keys(&k.lc, &b.be, ws, &lk, &bk, pk)) return false;
+  return !blacklist_op(bk, -1);
 }
 static bool pair_time(const tacker_lc_kernel &k, const tacker_be_kernel &b, double *tf) {
   std::string pk;

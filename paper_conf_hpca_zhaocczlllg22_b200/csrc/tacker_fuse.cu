@@ -16,6 +16,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <set>
 #include <memory>
 #include <string>
 #include <unordered_map>
@@ -747,6 +748,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   return TACKER_OK;
 }
 
+namespace tkrt {
+bool blacklist_op(const std::string &be_key, int op);
+}
+
 static std::atomic<int> g_overlap{TACKER_OVERLAP_DEFAULT};
 
 // cudaLaunchKernelEx with programmatic stream serialization (PDL) unless disabled for this
@@ -798,6 +803,69 @@ static tacker_status launch_plan(tacker_fused_s &F, cudaStream_t s) { return lau
 extern "C" {
 
 const char *tacker_last_error(void) { return g_err.c_str(); }
+
+tacker_status tacker_select_fusion(const tacker_lc_desc *lc, const tacker_be_desc *be, const int32_t *splits,
+                                   int32_t n_splits, int32_t reps, tacker_stream_t s, int32_t *best_ws,
+                                   double *best_ms, double *seq_ms, double *fused_ms) {
+  if (!lc || !be || !splits || n_splits <= 0 || reps <= 0 || !best_ws || !best_ms || !seq_ms)
+    return set_error("tacker_select_fusion: bad arguments"), TACKER_EINVAL;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(s);
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  auto time_it = [&](auto &&launch, double *ms) -> tacker_status {
+    if (tacker_status r = launch()) return r;   // warm-up
+    cudaEventRecord(e0, st);
+    for (int i = 0; i < reps; ++i)
+      if (tacker_status r = launch()) return r;
+    cudaEventRecord(e1, st);
+    cudaError_t e = cudaEventSynchronize(e1);
+    if (e != cudaSuccess) return cuda_fail("select_fusion sync", e);
+    float f = 0;
+    cudaEventElapsedTime(&f, e0, e1);
+    *ms = (double)f / reps;
+    return TACKER_OK;
+  };
+  tacker_status r = time_it([&] { return tacker_launch_original(lc, be, s); }, seq_ms);
+  *best_ws = 0;
+  *best_ms = *seq_ms;
+  for (int32_t i = 0; r == TACKER_OK && i < n_splits; ++i) {
+    if (fused_ms) fused_ms[i] = NAN;
+    tacker_fused_t f = nullptr;
+    tacker_status fs = tacker_fuse(lc, be, splits[i], tacker_ratio{0, 0}, &f);
+    if (fs == TACKER_ERESOURCE || fs == TACKER_EUNSUPPORTED) continue;   // not a candidate
+    if (fs) {
+      r = fs;
+      break;
+    }
+    double ms = 0;
+    r = time_it([&] { return tacker_launch_fused(f, s); }, &ms);
+    tacker_fused_destroy(f);
+    if (r) break;
+    if (fused_ms) fused_ms[i] = ms;
+    if (ms < *best_ms) {
+      *best_ms = ms;
+      *best_ws = splits[i];
+    }
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (r) return r;
+  if (*best_ws == 0) tkrt::blacklist_op(be_key_of(*be), 1);
+  return TACKER_OK;
+}
+
+tacker_status tacker_blacklist(const char *be_key, int32_t op, int32_t *listed) {
+  if (!be_key || op < -1 || op > 1) return set_error("tacker_blacklist: bad arguments"), TACKER_EINVAL;
+  const bool in = tkrt::blacklist_op(be_key, op);
+  if (listed) *listed = in ? 1 : 0;
+  return TACKER_OK;
+}
+
+tacker_status tacker_blacklist_clear(void) {
+  tkrt::blacklist_op("", 2);
+  return TACKER_OK;
+}
 
 tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n) {
   if (!out || n < 160 * 5 * 16) return set_error("need 12800 uint64 slots"), TACKER_EINVAL;
@@ -996,6 +1064,20 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
 
 // accessors used by the predictor / manager translation units
 namespace tkrt {
+// BE-kernel blacklist (NEXT-1): op 1 add, 0 remove, -1 query, 2 clear; returns membership
+bool blacklist_op(const std::string &be_key, int op) {
+  static std::mutex mu;
+  static std::set<std::string> listed;
+  std::lock_guard<std::mutex> g(mu);
+  if (op == 2) {
+    listed.clear();
+    return false;
+  }
+  if (op == 1) listed.insert(be_key);
+  if (op == 0) listed.erase(be_key);
+  return listed.count(be_key) != 0;
+}
+
 const std::string &fused_lc_key(tacker_fused_t f) { return f->lc_key; }
 const std::string &fused_be_key(tacker_fused_t f) { return f->be_key; }
 const std::string &fused_pair_key(tacker_fused_t f) { return f->pair_key; }

@@ -191,26 +191,21 @@ class QosRun:
                 self.t_be[(a, j)] = _time(lambda: tk.tacker_launch_original(None, bk.desc), reps)
                 if self.t_be[(a, j)] >= 0.01 and bk.desc.kind != tk.BE_JDS_SCAN:
                     self.lr_be[(a, j)] = self._fit_slice_lr(a, j, bk, reps)
-        # warp split per BE kernel (NEXT-1): the fastest fused launch with a
-        # representative LC kernel among the splits that fit the budget
+        # NEXT-1 through the C ABI: per BE kernel, every fused candidate
+        # (warp split) with a representative LC kernel and the sequential pair are timed; the fastest
+        # split is kept, and a BE kernel for which sequential wins is blacklisted (never fused)
         tcs = [k for k in self.svc.kernels if k.is_tc]
+        tk.tacker_blacklist_clear()
+        self.selection = {}
         for a, app in enumerate(self.apps):
             for j, bk in enumerate(app.kernels):
                 if self.t_be[(a, j)] < 0.01 or bk.is_tc:
                     continue
-                best = None
-                for ws in range(self.ws, 3, -4):
-                    try:
-                        f = tk.tacker_fuse(tcs[len(tcs) // 2].lc, bk.desc, ws)
-                    except tk.TackerError as e:
-                        if e.status not in (tk.ERESOURCE, tk.EUNSUPPORTED):
-                            raise
-                        continue
-                    t = _time(lambda: f.launch(), 3)
-                    if best is None or t < best[0]:
-                        best = (t, ws)
-                if best is not None:
-                    self.ws_of[(a, j)] = best[1]
+                best, best_ms, seq_ms, cand = tk.tacker_select_fusion(
+                    tcs[len(tcs) // 2].lc, bk.desc, splits=tuple(range(self.ws, 3, -4)), reps=3)
+                self.selection[bk.name] = {"best_ws": best, "best_ms": best_ms, "seq_ms": seq_ms, "fused_ms": cand}
+                if best > 0:
+                    self.ws_of[(a, j)] = best
         # two-stage models per (LC class, BE class, ws), trained on block prefixes
         off = 1 if getattr(self, "io", None) else 0      # t_lc index of svc.kernels[0]
         refit = set()

@@ -264,6 +264,10 @@ _PROTOS = {
     "tacker_launch_fused_slice": ([_V, _I64, _I64, _V], C.c_int),
     "tacker_set_launch_overlap": ([_I32], C.c_int),
     "tacker_debug_lc_timestamps": ([C.POINTER(C.c_uint64), _I64], C.c_int),
+    "tacker_select_fusion": ([C.POINTER(LcDesc), C.POINTER(BeDesc), C.POINTER(_I32), _I32, _I32, _V,
+                              C.POINTER(_I32), C.POINTER(_D), C.POINTER(_D), C.POINTER(_D)], C.c_int),
+    "tacker_blacklist": ([C.c_char_p, _I32, C.POINTER(_I32)], C.c_int),
+    "tacker_blacklist_clear": ([], C.c_int),
     "tacker_launch_original": ([C.POINTER(LcDesc), C.POINTER(BeDesc), _V], C.c_int),
     "tacker_model_add_sample": ([_S, _D, _D], C.c_int),
     "tacker_model_fit": ([_S, C.POINTER(_D), C.POINTER(_D)], C.c_int),
@@ -607,6 +611,29 @@ def tacker_fuse(lc: LcDesc, be: BeDesc | None, warp_split: int, block_ratio=(0, 
 
 def tacker_launch_fused(f: Fused, stream=None):
     f.launch(stream)
+
+
+def tacker_select_fusion(lc: LcDesc, be: BeDesc, splits=(24, 20, 16, 12, 8, 4), reps=5, stream=None):
+    """NEXT-1: time every fused candidate and the sequential pair; returns
+    (best warp split or 0 = do not fuse, best ms, sequential ms, {split: fused ms})."""
+    n = len(splits)
+    arr = (C.c_int32 * n)(*splits)
+    best, bms, sms = C.c_int32(), C.c_double(), C.c_double()
+    fms = (C.c_double * n)()
+    _chk(_lib.tacker_select_fusion(C.byref(lc), C.byref(be), arr, n, reps, _stream(stream), C.byref(best),
+                                   C.byref(bms), C.byref(sms), fms))
+    return best.value, bms.value, sms.value, {s: fms[i] for i, s in enumerate(splits) if fms[i] == fms[i]}
+
+
+def tacker_blacklist(be_key: str, op: int = -1) -> bool:
+    """op 1 add, 0 remove, -1 query; returns membership."""
+    v = C.c_int32()
+    _chk(_lib.tacker_blacklist(be_key.encode(), op, C.byref(v)))
+    return bool(v.value)
+
+
+def tacker_blacklist_clear():
+    _chk(_lib.tacker_blacklist_clear())
 
 
 def tacker_debug_lc_timestamps():

@@ -437,3 +437,35 @@ def test_manager_trace_replay_sim(tk, policy):
     bad[i]["thr"] += 0.5
     with pytest.raises(AssertionError):
         check_trace(bad, queries, apps, 50.0, mr.BAYMAX if policy == "baymax" else mr.TACKER, idle_cap=2.0, **rules)
+
+
+def test_blacklist_and_manager_never_fuses_listed_kernel(tk):
+    """NEXT-1: a blacklisted BE kernel is never fused; the C manager's decisions then
+    equal the reference's with that app's kernels marked never-fusable."""
+    tk.tacker_blacklist_clear()
+    assert not tk.tacker_blacklist("be:stencil:nz8")
+    assert tk.tacker_blacklist("be:stencil:nz8", 1)
+    assert tk.tacker_blacklist("be:stencil:nz8", -1)
+    assert not tk.tacker_blacklist("be:stencil:nz8", 0)
+    tk.tacker_model_clear()
+    tau = lambda r: max(1 + 0.25 * r, 0.4 + 0.93 * r)
+    fit_pair_closed_form(tk, tau)
+    fuse_pred = lambda ttc, tcd: ttc * tau(tcd / ttc)
+    rng = np.random.default_rng(23)
+    arrivals = np.cumsum(rng.exponential(6.0, 40))
+    shapes = [[(True, 1.21), (False, 0.3), (True, 0.83)], [(True, 0.52), (True, 0.49)]]
+    for listed in (False, True):
+        if listed:
+            tk.tacker_blacklist("be:stencil:nz8", 1)     # the BE kernels' model key (stencil nz=8)
+        m = tk.Manager(tk.POLICY_TACKER, simulate=True, idle_cap_ms=2.0)
+        qs = []
+        for i, t in enumerate(arrivals):
+            m.submit_lc([lc_kernel(tk, tc, d) for tc, d in shapes[i % 2]], float(t))
+            qs.append(mr.Query(i, float(t), list(shapes[i % 2])))
+        m.submit_be([be_kernel(tk, 1.53), be_kernel(tk, 0.71)])
+        app = mr.App([(mr.BE_OTHER if listed else mr.BE_CD, 1.53), (mr.BE_OTHER if listed else mr.BE_CD, 0.71)])
+        ref = mr.simulate(qs, [app], 50.0, mr.TACKER, fuse_pred, idle_cap=2.0)
+        m.run(50.0, float(arrivals[-1]))
+        assert m.stats().fused_launches == sum(d.action == mr.FUSED for d in ref["decisions"])
+        assert (m.stats().fused_launches == 0) == listed
+    tk.tacker_blacklist_clear()

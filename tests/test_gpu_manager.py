@@ -137,3 +137,22 @@ def test_gpu_manager_trace_replays_through_reference(tk, rules):
     n = check_trace(res["trace"], queries, apps, run.qos, mr.TACKER, idle_cap=cap if cap > 0 else None, **ref_rules)
     assert n == len(res["trace"])
     assert res["qos_met"], res
+
+
+def test_select_fusion_through_c_abi(tk):
+    """NEXT-1: tacker_select_fusion times every fused candidate and the sequential pair on the GPU;
+    the returned split is the fastest (or 0 = sequential, which blacklists the BE kernel)."""
+    from paper_conf_hpca_zhaocczlllg22_b200 import services as sv
+    cs = next(c for c in synth.resnet50_convs(8) if c.name == "layer2.1.conv2")
+    svc = sv.resnet50_service(8, convs=[cs])
+    mq = sv.mriq_app(64, 1024, 1024)
+    tk.tacker_launch_original(None, mq.kernels[0].desc)
+    tk.tacker_blacklist_clear()
+    best, best_ms, seq_ms, cand = tk.tacker_select_fusion(svc.kernels[0].lc, mq.kernels[1].desc, (24, 16, 8, 4), 3)
+    assert seq_ms > 0 and cand, (best, cand)
+    assert best_ms == min([seq_ms] + list(cand.values()))
+    key = tk.tacker_fuse(svc.kernels[0].lc, mq.kernels[1].desc, 4).keys()[1]
+    assert tk.tacker_blacklist(key) == (best == 0)
+    if best:
+        assert cand[best] == best_ms
+    tk.tacker_blacklist_clear()
