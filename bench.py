@@ -601,6 +601,9 @@ def run_tacker(args, comm):
         "fused_launches": res["fused"], "reordered_be": res["reordered"], "idle_be": res["idle_be"],
         "model_refits": res["model_refits"], "fused_pred_err_mean": res["fused_pred_err_mean"],
         "pair_pred_err_mean": statistics.mean(q.pair_err) if q.pair_err else None,
+        # NEXT-1 selection per BE kernel (tacker_select_fusion): best warp split, 0 = sequential won
+        # (blacklisted, never fused)
+        "fusion_selection": {k: v["best_ws"] for k, v in getattr(q, "selection", {}).items()},
         # Eq. 10 on normalised BE throughput (app-length independent) and on kernels/s
         "improvement_vs_baymax_same_rule_eq10_normalised": eq10(res, same, "be_norm_thpt"),
         "improvement_vs_baymax_same_rule_eq10": eq10(res, same, "be_kernels_per_s"),

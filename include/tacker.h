@@ -255,6 +255,15 @@ typedef struct {
 /* Whole-problem block counts ("number of blocks in non-PTB mode", §VI-C). */
 tacker_status tacker_be_num_blocks(const tacker_be_desc *be, int64_t *out);
 tacker_status tacker_lc_num_tiles(const tacker_lc_desc *lc, int32_t tile_n, int64_t *out);
+/* Per-kernel LR features (§VI-C) that follow the hardware's cost better than a block
+ * count.  LC: waves = ceil(work units / CTAs) of the LC-only persistent launch (tiles of one wave run
+ * concurrently: the time steps with the wave count, not the tile count).  BE: the algorithmic work
+ * of the first n original blocks -- spmv JDS: 8 nnz + 16 rows bytes of those rows (rows sorted by
+ * length, the first blocks are the heaviest); cutcp: (lattice point, neighbour-bin atom) pairs of
+ * those bins; every other kind: n.  Reads small device arrays (row lengths, bin counts) and
+ * synchronises: calibration only. */
+tacker_status tacker_lc_num_waves(const tacker_lc_desc *lc, int32_t tile_n, int64_t *out);
+tacker_status tacker_be_prefix_work(const tacker_be_desc *be, int64_t n_blocks, double *work);
 
 /* ======================================================================== fusion (a1)
  * tacker_fuse: admission + resource split of one fused kernel (§V-B/C P:1117-1309,

@@ -85,7 +85,9 @@ class TwoStage:
                 break
             nlo = [p for p in pts if p[0] <= rs]
             nhi = [p for p in pts if p[0] > rs]
-            if len(nlo) < 1 or len(nhi) < 1 or (nlo == lo and nhi == hi):
+            # each stage is a line through >= 2 samples (one LR per stage): a re-split
+            # leaving a stage one sample would fix no slope (OLS slope 0, a flat stage)
+            if len(nlo) < 2 or len(nhi) < 2 or (nlo == lo and nhi == hi):
                 break
             lo, hi = nlo, nhi
         return self.l1, self.l2

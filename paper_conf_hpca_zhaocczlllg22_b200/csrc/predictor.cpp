@@ -77,7 +77,9 @@ bool fit_pair(Pair &P, double split) {
     const double rs = (P.a2 - P.a1) / (P.b1 - P.b2);
     std::vector<std::pair<double, double>> nlo, nhi;
     for (auto &q : pts) (q.first <= rs ? nlo : nhi).push_back(q);
-    if (nlo.empty() || nhi.empty() || (nlo == lo && nhi == hi)) break;
+    // each stage is a line through >= 2 samples (one LR per stage): a re-split leaving
+    // a stage one sample would fix no slope (OLS slope 0, a flat stage)
+    if (nlo.size() < 2 || nhi.size() < 2 || (nlo == lo && nhi == hi)) break;
     lo.swap(nlo);
     hi.swap(nhi);
   }

@@ -16,6 +16,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <cmath>
+#include <vector>
 #include <set>
 #include <memory>
 #include <string>
@@ -897,6 +899,61 @@ tacker_status tacker_lc_num_tiles(const tacker_lc_desc *lc, int32_t tile_n, int6
   if (BN != 64 && BN != 128 && BN != 256) return set_error("tile_n must be 64/128/256"), TACKER_EINVAL;
   lc_tiles(L, BN);
   *out = L.num_tiles;
+  return TACKER_OK;
+}
+
+tacker_status tacker_lc_num_waves(const tacker_lc_desc *lc, int32_t tile_n, int64_t *out) {
+  if (!lc || !out) return set_error("null argument"), TACKER_EINVAL;
+  LcParams L;
+  tacker_status st = lc_view(*lc, L);
+  if (st) return st;
+  int BN = tile_n ? tile_n : pick_tile_n(*lc, L);
+  if (BN != 64 && BN != 128 && BN != 256) return set_error("tile_n must be 64/128/256"), TACKER_EINVAL;
+  lc_tiles(L, BN);
+  const int sms = sm_count() > 0 ? sm_count() : 148;
+  if (!(lc->epi_flags & TACKER_LC_NO_SPLIT)) lc_split(L, sms);
+  const int grid = L.num_units < sms ? L.num_units : sms;
+  *out = (L.num_units + grid - 1) / grid;
+  return TACKER_OK;
+}
+
+tacker_status tacker_be_prefix_work(const tacker_be_desc *be, int64_t n, double *work) {
+  if (!be || !work || n < 0) return set_error("bad argument"), TACKER_EINVAL;
+  int64_t full = 0;
+  if (!be_num_blocks(*be, &full)) return set_error("bad BE descriptor"), TACKER_EINVAL;
+  n = std::min(n, full);
+  if (be->kind == TACKER_BE_SPMV_JDS) {
+    const tacker_be_spmv &p = be->p.spmv;
+    const int64_t rows = std::min<int64_t>((int64_t)p.rows, n * 128);
+    std::vector<int32_t> len((size_t)rows);
+    cudaError_t e = cudaMemcpy(len.data(), p.row_len, (size_t)rows * 4, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_fail("prefix work (spmv row lengths)", e);
+    double nnz = 0;
+    for (int32_t l : len) nnz += l;
+    *work = 8.0 * nnz + 16.0 * (double)rows;
+    return TACKER_OK;
+  }
+  if (be->kind == TACKER_BE_CUTCP) {
+    const tacker_be_cutcp &p = be->p.cutcp;
+    const int64_t nb = (int64_t)p.bdim_x * p.bdim_y * p.bdim_z;
+    std::vector<int32_t> cnt((size_t)nb);
+    cudaError_t e = cudaMemcpy(cnt.data(), p.count, (size_t)nb * 4, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_fail("prefix work (cutcp bin counts)", e);
+    const int reach = (int)std::ceil(p.cutoff / p.bin_size);
+    double w = 0;
+    for (int64_t b = 0; b < n; ++b) {   // block b = bin b in (z, y, x) order: its 512 points x neighbour atoms
+      const int bx = (int)(b % p.bdim_x), by = (int)((b / p.bdim_x) % p.bdim_y), bz = (int)(b / ((int64_t)p.bdim_x * p.bdim_y));
+      int64_t atoms = 0;
+      for (int z = std::max(bz - reach, 0); z <= std::min(bz + reach, p.bdim_z - 1); ++z)
+        for (int y = std::max(by - reach, 0); y <= std::min(by + reach, p.bdim_y - 1); ++y)
+          for (int x = std::max(bx - reach, 0); x <= std::min(bx + reach, p.bdim_x - 1); ++x)
+            atoms += std::min(cnt[((size_t)z * p.bdim_y + y) * p.bdim_x + x], p.bin_depth);
+      w += 512.0 * (double)atoms;
+    }
+    *work = w;
+    return TACKER_OK;
+  }
+  *work = (double)n;
   return TACKER_OK;
 }
 

@@ -255,6 +255,8 @@ _PROTOS = {
     "tacker_last_error": ([], _S), "tacker_version": ([], _S), "tacker_device_sm_count": ([], C.c_int),
     "tacker_be_num_blocks": ([C.POINTER(BeDesc), C.POINTER(_I64)], C.c_int),
     "tacker_lc_num_tiles": ([C.POINTER(LcDesc), _I32, C.POINTER(_I64)], C.c_int),
+    "tacker_lc_num_waves": ([C.POINTER(LcDesc), _I32, C.POINTER(_I64)], C.c_int),
+    "tacker_be_prefix_work": ([C.POINTER(BeDesc), _I64, C.POINTER(_D)], C.c_int),
     "tacker_fuse": ([C.POINTER(LcDesc), C.POINTER(BeDesc), _I32, Ratio, C.POINTER(_V)], C.c_int),
     "tacker_fused_destroy": ([_V], C.c_int),
     "tacker_fused_info": ([_V, C.POINTER(FusedInfo)], C.c_int),
@@ -552,6 +554,18 @@ def tacker_last_error() -> str:
 def tacker_be_num_blocks(be: BeDesc) -> int:
     v = C.c_int64()
     _chk(_lib.tacker_be_num_blocks(C.byref(be), C.byref(v)))
+    return v.value
+
+
+def tacker_lc_num_waves(lc: LcDesc, tile_n: int = 0) -> int:
+    v = C.c_int64()
+    _chk(_lib.tacker_lc_num_waves(C.byref(lc), tile_n, C.byref(v)))
+    return v.value
+
+
+def tacker_be_prefix_work(be: BeDesc, n_blocks: int) -> float:
+    v = C.c_double()
+    _chk(_lib.tacker_be_prefix_work(C.byref(be), n_blocks, C.byref(v)))
     return v.value
 
 

@@ -71,6 +71,7 @@ def test_managed_reverse_fusion_outputs_match_standalone(tk):
     assert host(svc.outputs[-1]).tobytes() == ref
     # the GPU reverse-fused launch path, whatever this box measured: a model with a sure gain
     tk.tacker_model_clear()
+    tk.tacker_blacklist_clear()
     for r in (0.1, 0.2, 1.8, 1.9):
         tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0, r) + 0.05)
     tk.tacker_pair_fit(pk)
@@ -98,8 +99,9 @@ def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
     run.measure_service(n=20)
     assert run.pairs, "no fusable pair calibrated"
     # the launch paths under test must run whatever this box measured: pair models with a sure
-    # gain (tau = max(1 + 0.1 r, 0.5 + r), opportune ratio 5/9)
+    # gain (tau = max(1 + 0.1 r, 0.5 + r), opportune ratio 5/9), no BE kernel blacklisted
     tk.tacker_model_clear()
+    tk.tacker_blacklist_clear()
     for pk in run.pairs:
         for r in (0.1, 0.2, 1.8, 1.9):
             tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0 + 0.1 * r, 0.5 + r))

@@ -288,3 +288,21 @@ def test_overlap_rate_bounds():
 def test_rel_err_uses_abs_sum():
     assert metrics.max_rel_err([1e-3], [0.0], [1.0]) == pytest.approx(1e-3)
     assert metrics.max_rel_err([2.0], [1.0]) == 1.0
+
+
+def test_two_stage_refit_keeps_two_samples_per_stage():
+    """Reading 5: the iterative re-split at r* never leaves a stage one sample.  Pin:
+    the samples of a measured pair (BERT O-projection GEMM x cutcp, ws 24; r = X_cd / X_tc,
+    tau = T_fused / X_tc) whose two stages are nearly parallel: r* lands beyond all but the last
+    sample, and the old rule re-split to {5 | 1} samples, fitting a flat stage 2 (slope 0) through the
+    single point -- every prediction below r = 17 became that point's tau (errors up to 3.7x on the
+    pair's held-out prefixes).  Kept at the median split, both stages have slope ~1."""
+    r = [1.529, 2.027, 3.333, 4.558, 8.204, 16.31]
+    tau = [2.471, 3.288, 4.258, 5.623, 8.747, 17.416]
+    m = predictor.TwoStage()
+    for x, y in zip(r, tau):
+        m.add(1.0, x, y)
+    (a1, b1), (a2, b2) = m.fit()
+    assert b2 > 0.5 and b1 > 0.5                     # neither stage flat
+    for x, y in ((3.456, 4.383), (8.581, 8.787), (11.902, 12.80), (15.312, 17.09)):   # held-out prefixes
+        assert abs(m.tau(x) - y) / y < 0.12, (x, m.tau(x), y)

@@ -82,6 +82,9 @@ def main():
     ap.add_argument("--out", default="")
     ap.add_argument("--models", default="")
     ap.add_argument("--batch", type=int, default=128, help="BERT-base seq-128 batch (LC GEMM M = 128 x batch)")
+    ap.add_argument("--features", default="hw", choices=["hw", "blocks"],
+                    help="per-kernel LR feature: hw = LC waves / BE prefix work (tacker_lc_num_waves, "
+                         "tacker_be_prefix_work); blocks = tiles / original blocks (round 1)")
     args = ap.parse_args()
     wss = [int(w) for w in args.ws.split(",")]
     tk.tacker_model_clear()
@@ -98,7 +101,7 @@ def main():
         key = None
         for M in Ms + held:
             d = tk.lc_gemm(dA, dB, D, M=M)
-            tiles = tk.tacker_lc_num_tiles(d)
+            tiles = tk.tacker_lc_num_waves(d) if args.features == "hw" else tk.tacker_lc_num_tiles(d)
             t = timeit(lambda: tk.tacker_launch_original(d, None))
             if key is None:
                 f = tk.tacker_fuse(d, None, 0)
@@ -114,6 +117,7 @@ def main():
     # ---------------- BE per-kernel LR over original blocks
     bes = be_kernels()
     be_lr = {}
+    be_x = {}
     for name, (mk, keep) in bes.items():
         full = tk.tacker_be_num_blocks(mk())
         fr = [0.05, 0.1, 0.2, 0.35, 0.5, 0.75, 1.0]
@@ -128,11 +132,14 @@ def main():
                 A = torch.zeros(128, 64, dtype=torch.float16, device="cuda")
                 Dd = torch.zeros(128, 8, device="cuda")
                 key = tk.tacker_fuse(tk.lc_gemm(A, A[:8], Dd), d, 8).keys()[1]
+            x = tk.tacker_be_prefix_work(d, n) if args.features == "hw" else n
             if f_ in fr:
-                tk.tacker_model_add_sample(key, n, t)
+                tk.tacker_model_add_sample(key, x, t)
             samples.append((n, t, f_ in held))
         a, b = tk.tacker_model_fit(key)
-        errs = [abs(tk.tacker_model_predict(key, n) - t) / t for n, t, h in samples if h]
+        xf = (lambda n: tk.tacker_be_prefix_work(mk(n), n)) if args.features == "hw" else (lambda n: n)
+        be_x[name] = xf
+        errs = [abs(tk.tacker_model_predict(key, xf(n)) - t) / t for n, t, h in samples if h]
         be_lr[name] = (key, a, b, full)
         res["be_lr"][name] = {"key": key, "a": a, "b": b, "full_blocks": full, "max_err": max(errs),
                               "samples": [(n, t) for n, t, _ in samples]}
@@ -140,7 +147,7 @@ def main():
     train_r = [0.1, 0.2, 1.8, 1.9]
     eval_r = [0.05, 0.3, 0.5, 0.7, 0.9, 1.0, 1.2, 1.4, 1.6, 2.2, 2.6, 3.0]
     for lname, (lcd, lkey, _) in lcs.items():
-        tiles = tk.tacker_lc_num_tiles(lcd)
+        tiles = tk.tacker_lc_num_waves(lcd) if args.features == "hw" else tk.tacker_lc_num_tiles(lcd)
         x_tc_pred = tk.tacker_model_predict(lkey, tiles)
         x_tc = timeit(lambda: tk.tacker_launch_original(lcd, None))
         for bname, (mk, _) in bes.items():
@@ -184,7 +191,7 @@ def main():
                 errs, errs_meas, ev = [], [], []
                 for n in er:
                     x_cd, t_f = run_n(n)
-                    pred = tk.tacker_pair_predict(pkey, x_tc_pred, tk.tacker_model_predict(bkey, n))
+                    pred = tk.tacker_pair_predict(pkey, x_tc_pred, tk.tacker_model_predict(bkey, be_x[bname](n)))
                     pred_m = tk.tacker_pair_predict(pkey, x_tc, x_cd)   # model error alone
                     errs.append(abs(pred - t_f) / t_f)
                     errs_meas.append(abs(pred_m - t_f) / t_f)
