@@ -27,7 +27,7 @@ Rules, in the paper's order:
     becomes ready when the previous one completes.
   * Baymax mode = the same manager with fusion disabled ("static scheduling").
   * Idle GPU (no active LC query; the paper is silent): launch one ready BE head whose
-    duration <= idle_cap, round robin over apps.
+    duration <= idle_cap, the apps taken round robin from the one after the last idle launch.
   * PTB slicing (B200 reading 13 in DESIGN.md §2; off by default): with slice_be, the BE part of
     a fused launch is a slice of n of the head kernel's N original blocks (PTB, Fig. 7), with
     predicted standalone time X_cd(n) = t_floor + t_block * n (the kernel's LR, §VI-C
@@ -196,6 +196,12 @@ def slice_blocks(app, ttc, r_opp, slice_be, slice_ratio):
     return n if n < R else -1
 
 
+def _round_robin(cands, rr):
+    """Idle-GPU candidates [(app, T)] in round-robin order from app rr[0] (B200 reading, the paper is
+    silent on an idle GPU: no BE app starves behind a lower-numbered one)."""
+    return [c for c in cands if c[0] >= rr[0]] + [c for c in cands if c[0] < rr[0]]
+
+
 def _first_issue(q, active, t, qos, heads, direct_eps, direct_rule, fuse_older):
     """Eq. 9 at the first issue of q and the direct rule."""
     q.issue = t
@@ -248,6 +254,7 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
     pending = sorted(queries, key=lambda q: q.arrival)
     timeline, decisions = [], []
     qi = 0
+    rr = [0]   # idle launches: round robin over the apps
     while True:
         while qi < len(pending) and pending[qi].arrival <= t:
             active.append(pending[qi])
@@ -309,9 +316,10 @@ def simulate(queries, apps, qos, policy, fuse_pred, direct_eps=0.0, idle_cap=Non
                 apps[a].ready_at = t
         else:
             nxt = pending[qi].arrival if qi < len(pending) else None
-            cands = [(a, d) for a, d, _ in heads if idle_cap is None or d <= idle_cap]
+            cands = _round_robin([(a, d) for a, d, _ in heads if idle_cap is None or d <= idle_cap], rr)
             if cands:
                 a, d = cands[0]
+                rr[0] = a + 1
                 timeline.append(("be", -1, -1, a, t, t + d))
                 decisions.append(Decision(IDLE_BE, None, -1, [a], 0.0))
                 apps[a].issue(-1)
@@ -343,14 +351,18 @@ def replay(trace, queries, apps, qos, policy, direct_eps=0.0, idle_cap=None, reo
     the manager reports it: the effective bound of an older query under reading 18)."""
     by_id = {q.qid: q for q in queries}
     out = []
+    rr = [0]
     for rec in trace:
         t, act_ids, tf, ready = rec["t"], rec["active"], rec["tk_fuse"], set(rec["ready"])
         active = [by_id[i] for i in act_ids]
         heads = [(a, app.rem(), app.head()[0]) for a, app in enumerate(apps) if a in ready]
         work = [q for q in active if q.pos < len(q.kernels)]
         if not work:
-            cands = [a for a, d, _ in heads if (idle_cap is None or d <= idle_cap)] if not active else []
+            cands = [a for a, _ in _round_robin([(a, d) for a, d, _ in heads if idle_cap is None or d <= idle_cap],
+                                                rr)] if not active else []
             a = cands[0] if cands else -1
+            if a >= 0:
+                rr[0] = a + 1
             out.append(Decision(IDLE_BE, None, -1, [a] if a >= 0 else [], 0.0))
             if a >= 0:
                 apps[a].issue(-1)

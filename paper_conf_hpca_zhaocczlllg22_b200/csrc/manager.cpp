@@ -26,6 +26,7 @@
 // manager launches on its stream and observes completion with CUDA events.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -132,6 +133,7 @@ struct tacker_manager_s {
   };
   std::deque<Observed> observed;   // fused launches awaiting their measured duration
   int64_t refits = 0;
+  int idle_rr = 0;                 // idle launches: the next app in round-robin order
   size_t prepared = 0;                                   // queries visited by tacker_manager_prepare
   std::set<std::array<const void *, 3>> prepared_lc;     // LC operand triples already prepared
   double be_work_ms = 0;           // sum of standalone (predicted) times of issued BE kernels
@@ -576,7 +578,9 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
     }
 
   if (qid < 0) {
-    // idle GPU (or only tails of earlier queries still running): one bounded BE kernel
+    // idle GPU (or only tails of earlier queries still running): one bounded BE kernel, the apps
+    // taken round robin from the one after the last idle launch (no app starves behind another)
+    std::rotate(heads.begin(), std::lower_bound(heads.begin(), heads.end(), m->idle_rr), heads.end());
     for (int a : heads) {
       const double tt = rem_ms(m->apps[a]);
       if (m->prm.idle_cap_ms > 0 && tt > m->prm.idle_cap_ms) continue;
@@ -584,6 +588,7 @@ static tacker_status step_impl(tacker_manager_t m, double qos, double *headroom,
       out->action = TACKER_DEC_IDLE_BE;
       out->n_reorder = 1;
       out->reorder_apps[0] = a;
+      m->idle_rr = a + 1;
       App &A = m->apps[a];
       if (m->sim()) {
         m->now += tt;

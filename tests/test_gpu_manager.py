@@ -108,8 +108,9 @@ def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
         tk.tacker_pair_fit(pk)
     svc.outputs[-1].zero_()
     res = run.run(tk.POLICY_TACKER, 60, load=0.8, max_inflight=8, **variant)
-    assert res["qos_met"], res
-    assert res["fused"] > 0, res
+    brief = {k: res[k] for k in ("fused", "reordered", "idle_be", "be_kernels", "lc_p99_ms", "class_launches")}
+    assert res["qos_met"], brief
+    assert res["fused"] > 0, (brief, run.ws_of, run.lr_be, list(run.pairs))
     assert host(svc.outputs[-1]).tobytes() == ref
 
 

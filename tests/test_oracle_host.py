@@ -306,3 +306,15 @@ def test_two_stage_refit_keeps_two_samples_per_stage():
     assert b2 > 0.5 and b1 > 0.5                     # neither stage flat
     for x, y in ((3.456, 4.383), (8.581, 8.787), (11.902, 12.80), (15.312, 17.09)):   # held-out prefixes
         assert abs(m.tau(x) - y) / y < 0.12, (x, m.tau(x), y)
+
+
+def test_manager_idle_round_robin():
+    """Idle GPU (B200 reading, DESIGN.md §2 reading 6): BE heads launched round robin over the apps
+    from the one after the last idle launch -- a 5 ms app 0 does not starve a 1 ms app 1."""
+    apps = [mr.App([(True, 5.0)]), mr.App([(True, 1.0)])]
+    q = mr.Query(0, 13.0, [(True, 1.0)])
+    res = mr.simulate([q], apps, 50.0, mr.TACKER, lambda a, b: None, idle_cap=10.0)
+    idle = [d.reorder[0] for d in res["decisions"] if d.action == mr.IDLE_BE]
+    assert idle[:4] == [0, 1, 0, 1]
+    # 0..5 app 0, 5..6 app 1, 6..11 app 0, 11..12 app 1, 12..17 app 0 -> the query (13) waits to 17
+    assert res["latency"][0] == 17.0 - 13.0 + 1.0
