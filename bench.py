@@ -368,43 +368,74 @@ def be_class_roofline(q, peaks, apps):
 
 
 # ----------------------------------------------------------------------------- CPU oracle baseline
-def cpu_oracle_sample(small=False, batch=32):
-    """The oracle as it stands on a bounded sample of the same workload: oracle conv of two
-    ResNet-50 layers on one image (time x batch: the conv is linear in the batch) + one stencil
-    sweep (512x512x64, or an 8-plane slab scaled x8 when small) + one mri-q 1024-k chunk on 4096
-    (small: 256) of the 64^3 voxels, time scaled to the full kernel.  Returns BE kernels/s =
-    1 / mean (LC conv + BE kernel) pair time."""
+def cpu_oracle_sample(small=False, batch=32, be="table2"):
+    """The oracle as it stands on a bounded sample of the same workload: the oracle conv of two
+    ResNet-50 layers on one image (time x batch: the conv is linear in the batch) paired with each
+    BE kernel of the queue, every BE kernel computed on a bounded part of its problem and its time
+    scaled to the whole kernel (the oracle's cost is linear in the part).  Table II queue: mri-q
+    and mri-fhd chunks on 256 of the 64^3 voxels (x1024), fft on 16 of the 16384 transforms
+    (x1024), cutcp on 512 of the 96^3 lattice points (x1728), cp on a 32x32 corner of the 512^2
+    slice (x256), sgemm on 64 of the 2048 rows (x32), lbm on a 120x120x10 slab (x15), tpacf DR on
+    1024 x 1024 of the 16384^2 pairs (x256); small = half of each part (scale x2).  Returns BE
+    kernels/s = 1 / mean (conv + BE kernel) time."""
     import synth
     from oracle import be as obe, lc as olc
     convs = synth.resnet50_convs(1)
-    t_pairs = []
-    nz, zscale = (10, 64 / 8) if small else (64, 1.0)
     t0 = time.perf_counter()
-    cs = convs[5]
-    x, w, _ = synth.conv_inputs(cs, 1)
-    olc.lc_conv(x, w, cs.stride, cs.pad)
-    tc = (time.perf_counter() - t0) * batch
-    A = synth.stencil_inputs(512, 512, nz, 2022)
-    t0 = time.perf_counter()
-    obe.stencil(A, np.float32(1 / 6), np.float32(1 / 36))
-    t_pairs.append(tc + (time.perf_counter() - t0) * zscale)
-    t0 = time.perf_counter()
-    cs = convs[20]
-    x, w, _ = synth.conv_inputs(cs, 2)
-    olc.lc_conv(x, w, cs.stride, cs.pad)
-    tc = (time.perf_counter() - t0) * batch
-    d = synth.mriq_inputs(64, 1024, 2022)
-    pm, _ = obe.mriq_phimag(d["phiR"], d["phiI"])
-    sub = 256 if small else 4096
-    t0 = time.perf_counter()
-    obe.mriq_q(d["x"][:sub], d["y"][:sub], d["z"][:sub], d["kx"], d["ky"], d["kz"], pm)
-    t_pairs.append(tc + (time.perf_counter() - t0) * (64 ** 3 / sub))
-    per = sum(t_pairs) / len(t_pairs)
-    desc = (f"oracle conv (2 ResNet-50 layers, 1 image, time x{batch}) + 1 stencil 512x512x64 sweep ({'8-plane slab x8' if small else 'full'})"
-            f" + 1 mri-q 1024-k chunk on {sub} of 64^3 voxels (time scaled x{64 ** 3 // sub}); "
-            "BE kernels/s = 1 / mean pair time")
+    for i in (5, 20):
+        cs = convs[i]
+        x, w, _ = synth.conv_inputs(cs, i)
+        olc.lc_conv(x, w, cs.stride, cs.pad)
+    t_conv = (time.perf_counter() - t0) / 2 * batch
+    f = 2 if small else 1
+    times = {}
+
+    def timed(name, fn, scale):
+        t = time.perf_counter()
+        fn()
+        times[name] = (time.perf_counter() - t) * scale
+
+    if be == "table2":
+        d = synth.mriq_inputs(64, 1024, 2022)
+        n = 256 // f
+        pm, _ = obe.mriq_phimag(d["phiR"], d["phiI"])
+        timed("mriq.q", lambda: obe.mriq_q(d["x"][:n], d["y"][:n], d["z"][:n], d["kx"], d["ky"], d["kz"], pm),
+              64 ** 3 / n)
+        dd = synth.mrifhd_inputs(64, 1024, 2022)
+        rr, ri, _, _ = obe.mrifhd_rhophi(dd["phiR"], dd["phiI"], dd["dR"], dd["dI"])
+        timed("mrifhd.fh", lambda: obe.mrifhd_fh(dd["x"][:n], dd["y"][:n], dd["z"][:n], dd["kx"], dd["ky"], dd["kz"],
+                                                 rr, ri), 64 ** 3 / n)
+        xf = synth.fft_inputs(16 // f, 1024, 2022)
+        timed("fft", lambda: obe.fft(xf), 16384 / (16 // f))
+        cu = synth.cutcp_inputs(48.0, 2022)
+        pts = np.random.default_rng(0).integers(0, cu["nx"] ** 3, size=512 // f)
+        timed("cutcp", lambda: obe.cutcp(cu["atoms"], cu["nx"], cu["nx"], cu["nx"], cu["h"], points=pts),
+              cu["nx"] ** 3 / (512 // f))
+        at, z = synth.cp_inputs(4000, 512, 512, 0.1, 2022)
+        m = 32 // f
+        timed("cp", lambda: obe.cp(at, m, m, 0.1, z), 512 * 512 / (m * m))
+        A, B = synth.sgemm_inputs(2048, 2048, 2048, 2022)
+        timed("sgemm", lambda: obe.sgemm(A[:64 // f], B), 2048 / (64 // f))
+        src, fl = synth.lbm_inputs(120, 120, 10 // f, 2022)
+        timed("lbm", lambda: obe.lbm_step(src, fl, src.copy()), 150 / (10 // f))
+        a = synth.tpacf_inputs(1024 // f, 2022)
+        b = synth.tpacf_inputs(1024 // f, 2023, "uniform")
+        e = synth.tpacf_edges()
+        timed("tpacf", lambda: obe.tpacf(a, b, e, False), (16384 / (1024 // f)) ** 2)
+        desc = ("oracle conv (2 ResNet-50 layers, 1 image, time x%d) paired with each Table II BE kernel on a bounded "
+                "part, time scaled to the whole kernel (%s)" % (batch, "; ".join(f"{k} {v:.3g} s" for k, v in times.items())))
+    else:
+        A = synth.stencil_inputs(512, 512, 10 if small else 64, 2022)
+        timed("stencil", lambda: obe.stencil(A, np.float32(1 / 6), np.float32(1 / 36)), 64 / 8 if small else 1.0)
+        d = synth.mriq_inputs(64, 1024, 2022)
+        pm, _ = obe.mriq_phimag(d["phiR"], d["phiI"])
+        n = 256 if small else 4096
+        timed("mriq.q", lambda: obe.mriq_q(d["x"][:n], d["y"][:n], d["z"][:n], d["kx"], d["ky"], d["kz"], pm),
+              64 ** 3 / n)
+        desc = "oracle conv (2 ResNet-50 layers, 1 image, time x%d) + stencil sweep + mri-q chunk, scaled" % batch
+    per = t_conv + sum(times.values()) / len(times)
     return {"value": 1.0 / per, "unit": "BE kernels/s", "cores": _oracle_threads(), "kind": "oracle",
-            "sample": desc, "seconds_per_be_kernel": per}
+            "sample": desc + "; BE kernels/s = 1 / mean (conv + BE kernel) time", "seconds_per_be_kernel": per}
 
 
 def _oracle_threads():
@@ -420,12 +451,12 @@ def run_reference(args, ws, rank):
     """--impl reference: the CPU oracle as it stands is this tier's reference arm."""
     if rank != 0:
         return
-    for _ in range(min(args.warmup, 3)):    # untimed warm-up steps (bounded)
-        cpu_oracle_sample(small=True, batch=args.batch)
+    for _ in range(min(args.warmup, 1)):    # untimed warm-up step (bounded)
+        cpu_oracle_sample(small=True, batch=args.batch, be=args.be)
     t0 = time.perf_counter()
     vals, r = [], None
     for _ in range(args.steps):
-        r = cpu_oracle_sample(small=True, batch=args.batch)
+        r = cpu_oracle_sample(small=True, batch=args.batch, be=args.be)
         vals.append(r["seconds_per_be_kernel"])
         if time.perf_counter() - t0 > 120.0:
             break
@@ -571,7 +602,7 @@ def run_tacker(args, comm):
     if not args.no_extra:
         extra = side_workloads(args, comm, peaks, flush, tk, qos, sv, torch)
 
-    cpu = cpu_oracle_sample(batch=args.batch) if (rank == 0 and ws == 1 and not args.no_cpu) else None
+    cpu = cpu_oracle_sample(batch=args.batch, be=args.be) if (rank == 0 and ws == 1 and not args.no_cpu) else None
     if cpu is not None:
         cpu.pop("seconds_per_be_kernel", None)
 
