@@ -297,7 +297,7 @@ typedef struct {
   int32_t lc_tma_store;      /* 1: TMA-store epilogue (LC-only fp16 plans) */
 } tacker_fused_info_t;
 enum { TACKER_LC_MODE_GEMM = 0, TACKER_LC_MODE_CONV_IM2COL = 1, TACKER_LC_MODE_CONV_TILED = 2,
-       TACKER_LC_MODE_CONV_C8 = 3, TACKER_LC_MODE_CONV_HALO = 4 };
+       TACKER_LC_MODE_CONV_C8 = 3, TACKER_LC_MODE_CONV_HALO = 4, TACKER_LC_MODE_CONV_S2C8 = 5 };
 tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *out);
 /* Model-store keys of the handle's LC kernel, BE kernel and fused pair (for the predictor). */
 tacker_status tacker_fused_keys(tacker_fused_t f, char *lc_key, char *be_key, char *pair_key, size_t buflen);

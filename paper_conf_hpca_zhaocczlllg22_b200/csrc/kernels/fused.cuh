@@ -50,6 +50,21 @@ struct LcParams {
                              // pixels x 64 channels (SW128) and the S taps' weights, and issues S x 4
                              // MMAs whose A descriptors start s rows into the halo (SBO = (8+S-1) rows)
   uint32_t stage_a, stage_bytes;   // shared-memory bytes of a ring stage's A part and of the stage
+  // stride-2 conv with C = 8 (ResNet conv1, 7x7 over 3 channels padded to 8), "phase halo" mode:
+  // M-tile = 16 x 8 output pixels; a stage holds the input halo split into the 4 parity phases
+  // (even/odd rows x even/odd columns, TMA traversal stride 2), each [rows][cols] pixels of 16 B,
+  // so that tap (r, s) of 8 consecutive output columns is 8 consecutive 16-byte rows: an unswizzled
+  // K-major core matrix.  The taps are paired in address order into K = 16 MMAs (start s2_a_off,
+  // second tap s2_a_lbo bytes later); the weights stay resident in shared memory (B region, one
+  // 64-row x 16-byte chunk per tap in the same order, chunk_tap = -1: zero padding).
+  int32_t conv_s2c8;
+  int32_t s2_pairs;                // K = 16 MMAs per tile
+  uint32_t s2_sbo;                 // bytes between output rows inside a phase (cols x 16)
+  uint32_t s2_phase_bytes;         // one phase's TMA box (rows x cols x 16) ...
+  uint32_t s2_phase_stride;        // ... and its slot in the stage (128-aligned)
+  uint32_t b_res_off;              // resident B: offset from the LC base
+  uint16_t s2_a_off[32], s2_a_lbo[32];
+  int16_t s2_chunk_tap[64];
   // split-K: work unit u = (tile u / splits, k-blocks [s kb_per_split, (s+1) kb_per_split) of split
   // s = u % splits).  splits > 1 only when every unit has its own CTA (num_units <= grid): the
   // splits of a tile write fp32 partials, meet on a counter, then each reduces 1/splits of the tile
@@ -113,6 +128,7 @@ struct LcGemm {
     uint64_t *full, *empty, *tfull, *tempty;
     uint32_t *tmem_holder;
     float *bias;             // the current tile's BN bias values (epilogue warps)
+    uint64_t *bres;          // resident weights landed (conv_s2c8)
   };
   static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
     return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
@@ -120,7 +136,7 @@ struct LcGemm {
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages, uint32_t stage_bytes) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * stage_bytes);
     return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4),
-                reinterpret_cast<float *>(b + 2 * stages + 6)};
+                reinterpret_cast<float *>(b + 2 * stages + 6), b + 2 * stages + 5};
   }
 
   static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
@@ -250,7 +266,7 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4)) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -260,6 +276,24 @@ struct LcGemm {
           mbar_arrive_expect_tx(&bb.full[i], L.stage_bytes);
           load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a, kb0 + i, nt);
         }
+      }
+      __syncwarp();
+    }
+    if (L.conv_s2c8) {
+      // resident weights: one 64 x 16-byte chunk per tap (TMA, before the dependency wait: weights
+      // are constant), the padding chunk zeroed here (generic stores, then the async-proxy fence)
+      uint8_t *bres = lc + L.b_res_off;
+      for (int c = 0; c < 2 * L.s2_pairs; ++c)
+        if (L.s2_chunk_tap[c] < 0)
+          for (int i = lane_id(); i < 64; i += 32) reinterpret_cast<uint4 *>(bres + c * 1024)[i] = make_uint4(0, 0, 0, 0);
+      fence_proxy_async();
+      __syncwarp();
+      if (elect_one()) {
+        uint32_t bytes = 0;
+        for (int c = 0; c < 2 * L.s2_pairs; ++c) bytes += L.s2_chunk_tap[c] >= 0 ? 1024u : 0u;
+        mbar_arrive_expect_tx(bb.bres, bytes);
+        for (int c = 0; c < 2 * L.s2_pairs; ++c)
+          if (L.s2_chunk_tap[c] >= 0) tma_load_2d(&P.tmap_b, bb.bres, bres + c * 1024, L.s2_chunk_tap[c] * 8, 0);
       }
       __syncwarp();
     }
@@ -306,6 +340,15 @@ struct LcGemm {
         if (elect_one()) {
           if (L.dbg & 4) {
             mbar_arrive(&bb.full[stage]);
+          } else if (L.conv_s2c8) {
+            // the 4 parity phases of the tile's input window (traversal stride 2, zero padding)
+            const int img = mt / (L.tiles_p * L.tiles_q);
+            const int rem = mt - img * L.tiles_p * L.tiles_q;
+            const int pt = rem / L.tiles_q, qt = rem - pt * L.tiles_q;
+            const int w0 = qt * L.tq * 2 - L.pad, h0 = pt * L.tp * 2 - L.pad;
+            mbar_arrive_expect_tx(&bb.full[stage], 4u * L.s2_phase_bytes);
+            for (int ph = 0; ph < 4; ++ph)
+              tma_load_4d(&P.tmap_a, &bb.full[stage], sa + ph * L.s2_phase_stride, 0, w0 + (ph & 1), h0 + (ph >> 1), img);
           } else if (L.conv_halo) {
             if (!first) {
               mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
@@ -351,6 +394,7 @@ struct LcGemm {
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
     int ui = 0;
+    if (L.conv_s2c8) mbar_wait(bb.bres, 0);   // resident weights landed
     for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1;
       unit_coords(L, u, t, sp, kb0, kb1);
@@ -366,6 +410,13 @@ struct LcGemm {
         if (elect_one()) {
           if (L.dbg & 2) {
             // diagnostics: no MMA
+          } else if (L.conv_s2c8) {
+            // K = 16 per MMA = the tap pair (t0, t1): A core matrices at a_off and a_off + lbo, 8-row
+            // groups (output rows) s2_sbo apart; B = chunks 2u, 2u+1 of the resident weights
+            const uint32_t bres = smem_u32(lc + L.b_res_off);
+            for (int pu = 0; pu < L.s2_pairs; ++pu)
+              umma_f16(d, umma_desc_kmajor_noswz(sa + L.s2_a_off[pu], L.s2_a_lbo[pu], L.s2_sbo),
+                       umma_desc_kmajor_noswz(bres + pu * 2048u, 1024u, 128u), kIdesc, pu != 0);
           } else if (L.conv_halo) {
             // tap s of this filter row: A = the halo from row s, 8-row groups (one output row of 8
             // pixels each) (8 + S - 1) rows apart; B = the tap's BN x 64 weight slot
@@ -455,7 +506,7 @@ struct LcGemm {
     fence_proxy_async();                  // generic-proxy writes visible to the TMA unit
     __syncwarp();
     if (lane == 0) {
-      if (L.conv_halo) tma_store_4d(&P.tmap_d, stg + buf * 4096, n0, at.q0, at.p0, at.img);
+      if (L.conv_halo || L.conv_s2c8) tma_store_4d(&P.tmap_d, stg + buf * 4096, n0, at.q0, at.p0, at.img);
       else tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, at.row0);
       bulk_commit();
     }
@@ -498,7 +549,7 @@ struct LcGemm {
       }
       const bool skip = (L.dbg & 1) != 0;
       BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
-      if (L.conv_halo) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
+      if (L.conv_halo || L.conv_s2c8) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
         at.img = mt / (L.tiles_p * L.tiles_q);
         at.p0 = ((mt / L.tiles_q) % L.tiles_p) * L.tp + 4 * quarter;
         at.q0 = (mt % L.tiles_q) * L.tq;
@@ -724,6 +775,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
         mbar_init(&bb.tfull[a], 1);
         mbar_init(&bb.tempty[a], 4 * 32);
       }
+      mbar_init(bb.bres, 1);
       fence_barrier_init();
     }
     if (warp == 1 && has_lc) tmem_alloc(bb.tmem_holder, P.tmem_cols);

@@ -347,11 +347,56 @@ static bool conv_halo_ok(const LcParams &L, int BN) {
          L.r == L.s && L.s <= 7 && 2 * L.pad == L.s - 1 && L.p >= 8 && L.q >= 8 && BN <= 128;
 }
 
+// Phase-halo mode for stride-2 convs over 8 channels (ResNet-50 conv1: 7x7, 3 channels padded to
+// 8), N <= 64: replaces the explicit im2col + GEMM of §VIII-H.  TACKER_CONV_S2C8=0 disables it.
+static bool conv_s2c8_ok(const LcParams &L, int BN) {
+  static const bool on = [] {
+    const char *e = getenv("TACKER_CONV_S2C8");
+    return !(e && e[0] == '0');
+  }();
+  return on && L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm && L.c == 8 && L.stride == 2 &&
+         L.r * L.s <= 63 && L.N <= 64 && BN == 64;
+}
+
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
   L.stage_a = kBM * kBK * 2;
   L.stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
-  if (conv_halo_ok(L, BN)) {
+  if (conv_s2c8_ok(L, BN)) {
+    L.conv_s2c8 = 1;
+    L.tq = 8;
+    L.tp = kBM / 8;
+    L.tiles_p = (L.p + L.tp - 1) / L.tp;
+    L.tiles_q = (L.q + L.tq - 1) / L.tq;
+    L.tiles_m = L.n * L.tiles_p * L.tiles_q;
+    L.c_blocks = 1;
+    L.num_kb = 1;                                   // one stage = every tap of the tile
+    const int rows = L.tp + (L.r - 1) / 2, cols = L.tq + (L.s - 1) / 2;
+    L.s2_phase_bytes = (uint32_t)rows * cols * 16u;
+    L.s2_phase_stride = (L.s2_phase_bytes + 127u) & ~127u;
+    L.s2_sbo = (uint32_t)cols * 16u;
+    L.stage_a = (4u * L.s2_phase_stride + 1023u) & ~1023u;
+    L.stage_bytes = L.stage_a;
+    // taps in shared-memory address order, paired into K = 16 MMAs (the second of a pair at a
+    // higher address: LBO > 0); an odd tap count ends with a zero-weight chunk reading the
+    // neighbouring (finite) pixel
+    std::vector<std::pair<uint32_t, int>> taps;
+    for (int r = 0; r < L.r; ++r)
+      for (int s = 0; s < L.s; ++s)
+        taps.emplace_back((uint32_t)((r % 2) * 2 + (s % 2)) * L.s2_phase_stride +
+                              (uint32_t)((r / 2) * cols + s / 2) * 16u,
+                          r * L.s + s);
+    std::sort(taps.begin(), taps.end());
+    L.s2_pairs = (int)(taps.size() + 1) / 2;
+    for (int u = 0; u < L.s2_pairs; ++u) {
+      const auto &t0 = taps[2 * u];
+      const bool two = 2 * u + 1 < (int)taps.size();
+      L.s2_a_off[u] = (uint16_t)t0.first;
+      L.s2_a_lbo[u] = (uint16_t)(two ? taps[2 * u + 1].first - t0.first : 16u);
+      L.s2_chunk_tap[2 * u] = (int16_t)t0.second;
+      L.s2_chunk_tap[2 * u + 1] = (int16_t)(two ? taps[2 * u + 1].second : -1);
+    }
+  } else if (conv_halo_ok(L, BN)) {
     L.conv_halo = 1;
     L.tq = 8;
     L.tp = kBM / 8;
@@ -450,6 +495,39 @@ static tacker_status encode_conv_x(CUtensorMap *m, const tacker_lc_desc &d, cons
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv x) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+static tacker_status encode_2d_raw(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                                   uint32_t box_outer, CUtensorMapSwizzle swz) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {inner * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(2d raw) failed: %d", (int)r), TACKER_ECUDA;
+  return TACKER_OK;
+}
+
+// Phase-halo A (conv_s2c8): NHWC as (C = 8, W, H, N), traversal stride 2 in W and H, box 8 channels x
+// 2 cols x 2 rows of the phase (cols x rows pixels of 16 B loaded, unswizzled); out-of-image pixels
+// zero-filled = the padding.
+static tacker_status encode_conv_s2c8(CUtensorMap *m, const tacker_lc_desc &d, const LcParams &L) {
+  auto enc = get_encode();
+  if (!enc) return set_error("cuTensorMapEncodeTiled unavailable"), TACKER_ECUDA;
+  const int rows = L.tp + (L.r - 1) / 2, cols = L.tq + (L.s - 1) / 2;
+  cuuint64_t dims[4] = {8, (cuuint64_t)d.w, (cuuint64_t)d.h, (cuuint64_t)d.n};
+  cuuint64_t strides[3] = {16, (cuuint64_t)d.w * 16, (cuuint64_t)d.w * d.h * 16};
+  cuuint32_t box[4] = {8, (cuuint32_t)(2 * cols), (cuuint32_t)(2 * rows), 1};
+  cuuint32_t es[4] = {1, 2, 2, 1};
+  if (box[1] > 256 || box[2] > 256) return set_error("conv s2c8: TMA box too large"), TACKER_EUNSUPPORTED;
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void *>(d.A), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error("cuTensorMapEncodeTiled(conv s2c8) failed: %d", (int)r), TACKER_ECUDA;
   return TACKER_OK;
 }
 
@@ -666,8 +744,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // stride-1 conv, im2col-mode conv), no residual, no split-K; 4 warps x 2 staging boxes of 4 KB
   L.tma_store = !has_be && tma_store_enabled() && lc->d_dtype == TACKER_F16 &&
                 !(lc->epi_flags & TACKER_EPI_RESIDUAL) && L.splits == 1 && BN >= 64 && L.N >= 64 &&
-                (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col || L.conv_halo);
-  const uint32_t epi_bytes = L.tma_store ? 4u * 2u * 4096u + 1024u : 0u;
+                (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col || L.conv_halo ||
+                 L.conv_s2c8);
+  const uint32_t epi_bytes = (L.tma_store ? 4u * 2u * 4096u + 1024u : 0u) +
+                             (L.conv_s2c8 ? 2u * L.s2_pairs * 1024u + 1024u : 0u);   // + resident weights
   L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
@@ -696,6 +776,10 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.P.tmem_cols = cols;
   F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
   F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + 256u + 4u * 256u + 1023u) & ~1023u : 0u;
+  if (L.conv_s2c8) {
+    const uint32_t after = L.tma_store ? F.P.epi_stage_off + 4u * 2u * 4096u : (uint32_t)stages * stage_bytes + 1280u;
+    L.b_res_off = (after + 1023u) & ~1023u;
+  }
   F.P.be_smem_per_vb = be_slice;
   F.P.be_vb_per_cta = vb;
   F.P.be_blocks = be_blocks;
@@ -715,17 +799,23 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
 
   // TMA tensor maps
   if (lc->kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) {
-    if ((st = L.conv_halo ? encode_conv_halo(&F.P.tmap_a, *lc, L)
-                          : L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc, L.conv_c8 != 0)
-                                          : encode_conv_x(&F.P.tmap_a, *lc, L)))
+    if ((st = L.conv_s2c8 ? encode_conv_s2c8(&F.P.tmap_a, *lc, L)
+              : L.conv_halo ? encode_conv_halo(&F.P.tmap_a, *lc, L)
+                            : L.conv_im2col ? encode_conv_im2col(&F.P.tmap_a, *lc, L.conv_c8 != 0)
+                                            : encode_conv_x(&F.P.tmap_a, *lc, L)))
       return st;
-    if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
+    if (L.conv_s2c8) {   // weights [N][R S 8]: one 16-byte tap chunk x 64 rows per load, unswizzled
+      if ((st = encode_2d_raw(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, 8, 64, CU_TENSOR_MAP_SWIZZLE_NONE)))
+        return st;
+    } else if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) {
+      return st;
+    }
   } else {
     if ((st = encode_2d(&F.P.tmap_a, lc->A, (uint64_t)L.K, (uint64_t)L.M, kBK, kBM))) return st;
     if ((st = encode_2d(&F.P.tmap_b, lc->B, (uint64_t)L.K, (uint64_t)L.N, kBK, BN))) return st;
   }
   if (has_be && (st = encode_be_tmap(*be, &F.P.tmap_be))) return st;
-  if (L.tma_store && L.conv_halo) {
+  if (L.tma_store && (L.conv_halo || L.conv_s2c8)) {
     if ((st = encode_conv_out_4d(&F.P.tmap_d, *lc, L))) return st;
   } else if (L.tma_store && (st = encode_2d(&F.P.tmap_d, lc->D, (uint64_t)L.N, (uint64_t)L.M, 64, 32))) {
     return st;
@@ -1011,6 +1101,7 @@ tacker_status tacker_fused_info(tacker_fused_t f, tacker_fused_info_t *o) {
   const LcParams &L = f->P.lc;
   const bool implicit = L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
   o->lc_mode = !implicit ? TACKER_LC_MODE_GEMM
+               : L.conv_s2c8 ? TACKER_LC_MODE_CONV_S2C8
                : L.conv_halo ? TACKER_LC_MODE_CONV_HALO
                : L.conv_c8 ? TACKER_LC_MODE_CONV_C8
                : L.conv_im2col ? TACKER_LC_MODE_CONV_IM2COL : TACKER_LC_MODE_CONV_TILED;

@@ -54,11 +54,11 @@ def _dev(a, dtype=None):
     return t.cuda()
 
 
-def resnet50_service(batch: int = 1, seed: int = 2022, convs=None, conv1_im2col: bool = True) -> LcService:
-    """conv1 (C = 3 padded to 8): the paper's explicit im2col (an LC CUDA-core kernel, §VIII-H
-    P:3350-3381) + GEMM by default; conv1_im2col=False runs it as one implicit GEMM over 8-tap
-    k-blocks (TMA im2col mode, unswizzled A) -- correct, but measured no faster at b32 (189 us vs
-    130 + 66 us: eight 2 KB TMA loads per k-block)."""
+def resnet50_service(batch: int = 1, seed: int = 2022, convs=None, conv1_im2col: bool = False) -> LcService:
+    """conv1 (C = 3 padded to 8, 7x7 stride 2) runs as one implicit-GEMM tensor-core kernel in the
+    phase-halo mode (TACKER_LC_MODE_CONV_S2C8: the 4 parity phases of the input window per 16 x 8
+    output tile, tap pairs as unswizzled K = 16 MMAs, resident weights); conv1_im2col=True keeps
+    the paper's explicit im2col (an LC CUDA-core kernel, §VIII-H) + GEMM."""
     convs = convs if convs is not None else synth.resnet50_convs(batch)
     ks, bufs, ins, outs = [], [], [], []
     for i, cs in enumerate(convs):

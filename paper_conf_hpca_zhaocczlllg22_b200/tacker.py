@@ -189,7 +189,7 @@ class FusedInfo(C.Structure):
                 ("lc_tma_store", C.c_int32)]
 
 
-LC_MODE_GEMM, LC_MODE_CONV_IM2COL, LC_MODE_CONV_TILED, LC_MODE_CONV_C8, LC_MODE_CONV_HALO = range(5)
+LC_MODE_GEMM, LC_MODE_CONV_IM2COL, LC_MODE_CONV_TILED, LC_MODE_CONV_C8, LC_MODE_CONV_HALO, LC_MODE_CONV_S2C8 = range(6)
 
 
 class LcKernel(C.Structure):

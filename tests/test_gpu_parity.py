@@ -443,3 +443,41 @@ def test_lc_conv_halo_fused_bit_identical(tk):
     f.launch()
     assert torch.equal(o0, o1)
     c["check"]([host(o) for o in c["outs"]])
+
+
+# ------------------------------------------------------------------ LC conv, stride-2 phase halo (conv1)
+S2C8_CASES = [synth.ConvShape("conv1_b2", 2, 224, 224, 8, 64, 7, 7, 2, 3),   # ResNet-50 conv1 (3 ch padded)
+              synth.ConvShape("odd", 3, 30, 27, 8, 64, 7, 7, 2, 3),         # ragged p and q
+              synth.ConvShape("5x5", 2, 33, 41, 8, 48, 5, 5, 2, 2),         # N 48 < 64, 13 tap pairs
+              synth.ConvShape("3x3", 1, 20, 20, 8, 64, 3, 3, 2, 1)]
+
+
+@pytest.mark.parametrize("epi", ["bias_relu", "residual"])
+@pytest.mark.parametrize("cs", S2C8_CASES, ids=lambda c: c.name)
+def test_lc_conv_s2c8_vs_oracle(tk, cs, epi):
+    """conv1 as one implicit GEMM (phase-split halo, tap pairs as unswizzled K = 16 MMAs, resident
+    weights), TMA-store (bias + ReLU) and register (residual) epilogues, vs the oracle."""
+    x, w, b = synth.conv_inputs(cs, seed=7, real_c=3)
+    res = np.random.default_rng(4).uniform(-1, 1, size=(cs.n, cs.p, cs.q, cs.k)).astype(np.float16)
+    out = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    lc = tk.lc_conv(t(x), t(w), out, cs.stride, cs.pad, bias=t(b), relu=True,
+                    residual=t(res) if epi == "residual" else None)
+    assert tk.tacker_fuse(lc, None, 0).info().lc_mode == tk.LC_MODE_CONV_S2C8
+    tk.tacker_launch_original(lc, None)
+    ref, S = olc.lc_conv(x, w, cs.stride, cs.pad, bias=b, relu=True, residual=res if epi == "residual" else None)
+    assert max_rel_err(host(out).astype(np.float64), ref, S) <= 1e-2
+
+
+def test_lc_conv_s2c8_fused_bit_identical(tk):
+    cs = S2C8_CASES[1]
+    x, w, b = synth.conv_inputs(cs, seed=8, real_c=3)
+    o0 = torch.zeros(cs.n, cs.p, cs.q, cs.k, dtype=torch.float16, device=dev())
+    o1 = torch.zeros_like(o0)
+    c = be_case(tk.BE_MRIQ_Q, seed=3)
+    c["reset"]()
+    tk.tacker_launch_original(tk.lc_conv(t(x), t(w), o0, 2, 3, bias=t(b), relu=True), None)
+    f = tk.tacker_fuse(tk.lc_conv(t(x), t(w), o1, 2, 3, bias=t(b), relu=True), c["desc"], 16)
+    assert f.info().lc_mode == tk.LC_MODE_CONV_S2C8
+    f.launch()
+    assert torch.equal(o0, o1)
+    c["check"]([host(o) for o in c["outs"]])
