@@ -98,14 +98,21 @@ def test_managed_runs_keep_lc_outputs_and_qos(tk, variant):
     run.calibrate(reps=3, pair_reps=3)
     run.measure_service(n=20)
     assert run.pairs, "no fusable pair calibrated"
-    # the launch paths under test must run whatever this box measured: pair models with a sure
-    # gain (tau = max(1 + 0.1 r, 0.5 + r), opportune ratio 5/9), no BE kernel blacklisted
+    # the launch paths under test must run whatever this box measured (the NEXT-1 selection may
+    # have kept a BE kernel out of fusion): every >= 10 us BE kernel fused at 16 warps, with a pair
+    # model of sure gain (tau = max(1 + 0.1 r, 0.5 + r), opportune ratio 5/9), none blacklisted
     tk.tacker_model_clear()
     tk.tacker_blacklist_clear()
-    for pk in run.pairs:
-        for r in (0.1, 0.2, 1.8, 1.9):
-            tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0 + 0.1 * r, 0.5 + r))
-        tk.tacker_pair_fit(pk)
+    for a, app in enumerate([st, mq]):
+        for j, bk in enumerate(app.kernels):
+            if run.t_be[(a, j)] < 0.01:
+                continue
+            run.ws_of[(a, j)] = 16
+            for k in svc.kernels:
+                pk = tk.tacker_fuse(k.lc, bk.desc, 16).keys()[2]
+                for r in (0.1, 0.2, 1.8, 1.9):
+                    tk.tacker_pair_add_sample(pk, 1.0, r, max(1.0 + 0.1 * r, 0.5 + r))
+                tk.tacker_pair_fit(pk)
     svc.outputs[-1].zero_()
     res = run.run(tk.POLICY_TACKER, 60, load=0.8, max_inflight=8, **variant)
     brief = {k: res[k] for k in ("fused", "reordered", "idle_be", "be_kernels", "lc_p99_ms", "class_launches")}

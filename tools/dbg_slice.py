@@ -18,6 +18,7 @@ for pk in run.pairs:
     print(pk, tk.tacker_pair_fit(pk))
 res = run.run_window(tk.POLICY_TACKER, 30.0, 5.0, load=0.8, max_inflight=8, trace=True, fuse_older=True, slice_be=True, reorder_rule=2)
 print({k: res[k] for k in ("fused", "reordered", "idle_be", "be_kernels")})
+print("first 40 actions", [(d["action"], d["query"], d["reorder"]) for d in res["trace"][:40]])
 n = 0
 for d in res["trace"]:
     if d["query"] >= 0:
@@ -33,3 +34,11 @@ for k in run.lc_kernels():
             print(ks[2], "blacklisted", tk.tacker_blacklist(ks[1]), "pred", tk.tacker_pair_predict(ks[2], k.t_pred_ms, 0.01) if ks[2] in run.pairs else None)
         except tk.TackerError as e:
             print("fuse err", e)
+m = tk.Manager(tk.POLICY_TACKER, simulate=True, idle_cap_ms=20.0, slice_be=True, reorder_rule=2, fuse_older=True, older_margin_ms=15.0)
+m.trace_enable(100000)
+for ks in run.be_apps():
+    m.submit_be(ks)
+m.submit_lc_batch(run.lc_kernels(), [0.5 + 0.3 * i for i in range(20)])
+m.run(50.0, 7.0)
+tr, _ = m.trace_dicts()
+print("SIM", m.stats().fused_launches, [(d["action"], d["query"], d["reorder"], d["tk_fuse"]) for d in tr[:30]])
