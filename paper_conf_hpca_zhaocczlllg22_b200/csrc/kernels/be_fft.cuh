@@ -45,6 +45,9 @@ template <> struct BeBody<TACKER_BE_FFT> {
   // all 128 threads busy (64 butterflies per transform) and every thread has twice the loads
   // in flight, so a vblock of the fused kernel (fewer resident warps) hides more latency.
   static constexpr int kT = TK_FFT_PER_BLOCK;
+#if TK_FFT_ODD_FIRST
+  static_assert(kMaxN == 1024, "run() dispatches the static plans of n = 2 .. 1024");
+#endif
   static constexpr uint32_t kSmem = kT * kMaxN * 8;
   static __device__ __forceinline__ int pad(int i) { return i ^ ((i >> 4) & 15); }
   static __host__ __device__ int64_t num_blocks(const tacker_be_fft &p) { return (p.batch + kT - 1) / kT; }
@@ -208,9 +211,60 @@ template <> struct BeBody<TACKER_BE_FFT> {
 
   static __device__ __forceinline__ void run(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
                                              uint8_t *smem) {
+#if TK_FFT_ODD_FIRST
+    // one straight-line pass sequence per n (compile-time plan): inside the fused PTB loop the
+    // generic plan (a runtime loop over radix-8 passes and a radix switch, nested in the block loop)
+    // was register-allocated to 2.4 KB of spills per thread at any cap; the static sequences are not
+    switch (p.n) {
+      case 2: run_static<1>(p, vb, tid, bar, smem); return;
+      case 4: run_static<2>(p, vb, tid, bar, smem); return;
+      case 8: run_static<3>(p, vb, tid, bar, smem); return;
+      case 16: run_static<4>(p, vb, tid, bar, smem); return;
+      case 32: run_static<5>(p, vb, tid, bar, smem); return;
+      case 64: run_static<6>(p, vb, tid, bar, smem); return;
+      case 128: run_static<7>(p, vb, tid, bar, smem); return;
+      case 256: run_static<8>(p, vb, tid, bar, smem); return;
+      case 512: run_static<9>(p, vb, tid, bar, smem); return;
+      default: run_static<10>(p, vb, tid, bar, smem); return;   // 1024 (validated on the host)
+    }
+#else
     if (p.n <= 512) run_n<(kMaxN < 512 ? kMaxN : 512)>(p, vb, tid, bar, smem);
     else if (p.n <= 1024) run_n<(kMaxN < 1024 ? kMaxN : 1024)>(p, vb, tid, bar, smem);
     else run_n<kMaxN>(p, vb, tid, bar, smem);
+#endif
+  }
+  // The same plan as run_n (radix-2^f pass first, then p8 radix-8 passes) with n = 2^L fixed at
+  // compile time: identical butterflies in identical order, so identical results.
+  template <int L>
+  static __device__ __forceinline__ void run_static(const tacker_be_fft &p, int64_t vb, int tid, uint32_t bar,
+                                                    uint8_t *smem) {
+    constexpr int N = 1 << L;
+    constexpr int P8 = L <= 4 ? 0 : L % 3 == 0 ? L / 3 - 1 : L % 3 == 1 ? (L - 4) / 3 : (L - 2) / 3;
+    constexpr int F = L <= 4 ? L : L % 3 == 0 ? 3 : L % 3 == 1 ? 4 : 2;
+    constexpr int R0 = 1 << F;
+    float2 *s = reinterpret_cast<float2 *>(smem);
+    const float2 *tw = reinterpret_cast<const float2 *>(p.twiddle);
+    const int nt = p.batch - vb * kT < kT ? (int)(p.batch - vb * kT) : kT;
+    const float2 *gx = reinterpret_cast<const float2 *>(p.x) + vb * kT * N;
+    float2 *gy = reinterpret_cast<float2 *>(p.y) + vb * kT * N;
+    named_bar_sync(bar, kVbThreads);        // the previous transform of this slot is done with s
+    if constexpr (P8 == 0) {
+      pass<R0, N, true, true>(s, gx, gy, tw, N, nt, 1, tid, bar);
+    } else {
+      pass<R0, N, true, false>(s, gx, gy, tw, N, nt, 1, tid, bar);
+      radix8_passes<N, P8 - 1>(s, gx, gy, tw, nt, R0, tid, bar);
+    }
+  }
+  // M middle radix-8 passes from sub-transform size Ns, then the last one (writes global memory)
+  template <int N, int M>
+  static __device__ __forceinline__ void radix8_passes(float2 *s, const float2 *gx, float2 *gy, const float2 *tw,
+                                                       int nt, int Ns, int tid, uint32_t bar) {
+    if constexpr (M == 0) {
+      pass<8, N, false, true>(s, gx, gy, tw, N, nt, Ns, tid, bar);
+    } else {
+      pass<8, N, false, false>(s, gx, gy, tw, N, nt, Ns, tid, bar);
+      radix8_passes<N, M - 1>(s, gx, gy, tw, nt, Ns * 8, tid, bar);
+    }
   }
   // Pass plan for n = 2^L: one radix-2^f pass (f in {1, 2, 3, 4}) and p8 radix-8 passes, the
   // radix-2^f one first (TK_FFT_ODD_FIRST) or last; n = 1024: 16, 8, 8 — two shared-memory

@@ -708,16 +708,22 @@ __device__ __noinline__ void be_run_coarse_outlined(const tacker_be_desc &d, int
                                                     uint8_t *smem, const CUtensorMap *tm) {
   be_run_coarse<KIND>(d, vb, nb, tid, bar, smem, tm);
 }
-template <int KIND>
+// SPEC: a compile-time specialisation of the body chosen once per launch outside the PTB loop
+// (fft: SPEC = log2 n, the static pass plan; 0 = the generic body).  ptxas allocates registers
+// for the loop as a whole: with the generic fft (a runtime pass loop and radix switch) inside the
+// block loop it spilled 2.4 KB per thread; one static plan per loop copy does not.
+template <int KIND, int SPEC>
 __device__ __forceinline__ void be_fused_body(const tacker_be_desc &d, int64_t vb, int nb, int tid, uint32_t bar,
                                               uint8_t *smem, const CUtensorMap *tm) {
-  if constexpr (KIND == TACKER_BE_FFT && TK_FFT_OUTLINED)
+  if constexpr (KIND == TACKER_BE_FFT && SPEC > 0)
+    BeBody<TACKER_BE_FFT>::run_static<SPEC>(BeSel<TACKER_BE_FFT>::get(d), vb, tid, bar, smem);
+  else if constexpr (KIND == TACKER_BE_FFT && TK_FFT_OUTLINED)
     be_run_coarse_outlined<KIND>(d, vb, nb, tid, bar, smem, tm);
   else
     be_run_coarse<KIND>(d, vb, nb, tid, bar, smem, tm);
 }
-template <int BE_KIND>
-__device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_smem) {
+template <int BE_KIND, int SPEC>
+__device__ __forceinline__ void be_ptb_loop_impl(const FusedParams &P, uint8_t *be_smem) {
   const int j = warp_id() >> 2;                     // virtual block slot in this CTA
   const int tid = (int)(threadIdx.x & (kVbThreads - 1));   // thread_step rebase (Fig. 5): threadIdx.x - 128 j, bounded for the compiler
   const uint32_t bar = 1 + j;                       // named barrier id (0 is reserved)
@@ -742,14 +748,14 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
     const int64_t lo = P.be_blocks * cta / gridDim.x, hi = P.be_blocks * (cta + 1) / gridDim.x;
     const int S = P.be_vb_per_cta;
     for (int64_t b = lo + (hi - lo) * j / S, e = lo + (hi - lo) * (j + 1) / S; b < e; b += kC)
-      be_fused_body<BE_KIND>(P.be, P.be_offset + b, (int)min((int64_t)kC, e - b), tid, bar, body_smem, &P.tmap_be);
+      be_fused_body<BE_KIND, SPEC>(P.be, P.be_offset + b, (int)min((int64_t)kC, e - b), tid, bar, body_smem, &P.tmap_be);
     return;
   }
   const int64_t units = (P.be_blocks + kC - 1) / kC;
   int64_t vb = (int64_t)j * gridDim.x + cta;
   while (vb < units) {
     const int64_t b0 = vb * kC;
-    be_fused_body<BE_KIND>(P.be, P.be_offset + b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem,
+    be_fused_body<BE_KIND, SPEC>(P.be, P.be_offset + b0, (int)min((int64_t)kC, P.be_blocks - b0), tid, bar, body_smem,
                            &P.tmap_be);
     if (tid == 0) *s_ticket = groups + atomicAdd(&P.work->ticket, 1u);
     named_bar_sync(bar, kVbThreads);
@@ -766,9 +772,34 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
   }
 }
 
+template <int BE_KIND>
+__device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_smem) {
+  if constexpr (BE_KIND == TACKER_BE_FFT && TK_FFT_ODD_FIRST) {
+    switch (P.be.p.fft.n) {   // one loop copy per length (n = 2 .. 1024, validated on the host)
+      case 2: be_ptb_loop_impl<BE_KIND, 1>(P, be_smem); return;
+      case 4: be_ptb_loop_impl<BE_KIND, 2>(P, be_smem); return;
+      case 8: be_ptb_loop_impl<BE_KIND, 3>(P, be_smem); return;
+      case 16: be_ptb_loop_impl<BE_KIND, 4>(P, be_smem); return;
+      case 32: be_ptb_loop_impl<BE_KIND, 5>(P, be_smem); return;
+      case 64: be_ptb_loop_impl<BE_KIND, 6>(P, be_smem); return;
+      case 128: be_ptb_loop_impl<BE_KIND, 7>(P, be_smem); return;
+      case 256: be_ptb_loop_impl<BE_KIND, 8>(P, be_smem); return;
+      case 512: be_ptb_loop_impl<BE_KIND, 9>(P, be_smem); return;
+      default: be_ptb_loop_impl<BE_KIND, 10>(P, be_smem); return;
+    }
+  } else {
+    be_ptb_loop_impl<BE_KIND, 0>(P, be_smem);
+  }
+}
+
 // ------------------------------------------------------------------------ the fused kernel
-template <int BN, int BE_KIND>
-__global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
+// WMAX: the largest BE warp split this instantiation launches with.  The launch bound, and with
+// it the per-thread register cap, follows the CTA's warp count: the default class (WMAX =
+// be_max_warps) holds 6 + 24 warps at 64 registers; the register-rich class (WMAX = 8, 6 + 8
+// warps) gives every warp up to 144, for bodies that spill at 64 (fft) and for wider LC
+// epilogue batches.  tacker_fuse picks the smallest class that holds the plan's warp split.
+template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND)>
+__global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();   // the next kernel on the stream may start its prologue
@@ -815,7 +846,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + be_max_warps(BE_KIND)), 1)
       } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
         LcGemm<BN>::epilogue_tma(P, bb, tmem, lc);
       } else {
-        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : 16>(P, bb, tmem);
+        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
       }
     }
   } else if constexpr (BE_KIND != TACKER_BE_NONE) {

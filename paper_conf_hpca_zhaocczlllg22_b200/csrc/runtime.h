@@ -15,6 +15,9 @@ bool model_predict(const std::string &key, double x, double *y);
 bool pair_predict(const std::string &key, double x_tc, double x_cd, double *y);
 bool pair_opportune(const std::string &key, double *r);
 
+// register-rich fused instantiations (fused_rich.cu): fused_kernel<BN, kind, 8> or nullptr
+void *pick_fused_rich(int BN, int be_kind);
+
 // kind names
 const char *be_kind_name(int kind);
 

@@ -627,6 +627,14 @@ static KernelFn fused_fn(int be_kind) {
     default: return nullptr;
   }
 }
+// TACKER_RICH=0 disables the register-rich class (A/B measurements)
+static bool rich_class_enabled() {
+  static const bool on = [] {
+    const char *e = getenv("TACKER_RICH");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
 static KernelFn pick_fused(int BN, int be_kind) {
   if (BN == 64) return fused_fn<64>(be_kind);
   if (BN == 128) return fused_fn<128>(be_kind);
@@ -794,7 +802,11 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   if (!has_be && F.smem < kMinLcSmem) F.smem = kMinLcSmem;
   F.grid = has_be ? sms : (L.num_units < sms ? L.num_units : sms);
   if (F.grid < 1) F.grid = 1;
-  F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
+  // register class: plans with at most 8 BE warps take the register-rich instantiation (up to
+  // 128 registers per thread) where one is compiled; wider plans the default class (64)
+  F.fn = nullptr;
+  if (has_be && warp_split <= 8 && rich_class_enabled()) F.fn = reinterpret_cast<KernelFn>(pick_fused_rich(BN, be->kind));
+  if (!F.fn) F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
   if (!F.fn) return set_error("no kernel instantiation for BN=%d BE=%d", BN, has_be ? be->kind : 0), TACKER_EUNSUPPORTED;
 
   // TMA tensor maps

@@ -94,6 +94,25 @@ def test_fft_lengths_vs_oracle(tk, size):
     c["check"]([host(o) for o in c["outs"]])
 
 
+@pytest.mark.parametrize("size", ["small", "odd", "mid", "tiny", "single16", "single8", "two"])
+@pytest.mark.parametrize("ws", [8, 24])
+def test_fft_lengths_fused_bit_identical(tk, size, ws):
+    # the fused fft runs one static pass plan per length in its own PTB loop copy (fused.cuh
+    # be_ptb_loop): every length, in the register-rich (ws 8) and the default (ws 24) class
+    c = be_case(tk.BE_FFT, seed=4, size=size)
+    c["reset"]()
+    tk.tacker_launch_original(None, c["desc"])
+    orig = [host(o).copy() for o in c["outs"]]
+    c["check"](orig)
+    A, B = synth.lc_gemm_inputs(256, 128, 128, seed=1)
+    D = torch.zeros(256, 128, device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), c["desc"], ws)
+    c["reset"]()
+    f.launch()
+    for a, o in zip(orig, c["outs"]):
+        assert a.tobytes() == host(o).tobytes()
+
+
 @pytest.mark.parametrize("variant", ["impulse", "tone"])
 def test_fft_closed_form_inputs(tk, variant):
     # impulse -> pure twiddle rows, tone -> n at one bin: vs the oracle's DFT of the same fp32 input
@@ -148,8 +167,12 @@ FUSE_KINDS = ["BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_LBM", "BE_SPMV_JDS", "B
               "BE_MRIFHD_RHOPHI", "BE_MRIFHD_FH", "BE_CP", "BE_FFT", "BE_TPACF"]
 
 
+RICH_KINDS = {"BE_SGEMM", "BE_STENCIL", "BE_MRIQ_Q", "BE_MRIFHD_FH", "BE_CUTCP", "BE_CP", "BE_LBM", "BE_FFT", "BE_TPACF",
+              "BE_SPMV_JDS"}
+
+
 @pytest.mark.parametrize("kind", FUSE_KINDS)
-@pytest.mark.parametrize("ws", [4, 16])
+@pytest.mark.parametrize("ws", [4, 8, 16])
 def test_fused_bit_identical_to_original(tk, kind, ws):
     M, N, K = 256, 256, 256
     A, B = synth.lc_gemm_inputs(M, N, K, seed=1)
@@ -164,6 +187,8 @@ def test_fused_bit_identical_to_original(tk, kind, ws):
     c["check"](orig)
     # fused launch, twice (the BE ticket must self-reset)
     f = tk.tacker_fuse(tk.lc_gemm(dA, dB, D1), c["desc"], ws)
+    if ws <= 8 and kind in RICH_KINDS:   # register-rich class (fused_rich.cu): above the 64 cap
+        assert f.info().regs_per_thread > 64
     for _ in range(2):
         c["reset"]()
         D1.zero_()

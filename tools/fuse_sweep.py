@@ -37,8 +37,9 @@ def main():
     ap.add_argument("--convs", default="0,5,20,40,52")
     ap.add_argument("--ws", default="8,16,24")
     ap.add_argument("--be", default="stencil,mriq")
+    ap.add_argument("--batch", type=int, default=1, help="ResNet-50 batch of the LC convs")
     args = ap.parse_args()
-    svc = sv.resnet50_service(1)
+    svc = sv.resnet50_service(args.batch)
     tcs = [k for k in svc.kernels if k.is_tc]
     bes = {}
     for b in args.be.split(","):
@@ -52,6 +53,12 @@ def main():
         elif b == "sgemm":
             app = sv.sgemm_app(2048, 2048, 2048)
             bes[b] = (app, app.kernels[0].desc)
+        elif b in ("fft", "lbm", "cp", "mrifhd", "tpacf"):
+            app = {"fft": sv.fft_app, "lbm": sv.lbm_app, "cp": sv.cp_app, "mrifhd": sv.mrifhd_app,
+                   "tpacf": sv.tpacf_app}[b]()
+            sv.prime_apps([app])
+            k0 = next(k for k in app.kernels if k.name not in ("mrifhd.rhophi",))
+            bes[b] = (app, k0.desc)
     for ci in [int(c) for c in args.convs.split(",")]:
         k = tcs[ci]
         t_lc = timeit(lambda: tk.tacker_launch_original(k.lc, None))
@@ -64,7 +71,7 @@ def main():
                     print(json.dumps({"conv": ci, "be": name, "ws": ws, "err": str(e)}))
                     continue
                 t_f = timeit(f.launch)
-                print(json.dumps({"conv": ci, "shape": k.name, "be": name, "ws": ws, "lc_us": round(t_lc, 2),
+                print(json.dumps({"conv": ci, "shape": k.name, "be": name, "ws": ws, "regs": f.info().regs_per_thread, "lc_us": round(t_lc, 2),
                                   "be_us": round(t_be, 2), "fused_us": round(t_f, 2),
                                   "seq_us": round(t_lc + t_be, 2), "ideal_us": round(max(t_lc, t_be), 2),
                                   "frac_of_ideal": round(max(t_lc, t_be) / t_f, 3),
