@@ -21,7 +21,12 @@
  *   Streams    tacker_stream_t is a cudaStream_t (NULL = legacy default stream).  Launches are
  *              asynchronous on that stream; predictor calls never touch the GPU.
  *   Threads    Fused handles are immutable after tacker_fuse() and may be launched from any
- *              thread.  A manager is single-threaded.  The model store is mutex-protected.
+ *              thread, but a handle owns device workspaces (the BE ticket counters, split-K
+ *              partials and counters) that reset themselves at the end of each launch: at most
+ *              one launch of a handle may be in flight at a time (launch it on one stream; fuse
+ *              a second handle for concurrent streams).  tacker_launch_original's internal LC
+ *              plans follow the same rule per LC descriptor.  A manager is single-threaded.
+ *              The model store is mutex-protected.
  */
 #ifndef TACKER_H
 #define TACKER_H
@@ -347,6 +352,11 @@ tacker_status tacker_blacklist_clear(void);
 /* Diagnostics: copies the LC role clock64 stamps recorded by plans built with TACKER_LC_DBG bit 3
  * ([160 CTAs][5 events][16 work units], see fused.cuh) into out (>= 12800 slots). */
 tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n);
+/* Diagnostics: synchronises the device, copies the per-launch %globaltimer stamps (ns) recorded by
+ * plans built with TACKER_LC_DBG bit 4 (value 16) into out ([256 launch slots][8], >= 2048 slots;
+ * slot layout in fused.cuh g_lc_gt), clears them and the slot counter; *next_slot (nullable) = the
+ * number of launches recorded since the last call (mod 256). */
+tacker_status tacker_debug_lc_globaltimer(uint64_t *out, int64_t n, int32_t *next_slot);
 
 /* One fused launch of handle f whose BE part runs only the PTB slice [block_offset,
  * block_offset + n_blocks) of the handle's BE kernel (the LC part is unchanged; n_blocks 0 = no

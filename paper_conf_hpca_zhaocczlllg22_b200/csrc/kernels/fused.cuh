@@ -21,7 +21,8 @@
 
 namespace tk {
 
-constexpr int kLcWarps = 6;
+constexpr int kLcWarps = 6;        // fused CTAs: producer, MMA, 4 epilogue warps
+constexpr int kLcWarpsSolo = 10;   // LC-only CTAs: producer, MMA, 2 epilogue groups of 4 warps
 constexpr int kBM = 128;   // UMMA M
 constexpr int kBK = 64;    // one 128-byte swizzle row of fp16
 constexpr int kUK = 16;    // UMMA K for kind::f16
@@ -50,6 +51,10 @@ struct LcParams {
                              // pixels x 64 channels (SW128) and the S taps' weights, and issues S x 4
                              // MMAs whose A descriptors start s rows into the halo (SBO = (8+S-1) rows)
   uint32_t stage_a, stage_bytes;   // shared-memory bytes of a ring stage's A part and of the stage
+  // k-blocks per ring stage (plain GEMM / 1x1 / im2col modes; 1 elsewhere): a stage holds kps A
+  // k-blocks then kps B k-blocks and one full/empty handshake covers 4 kps MMAs -- the handshake
+  // (~370 cycles) otherwise bounds N <= 128 mainloops (4 MMAs of 32-64 cycles per k-block)
+  int32_t kps;
   // stride-2 conv with C = 8 (ResNet conv1, 7x7 over 3 channels padded to 8), "phase halo" mode:
   // M-tile = 16 x 8 output pixels; a stage holds the input halo split into the 4 parity phases
   // (even/odd rows x even/odd columns, TMA traversal stride 2), each [rows][cols] pixels of 16 B,
@@ -74,10 +79,16 @@ struct LcParams {
   // warp stages its 32 rows x 64 columns (SW128) in shared memory and one lane stores the box
   // through tmap_d -- full-line global writes instead of 16-byte row-strided stores
   int32_t tma_store;
+  // resident bias: the whole bias vector (tiles_n x BN floats, zero past N) is loaded into shared
+  // memory at bias_off (from the LC base) once per CTA, before the dependency wait (it is a
+  // constant), instead of staging one tile's BN values per tile (a global load and two epilogue
+  // barriers on every tile's critical path); 0 = per-tile staging
+  uint32_t bias_off;
   // diagnostics (TACKER_LC_DBG, never set in production): bit 0 = epilogue drains TMEM without
   // math or stores; bit 1 = no MMAs (the issuer only releases stages and signals the epilogue);
   // bit 2 = no TMA loads (the producer arrives on the full barriers without data)
   int32_t dbg;
+  int32_t dbg_id;          // launch slot of the bit-4 (16) global-time stamps
   float *part;             // [num_tiles * splits][kBM][BN] fp32 partial tiles
   uint32_t *cnt;           // [2 * num_tiles]: arrivals, finished reductions (self-resetting)
 };
@@ -98,13 +109,14 @@ struct alignas(64) FusedParams {
   int64_t be_offset;       // first original block (a slice [be_offset, be_offset + be_blocks))
   BeWork *work;            // device workspace for the BE ticket
   int32_t be_vb_per_cta;   // virtual blocks per CTA
-  int32_t lc_warps;        // 6 or 0
+  int32_t lc_warps;        // 6 (one epilogue group), 10 (LC-only: two groups, one per TMEM accumulator stage) or 0
   int32_t stages;          // SMEM ring depth
   int32_t acc_stages;      // TMEM accumulator buffers
   uint32_t tmem_cols;
   uint32_t lc_smem_bytes;  // ring + barriers, 1024-aligned start
   uint32_t be_smem_per_vb; // per-vblock slice (incl. 16 B ticket slot)
-  uint32_t epi_stage_off;  // TMA-store staging (4 warps x 2 x 4 KB, 1024-aligned) from the LC base
+  uint32_t epi_stage_off;  // TMA-store staging (4 warps x epi_bufs x 4 KB, 1024-aligned) from the LC base
+  int32_t epi_bufs;        // staging boxes per epilogue warp (2 or 4): stores in flight per warp
 };
 
 // diagnostics (TACKER_LC_DBG bit 3): per-CTA clock64 stamps of the first 16 work units of each LC
@@ -114,6 +126,28 @@ struct alignas(64) FusedParams {
 __device__ unsigned long long g_lc_ts[160][5][16];
 __device__ __forceinline__ void lc_stamp(const LcParams &L, int ev, int i) {
   if ((L.dbg & 8) && i < 16 && blockIdx.x < 160) g_lc_ts[blockIdx.x][ev][i] = clock64();
+}
+
+// diagnostics (TACKER_LC_DBG bit 4 = 16): per-launch %globaltimer stamps (ns, comparable across
+// SMs and launches) of the kernel-boundary cost, slot = dbg_id: [0] CTA 0 entry, [1] CTA 0 prologue
+// done, [2] CTA 0 producer's dependency wait returned, [3] CTA 0 first ring stage landed (MMA
+// warp), [4] ~(earliest CTA entry), [5] latest epilogue end, [6] latest CTA exit; read and cleared
+// by tacker_debug_lc_globaltimer
+__device__ unsigned long long g_lc_gt[256][8];
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void lc_gt(const LcParams &L, int slot, bool cta0_only) {
+  if (!(L.dbg & 16)) return;
+  const unsigned long long t = gtime();
+  unsigned long long *g = &g_lc_gt[L.dbg_id & 255][slot];
+  if (cta0_only) {
+    if (blockIdx.x == 0) *g = t;
+  } else {
+    atomicMax(g, slot == 4 ? ~t : t);
+  }
 }
 
 // ------------------------------------------------------------------------ LC roles
@@ -139,6 +173,16 @@ struct LcGemm {
                 reinterpret_cast<float *>(b + 2 * stages + 6), b + 2 * stages + 5};
   }
 
+  // resident bias (L.bias_off != 0): the 128 epilogue threads copy tiles_n x BN bias values
+  // (zero past N) into shared memory once; returns the shared base
+  // (each epilogue group writes the same values and meets on its own barrier `ebar`)
+  static __device__ __forceinline__ float *load_bias_resident(const LcParams &L, uint8_t *lc, uint32_t ebar) {
+    float *b = reinterpret_cast<float *>(lc + L.bias_off);
+    const int et = (int)threadIdx.x % 128;
+    for (int c = et; c < L.tiles_n * BN; c += 128) b[c] = c < L.N ? __ldg(L.bias + c) : 0.f;
+    named_bar_sync(ebar, 128);
+    return b;
+  }
   static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
     // N-tiles fastest: consecutive CTAs share the A rows (L2 reuse of the activation tile)
     mt = t / L.tiles_n;
@@ -270,11 +314,15 @@ struct LcGemm {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
-      pre = min(P.stages, kb1 - kb0);
+      const int kps = L.kps, steps = (kb1 - kb0 + kps - 1) / kps;
+      const uint32_t kb_bytes = L.stage_bytes / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
+      pre = min(P.stages, steps);
       if (elect_one()) {
         for (int i = 0; i < pre; ++i) {
-          mbar_arrive_expect_tx(&bb.full[i], L.stage_bytes);
-          load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a, kb0 + i, nt);
+          const int n = min(kps, kb1 - kb0 - i * kps);
+          mbar_arrive_expect_tx(&bb.full[i], n * kb_bytes);
+          for (int j = 0; j < n; ++j)
+            load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a + j * b_bytes, kb0 + i * kps + j, nt);
         }
       }
       __syncwarp();
@@ -298,6 +346,8 @@ struct LcGemm {
       __syncwarp();
     }
     griddep_wait();
+    if (elect_one()) lc_gt(L, 2, true);
+    __syncwarp();
     int stage = 0;
     uint32_t phase = 0;
     int ui = 0;
@@ -331,9 +381,12 @@ struct LcGemm {
         rr = rs / L.s;
         ss = rs - rr * L.s;
       }
-      for (int kb = kb0; kb < kb1; ++kb) {
+      const int kps = L.kps;
+      const uint32_t a_bytes = L.stage_a / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
+      for (int kb = kb0; kb < kb1; kb += kps) {
         uint8_t *sa = lc + stage * L.stage_bytes;
         uint8_t *sb = sa + L.stage_a;
+        const int n = min(kps, kb1 - kb);   // k-blocks in this stage
         const bool first = pre > 0;   // first tile, stage == kb: B already in flight, its bytes expected
         if (first) --pre;
         else mbar_wait(&bb.empty[stage], phase ^ 1);
@@ -358,28 +411,43 @@ struct LcGemm {
             tma_load_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc + rr, n0);
           } else if (walk) {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
-              tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);   // K index rs*C + cb*64 = 64 kb
+              mbar_arrive_expect_tx(&bb.full[stage], n * (a_bytes + b_bytes));
+              for (int j = 0; j < n; ++j)   // K index rs*C + cb*64 = 64 kb
+                tma_load_2d(&P.tmap_b, &bb.full[stage], sb + j * b_bytes, (kb + j) * kBK, nt * BN);
             }
-            tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc, n0, (uint16_t)ss, (uint16_t)rr);
+            int c2 = cb, s2 = ss, r2 = rr;
+            for (int j = 0; j < n; ++j) {
+              tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa + j * a_bytes, c2 * kBK, wc, hc, n0, (uint16_t)s2,
+                                 (uint16_t)r2);
+              if (++c2 == L.c_blocks) {
+                c2 = 0;
+                if (++s2 == L.s) {
+                  s2 = 0;
+                  ++r2;
+                }
+              }
+            }
           } else {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
-              load_b(P, &bb.full[stage], sb, kb, nt);
+              mbar_arrive_expect_tx(&bb.full[stage], n * (a_bytes + b_bytes));
+              for (int j = 0; j < n; ++j) load_b(P, &bb.full[stage], sb + j * b_bytes, kb + j, nt);
             }
-            load_a(P, &bb.full[stage], sa, kb, mt);
+            for (int j = 0; j < n; ++j) load_a(P, &bb.full[stage], sa + j * a_bytes, kb + j, mt);
           }
         }
         __syncwarp();
         if (L.conv_halo && ++cb == L.c_blocks) {
           cb = 0;
           ++rr;
-        } else if (walk && ++cb == L.c_blocks) {
-          cb = 0;
-          if (++ss == L.s) {
-            ss = 0;
-            ++rr;
-          }
+        } else if (walk) {
+          for (int j = 0; j < n; ++j)
+            if (++cb == L.c_blocks) {
+              cb = 0;
+              if (++ss == L.s) {
+                ss = 0;
+                ++rr;
+              }
+            }
         }
         if (++stage == P.stages) {
           stage = 0;
@@ -402,9 +470,13 @@ struct LcGemm {
       tc_fence_after();
       lc_stamp(L, 1, ui);
       const uint32_t d = tmem + acc * BN;
-      for (int kb = kb0; kb < kb1; ++kb) {
+      const int kps = L.kps;
+      const uint32_t a_bytes = L.stage_a / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
+      for (int kb = kb0; kb < kb1; kb += kps) {
+        const int n = min(kps, kb1 - kb);
         mbar_wait(&bb.full[stage], phase);
         tc_fence_after();
+        if (ui == 0 && kb == kb0 && lane_id() == 0) lc_gt(L, 3, true);
         const uint32_t sa = smem_u32(lc + stage * L.stage_bytes);
         const uint32_t sb = sa + L.stage_a;
         if (elect_one()) {
@@ -434,10 +506,12 @@ struct LcGemm {
               umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
                        umma_desc_sw128(sb + k * kUK * 2), kIdesc, (kb != kb0 || k != 0));
           } else {
-            const uint64_t da = umma_desc_sw128(sa), db = umma_desc_sw128(sb);
+            for (int j = 0; j < n; ++j) {
+              const uint64_t da = umma_desc_sw128(sa + j * a_bytes), db = umma_desc_sw128(sb + j * b_bytes);
 #pragma unroll
-            for (int k = 0; k < kBK / kUK; ++k)   // K step of 16 fp16 = 32 B = +2 in the start-address field
-              umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || k != 0));
+              for (int k = 0; k < kBK / kUK; ++k)   // K step of 16 fp16 = 32 B = +2 in the start-address field
+                umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || j != 0 || k != 0));
+            }
           }
           umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
         }
@@ -472,31 +546,28 @@ struct LcGemm {
     int row0;              // 2-D: first GEMM row
     int q0, p0, img;       // 4-D
   };
+  template <bool BIAS, bool RELU>
   static __device__ __forceinline__ void epi_batch(const FusedParams &P, const uint32_t (&v)[64], uint32_t bias_s,
-                                                   bool bias, uint8_t *stg, int &buf, int n0, BoxAt at, int lane) {
+                                                   uint8_t *stg, int &buf, int n0, BoxAt at, int lane) {
     const LcParams &L = P.lc;
-    float b[64];
-    if (bias) {
-#pragma unroll
-      for (int i = 0; i < 16; ++i) {
-        const float4 q = ld_shared_v4f(bias_s + 16 * i);
-        b[4 * i] = q.x;
-        b[4 * i + 1] = q.y;
-        b[4 * i + 2] = q.z;
-        b[4 * i + 3] = q.w;
-      }
+    if (lane == 0) {   // this box's previous store has read it
+      if (P.epi_bufs == 4) bulk_wait_read<3>();
+      else bulk_wait_read<1>();
     }
-    if (lane == 0) bulk_wait_read<1>();   // this box's previous store has read it
     __syncwarp();
     const uint32_t box = smem_u32(stg + buf * 4096) + lane * 128;
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
-      float f[8];
+      float f[8], b[8];
+      if (BIAS) {   // 8 bias values per group of 8 columns (broadcast LDS.128; 64 held at once spilled)
+        const float4 q0 = ld_shared_v4f(bias_s + 32 * j), q1 = ld_shared_v4f(bias_s + 32 * j + 16);
+        b[0] = q0.x, b[1] = q0.y, b[2] = q0.z, b[3] = q0.w, b[4] = q1.x, b[5] = q1.y, b[6] = q1.z, b[7] = q1.w;
+      }
 #pragma unroll
       for (int e = 0; e < 8; ++e) {
         f[e] = __uint_as_float(v[8 * j + e]);
-        if (bias) f[e] = __fadd_rn(f[e], b[8 * j + e]);
-        if (L.epi & TACKER_EPI_RELU) f[e] = fmaxf(f[e], 0.f);
+        if (BIAS) f[e] = __fadd_rn(f[e], b[e]);
+        if (RELU) f[e] = fmaxf(f[e], 0.f);
       }
       __align__(16) __half2 hv[4];
 #pragma unroll
@@ -510,7 +581,7 @@ struct LcGemm {
       else tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, at.row0);
       bulk_commit();
     }
-    buf ^= 1;
+    buf = buf + 1 == P.epi_bufs ? 0 : buf + 1;
   }
   static __device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
     tmem_ld_32x32b_x16(taddr, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
@@ -518,34 +589,56 @@ struct LcGemm {
     tmem_ld_32x32b_x16(taddr + 32, *reinterpret_cast<uint32_t(*)[16]>(&v[32]));
     tmem_ld_32x32b_x16(taddr + 48, *reinterpret_cast<uint32_t(*)[16]>(&v[48]));
   }
+  // Epilogue groups (LC-only plans): group g of ng drains the work units u = cta + (g + i ng) grid,
+  // i.e. with two groups and two TMEM accumulator stages group g owns stage g -- two tiles'
+  // epilogues run at once (one group's TMEM drain / conversion / store issue was the bound of the
+  // short-K convs); `ew` = the warp's index among all epilogue warps (its staging boxes)
   static __device__ __forceinline__ void epilogue_tma(const FusedParams &P, const Bars &bb, uint32_t tmem,
-                                                      uint8_t *lc) {
+                                                      uint8_t *lc, int grp, int ngrp, int ew) {
+    const LcParams &L = P.lc;
+    const bool bias = (L.epi & TACKER_EPI_BIAS) != 0, relu = (L.epi & TACKER_EPI_RELU) != 0;
+    if (bias && relu) epilogue_tma_t<true, true>(P, bb, tmem, lc, grp, ngrp, ew);
+    else if (bias) epilogue_tma_t<true, false>(P, bb, tmem, lc, grp, ngrp, ew);
+    else if (relu) epilogue_tma_t<false, true>(P, bb, tmem, lc, grp, ngrp, ew);
+    else epilogue_tma_t<false, false>(P, bb, tmem, lc, grp, ngrp, ew);
+  }
+  template <bool BIAS, bool RELU>
+  static __device__ __forceinline__ void epilogue_tma_t(const FusedParams &P, const Bars &bb, uint32_t tmem,
+                                                        uint8_t *lc, int grp, int ngrp, int ew) {
     static_assert(BN % 64 == 0, "TMA-store epilogue: 64-column batches");
     constexpr int NB = BN / 64;
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;
     const int lane = lane_id();
-    uint8_t *stg = lc + P.epi_stage_off + quarter * 8192;
-    const uint32_t bias_s = smem_u32(bb.bias);
+    const uint32_t ebar = kLcEpiBar - (uint32_t)grp;
+    uint8_t *stg = lc + P.epi_stage_off + ew * P.epi_bufs * 4096;
+    const bool bias = BIAS;
+    const bool bias_res = bias && L.bias_off != 0;
+    const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
+    float *bias_all = bias_res && bconst ? load_bias_resident(L, lc, ebar) : nullptr;   // constant: before the wait
     int buf = 0;
     griddep_wait();
-    int acc = 0;
+    if (bias_res && !bconst) bias_all = load_bias_resident(L, lc, ebar);
+    int acc = grp;
     uint32_t acc_phase = 0;
     int ui = 0;
-    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
+    for (int u = blockIdx.x + grp * gridDim.x; u < L.num_units; u += ngrp * gridDim.x, ++ui) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
       mbar_wait(&bb.tfull[acc], acc_phase);
       tc_fence_after();
-      if (quarter == 0 && lane == 0) lc_stamp(L, 3, ui);
+      if (quarter == 0 && lane == 0 && grp == 0) lc_stamp(L, 3, ui);
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
-      const bool bias = (L.epi & TACKER_EPI_BIAS) != 0;
-      if (bias) {
+      float *tb = bb.bias + grp * BN;   // per-tile staging (one BN slot per group)
+      uint32_t bias_s = smem_u32(tb);
+      if (bias_res) {
+        bias_s = smem_u32(bias_all + nt * BN);
+      } else if (bias) {
         const int et = (int)threadIdx.x % 128;
-        named_bar_sync(kLcEpiBar, 128);
-        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
-        named_bar_sync(kLcEpiBar, 128);
+        named_bar_sync(ebar, 128);
+        for (int c = et; c < BN; c += 128) tb[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(ebar, 128);
       }
       const bool skip = (L.dbg & 1) != 0;
       BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
@@ -562,29 +655,33 @@ struct LcGemm {
         if (b + 1 < NB) tmem_ld64(tbase + 64 * (b + 1), (b % 2) ? va : vb);
         const int n0 = nt * BN + 64 * b;
         if (n0 < L.N && !skip)
-          epi_batch(P, (b % 2) ? vb : va, bias_s + 256 * b, bias, stg, buf, n0, at, lane);
+          epi_batch<BIAS, RELU>(P, (b % 2) ? vb : va, bias_s + 256 * b, stg, buf, n0, at, lane);
       }
       tc_fence_before();
       mbar_arrive(&bb.tempty[acc]);
-      if (quarter == 0 && lane == 0) lc_stamp(L, 4, ui);
-      if (++acc == P.acc_stages) {
-        acc = 0;
-        acc_phase ^= 1;
-      }
+      if (quarter == 0 && lane == 0 && grp == 0) lc_stamp(L, 4, ui);
+      for (acc += ngrp; acc >= P.acc_stages; acc -= P.acc_stages) acc_phase ^= 1;
     }
     if (lane == 0) bulk_wait<0>();            // every store performed before the CTA retires
+    if (lane == 0) lc_gt(L, 5, false);
   }
 
   template <int EC>
-  static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem) {
+  static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem, uint8_t *lc,
+                                                  int grp, int ngrp) {
     static_assert(EC % 16 == 0 && BN % EC == 0, "EC: multiple of 16 dividing BN");
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;          // TMEM lanes 32*quarter .. +31
     const int row_in_tile = quarter * 32 + lane_id();
+    const uint32_t ebar = kLcEpiBar - (uint32_t)grp;
+    const bool bias_res = (L.epi & TACKER_EPI_BIAS) && L.bias_off != 0;
+    const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
+    float *bias_all = bias_res && bconst ? load_bias_resident(L, lc, ebar) : nullptr;   // constant: before the wait
     griddep_wait();                             // residual / D of earlier kernels
-    int acc = 0;
+    if (bias_res && !bconst) bias_all = load_bias_resident(L, lc, ebar);
+    int acc = grp;
     uint32_t acc_phase = 0;
-    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
+    for (int u = blockIdx.x + grp * gridDim.x; u < L.num_units; u += ngrp * gridDim.x) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -594,11 +691,12 @@ struct LcGemm {
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
       float *prow = L.splits > 1 ? L.part + ((size_t)u * kBM + row_in_tile) * BN : nullptr;
       const bool bias = !prow && (L.epi & TACKER_EPI_BIAS);
-      if (bias) {   // stage this tile's bias in shared memory (read as a broadcast per column)
+      float *tbias = bias_res ? bias_all + nt * BN : bb.bias + grp * BN;
+      if (bias && !bias_res) {   // stage this tile's bias in shared memory (read as a broadcast per column)
         const int et = (int)threadIdx.x % 128;
-        named_bar_sync(kLcEpiBar, 128);           // the previous tile's readers are done
-        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
-        named_bar_sync(kLcEpiBar, 128);
+        named_bar_sync(ebar, 128);                // the previous tile's readers are done
+        for (int c = et; c < BN; c += 128) tbias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(ebar, 128);
       }
       const bool res = !prow && (L.epi & TACKER_EPI_RESIDUAL) && orow >= 0;
 #pragma unroll 1
@@ -629,8 +727,8 @@ struct LcGemm {
               for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j / 16][j % 16 + u]);
               __align__(16) float b8[8];
               if (bias) {   // shared-space loads (a generic pointer would compile to LD.E)
-                *reinterpret_cast<float4 *>(b8) = ld_shared_v4f(smem_u32(bb.bias + c0 + j));
-                *reinterpret_cast<float4 *>(b8 + 4) = ld_shared_v4f(smem_u32(bb.bias + c0 + j + 4));
+                *reinterpret_cast<float4 *>(b8) = ld_shared_v4f(smem_u32(tbias + c0 + j));
+                *reinterpret_cast<float4 *>(b8 + 4) = ld_shared_v4f(smem_u32(tbias + c0 + j + 4));
               }
               store8(L, orow, n0 + j, f, b8, rv[j / 8]);
             }
@@ -638,29 +736,27 @@ struct LcGemm {
       }
       tc_fence_before();
       mbar_arrive(&bb.tempty[acc]);
-      if (++acc == P.acc_stages) {
-        acc = 0;
-        acc_phase ^= 1;
-      }
-      if (L.splits > 1) reduce_split(L, t, sp, mt, nt);
+      for (acc += ngrp; acc >= P.acc_stages; acc -= P.acc_stages) acc_phase ^= 1;
+      if (L.splits > 1) reduce_split(L, t, sp, mt, nt, ebar);
     }
+    if (lane_id() == 0) lc_gt(L, 5, false);
   }
 
   // Split-K fixup of tile t by split sp (all splits of the tile run concurrently, one per CTA):
   // wait until every split has written its partial, then reduce elements [sp E/S, (sp+1) E/S) of
   // the tile (E = kBM x BN, in groups of 4 columns) over the splits in order 0..S-1 and store them.
-  static __device__ __forceinline__ void reduce_split(const LcParams &L, int t, int sp, int mt, int nt) {
+  static __device__ __forceinline__ void reduce_split(const LcParams &L, int t, int sp, int mt, int nt, uint32_t ebar) {
     const int S = L.splits;
     const int et = (int)threadIdx.x % 128;      // the 4 epilogue warps are 128 consecutive threads
     uint32_t *arrive = L.cnt + 2 * t, *finish = arrive + 1;
     __threadfence();                            // partial visible before the arrival
-    named_bar_sync(kLcEpiBar, 128);
+    named_bar_sync(ebar, 128);
     if (et == 0) {
       atomicAdd(arrive, 1u);
       while (ld_acquire_gpu(arrive) < (uint32_t)S) {
       }
     }
-    named_bar_sync(kLcEpiBar, 128);
+    named_bar_sync(ebar, 128);
     constexpr int G = BN / 8;                   // 8-column groups per row
     const int E = kBM * G;
     const float *base = L.part + (size_t)t * S * kBM * BN;
@@ -687,7 +783,7 @@ struct LcGemm {
                                                      : make_uint4(0, 0, 0, 0);
       store8(L, orow, n, f, bias, rv);
     }
-    named_bar_sync(kLcEpiBar, 128);
+    named_bar_sync(ebar, 128);
     if (et == 0 && atomicAdd(finish, 1u) == (uint32_t)S - 1) {   // last reducer: reset for the next launch
       *arrive = 0;
       *finish = 0;
@@ -799,7 +895,7 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 // warps) gives every warp up to 144, for bodies that spill at 64 (fft) and for wider LC
 // epilogue batches.  tacker_fuse picks the smallest class that holds the plan's warp split.
 template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND)>
-__global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
+__global__ void __launch_bounds__(32 * ((BE_KIND == TACKER_BE_NONE ? kLcWarpsSolo : kLcWarps) + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();   // the next kernel on the stream may start its prologue
@@ -813,6 +909,10 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
   const int be_warps = 4 * P.be_vb_per_cta;
   const int warp = (int)warp_id() - be_warps;       // LC role index (< 0: BE warp)
   const bool has_lc = P.lc_warps > 0 && P.lc.num_units > 0;
+  if (threadIdx.x == 0) {
+    lc_gt(P.lc, 0, true);
+    lc_gt(P.lc, 4, false);
+  }
   typename LcGemm<BN>::Bars bb{};
   if (P.lc_warps > 0) {
     bb = LcGemm<BN>::bars(lc, P.stages, P.lc.stage_bytes);
@@ -835,6 +935,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
   tc_fence_before();
   __syncthreads();   // bar.sync 0: prologue only
   tc_fence_after();
+  if (threadIdx.x == 0) lc_gt(P.lc, 1, true);
 
   if (warp >= 0) {
     if (has_lc) {
@@ -843,10 +944,13 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
         LcGemm<BN>::producer(P, lc, bb);      // warp-wide loop, elected issue
       } else if (warp == 1) {
         LcGemm<BN>::mma(P, lc, bb, tmem);
-      } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
-        LcGemm<BN>::epilogue_tma(P, bb, tmem, lc);
       } else {
-        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
+        const int ew = warp - 2, grp = ew >> 2, ngrp = (P.lc_warps - 2) >> 2;   // epilogue group
+        if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store)
+          LcGemm<BN>::epilogue_tma(P, bb, tmem, lc, grp, ngrp, ew);
+        else
+          LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(
+              P, bb, tmem, lc, grp, ngrp);
       }
     }
   } else if constexpr (BE_KIND != TACKER_BE_NONE) {
@@ -859,6 +963,7 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     tc_fence_after();
     tmem_dealloc(*bb.tmem_holder, P.tmem_cols);
   }
+  if (threadIdx.x == 0) lc_gt(P.lc, 6, false);
 }
 
 // ------------------------------------------------------------------------ BE original kernel

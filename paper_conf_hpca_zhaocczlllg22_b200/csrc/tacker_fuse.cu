@@ -80,6 +80,7 @@ static constexpr int kSmemCap = 232448;      // max dynamic SMEM per CTA on sm_1
 static constexpr int kTmemCols = 512;
 static constexpr int kMaxWarps = 32;
 static constexpr int kMinLcSmem = 120 * 1024;  // forces one LC CTA per SM (TMEM ownership)
+static constexpr uint32_t kLcHdr = 256 + 8 * 256;  // LC region after the ring: mbarriers + TMEM address, 2 x 256 bias floats
 
 // ============================================================================ BE helpers
 template <int K>
@@ -308,6 +309,54 @@ static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
   return 128;
 }
 
+static int epi_bufs_cfg() {   // TACKER_EPI_BUFS: 2 (default) or 4 TMA-store staging boxes per epilogue warp
+  static const int v = [] {
+    const char *e = getenv("TACKER_EPI_BUFS");
+    return e && atoi(e) == 4 ? 4 : 2;
+  }();
+  return v;
+}
+static int epi_groups_cfg() {   // TACKER_EPI_GROUPS: 1 / 2 forces the LC-only epilogue groups, 0 (default) = heuristic
+  static const int v = [] {
+    const char *e = getenv("TACKER_EPI_GROUPS");
+    const int g = e ? atoi(e) : 0;
+    return g == 1 || g == 2 ? g : 0;
+  }();
+  return v;
+}
+static int lc_kps() {
+  static const int v = [] {
+    const char *e = getenv("TACKER_KPS");
+    const int k = e ? atoi(e) : 2;
+    return k < 1 ? 1 : k > 4 ? 4 : k;
+  }();
+  return v;
+}
+static int lc_kps64() {   // BN = 64 override (0: TACKER_KPS); 3 measured best (b32 ResNet-50 query)
+  static const int v = [] {
+    const char *e = getenv("TACKER_KPS64");
+    const int k = e ? atoi(e) : 3;
+    return k < 0 ? 0 : k > 4 ? 4 : k;
+  }();
+  return v;
+}
+static int lc_kps_max_bn() {
+  static const int v = [] {
+    const char *e = getenv("TACKER_KPS_MAXBN");
+    return e ? atoi(e) : 128;
+  }();
+  return v;
+}
+
+// resident bias (TACKER_BIAS_RES=0 restores per-tile staging)
+static bool bias_resident_enabled() {
+  static const bool on = [] {
+    const char *e = getenv("TACKER_BIAS_RES");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 // TMA-store epilogue for eligible LC-only plans (TACKER_EPI_TMA=0 restores the register path)
 static bool tma_store_enabled() {
   static const bool on = [] {
@@ -360,6 +409,7 @@ static bool conv_s2c8_ok(const LcParams &L, int BN) {
 
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
+  L.kps = 1;
   L.stage_a = kBM * kBK * 2;
   L.stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
   if (conv_s2c8_ok(L, BN)) {
@@ -727,6 +777,15 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   lc_tiles(L, BN);
   if (!(lc->epi_flags & TACKER_LC_NO_SPLIT)) lc_split(L, sms);
   F.BN = BN;
+  // two k-blocks per ring stage for LC-only plain-GEMM / 1x1 / im2col-mode plans with narrow tiles
+  // (fused.cuh LcParams::kps); TACKER_KPS=1 restores one, TACKER_KPS_MAXBN the widest tile using it
+  const int kps = BN == 64 && lc_kps64() > 0 ? lc_kps64() : lc_kps();
+  if (!has_be && kps > 1 && BN <= lc_kps_max_bn() && L.num_kb >= 2 && !L.conv_halo && !L.conv_s2c8 &&
+      !L.conv_c8 && (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col)) {
+    L.kps = kps;
+    L.stage_a *= (uint32_t)L.kps;
+    L.stage_bytes *= (uint32_t)L.kps;
+  }
 
   int64_t be_blocks = 0;
   int vb = 0;
@@ -754,13 +813,30 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
                 !(lc->epi_flags & TACKER_EPI_RESIDUAL) && L.splits == 1 && BN >= 64 && L.N >= 64 &&
                 (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col || L.conv_halo ||
                  L.conv_s2c8);
-  const uint32_t epi_bytes = (L.tma_store ? 4u * 2u * 4096u + 1024u : 0u) +
+  // epilogue warps: LC-only plans with two TMEM accumulator stages run two epilogue groups (one per
+  // stage, fused.cuh epilogue_tma); fused CTAs keep one group of 4 (their warps go to the BE)
+  // when the epilogue work per CTA is large (units / SMs x BN >= 512 columns: the 1x1 convs with
+  // many short-K tiles measured faster; below it the larger staging costs ring stages)
+  const bool two_groups = !has_be && acc == 2 &&
+                          (epi_groups_cfg() == 2 ||
+                           (epi_groups_cfg() == 0 && (int64_t)L.num_units * BN >= 512LL * sms));
+  const int lc_warps = two_groups ? kLcWarpsSolo : kLcWarps;
+  const uint32_t epi_warps = (uint32_t)lc_warps - 2u;
+  const uint32_t epi_bufs = L.tma_store ? (uint32_t)epi_bufs_cfg() : 0u;   // staging boxes per epilogue warp
+  const uint32_t epi_bytes = (L.tma_store ? epi_warps * epi_bufs * 4096u + 1024u : 0u) +
                              (L.conv_s2c8 ? 2u * L.s2_pairs * 1024u + 1024u : 0u);   // + resident weights
   L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
   const uint32_t stage_bytes = L.stage_bytes;
-  const uint32_t bar_bytes = 256 + 4 * 256 + epi_bytes;   // mbarriers + TMEM address + one tile's bias (BN <= 256) + staging
+  // resident bias (fused.cuh LcParams::bias_off): tiles_n x BN floats, when at most 16 KB
+  const uint32_t bias_bytes = (lc->epi_flags & TACKER_EPI_BIAS) && bias_resident_enabled() &&
+                                      (uint32_t)L.tiles_n * BN * 4u <= 16384u
+                                  ? (uint32_t)L.tiles_n * BN * 4u
+                                  : 0u;
+  // mbarriers + TMEM address (256) + one tile's bias per epilogue group (2 x BN <= 256 floats) +
+  // staging + resident bias
+  const uint32_t bar_bytes = kLcHdr + epi_bytes + (bias_bytes ? bias_bytes + 16 : 0);
   const uint32_t be_total = (uint32_t)vb * be_slice;
   // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
   // SM for the latency-bound implicit-GEMM loads); fused plans stop at 4 so the BE keeps L1
@@ -776,23 +852,33 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     set_error("fused budget exceeds one SM: LC ring %u B x2 + BE %d x %u B > %d B", stage_bytes, vb, be_slice, kSmemCap);
     return TACKER_ERESOURCE;
   }
-  const int warps = kLcWarps + warp_split;
+  const int warps = lc_warps + warp_split;
   if (warps > kMaxWarps) return set_error("too many warps"), TACKER_ERESOURCE;
 
   F.P.stages = stages;
   F.P.acc_stages = acc;
   F.P.tmem_cols = cols;
   F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
-  F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + 256u + 4u * 256u + 1023u) & ~1023u : 0u;
+  F.P.epi_bufs = (int32_t)epi_bufs;
+  F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + kLcHdr + 1023u) & ~1023u : 0u;
   if (L.conv_s2c8) {
-    const uint32_t after = L.tma_store ? F.P.epi_stage_off + 4u * 2u * 4096u : (uint32_t)stages * stage_bytes + 1280u;
+    const uint32_t after = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
     L.b_res_off = (after + 1023u) & ~1023u;
+  }
+  {   // resident bias after everything else of the LC region (16-aligned)
+    uint32_t end = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
+    if (L.conv_s2c8) end = L.b_res_off + 2u * L.s2_pairs * 1024u;
+    L.bias_off = bias_bytes ? ((end + 15u) & ~15u) : 0u;
+    if (bias_bytes && L.bias_off + bias_bytes > F.P.lc_smem_bytes) {
+      set_error("internal: resident bias outside the LC region (%u + %u > %u)", L.bias_off, bias_bytes, F.P.lc_smem_bytes);
+      return TACKER_ERESOURCE;
+    }
   }
   F.P.be_smem_per_vb = be_slice;
   F.P.be_vb_per_cta = vb;
   F.P.be_blocks = be_blocks;
   F.P.be_offset = has_be ? be->block_offset : 0;
-  F.P.lc_warps = kLcWarps;
+  F.P.lc_warps = lc_warps;
   F.warp_split = warp_split;
   F.block = 32 * warps;
   F.smem = 1024 + F.P.lc_smem_bytes + be_total;
@@ -896,7 +982,9 @@ static tacker_status alloc_lc_workspace(tacker_fused_s &F) {
   return TACKER_OK;
 }
 
+static std::atomic<int> g_dbg_launch{0};
 static tacker_status launch_params(const tacker_fused_s &F, FusedParams &P, cudaStream_t s) {
+  if (P.lc.dbg & 16) P.lc.dbg_id = g_dbg_launch.fetch_add(1) & 255;   // diagnostics slot
   cudaError_t e = launch_ex(F.fn, dim3(F.grid), dim3(F.block), F.smem, s, P);
   if (e != cudaSuccess) return cuda_fail("launch fused_kernel", e);
   return TACKER_OK;
@@ -975,6 +1063,17 @@ tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n) {
   if (!out || n < 160 * 5 * 16) return set_error("need 12800 uint64 slots"), TACKER_EINVAL;
   cudaError_t e = cudaMemcpyFromSymbol(out, tk::g_lc_ts, sizeof(tk::g_lc_ts));
   if (e != cudaSuccess) return cuda_fail("debug timestamps", e);
+  return TACKER_OK;
+}
+
+tacker_status tacker_debug_lc_globaltimer(uint64_t *out, int64_t n, int32_t *next_slot) {
+  if (!out || n < 256 * 8) return set_error("need 2048 uint64 slots"), TACKER_EINVAL;
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpyFromSymbol(out, tk::g_lc_gt, sizeof(tk::g_lc_gt));
+  static const unsigned long long zero[256][8] = {};
+  if (e == cudaSuccess) e = cudaMemcpyToSymbol(tk::g_lc_gt, zero, sizeof zero);
+  if (e != cudaSuccess) return cuda_fail("debug globaltimer", e);
+  if (next_slot) *next_slot = g_dbg_launch.exchange(0) & 255;
   return TACKER_OK;
 }
 
@@ -1183,6 +1282,8 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
   if (lc && lc->kind != TACKER_LC_NONE) {
     // LC-only plans (tensor maps, smem attribute) are cached by descriptor bytes: the manager
     // re-launches the same LC kernels every query.
+    // Entries are never evicted: a plan (and its split-K workspace) may still be in use by a
+    // launch in flight, and a service has a bounded set of LC descriptors.
     static std::mutex mu;
     static std::unordered_map<std::string, std::unique_ptr<tacker_fused_s>> cache;
     const std::string key(reinterpret_cast<const char *>(lc), sizeof *lc);
@@ -1198,8 +1299,13 @@ tacker_status tacker_launch_original(const tacker_lc_desc *lc, const tacker_be_d
       P->P.work = nullptr;
       if ((st = alloc_lc_workspace(*P))) return st;
       std::lock_guard<std::mutex> g(mu);
-      if (cache.size() > 4096) cache.clear();
-      F = (cache[key] = std::move(P)).get();
+      auto it = cache.find(key);   // another thread may have planned the same descriptor meanwhile
+      if (it != cache.end()) {
+        if (P->P.lc.part) cudaFree(P->P.lc.part);
+        F = it->second.get();
+      } else {
+        F = (cache[key] = std::move(P)).get();
+      }
     }
     if ((st = launch_plan(*F, s))) return st;
   }

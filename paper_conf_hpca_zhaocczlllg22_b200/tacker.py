@@ -266,6 +266,7 @@ _PROTOS = {
     "tacker_launch_fused_slice": ([_V, _I64, _I64, _V], C.c_int),
     "tacker_set_launch_overlap": ([_I32], C.c_int),
     "tacker_debug_lc_timestamps": ([C.POINTER(C.c_uint64), _I64], C.c_int),
+    "tacker_debug_lc_globaltimer": ([C.POINTER(C.c_uint64), _I64, C.POINTER(C.c_int32)], C.c_int),
     "tacker_select_fusion": ([C.POINTER(LcDesc), C.POINTER(BeDesc), C.POINTER(_I32), _I32, _I32, _V,
                               C.POINTER(_I32), C.POINTER(_D), C.POINTER(_D), C.POINTER(_D)], C.c_int),
     "tacker_blacklist": ([C.c_char_p, _I32, C.POINTER(_I32)], C.c_int),
@@ -648,6 +649,16 @@ def tacker_blacklist(be_key: str, op: int = -1) -> bool:
 
 def tacker_blacklist_clear():
     _chk(_lib.tacker_blacklist_clear())
+
+
+def tacker_debug_lc_globaltimer():
+    """([256][8] %globaltimer stamps per LC launch (plans built with TACKER_LC_DBG bit 4 = 16),
+    number of launches recorded); clears the buffer."""
+    import numpy as np
+    buf = (C.c_uint64 * (256 * 8))()
+    n = C.c_int32()
+    _chk(_lib.tacker_debug_lc_globaltimer(buf, len(buf), C.byref(n)))
+    return np.frombuffer(buf, dtype=np.uint64).reshape(256, 8).copy(), n.value
 
 
 def tacker_debug_lc_timestamps():
