@@ -8,8 +8,20 @@
 
 namespace tk {
 constexpr int kVbThreads = 128;
+#ifndef TK_MRIQ_RINT
+#define TK_MRIQ_RINT 0   // 1: rintf (FRND) in the mri-q range reduction: measured 0.150 -> 0.189 ms (slow pipe)
+#endif
+// stencil: planes per thread and resident blocks of the original launch.  Measured (512x512x64,
+// standalone): ZC 4 / 8 blocks 31.5 us, ZC 2 / 12 blocks 30 us, ZC 4 / 1 block (74 regs) 37 us;
+// fused (ws 24 beside a b1 conv) ZC 4 48 us, ZC 2 55 us -- ZC 4 / 8 blocks kept
 #ifndef TK_STENCIL_ZC
 #define TK_STENCIL_ZC 4
+#endif
+#ifndef TK_STENCIL_COARSEN
+#define TK_STENCIL_COARSEN 1
+#endif
+#ifndef TK_STENCIL_MIN_BLOCKS
+#define TK_STENCIL_MIN_BLOCKS 8
 #endif
 #ifndef TK_STENCIL_HOIST
 #define TK_STENCIL_HOIST 0

@@ -60,7 +60,9 @@ __host__ __device__ constexpr int be_max_warps(int kind) {
 }
 // Minimum resident blocks per SM of an original (standalone) BE launch: caps the registers of
 // bodies whose latency hiding needs many blocks (fft: TK_FFT_MIN_BLOCKS = 8 blocks -> <= 64 registers).
-__host__ __device__ constexpr int be_orig_min_blocks(int kind) { return kind == TACKER_BE_FFT ? TK_FFT_MIN_BLOCKS : 1; }
+__host__ __device__ constexpr int be_orig_min_blocks(int kind) {
+  return kind == TACKER_BE_FFT ? TK_FFT_MIN_BLOCKS : kind == TACKER_BE_STENCIL ? TK_STENCIL_MIN_BLOCKS : 1;
+}
 
 // Body call with the optional per-kind TMA tensor map (only the stencil uses one).
 template <int KIND>
@@ -73,6 +75,7 @@ __device__ __forceinline__ void be_run(const tacker_be_desc &d, int64_t vb, int 
 template <int KIND> struct BeCoarsen { static constexpr int value = 1; };
 template <> struct BeCoarsen<TACKER_BE_MRIQ_Q> { static constexpr int value = BeBody<TACKER_BE_MRIQ_Q>::kCoarsen; };
 template <> struct BeCoarsen<TACKER_BE_MRIFHD_FH> { static constexpr int value = BeBody<TACKER_BE_MRIFHD_FH>::kCoarsen; };
+template <> struct BeCoarsen<TACKER_BE_STENCIL> { static constexpr int value = BeBody<TACKER_BE_STENCIL>::kCoarsen; };
 template <int KIND>
 __device__ __forceinline__ void be_run_coarse(const tacker_be_desc &d, int64_t vb, int nb, int tid, uint32_t bar,
                                               uint8_t *smem, const CUtensorMap *tm) {

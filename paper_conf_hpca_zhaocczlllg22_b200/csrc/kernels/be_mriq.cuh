@@ -59,8 +59,12 @@ template <> struct BeBody<TACKER_BE_MRIQ_Q> {
     const float kTwoPi = 6.2831853071795864769f;
     float t = __fmaf_rn(kv.z, z, __fmaf_rn(kv.y, y, __fmul_rn(kv.x, x)));
 #if TK_MRIQ_REDUCE
+#if TK_MRIQ_RINT
+    t = __fsub_rn(t, rintf(t));         // FRND: the same value as the magic-number form, one instruction
+#else
     const float kMagic = 12582912.0f;   // 1.5 * 2^23: (t + M) - M == rint(t) for |t| < 2^22
     t = __fsub_rn(t, __fsub_rn(__fadd_rn(t, kMagic), kMagic));
+#endif
 #endif
     float s, c;
     __sincosf(__fmul_rn(kTwoPi, t), &s, &c);

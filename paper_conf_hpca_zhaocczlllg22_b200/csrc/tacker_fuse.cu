@@ -124,6 +124,7 @@ static tacker_status validate_be(const tacker_be_desc &d, int64_t *blocks) {
     case TACKER_BE_STENCIL: {
       const auto &p = d.p.stencil;
       if (p.nx <= 0 || p.ny <= 0 || p.nz <= 0 || !p.A0 || !p.Anext) return set_error("stencil: bad args"), TACKER_EINVAL;
+      if (full > 0x7fffffffLL) return set_error("stencil: more than 2^31 - 1 blocks"), TACKER_EUNSUPPORTED;
       break;
     }
     case TACKER_BE_MRIQ_PHIMAG:
