@@ -90,6 +90,12 @@ class TwoStage:
             if len(nlo) < 2 or len(nhi) < 2 or (nlo == lo and nhi == hi):
                 break
             lo, hi = nlo, nhi
+        if self.l1[1] >= self.l2[1]:
+            # DESIGN.md reading 5: the two stages of Fig. 10 are co-run (slope below the CD-solo
+            # stage's) then CD solo; fitted slopes in the other order describe no such
+            # curve (max() would put the steeper first stage at large r), so one LR over all samples
+            b, a = ols([p[0] for p in pts], [p[1] for p in pts])
+            self.l1 = self.l2 = (a, b)
         return self.l1, self.l2
 
     def inflection(self):

@@ -83,6 +83,14 @@ bool fit_pair(Pair &P, double split) {
     lo.swap(nlo);
     hi.swap(nhi);
   }
+  // Fig. 10's stages are co-run (slope below the CD-solo stage's) then CD solo; fitted
+  // slopes in the other order describe no such curve (max() would put the steeper first stage at
+  // large r): one LR over all samples (reading 5)
+  if (P.b1 >= P.b2) {
+    ols(pts, P.b1, P.a1);
+    P.a2 = P.a1;
+    P.b2 = P.b1;
+  }
   P.fitted = true;
   return true;
 }

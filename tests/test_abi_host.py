@@ -132,6 +132,21 @@ def test_two_stage_c_matches_oracle_and_refits(tk):
     assert abs(tk.tacker_pair_predict("p", 1.0, 1.0) - m.predict(1.0, 1.0)) < 1e-12
 
 
+def test_two_stage_inverted_slopes_c_matches_oracle(tk):
+    # the single-LR fallback of reading 5 (stage slopes b1 >= b2): C == oracle
+    tk.tacker_model_clear()
+    m = op.TwoStage()
+    for r in (0.2, 0.4, 0.6, 0.8, 1.5, 2.5, 4.0, 6.0):
+        tau = 1 + 2.0 * r if r < 1 else 3.0 + (r - 1.0)
+        tk.tacker_pair_add_sample("inv", 1.0, r, tau)
+        m.add(1.0, r, tau)
+    c = tk.tacker_pair_fit("inv")
+    (a1, b1), (a2, b2) = m.fit()
+    assert np.allclose(c, (a1, b1, a2, b2), rtol=0, atol=1e-12) and c[1] == c[3]
+    for r in (0.1, 1.0, 7.0):
+        assert abs(tk.tacker_pair_predict("inv", 1.0, r) - m.predict(1.0, r)) < 1e-12
+
+
 def test_model_save_load_roundtrip(tk, tmp_path):
     tk.tacker_model_clear()
     for x in (1, 2, 3):

@@ -318,3 +318,30 @@ def test_manager_idle_round_robin():
     assert idle[:4] == [0, 1, 0, 1]
     # 0..5 app 0, 5..6 app 1, 6..11 app 0, 11..12 app 1, 12..17 app 0 -> the query (13) waits to 17
     assert res["latency"][0] == 17.0 - 13.0 + 1.0
+
+
+def test_two_stage_inverted_slopes_fall_back_to_one_lr():
+    # DESIGN.md reading 5: samples of a concave curve (steep, then slope 1) give stage slopes in
+    # the wrong order for Fig. 10's co-run -> CD-solo shape; the model must be the single LR over
+    # all samples (pinned against numpy.polyfit), not max() of the two lines
+    import numpy as np
+    from oracle import predictor as op
+    rs = [0.2, 0.4, 0.6, 0.8, 1.5, 2.5, 4.0, 6.0]
+    taus = [1 + 2.0 * r if r < 1 else 3.0 + (r - 1.0) for r in rs]
+    m = op.TwoStage()
+    for r, t in zip(rs, taus):
+        m.add(1.0, r, t)
+    (a1, b1), (a2, b2) = m.fit()
+    b, a = np.polyfit(rs, taus, 1)
+    assert (a1, b1) == (a2, b2)
+    assert abs(b1 - b) < 1e-12 and abs(a1 - a) < 1e-12
+    assert m.inflection() is None
+    for r in (0.3, 1.0, 5.0):
+        assert abs(m.tau(r) - (a + b * r)) < 1e-12
+    # a convex curve keeps its two stages (b1 < b2)
+    m2 = op.TwoStage()
+    for r in rs:
+        m2.add(1.0, r, max(1 + 0.3 * r, 0.55 + r))
+    (c1, d1), (c2, d2) = m2.fit()
+    assert d1 < d2 and abs(d2 - 1.0) < 1e-9
+
