@@ -26,6 +26,7 @@ constexpr int kLcWarpsSolo = 10;   // LC-only CTAs: producer, MMA, 2 epilogue gr
 constexpr int kBM = 128;   // UMMA M
 constexpr int kBK = 64;    // one 128-byte swizzle row of fp16
 constexpr int kUK = 16;    // UMMA K for kind::f16
+constexpr int kMaxAcc = 4;          // TMEM accumulator stages (tiles in flight between MMA and epilogue)
 constexpr uint32_t kLcEpiBar = 15;   // named barrier of the 4 LC epilogue warps (BE uses 1..14)
 
 struct LcParams {
@@ -46,6 +47,9 @@ struct LcParams {
                              // 16 B, loaded as 8 unswizzled 128 x 16 B boxes (K-major, no swizzle)
   int32_t conv_im2col;       // implicit conv through the TMA im2col mode: M-tile = 128 consecutive
                              // output pixels (n, p, q linear); else tp x tq windows of one image
+  int32_t halo_bres;         // halo mode with the whole filter resident in shared memory (one N tile): B
+                             // loaded once per CTA at b_res_off, chunk ((r S + s) c_blocks + cb) x BN x 128 B;
+                             // a ring stage holds only the input halo
   int32_t conv_halo;         // stride-1 conv, C % 64 == 0: M-tile = 16 x 8 output pixels; a k-step =
                              // (filter row r, channel block cb) loads ONE input halo of 16 x (8+S-1)
                              // pixels x 64 channels (SW128) and the S taps' weights, and issues S x 4
@@ -169,8 +173,10 @@ struct LcGemm {
   }
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages, uint32_t stage_bytes) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * stage_bytes);
-    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4),
-                reinterpret_cast<float *>(b + 2 * stages + 6), b + 2 * stages + 5};
+    // full[S], empty[S], tfull[4], tempty[4] (up to kMaxAcc TMEM accumulator stages), TMEM address,
+    // resident-weights barrier, then the per-tile bias slots (16-byte aligned)
+    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + kMaxAcc, reinterpret_cast<uint32_t *>(b + 2 * stages + 2 * kMaxAcc),
+                reinterpret_cast<float *>(b + 2 * stages + 2 * kMaxAcc + 2), b + 2 * stages + 2 * kMaxAcc + 1};
   }
 
   // resident bias (L.bias_off != 0): the 128 epilogue threads copy tiles_n x BN bias values
@@ -310,7 +316,8 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8 &&
+        !L.halo_bres) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -342,6 +349,21 @@ struct LcGemm {
         mbar_arrive_expect_tx(bb.bres, bytes);
         for (int c = 0; c < 2 * L.s2_pairs; ++c)
           if (L.s2_chunk_tap[c] >= 0) tma_load_2d(&P.tmap_b, bb.bres, bres + c * 1024, L.s2_chunk_tap[c] * 8, 0);
+      }
+      __syncwarp();
+    }
+    if (L.halo_bres) {
+      // the whole filter (one N tile), once per CTA; constant weights load before the dependency
+      // wait (TACKER_LC_B_CONST), others after it
+      const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
+      if (!bconst) griddep_wait();
+      if (elect_one()) {
+        uint8_t *bres = lc + L.b_res_off;
+        const int chunks = L.r * L.s * L.c_blocks;
+        mbar_arrive_expect_tx(bb.bres, (uint32_t)chunks * BN * 128u);
+        for (int rs = 0; rs < L.r * L.s; ++rs)
+          for (int cb = 0; cb < L.c_blocks; ++cb)
+            tma_load_2d(&P.tmap_b, bb.bres, bres + (uint32_t)(rs * L.c_blocks + cb) * BN * 128u, rs * L.c + cb * kBK, 0);
       }
       __syncwarp();
     }
@@ -403,7 +425,9 @@ struct LcGemm {
             for (int ph = 0; ph < 4; ++ph)
               tma_load_4d(&P.tmap_a, &bb.full[stage], sa + ph * L.s2_phase_stride, 0, w0 + (ph & 1), h0 + (ph >> 1), img);
           } else if (L.conv_halo) {
-            if (!first) {
+            if (L.halo_bres) {
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);   // the halo only (stage_bytes = stage_a)
+            } else if (!first) {
               mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
               for (int t = 0; t < L.s; ++t)   // the filter row's S taps: K columns (rr S + t) C + 64 cb
                 tma_load_2d(&P.tmap_b, &bb.full[stage], sb + t * BN * 128, (rr * L.s + t) * L.c + cb * kBK, nt * BN);
@@ -462,7 +486,7 @@ struct LcGemm {
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
     int ui = 0;
-    if (L.conv_s2c8) mbar_wait(bb.bres, 0);   // resident weights landed
+    if (L.conv_s2c8 || L.halo_bres) mbar_wait(bb.bres, 0);   // resident weights landed
     for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1;
       unit_coords(L, u, t, sp, kb0, kb1);
@@ -493,9 +517,13 @@ struct LcGemm {
             // tap s of this filter row: A = the halo from row s, 8-row groups (one output row of 8
             // pixels each) (8 + S - 1) rows apart; B = the tap's BN x 64 weight slot
             const uint32_t sbo = (uint32_t)(8 + L.s - 1) * 128u;
+            // B of tap t: the stage's slot, or chunk ((r S + t) c_blocks + cb) of the resident filter
+            const int hcb = kb % L.c_blocks, hr = kb / L.c_blocks;
+            const uint32_t bres0 = smem_u32(lc + L.b_res_off) + (uint32_t)(hr * L.s * L.c_blocks + hcb) * BN * 128u;
             for (int t = 0; t < L.s; ++t) {
               const uint64_t da = umma_desc_sw128_sbo(sa + 128u * t, sbo);
-              const uint64_t db = umma_desc_sw128(sb + (uint32_t)t * BN * 128u);
+              const uint64_t db = umma_desc_sw128(L.halo_bres ? bres0 + (uint32_t)(t * L.c_blocks) * BN * 128u
+                                                              : sb + (uint32_t)t * BN * 128u);
 #pragma unroll
               for (int k = 0; k < kBK / kUK; ++k)
                 umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || t != 0 || k != 0));
@@ -923,7 +951,7 @@ __global__ void __launch_bounds__(32 * ((BE_KIND == TACKER_BE_NONE ? kLcWarpsSol
         mbar_init(&bb.full[s], 1);
         mbar_init(&bb.empty[s], 1);
       }
-      for (int a = 0; a < 2; ++a) {
+      for (int a = 0; a < kMaxAcc; ++a) {
         mbar_init(&bb.tfull[a], 1);
         mbar_init(&bb.tempty[a], 4 * 32);
       }

@@ -397,6 +397,21 @@ static bool conv_halo_ok(const LcParams &L, int BN) {
          L.r == L.s && L.s <= 7 && 2 * L.pad == L.s - 1 && L.p >= 8 && L.q >= 8 && BN <= 128;
 }
 
+static int acc_cfg() {   // TACKER_ACC: TMEM accumulator stages wanted for LC-only plans (2 or 4)
+  static const int v = [] {
+    const char *e = getenv("TACKER_ACC");
+    return e && atoi(e) == 4 ? 4 : 2;
+  }();
+  return v;
+}
+static bool halo_bres_enabled() {   // TACKER_HALO_BRES=0: halo plans reload the filter per k-step
+  static const bool on = [] {
+    const char *e = getenv("TACKER_HALO_BRES");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 // Phase-halo mode for stride-2 convs over 8 channels (ResNet-50 conv1: 7x7, 3 channels padded to
 // 8), N <= 64: replaces the explicit im2col + GEMM of §VIII-H.  TACKER_CONV_S2C8=0 disables it.
 static bool conv_s2c8_ok(const LcParams &L, int BN) {
@@ -802,8 +817,15 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     be_slice = (16 + be_smem_bytes(be->kind) + 127) & ~127u;
     F.P.be = *be;
   }
-  const int acc = ratio.lc ? ratio.lc : (2 * BN <= kTmemCols ? 2 : 1);
-  if (acc < 1 || acc > 2 || acc * BN > kTmemCols)
+  // TMEM accumulator stages: 2 by default; LC-only plans of narrow tiles take up to 4 (TACKER_ACC)
+  // so more tiles are in flight between the MMA warp and the epilogue (the commit -> epilogue ->
+  // tempty round trip per tile bounded the many-tile N = 64 convs)
+  int acc = ratio.lc ? ratio.lc : (2 * BN <= kTmemCols ? 2 : 1);
+  if (!ratio.lc && !has_be) {
+    const int want = acc_cfg();
+    while (acc < want && acc < kMaxAcc && 2 * acc * BN <= kTmemCols) acc *= 2;
+  }
+  if (acc < 1 || acc > kMaxAcc || acc * BN > kTmemCols)
     return set_error("block_ratio.lc (TMEM accumulator stages) %d does not fit %d columns", acc, kTmemCols), TACKER_ERESOURCE;
   uint32_t cols = 32;
   while (cols < (uint32_t)(acc * BN)) cols <<= 1;
@@ -818,14 +840,22 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // stage, fused.cuh epilogue_tma); fused CTAs keep one group of 4 (their warps go to the BE)
   // when the epilogue work per CTA is large (units / SMs x BN >= 512 columns: the 1x1 convs with
   // many short-K tiles measured faster; below it the larger staging costs ring stages)
-  const bool two_groups = !has_be && acc == 2 &&
+  const bool two_groups = !has_be && acc % 2 == 0 &&
                           (epi_groups_cfg() == 2 ||
                            (epi_groups_cfg() == 0 && (int64_t)L.num_units * BN >= 512LL * sms));
   const int lc_warps = two_groups ? kLcWarpsSolo : kLcWarps;
   const uint32_t epi_warps = (uint32_t)lc_warps - 2u;
+  // halo mode, LC-only, one N tile: the whole filter resident in shared memory (<= 96 KB), a ring
+  // stage then holds only the input halo (the B re-load per tile was half of the L2 -> SMEM bytes)
+  const uint32_t halo_bres_bytes = (uint32_t)L.r * L.s * L.c_blocks * BN * 128u;
+  if (!has_be && L.conv_halo && L.tiles_n == 1 && L.splits == 1 && halo_bres_enabled() && halo_bres_bytes <= 96u * 1024u) {
+    L.halo_bres = 1;
+    L.stage_bytes = L.stage_a;
+  }
+  const uint32_t res_bytes = L.conv_s2c8 ? 2u * L.s2_pairs * 1024u : L.halo_bres ? halo_bres_bytes : 0u;
   const uint32_t epi_bufs = L.tma_store ? (uint32_t)epi_bufs_cfg() : 0u;   // staging boxes per epilogue warp
   const uint32_t epi_bytes = (L.tma_store ? epi_warps * epi_bufs * 4096u + 1024u : 0u) +
-                             (L.conv_s2c8 ? 2u * L.s2_pairs * 1024u + 1024u : 0u);   // + resident weights
+                             (res_bytes ? res_bytes + 1024u : 0u);   // + resident weights
   L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
@@ -862,13 +892,13 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
   F.P.epi_bufs = (int32_t)epi_bufs;
   F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + kLcHdr + 1023u) & ~1023u : 0u;
-  if (L.conv_s2c8) {
+  if (res_bytes) {
     const uint32_t after = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
     L.b_res_off = (after + 1023u) & ~1023u;
   }
   {   // resident bias after everything else of the LC region (16-aligned)
     uint32_t end = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
-    if (L.conv_s2c8) end = L.b_res_off + 2u * L.s2_pairs * 1024u;
+    if (res_bytes) end = L.b_res_off + res_bytes;
     L.bias_off = bias_bytes ? ((end + 15u) & ~15u) : 0u;
     if (bias_bytes && L.bias_off + bias_bytes > F.P.lc_smem_bytes) {
       set_error("internal: resident bias outside the LC region (%u + %u > %u)", L.bias_off, bias_bytes, F.P.lc_smem_bytes);
