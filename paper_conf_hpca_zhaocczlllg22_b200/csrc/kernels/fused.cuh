@@ -59,6 +59,7 @@ struct LcParams {
   // k-blocks then kps B k-blocks and one full/empty handshake covers 4 kps MMAs -- the handshake
   // (~370 cycles) otherwise bounds N <= 128 mainloops (4 MMAs of 32-64 cycles per k-block)
   int32_t kps;
+  int32_t raster_g;          // > 1: grouped tile raster (tile_coords), plain GEMMs with many tiles
   // stride-2 conv with C = 8 (ResNet conv1, 7x7 over 3 channels padded to 8), "phase halo" mode:
   // M-tile = 16 x 8 output pixels; a stage holds the input halo split into the 4 parity phases
   // (even/odd rows x even/odd columns, TMA traversal stride 2), each [rows][cols] pixels of 16 B,
@@ -190,6 +191,18 @@ struct LcGemm {
     return b;
   }
   static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
+    if (L.raster_g > 1) {
+      // grouped raster (large GEMMs): groups of raster_g M-tiles, M fastest inside a group, so a
+      // wave of CTAs covers raster_g x (grid / raster_g) tiles whose A rows and B columns stay in
+      // L2 (N-fastest order streamed all of B once per ~grid / tiles_n M-tiles: 7.8x the
+      // algorithmic DRAM bytes at 8192^3)
+      const int per = L.raster_g * L.tiles_n;
+      const int g = t / per, r = t - g * per;
+      const int m0 = g * L.raster_g, gm = min(L.raster_g, L.tiles_m - m0);
+      mt = m0 + r % gm;
+      nt = r / gm;
+      return;
+    }
     // N-tiles fastest: consecutive CTAs share the A rows (L2 reuse of the activation tile)
     mt = t / L.tiles_n;
     nt = t % L.tiles_n;

@@ -397,6 +397,21 @@ static bool conv_halo_ok(const LcParams &L, int BN) {
          L.r == L.s && L.s <= 7 && 2 * L.pad == L.s - 1 && L.p >= 8 && L.q >= 8 && BN <= 128;
 }
 
+static int raster_cfg() {   // TACKER_RASTER: M-tiles per raster group of large GEMMs (0/1 = N-fastest order)
+  static const int v = [] {
+    const char *e = getenv("TACKER_RASTER");
+    return e ? atoi(e) : 8;
+  }();
+  return v;
+}
+static int fused_stages_cfg() {   // TACKER_FUSED_STAGES: deepest LC ring of a fused plan (2..4, default 4)
+  static const int v = [] {
+    const char *e = getenv("TACKER_FUSED_STAGES");
+    const int k = e ? atoi(e) : 4;
+    return k < 2 ? 2 : k > 4 ? 4 : k;
+  }();
+  return v;
+}
 static int acc_cfg() {   // TACKER_ACC: TMEM accumulator stages wanted for LC-only plans (2 or 4)
   static const int v = [] {
     const char *e = getenv("TACKER_ACC");
@@ -793,6 +808,11 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   lc_tiles(L, BN);
   if (!(lc->epi_flags & TACKER_LC_NO_SPLIT)) lc_split(L, sms);
   F.BN = BN;
+  // grouped raster for plain GEMMs whose B does not stay in L2 across an N-fastest sweep
+  L.raster_g = (lc->kind == TACKER_LC_GEMM_F16 && raster_cfg() > 1 && L.splits == 1 && L.tiles_m >= 2 * raster_cfg() &&
+                L.tiles_n >= 16)
+                   ? raster_cfg()
+                   : 0;
   // two k-blocks per ring stage for LC-only plain-GEMM / 1x1 / im2col-mode plans with narrow tiles
   // (fused.cuh LcParams::kps); TACKER_KPS=1 restores one, TACKER_KPS_MAXBN the widest tile using it
   const int kps = BN == 64 && lc_kps64() > 0 ? lc_kps64() : lc_kps();
@@ -872,7 +892,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
   // SM for the latency-bound implicit-GEMM loads); fused plans stop at 4 so the BE keeps L1
   int stages = 0;
-  for (int s = has_be ? 4 : 8; s >= 2; --s) {
+  for (int s = has_be ? fused_stages_cfg() : 8; s >= 2; --s) {
     const uint32_t need = 1024 + s * stage_bytes + bar_bytes + be_total;
     if (need <= (uint32_t)kSmemCap) {
       stages = s;

@@ -42,6 +42,25 @@ def test_lc_gemm_exact_variants(tk, variant):
     assert np.array_equal(host(D).astype(np.float64), ref)
 
 
+@pytest.mark.parametrize("M,N,K", [(2304, 2176, 128), (4096 + 200, 2048, 192)])
+def test_lc_gemm_grouped_raster_exact(tk, M, N, K):
+    # >= 16 x 16 tiles: the grouped tile raster (8 M-tiles per group, a ragged last group, ragged M)
+    # must cover every tile once -- integer inputs, so the whole output is exact; and the fused
+    # launch (same raster) bit-identical to the original
+    A, B = synth.lc_gemm_inputs(M, N, K, seed=17, variant="int")
+    D = torch.zeros(M, N, device=dev())
+    f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), None, 0)
+    assert f.info().lc_tiles >= 256
+    tk.tacker_launch_original(tk.lc_gemm(t(A), t(B), D), None)
+    ref = A.astype(np.float64) @ B.astype(np.float64).T
+    assert np.array_equal(host(D).astype(np.float64), ref)
+    c = be_case(tk.BE_SGEMM, seed=3)
+    D1 = torch.zeros(M, N, device=dev())
+    c["reset"]()
+    tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D1), c["desc"], 16).launch()
+    assert host(D1).tobytes() == host(D).tobytes()
+
+
 def test_lc_gemm_f16_epilogue(tk):
     M, N, K = 200, 192, 128
     A, B = synth.lc_gemm_inputs(M, N, K, seed=9)
