@@ -278,7 +278,7 @@ tacker_status tacker_be_prefix_work(const tacker_be_desc *be, int64_t n_blocks, 
  *   warps [6, 6+warp_split) BE: block_ratio.be virtual blocks of 4 warps, each with its own
  *                          named barrier (bar.sync 1+j, 128; Fig. 9) and SMEM slice
  * warp_split  BE warps per CTA, a multiple of 4 in [4, 24] (0 = LC only; requires be NULL/NONE)
- * block_ratio.lc  LC accumulator pipelines per CTA (TMEM stages, 1, 2 or 4 with acc x BN <= 512; 0 = auto)
+ * block_ratio.lc  LC accumulator pipelines per CTA (TMEM stages, 1 or 2; 0 = auto)
  * block_ratio.be  BE virtual blocks per CTA = warp_split/4 (0 = auto)
  * LC is budgeted first (SMEM ring stages, TMEM columns), BE gets the rest (TC-first, §V-C).
  * Returns TACKER_ERESOURCE when the aggregate does not fit (232,448 B SMEM, 512 TMEM columns,

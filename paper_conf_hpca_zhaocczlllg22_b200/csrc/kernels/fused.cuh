@@ -21,12 +21,10 @@
 
 namespace tk {
 
-constexpr int kLcWarps = 6;        // fused CTAs: producer, MMA, 4 epilogue warps
-constexpr int kLcWarpsSolo = 10;   // LC-only CTAs: producer, MMA, 2 epilogue groups of 4 warps
+constexpr int kLcWarps = 6;
 constexpr int kBM = 128;   // UMMA M
 constexpr int kBK = 64;    // one 128-byte swizzle row of fp16
 constexpr int kUK = 16;    // UMMA K for kind::f16
-constexpr int kMaxAcc = 4;          // TMEM accumulator stages (tiles in flight between MMA and epilogue)
 constexpr uint32_t kLcEpiBar = 15;   // named barrier of the 4 LC epilogue warps (BE uses 1..14)
 
 struct LcParams {
@@ -47,19 +45,11 @@ struct LcParams {
                              // 16 B, loaded as 8 unswizzled 128 x 16 B boxes (K-major, no swizzle)
   int32_t conv_im2col;       // implicit conv through the TMA im2col mode: M-tile = 128 consecutive
                              // output pixels (n, p, q linear); else tp x tq windows of one image
-  int32_t halo_bres;         // halo mode with the whole filter resident in shared memory (one N tile): B
-                             // loaded once per CTA at b_res_off, chunk ((r S + s) c_blocks + cb) x BN x 128 B;
-                             // a ring stage holds only the input halo
   int32_t conv_halo;         // stride-1 conv, C % 64 == 0: M-tile = 16 x 8 output pixels; a k-step =
                              // (filter row r, channel block cb) loads ONE input halo of 16 x (8+S-1)
                              // pixels x 64 channels (SW128) and the S taps' weights, and issues S x 4
                              // MMAs whose A descriptors start s rows into the halo (SBO = (8+S-1) rows)
   uint32_t stage_a, stage_bytes;   // shared-memory bytes of a ring stage's A part and of the stage
-  // k-blocks per ring stage (plain GEMM / 1x1 / im2col modes; 1 elsewhere): a stage holds kps A
-  // k-blocks then kps B k-blocks and one full/empty handshake covers 4 kps MMAs -- the handshake
-  // (~370 cycles) otherwise bounds N <= 128 mainloops (4 MMAs of 32-64 cycles per k-block)
-  int32_t kps;
-  int32_t raster_g;          // > 1: grouped tile raster (tile_coords), plain GEMMs with many tiles
   // stride-2 conv with C = 8 (ResNet conv1, 7x7 over 3 channels padded to 8), "phase halo" mode:
   // M-tile = 16 x 8 output pixels; a stage holds the input halo split into the 4 parity phases
   // (even/odd rows x even/odd columns, TMA traversal stride 2), each [rows][cols] pixels of 16 B,
@@ -84,11 +74,6 @@ struct LcParams {
   // warp stages its 32 rows x 64 columns (SW128) in shared memory and one lane stores the box
   // through tmap_d -- full-line global writes instead of 16-byte row-strided stores
   int32_t tma_store;
-  // resident bias: the whole bias vector (tiles_n x BN floats, zero past N) is loaded into shared
-  // memory at bias_off (from the LC base) once per CTA, before the dependency wait (it is a
-  // constant), instead of staging one tile's BN values per tile (a global load and two epilogue
-  // barriers on every tile's critical path); 0 = per-tile staging
-  uint32_t bias_off;
   // diagnostics (TACKER_LC_DBG, never set in production): bit 0 = epilogue drains TMEM without
   // math or stores; bit 1 = no MMAs (the issuer only releases stages and signals the epilogue);
   // bit 2 = no TMA loads (the producer arrives on the full barriers without data)
@@ -114,14 +99,13 @@ struct alignas(64) FusedParams {
   int64_t be_offset;       // first original block (a slice [be_offset, be_offset + be_blocks))
   BeWork *work;            // device workspace for the BE ticket
   int32_t be_vb_per_cta;   // virtual blocks per CTA
-  int32_t lc_warps;        // 6 (one epilogue group), 10 (LC-only: two groups, one per TMEM accumulator stage) or 0
+  int32_t lc_warps;        // 6 or 0
   int32_t stages;          // SMEM ring depth
   int32_t acc_stages;      // TMEM accumulator buffers
   uint32_t tmem_cols;
   uint32_t lc_smem_bytes;  // ring + barriers, 1024-aligned start
   uint32_t be_smem_per_vb; // per-vblock slice (incl. 16 B ticket slot)
-  uint32_t epi_stage_off;  // TMA-store staging (4 warps x epi_bufs x 4 KB, 1024-aligned) from the LC base
-  int32_t epi_bufs;        // staging boxes per epilogue warp (2 or 4): stores in flight per warp
+  uint32_t epi_stage_off;  // TMA-store staging (4 warps x 2 x 4 KB, 1024-aligned) from the LC base
 };
 
 // diagnostics (TACKER_LC_DBG bit 3): per-CTA clock64 stamps of the first 16 work units of each LC
@@ -134,25 +118,35 @@ __device__ __forceinline__ void lc_stamp(const LcParams &L, int ev, int i) {
 }
 
 // diagnostics (TACKER_LC_DBG bit 4 = 16): per-launch %globaltimer stamps (ns, comparable across
-// SMs and launches) of the kernel-boundary cost, slot = dbg_id: [0] CTA 0 entry, [1] CTA 0 prologue
-// done, [2] CTA 0 producer's dependency wait returned, [3] CTA 0 first ring stage landed (MMA
-// warp), [4] ~(earliest CTA entry), [5] latest epilogue end, [6] latest CTA exit; read and cleared
-// by tacker_debug_lc_globaltimer
+// SMs and launches), slot = dbg_id: [0] CTA 0 entry, [1] CTA 0 prologue done, [2] CTA 0 producer's
+// dependency wait returned, [3] unused, [4] ~(earliest CTA entry), [5] latest epilogue end,
+// [6] latest CTA exit; read and cleared by tacker_debug_lc_globaltimer.  The recorder is out of
+// line and called only outside the roles' loops (the LC-only kernel's code size is what the
+// kernel-boundary cost of a query chain is sensitive to).
 __device__ unsigned long long g_lc_gt[256][8];
-__device__ __forceinline__ unsigned long long gtime() {
+#if TK_LC_GT
+static __device__ __noinline__ void lc_gt_record(int id, int slot, bool cta0_only) {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-__device__ __forceinline__ void lc_gt(const LcParams &L, int slot, bool cta0_only) {
-  if (!(L.dbg & 16)) return;
-  const unsigned long long t = gtime();
-  unsigned long long *g = &g_lc_gt[L.dbg_id & 255][slot];
+  unsigned long long *g = &g_lc_gt[id & 255][slot];
   if (cta0_only) {
     if (blockIdx.x == 0) *g = t;
   } else {
     atomicMax(g, slot == 4 ? ~t : t);
   }
+}
+#endif
+// Compiled in only with -DTK_LC_GT=1 (tools/gpu/lc_gaps.sh builds that variant): even never-taken
+// calls to the out-of-line recorder made the LC-only kernel 3 % slower in a query chain.
+#ifndef TK_LC_GT
+#define TK_LC_GT 0
+#endif
+__device__ __forceinline__ void lc_gt(const LcParams &L, int slot, bool cta0_only) {
+#if TK_LC_GT
+  if (L.dbg & 16) lc_gt_record(L.dbg_id, slot, cta0_only);
+#else
+  (void)L, (void)slot, (void)cta0_only;
+#endif
 }
 
 // ------------------------------------------------------------------------ LC roles
@@ -174,35 +168,11 @@ struct LcGemm {
   }
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages, uint32_t stage_bytes) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * stage_bytes);
-    // full[S], empty[S], tfull[4], tempty[4] (up to kMaxAcc TMEM accumulator stages), TMEM address,
-    // resident-weights barrier, then the per-tile bias slots (16-byte aligned)
-    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + kMaxAcc, reinterpret_cast<uint32_t *>(b + 2 * stages + 2 * kMaxAcc),
-                reinterpret_cast<float *>(b + 2 * stages + 2 * kMaxAcc + 2), b + 2 * stages + 2 * kMaxAcc + 1};
+    return Bars{b, b + stages, b + 2 * stages, b + 2 * stages + 2, reinterpret_cast<uint32_t *>(b + 2 * stages + 4),
+                reinterpret_cast<float *>(b + 2 * stages + 6), b + 2 * stages + 5};
   }
 
-  // resident bias (L.bias_off != 0): the 128 epilogue threads copy tiles_n x BN bias values
-  // (zero past N) into shared memory once; returns the shared base
-  // (each epilogue group writes the same values and meets on its own barrier `ebar`)
-  static __device__ __forceinline__ float *load_bias_resident(const LcParams &L, uint8_t *lc, uint32_t ebar) {
-    float *b = reinterpret_cast<float *>(lc + L.bias_off);
-    const int et = (int)threadIdx.x % 128;
-    for (int c = et; c < L.tiles_n * BN; c += 128) b[c] = c < L.N ? __ldg(L.bias + c) : 0.f;
-    named_bar_sync(ebar, 128);
-    return b;
-  }
   static __device__ __forceinline__ void tile_coords(const LcParams &L, int t, int &mt, int &nt) {
-    if (L.raster_g > 1) {
-      // grouped raster (large GEMMs): groups of raster_g M-tiles, M fastest inside a group, so a
-      // wave of CTAs covers raster_g x (grid / raster_g) tiles whose A rows and B columns stay in
-      // L2 (N-fastest order streamed all of B once per ~grid / tiles_n M-tiles: 7.8x the
-      // algorithmic DRAM bytes at 8192^3)
-      const int per = L.raster_g * L.tiles_n;
-      const int g = t / per, r = t - g * per;
-      const int m0 = g * L.raster_g, gm = min(L.raster_g, L.tiles_m - m0);
-      mt = m0 + r % gm;
-      nt = r / gm;
-      return;
-    }
     // N-tiles fastest: consecutive CTAs share the A rows (L2 reuse of the activation tile)
     mt = t / L.tiles_n;
     nt = t % L.tiles_n;
@@ -329,20 +299,15 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8 &&
-        !L.halo_bres) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
-      const int kps = L.kps, steps = (kb1 - kb0 + kps - 1) / kps;
-      const uint32_t kb_bytes = L.stage_bytes / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
-      pre = min(P.stages, steps);
+      pre = min(P.stages, kb1 - kb0);
       if (elect_one()) {
         for (int i = 0; i < pre; ++i) {
-          const int n = min(kps, kb1 - kb0 - i * kps);
-          mbar_arrive_expect_tx(&bb.full[i], n * kb_bytes);
-          for (int j = 0; j < n; ++j)
-            load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a + j * b_bytes, kb0 + i * kps + j, nt);
+          mbar_arrive_expect_tx(&bb.full[i], L.stage_bytes);
+          load_b(P, &bb.full[i], lc + i * L.stage_bytes + L.stage_a, kb0 + i, nt);
         }
       }
       __syncwarp();
@@ -365,24 +330,8 @@ struct LcGemm {
       }
       __syncwarp();
     }
-    if (L.halo_bres) {
-      // the whole filter (one N tile), once per CTA; constant weights load before the dependency
-      // wait (TACKER_LC_B_CONST), others after it
-      const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
-      if (!bconst) griddep_wait();
-      if (elect_one()) {
-        uint8_t *bres = lc + L.b_res_off;
-        const int chunks = L.r * L.s * L.c_blocks;
-        mbar_arrive_expect_tx(bb.bres, (uint32_t)chunks * BN * 128u);
-        for (int rs = 0; rs < L.r * L.s; ++rs)
-          for (int cb = 0; cb < L.c_blocks; ++cb)
-            tma_load_2d(&P.tmap_b, bb.bres, bres + (uint32_t)(rs * L.c_blocks + cb) * BN * 128u, rs * L.c + cb * kBK, 0);
-      }
-      __syncwarp();
-    }
     griddep_wait();
-    if (elect_one()) lc_gt(L, 2, true);
-    __syncwarp();
+    if (lane_id() == 0) lc_gt(L, 2, true);
     int stage = 0;
     uint32_t phase = 0;
     int ui = 0;
@@ -416,12 +365,9 @@ struct LcGemm {
         rr = rs / L.s;
         ss = rs - rr * L.s;
       }
-      const int kps = L.kps;
-      const uint32_t a_bytes = L.stage_a / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
-      for (int kb = kb0; kb < kb1; kb += kps) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         uint8_t *sa = lc + stage * L.stage_bytes;
         uint8_t *sb = sa + L.stage_a;
-        const int n = min(kps, kb1 - kb);   // k-blocks in this stage
         const bool first = pre > 0;   // first tile, stage == kb: B already in flight, its bytes expected
         if (first) --pre;
         else mbar_wait(&bb.empty[stage], phase ^ 1);
@@ -438,9 +384,7 @@ struct LcGemm {
             for (int ph = 0; ph < 4; ++ph)
               tma_load_4d(&P.tmap_a, &bb.full[stage], sa + ph * L.s2_phase_stride, 0, w0 + (ph & 1), h0 + (ph >> 1), img);
           } else if (L.conv_halo) {
-            if (L.halo_bres) {
-              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);   // the halo only (stage_bytes = stage_a)
-            } else if (!first) {
+            if (!first) {
               mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
               for (int t = 0; t < L.s; ++t)   // the filter row's S taps: K columns (rr S + t) C + 64 cb
                 tma_load_2d(&P.tmap_b, &bb.full[stage], sb + t * BN * 128, (rr * L.s + t) * L.c + cb * kBK, nt * BN);
@@ -448,43 +392,28 @@ struct LcGemm {
             tma_load_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc + rr, n0);
           } else if (walk) {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], n * (a_bytes + b_bytes));
-              for (int j = 0; j < n; ++j)   // K index rs*C + cb*64 = 64 kb
-                tma_load_2d(&P.tmap_b, &bb.full[stage], sb + j * b_bytes, (kb + j) * kBK, nt * BN);
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
+              tma_load_2d(&P.tmap_b, &bb.full[stage], sb, kb * kBK, nt * BN);   // K index rs*C + cb*64 = 64 kb
             }
-            int c2 = cb, s2 = ss, r2 = rr;
-            for (int j = 0; j < n; ++j) {
-              tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa + j * a_bytes, c2 * kBK, wc, hc, n0, (uint16_t)s2,
-                                 (uint16_t)r2);
-              if (++c2 == L.c_blocks) {
-                c2 = 0;
-                if (++s2 == L.s) {
-                  s2 = 0;
-                  ++r2;
-                }
-              }
-            }
+            tma_load_im2col_4d(&P.tmap_a, &bb.full[stage], sa, cb * kBK, wc, hc, n0, (uint16_t)ss, (uint16_t)rr);
           } else {
             if (!first) {
-              mbar_arrive_expect_tx(&bb.full[stage], n * (a_bytes + b_bytes));
-              for (int j = 0; j < n; ++j) load_b(P, &bb.full[stage], sb + j * b_bytes, kb + j, nt);
+              mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
+              load_b(P, &bb.full[stage], sb, kb, nt);
             }
-            for (int j = 0; j < n; ++j) load_a(P, &bb.full[stage], sa + j * a_bytes, kb + j, mt);
+            load_a(P, &bb.full[stage], sa, kb, mt);
           }
         }
         __syncwarp();
         if (L.conv_halo && ++cb == L.c_blocks) {
           cb = 0;
           ++rr;
-        } else if (walk) {
-          for (int j = 0; j < n; ++j)
-            if (++cb == L.c_blocks) {
-              cb = 0;
-              if (++ss == L.s) {
-                ss = 0;
-                ++rr;
-              }
-            }
+        } else if (walk && ++cb == L.c_blocks) {
+          cb = 0;
+          if (++ss == L.s) {
+            ss = 0;
+            ++rr;
+          }
         }
         if (++stage == P.stages) {
           stage = 0;
@@ -499,7 +428,7 @@ struct LcGemm {
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
     int ui = 0;
-    if (L.conv_s2c8 || L.halo_bres) mbar_wait(bb.bres, 0);   // resident weights landed
+    if (L.conv_s2c8) mbar_wait(bb.bres, 0);   // resident weights landed
     for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1;
       unit_coords(L, u, t, sp, kb0, kb1);
@@ -507,13 +436,9 @@ struct LcGemm {
       tc_fence_after();
       lc_stamp(L, 1, ui);
       const uint32_t d = tmem + acc * BN;
-      const int kps = L.kps;
-      const uint32_t a_bytes = L.stage_a / kps, b_bytes = (L.stage_bytes - L.stage_a) / kps;
-      for (int kb = kb0; kb < kb1; kb += kps) {
-        const int n = min(kps, kb1 - kb);
+      for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&bb.full[stage], phase);
         tc_fence_after();
-        if (ui == 0 && kb == kb0 && lane_id() == 0) lc_gt(L, 3, true);
         const uint32_t sa = smem_u32(lc + stage * L.stage_bytes);
         const uint32_t sb = sa + L.stage_a;
         if (elect_one()) {
@@ -530,13 +455,9 @@ struct LcGemm {
             // tap s of this filter row: A = the halo from row s, 8-row groups (one output row of 8
             // pixels each) (8 + S - 1) rows apart; B = the tap's BN x 64 weight slot
             const uint32_t sbo = (uint32_t)(8 + L.s - 1) * 128u;
-            // B of tap t: the stage's slot, or chunk ((r S + t) c_blocks + cb) of the resident filter
-            const int hcb = kb % L.c_blocks, hr = kb / L.c_blocks;
-            const uint32_t bres0 = smem_u32(lc + L.b_res_off) + (uint32_t)(hr * L.s * L.c_blocks + hcb) * BN * 128u;
             for (int t = 0; t < L.s; ++t) {
               const uint64_t da = umma_desc_sw128_sbo(sa + 128u * t, sbo);
-              const uint64_t db = umma_desc_sw128(L.halo_bres ? bres0 + (uint32_t)(t * L.c_blocks) * BN * 128u
-                                                              : sb + (uint32_t)t * BN * 128u);
+              const uint64_t db = umma_desc_sw128(sb + (uint32_t)t * BN * 128u);
 #pragma unroll
               for (int k = 0; k < kBK / kUK; ++k)
                 umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || t != 0 || k != 0));
@@ -547,12 +468,10 @@ struct LcGemm {
               umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
                        umma_desc_sw128(sb + k * kUK * 2), kIdesc, (kb != kb0 || k != 0));
           } else {
-            for (int j = 0; j < n; ++j) {
-              const uint64_t da = umma_desc_sw128(sa + j * a_bytes), db = umma_desc_sw128(sb + j * b_bytes);
+            const uint64_t da = umma_desc_sw128(sa), db = umma_desc_sw128(sb);
 #pragma unroll
-              for (int k = 0; k < kBK / kUK; ++k)   // K step of 16 fp16 = 32 B = +2 in the start-address field
-                umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || j != 0 || k != 0));
-            }
+            for (int k = 0; k < kBK / kUK; ++k)   // K step of 16 fp16 = 32 B = +2 in the start-address field
+              umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || k != 0));
           }
           umma_commit(&bb.empty[stage]);   // frees the ring slot when these MMAs retire
         }
@@ -587,28 +506,31 @@ struct LcGemm {
     int row0;              // 2-D: first GEMM row
     int q0, p0, img;       // 4-D
   };
-  template <bool BIAS, bool RELU>
   static __device__ __forceinline__ void epi_batch(const FusedParams &P, const uint32_t (&v)[64], uint32_t bias_s,
-                                                   uint8_t *stg, int &buf, int n0, BoxAt at, int lane) {
+                                                   bool bias, uint8_t *stg, int &buf, int n0, BoxAt at, int lane) {
     const LcParams &L = P.lc;
-    if (lane == 0) {   // this box's previous store has read it
-      if (P.epi_bufs == 4) bulk_wait_read<3>();
-      else bulk_wait_read<1>();
+    float b[64];
+    if (bias) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const float4 q = ld_shared_v4f(bias_s + 16 * i);
+        b[4 * i] = q.x;
+        b[4 * i + 1] = q.y;
+        b[4 * i + 2] = q.z;
+        b[4 * i + 3] = q.w;
+      }
     }
+    if (lane == 0) bulk_wait_read<1>();   // this box's previous store has read it
     __syncwarp();
     const uint32_t box = smem_u32(stg + buf * 4096) + lane * 128;
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
-      float f[8], b[8];
-      if (BIAS) {   // 8 bias values per group of 8 columns (broadcast LDS.128; 64 held at once spilled)
-        const float4 q0 = ld_shared_v4f(bias_s + 32 * j), q1 = ld_shared_v4f(bias_s + 32 * j + 16);
-        b[0] = q0.x, b[1] = q0.y, b[2] = q0.z, b[3] = q0.w, b[4] = q1.x, b[5] = q1.y, b[6] = q1.z, b[7] = q1.w;
-      }
+      float f[8];
 #pragma unroll
       for (int e = 0; e < 8; ++e) {
         f[e] = __uint_as_float(v[8 * j + e]);
-        if (BIAS) f[e] = __fadd_rn(f[e], b[e]);
-        if (RELU) f[e] = fmaxf(f[e], 0.f);
+        if (bias) f[e] = __fadd_rn(f[e], b[8 * j + e]);
+        if (L.epi & TACKER_EPI_RELU) f[e] = fmaxf(f[e], 0.f);
       }
       __align__(16) __half2 hv[4];
 #pragma unroll
@@ -622,7 +544,7 @@ struct LcGemm {
       else tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, at.row0);
       bulk_commit();
     }
-    buf = buf + 1 == P.epi_bufs ? 0 : buf + 1;
+    buf ^= 1;
   }
   static __device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
     tmem_ld_32x32b_x16(taddr, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
@@ -630,56 +552,34 @@ struct LcGemm {
     tmem_ld_32x32b_x16(taddr + 32, *reinterpret_cast<uint32_t(*)[16]>(&v[32]));
     tmem_ld_32x32b_x16(taddr + 48, *reinterpret_cast<uint32_t(*)[16]>(&v[48]));
   }
-  // Epilogue groups (LC-only plans): group g of ng drains the work units u = cta + (g + i ng) grid,
-  // i.e. with two groups and two TMEM accumulator stages group g owns stage g -- two tiles'
-  // epilogues run at once (one group's TMEM drain / conversion / store issue was the bound of the
-  // short-K convs); `ew` = the warp's index among all epilogue warps (its staging boxes)
   static __device__ __forceinline__ void epilogue_tma(const FusedParams &P, const Bars &bb, uint32_t tmem,
-                                                      uint8_t *lc, int grp, int ngrp, int ew) {
-    const LcParams &L = P.lc;
-    const bool bias = (L.epi & TACKER_EPI_BIAS) != 0, relu = (L.epi & TACKER_EPI_RELU) != 0;
-    if (bias && relu) epilogue_tma_t<true, true>(P, bb, tmem, lc, grp, ngrp, ew);
-    else if (bias) epilogue_tma_t<true, false>(P, bb, tmem, lc, grp, ngrp, ew);
-    else if (relu) epilogue_tma_t<false, true>(P, bb, tmem, lc, grp, ngrp, ew);
-    else epilogue_tma_t<false, false>(P, bb, tmem, lc, grp, ngrp, ew);
-  }
-  template <bool BIAS, bool RELU>
-  static __device__ __forceinline__ void epilogue_tma_t(const FusedParams &P, const Bars &bb, uint32_t tmem,
-                                                        uint8_t *lc, int grp, int ngrp, int ew) {
+                                                      uint8_t *lc) {
     static_assert(BN % 64 == 0, "TMA-store epilogue: 64-column batches");
     constexpr int NB = BN / 64;
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;
     const int lane = lane_id();
-    const uint32_t ebar = kLcEpiBar - (uint32_t)grp;
-    uint8_t *stg = lc + P.epi_stage_off + ew * P.epi_bufs * 4096;
-    const bool bias = BIAS;
-    const bool bias_res = bias && L.bias_off != 0;
-    const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
-    float *bias_all = bias_res && bconst ? load_bias_resident(L, lc, ebar) : nullptr;   // constant: before the wait
+    uint8_t *stg = lc + P.epi_stage_off + quarter * 8192;
+    const uint32_t bias_s = smem_u32(bb.bias);
     int buf = 0;
     griddep_wait();
-    if (bias_res && !bconst) bias_all = load_bias_resident(L, lc, ebar);
-    int acc = grp;
+    int acc = 0;
     uint32_t acc_phase = 0;
     int ui = 0;
-    for (int u = blockIdx.x + grp * gridDim.x; u < L.num_units; u += ngrp * gridDim.x, ++ui) {
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
       mbar_wait(&bb.tfull[acc], acc_phase);
       tc_fence_after();
-      if (quarter == 0 && lane == 0 && grp == 0) lc_stamp(L, 3, ui);
+      if (quarter == 0 && lane == 0) lc_stamp(L, 3, ui);
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
-      float *tb = bb.bias + grp * BN;   // per-tile staging (one BN slot per group)
-      uint32_t bias_s = smem_u32(tb);
-      if (bias_res) {
-        bias_s = smem_u32(bias_all + nt * BN);
-      } else if (bias) {
+      const bool bias = (L.epi & TACKER_EPI_BIAS) != 0;
+      if (bias) {
         const int et = (int)threadIdx.x % 128;
-        named_bar_sync(ebar, 128);
-        for (int c = et; c < BN; c += 128) tb[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
-        named_bar_sync(ebar, 128);
+        named_bar_sync(kLcEpiBar, 128);
+        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(kLcEpiBar, 128);
       }
       const bool skip = (L.dbg & 1) != 0;
       BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
@@ -696,33 +596,30 @@ struct LcGemm {
         if (b + 1 < NB) tmem_ld64(tbase + 64 * (b + 1), (b % 2) ? va : vb);
         const int n0 = nt * BN + 64 * b;
         if (n0 < L.N && !skip)
-          epi_batch<BIAS, RELU>(P, (b % 2) ? vb : va, bias_s + 256 * b, stg, buf, n0, at, lane);
+          epi_batch(P, (b % 2) ? vb : va, bias_s + 256 * b, bias, stg, buf, n0, at, lane);
       }
       tc_fence_before();
       mbar_arrive(&bb.tempty[acc]);
-      if (quarter == 0 && lane == 0 && grp == 0) lc_stamp(L, 4, ui);
-      for (acc += ngrp; acc >= P.acc_stages; acc -= P.acc_stages) acc_phase ^= 1;
+      if (quarter == 0 && lane == 0) lc_stamp(L, 4, ui);
+      if (++acc == P.acc_stages) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
     }
     if (lane == 0) bulk_wait<0>();            // every store performed before the CTA retires
     if (lane == 0) lc_gt(L, 5, false);
   }
 
   template <int EC>
-  static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem, uint8_t *lc,
-                                                  int grp, int ngrp) {
+  static __device__ __forceinline__ void epilogue(const FusedParams &P, const Bars &bb, uint32_t tmem) {
     static_assert(EC % 16 == 0 && BN % EC == 0, "EC: multiple of 16 dividing BN");
     const LcParams &L = P.lc;
     const int quarter = warp_id() & 3;          // TMEM lanes 32*quarter .. +31
     const int row_in_tile = quarter * 32 + lane_id();
-    const uint32_t ebar = kLcEpiBar - (uint32_t)grp;
-    const bool bias_res = (L.epi & TACKER_EPI_BIAS) && L.bias_off != 0;
-    const bool bconst = (L.epi & TACKER_LC_B_CONST) != 0;
-    float *bias_all = bias_res && bconst ? load_bias_resident(L, lc, ebar) : nullptr;   // constant: before the wait
     griddep_wait();                             // residual / D of earlier kernels
-    if (bias_res && !bconst) bias_all = load_bias_resident(L, lc, ebar);
-    int acc = grp;
+    int acc = 0;
     uint32_t acc_phase = 0;
-    for (int u = blockIdx.x + grp * gridDim.x; u < L.num_units; u += ngrp * gridDim.x) {
+    for (int u = blockIdx.x; u < L.num_units; u += gridDim.x) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -732,12 +629,11 @@ struct LcGemm {
       const uint32_t tbase = tmem + acc * BN + ((uint32_t)(quarter * 32) << 16);
       float *prow = L.splits > 1 ? L.part + ((size_t)u * kBM + row_in_tile) * BN : nullptr;
       const bool bias = !prow && (L.epi & TACKER_EPI_BIAS);
-      float *tbias = bias_res ? bias_all + nt * BN : bb.bias + grp * BN;
-      if (bias && !bias_res) {   // stage this tile's bias in shared memory (read as a broadcast per column)
+      if (bias) {   // stage this tile's bias in shared memory (read as a broadcast per column)
         const int et = (int)threadIdx.x % 128;
-        named_bar_sync(ebar, 128);                // the previous tile's readers are done
-        for (int c = et; c < BN; c += 128) tbias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
-        named_bar_sync(ebar, 128);
+        named_bar_sync(kLcEpiBar, 128);           // the previous tile's readers are done
+        for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
+        named_bar_sync(kLcEpiBar, 128);
       }
       const bool res = !prow && (L.epi & TACKER_EPI_RESIDUAL) && orow >= 0;
 #pragma unroll 1
@@ -768,8 +664,8 @@ struct LcGemm {
               for (int u = 0; u < 8; ++u) f[u] = __uint_as_float(v[j / 16][j % 16 + u]);
               __align__(16) float b8[8];
               if (bias) {   // shared-space loads (a generic pointer would compile to LD.E)
-                *reinterpret_cast<float4 *>(b8) = ld_shared_v4f(smem_u32(tbias + c0 + j));
-                *reinterpret_cast<float4 *>(b8 + 4) = ld_shared_v4f(smem_u32(tbias + c0 + j + 4));
+                *reinterpret_cast<float4 *>(b8) = ld_shared_v4f(smem_u32(bb.bias + c0 + j));
+                *reinterpret_cast<float4 *>(b8 + 4) = ld_shared_v4f(smem_u32(bb.bias + c0 + j + 4));
               }
               store8(L, orow, n0 + j, f, b8, rv[j / 8]);
             }
@@ -777,8 +673,11 @@ struct LcGemm {
       }
       tc_fence_before();
       mbar_arrive(&bb.tempty[acc]);
-      for (acc += ngrp; acc >= P.acc_stages; acc -= P.acc_stages) acc_phase ^= 1;
-      if (L.splits > 1) reduce_split(L, t, sp, mt, nt, ebar);
+      if (++acc == P.acc_stages) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+      if (L.splits > 1) reduce_split(L, t, sp, mt, nt);
     }
     if (lane_id() == 0) lc_gt(L, 5, false);
   }
@@ -786,18 +685,18 @@ struct LcGemm {
   // Split-K fixup of tile t by split sp (all splits of the tile run concurrently, one per CTA):
   // wait until every split has written its partial, then reduce elements [sp E/S, (sp+1) E/S) of
   // the tile (E = kBM x BN, in groups of 4 columns) over the splits in order 0..S-1 and store them.
-  static __device__ __forceinline__ void reduce_split(const LcParams &L, int t, int sp, int mt, int nt, uint32_t ebar) {
+  static __device__ __forceinline__ void reduce_split(const LcParams &L, int t, int sp, int mt, int nt) {
     const int S = L.splits;
     const int et = (int)threadIdx.x % 128;      // the 4 epilogue warps are 128 consecutive threads
     uint32_t *arrive = L.cnt + 2 * t, *finish = arrive + 1;
     __threadfence();                            // partial visible before the arrival
-    named_bar_sync(ebar, 128);
+    named_bar_sync(kLcEpiBar, 128);
     if (et == 0) {
       atomicAdd(arrive, 1u);
       while (ld_acquire_gpu(arrive) < (uint32_t)S) {
       }
     }
-    named_bar_sync(ebar, 128);
+    named_bar_sync(kLcEpiBar, 128);
     constexpr int G = BN / 8;                   // 8-column groups per row
     const int E = kBM * G;
     const float *base = L.part + (size_t)t * S * kBM * BN;
@@ -824,7 +723,7 @@ struct LcGemm {
                                                      : make_uint4(0, 0, 0, 0);
       store8(L, orow, n, f, bias, rv);
     }
-    named_bar_sync(ebar, 128);
+    named_bar_sync(kLcEpiBar, 128);
     if (et == 0 && atomicAdd(finish, 1u) == (uint32_t)S - 1) {   // last reducer: reset for the next launch
       *arrive = 0;
       *finish = 0;
@@ -936,7 +835,7 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 // warps) gives every warp up to 144, for bodies that spill at 64 (fft) and for wider LC
 // epilogue batches.  tacker_fuse picks the smallest class that holds the plan's warp split.
 template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND)>
-__global__ void __launch_bounds__(32 * ((BE_KIND == TACKER_BE_NONE ? kLcWarpsSolo : kLcWarps) + WMAX), 1)
+__global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();   // the next kernel on the stream may start its prologue
@@ -964,7 +863,7 @@ __global__ void __launch_bounds__(32 * ((BE_KIND == TACKER_BE_NONE ? kLcWarpsSol
         mbar_init(&bb.full[s], 1);
         mbar_init(&bb.empty[s], 1);
       }
-      for (int a = 0; a < kMaxAcc; ++a) {
+      for (int a = 0; a < 2; ++a) {
         mbar_init(&bb.tfull[a], 1);
         mbar_init(&bb.tempty[a], 4 * 32);
       }
@@ -985,13 +884,10 @@ __global__ void __launch_bounds__(32 * ((BE_KIND == TACKER_BE_NONE ? kLcWarpsSol
         LcGemm<BN>::producer(P, lc, bb);      // warp-wide loop, elected issue
       } else if (warp == 1) {
         LcGemm<BN>::mma(P, lc, bb, tmem);
+      } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
+        LcGemm<BN>::epilogue_tma(P, bb, tmem, lc);
       } else {
-        const int ew = warp - 2, grp = ew >> 2, ngrp = (P.lc_warps - 2) >> 2;   // epilogue group
-        if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store)
-          LcGemm<BN>::epilogue_tma(P, bb, tmem, lc, grp, ngrp, ew);
-        else
-          LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(
-              P, bb, tmem, lc, grp, ngrp);
+        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
       }
     }
   } else if constexpr (BE_KIND != TACKER_BE_NONE) {

@@ -80,7 +80,6 @@ static constexpr int kSmemCap = 232448;      // max dynamic SMEM per CTA on sm_1
 static constexpr int kTmemCols = 512;
 static constexpr int kMaxWarps = 32;
 static constexpr int kMinLcSmem = 120 * 1024;  // forces one LC CTA per SM (TMEM ownership)
-static constexpr uint32_t kLcHdr = 256 + 8 * 256;  // LC region after the ring: mbarriers + TMEM address, 2 x 256 bias floats
 
 // ============================================================================ BE helpers
 template <int K>
@@ -310,54 +309,6 @@ static int pick_tile_n(const tacker_lc_desc &d, const LcParams &L) {
   return 128;
 }
 
-static int epi_bufs_cfg() {   // TACKER_EPI_BUFS: 2 (default) or 4 TMA-store staging boxes per epilogue warp
-  static const int v = [] {
-    const char *e = getenv("TACKER_EPI_BUFS");
-    return e && atoi(e) == 4 ? 4 : 2;
-  }();
-  return v;
-}
-static int epi_groups_cfg() {   // TACKER_EPI_GROUPS: 1 / 2 forces the LC-only epilogue groups, 0 (default) = heuristic
-  static const int v = [] {
-    const char *e = getenv("TACKER_EPI_GROUPS");
-    const int g = e ? atoi(e) : 0;
-    return g == 1 || g == 2 ? g : 0;
-  }();
-  return v;
-}
-static int lc_kps() {
-  static const int v = [] {
-    const char *e = getenv("TACKER_KPS");
-    const int k = e ? atoi(e) : 2;
-    return k < 1 ? 1 : k > 4 ? 4 : k;
-  }();
-  return v;
-}
-static int lc_kps64() {   // BN = 64 override (0: TACKER_KPS); 3 measured best (b32 ResNet-50 query)
-  static const int v = [] {
-    const char *e = getenv("TACKER_KPS64");
-    const int k = e ? atoi(e) : 3;
-    return k < 0 ? 0 : k > 4 ? 4 : k;
-  }();
-  return v;
-}
-static int lc_kps_max_bn() {
-  static const int v = [] {
-    const char *e = getenv("TACKER_KPS_MAXBN");
-    return e ? atoi(e) : 128;
-  }();
-  return v;
-}
-
-// resident bias (TACKER_BIAS_RES=0 restores per-tile staging)
-static bool bias_resident_enabled() {
-  static const bool on = [] {
-    const char *e = getenv("TACKER_BIAS_RES");
-    return !(e && e[0] == '0');
-  }();
-  return on;
-}
-
 // TMA-store epilogue for eligible LC-only plans (TACKER_EPI_TMA=0 restores the register path)
 static bool tma_store_enabled() {
   static const bool on = [] {
@@ -397,36 +348,6 @@ static bool conv_halo_ok(const LcParams &L, int BN) {
          L.r == L.s && L.s <= 7 && 2 * L.pad == L.s - 1 && L.p >= 8 && L.q >= 8 && BN <= 128;
 }
 
-static int raster_cfg() {   // TACKER_RASTER: M-tiles per raster group of large GEMMs (0/1 = N-fastest order)
-  static const int v = [] {
-    const char *e = getenv("TACKER_RASTER");
-    return e ? atoi(e) : 8;
-  }();
-  return v;
-}
-static int fused_stages_cfg() {   // TACKER_FUSED_STAGES: deepest LC ring of a fused plan (2..4, default 4)
-  static const int v = [] {
-    const char *e = getenv("TACKER_FUSED_STAGES");
-    const int k = e ? atoi(e) : 4;
-    return k < 2 ? 2 : k > 4 ? 4 : k;
-  }();
-  return v;
-}
-static int acc_cfg() {   // TACKER_ACC: TMEM accumulator stages wanted for LC-only plans (2 or 4)
-  static const int v = [] {
-    const char *e = getenv("TACKER_ACC");
-    return e && atoi(e) == 4 ? 4 : 2;
-  }();
-  return v;
-}
-static bool halo_bres_enabled() {   // TACKER_HALO_BRES=0: halo plans reload the filter per k-step
-  static const bool on = [] {
-    const char *e = getenv("TACKER_HALO_BRES");
-    return !(e && e[0] == '0');
-  }();
-  return on;
-}
-
 // Phase-halo mode for stride-2 convs over 8 channels (ResNet-50 conv1: 7x7, 3 channels padded to
 // 8), N <= 64: replaces the explicit im2col + GEMM of §VIII-H.  TACKER_CONV_S2C8=0 disables it.
 static bool conv_s2c8_ok(const LcParams &L, int BN) {
@@ -440,7 +361,6 @@ static bool conv_s2c8_ok(const LcParams &L, int BN) {
 
 static void lc_tiles(LcParams &L, int BN) {
   L.tiles_n = (L.N + BN - 1) / BN;
-  L.kps = 1;
   L.stage_a = kBM * kBK * 2;
   L.stage_bytes = (uint32_t)(kBM + BN) * kBK * 2;
   if (conv_s2c8_ok(L, BN)) {
@@ -808,20 +728,6 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   lc_tiles(L, BN);
   if (!(lc->epi_flags & TACKER_LC_NO_SPLIT)) lc_split(L, sms);
   F.BN = BN;
-  // grouped raster for plain GEMMs whose B does not stay in L2 across an N-fastest sweep
-  L.raster_g = (lc->kind == TACKER_LC_GEMM_F16 && raster_cfg() > 1 && L.splits == 1 && L.tiles_m >= 2 * raster_cfg() &&
-                L.tiles_n >= 16)
-                   ? raster_cfg()
-                   : 0;
-  // two k-blocks per ring stage for LC-only plain-GEMM / 1x1 / im2col-mode plans with narrow tiles
-  // (fused.cuh LcParams::kps); TACKER_KPS=1 restores one, TACKER_KPS_MAXBN the widest tile using it
-  const int kps = BN == 64 && lc_kps64() > 0 ? lc_kps64() : lc_kps();
-  if (!has_be && kps > 1 && BN <= lc_kps_max_bn() && L.num_kb >= 2 && !L.conv_halo && !L.conv_s2c8 &&
-      !L.conv_c8 && (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col)) {
-    L.kps = kps;
-    L.stage_a *= (uint32_t)L.kps;
-    L.stage_bytes *= (uint32_t)L.kps;
-  }
 
   int64_t be_blocks = 0;
   int vb = 0;
@@ -837,15 +743,8 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     be_slice = (16 + be_smem_bytes(be->kind) + 127) & ~127u;
     F.P.be = *be;
   }
-  // TMEM accumulator stages: 2 by default; LC-only plans of narrow tiles take up to 4 (TACKER_ACC)
-  // so more tiles are in flight between the MMA warp and the epilogue (the commit -> epilogue ->
-  // tempty round trip per tile bounded the many-tile N = 64 convs)
-  int acc = ratio.lc ? ratio.lc : (2 * BN <= kTmemCols ? 2 : 1);
-  if (!ratio.lc && !has_be) {
-    const int want = acc_cfg();
-    while (acc < want && acc < kMaxAcc && 2 * acc * BN <= kTmemCols) acc *= 2;
-  }
-  if (acc < 1 || acc > kMaxAcc || acc * BN > kTmemCols)
+  const int acc = ratio.lc ? ratio.lc : (2 * BN <= kTmemCols ? 2 : 1);
+  if (acc < 1 || acc > 2 || acc * BN > kTmemCols)
     return set_error("block_ratio.lc (TMEM accumulator stages) %d does not fit %d columns", acc, kTmemCols), TACKER_ERESOURCE;
   uint32_t cols = 32;
   while (cols < (uint32_t)(acc * BN)) cols <<= 1;
@@ -856,43 +755,18 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
                 !(lc->epi_flags & TACKER_EPI_RESIDUAL) && L.splits == 1 && BN >= 64 && L.N >= 64 &&
                 (lc->kind == TACKER_LC_GEMM_F16 || L.conv_direct_gemm || L.conv_im2col || L.conv_halo ||
                  L.conv_s2c8);
-  // epilogue warps: LC-only plans with two TMEM accumulator stages run two epilogue groups (one per
-  // stage, fused.cuh epilogue_tma); fused CTAs keep one group of 4 (their warps go to the BE)
-  // when the epilogue work per CTA is large (units / SMs x BN >= 512 columns: the 1x1 convs with
-  // many short-K tiles measured faster; below it the larger staging costs ring stages)
-  const bool two_groups = !has_be && acc % 2 == 0 &&
-                          (epi_groups_cfg() == 2 ||
-                           (epi_groups_cfg() == 0 && (int64_t)L.num_units * BN >= 512LL * sms));
-  const int lc_warps = two_groups ? kLcWarpsSolo : kLcWarps;
-  const uint32_t epi_warps = (uint32_t)lc_warps - 2u;
-  // halo mode, LC-only, one N tile: the whole filter resident in shared memory (<= 96 KB), a ring
-  // stage then holds only the input halo (the B re-load per tile was half of the L2 -> SMEM bytes)
-  const uint32_t halo_bres_bytes = (uint32_t)L.r * L.s * L.c_blocks * BN * 128u;
-  if (!has_be && L.conv_halo && L.tiles_n == 1 && L.splits == 1 && halo_bres_enabled() && halo_bres_bytes <= 96u * 1024u) {
-    L.halo_bres = 1;
-    L.stage_bytes = L.stage_a;
-  }
-  const uint32_t res_bytes = L.conv_s2c8 ? 2u * L.s2_pairs * 1024u : L.halo_bres ? halo_bres_bytes : 0u;
-  const uint32_t epi_bufs = L.tma_store ? (uint32_t)epi_bufs_cfg() : 0u;   // staging boxes per epilogue warp
-  const uint32_t epi_bytes = (L.tma_store ? epi_warps * epi_bufs * 4096u + 1024u : 0u) +
-                             (res_bytes ? res_bytes + 1024u : 0u);   // + resident weights
+  const uint32_t epi_bytes = (L.tma_store ? 4u * 2u * 4096u + 1024u : 0u) +
+                             (L.conv_s2c8 ? 2u * L.s2_pairs * 1024u + 1024u : 0u);   // + resident weights
   L.dbg = lc_dbg_flags();
   // LC first (TC-first rule, §V-C): the deepest ring (<= 4 stages fused, <= 8 LC-only,
   // >= 2) that still leaves room for the requested BE virtual blocks.
   const uint32_t stage_bytes = L.stage_bytes;
-  // resident bias (fused.cuh LcParams::bias_off): tiles_n x BN floats, when at most 16 KB
-  const uint32_t bias_bytes = (lc->epi_flags & TACKER_EPI_BIAS) && bias_resident_enabled() &&
-                                      (uint32_t)L.tiles_n * BN * 4u <= 16384u
-                                  ? (uint32_t)L.tiles_n * BN * 4u
-                                  : 0u;
-  // mbarriers + TMEM address (256) + one tile's bias per epilogue group (2 x BN <= 256 floats) +
-  // staging + resident bias
-  const uint32_t bar_bytes = kLcHdr + epi_bytes + (bias_bytes ? bias_bytes + 16 : 0);
+  const uint32_t bar_bytes = 256 + 4 * 256 + epi_bytes;   // mbarriers + TMEM address + one tile's bias (BN <= 256) + staging
   const uint32_t be_total = (uint32_t)vb * be_slice;
   // LC-only launches take the deepest ring that fits (up to 8 stages: more TMA bytes in flight per
   // SM for the latency-bound implicit-GEMM loads); fused plans stop at 4 so the BE keeps L1
   int stages = 0;
-  for (int s = has_be ? fused_stages_cfg() : 8; s >= 2; --s) {
+  for (int s = has_be ? 4 : 8; s >= 2; --s) {
     const uint32_t need = 1024 + s * stage_bytes + bar_bytes + be_total;
     if (need <= (uint32_t)kSmemCap) {
       stages = s;
@@ -903,33 +777,23 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
     set_error("fused budget exceeds one SM: LC ring %u B x2 + BE %d x %u B > %d B", stage_bytes, vb, be_slice, kSmemCap);
     return TACKER_ERESOURCE;
   }
-  const int warps = lc_warps + warp_split;
+  const int warps = kLcWarps + warp_split;
   if (warps > kMaxWarps) return set_error("too many warps"), TACKER_ERESOURCE;
 
   F.P.stages = stages;
   F.P.acc_stages = acc;
   F.P.tmem_cols = cols;
   F.P.lc_smem_bytes = (stages * stage_bytes + bar_bytes + 127) & ~127u;
-  F.P.epi_bufs = (int32_t)epi_bufs;
-  F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + kLcHdr + 1023u) & ~1023u : 0u;
-  if (res_bytes) {
-    const uint32_t after = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
+  F.P.epi_stage_off = L.tma_store ? ((uint32_t)stages * stage_bytes + 256u + 4u * 256u + 1023u) & ~1023u : 0u;
+  if (L.conv_s2c8) {
+    const uint32_t after = L.tma_store ? F.P.epi_stage_off + 4u * 2u * 4096u : (uint32_t)stages * stage_bytes + 1280u;
     L.b_res_off = (after + 1023u) & ~1023u;
-  }
-  {   // resident bias after everything else of the LC region (16-aligned)
-    uint32_t end = L.tma_store ? F.P.epi_stage_off + epi_warps * epi_bufs * 4096u : (uint32_t)stages * stage_bytes + kLcHdr;
-    if (res_bytes) end = L.b_res_off + res_bytes;
-    L.bias_off = bias_bytes ? ((end + 15u) & ~15u) : 0u;
-    if (bias_bytes && L.bias_off + bias_bytes > F.P.lc_smem_bytes) {
-      set_error("internal: resident bias outside the LC region (%u + %u > %u)", L.bias_off, bias_bytes, F.P.lc_smem_bytes);
-      return TACKER_ERESOURCE;
-    }
   }
   F.P.be_smem_per_vb = be_slice;
   F.P.be_vb_per_cta = vb;
   F.P.be_blocks = be_blocks;
   F.P.be_offset = has_be ? be->block_offset : 0;
-  F.P.lc_warps = lc_warps;
+  F.P.lc_warps = kLcWarps;
   F.warp_split = warp_split;
   F.block = 32 * warps;
   F.smem = 1024 + F.P.lc_smem_bytes + be_total;

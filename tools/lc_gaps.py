@@ -3,6 +3,8 @@ before import) of one ResNet-50 query's convs launched back to back; prints per 
 from the previous kernel's last CTA exit to this kernel's CTA-0 entry, prologue, dependency-wait
 release, first stage landed, and its own span.
 
+  (the stamps are compiled in only with -DTK_LC_GT=1: python -m paper_conf_hpca_zhaocczlllg22_b200.build
+   --out variants/lib_gt.so -DTK_LC_GT=1, then TACKER_LIB=variants/lib_gt.so)
   TACKER_LC_DBG=16 python tools/lc_gaps.py [--batch 32] [--overlap 2]"""
 import argparse
 import json
