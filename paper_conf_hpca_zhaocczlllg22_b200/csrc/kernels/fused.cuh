@@ -150,8 +150,21 @@ __device__ __forceinline__ void lc_gt(const LcParams &L, int slot, bool cta0_onl
 }
 
 // ------------------------------------------------------------------------ LC roles
-template <int BN>
+// LC mode of an instantiation (MODE): 0 = any (decided at run time from LcParams: fused
+// kernels), else compiled for one mode only (LC-only kernels: each instantiation carries only its
+// mode's producer / MMA / epilogue code -- the kernel-switch cost of a query chain grows with the
+// instruction footprint)
+enum LcMode { kModeAny = 0, kModeGemm = 1, kModeIm2col = 2, kModeHalo = 3, kModeS2c8 = 4, kModeC8 = 5, kModeTiled = 6 };
+
+template <int BN, int MODE = kModeAny>
 struct LcGemm {
+  static constexpr bool kAny = MODE == kModeAny;
+  static __device__ __forceinline__ bool halo_(const LcParams &L) { return kAny ? L.conv_halo != 0 : MODE == kModeHalo; }
+  static __device__ __forceinline__ bool s2c8_(const LcParams &L) { return kAny ? L.conv_s2c8 != 0 : MODE == kModeS2c8; }
+  static __device__ __forceinline__ bool c8_(const LcParams &L) { return kAny ? L.conv_c8 != 0 : MODE == kModeC8; }
+  static __device__ __forceinline__ bool im2col_(const LcParams &L) {
+    return kAny ? L.conv_im2col != 0 : (MODE == kModeIm2col || MODE == kModeC8);
+  }
   static constexpr uint32_t kStageA = kBM * kBK * 2;
   static constexpr uint32_t kStageB = BN * kBK * 2;
   static constexpr uint32_t kStage = kStageA + kStageB;
@@ -164,7 +177,7 @@ struct LcGemm {
     uint64_t *bres;          // resident weights landed (conv_s2c8)
   };
   static __device__ __forceinline__ bool implicit_conv(const LcParams &L) {
-    return L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm;
+    return kAny ? (L.kind == TACKER_LC_CONV_F16 && !L.conv_direct_gemm) : MODE != kModeGemm;
   }
   static __device__ __forceinline__ Bars bars(uint8_t *lc, int stages, uint32_t stage_bytes) {
     uint64_t *b = reinterpret_cast<uint64_t *>(lc + stages * stage_bytes);
@@ -186,7 +199,7 @@ struct LcGemm {
   }
   // output row (GEMM row of D) of row r of M-tile mt, or -1 outside the problem
   static __device__ __forceinline__ int64_t out_row(const LcParams &L, int mt, int r) {
-    if (implicit_conv(L) && !L.conv_im2col) {
+    if (implicit_conv(L) && !im2col_(L)) {
       const int img = mt / (L.tiles_p * L.tiles_q);
       const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
       const int pp = pt * L.tp + r / L.tq, qq = qt * L.tq + r % L.tq;
@@ -231,12 +244,12 @@ struct LcGemm {
   // B (weights) k-block kb of N-tile nt
   static __device__ __forceinline__ void load_b(const FusedParams &P, uint64_t *bar, uint8_t *sb, int kb, int nt) {
     const LcParams &L = P.lc;
-    if (L.conv_halo) {
+    if (halo_(L)) {
       // k-step kb = (filter row r, channel block cb): the S taps' weight columns (r S + t) C + 64 cb
       const int cb = kb % L.c_blocks, r = kb / L.c_blocks;
       for (int t = 0; t < L.s; ++t)
         tma_load_2d(&P.tmap_b, bar, sb + t * BN * 128, (r * L.s + t) * L.c + cb * kBK, nt * BN);
-    } else if (implicit_conv(L) && L.conv_c8) {
+    } else if (implicit_conv(L) && c8_(L)) {
       tma_load_2d(&P.tmap_b, bar, sb, kb * kBK, nt * BN);   // K = R*S*8 linear (OOB tail zero-filled)
     } else if (implicit_conv(L)) {
       // filter viewed as [K, R*S*C]: k-block column = (rs*C + cb*64)
@@ -249,14 +262,14 @@ struct LcGemm {
   // A (activations) k-block kb of M-tile mt
   static __device__ __forceinline__ void load_a(const FusedParams &P, uint64_t *bar, uint8_t *sa, int kb, int mt) {
     const LcParams &L = P.lc;
-    if (L.conv_halo) {
+    if (halo_(L)) {
       // the input rows of filter row r for the tile's 16 output rows, 8 + S - 1 columns, 64 channels
       // (out-of-image rows / columns zero-filled = the padding)
       const int cb = kb % L.c_blocks, r = kb / L.c_blocks;
       const int img = mt / (L.tiles_p * L.tiles_q);
       const int pt = (mt / L.tiles_q) % L.tiles_p, qt = mt % L.tiles_q;
       tma_load_4d(&P.tmap_a, bar, sa, cb * kBK, qt * L.tq - L.pad, pt * L.tp - L.pad + r, img);
-    } else if (implicit_conv(L) && L.conv_c8) {
+    } else if (implicit_conv(L) && c8_(L)) {
       // k-block kb = filter taps 8 kb .. 8 kb + 7 (K index = tap * 8 + c); tap t lands at sa + 2 KB t
       // as 128 pixel rows of 16 B; taps past R*S reload tap 0 (their weights are the zero padding)
       const int pq = L.p * L.q, m0 = mt * kBM;
@@ -270,7 +283,7 @@ struct LcGemm {
         tma_load_im2col_4d(&P.tmap_a, bar, sa + t * kBM * 16, 0, q0 * L.stride - L.pad, p0 * L.stride - L.pad, n0,
                            (uint16_t)(tap % L.s), (uint16_t)(tap / L.s));
       }
-    } else if (implicit_conv(L) && L.conv_im2col) {
+    } else if (implicit_conv(L) && im2col_(L)) {
       // k-block -> (filter tap r,s ; channel block cb); A = 128 output pixels from m0 = 128 mt,
       // first pixel (n0, p0, q0) -> input corner (q0 stride - pad, p0 stride - pad), tap offset (s, r)
       const int cb = kb % L.c_blocks, rs = kb / L.c_blocks;
@@ -299,7 +312,7 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !L.conv_s2c8) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !s2c8_(L)) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -312,7 +325,7 @@ struct LcGemm {
       }
       __syncwarp();
     }
-    if (L.conv_s2c8) {
+    if (s2c8_(L)) {
       // resident weights: one 64 x 16-byte chunk per tap (TMA, before the dependency wait: weights
       // are constant), the padding chunk zeroed here (generic stores, then the async-proxy fence)
       uint8_t *bres = lc + L.b_res_off;
@@ -338,14 +351,14 @@ struct LcGemm {
     // im2col-mode implicit conv (C % 64 == 0): the k-block -> (channel block, filter tap) walk and
     // the tile's first output pixel are computed once per unit and advanced incrementally, so the
     // single producer thread does no integer division per k-block (it was the loop's bound)
-    const bool walk = implicit_conv(L) && L.conv_im2col && !L.conv_c8;
+    const bool walk = implicit_conv(L) && im2col_(L) && !c8_(L);
     for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, u, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
       lc_stamp(L, 0, ui);
       int wc = 0, hc = 0, n0 = 0, cb = 0, ss = 0, rr = 0;
-      if (L.conv_halo) {   // halo tile origin (input coordinates of output pixel (p0, q0) minus pad)
+      if (halo_(L)) {   // halo tile origin (input coordinates of output pixel (p0, q0) minus pad)
         n0 = mt / (L.tiles_p * L.tiles_q);
         const int rem = mt - n0 * L.tiles_p * L.tiles_q;
         const int pt = rem / L.tiles_q, qt = rem - pt * L.tiles_q;
@@ -374,7 +387,7 @@ struct LcGemm {
         if (elect_one()) {
           if (L.dbg & 4) {
             mbar_arrive(&bb.full[stage]);
-          } else if (L.conv_s2c8) {
+          } else if (s2c8_(L)) {
             // the 4 parity phases of the tile's input window (traversal stride 2, zero padding)
             const int img = mt / (L.tiles_p * L.tiles_q);
             const int rem = mt - img * L.tiles_p * L.tiles_q;
@@ -383,7 +396,7 @@ struct LcGemm {
             mbar_arrive_expect_tx(&bb.full[stage], 4u * L.s2_phase_bytes);
             for (int ph = 0; ph < 4; ++ph)
               tma_load_4d(&P.tmap_a, &bb.full[stage], sa + ph * L.s2_phase_stride, 0, w0 + (ph & 1), h0 + (ph >> 1), img);
-          } else if (L.conv_halo) {
+          } else if (halo_(L)) {
             if (!first) {
               mbar_arrive_expect_tx(&bb.full[stage], L.stage_bytes);
               for (int t = 0; t < L.s; ++t)   // the filter row's S taps: K columns (rr S + t) C + 64 cb
@@ -405,7 +418,7 @@ struct LcGemm {
           }
         }
         __syncwarp();
-        if (L.conv_halo && ++cb == L.c_blocks) {
+        if (halo_(L) && ++cb == L.c_blocks) {
           cb = 0;
           ++rr;
         } else if (walk && ++cb == L.c_blocks) {
@@ -428,7 +441,7 @@ struct LcGemm {
     int stage = 0, acc = 0;
     uint32_t phase = 0, acc_phase = 0;
     int ui = 0;
-    if (L.conv_s2c8) mbar_wait(bb.bres, 0);   // resident weights landed
+    if (s2c8_(L)) mbar_wait(bb.bres, 0);   // resident weights landed
     for (int u = blockIdx.x; u < L.num_units; u += gridDim.x, ++ui) {
       int t, sp, kb0, kb1;
       unit_coords(L, u, t, sp, kb0, kb1);
@@ -444,14 +457,14 @@ struct LcGemm {
         if (elect_one()) {
           if (L.dbg & 2) {
             // diagnostics: no MMA
-          } else if (L.conv_s2c8) {
+          } else if (s2c8_(L)) {
             // K = 16 per MMA = the tap pair (t0, t1): A core matrices at a_off and a_off + lbo, 8-row
             // groups (output rows) s2_sbo apart; B = chunks 2u, 2u+1 of the resident weights
             const uint32_t bres = smem_u32(lc + L.b_res_off);
             for (int pu = 0; pu < L.s2_pairs; ++pu)
               umma_f16(d, umma_desc_kmajor_noswz(sa + L.s2_a_off[pu], L.s2_a_lbo[pu], L.s2_sbo),
                        umma_desc_kmajor_noswz(bres + pu * 2048u, 1024u, 128u), kIdesc, pu != 0);
-          } else if (L.conv_halo) {
+          } else if (halo_(L)) {
             // tap s of this filter row: A = the halo from row s, 8-row groups (one output row of 8
             // pixels each) (8 + S - 1) rows apart; B = the tap's BN x 64 weight slot
             const uint32_t sbo = (uint32_t)(8 + L.s - 1) * 128u;
@@ -462,7 +475,7 @@ struct LcGemm {
               for (int k = 0; k < kBK / kUK; ++k)
                 umma_f16(d, da + 2 * k, db + 2 * k, kIdesc, (kb != kb0 || t != 0 || k != 0));
             }
-          } else if (L.conv_c8) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
+          } else if (c8_(L)) {   // A: 8 tap boxes of 128 x 16 B; K = 16 spans taps 2k, 2k+1 (LBO = one box)
 #pragma unroll
             for (int k = 0; k < kBK / kUK; ++k)
               umma_f16(d, umma_desc_kmajor_noswz(sa + 2 * k * kBM * 16, kBM * 16, 128),
@@ -540,7 +553,7 @@ struct LcGemm {
     fence_proxy_async();                  // generic-proxy writes visible to the TMA unit
     __syncwarp();
     if (lane == 0) {
-      if (L.conv_halo || L.conv_s2c8) tma_store_4d(&P.tmap_d, stg + buf * 4096, n0, at.q0, at.p0, at.img);
+      if (halo_(L) || s2c8_(L)) tma_store_4d(&P.tmap_d, stg + buf * 4096, n0, at.q0, at.p0, at.img);
       else tma_store_2d(&P.tmap_d, stg + buf * 4096, n0, at.row0);
       bulk_commit();
     }
@@ -583,7 +596,7 @@ struct LcGemm {
       }
       const bool skip = (L.dbg & 1) != 0;
       BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
-      if (L.conv_halo || L.conv_s2c8) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
+      if (halo_(L) || s2c8_(L)) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
         at.img = mt / (L.tiles_p * L.tiles_q);
         at.p0 = ((mt / L.tiles_q) % L.tiles_p) * L.tp + 4 * quarter;
         at.q0 = (mt % L.tiles_q) * L.tq;
@@ -834,9 +847,10 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 // be_max_warps) holds 6 + 24 warps at 64 registers; the register-rich class (WMAX = 8, 6 + 8
 // warps) gives every warp up to 144, for bodies that spill at 64 (fft) and for wider LC
 // epilogue batches.  tacker_fuse picks the smallest class that holds the plan's warp split.
-template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND)>
+template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND), int MODE = kModeAny>
 __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
+  using LC = LcGemm<BN, MODE>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();   // the next kernel on the stream may start its prologue
   // 1024-aligned LC base by pointer arithmetic on the shared array (an integer round trip would
@@ -853,9 +867,9 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     lc_gt(P.lc, 0, true);
     lc_gt(P.lc, 4, false);
   }
-  typename LcGemm<BN>::Bars bb{};
+  typename LC::Bars bb{};
   if (P.lc_warps > 0) {
-    bb = LcGemm<BN>::bars(lc, P.stages, P.lc.stage_bytes);
+    bb = LC::bars(lc, P.stages, P.lc.stage_bytes);
     if (warp == 0 && lane_id() == 0) {
       tma_prefetch_desc(&P.tmap_a);
       tma_prefetch_desc(&P.tmap_b);
@@ -881,13 +895,13 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     if (has_lc) {
       const uint32_t tmem = *bb.tmem_holder;
       if (warp == 0) {
-        LcGemm<BN>::producer(P, lc, bb);      // warp-wide loop, elected issue
+        LC::producer(P, lc, bb);      // warp-wide loop, elected issue
       } else if (warp == 1) {
-        LcGemm<BN>::mma(P, lc, bb, tmem);
+        LC::mma(P, lc, bb, tmem);
       } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
-        LcGemm<BN>::epilogue_tma(P, bb, tmem, lc);
+        LC::epilogue_tma(P, bb, tmem, lc);
       } else {
-        LcGemm<BN>::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
+        LC::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
       }
     }
   } else if constexpr (BE_KIND != TACKER_BE_NONE) {
