@@ -847,7 +847,9 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 // be_max_warps) holds 6 + 24 warps at 64 registers; the register-rich class (WMAX = 8, 6 + 8
 // warps) gives every warp up to 144, for bodies that spill at 64 (fft) and for wider LC
 // epilogue batches.  tacker_fuse picks the smallest class that holds the plan's warp split.
-template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND), int MODE = kModeAny>
+// EPI (LC-only kernels): 0 = epilogue chosen at run time, 1 = TMA-store epilogue only, 2 = register
+// epilogue (residual / split-K / fp32) only -- like MODE, one path's code per instantiation
+template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND), int MODE = kModeAny, int EPI = 0>
 __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
   using LC = LcGemm<BN, MODE>;
@@ -898,9 +900,9 @@ __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
         LC::producer(P, lc, bb);      // warp-wide loop, elected issue
       } else if (warp == 1) {
         LC::mma(P, lc, bb, tmem);
-      } else if (BE_KIND == TACKER_BE_NONE && BN >= 64 && P.lc.tma_store) {
+      } else if (EPI != 2 && BE_KIND == TACKER_BE_NONE && BN >= 64 && (EPI == 1 || P.lc.tma_store)) {
         LC::epilogue_tma(P, bb, tmem, lc);
-      } else {
+      } else if constexpr (EPI != 1) {
         LC::template epilogue<(BE_KIND == TACKER_BE_NONE && BN >= 64) ? 64 : (WMAX <= 8 && BN >= 32) ? 32 : 16>(P, bb, tmem);
       }
     }

@@ -18,6 +18,9 @@ bool pair_opportune(const std::string &key, double *r);
 // register-rich fused instantiations (fused_rich.cu): fused_kernel<BN, kind, 8> or nullptr
 void *pick_fused_rich(int BN, int be_kind);
 
+// LC-only kernels per (BN, LC mode, epilogue 1 = TMA store / 2 = register) (fused_lc.cu) or nullptr
+void *pick_lc_only_kernel(int BN, int mode, int epi);
+
 // kind names
 const char *be_kind_name(int kind);
 

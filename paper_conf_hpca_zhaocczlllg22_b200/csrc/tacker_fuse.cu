@@ -636,29 +636,14 @@ static bool rich_class_enabled() {
   }();
   return on;
 }
-// LC-only kernels compiled for one LC mode each (fused.cuh LcMode): only that mode's code
-template <int BN>
-static KernelFn lc_only_fn(int mode) {
-  switch (mode) {
-    case kModeGemm: return fused_kernel<BN, TACKER_BE_NONE, 0, kModeGemm>;
-    case kModeIm2col: return fused_kernel<BN, TACKER_BE_NONE, 0, kModeIm2col>;
-    case kModeHalo: return BN <= 128 ? fused_kernel<BN, TACKER_BE_NONE, 0, kModeHalo> : nullptr;
-    case kModeS2c8: return BN == 64 ? fused_kernel<BN, TACKER_BE_NONE, 0, kModeS2c8> : nullptr;
-    case kModeC8: return fused_kernel<BN, TACKER_BE_NONE, 0, kModeC8>;
-    case kModeTiled: return fused_kernel<BN, TACKER_BE_NONE, 0, kModeTiled>;
-    default: return nullptr;
-  }
-}
-static KernelFn pick_lc_only(int BN, int mode) {
+// LC-only kernels compiled for one LC mode and epilogue each (fused_lc.cu)
+static KernelFn pick_lc_only(int BN, int mode, int epi) {
   static const bool on = [] {   // TACKER_LC_MODE_KERNELS=0: the run-time-mode kernel
     const char *e = getenv("TACKER_LC_MODE_KERNELS");
     return !(e && e[0] == '0');
   }();
   if (!on) return nullptr;
-  if (BN == 64) return lc_only_fn<64>(mode);
-  if (BN == 128) return lc_only_fn<128>(mode);
-  if (BN == 256) return lc_only_fn<256>(mode);
-  return nullptr;
+  return reinterpret_cast<KernelFn>(pick_lc_only_kernel(BN, mode, epi));
 }
 static int lc_mode_of(const LcParams &L) {
   if (L.kind != TACKER_LC_CONV_F16 || L.conv_direct_gemm) return kModeGemm;
@@ -839,7 +824,7 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   // 128 registers per thread) where one is compiled; wider plans the default class (64)
   F.fn = nullptr;
   if (has_be && warp_split <= 8 && rich_class_enabled()) F.fn = reinterpret_cast<KernelFn>(pick_fused_rich(BN, be->kind));
-  if (!F.fn && !has_be) F.fn = pick_lc_only(BN, lc_mode_of(L));
+  if (!F.fn && !has_be) F.fn = pick_lc_only(BN, lc_mode_of(L), L.tma_store && BN >= 64 ? 1 : 2);
   if (!F.fn) F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
   if (!F.fn) return set_error("no kernel instantiation for BN=%d BE=%d", BN, has_be ? be->kind : 0), TACKER_EUNSUPPORTED;
 
