@@ -1,6 +1,6 @@
 # round-2b final capture: default bench (K = 100), reference arm, launch list of the timed region,
 # per-launch DRAM traffic of one b32 LC query, ncu --set full of the dominant LC conv class
-D=gpurun_out/r02b_final
+D=gpurun_out/r02c_final
 mkdir -p $D
 timeout 1500 python bench.py > $D/bench_default.json 2> $D/bench_default.err
 timeout 600 python bench.py --impl reference --steps 20 --warmup 5 > $D/bench_reference.json 2> $D/bench_reference.err
