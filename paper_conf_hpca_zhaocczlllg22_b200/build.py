@@ -12,7 +12,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libtacker.so")
-SOURCES = ["tacker_fuse.cu", "fused_rich.cu", "fused_lc.cu", "predictor.cpp", "manager.cpp"]
+SOURCES = ["tacker_fuse.cu", "fused_rich.cu", "fused_lc.cu", "fused_mode.cu", "predictor.cpp", "manager.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
          "-Xcompiler", "-fPIC", "-diag-suppress", "1886",

@@ -21,6 +21,9 @@ void *pick_fused_rich(int BN, int be_kind);
 // LC-only kernels per (BN, LC mode, epilogue 1 = TMA store / 2 = register) (fused_lc.cu) or nullptr
 void *pick_lc_only_kernel(int BN, int mode, int epi);
 
+// default-class fused kernels per (BN, BE kind, LC mode) for the bench's kinds (fused_mode.cu) or nullptr
+void *pick_fused_mode_kernel(int BN, int be_kind, int mode);
+
 // kind names
 const char *be_kind_name(int kind);
 

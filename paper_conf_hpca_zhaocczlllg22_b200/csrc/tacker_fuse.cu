@@ -637,12 +637,15 @@ static bool rich_class_enabled() {
   return on;
 }
 // LC-only kernels compiled for one LC mode and epilogue each (fused_lc.cu)
-static KernelFn pick_lc_only(int BN, int mode, int epi) {
-  static const bool on = [] {   // TACKER_LC_MODE_KERNELS=0: the run-time-mode kernel
+static bool lc_mode_kernels_on() {   // TACKER_LC_MODE_KERNELS=0: the run-time-mode kernels
+  static const bool on = [] {
     const char *e = getenv("TACKER_LC_MODE_KERNELS");
     return !(e && e[0] == '0');
   }();
-  if (!on) return nullptr;
+  return on;
+}
+static KernelFn pick_lc_only(int BN, int mode, int epi) {
+  if (!lc_mode_kernels_on()) return nullptr;
   return reinterpret_cast<KernelFn>(pick_lc_only_kernel(BN, mode, epi));
 }
 static int lc_mode_of(const LcParams &L) {
@@ -825,6 +828,8 @@ static tacker_status plan(const tacker_lc_desc *lc, const tacker_be_desc *be, in
   F.fn = nullptr;
   if (has_be && warp_split <= 8 && rich_class_enabled()) F.fn = reinterpret_cast<KernelFn>(pick_fused_rich(BN, be->kind));
   if (!F.fn && !has_be) F.fn = pick_lc_only(BN, lc_mode_of(L), L.tma_store && BN >= 64 ? 1 : 2);
+  if (!F.fn && has_be && lc_mode_kernels_on())   // default register class, compiled per LC mode
+    F.fn = reinterpret_cast<KernelFn>(pick_fused_mode_kernel(BN, be->kind, lc_mode_of(L)));
   if (!F.fn) F.fn = pick_fused(BN, has_be ? be->kind : TACKER_BE_NONE);
   if (!F.fn) return set_error("no kernel instantiation for BN=%d BE=%d", BN, has_be ? be->kind : 0), TACKER_EUNSUPPORTED;
 
