@@ -156,9 +156,12 @@ __device__ __forceinline__ void lc_gt(const LcParams &L, int slot, bool cta0_onl
 // instruction footprint)
 enum LcMode { kModeAny = 0, kModeGemm = 1, kModeIm2col = 2, kModeHalo = 3, kModeS2c8 = 4, kModeC8 = 5, kModeTiled = 6 };
 
-template <int BN, int MODE = kModeAny>
+// EPI (LC-only kernels, see fused_kernel): 1 = TMA-store epilogue (never split-K), 2 = register
+// epilogue, 0 = decided at run time
+template <int BN, int MODE = kModeAny, int EPI = 0>
 struct LcGemm {
   static constexpr bool kAny = MODE == kModeAny;
+  static constexpr bool kNoSplit = EPI == 1;   // TMA-store plans are never split-K
   static __device__ __forceinline__ bool halo_(const LcParams &L) { return kAny ? L.conv_halo != 0 : MODE == kModeHalo; }
   static __device__ __forceinline__ bool s2c8_(const LcParams &L) { return kAny ? L.conv_s2c8 != 0 : MODE == kModeS2c8; }
   static __device__ __forceinline__ bool c8_(const LcParams &L) { return kAny ? L.conv_c8 != 0 : MODE == kModeC8; }
@@ -192,6 +195,13 @@ struct LcGemm {
   }
   // work unit -> tile, split and its k-block range
   static __device__ __forceinline__ void unit_coords(const LcParams &L, int u, int &t, int &sp, int &kb0, int &kb1) {
+    if constexpr (kNoSplit) {   // one unit per tile: no division in the roles' code
+      t = u;
+      sp = 0;
+      kb0 = 0;
+      kb1 = L.num_kb;
+      return;
+    }
     t = u / L.splits;
     sp = u % L.splits;
     kb0 = sp * L.kb_per_split;
@@ -852,7 +862,7 @@ __device__ __forceinline__ void be_ptb_loop(const FusedParams &P, uint8_t *be_sm
 template <int BN, int BE_KIND, int WMAX = be_max_warps(BE_KIND), int MODE = kModeAny, int EPI = 0>
 __global__ void __launch_bounds__(32 * (kLcWarps + WMAX), 1)
     fused_kernel(const __grid_constant__ FusedParams P) {
-  using LC = LcGemm<BN, MODE>;
+  using LC = LcGemm<BN, MODE, EPI>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   griddep_launch_dependents();   // the next kernel on the stream may start its prologue
   // 1024-aligned LC base by pointer arithmetic on the shared array (an integer round trip would
