@@ -195,7 +195,7 @@ struct LcGemm {
   }
   // work unit -> tile, split and its k-block range
   static __device__ __forceinline__ void unit_coords(const LcParams &L, int u, int &t, int &sp, int &kb0, int &kb1) {
-    if constexpr (kNoSplit) {   // one unit per tile: no division in the roles' code
+    if (kNoSplit || L.splits == 1) {   // one unit per tile: no division on the roles' critical path
       t = u;
       sp = 0;
       kb0 = 0;
