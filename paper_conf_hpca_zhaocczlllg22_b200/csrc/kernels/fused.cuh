@@ -113,8 +113,16 @@ struct alignas(64) FusedParams {
 // [3] epilogue start (tfull seen), [4] epilogue end (tempty arrive); read by
 // tacker_debug_lc_timestamps
 __device__ unsigned long long g_lc_ts[160][5][16];
+// The TACKER_LC_DBG switches (bits 0-3: skip epilogue math / MMAs / TMA loads, clock64 stamps) are
+// compiled in only with -DTK_LC_DIAG=1 (the decomposition tools build that variant): in production
+// builds the roles' loops carry no diagnostic branches (the LC chain is sensitive to the roles'
+// instruction footprint).
+#ifndef TK_LC_DIAG
+#define TK_LC_DIAG 0
+#endif
+__device__ __forceinline__ int lc_dbg(const LcParams &L) { return TK_LC_DIAG ? L.dbg : 0; }
 __device__ __forceinline__ void lc_stamp(const LcParams &L, int ev, int i) {
-  if ((L.dbg & 8) && i < 16 && blockIdx.x < 160) g_lc_ts[blockIdx.x][ev][i] = clock64();
+  if ((lc_dbg(L) & 8) && i < 16 && blockIdx.x < 160) g_lc_ts[blockIdx.x][ev][i] = clock64();
 }
 
 // diagnostics (TACKER_LC_DBG bit 4 = 16): per-launch %globaltimer stamps (ns, comparable across
@@ -322,7 +330,7 @@ struct LcGemm {
     // Weights do not depend on the stream predecessor (TACKER_LC_B_CONST): the first ring's worth
     // of B k-blocks is requested before the dependency wait, overlapping the previous kernel.
     int pre = 0;
-    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(L.dbg & 4) && !s2c8_(L)) {
+    if ((L.epi & TACKER_LC_B_CONST) && (int)blockIdx.x < L.num_units && !(lc_dbg(L) & 4) && !s2c8_(L)) {
       int t, sp, kb0, kb1, mt, nt;
       unit_coords(L, blockIdx.x, t, sp, kb0, kb1);
       tile_coords(L, t, mt, nt);
@@ -395,7 +403,7 @@ struct LcGemm {
         if (first) --pre;
         else mbar_wait(&bb.empty[stage], phase ^ 1);
         if (elect_one()) {
-          if (L.dbg & 4) {
+          if (lc_dbg(L) & 4) {
             mbar_arrive(&bb.full[stage]);
           } else if (s2c8_(L)) {
             // the 4 parity phases of the tile's input window (traversal stride 2, zero padding)
@@ -465,7 +473,7 @@ struct LcGemm {
         const uint32_t sa = smem_u32(lc + stage * L.stage_bytes);
         const uint32_t sb = sa + L.stage_a;
         if (elect_one()) {
-          if (L.dbg & 2) {
+          if (lc_dbg(L) & 2) {
             // diagnostics: no MMA
           } else if (s2c8_(L)) {
             // K = 16 per MMA = the tap pair (t0, t1): A core matrices at a_off and a_off + lbo, 8-row
@@ -604,7 +612,7 @@ struct LcGemm {
         for (int c = et; c < BN; c += 128) bb.bias[c] = nt * BN + c < L.N ? __ldg(L.bias + nt * BN + c) : 0.f;
         named_bar_sync(kLcEpiBar, 128);
       }
-      const bool skip = (L.dbg & 1) != 0;
+      const bool skip = (lc_dbg(L) & 1) != 0;
       BoxAt at{mt * kBM + quarter * 32, 0, 0, 0};
       if (halo_(L) || s2c8_(L)) {   // tile = 16 output rows x 8 columns; this warp's TMEM lanes = rows 4 quarter ..
         at.img = mt / (L.tiles_p * L.tiles_q);
@@ -671,7 +679,7 @@ struct LcGemm {
           rv[g] = (res && n0 + 8 * g < L.N) ? *reinterpret_cast<const uint4 *>(L.residual + orow * L.N + n0 + 8 * g)
                                             : make_uint4(0, 0, 0, 0);
         tmem_ld_wait();
-        if (orow < 0 || n0 >= L.N || (L.dbg & 1)) continue;
+        if (orow < 0 || n0 >= L.N || (lc_dbg(L) & 1)) continue;
         if (prow) {   // split-K partial, fp32
 #pragma unroll
           for (int j = 0; j < EC; j += 4)

@@ -1,5 +1,6 @@
 """Per-role timeline of one LC conv launch (TACKER_LC_DBG must include bit 3, set before import):
-clock64 stamps of the producer / MMA / epilogue per work unit on a few CTAs, as cycles from the
+clock64 stamps of the producer / MMA / epilogue per work unit on a few CTAs (a -DTK_LC_DIAG=1 build via
+TACKER_LIB: production kernels carry no diagnostics), as cycles from the
 first producer stamp.   TACKER_LC_DBG=8 python tools/lc_timeline.py --bn 64 layer1.0.conv2"""
 import argparse
 import os
