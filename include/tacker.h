@@ -350,10 +350,13 @@ tacker_status tacker_blacklist(const char *be_key, int32_t op, int32_t *listed);
 tacker_status tacker_blacklist_clear(void);
 
 /* Diagnostics: copies the LC role clock64 stamps recorded by plans built with TACKER_LC_DBG bit 3
- * ([160 CTAs][5 events][16 work units], see fused.cuh) into out (>= 12800 slots). */
+ * ([160 CTAs][5 events][16 work units], see fused.cuh) into out (>= 12800 slots).  The stamps (and
+ * the TACKER_LC_DBG skip switches) exist only in a library built with -DTK_LC_DIAG=1; production
+ * builds record nothing (zeros). */
 tacker_status tacker_debug_lc_timestamps(uint64_t *out, int64_t n);
 /* Diagnostics: synchronises the device, copies the per-launch %globaltimer stamps (ns) recorded by
- * plans built with TACKER_LC_DBG bit 4 (value 16) into out ([256 launch slots][8], >= 2048 slots;
+ * plans built with TACKER_LC_DBG bit 4 (value 16) in a library built with -DTK_LC_GT=1 (zeros
+ * otherwise) into out ([256 launch slots][8], >= 2048 slots;
  * slot layout in fused.cuh g_lc_gt), clears them and the slot counter; *next_slot (nullable) = the
  * number of launches recorded since the last call (mod 256). */
 tacker_status tacker_debug_lc_globaltimer(uint64_t *out, int64_t n, int32_t *next_slot);
