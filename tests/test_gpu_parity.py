@@ -43,10 +43,10 @@ def test_lc_gemm_exact_variants(tk, variant):
 
 
 @pytest.mark.parametrize("M,N,K", [(2304, 2176, 128), (4096 + 200, 2048, 192)])
-def test_lc_gemm_grouped_raster_exact(tk, M, N, K):
-    # >= 16 x 16 tiles: the grouped tile raster (8 M-tiles per group, a ragged last group, ragged M)
-    # must cover every tile once -- integer inputs, so the whole output is exact; and the fused
-    # launch (same raster) bit-identical to the original
+def test_lc_gemm_many_tiles_exact(tk, M, N, K):
+    # >= 256 tiles over the persistent grid (several tiles per CTA, ragged M): every tile covered
+    # once -- integer inputs, so the whole output is exact; and the fused launch bit-identical to
+    # the original (the mode-specialised LC-only kernel vs the run-time-mode fused kernel)
     A, B = synth.lc_gemm_inputs(M, N, K, seed=17, variant="int")
     D = torch.zeros(M, N, device=dev())
     f = tk.tacker_fuse(tk.lc_gemm(t(A), t(B), D), None, 0)
