@@ -529,6 +529,7 @@ def run_tacker(args, comm):
     seed = 2022 + rank
     svc = sv.resnet50_service(args.batch, seed)
     sv.autotune_tile_n(svc)                                      # LC tile width per conv, measured
+    chain_tune = sv.chain_autotune_tile_n(svc)                   # ... refined on the query chain
     names = sv.TABLE2_BE if args.be == "table2" else tuple(args.be.split(","))
     apps = sv.be_apps(names, seed)
     sv.prime_apps(apps)
@@ -613,7 +614,10 @@ def run_tacker(args, comm):
         "vs_baseline": None, "dtype": "f16xf16->f32 (LC tcgen05) + f32 (BE CUDA cores)",
         "data": "synthetic (seeded inputs, random weights)",
         "config": {"workload": WORKLOAD.format(b=args.batch, be=",".join(names)),
-                   "lc": f"ResNet-50 batch-{args.batch} (Table II), 53 convs, fp16 NHWC, implicit GEMM tcgen05",
+                   "lc": f"ResNet-50 batch-{args.batch} (Table II), 53 convs, fp16 NHWC, implicit GEMM tcgen05, "
+                         f"tile widths measured per kernel then on the query chain "
+                         f"({chain_tune['before_ms']:.3f} -> {chain_tune['after_ms']:.3f} ms per query, "
+                         f"{len(chain_tune['changed'])} changed)",
                    "be": " | ".join(a.name for a in apps),
                    "arrivals": f"Poisson at {LOAD:.0%} of lambda_peak (LC-only p99 <= QoS, bisection) = "
                                f"{load:.3f} x the LC-only service rate",

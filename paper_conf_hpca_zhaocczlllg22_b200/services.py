@@ -120,6 +120,42 @@ def autotune_tile_n(svc: LcService, reps: int = 8, choices=(64, 128, 256)) -> di
     return out
 
 
+def chain_autotune_tile_n(svc: LcService, reps: int = 9, choices=(64, 128, 256), min_gain: float = 0.003) -> dict:
+    """Refine the per-kernel tile widths (autotune_tile_n first) on the query chain itself: the
+    query's kernels launched back to back are what the manager runs, and a kernel that follows
+    another instantiation starts with a cold instruction cache, so the fastest
+    width of a kernel repeated alone is not always the fastest in the chain.  One greedy pass over
+    the tensor-core kernels: each alternative width is kept if the whole query's CUDA-event time
+    (median of `reps`) improves by more than `min_gain`.  Returns {"before_ms", "after_ms",
+    "changed": {name: (old, new)}}."""
+    from .qos import _time
+
+    def query():
+        for k in svc.kernels:
+            tk.tacker_launch_original(k.lc if k.is_tc else None, None if k.is_tc else k.cd)
+
+    base = _time(query, reps)
+    out = {"before_ms": base, "changed": {}}
+    for k in svc.kernels:
+        if not k.is_tc:
+            continue
+        cur = k.lc.tile_n
+        for bn in choices:
+            if bn == cur:
+                continue
+            k.lc.tile_n = bn
+            try:
+                t = _time(query, reps)
+            except tk.TackerError:
+                t = None
+            if t is not None and t < base * (1.0 - min_gain):
+                base, cur = t, bn
+                out["changed"][k.name] = (out["changed"].get(k.name, (k.lc.tile_n,))[0], bn)
+            k.lc.tile_n = cur
+    out["after_ms"] = base
+    return out
+
+
 def vgg16_service(batch: int = 1, seed: int = 2023) -> LcService:
     return _named(resnet50_service(batch, seed, convs=synth.vgg16_convs(batch)), f"vgg16_b{batch}")
 

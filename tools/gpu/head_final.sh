@@ -1,4 +1,4 @@
-D=gpurun_out/head_final2
+D=gpurun_out/head_final3
 mkdir -p $D
 timeout 1500 python -m pytest tests -m gpu -q > $D/gpu_tests.log 2>&1; echo "pytest_rc=$?" >> $D/gpu_tests.log
 python -c "import __graft_entry__ as g; g.smoke()" > $D/smoke.log 2>&1

@@ -43,10 +43,13 @@ def main():
     ap.add_argument("--batch", type=int, default=1)
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--autotune", action="store_true", help="measured LC tile width per conv (services.autotune_tile_n)")
+    ap.add_argument("--chain-autotune", action="store_true", help="then refine the widths on the query chain")
     args = ap.parse_args()
     svc = sv.resnet50_service(args.batch) if args.service == "resnet50" else sv.vgg16_service(args.batch)
     if args.autotune:
         sv.autotune_tile_n(svc)
+    if args.chain_autotune:
+        sv.chain_autotune_tile_n(svc)
     res = {"service": svc.name, "kernels": len(svc.kernels), "autotune": bool(args.autotune)}
     for on in (False, True):
         tk.tacker_set_launch_overlap(on)
